@@ -1,0 +1,295 @@
+/*
+ * sh.h -- C ABI of the STRONGHOLD working-window offload engine (B200 / sm_100a).
+ *
+ * The engine trains a layer-sequential model whose parameters, gradients and Adam
+ * states live in pinned host RAM while only a sliding window of layers sits in a
+ * ring of GPU layer slots (§III-A; §III-C,
+ * Fig. 3b/3c).  The caller's model code drives it through per-layer hooks, the way
+ * STRONGHOLD's pre_forward / post_forward / pre_backward callbacks are driven by
+ * framework hooks.
+ *
+ * Step protocol (any other order returns SH_ERR_STATE):
+ *     for i in 0..L-1:    sh_forward_layer(i, SH_PRE)  -> compute FP of layer i -> sh_forward_layer(i, SH_POST)
+ *     (caller: head / loss using sh_resident views)
+ *     for i in L-1..0:    sh_backward_layer(i, SH_PRE) -> recompute + BP of layer i -> sh_backward_layer(i, SH_POST)
+ *     (caller: embedding backward into the sh_resident grad views)
+ *     sh_step()
+ * Every device pointer handed out is valid on the caller's compute stream between
+ * the PRE that returned it and the matching POST (layers) or the next sh_step
+ * (resident set).  The caller must enqueue its layer computation on that compute
+ * stream.  Hooks never block the host on the GPU; they may block on a true data
+ * dependency (the CPU Adam update of a layer that is about to be prefetched, or a
+ * full host landing ring).
+ *
+ * Window convention (eq. 1b-1c are garbled; reading R4):
+ *   window w = the paper's m = prefetch distance.  The ring has w+1 slots (the
+ *   extra slot is the landing slot s^j of (1c)).  Layers [0, w) plus the resident
+ *   set (embedding, positions, final LN) are GPU-optimised ("the first few layers
+ *   ... layers of the first working window"; Fig. 3 caption
+ *   PAPER.md:130).  Layers [w, L) are host-optimised by the multi-threaded CPU AdamW
+ *   (PAPER.md:201-205).  w = L is the all-resident configuration; w = 0 is
+ *   serial fetch-then-compute (L2L-like).
+ *
+ * Numerics contract (makes results bit-identical for
+ * every window): the GPU Adam (K2) and the CPU Adam execute per
+ * element, in IEEE fp32 round-to-nearest, no FTZ/DAZ:
+ *     g = g*coef (only when clipping is on);  m = fma(b1, m, omb1*g);
+ *     v = fma(b2, v, omb2*(g*g));  d = sqrt(v)/sqrt_bc2 + eps;
+ *     p = fma(-step_size, m/d, wd ? p*decay : p);  p16 = rne_bf16(p)
+ *   with omb1 = 1-b1, omb2 = 1-b2, sqrt_bc2 = sqrt(1-b2^t), step_size = lr/(1-b1^t),
+ *   decay = 1 - lr*lambda computed in double on the host and rounded once to fp32.
+ *   rne_bf16 is integer round-to-nearest-even with canonical NaN 0x7FC0.
+ *
+ * Errors: every call returns sh_status; no exception crosses the ABI.  The message
+ * of the last failing call on this thread is sh_last_error().  After SH_ERR_CUDA /
+ * SH_ERR_NCCL / SH_ERR_OOM_* inside a step, the context is failed: every call except
+ * sh_destroy, sh_stats and sh_last_error returns SH_ERR_STATE.
+ * Threading: one driver thread per context.  Internally the engine runs an H2D
+ * issuer thread, a D2H issuer thread and the CPU Adam pool.
+ */
+#ifndef SH_H_
+#define SH_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SH_ABI_VERSION 1
+
+typedef struct sh_ctx sh_ctx;
+
+typedef enum {
+  SH_OK = 0,
+  SH_ERR_INVALID = -1,     /* bad argument / configuration (message says which) */
+  SH_ERR_CUDA = -2,        /* CUDA runtime error (sync or async) */
+  SH_ERR_OOM_DEVICE = -3,  /* device allocation failed */
+  SH_ERR_OOM_HOST = -4,    /* host allocation or page-locking failed */
+  SH_ERR_NCCL = -5,        /* NCCL error (world_size > 1) */
+  SH_ERR_STATE = -6,       /* call out of protocol order, or context failed */
+  SH_ERR_UNSUPPORTED = -7  /* feature not available on this build / device */
+} sh_status;
+
+typedef enum { SH_FP32 = 0, SH_BF16_MIXED = 1 } sh_precision;
+typedef enum { SH_PRE = 0, SH_POST = 1 } sh_phase;
+
+/* What sh_read_layer returns. */
+typedef enum {
+  SH_READ_PARAM = 0,   /* fp32 master parameters (float[numel]) */
+  SH_READ_M = 1,       /* fp32 Adam first moment */
+  SH_READ_V = 2,       /* fp32 Adam second moment */
+  SH_READ_COMPUTE = 3  /* compute copy: uint16 bf16 bits (bf16 mode) or float (fp32 mode) */
+} sh_read_what;
+
+/* One layer (offload unit): its tensors in the caller's order.
+ * numel[k] > 0.  weight_decay[k] != 0: decoupled decay applies to tensor k. */
+typedef struct {
+  int32_t n_tensors;             /* 1..64 */
+  const int64_t* numel;          /* [n_tensors] */
+  const uint8_t* weight_decay;   /* [n_tensors] */
+} sh_layer_shape;
+
+/* Flags */
+#define SH_FLAG_PROFILE   (1ull << 0) /* record per-layer CUDA events every step (else warm-up only) */
+#define SH_FLAG_POISON    (1ull << 1) /* debug: fill a slot's param half with NaN before every refill */
+#define SH_FLAG_DUPLEX    (1ull << 2) /* autotuner: full-duplex link, max() instead of sum in (1d)/(2d) */
+#define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline on the D2H issuer (no pool) */
+
+typedef struct {
+  int32_t n_layers;                 /* L >= 1, execution order */
+  const sh_layer_shape* layers;     /* [n_layers] */
+  sh_layer_shape resident;          /* embedding / positions / final LN: always in HBM */
+  int32_t window;                   /* 0..n_layers, or -1: w0 = min(2, w_max) then autotune after warm-up */
+  int32_t precision;                /* sh_precision */
+  float lr;                         /* initial learning rate (sh_set_lr changes it) */
+  float beta1, beta2, eps, weight_decay;
+  float max_grad_norm;              /* <= 0: no clipping (throughput mode, R3) */
+  int32_t device;                   /* CUDA ordinal */
+  void* compute_stream;             /* caller-owned cudaStream_t for all layer compute (required) */
+  int32_t cpu_threads;              /* CPU Adam threads; 0 = all online cores */
+  int32_t grad_ring_depth;          /* host landing buffers for offloaded grads; 0 = one per host layer */
+  int32_t warmup_steps;             /* profiled steps before autotune (default 5); 0 = default */
+  int64_t device_budget_bytes;      /* S_avail for ring + G states; 0 = free memory - 2 GiB */
+  int32_t world_size;               /* data-parallel ranks (1 = single GPU) */
+  int32_t rank;
+  const void* nccl_unique_id;       /* 128-byte ncclUniqueId, required when world_size > 1 */
+  uint64_t flags;                   /* SH_FLAG_* */
+} sh_config;
+
+/* Per-layer profile consumed by the window solver (PAPER.md:132 notation; times in ms,
+ * sizes in bytes).  Arrays have n_layers entries; NULL arrays are treated as zeros. */
+typedef struct {
+  int32_t n_layers;
+  const double* t_fp;       /* FP compute time of layer i */
+  const double* t_bp;       /* BP time incl. recompute (PAPER.md:153 fn. 2) */
+  const double* t_c2g;      /* host -> device fetch of layer i */
+  const double* t_g2c;      /* device -> host gradient offload of layer i */
+  const double* t_stage;    /* K1 restage of a GPU-optimised layer in BP (replaces t_c2g for i < w) */
+  const double* t_opt_gpu;  /* K2 time of layer i */
+  const double* t_opt_cpu;  /* CPU Adam time of layer i */
+  double t_async;           /* one asynchronous hook call (eq. 4) */
+  const int64_t* slot_bytes;   /* s_bp of layer i: bytes of one ring slot holding i (param + grad half) */
+  const int64_t* gstate_bytes; /* HBM bytes of layer i's master/m/v when GPU-optimised */
+  int64_t fixed_bytes;         /* HBM always used by the engine (resident set, scratch) */
+  int64_t s_avail;             /* S_avail */
+  int32_t duplex;              /* 1: soft constraints use max(Σc2g, Σg2c) (R7) */
+} sh_profile;
+
+typedef struct {
+  int32_t window;          /* chosen w* */
+  int32_t w_max_memory;    /* largest w meeting (1c)/(2c) */
+  int32_t reason;          /* 0: hard+soft met; 1: hard only; 2: memory fallback */
+  int32_t fp_hard_ok, bp_hard_ok, soft_ok;  /* at the chosen window */
+  double eq3_min_slack_ms; /* min_k [Σ_{i<=k}(t_fp+t_bp) + Σ_{i<w} t_opt_gpu - t_opt_cpu_k]  (eq. 3) */
+  int32_t eq3_ok;
+  double eq4_lhs_ms, eq4_rhs_ms; /* 5 n t_async  vs  Σ_{i=w}^{n-1} t_opt_gpu (eq. 4) */
+} sh_solve_report;
+
+typedef struct {
+  int64_t step;                 /* completed sh_step calls */
+  int32_t window;
+  int32_t n_slots;
+  int64_t host_bytes;           /* pinned host store */
+  int64_t device_bytes;         /* ring + G states + resident + scratch */
+  int64_t h2d_bytes, d2h_bytes; /* cumulative algorithmic bytes moved by the engine */
+  int64_t h2d_copies, d2h_copies, stage_launches;
+  double h2d_busy_ms, d2h_busy_ms; /* cumulative copy durations (profiled steps only) */
+  int64_t h2d_profiled_bytes, d2h_profiled_bytes;
+  double cpu_adam_ms;           /* cumulative wall time of CPU Adam tasks (summed over threads) */
+  int64_t cpu_adam_elems;
+  double cpu_wait_ms;           /* cumulative time the H2D issuer waited on CPU Adam (eq. 3 violation) */
+  double k2_ms_last;            /* duration of the last sh_step K2 launch(es) when profiled */
+  int64_t k2_bytes_last;        /* algorithmic HBM bytes of that K2 */
+  int32_t k2_launches_last;
+  int32_t cpu_threads;
+  int32_t profiled_steps;
+} sh_stats_t;
+
+/* ---- lifecycle ------------------------------------------------------------------ */
+
+/* Validate cfg, build the size table (a0), allocate and page-lock the
+ * host store (D1), reserve the ring of w+1 slots and the GPU states
+ * once (D2), start the issuer threads and the CPU Adam pool.
+ * Returns SH_ERR_INVALID for bad shapes, SH_ERR_OOM_* when memory is short. */
+sh_status sh_init(const sh_config* cfg, sh_ctx** out);
+
+/* Copy in the initial fp32 state of `layer` (-1 = resident set).  params / m / v are
+ * host arrays of Σ numel floats, tensors concatenated in the caller's order; m and v
+ * may be NULL (zeros).  `step` = number of updates already applied (0 for fresh
+ * training; used for bias correction on resume).  Caller keeps ownership.  Must be
+ * called for every layer and the resident set before the first forward hook. */
+sh_status sh_register_host_store(sh_ctx* ctx, int32_t layer, const float* params,
+                                 const float* m, const float* v, int64_t step);
+
+/* Block until the engine is idle (all streams, issuers and CPU Adam tasks). */
+sh_status sh_synchronize(sh_ctx* ctx);
+
+sh_status sh_destroy(sh_ctx* ctx);
+
+/* ---- hooks (hot path) ----------------------------------------------------------- */
+
+/* FP hook.  SH_PRE: issue the async prefetch of the layer that enters the window
+ * (PAPER.md:108 step 1; position c+w of the step's use sequence), make the compute
+ * stream wait for layer `layer`'s arrival, and write its n_tensors device pointers
+ * (bf16 in SH_BF16_MIXED, fp32 in SH_FP32) into dev_params.  SH_POST: mark the
+ * layer's slot reusable once the compute enqueued so far finishes (step 3; no
+ * parameter write-back: FP does not change parameters, R10). */
+sh_status sh_forward_layer(sh_ctx* ctx, int32_t layer, int32_t phase, void** dev_params);
+
+/* BP hook.  SH_PRE: as FP, plus a zeroed fp32 gradient buffer per tensor in dev_grads
+ * (the caller writes, not accumulates, unless it wants to accumulate into zeros).
+ * GPU-optimised layers evicted during FP are restaged from their HBM master by K1.
+ * SH_POST: per-layer Σg² (K3), [world_size>1: NCCL average allreduce], then for a
+ * host-optimised layer the D2H gradient offload (PAPER.md:111 step 2) and the CPU
+ * Adam dispatch (step 3) that runs while the GPU continues. */
+sh_status sh_backward_layer(sh_ctx* ctx, int32_t layer, int32_t phase, void** dev_params,
+                            float** dev_grads);
+
+/* Views of the resident set: compute copies (bf16 or fp32) and fp32 grads.  The grads
+ * are zeroed at the first forward hook of every step. */
+sh_status sh_resident(sh_ctx* ctx, void** dev_params, float** dev_grads);
+
+/* Learning rate for the steps whose backward starts after this call. */
+sh_status sh_set_lr(sh_ctx* ctx, float lr);
+
+/* End of step: finalize the global gradient norm in fixed order (K3
+ * partials), then one fused multi-tensor AdamW (K2) over layers [0, w) and the
+ * resident set writing their new compute copies in place; in clip mode release the
+ * CPU Adam tasks with the clip coefficient.  Does not block unless grad_norm_out is
+ * non-NULL (then it synchronises and returns ||g||_2). */
+sh_status sh_step(sh_ctx* ctx, double* grad_norm_out);
+
+/* ---- window ----------------------------------------------------------------------- */
+
+/* Pure solver of the paper's analytic model P1 (eq. 1a-1d), P2 (eq. 2a-2d) and the
+ * window rule of PAPER.md:195, with the eq. 3 / eq. 4 checks reported.  No context,
+ * no GPU.  Returns SH_ERR_INVALID for inconsistent profiles. */
+sh_status sh_solve_window(const sh_profile* prof, sh_solve_report* report);
+
+/* Solve on the measured warm-up profile (or on `override` when non-NULL) and apply the
+ * result between steps (ring grows, never shrinks).  window_out may be NULL. */
+sh_status sh_autotune_window(sh_ctx* ctx, const sh_profile* override_profile, int32_t* window_out);
+
+/* Change the window between steps (after sh_step, before the next forward hook). */
+sh_status sh_set_window(sh_ctx* ctx, int32_t window);
+
+/* Fill the engine's measured profile (arrays owned by ctx, valid until the next call). */
+sh_status sh_get_profile(sh_ctx* ctx, sh_profile* out);
+
+/* ---- inspection ------------------------------------------------------------------- */
+
+/* Blocking copy of one layer's state (layer -1: resident) into host dst, in the caller's
+ * tensor order without padding.  Waits for any pending update of that layer. */
+sh_status sh_read_layer(sh_ctx* ctx, int32_t layer, int32_t what, void* dst);
+
+sh_status sh_stats(sh_ctx* ctx, sh_stats_t* out);
+
+/* Thread-local message of the last failed call ("" if none). */
+const char* sh_last_error(void);
+
+int32_t sh_abi_version(void);
+
+/* Rank 0 of a data-parallel job: fill a 128-byte ncclUniqueId (dlopen'ed libnccl.so.2, the
+ * one torch loads) to be broadcast through torch.distributed before sh_init. */
+sh_status sh_nccl_get_unique_id(void* out128);
+
+/* ---- op-level entry points (the kernels of the path, for parity tests) -------------
+ * All device pointers must be 16-byte aligned and n a multiple of 8.  `stream` is a
+ * cudaStream_t (NULL = legacy default).  Asynchronous; errors from the launch only. */
+
+typedef struct {
+  float beta1, beta2, omb1, omb2, eps, step_size, sqrt_bc2, decay;
+} sh_adam_scalars;
+
+/* Host-side derivation of the per-step fp32 scalars from (lr, t) in double. */
+sh_status sh_adam_scalars_for(float lr, float beta1, float beta2, float eps, float weight_decay,
+                              int64_t t, sh_adam_scalars* out);
+
+/* K2 on one flat tensor range: elements [0, n_decay) get weight decay, [n_decay, n) not.
+ * p, m, v: fp32 in/out; g: fp32 in; out16: bf16 compute copy out (uint16 bits) or NULL;
+ * out32: fp32 compute copy out or NULL; coef: device float (clip coefficient) or NULL. */
+sh_status sh_op_adamw_gpu(float* p, float* m, float* v, const float* g, uint16_t* out16,
+                          float* out32, int64_t n, int64_t n_decay, const sh_adam_scalars* sc,
+                          const float* coef, void* stream);
+
+/* The CPU AdamW of the pool on host arrays (same contract as above; coef is a host
+ * value, ignored when use_coef == 0).  n_threads <= 0: all cores. */
+sh_status sh_op_adamw_cpu(float* p, float* m, float* v, const float* g, uint16_t* out16,
+                          int64_t n, int64_t n_decay, const sh_adam_scalars* sc, int32_t use_coef,
+                          float coef, int32_t n_threads);
+
+/* K1: dst16[i] = rne_bf16(src[i]) on the device. */
+sh_status sh_op_cast_bf16_gpu(const float* src, uint16_t* dst16, int64_t n, void* stream);
+
+/* CPU rne_bf16 (the shadow writer of the CPU Adam). */
+sh_status sh_op_cast_bf16_cpu(const float* src, uint16_t* dst16, int64_t n);
+
+/* K3: out[0] = Σ g[i]^2 accumulated in fp64 with a fixed reduction tree (deterministic). */
+sh_status sh_op_sumsq_gpu(const float* g, int64_t n, double* out_dev, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SH_H_ */

@@ -1,0 +1,119 @@
+// Window-size solver: the paper's analytic model (§III-D).
+//
+//   P1 (FP, eq. 1a-1d):  min m  s.t.  (1b) window compute >= fetch of the layer entering it,
+//                        (1c) memory <= S_avail (hard), (1d) window compute >= Σc2g + Σg2c (soft)
+//   P2 (BP, eq. 2a-2d):  min m  s.t.  (2b) window BP time >= transfers of the layer entering it,
+//                        (2c) memory (hard), (2d) soft as (1d)
+//   window rule: m meeting P1 and P2 for all layers; otherwise the largest m
+//                        the memory permits.
+//   eq. 3 / eq. 4 are evaluated and reported, not used to choose m.
+//
+// Readings (R4-R8): m = w = prefetch distance; the sums of (1b)/(1d) run over the
+// w layers before the entering layer j; (2b) uses the decoupled param/grad slot halves of this
+// engine, so the entering layer's fetch and the leaving layer's offload proceed in opposite
+// link directions and the constraint is max(g2c, c2g) (a GPU-optimised entering layer is
+// restaged by K1: t_stage replaces t_c2g); the soft constraints use the paper's half-duplex
+// sum unless `duplex` is set (then max); "min m" with soft constraints is lexicographic:
+// hard and soft -> hard only -> memory maximum.  The implementation uses prefix sums; the
+// oracle (oracle/autotune_oracle.py) evaluates the same definitions with plain loops.
+#include <algorithm>
+#include <cmath>
+#include <vector>
+
+#include "sh_internal.hpp"
+
+namespace sh {
+
+namespace {
+struct Prefix {
+  std::vector<double> s;  // s[i] = Σ_{k<i} a[k]
+  explicit Prefix(const double* a, int n) : s(n + 1, 0.0) {
+    for (int i = 0; i < n; ++i) s[i + 1] = s[i] + (a ? a[i] : 0.0);
+  }
+  double sum(int b, int e) const {  // Σ_{k=b}^{e-1}
+    if (e <= b) return 0.0;
+    return s[e] - s[b];
+  }
+};
+inline double at(const double* a, int i) { return a ? a[i] : 0.0; }
+}  // namespace
+
+}  // namespace sh
+
+using namespace sh;
+
+extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
+  clear_error();
+  if (!P || !R || P->n_layers < 1) {
+    set_error("sh_solve_window: null profile/report or n_layers < 1");
+    return SH_ERR_INVALID;
+  }
+  const int L = P->n_layers;
+  const Prefix fp(P->t_fp, L), bp(P->t_bp, L), c2g(P->t_c2g, L), g2c(P->t_g2c, L);
+  const Prefix ogpu(P->t_opt_gpu, L);
+  int64_t slot = 0;
+  for (int i = 0; i < L; ++i) slot = std::max<int64_t>(slot, P->slot_bytes ? P->slot_bytes[i] : 0);
+
+  auto mem_ok = [&](int w) {
+    int64_t need = P->fixed_bytes + (int64_t)(w + 1) * slot;
+    for (int i = 0; i < w; ++i) need += P->gstate_bytes ? P->gstate_bytes[i] : 0;
+    return need <= P->s_avail;
+  };
+  auto fp_hard = [&](int w) {  // (1b): ∀ j ∈ [w, L): Σ_{i=j-w}^{j-1} t_fp ≥ t_c2g[j]
+    for (int j = w; j < L; ++j)
+      if (fp.sum(j - w, j) < at(P->t_c2g, j)) return false;
+    return true;
+  };
+  auto bp_hard = [&](int w) {  // (2b): ∀ j ∈ [0, L-w-2]: Σ_{i=j+1}^{j+w} t_bp ≥ max(g2c[j+w+1], fetch_j)
+    for (int j = 0; j + w + 1 < L; ++j) {
+      const double fetch = j < w ? at(P->t_stage, j) : at(P->t_c2g, j);
+      const double need = std::max(at(P->t_g2c, j + w + 1), fetch);
+      if (bp.sum(j + 1, j + w + 1) < need) return false;
+    }
+    return true;
+  };
+  auto soft = [&](int w) {  // (1d) over FP windows, (2d) over BP windows
+    for (int j = w; j < L; ++j) {
+      const double a = c2g.sum(j - w, j), b = g2c.sum(j - w, j);
+      if (fp.sum(j - w, j) < (P->duplex ? std::max(a, b) : a + b)) return false;
+    }
+    for (int j = 0; j + w + 1 < L; ++j) {
+      const double a = c2g.sum(j + 1, j + w + 1), b = g2c.sum(j + 1, j + w + 1);
+      if (bp.sum(j + 1, j + w + 1) < (P->duplex ? std::max(a, b) : a + b)) return false;
+    }
+    return true;
+  };
+
+  int wmax = -1;
+  for (int w = 0; w <= L; ++w)
+    if (mem_ok(w)) wmax = w;
+  if (wmax < 0) {
+    set_error("sh_solve_window: even w=0 exceeds S_avail (%lld bytes)", (long long)P->s_avail);
+    return SH_ERR_OOM_DEVICE;
+  }
+  int best = -1, reason = 2;
+  for (int w = 0; w <= L && best < 0; ++w)
+    if (mem_ok(w) && fp_hard(w) && bp_hard(w) && soft(w)) best = w, reason = 0;
+  for (int w = 0; w <= L && best < 0; ++w)
+    if (mem_ok(w) && fp_hard(w) && bp_hard(w)) best = w, reason = 1;
+  if (best < 0) best = wmax, reason = 2;
+
+  R->window = best;
+  R->w_max_memory = wmax;
+  R->reason = reason;
+  R->fp_hard_ok = fp_hard(best);
+  R->bp_hard_ok = bp_hard(best);
+  R->soft_ok = soft(best);
+  // eq. 3: t_opt_cpu^k ≤ Σ_{i=0}^{k}(t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i,  k ∈ [w, L)
+  double slack = INFINITY;
+  for (int k = best; k < L; ++k) {
+    const double rhs = fp.sum(0, k + 1) + bp.sum(0, k + 1) + ogpu.sum(0, best);
+    slack = std::min(slack, rhs - at(P->t_opt_cpu, k));
+  }
+  R->eq3_min_slack_ms = std::isinf(slack) ? 0.0 : slack;
+  R->eq3_ok = !(slack < 0.0);
+  // eq. 4: 5 n t_async ≤ Σ_{i=w}^{n-1} t_opt_gpu
+  R->eq4_lhs_ms = 5.0 * L * P->t_async;
+  R->eq4_rhs_ms = ogpu.sum(best, L);
+  return SH_OK;
+}

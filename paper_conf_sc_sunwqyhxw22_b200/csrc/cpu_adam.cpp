@@ -1,0 +1,142 @@
+// CPU AdamW of the concurrent optimizer pool (§III-E1) and the bf16 shadow
+// writer.  Executes exactly the op sequence of K2 (kernels.cu) in IEEE fp32 so that a layer
+// updated here is bit-identical to the same layer updated on the GPU (DESIGN.md "Engine
+// numerics"; the property behind PAPER.md:87's "no stale updates, no precision change").
+//
+// Built with -ffp-contract=off and without -ffast-math: no implicit FMA, no reassociation,
+// no FTZ/DAZ (MXCSR defaults).  FMAs are explicit (std::fmaf / _mm512_fmadd_ps, both
+// correctly rounded).  bf16 rounding uses the integer RNE trick (vcvtneps2bf16 flushes
+// denormals, so it is not used).
+#include <immintrin.h>
+
+#include <cmath>
+#include <cstdint>
+#include <cstring>
+
+#include "sh_internal.hpp"
+
+namespace sh {
+namespace cpu {
+
+uint16_t rne_bf16(float x) {
+  uint32_t u;
+  std::memcpy(&u, &x, 4);
+  if ((u & 0x7fffffffu) > 0x7f800000u) return 0x7fc0u;
+  return (uint16_t)((u + 0x7fffu + ((u >> 16) & 1u)) >> 16);
+}
+
+static inline void adam_scalar(float& p, float& m, float& v, float g, const sh_adam_scalars& s,
+                               bool wd, bool use_coef, float coef) {
+  if (use_coef) g = g * coef;
+  m = std::fmaf(s.beta1, m, s.omb1 * g);
+  v = std::fmaf(s.beta2, v, s.omb2 * (g * g));
+  const float d = std::sqrt(v) / s.sqrt_bc2 + s.eps;
+  const float pp = wd ? p * s.decay : p;
+  p = std::fmaf(-s.step_size, m / d, pp);
+}
+
+static void adam_scalar_range(float* p, float* m, float* v, const float* g, uint16_t* out16,
+                              int64_t b, int64_t e, int64_t n_decay, const sh_adam_scalars& s,
+                              bool use_coef, float coef) {
+  for (int64_t i = b; i < e; ++i) {
+    adam_scalar(p[i], m[i], v[i], g[i], s, i < n_decay, use_coef, coef);
+    if (out16) out16[i] = rne_bf16(p[i]);
+  }
+}
+
+__attribute__((target("avx512f"))) static inline __m256i rne_bf16_16(__m512 x) {
+  const __m512i u = _mm512_castps_si512(x);
+  const __m512i one = _mm512_set1_epi32(1);
+  const __m512i c7fff = _mm512_set1_epi32(0x7fff);
+  const __m512i absm = _mm512_set1_epi32(0x7fffffff);
+  const __m512i inf = _mm512_set1_epi32(0x7f800000);
+  const __m512i qnan = _mm512_set1_epi32(0x7fc0);
+  const __m512i lsb = _mm512_and_si512(_mm512_srli_epi32(u, 16), one);
+  __m512i r = _mm512_srli_epi32(_mm512_add_epi32(u, _mm512_add_epi32(lsb, c7fff)), 16);
+  const __mmask16 nan = _mm512_cmpgt_epu32_mask(_mm512_and_si512(u, absm), inf);
+  r = _mm512_mask_mov_epi32(r, nan, qnan);
+  return _mm512_cvtepi32_epi16(r);
+}
+
+template <bool kWd, bool kCoef, bool kOut>
+__attribute__((target("avx512f"))) static void adam_avx512_block(
+    float* __restrict p, float* __restrict m, float* __restrict v, const float* __restrict g,
+    uint16_t* __restrict out16, int64_t b, int64_t e, const sh_adam_scalars& s, float coef) {
+  const __m512 b1 = _mm512_set1_ps(s.beta1), b2 = _mm512_set1_ps(s.beta2);
+  const __m512 omb1 = _mm512_set1_ps(s.omb1), omb2 = _mm512_set1_ps(s.omb2);
+  const __m512 eps = _mm512_set1_ps(s.eps), nss = _mm512_set1_ps(-s.step_size);
+  const __m512 sbc2 = _mm512_set1_ps(s.sqrt_bc2), decay = _mm512_set1_ps(s.decay);
+  const __m512 vc = _mm512_set1_ps(coef);
+  for (int64_t i = b; i < e; i += 16) {
+    __m512 gg = _mm512_loadu_ps(g + i);
+    if (kCoef) gg = _mm512_mul_ps(gg, vc);
+    __m512 mm = _mm512_loadu_ps(m + i);
+    __m512 vv = _mm512_loadu_ps(v + i);
+    __m512 pp = _mm512_loadu_ps(p + i);
+    mm = _mm512_fmadd_ps(b1, mm, _mm512_mul_ps(omb1, gg));
+    vv = _mm512_fmadd_ps(b2, vv, _mm512_mul_ps(omb2, _mm512_mul_ps(gg, gg)));
+    const __m512 d = _mm512_add_ps(_mm512_div_ps(_mm512_sqrt_ps(vv), sbc2), eps);
+    if (kWd) pp = _mm512_mul_ps(pp, decay);
+    pp = _mm512_fmadd_ps(nss, _mm512_div_ps(mm, d), pp);
+    _mm512_storeu_ps(m + i, mm);
+    _mm512_storeu_ps(v + i, vv);
+    _mm512_storeu_ps(p + i, pp);
+    if (kOut) _mm256_storeu_si256(reinterpret_cast<__m256i*>(out16 + i), rne_bf16_16(pp));
+  }
+}
+
+template <bool kWd>
+static void adam_vec_dispatch(float* p, float* m, float* v, const float* g, uint16_t* out16,
+                              int64_t b, int64_t e, const sh_adam_scalars& s, bool use_coef,
+                              float coef) {
+  if (use_coef) {
+    if (out16) adam_avx512_block<kWd, true, true>(p, m, v, g, out16, b, e, s, coef);
+    else adam_avx512_block<kWd, true, false>(p, m, v, g, out16, b, e, s, coef);
+  } else {
+    if (out16) adam_avx512_block<kWd, false, true>(p, m, v, g, out16, b, e, s, coef);
+    else adam_avx512_block<kWd, false, false>(p, m, v, g, out16, b, e, s, coef);
+  }
+}
+
+bool has_avx512() {
+  static const bool ok = __builtin_cpu_supports("avx512f");
+  return ok;
+}
+
+void adamw_range(float* p, float* m, float* v, const float* g, uint16_t* out16, int64_t begin,
+                 int64_t end, int64_t n_decay, const sh_adam_scalars& sc, bool use_coef,
+                 float coef) {
+  if (!has_avx512()) {
+    adam_scalar_range(p, m, v, g, out16, begin, end, n_decay, sc, use_coef, coef);
+    return;
+  }
+  // decayed part [begin, min(end, n_decay)), then the rest; vector body in 16s, scalar tails
+  const int64_t split = end < n_decay ? end : (begin > n_decay ? begin : n_decay);
+  const int64_t parts[2][2] = {{begin, split}, {split, end}};
+  for (int k = 0; k < 2; ++k) {
+    const int64_t b = parts[k][0], e = parts[k][1];
+    if (b >= e) continue;
+    const int64_t ev = b + ((e - b) / 16) * 16;
+    if (k == 0) adam_vec_dispatch<true>(p, m, v, g, out16, b, ev, sc, use_coef, coef);
+    else adam_vec_dispatch<false>(p, m, v, g, out16, b, ev, sc, use_coef, coef);
+    adam_scalar_range(p, m, v, g, out16, ev, e, n_decay, sc, use_coef, coef);
+  }
+}
+
+__attribute__((target("avx512f"))) static void cast_avx512(const float* src, uint16_t* dst,
+                                                           int64_t b, int64_t e) {
+  for (int64_t i = b; i < e; i += 16)
+    _mm256_storeu_si256(reinterpret_cast<__m256i*>(dst + i), rne_bf16_16(_mm512_loadu_ps(src + i)));
+}
+
+void cast_bf16_range(const float* src, uint16_t* dst, int64_t begin, int64_t end) {
+  int64_t ev = begin;
+  if (has_avx512()) {
+    ev = begin + ((end - begin) / 16) * 16;
+    cast_avx512(src, dst, begin, ev);
+  }
+  for (int64_t i = ev; i < end; ++i) dst[i] = rne_bf16(src[i]);
+}
+
+}  // namespace cpu
+}  // namespace sh

@@ -1,0 +1,1741 @@
+// STRONGHOLD working-window offload engine for B200.
+//
+// Paper mechanism -> this file:
+//   pinned per-layer CPU buffers            -> HostStore: one mmap'ed, THP-advised,
+//                                                              page-locked region; per layer fp32
+//                                                              master | m | v | bf16 shadow
+//   reserved round-robin GPU buffer queue -> ring of w+1 slots, one cudaMalloc,
+//                                                              grow-only; param half + grad half
+//   pre_forward / post_forward (Fig. 3b)      -> sh_forward_layer PRE/POST
+//   pre_backward (Fig. 3c)                    -> sh_backward_layer PRE/POST
+//   "idle CUDA stream" async copies          -> H2D and D2H copy-engine streams, each
+//                                                              owned by an issuer thread
+//   concurrent CPU optimizers            -> AdamPool: worker threads, per-layer
+//                                                              jobs split into chunks, lowest layer
+//                                                              (needed first by the next FP) first
+//   first window + embedding updated on GPU  -> K2 over layers [0,w) + resident set
+//   warm-up profiling                         -> CUDA events per layer / transfer
+//   NCCL data-parallel gradient sync    -> per-layer ncclAllReduce(avg) on a
+//                                                              comm stream before the offload
+//
+// Which slot a fetch lands in: the use sequence of one step is fixed (FP 0..L-1, BP L-1..0), so
+// the victim is chosen by farthest next use (Belady) among slots whose occupant is not needed
+// before the fetched layer; this reproduces the paper's sliding window (FP: the slot of layer
+// i-1 receives layer i+w; BP: the slot of layer i+1 receives layer i-w) and handles the FP/BP
+// turn, w = 0 and w = L uniformly.
+//
+// No host stall on the GPU: PRE/POST only enqueue work and record events.  The single true
+// cross-device dependency -- "the prefetch of host layer j for step t must read the parameters
+// the CPU Adam produced in step t-1" -- is enforced by the H2D issuer thread waiting on the
+// layer's ready counter before it enqueues the copy (this B200 box reports no stream-memop
+// support, profiles/r01_probe_box.json, so cuStreamWaitValue32 is not used).
+#include <dlfcn.h>
+#include <pthread.h>
+#include <sched.h>
+#include <sys/mman.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cmath>
+#include <condition_variable>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <deque>
+#include <functional>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include <nccl.h>
+
+#include "sh_internal.hpp"
+
+namespace sh {
+const char* last_error_cstr();
+}
+
+using namespace sh;
+
+namespace {
+
+constexpr int64_t kInf = INT64_MAX / 4;
+constexpr int64_t kPinned = -1;
+constexpr int64_t kCpuChunk = 1 << 18;  // elements per CPU Adam task chunk (~7.5 MB of traffic)
+
+double now_ms() {
+  return std::chrono::duration<double, std::milli>(
+             std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
+int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+double wait_timeout_s() {
+  const char* e = getenv("SH_WAIT_TIMEOUT_S");
+  return e ? atof(e) : 600.0;
+}
+
+// ---- NCCL (dlopen'ed: the process must share torch's libnccl.so.2) ------------------------
+struct Nccl {
+  void* h = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+  bool load() {
+    if (h) return true;
+    const char* names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char* n : names) {
+      h = dlopen(n, RTLD_NOW | RTLD_NOLOAD | RTLD_GLOBAL);
+      if (!h) h = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+      if (h) break;
+    }
+    if (!h) return false;
+    GetUniqueId = (decltype(GetUniqueId))dlsym(h, "ncclGetUniqueId");
+    CommInitRank = (decltype(CommInitRank))dlsym(h, "ncclCommInitRank");
+    AllReduce = (decltype(AllReduce))dlsym(h, "ncclAllReduce");
+    CommDestroy = (decltype(CommDestroy))dlsym(h, "ncclCommDestroy");
+    GetErrorString = (decltype(GetErrorString))dlsym(h, "ncclGetErrorString");
+    return GetUniqueId && CommInitRank && AllReduce && CommDestroy && GetErrorString;
+  }
+};
+Nccl g_nccl;
+
+// ---- FIFO issuer thread (owns one copy stream) --------------------------------------------
+class Issuer {
+ public:
+  void start() { th_ = std::thread([this] { loop(); }); }
+  void push(std::function<void()> f) {
+    {
+      std::lock_guard<std::mutex> g(mu_);
+      q_.push_back(std::move(f));
+      ++pushed_;
+    }
+    cv_.notify_one();
+  }
+  void drain() {  // block until every pushed closure has run
+    std::unique_lock<std::mutex> g(mu_);
+    cv_done_.wait(g, [&] { return done_ == pushed_; });
+  }
+  void stop() {
+    {
+      std::lock_guard<std::mutex> g(mu_);
+      stop_ = true;
+    }
+    cv_.notify_one();
+    if (th_.joinable()) th_.join();
+  }
+
+ private:
+  void loop() {
+    for (;;) {
+      std::function<void()> f;
+      {
+        std::unique_lock<std::mutex> g(mu_);
+        cv_.wait(g, [&] { return stop_ || !q_.empty(); });
+        if (q_.empty()) return;
+        f = std::move(q_.front());
+        q_.pop_front();
+      }
+      f();
+      {
+        std::lock_guard<std::mutex> g(mu_);
+        ++done_;
+      }
+      cv_done_.notify_all();
+    }
+  }
+  std::thread th_;
+  std::mutex mu_;
+  std::condition_variable cv_, cv_done_;
+  std::deque<std::function<void()>> q_;
+  int64_t pushed_ = 0, done_ = 0;
+  bool stop_ = false;
+};
+
+struct ProfSet {  // CUDA timing events of one step (double-buffered by step parity)
+  std::vector<cudaEvent_t> fp0, fp1, bp0, bp1, c2g0[2], c2g1[2], g2c0, g2c1, st0, st1;
+  std::vector<std::atomic<uint8_t>> rec_c2g[2], rec_g2c, rec_st;
+  std::vector<uint8_t> rec_fp, rec_bp;
+  cudaEvent_t k2a = nullptr, k2b = nullptr;
+  bool rec_k2 = false;
+  bool active = false;
+  int64_t step = -1;
+  int64_t k2_bytes = 0;
+  int k2_launches = 0;
+};
+
+}  // namespace
+
+struct GState {
+  float* master = nullptr;
+  float* m = nullptr;
+  float* v = nullptr;
+};
+
+struct Job {
+  int layer;
+  int64_t step;
+  int landing;
+  int64_t n_chunks;
+  int64_t next = 0;
+  std::atomic<int64_t> done{0};
+  sh_adam_scalars sc;
+};
+
+struct sh_ctx {
+  // ---- configuration
+  sh_config cfg{};
+  int L = 0;
+  std::vector<LayerLayout> lay;
+  LayerLayout res;
+  bool bf16 = true;
+  int cb = 2;
+  int64_t max_pad = 0;
+  int64_t slot_param_bytes = 0, slot_grad_bytes = 0, slot_bytes = 0;
+  int w = 0;
+  int n_slots = 0;   // allocated
+  int n_active = 0;  // used = w+1
+  int D = 0;         // host landing buffers
+  bool clip = false;
+  int warmup = 5;
+  bool autotune_pending = false;
+  int W = 1, rank = 0;
+
+  // ---- streams
+  cudaStream_t cs = nullptr, h2d = nullptr, d2h = nullptr, stage = nullptr, comm = nullptr;
+  ncclComm_t nccl = nullptr;
+
+  // ---- device memory
+  char* ring = nullptr;
+  std::vector<GState> g;  // [L]
+  float *res_master = nullptr, *res_m = nullptr, *res_v = nullptr, *res_grad = nullptr;
+  void* res_compute = nullptr;
+  double* partials = nullptr;  // [L+1]
+  double* scratch_cs = nullptr;
+  double* scratch_comm = nullptr;
+  double* norm_dev = nullptr;
+  float* coef_dev = nullptr;
+  int64_t device_bytes = 0;
+
+  // ---- host store
+  char* host_base = nullptr;
+  size_t host_bytes = 0;
+  std::vector<float*> h_master, h_m, h_v;
+  std::vector<uint16_t*> h_shadow;
+  std::vector<float*> landing;
+  float* h_coef = nullptr;  // pinned [2]
+  std::vector<uint8_t> registered;
+
+  // ---- ring state (driver thread only, except *_pub / ready / landing_done)
+  std::vector<int> slot_layer, layer_slot;
+  std::vector<cudaEvent_t> ev_param_free, ev_grad_done, ev_grad_free, ev_reduced;
+  std::vector<int64_t> gradfree_gen, gradfree_waited;
+  std::unique_ptr<std::atomic<int64_t>[]> gradfree_pub;
+  std::vector<cudaEvent_t> ev_arrive;
+  std::vector<int64_t> arrive_gen, compute_waited;
+  std::vector<uint8_t> arrive_by_issuer;
+  std::unique_ptr<std::atomic<int64_t>[]> arrive_pub;
+  std::unique_ptr<std::atomic<int64_t>[]> ready;  // updates applied to layer j
+  std::unique_ptr<std::atomic<int64_t>[]> landing_done;
+  std::vector<int64_t> landing_uses;
+  int64_t landing_rr = 0;
+  int64_t gen = 0;
+  std::mutex smu;
+  std::condition_variable scv;
+
+  // ---- protocol
+  enum Phase { IDLE, FP, BP } phase = IDLE;
+  int last_layer = -1;
+  int last_hook = SH_POST;
+  int64_t step = 0;
+  bool registered_all = false;
+  std::vector<uint8_t> reg_done;
+  bool res_reg = false;
+  float lr = 0;
+  sh_adam_scalars sc{};
+  cudaEvent_t ev_comm_done = nullptr, ev_cs_mark = nullptr;
+
+  // ---- CPU Adam pool
+  std::vector<std::thread> workers;
+  std::mutex pmu;
+  std::condition_variable pcv;
+  std::deque<std::unique_ptr<Job>> jobs;
+  std::vector<float> coef_of_step;  // clip coefficient per step parity slot
+  std::vector<int64_t> coef_step;   // which step the value belongs to
+  bool pool_stop = false;
+  int n_threads = 0;
+
+  // ---- issuers
+  Issuer ih2d, id2h;
+
+  // ---- profiling
+  ProfSet prof[2];
+  std::vector<double> p_fp, p_bp, p_c2g, p_g2c, p_stage, p_ogpu, p_ocpu, p_slot, p_gstate;
+  std::vector<int64_t> p_slot_i, p_gstate_i;
+  std::vector<double> cpu_ms_layer;  // host timing of CPU Adam per layer (last)
+  double t_async_ms = 0.0;
+  int64_t n_async = 0;
+  int profiled_steps = 0;
+
+  // ---- stats
+  std::atomic<int64_t> h2d_bytes{0}, d2h_bytes{0}, h2d_copies{0}, d2h_copies{0}, stage_launches{0};
+  std::atomic<int64_t> cpu_elems{0};
+  std::atomic<double> cpu_ms{0.0}, cpu_wait_ms{0.0};
+  double h2d_busy = 0, d2h_busy = 0;
+  int64_t h2d_prof_bytes = 0, d2h_prof_bytes = 0;
+  double k2_ms_last = 0;
+  int64_t k2_bytes_last = 0;
+  int k2_launches_last = 0;
+
+  // ---- failure
+  std::atomic<int> failed{0};
+  std::mutex emu;
+  std::string async_err;
+  int async_status = SH_OK;
+
+  bool is_g(int x) const { return x < w; }
+  char* slot_param(int s) const { return ring + (int64_t)s * slot_bytes; }
+  float* slot_grad(int s) const {
+    return reinterpret_cast<float*>(ring + (int64_t)s * slot_bytes + slot_param_bytes);
+  }
+  int layer_at(int pos) const { return pos < L ? pos : 2 * L - 1 - pos; }
+};
+
+namespace {
+
+// ---------------------------------------------------------------------------- failure
+void async_fail(sh_ctx* c, int status, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  {
+    std::lock_guard<std::mutex> g(c->emu);
+    if (c->async_status == SH_OK) {
+      c->async_status = status;
+      c->async_err = buf;
+    }
+  }
+  c->failed.store(1);
+  {
+    std::lock_guard<std::mutex> g(c->smu);
+  }
+  c->scv.notify_all();
+  c->pcv.notify_all();
+}
+
+sh_status check_failed(sh_ctx* c) {
+  if (!c->failed.load()) return SH_OK;
+  std::lock_guard<std::mutex> g(c->emu);
+  set_error("context failed: %s", c->async_err.c_str());
+  return SH_ERR_STATE;
+}
+
+#define CKC(c, expr)                                                                     \
+  do {                                                                                   \
+    cudaError_t e_ = (expr);                                                             \
+    if (e_ != cudaSuccess) {                                                             \
+      async_fail((c), SH_ERR_CUDA, "%s failed: %s", #expr, cudaGetErrorString(e_));      \
+      set_error("%s failed: %s", #expr, cudaGetErrorString(e_));                         \
+      return SH_ERR_CUDA;                                                                \
+    }                                                                                    \
+  } while (0)
+
+#define CKA(c, expr)                                                                     \
+  do {                                                                                   \
+    cudaError_t e_ = (expr);                                                             \
+    if (e_ != cudaSuccess) async_fail((c), SH_ERR_CUDA, "%s: %s", #expr, cudaGetErrorString(e_)); \
+  } while (0)
+
+// Wait on the engine state condition (timeout => fail, never hang the box).
+template <class Pred>
+bool state_wait(sh_ctx* c, Pred pred, const char* what, double* waited_ms = nullptr) {
+  if (pred()) return true;
+  const double t0 = now_ms();
+  std::unique_lock<std::mutex> g(c->smu);
+  const bool ok = c->scv.wait_for(g, std::chrono::duration<double>(wait_timeout_s()),
+                                  [&] { return c->failed.load() || pred(); });
+  if (waited_ms) *waited_ms = now_ms() - t0;
+  if (!ok) {
+    g.unlock();
+    async_fail(c, SH_ERR_STATE, "timeout waiting for %s", what);
+    return false;
+  }
+  return !c->failed.load();
+}
+
+void notify_state(sh_ctx* c) {
+  { std::lock_guard<std::mutex> g(c->smu); }
+  c->scv.notify_all();
+}
+
+// ---------------------------------------------------------------------------- host store
+void* host_alloc(size_t bytes) {
+  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+  if (p == MAP_FAILED) return nullptr;
+  madvise(p, bytes, MADV_HUGEPAGE);
+  return p;
+}
+
+// first touch in parallel (pages land on the toucher's node; THP => 2 MiB pages)
+void parallel_touch(char* p, size_t bytes, int threads) {
+  const size_t chunk = align_up((int64_t)(bytes / std::max(threads, 1) + 1), 1 << 21);
+  std::vector<std::thread> ts;
+  for (size_t off = 0; off < bytes; off += chunk) {
+    const size_t n = std::min(chunk, bytes - off);
+    ts.emplace_back([=] { std::memset(p + off, 0, n); });
+  }
+  for (auto& t : ts) t.join();
+}
+
+// ---------------------------------------------------------------------------- CPU Adam pool
+void finish_job(sh_ctx* c, Job* j) {
+  c->ready[j->layer].store(j->step + 1, std::memory_order_release);
+  c->landing_done[j->landing].fetch_add(1, std::memory_order_release);
+  notify_state(c);
+}
+
+void worker_loop(sh_ctx* c, int tid) {
+  (void)tid;
+  for (;;) {
+    Job* job = nullptr;
+    int64_t chunk = -1;
+    float coef = 1.0f;
+    {
+      std::unique_lock<std::mutex> g(c->pmu);
+      c->pcv.wait(g, [&] {
+        if (c->pool_stop || c->failed.load()) return true;
+        for (auto& jp : c->jobs) {
+          if (jp->next >= jp->n_chunks) continue;
+          if (c->clip && c->coef_step[jp->step & 1] != jp->step) continue;
+          return true;
+        }
+        return false;
+      });
+      if (c->pool_stop || c->failed.load()) return;
+      // lowest layer first: it is prefetched first by the next FP (eq. 3)
+      for (auto& jp : c->jobs) {
+        if (jp->next >= jp->n_chunks) continue;
+        if (c->clip && c->coef_step[jp->step & 1] != jp->step) continue;
+        if (!job || jp->step < job->step || (jp->step == job->step && jp->layer < job->layer))
+          job = jp.get();
+      }
+      chunk = job->next++;
+      if (c->clip) coef = c->coef_of_step[job->step & 1];
+    }
+    const double t0 = now_ms();
+    const int x = job->layer;
+    const LayerLayout& Lx = c->lay[x];
+    const int64_t b = chunk * kCpuChunk, e = std::min(Lx.n_pad, b + kCpuChunk);
+    cpu::adamw_range(c->h_master[x], c->h_m[x], c->h_v[x], c->landing[job->landing],
+                     c->bf16 ? c->h_shadow[x] : nullptr, b, e, Lx.n_decay, job->sc, c->clip, coef);
+    const double dt = now_ms() - t0;
+    double cur = c->cpu_ms.load();
+    while (!c->cpu_ms.compare_exchange_weak(cur, cur + dt)) {
+    }
+    c->cpu_elems.fetch_add(e - b);
+    if (job->done.fetch_add(1) + 1 == job->n_chunks) {
+      finish_job(c, job);
+      std::lock_guard<std::mutex> g(c->pmu);
+      for (auto it = c->jobs.begin(); it != c->jobs.end(); ++it)
+        if (it->get() == job) {
+          c->jobs.erase(it);
+          break;
+        }
+    }
+  }
+}
+
+struct Landed {
+  sh_ctx* c;
+  int layer;
+  int64_t step;
+  int landing;
+  sh_adam_scalars sc;
+};
+
+void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA calls here
+  std::unique_ptr<Landed> L(static_cast<Landed*>(arg));
+  sh_ctx* c = L->c;
+  auto j = std::make_unique<Job>();
+  j->layer = L->layer;
+  j->step = L->step;
+  j->landing = L->landing;
+  j->n_chunks = (c->lay[L->layer].n_pad + kCpuChunk - 1) / kCpuChunk;
+  j->sc = L->sc;
+  if (c->cfg.flags & SH_FLAG_SYNC_CPU) {  // debug: inline, single-threaded
+    Job* jp = j.get();
+    float coef = c->clip ? c->coef_of_step[jp->step & 1] : 1.0f;
+    cpu::adamw_range(c->h_master[jp->layer], c->h_m[jp->layer], c->h_v[jp->layer],
+                     c->landing[jp->landing], c->bf16 ? c->h_shadow[jp->layer] : nullptr, 0,
+                     c->lay[jp->layer].n_pad, c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
+    finish_job(c, jp);
+    return;
+  }
+  {
+    std::lock_guard<std::mutex> g(c->pmu);
+    c->jobs.push_back(std::move(j));
+  }
+  c->pcv.notify_all();
+}
+
+struct CoefMsg {
+  sh_ctx* c;
+  int64_t step;
+};
+void CUDART_CB coef_cb(void* arg) {
+  std::unique_ptr<CoefMsg> m(static_cast<CoefMsg*>(arg));
+  sh_ctx* c = m->c;
+  {
+    std::lock_guard<std::mutex> g(c->pmu);
+    c->coef_of_step[m->step & 1] = c->h_coef[m->step & 1];
+    c->coef_step[m->step & 1] = m->step;
+  }
+  c->pcv.notify_all();
+}
+
+// ---------------------------------------------------------------------------- profiling
+sh_status prof_alloc(sh_ctx* c, ProfSet& P) {
+  auto mk = [&](std::vector<cudaEvent_t>& v) -> cudaError_t {
+    v.assign(c->L, nullptr);
+    for (auto& e : v) {
+      cudaError_t r = cudaEventCreate(&e);
+      if (r != cudaSuccess) return r;
+    }
+    return cudaSuccess;
+  };
+  cudaError_t r = cudaSuccess;
+  for (auto* v : {&P.fp0, &P.fp1, &P.bp0, &P.bp1, &P.c2g0[0], &P.c2g1[0], &P.c2g0[1], &P.c2g1[1],
+                  &P.g2c0, &P.g2c1, &P.st0, &P.st1})
+    if (r == cudaSuccess) r = mk(*v);
+  if (r == cudaSuccess) r = cudaEventCreate(&P.k2a);
+  if (r == cudaSuccess) r = cudaEventCreate(&P.k2b);
+  if (r != cudaSuccess) {
+    set_error("cudaEventCreate: %s", cudaGetErrorString(r));
+    return SH_ERR_CUDA;
+  }
+  P.rec_c2g[0] = std::vector<std::atomic<uint8_t>>(c->L);
+  P.rec_c2g[1] = std::vector<std::atomic<uint8_t>>(c->L);
+  P.rec_g2c = std::vector<std::atomic<uint8_t>>(c->L);
+  P.rec_st = std::vector<std::atomic<uint8_t>>(c->L);
+  P.rec_fp.assign(c->L, 0);
+  P.rec_bp.assign(c->L, 0);
+  return SH_OK;
+}
+
+void prof_reset(sh_ctx* c, ProfSet& P, int64_t step) {
+  for (int i = 0; i < c->L; ++i) {
+    P.rec_c2g[0][i] = 0;
+    P.rec_c2g[1][i] = 0;
+    P.rec_g2c[i] = 0;
+    P.rec_st[i] = 0;
+    P.rec_fp[i] = 0;
+    P.rec_bp[i] = 0;
+  }
+  P.rec_k2 = false;
+  P.active = true;
+  P.step = step;
+}
+
+float ev_ms(cudaEvent_t a, cudaEvent_t b) {
+  float ms = 0;
+  if (cudaEventSynchronize(b) != cudaSuccess) return 0;
+  if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) return 0;
+  return ms;
+}
+
+// Read the events of a finished profiled step into the profile arrays and the stats.
+void prof_harvest(sh_ctx* c, ProfSet& P) {
+  if (!P.active) return;
+  P.active = false;
+  const int L = c->L;
+  for (int i = 0; i < L; ++i) {
+    if (P.rec_fp[i]) c->p_fp[i] = ev_ms(P.fp0[i], P.fp1[i]);
+    if (P.rec_bp[i]) c->p_bp[i] = ev_ms(P.bp0[i], P.bp1[i]);
+    for (int ph = 0; ph < 2; ++ph)
+      if (P.rec_c2g[ph][i]) {
+        const double ms = ev_ms(P.c2g0[ph][i], P.c2g1[ph][i]);
+        c->p_c2g[i] = ms;
+        c->h2d_busy += ms;
+        c->h2d_prof_bytes += (int64_t)c->cb * c->lay[i].n_pad;
+      }
+    if (P.rec_g2c[i]) {
+      const double ms = ev_ms(P.g2c0[i], P.g2c1[i]);
+      c->p_g2c[i] = ms;
+      c->d2h_busy += ms;
+      c->d2h_prof_bytes += 4 * c->lay[i].n_pad;
+    }
+    if (P.rec_st[i]) c->p_stage[i] = ev_ms(P.st0[i], P.st1[i]);
+  }
+  if (P.rec_k2) {
+    c->k2_ms_last = ev_ms(P.k2a, P.k2b);
+    c->k2_bytes_last = P.k2_bytes;
+    c->k2_launches_last = P.k2_launches;
+    // apportion K2 time to layers by bytes (one fused launch covers all of them)
+    double tot = 0;
+    for (int i = 0; i < L; ++i) tot += c->lay[i].n_pad;
+    for (int i = 0; i < L; ++i)
+      c->p_ogpu[i] = P.k2_bytes > 0 ? c->k2_ms_last * (30.0 * c->lay[i].n_pad) / P.k2_bytes : 0.0;
+  }
+  c->profiled_steps++;
+}
+
+bool step_profiled(sh_ctx* c, int64_t step) {
+  return (c->cfg.flags & SH_FLAG_PROFILE) || step < c->warmup || c->autotune_pending;
+}
+
+ProfSet* cur_prof(sh_ctx* c) {
+  ProfSet& P = c->prof[c->step & 1];
+  return (P.active && P.step == c->step) ? &P : nullptr;
+}
+
+// ---------------------------------------------------------------------------- ring logic
+int64_t next_use(const sh_ctx* c, int x, int cur) {
+  if (x >= cur) return x;  // FP use still ahead
+  const int b = 2 * c->L - 1 - x;
+  if (b >= cur) return b;  // BP use still ahead
+  return c->is_g(x) ? kPinned : kInf;  // G grads wait for K2; host copies go stale
+}
+
+sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
+  const int old = c->slot_layer[s];
+  if (old >= 0) c->layer_slot[old] = -1;
+  c->slot_layer[s] = y;
+  c->layer_slot[y] = s;
+  const int64_t gen = ++c->gen;
+  c->arrive_gen[y] = gen;
+  char* dst = c->slot_param(s);
+  const int64_t n = c->lay[y].n_pad;
+  const bool poison = c->cfg.flags & SH_FLAG_POISON;
+  ProfSet* P = cur_prof(c);
+  const int ph = pos < c->L ? 0 : 1;
+  if (c->is_g(y)) {
+    // K1 restage from the HBM master (GPU-optimised layer evicted during FP)
+    CKC(c, cudaStreamWaitEvent(c->stage, c->ev_param_free[s], 0));
+    if (poison) CKC(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->stage));
+    if (P) CKC(c, cudaEventRecord(P->st0[y], c->stage));
+    if (c->bf16)
+      CKC(c, kern::cast_bf16(c->g[y].master, reinterpret_cast<uint16_t*>(dst), n, c->stage));
+    else
+      CKC(c, cudaMemcpyAsync(dst, c->g[y].master, 4 * n, cudaMemcpyDeviceToDevice, c->stage));
+    if (P) {
+      CKC(c, cudaEventRecord(P->st1[y], c->stage));
+      P->rec_st[y] = 1;
+    }
+    CKC(c, cudaEventRecord(c->ev_arrive[y], c->stage));
+    c->arrive_by_issuer[y] = 0;
+    c->arrive_pub[y].store(gen);
+    c->stage_launches++;
+    return SH_OK;
+  }
+  c->arrive_by_issuer[y] = 1;
+  const int64_t need = c->step;
+  const void* src = c->bf16 ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];
+  const int64_t bytes = (int64_t)c->cb * n;
+  cudaEvent_t pf = c->ev_param_free[s];
+  c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph] {
+    double waited = 0;
+    if (!state_wait(c, [&] { return c->ready[y].load(std::memory_order_acquire) >= need; },
+                    "CPU Adam of a layer to prefetch", &waited)) {
+      c->arrive_pub[y].store(kInf);
+      notify_state(c);
+      return;
+    }
+    if (waited > 0) {
+      double cur = c->cpu_wait_ms.load();
+      while (!c->cpu_wait_ms.compare_exchange_weak(cur, cur + waited)) {
+      }
+    }
+    CKA(c, cudaStreamWaitEvent(c->h2d, pf, 0));
+    if (poison) CKA(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->h2d));
+    if (P) CKA(c, cudaEventRecord(P->c2g0[ph][y], c->h2d));
+    CKA(c, cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, c->h2d));
+    if (P) {
+      CKA(c, cudaEventRecord(P->c2g1[ph][y], c->h2d));
+      P->rec_c2g[ph][y] = 1;
+    }
+    CKA(c, cudaEventRecord(c->ev_arrive[y], c->h2d));
+    c->h2d_bytes += bytes;
+    c->h2d_copies++;
+    c->arrive_pub[y].store(gen);
+    notify_state(c);
+  });
+  return SH_OK;
+}
+
+// Make sure the layer used at position p is in the ring; false if no slot can take it yet.
+bool ensure_at(sh_ctx* c, int p, int cur, sh_status* st) {
+  *st = SH_OK;
+  const int y = c->layer_at(p);
+  if (c->layer_slot[y] >= 0) return true;
+  int best = -1;
+  int64_t best_nu = -2;
+  for (int s = 0; s < c->n_active; ++s) {
+    const int o = c->slot_layer[s];
+    const int64_t nu = o < 0 ? kInf + 1 : next_use(c, o, cur);
+    if (nu == kPinned || nu <= p) continue;
+    if (nu > best_nu) best_nu = nu, best = s;
+  }
+  if (best < 0) return false;
+  *st = issue_fetch(c, y, best, p);
+  return *st == SH_OK;
+}
+
+// Common PRE work: ensure the current layer, prefetch the window ahead, wait for arrival.
+sh_status pre_common(sh_ctx* c, int x, int pos) {
+  sh_status st;
+  const int last = std::min(pos + c->w, 2 * c->L - 1);
+  for (int p = pos; p <= last; ++p) {
+    const bool ok = ensure_at(c, p, pos, &st);
+    if (st != SH_OK) return st;
+    if (!ok) {
+      if (p == pos) {
+        set_error("internal: no ring slot for layer %d at position %d", x, pos);
+        return SH_ERR_STATE;
+      }
+      break;
+    }
+  }
+  if (c->arrive_gen[x] > c->compute_waited[x]) {
+    const int64_t gen = c->arrive_gen[x];
+    if (c->arrive_by_issuer[x] &&
+        !state_wait(c, [&] { return c->arrive_pub[x].load() >= gen; }, "prefetch issue"))
+      return check_failed(c);
+    CKC(c, cudaStreamWaitEvent(c->cs, c->ev_arrive[x], 0));
+    c->compute_waited[x] = gen;
+  }
+  return check_failed(c);
+}
+
+void fill_param_ptrs(sh_ctx* c, int x, void** out) {
+  const LayerLayout& Lx = c->lay[x];
+  char* base = c->slot_param(c->layer_slot[x]);
+  for (int k = 0; k < Lx.n_tensors; ++k) out[k] = base + (int64_t)c->cb * Lx.offset[k];
+}
+
+sh_status stage_g_layers(sh_ctx* c) {
+  // ring reset: G layers 0..w-1 into slots 0..w-1 (compute stream), the rest empty
+  for (int s = 0; s < c->n_slots; ++s) c->slot_layer[s] = -1;
+  for (int x = 0; x < c->L; ++x) c->layer_slot[x] = -1;
+  for (int x = 0; x < c->w; ++x) {
+    c->slot_layer[x] = x;
+    c->layer_slot[x] = x;
+    char* dst = c->slot_param(x);
+    if (c->bf16)
+      CKC(c, kern::cast_bf16(c->g[x].master, reinterpret_cast<uint16_t*>(dst), c->lay[x].n_pad, c->cs));
+    else
+      CKC(c, cudaMemcpyAsync(dst, c->g[x].master, 4 * c->lay[x].n_pad, cudaMemcpyDeviceToDevice, c->cs));
+  }
+  return SH_OK;
+}
+
+sh_status alloc_g(sh_ctx* c, int x) {
+  if (c->g[x].master) return SH_OK;
+  const int64_t n = c->lay[x].n_pad;
+  float* p = nullptr;
+  if (cudaMalloc(&p, 3 * 4 * n) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("cudaMalloc of GPU-optimised state for layer %d (%lld B) failed", x, (long long)(12 * n));
+    return SH_ERR_OOM_DEVICE;
+  }
+  c->g[x].master = p;
+  c->g[x].m = p + n;
+  c->g[x].v = p + 2 * n;
+  c->device_bytes += 12 * n;
+  return SH_OK;
+}
+
+void free_g(sh_ctx* c, int x) {
+  if (!c->g[x].master) return;
+  cudaFree(c->g[x].master);
+  c->device_bytes -= 12 * c->lay[x].n_pad;
+  c->g[x] = GState{};
+}
+
+sh_status alloc_ring(sh_ctx* c, int n_slots) {
+  if (n_slots <= c->n_slots) return SH_OK;
+  char* r = nullptr;
+  if (cudaMalloc(&r, (int64_t)n_slots * c->slot_bytes) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("cudaMalloc of %d ring slots (%lld B each) failed", n_slots, (long long)c->slot_bytes);
+    return SH_ERR_OOM_DEVICE;
+  }
+  if (c->ring) {
+    cudaFree(c->ring);
+    c->device_bytes -= (int64_t)c->n_slots * c->slot_bytes;
+  }
+  c->ring = r;
+  c->device_bytes += (int64_t)n_slots * c->slot_bytes;
+  cudaMemset(r, 0, (int64_t)n_slots * c->slot_bytes);
+  const int old = c->n_slots;
+  c->slot_layer.resize(n_slots, -1);
+  c->ev_param_free.resize(n_slots, nullptr);
+  c->ev_grad_done.resize(n_slots, nullptr);
+  c->ev_grad_free.resize(n_slots, nullptr);
+  c->ev_reduced.resize(n_slots, nullptr);
+  c->gradfree_gen.resize(n_slots, 0);
+  c->gradfree_waited.resize(n_slots, 0);
+  auto pub = std::make_unique<std::atomic<int64_t>[]>(n_slots);
+  for (int s = 0; s < n_slots; ++s) pub[s].store(s < old ? c->gradfree_pub[s].load() : 0);
+  c->gradfree_pub = std::move(pub);
+  for (int s = old; s < n_slots; ++s) {
+    for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced})
+      if (cudaEventCreateWithFlags(&(*v)[s], cudaEventDisableTiming) != cudaSuccess) {
+        set_error("cudaEventCreate failed");
+        return SH_ERR_CUDA;
+      }
+    // a fresh slot is free: record once so every wait has a completed event
+    cudaEventRecord(c->ev_param_free[s], c->cs);
+    cudaEventRecord(c->ev_grad_free[s], c->cs);
+  }
+  c->n_slots = n_slots;
+  return SH_OK;
+}
+
+sh_status sync_all(sh_ctx* c) {
+  c->ih2d.drain();
+  c->id2h.drain();
+  for (cudaStream_t s : {c->cs, c->h2d, c->d2h, c->stage, c->comm})
+    if (s) CKC(c, cudaStreamSynchronize(s));
+  // all host layers updated for the steps taken so far
+  if (!state_wait(c, [&] {
+        for (int x = 0; x < c->L; ++x)
+          if (!c->is_g(x) && c->ready[x].load() < c->step) return false;
+        return true;
+      }, "CPU Adam drain"))
+    return check_failed(c);
+  for (auto& P : c->prof) prof_harvest(c, P);
+  return check_failed(c);
+}
+
+// Move the G boundary from c->w to w_new (between steps, everything idle).
+sh_status apply_window(sh_ctx* c, int w_new) {
+  sh_status st = sync_all(c);
+  if (st != SH_OK) return st;
+  const int w_old = c->w;
+  // leaving G: HBM -> host store (bitwise), shadow recomputed with the same RNE
+  for (int x = w_new; x < w_old; ++x) {
+    const int64_t n = c->lay[x].n_pad;
+    CKC(c, cudaMemcpy(c->h_master[x], c->g[x].master, 4 * n, cudaMemcpyDeviceToHost));
+    CKC(c, cudaMemcpy(c->h_m[x], c->g[x].m, 4 * n, cudaMemcpyDeviceToHost));
+    CKC(c, cudaMemcpy(c->h_v[x], c->g[x].v, 4 * n, cudaMemcpyDeviceToHost));
+    if (c->bf16) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], 0, n);
+    c->ready[x].store(c->step);
+    free_g(c, x);
+  }
+  // joining G: host store -> HBM
+  for (int x = w_old; x < w_new; ++x) {
+    st = alloc_g(c, x);
+    if (st != SH_OK) return st;
+    const int64_t n = c->lay[x].n_pad;
+    CKC(c, cudaMemcpy(c->g[x].master, c->h_master[x], 4 * n, cudaMemcpyHostToDevice));
+    CKC(c, cudaMemcpy(c->g[x].m, c->h_m[x], 4 * n, cudaMemcpyHostToDevice));
+    CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
+  }
+  st = alloc_ring(c, w_new + 1);
+  if (st != SH_OK) return st;
+  c->w = w_new;
+  c->n_active = w_new + 1;
+  st = stage_g_layers(c);
+  if (st != SH_OK) return st;
+  CKC(c, cudaStreamSynchronize(c->cs));
+  return SH_OK;
+}
+
+sh_status push_k2(sh_ctx* c, kern::K2Args& a, int64_t* bytes, int* launches) {
+  if (a.n_entries == 0) return SH_OK;
+  for (int i = 0; i < a.n_entries; ++i) *bytes += (c->bf16 ? 30 : 32) * a.e[i].n;
+  CKC(c, kern::adamw_multi(a, c->cs));
+  (*launches)++;
+  a.n_entries = 0;
+  return SH_OK;
+}
+
+sh_status nccl_check(sh_ctx* c, ncclResult_t r, const char* what) {
+  if (r == ncclSuccess) return SH_OK;
+  async_fail(c, SH_ERR_NCCL, "%s: %s", what, g_nccl.GetErrorString(r));
+  set_error("%s: %s", what, g_nccl.GetErrorString(r));
+  return SH_ERR_NCCL;
+}
+
+}  // namespace
+
+// =============================================================================== C ABI
+extern "C" {
+
+int32_t sh_abi_version(void) { return SH_ABI_VERSION; }
+const char* sh_last_error(void) { return sh::last_error_cstr(); }
+
+sh_status sh_nccl_get_unique_id(void* out128) {
+  clear_error();
+  if (!out128) return SH_ERR_INVALID;
+  if (!g_nccl.load()) {
+    set_error("libnccl.so.2 not loadable");
+    return SH_ERR_UNSUPPORTED;
+  }
+  ncclUniqueId id;
+  if (g_nccl.GetUniqueId(&id) != ncclSuccess) {
+    set_error("ncclGetUniqueId failed");
+    return SH_ERR_NCCL;
+  }
+  std::memcpy(out128, &id, sizeof(id));
+  return SH_OK;
+}
+
+sh_status sh_adam_scalars_for(float lr, float beta1, float beta2, float eps, float weight_decay,
+                              int64_t t, sh_adam_scalars* o) {
+  if (!o || t < 1) {
+    set_error("sh_adam_scalars_for: t must be >= 1");
+    return SH_ERR_INVALID;
+  }
+  const double bc1 = 1.0 - std::pow((double)beta1, (double)t);
+  const double bc2 = 1.0 - std::pow((double)beta2, (double)t);
+  o->beta1 = beta1;
+  o->beta2 = beta2;
+  o->omb1 = (float)(1.0 - (double)beta1);
+  o->omb2 = (float)(1.0 - (double)beta2);
+  o->eps = eps;
+  o->step_size = (float)((double)lr / bc1);
+  o->sqrt_bc2 = (float)std::sqrt(bc2);
+  o->decay = (float)(1.0 - (double)lr * (double)weight_decay);
+  return SH_OK;
+}
+
+sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
+  clear_error();
+  if (!cfg || !out) {
+    set_error("sh_init: null argument");
+    return SH_ERR_INVALID;
+  }
+  *out = nullptr;
+  if (cfg->n_layers < 1 || !cfg->layers) {
+    set_error("sh_init: n_layers must be >= 1 with a layers array");
+    return SH_ERR_INVALID;
+  }
+  if (cfg->window < -1 || cfg->window > cfg->n_layers) {
+    set_error("sh_init: window %d outside -1..n_layers (%d)", cfg->window, cfg->n_layers);
+    return SH_ERR_INVALID;
+  }
+  if (cfg->precision != SH_FP32 && cfg->precision != SH_BF16_MIXED) {
+    set_error("sh_init: unknown precision %d", cfg->precision);
+    return SH_ERR_INVALID;
+  }
+  if (!cfg->compute_stream) {
+    set_error("sh_init: compute_stream is required (the caller's cudaStream_t)");
+    return SH_ERR_INVALID;
+  }
+  const int W = cfg->world_size < 1 ? 1 : cfg->world_size;
+  if (W > 1 && (!cfg->nccl_unique_id || cfg->rank < 0 || cfg->rank >= W)) {
+    set_error("sh_init: world_size > 1 needs nccl_unique_id and 0 <= rank < world_size");
+    return SH_ERR_INVALID;
+  }
+  auto c = std::make_unique<sh_ctx>();
+  c->cfg = *cfg;
+  c->L = cfg->n_layers;
+  c->W = W;
+  c->rank = cfg->rank;
+  c->bf16 = cfg->precision == SH_BF16_MIXED;
+  c->cb = c->bf16 ? 2 : 4;
+  c->clip = cfg->max_grad_norm > 0.0f;
+  c->warmup = cfg->warmup_steps > 0 ? cfg->warmup_steps : 5;
+  c->lr = cfg->lr;
+  c->lay.resize(c->L);
+  for (int i = 0; i < c->L; ++i) {
+    if (!make_layout(cfg->layers[i], &c->lay[i])) return SH_ERR_INVALID;
+    c->max_pad = std::max(c->max_pad, c->lay[i].n_pad);
+  }
+  if (!make_layout(cfg->resident, &c->res)) return SH_ERR_INVALID;
+  c->slot_param_bytes = align_up((int64_t)c->cb * c->max_pad, 256);
+  c->slot_grad_bytes = align_up(4 * c->max_pad, 256);
+  c->slot_bytes = c->slot_param_bytes + c->slot_grad_bytes;
+  const int w0 = cfg->window >= 0 ? cfg->window : std::min(2, c->L);
+  c->autotune_pending = cfg->window < 0;
+  c->D = cfg->grad_ring_depth > 0 ? cfg->grad_ring_depth : c->L;
+  if (c->clip && c->D < c->L) {
+    set_error("sh_init: clip mode needs grad_ring_depth 0 (one landing buffer per layer): "
+              "every host gradient must be stored until the global norm is known");
+    return SH_ERR_INVALID;
+  }
+
+  CKC(c.get(), cudaSetDevice(cfg->device));
+  c->cs = static_cast<cudaStream_t>(cfg->compute_stream);
+  CKC(c.get(), cudaStreamCreateWithFlags(&c->h2d, cudaStreamNonBlocking));
+  CKC(c.get(), cudaStreamCreateWithFlags(&c->d2h, cudaStreamNonBlocking));
+  CKC(c.get(), cudaStreamCreateWithFlags(&c->stage, cudaStreamNonBlocking));
+  CKC(c.get(), cudaEventCreateWithFlags(&c->ev_cs_mark, cudaEventDisableTiming));
+  CKC(c.get(), cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
+  if (W > 1) {
+    CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
+    if (!g_nccl.load()) {
+      set_error("sh_init: world_size > 1 but libnccl.so.2 cannot be loaded");
+      return SH_ERR_UNSUPPORTED;
+    }
+    ncclUniqueId id;
+    std::memcpy(&id, cfg->nccl_unique_id, sizeof(id));
+    sh_status s = nccl_check(c.get(), g_nccl.CommInitRank(&c->nccl, W, id, cfg->rank), "ncclCommInitRank");
+    if (s != SH_OK) return s;
+  }
+
+  // ---- host store: per layer master | m | v | shadow, plus landing buffers, 2 MiB aligned
+  c->n_threads = cfg->cpu_threads > 0 ? cfg->cpu_threads : (int)std::thread::hardware_concurrency();
+  if (c->n_threads < 1) c->n_threads = 1;
+  std::vector<int64_t> off(c->L);
+  int64_t hb = 0;
+  for (int x = 0; x < c->L; ++x) {
+    off[x] = hb;
+    const int64_t n = c->lay[x].n_pad;
+    hb += align_up(12 * n + (c->bf16 ? 2 * n : 0), 4096);
+  }
+  const int64_t land_off = align_up(hb, 1 << 21);
+  hb = land_off + (int64_t)c->D * align_up(4 * c->max_pad, 4096);
+  const int64_t coef_off = hb;
+  hb = align_up(hb + 4096, 1 << 21);
+  c->host_bytes = hb;
+  c->host_base = static_cast<char*>(host_alloc(hb));
+  if (!c->host_base) {
+    set_error("sh_init: mmap of %lld B host store failed", (long long)hb);
+    return SH_ERR_OOM_HOST;
+  }
+  parallel_touch(c->host_base, hb, c->n_threads);
+  if (cudaHostRegister(c->host_base, hb, cudaHostRegisterPortable) != cudaSuccess) {
+    cudaGetLastError();
+    munmap(c->host_base, hb);
+    c->host_base = nullptr;
+    set_error("sh_init: cudaHostRegister of %lld B failed (memlock?)", (long long)hb);
+    return SH_ERR_OOM_HOST;
+  }
+  c->h_master.resize(c->L);
+  c->h_m.resize(c->L);
+  c->h_v.resize(c->L);
+  c->h_shadow.assign(c->L, nullptr);
+  for (int x = 0; x < c->L; ++x) {
+    const int64_t n = c->lay[x].n_pad;
+    float* b = reinterpret_cast<float*>(c->host_base + off[x]);
+    c->h_master[x] = b;
+    c->h_m[x] = b + n;
+    c->h_v[x] = b + 2 * n;
+    if (c->bf16) c->h_shadow[x] = reinterpret_cast<uint16_t*>(b + 3 * n);
+  }
+  c->landing.resize(c->D);
+  for (int k = 0; k < c->D; ++k)
+    c->landing[k] = reinterpret_cast<float*>(c->host_base + land_off + (int64_t)k * align_up(4 * c->max_pad, 4096));
+  c->h_coef = reinterpret_cast<float*>(c->host_base + coef_off);
+
+  // ---- device: resident set, partials, ring, G states
+  {
+    const int64_t n = c->res.n_pad;
+    float* p = nullptr;
+    if (cudaMalloc(&p, 16 * n + (int64_t)c->cb * n) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("sh_init: cudaMalloc of resident set failed");
+      return SH_ERR_OOM_DEVICE;
+    }
+    c->res_master = p;
+    c->res_m = p + n;
+    c->res_v = p + 2 * n;
+    c->res_grad = p + 3 * n;
+    c->res_compute = p + 4 * n;
+    c->device_bytes += 16 * n + (int64_t)c->cb * n;
+    CKC(c.get(), cudaMemset(p, 0, 16 * n + (int64_t)c->cb * n));
+    double* d = nullptr;
+    const int64_t nd = (c->L + 1) + 2 * kern::kSumsqMaxBlocks + 1;
+    if (cudaMalloc(&d, nd * 8 + 64) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("sh_init: cudaMalloc of scratch failed");
+      return SH_ERR_OOM_DEVICE;
+    }
+    CKC(c.get(), cudaMemset(d, 0, nd * 8 + 64));
+    c->partials = d;
+    c->scratch_cs = d + (c->L + 1);
+    c->scratch_comm = c->scratch_cs + kern::kSumsqMaxBlocks;
+    c->norm_dev = c->scratch_comm + kern::kSumsqMaxBlocks;
+    c->coef_dev = reinterpret_cast<float*>(c->norm_dev + 1);
+  }
+  c->g.assign(c->L, GState{});
+  c->layer_slot.assign(c->L, -1);
+  c->ev_arrive.assign(c->L, nullptr);
+  for (auto& e : c->ev_arrive) CKC(c.get(), cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  c->arrive_gen.assign(c->L, 0);
+  c->compute_waited.assign(c->L, 0);
+  c->arrive_by_issuer.assign(c->L, 0);
+  c->arrive_pub = std::make_unique<std::atomic<int64_t>[]>(c->L);
+  c->ready = std::make_unique<std::atomic<int64_t>[]>(c->L);
+  for (int x = 0; x < c->L; ++x) {
+    c->arrive_pub[x].store(0);
+    c->ready[x].store(0);
+  }
+  c->landing_done = std::make_unique<std::atomic<int64_t>[]>(c->D);
+  for (int k = 0; k < c->D; ++k) c->landing_done[k].store(0);
+  c->landing_uses.assign(c->D, 0);
+  c->reg_done.assign(c->L, 0);
+  c->coef_of_step.assign(2, 1.0f);
+  c->coef_step.assign(2, -1);
+  for (auto* v : {&c->p_fp, &c->p_bp, &c->p_c2g, &c->p_g2c, &c->p_stage, &c->p_ogpu, &c->p_ocpu})
+    v->assign(c->L, 0.0);
+  c->p_slot_i.assign(c->L, c->slot_bytes);
+  c->p_gstate_i.resize(c->L);
+  for (int x = 0; x < c->L; ++x) c->p_gstate_i[x] = 12 * c->lay[x].n_pad;
+  for (auto& P : c->prof) {
+    sh_status s = prof_alloc(c.get(), P);
+    if (s != SH_OK) return s;
+  }
+  c->w = w0;
+  c->n_active = w0 + 1;
+  {
+    sh_status s = alloc_ring(c.get(), w0 + 1);
+    if (s != SH_OK) return s;
+    for (int x = 0; x < w0; ++x) {
+      s = alloc_g(c.get(), x);
+      if (s != SH_OK) return s;
+    }
+  }
+  CKC(c.get(), cudaDeviceSynchronize());
+
+  c->ih2d.start();
+  c->id2h.start();
+  for (int t = 0; t < c->n_threads; ++t) {
+    sh_ctx* cp = c.get();
+    c->workers.emplace_back([cp, t] { worker_loop(cp, t); });
+  }
+  *out = c.release();
+  return SH_OK;
+}
+
+sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, const float* m,
+                                 const float* v, int64_t step) {
+  clear_error();
+  if (!c || !params) {
+    set_error("sh_register_host_store: null argument");
+    return SH_ERR_INVALID;
+  }
+  if (c->phase != sh_ctx::IDLE || (c->step > 0 && step != c->step)) {
+    set_error("sh_register_host_store: only before the first step (or between steps with step == current)");
+    return SH_ERR_STATE;
+  }
+  if (layer < -1 || layer >= c->L) {
+    set_error("sh_register_host_store: layer %d out of range", layer);
+    return SH_ERR_INVALID;
+  }
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  if (step < 0) step = 0;
+  if (layer == -1) {
+    const int64_t n = c->res.n_pad;
+    std::vector<float> tmp(n);
+    pack_layer(c->res, params, tmp.data());
+    CKC(c, cudaMemcpy(c->res_master, tmp.data(), 4 * n, cudaMemcpyHostToDevice));
+    pack_layer(c->res, m, tmp.data());
+    CKC(c, cudaMemcpy(c->res_m, tmp.data(), 4 * n, cudaMemcpyHostToDevice));
+    pack_layer(c->res, v, tmp.data());
+    CKC(c, cudaMemcpy(c->res_v, tmp.data(), 4 * n, cudaMemcpyHostToDevice));
+    if (c->bf16)
+      CKC(c, kern::cast_bf16(c->res_master, static_cast<uint16_t*>(c->res_compute), n, c->cs));
+    else
+      CKC(c, cudaMemcpyAsync(c->res_compute, c->res_master, 4 * n, cudaMemcpyDeviceToDevice, c->cs));
+    CKC(c, cudaStreamSynchronize(c->cs));
+    c->res_reg = true;
+  } else {
+    const int x = layer;
+    const int64_t n = c->lay[x].n_pad;
+    pack_layer(c->lay[x], params, c->h_master[x]);
+    pack_layer(c->lay[x], m, c->h_m[x]);
+    pack_layer(c->lay[x], v, c->h_v[x]);
+    if (c->bf16) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], 0, n);
+    c->ready[x].store(step);
+    if (c->is_g(x)) {
+      CKC(c, cudaMemcpy(c->g[x].master, c->h_master[x], 4 * n, cudaMemcpyHostToDevice));
+      CKC(c, cudaMemcpy(c->g[x].m, c->h_m[x], 4 * n, cudaMemcpyHostToDevice));
+      CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
+    }
+    c->reg_done[x] = 1;
+  }
+  c->step = step;
+  bool all = c->res_reg;
+  for (int x = 0; x < c->L; ++x) all = all && c->reg_done[x];
+  if (all && !c->registered_all) {
+    c->registered_all = true;
+    st = stage_g_layers(c);
+    if (st != SH_OK) return st;
+    CKC(c, cudaStreamSynchronize(c->cs));
+  }
+  return SH_OK;
+}
+
+sh_status sh_set_lr(sh_ctx* c, float lr) {
+  if (!c) return SH_ERR_INVALID;
+  c->lr = lr;
+  return SH_OK;
+}
+
+sh_status sh_forward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_params) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  const double t0 = now_ms();
+  if (phase == SH_PRE) {
+    const bool start = c->phase == sh_ctx::IDLE && x == 0;
+    const bool cont = c->phase == sh_ctx::FP && c->last_hook == SH_POST && x == c->last_layer + 1;
+    if (!(start || cont) || !dev_params) {
+      set_error("sh_forward_layer(%d, PRE) out of order (phase %d, last layer %d)", x, (int)c->phase, c->last_layer);
+      return SH_ERR_STATE;
+    }
+    if (start) {
+      if (!c->registered_all) {
+        set_error("sh_forward_layer: register every layer and the resident set first");
+        return SH_ERR_STATE;
+      }
+      // harvest the profile of step-2 (its issuer work is complete by the ready chain)
+      prof_harvest(c, c->prof[c->step & 1]);
+      if (step_profiled(c, c->step)) prof_reset(c, c->prof[c->step & 1], c->step);
+      CKC(c, cudaMemsetAsync(c->res_grad, 0, 4 * c->res.n_pad, c->cs));
+      c->phase = sh_ctx::FP;
+    }
+    st = pre_common(c, x, x);
+    if (st != SH_OK) return st;
+    if (ProfSet* P = cur_prof(c)) {
+      CKC(c, cudaEventRecord(P->fp0[x], c->cs));
+    }
+    fill_param_ptrs(c, x, dev_params);
+    c->last_layer = x;
+    c->last_hook = SH_PRE;
+  } else if (phase == SH_POST) {
+    if (!(c->phase == sh_ctx::FP && c->last_hook == SH_PRE && x == c->last_layer)) {
+      set_error("sh_forward_layer(%d, POST) out of order", x);
+      return SH_ERR_STATE;
+    }
+    if (ProfSet* P = cur_prof(c)) {
+      CKC(c, cudaEventRecord(P->fp1[x], c->cs));
+      P->rec_fp[x] = 1;
+    }
+    CKC(c, cudaEventRecord(c->ev_param_free[c->layer_slot[x]], c->cs));
+    c->last_hook = SH_POST;
+  } else {
+    set_error("sh_forward_layer: bad phase %d", phase);
+    return SH_ERR_INVALID;
+  }
+  c->t_async_ms += now_ms() - t0;
+  c->n_async++;
+  return SH_OK;
+}
+
+sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_params, float** dev_grads) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  const double t0 = now_ms();
+  const int L = c->L;
+  if (phase == SH_PRE) {
+    const bool start = c->phase == sh_ctx::FP && c->last_hook == SH_POST && c->last_layer == L - 1 && x == L - 1;
+    const bool cont = c->phase == sh_ctx::BP && c->last_hook == SH_POST && x == c->last_layer - 1;
+    if (!(start || cont) || !dev_params || !dev_grads) {
+      set_error("sh_backward_layer(%d, PRE) out of order (phase %d, last layer %d)", x, (int)c->phase, c->last_layer);
+      return SH_ERR_STATE;
+    }
+    if (start) {
+      c->phase = sh_ctx::BP;
+      // per-step Adam scalars: fixed once BP starts (the CPU updates begin during BP)
+      st = sh_adam_scalars_for(c->lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, c->cfg.weight_decay,
+                               c->step + 1, &c->sc);
+      if (st != SH_OK) return st;
+    }
+    const int pos = 2 * L - 1 - x;
+    st = pre_common(c, x, pos);
+    if (st != SH_OK) return st;
+    const int s = c->layer_slot[x];
+    if (c->gradfree_gen[s] > c->gradfree_waited[s]) {
+      const int64_t gen = c->gradfree_gen[s];
+      if (!state_wait(c, [&] { return c->gradfree_pub[s].load() >= gen; }, "gradient offload issue"))
+        return check_failed(c);
+      CKC(c, cudaStreamWaitEvent(c->cs, c->ev_grad_free[s], 0));
+      c->gradfree_waited[s] = gen;
+    }
+    CKC(c, cudaMemsetAsync(c->slot_grad(s), 0, 4 * c->lay[x].n_pad, c->cs));
+    if (ProfSet* P = cur_prof(c)) CKC(c, cudaEventRecord(P->bp0[x], c->cs));
+    fill_param_ptrs(c, x, dev_params);
+    const LayerLayout& Lx = c->lay[x];
+    for (int k = 0; k < Lx.n_tensors; ++k) dev_grads[k] = c->slot_grad(s) + Lx.offset[k];
+    c->last_layer = x;
+    c->last_hook = SH_PRE;
+  } else if (phase == SH_POST) {
+    if (!(c->phase == sh_ctx::BP && c->last_hook == SH_PRE && x == c->last_layer)) {
+      set_error("sh_backward_layer(%d, POST) out of order", x);
+      return SH_ERR_STATE;
+    }
+    const int s = c->layer_slot[x];
+    const int64_t n = c->lay[x].n_pad;
+    ProfSet* P = cur_prof(c);
+    if (P) {
+      CKC(c, cudaEventRecord(P->bp1[x], c->cs));
+      P->rec_bp[x] = 1;
+    }
+    CKC(c, cudaEventRecord(c->ev_param_free[s], c->cs));
+    cudaEvent_t grads_ready = c->ev_grad_done[s];
+    if (c->W > 1) {
+      // data parallel: average this layer's grads across ranks before the offload (K-e)
+      CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
+      CKC(c, cudaStreamWaitEvent(c->comm, c->ev_grad_done[s], 0));
+      st = nccl_check(c, g_nccl.AllReduce(c->slot_grad(s), c->slot_grad(s), n, ncclFloat, ncclAvg, c->nccl, c->comm),
+                      "ncclAllReduce(layer grads)");
+      if (st != SH_OK) return st;
+      CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_comm, c->partials + x, c->comm));
+      CKC(c, cudaEventRecord(c->ev_reduced[s], c->comm));
+      grads_ready = c->ev_reduced[s];
+    } else {
+      CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_cs, c->partials + x, c->cs));
+      CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
+    }
+    if (!c->is_g(x)) {
+      const int k = (int)(c->landing_rr++ % c->D);
+      const int64_t use = c->landing_uses[k]++;
+      const int64_t gen = ++c->gen;
+      c->gradfree_gen[s] = gen;
+      float* src = c->slot_grad(s);
+      float* dst = c->landing[k];
+      const int64_t step = c->step;
+      const sh_adam_scalars sc = c->sc;
+      cudaEvent_t gf = c->ev_grad_free[s];
+      c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P] {
+        if (!state_wait(c, [&] { return c->landing_done[k].load(std::memory_order_acquire) >= use; },
+                        "host landing buffer")) {
+          c->gradfree_pub[s].store(kInf);
+          notify_state(c);
+          return;
+        }
+        CKA(c, cudaStreamWaitEvent(c->d2h, grads_ready, 0));
+        if (P) CKA(c, cudaEventRecord(P->g2c0[x], c->d2h));
+        CKA(c, cudaMemcpyAsync(dst, src, 4 * n, cudaMemcpyDeviceToHost, c->d2h));
+        if (P) {
+          CKA(c, cudaEventRecord(P->g2c1[x], c->d2h));
+          P->rec_g2c[x] = 1;
+        }
+        CKA(c, cudaEventRecord(gf, c->d2h));
+        CKA(c, cudaLaunchHostFunc(c->d2h, landed_cb, new Landed{c, x, step, k, sc}));
+        c->d2h_bytes += 4 * n;
+        c->d2h_copies++;
+        c->gradfree_pub[s].store(gen);
+        notify_state(c);
+      });
+    }
+    c->last_hook = SH_POST;
+  } else {
+    set_error("sh_backward_layer: bad phase %d", phase);
+    return SH_ERR_INVALID;
+  }
+  c->t_async_ms += now_ms() - t0;
+  c->n_async++;
+  return SH_OK;
+}
+
+sh_status sh_resident(sh_ctx* c, void** dev_params, float** dev_grads) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  for (int k = 0; k < c->res.n_tensors; ++k) {
+    if (dev_params) dev_params[k] = static_cast<char*>(c->res_compute) + (int64_t)c->cb * c->res.offset[k];
+    if (dev_grads) dev_grads[k] = c->res_grad + c->res.offset[k];
+  }
+  return SH_OK;
+}
+
+sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  if (!(c->phase == sh_ctx::BP && c->last_layer == 0 && c->last_hook == SH_POST)) {
+    set_error("sh_step: the backward of layer 0 must be the last hook before sh_step");
+    return SH_ERR_STATE;
+  }
+  const int L = c->L;
+  if (c->W > 1) {
+    // resident grads: average too, on the comm stream after the caller's embedding backward
+    CKC(c, cudaEventRecord(c->ev_cs_mark, c->cs));
+    CKC(c, cudaStreamWaitEvent(c->comm, c->ev_cs_mark, 0));
+    st = nccl_check(c, g_nccl.AllReduce(c->res_grad, c->res_grad, c->res.n_pad, ncclFloat, ncclAvg, c->nccl, c->comm),
+                    "ncclAllReduce(resident grads)");
+    if (st != SH_OK) return st;
+    CKC(c, kern::sumsq(c->res_grad, c->res.n_pad, c->scratch_comm, c->partials + L, c->comm));
+    CKC(c, cudaEventRecord(c->ev_comm_done, c->comm));
+    CKC(c, cudaStreamWaitEvent(c->cs, c->ev_comm_done, 0));
+  } else {
+    CKC(c, kern::sumsq(c->res_grad, c->res.n_pad, c->scratch_cs, c->partials + L, c->cs));
+  }
+  CKC(c, kern::norm_finalize(c->partials, L + 1, c->cfg.max_grad_norm, c->norm_dev, c->coef_dev, c->cs));
+  ProfSet* P = cur_prof(c);
+  if (P) CKC(c, cudaEventRecord(P->k2a, c->cs));
+  kern::K2Args a{};
+  a.sc = c->sc;
+  a.coef = c->clip ? c->coef_dev : nullptr;
+  a.out_bf16 = c->bf16;
+  int64_t bytes = 0;
+  int launches = 0;
+  // layer 0 first: the next FP starts with it
+  for (int x = 0; x < c->w; ++x) {
+    const int s = c->layer_slot[x];
+    if (s < 0) {
+      set_error("internal: GPU-optimised layer %d not in the ring at sh_step", x);
+      return SH_ERR_STATE;
+    }
+    a.e[a.n_entries++] = kern::K2Entry{c->g[x].master, c->g[x].m, c->g[x].v, c->slot_grad(s),
+                                       c->slot_param(s), c->lay[x].n_pad, c->lay[x].n_decay};
+    if (a.n_entries == kern::kK2MaxEntries) {
+      st = push_k2(c, a, &bytes, &launches);
+      if (st != SH_OK) return st;
+    }
+  }
+  a.e[a.n_entries++] = kern::K2Entry{c->res_master, c->res_m, c->res_v, c->res_grad, c->res_compute,
+                                     c->res.n_pad, c->res.n_decay};
+  st = push_k2(c, a, &bytes, &launches);
+  if (st != SH_OK) return st;
+  if (P) {
+    CKC(c, cudaEventRecord(P->k2b, c->cs));
+    P->rec_k2 = true;
+    P->k2_bytes = bytes;
+    P->k2_launches = launches;
+  }
+  if (c->clip) {
+    const int64_t t = c->step;
+    CKC(c, cudaMemcpyAsync(c->h_coef + (t & 1), c->coef_dev, 4, cudaMemcpyDeviceToHost, c->cs));
+    CKC(c, cudaLaunchHostFunc(c->cs, coef_cb, new CoefMsg{c, t}));
+  }
+  // host-optimised copies in the ring are stale after this step's CPU update
+  for (int s = 0; s < c->n_active; ++s) {
+    const int o = c->slot_layer[s];
+    if (o >= 0 && !c->is_g(o)) {
+      c->layer_slot[o] = -1;
+      c->slot_layer[s] = -1;
+    }
+  }
+  c->step++;
+  c->phase = sh_ctx::IDLE;
+  c->last_layer = -1;
+  c->last_hook = SH_POST;
+  if (c->autotune_pending && c->step >= c->warmup) {
+    int32_t wout = 0;
+    st = sh_autotune_window(c, nullptr, &wout);
+    if (st != SH_OK) return st;
+  }
+  if (grad_norm_out) {
+    CKC(c, cudaStreamSynchronize(c->cs));
+    CKC(c, cudaMemcpy(grad_norm_out, c->norm_dev, 8, cudaMemcpyDeviceToHost));
+  }
+  return check_failed(c);
+}
+
+sh_status sh_synchronize(sh_ctx* c) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  return sync_all(c);
+}
+
+sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
+  clear_error();
+  if (!c || !o) return SH_ERR_INVALID;
+  if (c->phase != sh_ctx::IDLE) {
+    set_error("sh_get_profile: only between steps");
+    return SH_ERR_STATE;
+  }
+  sh_status st = sync_all(c);
+  if (st != SH_OK) return st;
+  // t_c2g of GPU-optimised layers is not observed (they are never fetched): use the bytes
+  // rate of the measured host layers (same link, same size class)
+  double rate = 0;  // ms per byte
+  int nr = 0;
+  for (int x = 0; x < c->L; ++x)
+    if (c->p_c2g[x] > 0) rate += c->p_c2g[x] / ((double)c->cb * c->lay[x].n_pad), nr++;
+  double grate = 0;
+  int ng = 0;
+  for (int x = 0; x < c->L; ++x)
+    if (c->p_g2c[x] > 0) grate += c->p_g2c[x] / (4.0 * c->lay[x].n_pad), ng++;
+  for (int x = 0; x < c->L; ++x) {
+    if (c->p_c2g[x] <= 0 && nr) c->p_c2g[x] = rate / nr * c->cb * c->lay[x].n_pad;
+    if (c->p_g2c[x] <= 0 && ng) c->p_g2c[x] = grate / ng * 4.0 * c->lay[x].n_pad;
+    c->p_ocpu[x] = c->cpu_elems.load() > 0
+                       ? c->cpu_ms.load() / c->n_threads / (double)c->cpu_elems.load() * c->lay[x].n_pad
+                       : 0.0;
+  }
+  o->n_layers = c->L;
+  o->t_fp = c->p_fp.data();
+  o->t_bp = c->p_bp.data();
+  o->t_c2g = c->p_c2g.data();
+  o->t_g2c = c->p_g2c.data();
+  o->t_stage = c->p_stage.data();
+  o->t_opt_gpu = c->p_ogpu.data();
+  o->t_opt_cpu = c->p_ocpu.data();
+  o->t_async = c->n_async ? c->t_async_ms / c->n_async : 0.0;
+  o->slot_bytes = c->p_slot_i.data();
+  o->gstate_bytes = c->p_gstate_i.data();
+  o->fixed_bytes = 0;
+  size_t fr = 0, tot = 0;
+  cudaMemGetInfo(&fr, &tot);
+  // S_avail = what the engine holds now (ring + G states) + what is still free - margin
+  int64_t held = (int64_t)c->n_slots * c->slot_bytes;
+  for (int x = 0; x < c->L; ++x)
+    if (c->g[x].master) held += 12 * c->lay[x].n_pad;
+  o->s_avail = c->cfg.device_budget_bytes > 0 ? c->cfg.device_budget_bytes
+                                              : held + (int64_t)fr - ((int64_t)2 << 30);
+  o->duplex = (c->cfg.flags & SH_FLAG_DUPLEX) ? 1 : 0;
+  return SH_OK;
+}
+
+sh_status sh_set_window(sh_ctx* c, int32_t w) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  if (c->phase != sh_ctx::IDLE) {
+    set_error("sh_set_window: only between steps");
+    return SH_ERR_STATE;
+  }
+  if (w < 0 || w > c->L) {
+    set_error("sh_set_window: window %d outside 0..%d", w, c->L);
+    return SH_ERR_INVALID;
+  }
+  if (c->clip && c->D < c->L - w) {
+    set_error("sh_set_window: clip mode needs a landing buffer per host layer");
+    return SH_ERR_INVALID;
+  }
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  if (w == c->w) return SH_OK;
+  return apply_window(c, w);
+}
+
+sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  sh_profile p{};
+  if (ov) {
+    p = *ov;
+  } else {
+    sh_status st = sh_get_profile(c, &p);
+    if (st != SH_OK) return st;
+  }
+  sh_solve_report rep{};
+  sh_status st = sh_solve_window(&p, &rep);
+  if (st != SH_OK) return st;
+  c->autotune_pending = false;
+  if (wout) *wout = rep.window;
+  if (rep.window != c->w) return sh_set_window(c, rep.window);
+  return SH_OK;
+}
+
+sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
+  clear_error();
+  if (!c || !dst) return SH_ERR_INVALID;
+  if (layer < -1 || layer >= c->L || what < 0 || what > 3) {
+    set_error("sh_read_layer: bad layer %d / what %d", layer, what);
+    return SH_ERR_INVALID;
+  }
+  if (c->phase != sh_ctx::IDLE) {
+    set_error("sh_read_layer: only between steps");
+    return SH_ERR_STATE;
+  }
+  sh_status st = sync_all(c);
+  if (st != SH_OK && !c->failed.load()) return st;
+  const LayerLayout& Lx = layer < 0 ? c->res : c->lay[layer];
+  const int64_t n = Lx.n_pad;
+  if (what == SH_READ_COMPUTE) {
+    std::vector<uint8_t> tmp((size_t)c->cb * n);
+    if (layer < 0) {
+      CKC(c, cudaMemcpy(tmp.data(), c->res_compute, tmp.size(), cudaMemcpyDeviceToHost));
+    } else if (c->is_g(layer)) {
+      if (c->layer_slot[layer] < 0) {
+        set_error("sh_read_layer: layer %d not staged", layer);
+        return SH_ERR_STATE;
+      }
+      CKC(c, cudaMemcpy(tmp.data(), c->slot_param(c->layer_slot[layer]), tmp.size(), cudaMemcpyDeviceToHost));
+    } else {
+      std::memcpy(tmp.data(), c->bf16 ? (void*)c->h_shadow[layer] : (void*)c->h_master[layer], tmp.size());
+    }
+    if (c->bf16)
+      unpack_layer_u16(Lx, reinterpret_cast<uint16_t*>(tmp.data()), static_cast<uint16_t*>(dst));
+    else
+      unpack_layer(Lx, reinterpret_cast<float*>(tmp.data()), static_cast<float*>(dst));
+    return SH_OK;
+  }
+  std::vector<float> tmp(n);
+  if (layer < 0 || c->is_g(layer)) {
+    const float* src = layer < 0 ? (what == 0 ? c->res_master : what == 1 ? c->res_m : c->res_v)
+                                 : (what == 0 ? c->g[layer].master : what == 1 ? c->g[layer].m : c->g[layer].v);
+    CKC(c, cudaMemcpy(tmp.data(), src, 4 * n, cudaMemcpyDeviceToHost));
+  } else {
+    const float* src = what == 0 ? c->h_master[layer] : what == 1 ? c->h_m[layer] : c->h_v[layer];
+    std::memcpy(tmp.data(), src, 4 * n);
+  }
+  unpack_layer(Lx, tmp.data(), static_cast<float*>(dst));
+  return SH_OK;
+}
+
+sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
+  clear_error();
+  if (!c || !o) return SH_ERR_INVALID;
+  if (c->phase == sh_ctx::IDLE) sync_all(c);
+  o->step = c->step;
+  o->window = c->w;
+  o->n_slots = c->n_slots;
+  o->host_bytes = (int64_t)c->host_bytes;
+  o->device_bytes = c->device_bytes;
+  o->h2d_bytes = c->h2d_bytes.load();
+  o->d2h_bytes = c->d2h_bytes.load();
+  o->h2d_copies = c->h2d_copies.load();
+  o->d2h_copies = c->d2h_copies.load();
+  o->stage_launches = c->stage_launches.load();
+  o->h2d_busy_ms = c->h2d_busy;
+  o->d2h_busy_ms = c->d2h_busy;
+  o->h2d_profiled_bytes = c->h2d_prof_bytes;
+  o->d2h_profiled_bytes = c->d2h_prof_bytes;
+  o->cpu_adam_ms = c->cpu_ms.load();
+  o->cpu_adam_elems = c->cpu_elems.load();
+  o->cpu_wait_ms = c->cpu_wait_ms.load();
+  o->k2_ms_last = c->k2_ms_last;
+  o->k2_bytes_last = c->k2_bytes_last;
+  o->k2_launches_last = c->k2_launches_last;
+  o->cpu_threads = c->n_threads;
+  o->profiled_steps = c->profiled_steps;
+  return SH_OK;
+}
+
+sh_status sh_destroy(sh_ctx* c) {
+  clear_error();
+  if (!c) return SH_OK;
+  if (!c->failed.load()) sync_all(c);
+  {
+    std::lock_guard<std::mutex> g(c->pmu);
+    c->pool_stop = true;
+  }
+  c->pcv.notify_all();
+  for (auto& t : c->workers) t.join();
+  c->failed.store(1);  // release any issuer wait
+  notify_state(c);
+  c->ih2d.stop();
+  c->id2h.stop();
+  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
+    if (s) cudaStreamSynchronize(s);
+  if (c->cs) cudaStreamSynchronize(c->cs);
+  if (c->nccl) g_nccl.CommDestroy(c->nccl);
+  for (int x = 0; x < c->L; ++x) free_g(c, x);
+  if (c->ring) cudaFree(c->ring);
+  if (c->res_master) cudaFree(c->res_master);
+  if (c->partials) cudaFree(c->partials);
+  for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced, &c->ev_arrive})
+    for (auto e : *v)
+      if (e) cudaEventDestroy(e);
+  for (auto& P : c->prof) {
+    for (auto* v : {&P.fp0, &P.fp1, &P.bp0, &P.bp1, &P.c2g0[0], &P.c2g1[0], &P.c2g0[1], &P.c2g1[1],
+                    &P.g2c0, &P.g2c1, &P.st0, &P.st1})
+      for (auto e : *v)
+        if (e) cudaEventDestroy(e);
+    if (P.k2a) cudaEventDestroy(P.k2a);
+    if (P.k2b) cudaEventDestroy(P.k2b);
+  }
+  if (c->ev_cs_mark) cudaEventDestroy(c->ev_cs_mark);
+  if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
+  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
+    if (s) cudaStreamDestroy(s);
+  if (c->host_base) {
+    cudaHostUnregister(c->host_base);
+    munmap(c->host_base, c->host_bytes);
+  }
+  delete c;
+  return SH_OK;
+}
+
+// ---- op-level entry points ------------------------------------------------------------
+static bool ops_args_ok(int64_t n, int64_t n_decay, const void* const* ptrs, int np) {
+  if (n < 0 || n % 8 != 0 || n_decay < 0 || n_decay > n || n_decay % 8 != 0) {
+    set_error("op: n and n_decay must be multiples of 8 with 0 <= n_decay <= n");
+    return false;
+  }
+  for (int i = 0; i < np; ++i)
+    if (ptrs[i] && (reinterpret_cast<uintptr_t>(ptrs[i]) & 15)) {
+      set_error("op: pointers must be 16-byte aligned");
+      return false;
+    }
+  return true;
+}
+
+sh_status sh_op_adamw_gpu(float* p, float* m, float* v, const float* g, uint16_t* out16, float* out32,
+                          int64_t n, int64_t n_decay, const sh_adam_scalars* sc, const float* coef,
+                          void* stream) {
+  clear_error();
+  const void* ptrs[] = {p, m, v, g, out16, out32};
+  if (!p || !m || !v || !g || !sc || (out16 && out32) || !ops_args_ok(n, n_decay, ptrs, 6))
+    return SH_ERR_INVALID;
+  kern::K2Args a{};
+  a.sc = *sc;
+  a.coef = coef;
+  a.out_bf16 = out16 != nullptr;
+  a.n_entries = 1;
+  a.e[0] = kern::K2Entry{p, m, v, g, out16 ? (void*)out16 : (void*)out32, n, n_decay};
+  const cudaError_t e = kern::adamw_multi(a, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) {
+    set_error("K2 launch: %s", cudaGetErrorString(e));
+    return SH_ERR_CUDA;
+  }
+  return SH_OK;
+}
+
+sh_status sh_op_adamw_cpu(float* p, float* m, float* v, const float* g, uint16_t* out16, int64_t n,
+                          int64_t n_decay, const sh_adam_scalars* sc, int32_t use_coef, float coef,
+                          int32_t n_threads) {
+  clear_error();
+  if (!p || !m || !v || !g || !sc || !ops_args_ok(n, n_decay, nullptr, 0)) return SH_ERR_INVALID;
+  int T = n_threads > 0 ? n_threads : (int)std::thread::hardware_concurrency();
+  if (T < 1) T = 1;
+  const int64_t per = align_up(n / T + 1, 16);
+  std::vector<std::thread> ts;
+  for (int64_t b = 0; b < n; b += per) {
+    const int64_t e = std::min(n, b + per);
+    ts.emplace_back([=] { cpu::adamw_range(p, m, v, g, out16, b, e, n_decay, *sc, use_coef != 0, coef); });
+  }
+  for (auto& t : ts) t.join();
+  return SH_OK;
+}
+
+sh_status sh_op_cast_bf16_gpu(const float* src, uint16_t* dst16, int64_t n, void* stream) {
+  clear_error();
+  const void* ptrs[] = {src, dst16};
+  if (!src || !dst16 || !ops_args_ok(n, 0, ptrs, 2)) return SH_ERR_INVALID;
+  const cudaError_t e = kern::cast_bf16(src, dst16, n, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) {
+    set_error("K1 launch: %s", cudaGetErrorString(e));
+    return SH_ERR_CUDA;
+  }
+  return SH_OK;
+}
+
+sh_status sh_op_cast_bf16_cpu(const float* src, uint16_t* dst16, int64_t n) {
+  clear_error();
+  if (!src || !dst16 || n < 0) return SH_ERR_INVALID;
+  cpu::cast_bf16_range(src, dst16, 0, n);
+  return SH_OK;
+}
+
+sh_status sh_op_sumsq_gpu(const float* g, int64_t n, double* out_dev, void* stream) {
+  clear_error();
+  const void* ptrs[] = {g};
+  if (!g || !out_dev || !ops_args_ok(n, 0, ptrs, 1)) return SH_ERR_INVALID;
+  static double* scratch = nullptr;
+  if (!scratch && cudaMalloc(&scratch, 8 * kern::kSumsqMaxBlocks) != cudaSuccess) {
+    set_error("K3 scratch allocation failed");
+    return SH_ERR_OOM_DEVICE;
+  }
+  const cudaError_t e = kern::sumsq(g, n, scratch, out_dev, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) {
+    set_error("K3 launch: %s", cudaGetErrorString(e));
+    return SH_ERR_CUDA;
+  }
+  return SH_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,239 @@
+// Hot-path kernels of the offload engine for sm_100a.
+//
+//  K1 cast_bf16    fp32 master -> bf16 slot copy (restage of GPU-optimised layers in BP and
+//                  the bf16 compute copy; PAPER.md:205 keeps the first window on the GPU).
+//                  HBM-bound: 6 B/element.
+//  K2 adamw_multi  fused multi-tensor AdamW over the GPU-optimised set (layers [0,w) and the
+//                  resident embedding / positions / final LN), writing the
+//                  new compute copy in place.  HBM-bound: 30 B/element (bf16 mode).
+//  K3 sumsq        per-layer Σg² in fp64 with a fixed reduction tree (grad-norm for clipping;
+//                  deterministic, no float atomics).  HBM-bound: 4 B/element.
+//
+// None of these is a contraction, so there is no tensor-core work here: the rules that matter
+// are 128-bit coalesced accesses, enough bytes in flight per SM, and a grid sized in
+// multiples of the 148 SMs (persistent blocks striding over work items).
+//
+// Numerics: every floating-point op is an explicit
+// round-to-nearest intrinsic so the compiler can neither contract nor reassociate, and the
+// CPU AdamW (cpu_adam.cpp) executes the identical sequence => bitwise-identical results for
+// any split of layers between GPU and CPU, i.e. for every window size.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "sh_internal.hpp"
+
+namespace sh {
+namespace kern {
+
+namespace {
+
+__device__ __forceinline__ uint32_t rne_bf16_bits(float x) {
+  uint32_t u = __float_as_uint(x);
+  if ((u & 0x7fffffffu) > 0x7f800000u) return 0x7fc0u;  // canonical quiet NaN
+  return (u + 0x7fffu + ((u >> 16) & 1u)) >> 16;
+}
+
+__device__ __forceinline__ float4 ld_stream(const float* p) {
+  float4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float4 ld_rw(const float* p) {
+  return *reinterpret_cast<const float4*>(p);
+}
+__device__ __forceinline__ void st_f4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+
+struct AdamS {
+  float b1, b2, omb1, omb2, eps, nss, sqrt_bc2, decay;
+};
+
+__device__ __forceinline__ void adam_elem(float& p, float& m, float& v, float g, const AdamS& s,
+                                          bool wd, bool use_coef, float coef) {
+  if (use_coef) g = __fmul_rn(g, coef);
+  m = __fmaf_rn(s.b1, m, __fmul_rn(s.omb1, g));
+  v = __fmaf_rn(s.b2, v, __fmul_rn(s.omb2, __fmul_rn(g, g)));
+  const float d = __fadd_rn(__fdiv_rn(__fsqrt_rn(v), s.sqrt_bc2), s.eps);
+  const float pp = wd ? __fmul_rn(p, s.decay) : p;
+  p = __fmaf_rn(s.nss, __fdiv_rn(m, d), pp);
+}
+
+// K2: one work item = kK2Chunk consecutive elements of one entry.  Thread t of the block
+// handles elements base + u*1024 + 4t .. +3 for u in {0,1}: every float4 load/store of a
+// warp touches 512 contiguous bytes.  8 independent 16-B loads in flight per thread.
+template <bool kBf16Out>
+__global__ void __launch_bounds__(256) k2_adamw_kernel(const __grid_constant__ K2Args a) {
+  const AdamS s{a.sc.beta1, a.sc.beta2, a.sc.omb1, a.sc.omb2, a.sc.eps, -a.sc.step_size,
+                a.sc.sqrt_bc2, a.sc.decay};
+  const bool use_coef = a.coef != nullptr;
+  const float coef = use_coef ? *a.coef : 1.0f;
+  const int64_t n_items = a.item_start[a.n_entries];
+  int e = 0;
+  for (int64_t item = blockIdx.x; item < n_items; item += gridDim.x) {
+    while (item >= a.item_start[e + 1]) ++e;  // items are visited in increasing order
+    const K2Entry& E = a.e[e];
+    const int64_t base = (item - a.item_start[e]) * kK2Chunk;
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int64_t i = base + u * 1024 + 4 * threadIdx.x;
+      if (i >= E.n) continue;
+      float4 p = ld_rw(E.p + i), m = ld_rw(E.m + i), v = ld_rw(E.v + i);
+      const float4 g = ld_stream(E.g + i);
+      const bool wd = i < E.n_decay;  // n_decay is a multiple of 8: uniform per float4
+      adam_elem(p.x, m.x, v.x, g.x, s, wd, use_coef, coef);
+      adam_elem(p.y, m.y, v.y, g.y, s, wd, use_coef, coef);
+      adam_elem(p.z, m.z, v.z, g.z, s, wd, use_coef, coef);
+      adam_elem(p.w, m.w, v.w, g.w, s, wd, use_coef, coef);
+      st_f4(E.p + i, p);
+      st_f4(E.m + i, m);
+      st_f4(E.v + i, v);
+      if (E.out != nullptr) {
+        if constexpr (kBf16Out) {
+          uint2 o;
+          o.x = rne_bf16_bits(p.x) | (rne_bf16_bits(p.y) << 16);
+          o.y = rne_bf16_bits(p.z) | (rne_bf16_bits(p.w) << 16);
+          *reinterpret_cast<uint2*>(static_cast<uint16_t*>(E.out) + i) = o;
+        } else {
+          st_f4(static_cast<float*>(E.out) + i, p);
+        }
+      }
+    }
+  }
+}
+
+// K1: 8 elements per thread per iteration: 2 x 16-B loads -> 1 x 16-B store.
+__global__ void __launch_bounds__(256) k1_cast_kernel(const float* __restrict__ src,
+                                                     uint16_t* __restrict__ dst, int64_t n8) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n8;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    const float4 a = ld_stream(src + 8 * j);
+    const float4 b = ld_stream(src + 8 * j + 4);
+    uint4 o;
+    o.x = rne_bf16_bits(a.x) | (rne_bf16_bits(a.y) << 16);
+    o.y = rne_bf16_bits(a.z) | (rne_bf16_bits(a.w) << 16);
+    o.z = rne_bf16_bits(b.x) | (rne_bf16_bits(b.y) << 16);
+    o.w = rne_bf16_bits(b.z) | (rne_bf16_bits(b.w) << 16);
+    *reinterpret_cast<uint4*>(dst + 8 * j) = o;
+  }
+}
+
+__device__ __forceinline__ double warp_sum(double x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+  return x;
+}
+
+// Block-level fixed-tree sum of a per-thread double (blockDim == 256).
+__device__ __forceinline__ double block_sum256(double x) {
+  __shared__ double ws[8];
+  x = warp_sum(x);
+  if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = x;
+  __syncthreads();
+  double r = 0.0;
+  if (threadIdx.x < 32) {
+    r = threadIdx.x < 8 ? ws[threadIdx.x] : 0.0;
+    r = warp_sum(r);
+  }
+  return r;  // valid in thread 0
+}
+
+// K3 pass 1: block b sums elements of float4 groups b*256+t, stepping by grid*256.
+// The grid depends only on n (never on the device), so the tree is fixed.
+__global__ void __launch_bounds__(256) k3_partial_kernel(const float* __restrict__ g, int64_t n4,
+                                                        double* __restrict__ partial) {
+  double acc = 0.0;
+  for (int64_t j = blockIdx.x * 256ll + threadIdx.x; j < n4; j += (int64_t)gridDim.x * 256) {
+    const float4 a = ld_stream(g + 4 * j);
+    acc = fma((double)a.x, (double)a.x, acc);
+    acc = fma((double)a.y, (double)a.y, acc);
+    acc = fma((double)a.z, (double)a.z, acc);
+    acc = fma((double)a.w, (double)a.w, acc);
+  }
+  const double s = block_sum256(acc);
+  if (threadIdx.x == 0) partial[blockIdx.x] = s;
+}
+
+__global__ void __launch_bounds__(256) k3_final_kernel(const double* __restrict__ partial, int nb,
+                                                      double* __restrict__ out) {
+  double acc = 0.0;
+  for (int i = threadIdx.x; i < nb; i += 256) acc += partial[i];
+  const double s = block_sum256(acc);
+  if (threadIdx.x == 0) *out = s;
+}
+
+__global__ void norm_finalize_kernel(const double* __restrict__ partials, int n, float max_norm,
+                                     double* norm_out, float* coef_out) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  double s = 0.0;
+  for (int i = 0; i < n; ++i) s += partials[i];  // index order: fixed
+  const double norm = sqrt(s);
+  *norm_out = norm;
+  double c = 1.0;
+  if (max_norm > 0.0f) {
+    c = (double)max_norm / (norm + 1e-6);
+    if (c > 1.0) c = 1.0;
+  }
+  *coef_out = (float)c;
+}
+
+int g_sm_count = 0;
+
+}  // namespace
+
+int sm_count() {
+  if (g_sm_count == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_sm_count, cudaDevAttrMultiProcessorCount, dev);
+    if (g_sm_count <= 0) g_sm_count = 148;
+  }
+  return g_sm_count;
+}
+
+cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
+  a.item_start[0] = 0;
+  for (int i = 0; i < a.n_entries; ++i)
+    a.item_start[i + 1] = a.item_start[i] + (a.e[i].n + kK2Chunk - 1) / kK2Chunk;
+  const int64_t items = a.item_start[a.n_entries];
+  if (items == 0) return cudaSuccess;
+  // Persistent-style grid: 4 resident 256-thread blocks per SM (8 KB of loads in flight per
+  // block-iteration), never more blocks than items.
+  const int64_t cap = (int64_t)sm_count() * 4;
+  const int grid = (int)(items < cap ? items : cap);
+  if (grid_out) *grid_out = grid;
+  if (a.out_bf16)
+    k2_adamw_kernel<true><<<grid, 256, 0, st>>>(a);
+  else
+    k2_adamw_kernel<false><<<grid, 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t cast_bf16(const float* src, uint16_t* dst, int64_t n, cudaStream_t st) {
+  const int64_t n8 = n / 8;
+  if (n8 == 0) return cudaSuccess;
+  const int64_t cap = (int64_t)sm_count() * 8;
+  const int64_t need = (n8 + 255) / 256;
+  k1_cast_kernel<<<(int)(need < cap ? need : cap), 256, 0, st>>>(src, dst, n8);
+  return cudaGetLastError();
+}
+
+cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaStream_t st) {
+  const int64_t n4 = n / 4;
+  if (n4 == 0) return cudaMemsetAsync(out, 0, sizeof(double), st);
+  int64_t nb = (n4 + 2047) / 2048;  // >= 8 float4 per thread before striding
+  if (nb > kSumsqMaxBlocks) nb = kSumsqMaxBlocks;
+  k3_partial_kernel<<<(int)nb, 256, 0, st>>>(g, n4, scratch);
+  k3_final_kernel<<<1, 256, 0, st>>>(scratch, (int)nb, out);
+  return cudaGetLastError();
+}
+
+cudaError_t norm_finalize(const double* partials, int n, float max_norm, double* norm_out,
+                          float* coef_out, cudaStream_t st) {
+  norm_finalize_kernel<<<1, 32, 0, st>>>(partials, n, max_norm, norm_out, coef_out);
+  return cudaGetLastError();
+}
+
+}  // namespace kern
+}  // namespace sh

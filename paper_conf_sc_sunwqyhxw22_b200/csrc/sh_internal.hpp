@@ -1,0 +1,84 @@
+// Internal declarations shared by the engine translation units (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "sh.h"
+
+namespace sh {
+
+// ---- errors -----------------------------------------------------------------------
+void set_error(const char* fmt, ...) __attribute__((format(printf, 1, 2)));
+void clear_error();
+
+// ---- layout -------------------------------------------------------
+// Each tensor is padded to kPad elements (512 B of fp32, 256 B of bf16) so every tensor
+// starts 256-B aligned in every slot (fixed cuBLAS alignment class => same kernels for
+// every window) and K1/K2/K3 can use 128-bit accesses with no tail.  Tensors with weight
+// decay are placed first, so one split point n_decay describes the whole layer.
+constexpr int64_t kPad = 128;
+
+struct LayerLayout {
+  int n_tensors = 0;
+  std::vector<int64_t> numel;   // caller order
+  std::vector<uint8_t> wd;      // caller order
+  std::vector<int64_t> offset;  // caller tensor k -> element offset inside the padded layer
+  int64_t n_raw = 0;            // Σ numel
+  int64_t n_pad = 0;            // padded total (multiple of kPad)
+  int64_t n_decay = 0;          // [0, n_decay) decayed
+};
+
+bool make_layout(const sh_layer_shape& s, LayerLayout* out);
+void pack_layer(const LayerLayout& L, const float* src, float* dst);    // caller order -> padded
+void unpack_layer(const LayerLayout& L, const float* src, float* dst);  // padded -> caller order
+void unpack_layer_u16(const LayerLayout& L, const uint16_t* src, uint16_t* dst);
+
+// ---- kernels (kernels.cu) -----------------------------------------------------------
+namespace kern {
+struct K2Entry {
+  float* p;
+  float* m;
+  float* v;
+  const float* g;
+  void* out;        // bf16 (uint16) or fp32 compute copy; may be null
+  int64_t n;        // multiple of 8
+  int64_t n_decay;  // multiple of 8
+};
+constexpr int kK2MaxEntries = 40;
+constexpr int kK2Chunk = 2048;  // elements per work item (256 threads x 2 x float4)
+struct K2Args {
+  sh_adam_scalars sc;
+  const float* coef;  // null: no clipping
+  int n_entries;
+  int out_bf16;
+  K2Entry e[kK2MaxEntries];
+  int64_t item_start[kK2MaxEntries + 1];
+};
+// Launch K2 over args (item_start filled by the callee).  Returns the grid used.
+cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out = nullptr);
+cudaError_t cast_bf16(const float* src, uint16_t* dst, int64_t n, cudaStream_t st);
+constexpr int kSumsqMaxBlocks = 1184;  // 148 SMs x 8
+// Deterministic Σ g^2 in fp64 -> *out (device).  scratch: kSumsqMaxBlocks doubles.
+cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaStream_t st);
+// norm = sqrt(Σ partials[0..n)) in index order; coef = min(1, max_norm/(norm+1e-6)) (fp32)
+cudaError_t norm_finalize(const double* partials, int n, float max_norm, double* norm_out,
+                          float* coef_out, cudaStream_t st);
+int sm_count();
+}  // namespace kern
+
+// ---- CPU Adam (cpu_adam.cpp) ----------------------------------------------------------
+namespace cpu {
+// Elements [begin, end) of one padded layer (begin/end multiples of 16 or end == n).
+void adamw_range(float* p, float* m, float* v, const float* g, uint16_t* out16, int64_t begin,
+                 int64_t end, int64_t n_decay, const sh_adam_scalars& sc, bool use_coef,
+                 float coef);
+void cast_bf16_range(const float* src, uint16_t* dst, int64_t begin, int64_t end);
+uint16_t rne_bf16(float x);
+bool has_avx512();
+}  // namespace cpu
+
+}  // namespace sh

@@ -1,0 +1,164 @@
+"""End-to-end parity of the CUDA path (engine + GPT driver) on the tiny configuration.
+
+Bars (BASELINE.json north_star, R16):
+  * windowed == all-resident (w = L) BITWISE for every window 0..L: params, m, v, compute copies
+  * vs the fp64 oracle after 3 steps: per offload unit ∞-norm relative error <= 1e-4 (fp32),
+    <= 2e-2 (bf16 mixed); loss per step within 1e-5 relative (fp32)
+"""
+import numpy as np
+import pytest
+
+import synth
+from tests._common import (BF16_TOL, FP32_TOL, TINY, engine_run, engine_state, oracle_run, states_bitwise_equal,
+                           unit_errors)
+
+pytestmark = pytest.mark.gpu
+
+sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
+
+STEPS = 3
+
+
+@pytest.fixture(scope="module")
+def oracle_noclip():
+    return oracle_run(TINY, STEPS)
+
+
+@pytest.fixture(scope="module")
+def oracle_clip():
+    return oracle_run(TINY, STEPS, max_grad_norm=0.5)
+
+
+def _errors(tr, st):
+    L = tr.mc.n_layers
+    layers = [tr.read_layer_tensors(i) for i in range(L)]
+    res = tr.read_layer_tensors(-1)
+    return unit_errors(layers, res, st)
+
+
+@pytest.mark.parametrize("window", [TINY["L"], 2])
+def test_fp32_vs_oracle(oracle_noclip, window):
+    st, olosses, onorms = oracle_noclip
+    tr, losses, norms = engine_run(TINY, STEPS, window, sh.SH_FP32)
+    try:
+        errs = _errors(tr, st)
+        assert max(errs.values()) <= FP32_TOL, errs
+        for a, b in zip(losses, olosses):
+            assert abs(a - b) <= 1e-5 * abs(b), (losses, olosses)
+        for a, b in zip(norms, onorms):
+            assert abs(a - b) <= 1e-4 * b, (norms, onorms)
+    finally:
+        tr.close()
+
+
+def test_bf16_vs_oracle(oracle_noclip):
+    st, olosses, _ = oracle_noclip
+    tr, losses, _ = engine_run(TINY, STEPS, 2, sh.SH_BF16_MIXED)
+    try:
+        errs = _errors(tr, st)
+        assert max(errs.values()) <= BF16_TOL, errs
+        for a, b in zip(losses, olosses):
+            assert abs(a - b) <= 2e-2 * abs(b)
+    finally:
+        tr.close()
+
+
+def test_clip_fp32_vs_oracle(oracle_clip):
+    st, olosses, onorms = oracle_clip
+    assert onorms[0] > 0.5  # clipping is active in this run
+    tr, losses, norms = engine_run(TINY, STEPS, 1, sh.SH_FP32, max_grad_norm=0.5)
+    try:
+        errs = _errors(tr, st)
+        assert max(errs.values()) <= FP32_TOL, errs
+    finally:
+        tr.close()
+
+
+@pytest.mark.parametrize("precision", [sh.SH_FP32, sh.SH_BF16_MIXED])
+def test_windowed_bitwise_equals_resident(precision):
+    L = TINY["L"]
+    ref, ref_losses, _ = engine_run(TINY, STEPS, L, precision)
+    ref_state = engine_state(ref)
+    ref.close()
+    for w in range(0, L):
+        tr, losses, _ = engine_run(TINY, STEPS, w, precision)
+        try:
+            ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+            assert ok, f"window {w}: {what} differs from resident"
+            assert [np.float32(x).tobytes() for x in losses] == [np.float32(x).tobytes() for x in ref_losses]
+            s = tr.engine.stats()
+            if w < L:
+                assert s["h2d_bytes"] > 0 and s["d2h_bytes"] > 0
+        finally:
+            tr.close()
+
+
+def test_clip_windowed_bitwise_and_poison():
+    L = TINY["L"]
+    ref, _, _ = engine_run(TINY, STEPS, L, sh.SH_BF16_MIXED, max_grad_norm=0.5)
+    ref_state = engine_state(ref)
+    ref.close()
+    for w, flags in ((0, 0), (2, sh.SH_FLAG_POISON), (3, sh.SH_FLAG_SYNC_CPU)):
+        tr, _, _ = engine_run(TINY, STEPS, w, sh.SH_BF16_MIXED, max_grad_norm=0.5, flags=flags)
+        try:
+            ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+            assert ok, f"clip window {w} flags {flags}: {what}"
+        finally:
+            tr.close()
+
+
+def test_window_change_mid_run_bitwise():
+    L = TINY["L"]
+    ref, _, _ = engine_run(TINY, 4, L, sh.SH_BF16_MIXED)
+    ref_state = engine_state(ref)
+    ref.close()
+    tr, _, _ = engine_run(TINY, 4, 1, sh.SH_BF16_MIXED, set_window_at={1: 3, 2: 0, 3: 2})
+    try:
+        ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+        assert ok, what
+    finally:
+        tr.close()
+
+
+def test_small_landing_ring_and_one_thread_bitwise():
+    L = TINY["L"]
+    ref, _, _ = engine_run(TINY, STEPS, L, sh.SH_FP32)
+    ref_state = engine_state(ref)
+    ref.close()
+    tr, _, _ = engine_run(TINY, STEPS, 1, sh.SH_FP32, cpu_threads=1, grad_ring_depth=1)
+    try:
+        ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+        assert ok, what
+    finally:
+        tr.close()
+
+
+def test_lr_zero_leaves_params_unchanged():
+    tr, _, _ = engine_run(TINY, 2, 1, sh.SH_FP32, lr=0.0)
+    try:
+        for i in range(TINY["L"]):
+            got = tr.read_layer_tensors(i)
+            init = synth.init_layer(1234, i, TINY["L"], TINY["h"])
+            for a, b in zip(got, init):
+                assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
+    finally:
+        tr.close()
+
+
+def test_protocol_errors():
+    tr, _, _ = engine_run(TINY, 1, 1, sh.SH_FP32)
+    try:
+        with pytest.raises(sh.ShError) as e:
+            tr.engine.forward_pre(1)  # must start at layer 0
+        assert e.value.status == sh.SH_ERR_STATE
+        with pytest.raises(sh.ShError):
+            tr.engine.step()
+        with pytest.raises(sh.ShError) as e:
+            tr.engine.set_window(99)
+        assert e.value.status == sh.SH_ERR_INVALID
+        # the context is still usable after protocol errors
+        tr.set_tokens(synth.tokens(5, TINY["b"], TINY["s"], TINY["V"]))
+        tr.step_device()
+        assert np.isfinite(tr.loss())
+    finally:
+        tr.close()
