@@ -1,0 +1,362 @@
+"""Benchmark of the STRONGHOLD working-window engine on B200 (one JSON line on rank 0).
+
+  python bench.py [--gpus N --steps K --warmup W] [--config c2|c3|tiny] [--batch B] [--window w]
+  python bench.py --impl reference ...     # the CPU oracle, timed on this box's host cores
+
+Metric (BASELINE.json): samples/s at max trainable size per B200; host-link GB/s vs peak.
+Workload (N=1): BASELINE.json configs[1], GPT-2 XL-shaped 1.5B (48 layers, h 1600, 25 heads,
+seq 1024, V 50304), bf16 mixed precision, batch 16 per GPU, window 4 (the paper's artifact
+default), parameters + Adam states in pinned host RAM.  A "step" is one full
+training iteration through every §8(a) row: prefetch H2D, K1 restage, per-layer K3, grad D2H,
+CPU AdamW, K2 (and, outside the hot path, the GPT block compute that drives it).
+
+Timing: W untimed warm-up steps; K timed steps bracketed by barrier + synchronize; CUDA events
+on the engine's compute stream; the end event is recorded after sh_synchronize (all copies and
+all CPU Adam updates of the K steps complete); max over ranks.  Per-step traffic (GBs of weights,
+grads and states) is far larger than the 126 MB L2, so no explicit flush is needed.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: (L, h, nh, s, V, default batch, default window, description)
+    "tiny": (4, 256, 4, 128, 512, 2, 2, "BASELINE configs[0]: tiny GPT 4x256, seq 128"),
+    "c2": (48, 1600, 25, 1024, 50304, 16, 4, "BASELINE configs[1]: GPT-2 XL-shaped 1.5B (48 x 1600, seq 1024)"),
+    "c3": (48, 4096, 32, 1024, 50304, 16, 4, "BASELINE configs[2]: GPT-style ~10B (48 x 4096, seq 1024)"),
+}
+PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
+PROBE_D2H_GBS = 57.01
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = "clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown," \
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown," \
+             "clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def oracle_sample(L, h, nh, s, V, seed=1234):
+    """Bounded CPU-oracle sample of the workload: one block fwd+bwd and its AdamW, plus the head
+    (fwd+bwd) and the resident AdamW, at batch 1; extrapolated to one sample of the full model."""
+    from oracle import gpt_oracle as O
+    import synth
+    cfg = O.GPTConfig(1, h, nh, s, V)
+    P = [a.astype(np.float64) for a in synth.init_layer(seed, 0, L, h)]
+    R = [a.astype(np.float64) for a in synth.init_resident(seed, V, s, h)]
+    tok = synth.tokens(0, 1, s, V)
+    opt = O.AdamWConfig()
+    x = R[0][tok[:, :-1]] + R[1][None, :s]
+    t0 = time.perf_counter()
+    y, cache = O.block_fwd(x, P, nh)
+    dx, grads = O.block_bwd(np.ones_like(y) * 1e-3, cache, P)
+    for k, (p, g) in enumerate(zip(P, grads)):
+        O.adamw_update(p, g, np.zeros_like(p), np.zeros_like(p), 1, opt, p.ndim == 2)
+    t_layer = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    O.forward_backward(O.GPTConfig(0, h, nh, s, V), [], R, tok)
+    for p in R:
+        O.adamw_update(p, p, np.zeros_like(p), np.zeros_like(p), 1, opt, True)
+    t_head = time.perf_counter() - t0
+    per_sample = L * t_layer + t_head
+    return per_sample, t_layer, t_head
+
+
+def blas_threads():
+    try:
+        from threadpoolctl import threadpool_info
+        return max(int(i.get("num_threads", 1)) for i in threadpool_info()) or os.cpu_count()
+    except Exception:
+        return os.cpu_count()
+
+
+def run_reference(args, cfgname):
+    L, h, nh, s, V, b, w, desc = CONFIGS[cfgname]
+    b = args.batch or b
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    times = []
+    for i in range(args.warmup + args.steps):
+        per_sample, tl, th = oracle_sample(L, h, nh, s, V)
+        if i >= args.warmup:
+            times.append(per_sample)
+    per = float(np.mean(times))
+    val = 1.0 / per
+    line = {"impl": "reference", "metric": "samples/s (CPU oracle, extrapolated)", "value": val,
+            "unit": "samples/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": per * 1e3 * b, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic",
+            "config": {"workload": cfgname, "description": desc, "batch_per_gpu": b, "seq": s},
+            "cpu_baseline": {"value": val, "unit": "samples/s", "cores": blas_threads(), "kind": "oracle",
+                             "sample": "per step: one block fwd+bwd+AdamW and the head at batch 1 (numpy fp64), "
+                                       f"extrapolated x{L} layers"},
+            "e2e": {"value": val, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="sh", choices=["sh", "reference"])
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--batch", type=int, default=0)
+    ap.add_argument("--window", type=int, default=-2, help="-2: config default, -1: autotune, L: resident")
+    ap.add_argument("--precision", default="bf16", choices=["bf16", "fp32"])
+    ap.add_argument("--cpu-threads", type=int, default=0)
+    ap.add_argument("--grad-ring", type=int, default=0)
+    ap.add_argument("--no-resident", action="store_true", help="skip the all-resident comparison run")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args, args.config)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_sunwqyhxw22_b200 import gpt as G
+    from paper_conf_sc_sunwqyhxw22_b200 import sh
+    from paper_conf_sc_sunwqyhxw22_b200.trainer import ModelConfig, StrongholdTrainer
+    import synth
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    nccl_id = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        idt = torch.zeros(128, dtype=torch.uint8, device="cuda")
+        if rank == 0:
+            idt.copy_(torch.frombuffer(bytearray(sh.nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(idt, 0)
+        nccl_id = bytes(idt.cpu().numpy().tobytes())
+
+    L, h, nh, s, V, b0, w0, desc = CONFIGS[args.config]
+    b = args.batch or b0
+    w = w0 if args.window == -2 else args.window
+    prec = sh.SH_BF16_MIXED if args.precision == "bf16" else sh.SH_FP32
+    mc = ModelConfig(L, h, nh, s, V)
+    K, W = args.steps, args.warmup
+
+    def run(window, e2e: bool):
+        t_init = time.perf_counter()
+        tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
+                               flags=sh.SH_FLAG_PROFILE, world_size=world, rank=rank, nccl_id=nccl_id,
+                               cpu_threads=args.cpu_threads, grad_ring_depth=args.grad_ring,
+                               warmup_steps=W if window == -1 else 5)
+        t_init = time.perf_counter() - t_init
+        # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
+        host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + K)])
+        host = host.pin_memory()
+        dev = host.to(f"cuda:{local}")
+        for t in range(W):
+            tr.tok_dev.copy_(dev[t])
+            tr.step_device()
+        tr.engine.synchronize()
+        st0 = tr.engine.stats()
+        l0 = sh.kernel_launches() + G.kernel_launches()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        with ClockSampler(local) as clk:
+            ev0.record(tr.stream)
+            for t in range(W, W + K):
+                with torch.cuda.stream(tr.stream):
+                    tr.tok_dev.copy_(dev[t], non_blocking=True)
+                tr.step_device()
+            tr.engine.synchronize()
+            ev1.record(tr.stream)
+            torch.cuda.synchronize()
+        ms = ev0.elapsed_time(ev1)
+        launches = sh.kernel_launches() + G.kernel_launches() - l0
+        st1 = tr.engine.stats()
+        loss = tr.loss()
+        e2e_ms = None
+        if e2e:
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(tr.stream)
+            for t in range(W, W + K):
+                tr.step(host[t])  # public API: pinned host tokens -> H2D, step, loss -> host
+            tr.engine.synchronize()
+            e1.record(tr.stream)
+            torch.cuda.synchronize()
+            e2e_ms = e0.elapsed_time(e1)
+        prof = tr.engine.profile() if window != L else None
+        tr.close()
+        return dict(ms=ms, e2e_ms=e2e_ms, st0=st0, st1=st1, loss=loss, launches=launches, clocks=clk.summary(),
+                    init_s=t_init, prof=prof)
+
+    r = run(w, not args.no_e2e)
+    res = None
+    if not args.no_resident and w != L and args.config != "c3":
+        res = run(L, False)
+
+    def gmax(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    ms = gmax(r["ms"])
+    e2e_ms = gmax(r["e2e_ms"]) if r["e2e_ms"] is not None else None
+    res_ms = gmax(res["ms"]) if res else None
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+    st0, st1 = r["st0"], r["st1"]
+    d = {k: st1[k] - st0[k] for k in ("h2d_bytes", "d2h_bytes", "h2d_busy_ms", "d2h_busy_ms",
+                                      "h2d_profiled_bytes", "d2h_profiled_bytes", "cpu_adam_ms",
+                                      "cpu_adam_elems", "cpu_wait_ms", "k2_ms_sum", "k2_bytes_sum",
+                                      "k2_samples", "k3_ms_sum", "k3_bytes_sum", "k3_samples")}
+    step_ms = ms / K
+    samples = b * world * K / (ms / 1e3)
+    peak, peak_kind = measured_peaks()
+    k2_gbs = d["k2_bytes_sum"] / (d["k2_ms_sum"] / 1e3) / 1e9 if d["k2_ms_sum"] > 0 else None
+    k3_gbs = d["k3_bytes_sum"] / (d["k3_ms_sum"] / 1e3) / 1e9 if d["k3_ms_sum"] > 0 else None
+    h2d_gbs = d["h2d_profiled_bytes"] / (d["h2d_busy_ms"] / 1e3) / 1e9 if d["h2d_busy_ms"] > 0 else None
+    d2h_gbs = d["d2h_profiled_bytes"] / (d["d2h_busy_ms"] / 1e3) / 1e9 if d["d2h_busy_ms"] > 0 else None
+    flops_tok = mc.flops_per_token()
+    tokens_s = samples * s
+    line = {
+        "metric": "samples/s at max trainable size per B200; host-link GB/s vs peak",
+        "value": samples, "unit": "samples/s", "n_gpus": world, "steps": K, "warmup": W,
+        "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "bf16" if prec == sh.SH_BF16_MIXED else "f32", "data": "synthetic",
+        "config": {"workload": args.config, "description": desc, "layers": L, "hidden": h, "heads": nh, "seq": s,
+                   "vocab": V, "params": mc.n_params(), "batch_per_gpu": b, "global_batch": b * world,
+                   "window": w, "ring_slots": w + 1, "precision": "bf16_mixed" if prec else "fp32",
+                   "parallelism": f"dp{world}", "states": "fp32 master/m/v + bf16 shadow in pinned host RAM",
+                   "l2": "no flush: per-step traffic (GBs) >> 126 MB L2"},
+        "tokens_per_s": tokens_s,
+        "model_tflops": tokens_s * flops_tok / 1e12,
+        "final_loss": r["loss"],
+        "host_link": {
+            "h2d_bytes_per_step": d["h2d_bytes"] / K, "d2h_bytes_per_step": d["d2h_bytes"] / K,
+            "h2d_gbs_per_transfer": h2d_gbs, "d2h_gbs_per_transfer": d2h_gbs,
+            "h2d_peak_gbs": PROBE_H2D_GBS, "d2h_peak_gbs": PROBE_D2H_GBS,
+            "h2d_frac": h2d_gbs / PROBE_H2D_GBS if h2d_gbs else None,
+            "d2h_frac": d2h_gbs / PROBE_D2H_GBS if d2h_gbs else None,
+            "h2d_busy_frac_of_step": d["h2d_busy_ms"] / ms, "d2h_busy_frac_of_step": d["d2h_busy_ms"] / ms,
+            "peak_source": "profiles/r01_probe_box.json (pinned 1 GiB copies)"},
+        "cpu_adam": {"threads": st1["cpu_threads"], "elems_per_step": d["cpu_adam_elems"] / K,
+                     "thread_ms_per_step": d["cpu_adam_ms"] / K,
+                     "dram_gbs": 30.0 * d["cpu_adam_elems"] / (d["cpu_adam_ms"] / 1e3 / st1["cpu_threads"]) / 1e9
+                     if d["cpu_adam_ms"] > 0 else None,
+                     "prefetch_wait_ms_per_step": d["cpu_wait_ms"] / K},
+        "roofline": {"kernel": "K2 fused multi-tensor AdamW (sh_step)", "bound": "hbm", "achieved": k2_gbs,
+                     "peak": peak, "unit": "GB/s", "frac": k2_gbs / peak if k2_gbs else None, "traffic": None,
+                     "peak_source": peak_kind, "algorithmic_bytes_per_elem": 30 if prec else 32,
+                     "bytes_per_launch": d["k2_bytes_sum"] / max(1, d["k2_samples"]),
+                     "k3_sumsq_gbs": k3_gbs, "k3_frac": k3_gbs / peak if k3_gbs else None},
+        "gpu_launches": r["launches"],
+        "clocks": r["clocks"],
+        "init_s": r["init_s"],
+    }
+    if r["e2e_ms"] is not None:
+        line["e2e"] = {"value": b * world * K / (e2e_ms / 1e3), "unit": "samples/s",
+                       "h2d_bytes_per_step": b * (s + 1) * 4, "d2h_bytes_per_step": 4}
+    if res:
+        line["resident"] = {"window": L, "samples_per_s": b * world * K / (res_ms / 1e3),
+                            "ms_per_step": res_ms / K, "frac_windowed_over_resident": res_ms / ms}
+    if r["prof"]:
+        p = r["prof"]
+        rep = sh.solve_window(p["t_fp"], p["t_bp"], p["t_c2g"], p["t_g2c"], p["t_stage"], p["t_opt_gpu"],
+                              p["t_opt_cpu"], p["t_async"], p["slot_bytes"], p["gstate_bytes"], p["fixed_bytes"],
+                              p["s_avail"], p["duplex"])
+        line["autotune"] = {"window": rep["window"], "reason": rep["reason"], "eq3_ok": rep["eq3_ok"],
+                            "eq3_min_slack_ms": rep["eq3_min_slack_ms"],
+                            "t_fp_ms": float(np.median(p["t_fp"])), "t_bp_ms": float(np.median(p["t_bp"])),
+                            "t_c2g_ms": float(np.median(p["t_c2g"])), "t_g2c_ms": float(np.median(p["t_g2c"])),
+                            "t_opt_cpu_ms": float(np.median(p["t_opt_cpu"]))}
+    if world == 1 and not args.no_cpu_baseline:
+        per_sample, tl, th = oracle_sample(L, h, nh, s, V)
+        line["cpu_baseline"] = {"value": 1.0 / per_sample, "unit": "samples/s", "cores": blas_threads(),
+                                "kind": "oracle",
+                                "sample": f"one block fwd+bwd+AdamW ({tl:.2f} s) and the head ({th:.2f} s) at batch 1, "
+                                          f"numpy fp64, extrapolated x{L} layers"}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

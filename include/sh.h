@@ -95,7 +95,7 @@ typedef struct {
 #define SH_FLAG_PROFILE   (1ull << 0) /* record per-layer CUDA events every step (else warm-up only) */
 #define SH_FLAG_POISON    (1ull << 1) /* debug: fill a slot's param half with NaN before every refill */
 #define SH_FLAG_DUPLEX    (1ull << 2) /* autotuner: full-duplex link, max() instead of sum in (1d)/(2d) */
-#define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline on the D2H issuer (no pool) */
+#define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
 typedef struct {
   int32_t n_layers;                 /* L >= 1, execution order */
@@ -165,6 +165,12 @@ typedef struct {
   int32_t k2_launches_last;
   int32_t cpu_threads;
   int32_t profiled_steps;
+  double k2_ms_sum;             /* K2 durations summed over all profiled steps */
+  int64_t k2_bytes_sum;         /* their algorithmic HBM bytes */
+  int64_t k2_samples;           /* number of profiled K2 phases summed */
+  double k3_ms_sum;             /* per-layer K3 (Σg²) durations summed (profiled steps) */
+  int64_t k3_bytes_sum;
+  int64_t k3_samples;
 } sh_stats_t;
 
 /* ---- lifecycle ------------------------------------------------------------------ */
@@ -250,6 +256,9 @@ sh_status sh_stats(sh_ctx* ctx, sh_stats_t* out);
 const char* sh_last_error(void);
 
 int32_t sh_abi_version(void);
+
+/* Number of engine kernel launches (K1, K2, K3, norm finalize) since the library was loaded. */
+int64_t sh_kernel_launches(void);
 
 /* Rank 0 of a data-parallel job: fill a 128-byte ncclUniqueId (dlopen'ed libnccl.so.2, the
  * one torch loads) to be broadcast through torch.distributed before sh_init. */

@@ -47,6 +47,8 @@ typedef struct {
 int32_t gpt_create(const gpt_config* cfg, gpt_ctx** out);
 int32_t gpt_destroy(gpt_ctx* ctx);
 const char* gpt_last_error(void);
+/* Number of this library's own kernel launches (cuBLAS / CUB launches not counted). */
+int64_t gpt_kernel_launches(void);
 /* Device bytes of activations/workspace held by the context. */
 int64_t gpt_workspace_bytes(const gpt_ctx* ctx);
 

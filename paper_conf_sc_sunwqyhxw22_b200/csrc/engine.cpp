@@ -162,9 +162,9 @@ class Issuer {
 };
 
 struct ProfSet {  // CUDA timing events of one step (double-buffered by step parity)
-  std::vector<cudaEvent_t> fp0, fp1, bp0, bp1, c2g0[2], c2g1[2], g2c0, g2c1, st0, st1;
+  std::vector<cudaEvent_t> fp0, fp1, bp0, bp1, c2g0[2], c2g1[2], g2c0, g2c1, st0, st1, k30, k31;
   std::vector<std::atomic<uint8_t>> rec_c2g[2], rec_g2c, rec_st;
-  std::vector<uint8_t> rec_fp, rec_bp;
+  std::vector<uint8_t> rec_fp, rec_bp, rec_k3;
   cudaEvent_t k2a = nullptr, k2b = nullptr;
   bool rec_k2 = false;
   bool active = false;
@@ -292,8 +292,8 @@ struct sh_ctx {
   std::atomic<double> cpu_ms{0.0}, cpu_wait_ms{0.0};
   double h2d_busy = 0, d2h_busy = 0;
   int64_t h2d_prof_bytes = 0, d2h_prof_bytes = 0;
-  double k2_ms_last = 0;
-  int64_t k2_bytes_last = 0;
+  double k2_ms_last = 0, k2_ms_sum = 0, k3_ms_sum = 0;
+  int64_t k2_bytes_last = 0, k2_bytes_sum = 0, k2_samples = 0, k3_bytes_sum = 0, k3_samples = 0;
   int k2_launches_last = 0;
 
   // ---- failure
@@ -473,9 +473,9 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
   j->landing = L->landing;
   j->n_chunks = (c->lay[L->layer].n_pad + kCpuChunk - 1) / kCpuChunk;
   j->sc = L->sc;
-  if (c->cfg.flags & SH_FLAG_SYNC_CPU) {  // debug: inline, single-threaded
+  if ((c->cfg.flags & SH_FLAG_SYNC_CPU) && !c->clip) {  // debug: inline, single-threaded
     Job* jp = j.get();
-    float coef = c->clip ? c->coef_of_step[jp->step & 1] : 1.0f;
+    const float coef = 1.0f;
     cpu::adamw_range(c->h_master[jp->layer], c->h_m[jp->layer], c->h_v[jp->layer],
                      c->landing[jp->landing], c->bf16 ? c->h_shadow[jp->layer] : nullptr, 0,
                      c->lay[jp->layer].n_pad, c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
@@ -516,7 +516,7 @@ sh_status prof_alloc(sh_ctx* c, ProfSet& P) {
   };
   cudaError_t r = cudaSuccess;
   for (auto* v : {&P.fp0, &P.fp1, &P.bp0, &P.bp1, &P.c2g0[0], &P.c2g1[0], &P.c2g0[1], &P.c2g1[1],
-                  &P.g2c0, &P.g2c1, &P.st0, &P.st1})
+                  &P.g2c0, &P.g2c1, &P.st0, &P.st1, &P.k30, &P.k31})
     if (r == cudaSuccess) r = mk(*v);
   if (r == cudaSuccess) r = cudaEventCreate(&P.k2a);
   if (r == cudaSuccess) r = cudaEventCreate(&P.k2b);
@@ -530,6 +530,7 @@ sh_status prof_alloc(sh_ctx* c, ProfSet& P) {
   P.rec_st = std::vector<std::atomic<uint8_t>>(c->L);
   P.rec_fp.assign(c->L, 0);
   P.rec_bp.assign(c->L, 0);
+  P.rec_k3.assign(c->L, 0);
   return SH_OK;
 }
 
@@ -541,6 +542,7 @@ void prof_reset(sh_ctx* c, ProfSet& P, int64_t step) {
     P.rec_st[i] = 0;
     P.rec_fp[i] = 0;
     P.rec_bp[i] = 0;
+    P.rec_k3[i] = 0;
   }
   P.rec_k2 = false;
   P.active = true;
@@ -576,11 +578,19 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
       c->d2h_prof_bytes += 4 * c->lay[i].n_pad;
     }
     if (P.rec_st[i]) c->p_stage[i] = ev_ms(P.st0[i], P.st1[i]);
+    if (P.rec_k3[i]) {
+      c->k3_ms_sum += ev_ms(P.k30[i], P.k31[i]);
+      c->k3_bytes_sum += 4 * c->lay[i].n_pad;
+      c->k3_samples++;
+    }
   }
   if (P.rec_k2) {
     c->k2_ms_last = ev_ms(P.k2a, P.k2b);
     c->k2_bytes_last = P.k2_bytes;
     c->k2_launches_last = P.k2_launches;
+    c->k2_ms_sum += c->k2_ms_last;
+    c->k2_bytes_sum += P.k2_bytes;
+    c->k2_samples++;
     // apportion K2 time to layers by bytes (one fused launch covers all of them)
     double tot = 0;
     for (int i = 0; i < L; ++i) tot += c->lay[i].n_pad;
@@ -874,6 +884,7 @@ sh_status nccl_check(sh_ctx* c, ncclResult_t r, const char* what) {
 extern "C" {
 
 int32_t sh_abi_version(void) { return SH_ABI_VERSION; }
+int64_t sh_kernel_launches(void) { return kern::launches(); }
 const char* sh_last_error(void) { return sh::last_error_cstr(); }
 
 sh_status sh_nccl_get_unique_id(void* out128) {
@@ -1293,7 +1304,12 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       CKC(c, cudaEventRecord(c->ev_reduced[s], c->comm));
       grads_ready = c->ev_reduced[s];
     } else {
+      if (P) CKC(c, cudaEventRecord(P->k30[x], c->cs));
       CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_cs, c->partials + x, c->cs));
+      if (P) {
+        CKC(c, cudaEventRecord(P->k31[x], c->cs));
+        P->rec_k3[x] = 1;
+      }
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
     }
     if (!c->is_g(x)) {
@@ -1602,6 +1618,12 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->k2_launches_last = c->k2_launches_last;
   o->cpu_threads = c->n_threads;
   o->profiled_steps = c->profiled_steps;
+  o->k2_ms_sum = c->k2_ms_sum;
+  o->k2_bytes_sum = c->k2_bytes_sum;
+  o->k2_samples = c->k2_samples;
+  o->k3_ms_sum = c->k3_ms_sum;
+  o->k3_bytes_sum = c->k3_bytes_sum;
+  o->k3_samples = c->k3_samples;
   return SH_OK;
 }
 
@@ -1632,7 +1654,7 @@ sh_status sh_destroy(sh_ctx* c) {
       if (e) cudaEventDestroy(e);
   for (auto& P : c->prof) {
     for (auto* v : {&P.fp0, &P.fp1, &P.bp0, &P.bp1, &P.c2g0[0], &P.c2g1[0], &P.c2g0[1], &P.c2g1[1],
-                    &P.g2c0, &P.g2c1, &P.st0, &P.st1})
+                    &P.g2c0, &P.g2c1, &P.st0, &P.st1, &P.k30, &P.k31})
       for (auto e : *v)
         if (e) cudaEventDestroy(e);
     if (P.k2a) cudaEventDestroy(P.k2a);

@@ -10,6 +10,7 @@
 
 #include <cub/device/device_radix_sort.cuh>
 
+#include <atomic>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -21,6 +22,7 @@
 namespace {
 
 thread_local std::string g_err;
+std::atomic<int64_t> g_launches{0};
 void seterr(const char* fmt, ...) {
   char b[512];
   va_list ap;
@@ -390,30 +392,30 @@ int layer_fwd_impl(gpt_ctx* c, int l, void* const* P, bool write_out) {
   const float* xin = c->x + (int64_t)l * c->maxN * h;
   float* xout = c->x + (int64_t)(l + 1) * c->maxN * h;
   const int rows_per_blk = 8;
-  ln_fwd<T><<<(N + rows_per_blk - 1) / rows_per_blk, 256, 0, c->st>>>(xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
+  (g_launches++, 0), ln_fwd<T><<<(N + rows_per_blk - 1) / rows_per_blk, 256, 0, c->st>>>(xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
                                                                       c->ln1_m, c->ln1_r, N, h);
   CB(rm_gemm(c, false, true, N, 3 * h, h, 1.f, c->ln1, dt, P[2], dt, 0.f, c->f32big, CUDA_R_32F));
-  qkv_split<T><<<grid_for((int64_t)N * 3 * h), 256, 0, c->st>>>(c->f32big, (const T*)P[3], (T*)c->q, (T*)c->k,
+  (g_launches++, 0), qkv_split<T><<<grid_for((int64_t)N * 3 * h), 256, 0, c->st>>>(c->f32big, (const T*)P[3], (T*)c->q, (T*)c->k,
                                                                 (T*)c->v, S, h, nh, (int64_t)N * 3 * h);
   const int BH = B * nh;
   const float scale = 1.0f / sqrtf((float)hd);
   CB(rm_gemm_batched(c, false, true, S, S, hd, scale, c->q, dt, (int64_t)S * hd, c->k, dt, (int64_t)S * hd, 0.f,
                      c->scores, CUDA_R_32F, (int64_t)S * S, BH));
   const int64_t rows = (int64_t)BH * S;
-  softmax_causal<T><<<(int)((rows + 7) / 8), 256, 0, c->st>>>(c->scores, (T*)c->probs, S, rows);
+  (g_launches++, 0), softmax_causal<T><<<(int)((rows + 7) / 8), 256, 0, c->st>>>(c->scores, (T*)c->probs, S, rows);
   CB(rm_gemm_batched(c, false, false, S, hd, S, 1.f, c->probs, dt, (int64_t)S * S, c->v, dt, (int64_t)S * hd, 0.f,
                      c->atto, dt, (int64_t)S * hd, BH));
-  heads_to_rows<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>((const T*)c->atto, (T*)c->att, S, h, nh,
+  (g_launches++, 0), heads_to_rows<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>((const T*)c->atto, (T*)c->att, S, h, nh,
                                                                  (int64_t)N * h, h, 0);
-  resid_bias<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>(xin, (const T*)P[5], c->x_mid, h, (int64_t)N * h);
+  (g_launches++, 0), resid_bias<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>(xin, (const T*)P[5], c->x_mid, h, (int64_t)N * h);
   CB(rm_gemm(c, false, true, N, h, h, 1.f, c->att, dt, P[4], dt, 1.f, c->x_mid, CUDA_R_32F));
-  ln_fwd<T><<<(N + rows_per_blk - 1) / rows_per_blk, 256, 0, c->st>>>(c->x_mid, (const T*)P[6], (const T*)P[7],
+  (g_launches++, 0), ln_fwd<T><<<(N + rows_per_blk - 1) / rows_per_blk, 256, 0, c->st>>>(c->x_mid, (const T*)P[6], (const T*)P[7],
                                                                       (T*)c->ln2, c->ln2_m, c->ln2_r, N, h);
   CB(rm_gemm(c, false, true, N, 4 * h, h, 1.f, c->ln2, dt, P[8], dt, 0.f, c->f32big, CUDA_R_32F));
-  gelu_fwd<T><<<grid_for((int64_t)N * 4 * h), 256, 0, c->st>>>(c->f32big, (const T*)P[9], (T*)c->fc_pre,
+  (g_launches++, 0), gelu_fwd<T><<<grid_for((int64_t)N * 4 * h), 256, 0, c->st>>>(c->f32big, (const T*)P[9], (T*)c->fc_pre,
                                                                (T*)c->fc_act, 4 * h, (int64_t)N * 4 * h);
   if (write_out) {
-    resid_bias<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>(c->x_mid, (const T*)P[11], xout, h, (int64_t)N * h);
+    (g_launches++, 0), resid_bias<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>(c->x_mid, (const T*)P[11], xout, h, (int64_t)N * h);
     CB(rm_gemm(c, false, true, N, h, 4 * h, 1.f, c->fc_act, dt, P[10], dt, 1.f, xout, CUDA_R_32F));
   }
   CK(cudaGetLastError());
@@ -429,39 +431,39 @@ int layer_bwd_impl(gpt_ctx* c, int l, void* const* P, float* const* G) {
   const float* xin = c->x + (int64_t)l * c->maxN * h;
   const int64_t Nh = (int64_t)N * h;
   // ---- MLP
-  cast_f2t<T><<<grid_for(Nh), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh);
+  (g_launches++, 0), cast_f2t<T><<<grid_for(Nh), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh);
   CB(rm_gemm(c, true, false, h, 4 * h, N, 1.f, c->dy, dt, c->fc_act, dt, 0.f, G[10], CUDA_R_32F));
   if ((r = colsum(c, c->dres, true, N, h, G[11]))) return r;
   CB(rm_gemm(c, false, false, N, 4 * h, h, 1.f, c->dy, dt, P[10], dt, 0.f, c->d4h, dt));
-  gelu_bwd<T><<<grid_for(4 * Nh), 256, 0, c->st>>>((T*)c->d4h, (const T*)c->fc_pre, 4 * Nh);
+  (g_launches++, 0), gelu_bwd<T><<<grid_for(4 * Nh), 256, 0, c->st>>>((T*)c->d4h, (const T*)c->fc_pre, 4 * Nh);
   CB(rm_gemm(c, true, false, 4 * h, h, N, 1.f, c->d4h, dt, c->ln2, dt, 0.f, G[8], CUDA_R_32F));
   if ((r = colsum(c, c->d4h, false, N, 4 * h, G[9]))) return r;
   CB(rm_gemm(c, false, false, N, h, 4 * h, 1.f, c->d4h, dt, P[8], dt, 0.f, c->dln, CUDA_R_32F));
-  ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, c->x_mid, c->ln2_m, c->ln2_r, (const T*)P[6], c->dres, c->tmp, N, h);
+  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, c->x_mid, c->ln2_m, c->ln2_r, (const T*)P[6], c->dres, c->tmp, N, h);
   if ((r = colsum(c, c->tmp, true, N, h, G[6]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[7]))) return r;
   // ---- attention
-  cast_f2t<T><<<grid_for(Nh), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh);
+  (g_launches++, 0), cast_f2t<T><<<grid_for(Nh), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh);
   CB(rm_gemm(c, true, false, h, h, N, 1.f, c->dy, dt, c->att, dt, 0.f, G[4], CUDA_R_32F));
   if ((r = colsum(c, c->dres, true, N, h, G[5]))) return r;
   CB(rm_gemm(c, false, false, N, h, h, 1.f, c->dy, dt, P[4], dt, 0.f, c->datt, dt));
-  rows_to_heads<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->datt, (T*)c->dO, S, h, nh, Nh);
+  (g_launches++, 0), rows_to_heads<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->datt, (T*)c->dO, S, h, nh, Nh);
   const int BH = B * nh;
   const float scale = 1.0f / sqrtf((float)hd);
   const int64_t sQ = (int64_t)S * hd, sS = (int64_t)S * S;
   CB(rm_gemm_batched(c, false, true, S, S, hd, 1.f, c->dO, dt, sQ, c->v, dt, sQ, 0.f, c->scores, CUDA_R_32F, sS, BH));
   CB(rm_gemm_batched(c, true, false, S, hd, S, 1.f, c->probs, dt, sS, c->dO, dt, sQ, 0.f, c->dv, dt, sQ, BH));
   const int64_t rows = (int64_t)BH * S;
-  softmax_bwd<T><<<(int)((rows + 7) / 8), 256, 0, c->st>>>((T*)c->probs, c->scores, S, rows);
+  (g_launches++, 0), softmax_bwd<T><<<(int)((rows + 7) / 8), 256, 0, c->st>>>((T*)c->probs, c->scores, S, rows);
   CB(rm_gemm_batched(c, false, false, S, hd, S, scale, c->probs, dt, sS, c->k, dt, sQ, 0.f, c->dq, dt, sQ, BH));
   CB(rm_gemm_batched(c, true, false, S, hd, S, scale, c->probs, dt, sS, c->q, dt, sQ, 0.f, c->dk, dt, sQ, BH));
-  heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dq, (T*)c->dqkv, S, h, nh, Nh, 3 * h, 0);
-  heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dk, (T*)c->dqkv, S, h, nh, Nh, 3 * h, h);
-  heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dv, (T*)c->dqkv, S, h, nh, Nh, 3 * h, 2 * h);
+  (g_launches++, 0), heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dq, (T*)c->dqkv, S, h, nh, Nh, 3 * h, 0);
+  (g_launches++, 0), heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dk, (T*)c->dqkv, S, h, nh, Nh, 3 * h, h);
+  (g_launches++, 0), heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dv, (T*)c->dqkv, S, h, nh, Nh, 3 * h, 2 * h);
   CB(rm_gemm(c, true, false, 3 * h, h, N, 1.f, c->dqkv, dt, c->ln1, dt, 0.f, G[2], CUDA_R_32F));
   if ((r = colsum(c, c->dqkv, false, N, 3 * h, G[3]))) return r;
   CB(rm_gemm(c, false, false, N, h, 3 * h, 1.f, c->dqkv, dt, P[2], dt, 0.f, c->dln, CUDA_R_32F));
-  ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xin, c->ln1_m, c->ln1_r, (const T*)P[0], c->dres, c->tmp, N, h);
+  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xin, c->ln1_m, c->ln1_r, (const T*)P[0], c->dres, c->tmp, N, h);
   if ((r = colsum(c, c->tmp, true, N, h, G[0]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[1]))) return r;
   CK(cudaGetLastError());
@@ -473,13 +475,13 @@ int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float
   const int N = c->N, h = c->h, V = c->V, S = c->S;
   const cudaDataType_t dt = c->dt;
   const float* xL = c->x + (int64_t)c->L * c->maxN * h;
-  ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xL, (const T*)R[2], (const T*)R[3], (T*)c->lnf, c->lnf_m, c->lnf_r, N, h);
+  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xL, (const T*)R[2], (const T*)R[3], (T*)c->lnf, c->lnf_m, c->lnf_r, N, h);
   CB(rm_gemm(c, false, true, N, V, h, 1.f, c->lnf, dt, R[0], dt, 0.f, c->logits, CUDA_R_32F));
-  ce_fwd_bwd<T><<<N, 512, 0, c->st>>>(c->logits, tok, S, V, 1.0f / N, c->row_loss, (T*)c->dlogits);
-  mean_fixed<<<1, 512, 0, c->st>>>(c->row_loss, N, 1.0f / N, d_loss);
+  (g_launches++, 0), ce_fwd_bwd<T><<<N, 512, 0, c->st>>>(c->logits, tok, S, V, 1.0f / N, c->row_loss, (T*)c->dlogits);
+  (g_launches++, 0), mean_fixed<<<1, 512, 0, c->st>>>(c->row_loss, N, 1.0f / N, d_loss);
   CB(rm_gemm(c, false, false, N, h, V, 1.f, c->dlogits, dt, R[0], dt, 0.f, c->dln, CUDA_R_32F));
   CK(cudaMemsetAsync(c->dres, 0, sizeof(float) * (size_t)N * h, c->st));
-  ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xL, c->lnf_m, c->lnf_r, (const T*)R[2], c->dres, c->tmp, N, h);
+  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xL, c->lnf_m, c->lnf_r, (const T*)R[2], c->dres, c->tmp, N, h);
   int r;
   if ((r = colsum(c, c->tmp, true, N, h, G[2]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[3]))) return r;
@@ -493,6 +495,7 @@ int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float
 extern "C" {
 
 const char* gpt_last_error(void) { return g_err.c_str(); }
+int64_t gpt_kernel_launches(void) { return g_launches.load(); }
 int64_t gpt_workspace_bytes(const gpt_ctx* c) { return c ? c->bytes : 0; }
 float* gpt_checkpoint(gpt_ctx* c, int32_t l) {
   if (!c || l < 0 || l > c->L) return nullptr;
@@ -566,11 +569,11 @@ int32_t gpt_create(const gpt_config* cfg, gpt_ctx** out) {
   cublasSetWorkspace(c->cb, c->ws, c->ws_bytes);
   cublasSetMathMode(c->cb, CUBLAS_DEFAULT_MATH);  // no TF32 in fp32 mode
   cublasSetAtomicsMode(c->cb, CUBLAS_ATOMICS_NOT_ALLOWED);
-  fill_ones<float><<<grid_for(mN), 256, 0, c->st>>>(c->ones_f, mN);
+  (g_launches++, 0), fill_ones<float><<<grid_for(mN), 256, 0, c->st>>>(c->ones_f, mN);
   if (c->bf16)
-    fill_ones<bf16><<<grid_for(mN), 256, 0, c->st>>>((bf16*)c->ones_t, mN);
+    (g_launches++, 0), fill_ones<bf16><<<grid_for(mN), 256, 0, c->st>>>((bf16*)c->ones_t, mN);
   else
-    fill_ones<float><<<grid_for(mN), 256, 0, c->st>>>((float*)c->ones_t, mN);
+    (g_launches++, 0), fill_ones<float><<<grid_for(mN), 256, 0, c->st>>>((float*)c->ones_t, mN);
   if (cudaStreamSynchronize(c->st) != cudaSuccess) {
     seterr("gpt_create: init kernels failed");
     gpt_destroy(c);
@@ -598,9 +601,9 @@ int32_t gpt_embed_forward(gpt_ctx* c, const int32_t* tok, int32_t B, void* const
   c->B = B;
   c->N = B * c->S;
   if (c->bf16)
-    embed_fwd<bf16><<<c->N, 256, 0, c->st>>>(tok, (const bf16*)R[0], (const bf16*)R[1], c->x, c->S, c->h);
+    (g_launches++, 0), embed_fwd<bf16><<<c->N, 256, 0, c->st>>>(tok, (const bf16*)R[0], (const bf16*)R[1], c->x, c->S, c->h);
   else
-    embed_fwd<float><<<c->N, 256, 0, c->st>>>(tok, (const float*)R[0], (const float*)R[1], c->x, c->S, c->h);
+    (g_launches++, 0), embed_fwd<float><<<c->N, 256, 0, c->st>>>(tok, (const float*)R[0], (const float*)R[1], c->x, c->S, c->h);
   CK(cudaGetLastError());
   return 0;
 }
@@ -639,13 +642,13 @@ int32_t gpt_embed_backward(gpt_ctx* c, const int32_t* tok, float* const* G) {
     return -1;
   }
   const int N = c->N;
-  gather_tokens<<<(N + 255) / 256, 256, 0, c->st>>>(tok, c->S, N, c->keys, c->vals);
+  (g_launches++, 0), gather_tokens<<<(N + 255) / 256, 256, 0, c->st>>>(tok, c->S, N, c->keys, c->vals);
   int bits = 1;
   while ((1 << bits) < c->V) ++bits;
   size_t tb = c->cub_bytes;
   CK(cub::DeviceRadixSort::SortPairs(c->cub_tmp, tb, c->keys, c->keys2, c->vals, c->vals2, N, 0, bits, c->st));
-  embed_bwd_wte<<<N, 256, 0, c->st>>>(c->keys2, c->vals2, c->dres, G[0], N, c->h);
-  embed_bwd_wpe<<<c->S, 256, 0, c->st>>>(c->dres, G[1], c->B, c->S, c->h);
+  (g_launches++, 0), embed_bwd_wte<<<N, 256, 0, c->st>>>(c->keys2, c->vals2, c->dres, G[0], N, c->h);
+  (g_launches++, 0), embed_bwd_wpe<<<c->S, 256, 0, c->st>>>(c->dres, G[1], c->B, c->S, c->h);
   CK(cudaGetLastError());
   return 0;
 }

@@ -19,6 +19,7 @@
 // any split of layers between GPU and CPU, i.e. for every window size.
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdint>
 
 #include "sh_internal.hpp"
@@ -179,8 +180,14 @@ __global__ void norm_finalize_kernel(const double* __restrict__ partials, int n,
 }
 
 int g_sm_count = 0;
+__host__ std::atomic<int64_t>& launch_counter() {
+  static std::atomic<int64_t> n{0};
+  return n;
+}
 
 }  // namespace
+
+int64_t launches() { return launch_counter().load(); }
 
 int sm_count() {
   if (g_sm_count == 0) {
@@ -203,6 +210,7 @@ cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
   const int64_t cap = (int64_t)sm_count() * 4;
   const int grid = (int)(items < cap ? items : cap);
   if (grid_out) *grid_out = grid;
+  launch_counter()++;
   if (a.out_bf16)
     k2_adamw_kernel<true><<<grid, 256, 0, st>>>(a);
   else
@@ -215,6 +223,7 @@ cudaError_t cast_bf16(const float* src, uint16_t* dst, int64_t n, cudaStream_t s
   if (n8 == 0) return cudaSuccess;
   const int64_t cap = (int64_t)sm_count() * 8;
   const int64_t need = (n8 + 255) / 256;
+  launch_counter()++;
   k1_cast_kernel<<<(int)(need < cap ? need : cap), 256, 0, st>>>(src, dst, n8);
   return cudaGetLastError();
 }
@@ -224,6 +233,7 @@ cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaS
   if (n4 == 0) return cudaMemsetAsync(out, 0, sizeof(double), st);
   int64_t nb = (n4 + 2047) / 2048;  // >= 8 float4 per thread before striding
   if (nb > kSumsqMaxBlocks) nb = kSumsqMaxBlocks;
+  launch_counter() += 2;
   k3_partial_kernel<<<(int)nb, 256, 0, st>>>(g, n4, scratch);
   k3_final_kernel<<<1, 256, 0, st>>>(scratch, (int)nb, out);
   return cudaGetLastError();
@@ -231,6 +241,7 @@ cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaS
 
 cudaError_t norm_finalize(const double* partials, int n, float max_norm, double* norm_out,
                           float* coef_out, cudaStream_t st) {
+  launch_counter()++;
   norm_finalize_kernel<<<1, 32, 0, st>>>(partials, n, max_norm, norm_out, coef_out);
   return cudaGetLastError();
 }

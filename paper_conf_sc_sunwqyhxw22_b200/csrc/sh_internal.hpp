@@ -68,6 +68,7 @@ cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaS
 cudaError_t norm_finalize(const double* partials, int n, float max_norm, double* norm_out,
                           float* coef_out, cudaStream_t st);
 int sm_count();
+int64_t launches();
 }  // namespace kern
 
 // ---- CPU Adam (cpu_adam.cpp) ----------------------------------------------------------

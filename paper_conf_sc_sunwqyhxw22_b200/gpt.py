@@ -9,7 +9,7 @@ from .sh import LIBDIR
 
 EXPORTS = ("gpt_create", "gpt_destroy", "gpt_last_error", "gpt_workspace_bytes", "gpt_embed_forward",
            "gpt_layer_forward", "gpt_head_forward_backward", "gpt_layer_backward", "gpt_embed_backward",
-           "gpt_checkpoint")
+           "gpt_checkpoint", "gpt_kernel_launches")
 
 
 class GptConfig(C.Structure):
@@ -41,8 +41,13 @@ def lib() -> C.CDLL:
         L.gpt_workspace_bytes.restype = C.c_int64
         L.gpt_checkpoint.argtypes = [vp, i32]
         L.gpt_checkpoint.restype = C.c_void_p
+        L.gpt_kernel_launches.restype = C.c_int64
         _lib = L
     return _lib
+
+
+def kernel_launches() -> int:
+    return int(lib().gpt_kernel_launches())
 
 
 def _check(r):

@@ -28,7 +28,7 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_autotune_window", "sh_set_window", "sh_get_profile", "sh_read_layer", "sh_stats",
            "sh_last_error", "sh_abi_version", "sh_nccl_get_unique_id", "sh_adam_scalars_for",
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
-           "sh_op_sumsq_gpu")
+           "sh_op_sumsq_gpu", "sh_kernel_launches")
 
 
 class ShError(RuntimeError):
@@ -76,7 +76,9 @@ class Stats(C.Structure):
                 ("h2d_busy_ms", C.c_double), ("d2h_busy_ms", C.c_double), ("h2d_profiled_bytes", C.c_int64),
                 ("d2h_profiled_bytes", C.c_int64), ("cpu_adam_ms", C.c_double), ("cpu_adam_elems", C.c_int64),
                 ("cpu_wait_ms", C.c_double), ("k2_ms_last", C.c_double), ("k2_bytes_last", C.c_int64),
-                ("k2_launches_last", C.c_int32), ("cpu_threads", C.c_int32), ("profiled_steps", C.c_int32)]
+                ("k2_launches_last", C.c_int32), ("cpu_threads", C.c_int32), ("profiled_steps", C.c_int32),
+                ("k2_ms_sum", C.c_double), ("k2_bytes_sum", C.c_int64), ("k2_samples", C.c_int64),
+                ("k3_ms_sum", C.c_double), ("k3_bytes_sum", C.c_int64), ("k3_samples", C.c_int64)]
 
 
 class AdamScalars(C.Structure):
@@ -121,6 +123,7 @@ def lib() -> C.CDLL:
         L.sh_last_error.restype = C.c_char_p
         L.sh_last_error.argtypes = []
         L.sh_abi_version.restype = C.c_int32
+        L.sh_kernel_launches.restype = C.c_int64
         _lib = L
     return _lib
 
@@ -179,6 +182,10 @@ def op_cast_bf16_cpu(src, dst16, n):
 
 def op_sumsq_gpu(g, n, out_dev, stream=None):
     check(lib().sh_op_sumsq_gpu(_ptr(g), n, _ptr(out_dev), _stream_handle(stream)))
+
+
+def kernel_launches() -> int:
+    return int(lib().sh_kernel_launches())
 
 
 def nccl_unique_id() -> bytes:
