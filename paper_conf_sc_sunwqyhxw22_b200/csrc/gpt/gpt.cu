@@ -1,8 +1,11 @@
 // GPT-2 block compute that drives the offload engine -- OUTSIDE THE HOT PATH (see sh_gpt.h).
 //
-// GEMMs: cuBLAS (bf16 or fp32 operands, fp32 accumulation, CUBLAS_COMPUTE_32F, fixed
-// workspace => run-to-run bitwise reproducible; on sm_100 the bf16 GEMMs run on tcgen05 tensor
-// cores inside cuBLAS).  Everything else is small SIMT kernels with fixed reduction orders.
+// GEMMs: cuBLAS (bf16 or fp32 operands, fp32 accumulation, CUBLAS_COMPUTE_32F, fixed workspace,
+// atomics disallowed => run-to-run bitwise reproducible; on sm_100 the bf16 GEMMs run on the
+// tcgen05 tensor cores inside cuBLAS).  Attention runs as pointer-array batched GEMMs directly
+// on the [N, 3h] qkv layout (no permute kernels); biases are folded into the GEMMs by a
+// broadcast prefill + beta = 1 (one rounding of acc + bias).  The remaining SIMT kernels are
+// HBM-bound and move 16-byte vectors (8 bf16 / 2 x 4 fp32) with fixed reduction orders.
 // The math is DESIGN.md reading R1 / oracle/gpt_oracle.py (shared by definition, not code).
 #include <cublas_v2.h>
 #include <cuda_bf16.h>
@@ -41,6 +44,35 @@ template <class T> __device__ __forceinline__ T fromf(float x);
 template <> __device__ __forceinline__ float fromf<float>(float x) { return x; }
 template <> __device__ __forceinline__ bf16 fromf<bf16>(float x) { return __float2bfloat16_rn(x); }
 
+// 8-element vector load/store as floats (16 B for bf16, 2 x 16 B for fp32)
+__device__ __forceinline__ void ld8(const float* p, float (&v)[8]) {
+  const float4 a = reinterpret_cast<const float4*>(p)[0], b = reinterpret_cast<const float4*>(p)[1];
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+}
+__device__ __forceinline__ void ld8(const bf16* p, float (&v)[8]) {
+  const uint4 u = *reinterpret_cast<const uint4*>(p);
+  const uint32_t w[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    v[2 * i] = __uint_as_float(w[i] << 16);
+    v[2 * i + 1] = __uint_as_float(w[i] & 0xffff0000u);
+  }
+}
+__device__ __forceinline__ void st8(float* p, const float (&v)[8]) {
+  reinterpret_cast<float4*>(p)[0] = make_float4(v[0], v[1], v[2], v[3]);
+  reinterpret_cast<float4*>(p)[1] = make_float4(v[4], v[5], v[6], v[7]);
+}
+__device__ __forceinline__ void st8(bf16* p, const float (&v)[8]) {
+  uint32_t w[4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t lo = __bfloat16_as_ushort(__float2bfloat16_rn(v[2 * i]));
+    const uint32_t hi = __bfloat16_as_ushort(__float2bfloat16_rn(v[2 * i + 1]));
+    w[i] = lo | (hi << 16);
+  }
+  *reinterpret_cast<uint4*>(p) = make_uint4(w[0], w[1], w[2], w[3]);
+}
+
 __device__ __forceinline__ float warp_sum(float x) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
@@ -61,8 +93,10 @@ __device__ __forceinline__ float block_reduce(float x, bool is_max) {
   __syncthreads();
   float r = l < NT / 32 ? sh[l] : (is_max ? -INFINITY : 0.f);
   r = is_max ? warp_max(r) : warp_sum(r);
-  return r;  // every thread of warp 0.. holds the result (all warps compute it)
+  return r;  // every warp computes the same fixed-order result
 }
+
+#define GRID_STRIDE(i, n) for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (n); i += (int64_t)gridDim.x * blockDim.x)
 
 // ------------------------------------------------------------------------------ kernels
 template <class T>
@@ -70,10 +104,17 @@ __global__ void embed_fwd(const int* tok, const T* wte, const T* wpe, float* x, 
   const int n = blockIdx.x;  // token row b*S+s
   const int b = n / S, s = n % S;
   const int t = tok[b * (S + 1) + s];
-  for (int c = threadIdx.x; c < h; c += blockDim.x)
-    x[(int64_t)n * h + c] = tof(wte[(int64_t)t * h + c]) + tof(wpe[(int64_t)s * h + c]);
+  for (int c = 8 * threadIdx.x; c < h; c += 8 * blockDim.x) {
+    float a[8], p[8];
+    ld8(wte + (int64_t)t * h + c, a);
+    ld8(wpe + (int64_t)s * h + c, p);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a[i] += p[i];
+    st8(x + (int64_t)n * h + c, a);
+  }
 }
 
+// one warp per row; two-pass statistics (mean, then centred variance) in fp32
 template <class T>
 __global__ void ln_fwd(const float* x, const T* g, const T* b, T* out, float* mean, float* rstd, int N, int h) {
   const int row = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
@@ -81,16 +122,31 @@ __global__ void ln_fwd(const float* x, const T* g, const T* b, T* out, float* me
   if (row >= N) return;
   const float* xr = x + (int64_t)row * h;
   float s = 0.f;
-  for (int c = lane; c < h; c += 32) s += xr[c];
-  const float mu = warp_sum(s) / h;
-  float v = 0.f;
-  for (int c = lane; c < h; c += 32) {
-    const float d = xr[c] - mu;
-    v += d * d;
+  for (int c = 8 * lane; c < h; c += 256) {
+    float v[8];
+    ld8(xr + c, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) s += v[i];
   }
-  const float rs = 1.0f / sqrtf(warp_sum(v) / h + kLnEps);
+  const float mu = warp_sum(s) / h;
+  float var = 0.f;
+  for (int c = 8 * lane; c < h; c += 256) {
+    float v[8];
+    ld8(xr + c, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) var += (v[i] - mu) * (v[i] - mu);
+  }
+  const float rs = 1.0f / sqrtf(warp_sum(var) / h + kLnEps);
   T* o = out + (int64_t)row * h;
-  for (int c = lane; c < h; c += 32) o[c] = fromf<T>((xr[c] - mu) * rs * tof(g[c]) + tof(b[c]));
+  for (int c = 8 * lane; c < h; c += 256) {
+    float v[8], gg[8], bb[8];
+    ld8(xr + c, v);
+    ld8(g + c, gg);
+    ld8(b + c, bb);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = (v[i] - mu) * rs * gg[i] + bb[i];
+    st8(o + c, v);
+  }
   if (lane == 0) {
     mean[row] = mu;
     rstd[row] = rs;
@@ -108,99 +164,60 @@ __global__ void ln_bwd(const float* dy, const float* x, const float* mean, const
   const float* xr = x + (int64_t)row * h;
   const float mu = mean[row], rs = rstd[row];
   float a = 0.f, bb = 0.f;
-  for (int c = lane; c < h; c += 32) {
-    const float xh = (xr[c] - mu) * rs;
-    const float dxh = dr[c] * tof(g[c]);
-    a += dxh;
-    bb += dxh * xh;
+  for (int c = 8 * lane; c < h; c += 256) {
+    float d[8], xv[8], gg[8];
+    ld8(dr + c, d);
+    ld8(xr + c, xv);
+    ld8(g + c, gg);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const float dxh = d[i] * gg[i];
+      a += dxh;
+      bb += dxh * ((xv[i] - mu) * rs);
+    }
   }
   a = warp_sum(a) / h;
   bb = warp_sum(bb) / h;
   float* o = dres + (int64_t)row * h;
   float* t = tmp + (int64_t)row * h;
-  for (int c = lane; c < h; c += 32) {
-    const float xh = (xr[c] - mu) * rs;
-    const float dxh = dr[c] * tof(g[c]);
-    o[c] += rs * (dxh - a - xh * bb);
-    t[c] = dr[c] * xh;
+  for (int c = 8 * lane; c < h; c += 256) {
+    float d[8], xv[8], gg[8], ov[8], tv[8];
+    ld8(dr + c, d);
+    ld8(xr + c, xv);
+    ld8(g + c, gg);
+    ld8(o + c, ov);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const float xh = (xv[i] - mu) * rs;
+      ov[i] += rs * (d[i] * gg[i] - a - xh * bb);
+      tv[i] = d[i] * xh;
+    }
+    st8(o + c, ov);
+    st8(t + c, tv);
   }
 }
 
-// qkv (fp32, no bias) [N,3h] + bias -> q,k,v [B,nh,S,hd] in T
+// out[r, :] = bias (T) or x[r, :] + bias (fp32 residual); C % 8 == 0
 template <class T>
-__global__ void qkv_split(const float* qkv, const T* bias, T* q, T* k, T* v, int S, int h, int nh, int64_t total) {
-  const int hd = h / nh;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t n = i / (3 * h);
-    const int c = (int)(i % (3 * h));
-    const int which = c / h, cc = c % h, head = cc / hd, d = cc % hd;
-    const int64_t b = n / S, s = n % S;
-    const int64_t dst = ((b * nh + head) * S + s) * hd + d;
-    const T val = fromf<T>(qkv[i] + tof(bias[c]));
-    (which == 0 ? q : which == 1 ? k : v)[dst] = val;
-  }
-}
-
-// [B,nh,S,hd] <-> [N,h]
-template <class T>
-__global__ void heads_to_rows(const T* src, T* dst, int S, int h, int nh, int64_t total, int rows_stride, int col_off) {
-  const int hd = h / nh;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t n = i / h;
-    const int c = (int)(i % h), head = c / hd, d = c % hd;
-    const int64_t b = n / S, s = n % S;
-    dst[n * rows_stride + col_off + c] = src[((b * nh + head) * S + s) * hd + d];
+__global__ void bias_fill(T* out, const T* bias, int C, int64_t n8) {
+  const int c8 = C / 8;
+  GRID_STRIDE(j, n8) {
+    float v[8];
+    ld8(bias + (j % c8) * 8, v);
+    st8(out + 8 * j, v);
   }
 }
 template <class T>
-__global__ void rows_to_heads(const T* src, T* dst, int S, int h, int nh, int64_t total) {
-  const int hd = h / nh;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t n = i / h;
-    const int c = (int)(i % h), head = c / hd, d = c % hd;
-    const int64_t b = n / S, s = n % S;
-    dst[((b * nh + head) * S + s) * hd + d] = src[i];
+__global__ void resid_bias(const float* x, const T* bias, float* out, int C, int64_t n8) {
+  const int c8 = C / 8;
+  GRID_STRIDE(j, n8) {
+    float v[8], b[8];
+    ld8(x + 8 * j, v);
+    ld8(bias + (j % c8) * 8, b);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] += b[i];
+    st8(out + 8 * j, v);
   }
-}
-
-// causal softmax, one warp per row: scores already scaled by 1/sqrt(hd)
-template <class T>
-__global__ void softmax_causal(const float* sc, T* p, int S, int64_t rows) {
-  const int64_t row = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5);
-  const int lane = threadIdx.x & 31;
-  if (row >= rows) return;
-  const int r = (int)(row % S);
-  const float* s = sc + row * S;
-  T* o = p + row * S;
-  float m = -INFINITY;
-  for (int c = lane; c <= r; c += 32) m = fmaxf(m, s[c]);
-  m = warp_max(m);
-  float z = 0.f;
-  for (int c = lane; c <= r; c += 32) z += expf(s[c] - m);
-  z = warp_sum(z);
-  const float inv = 1.0f / z;
-  for (int c = lane; c < S; c += 32) o[c] = fromf<T>(c <= r ? expf(s[c] - m) * inv : 0.f);
-}
-
-// dS = P * (dP - Σ dP*P), written in place over P
-template <class T>
-__global__ void softmax_bwd(T* p, const float* dp, int S, int64_t rows) {
-  const int64_t row = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5);
-  const int lane = threadIdx.x & 31;
-  if (row >= rows) return;
-  const int r = (int)(row % S);
-  T* pr = p + row * S;
-  const float* d = dp + row * S;
-  float a = 0.f;
-  for (int c = lane; c <= r; c += 32) a += tof(pr[c]) * d[c];
-  a = warp_sum(a);
-  for (int c = lane; c <= r; c += 32) pr[c] = fromf<T>(tof(pr[c]) * (d[c] - a));
-}
-
-template <class T>
-__global__ void resid_bias(const float* x, const T* b, float* out, int h, int64_t total) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
-    out[i] = x[i] + tof(b[i % h]);
 }
 
 __device__ __forceinline__ float gelu_f(float u) {
@@ -214,27 +231,120 @@ __device__ __forceinline__ float gelu_grad(float u) {
 }
 
 template <class T>
-__global__ void gelu_fwd(const float* f, const T* b, T* pre, T* act, int C, int64_t total) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const T u = fromf<T>(f[i] + tof(b[i % C]));
-    pre[i] = u;
-    act[i] = fromf<T>(gelu_f(tof(u)));
+__global__ void gelu_fwd(const T* pre, T* act, int64_t n8) {
+  GRID_STRIDE(j, n8) {
+    float v[8];
+    ld8(pre + 8 * j, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = gelu_f(v[i]);
+    st8(act + 8 * j, v);
   }
 }
 template <class T>
-__global__ void gelu_bwd(T* d, const T* pre, int64_t total) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
-    d[i] = fromf<T>(tof(d[i]) * gelu_grad(tof(pre[i])));
+__global__ void gelu_bwd(T* d, const T* pre, int64_t n8) {
+  GRID_STRIDE(j, n8) {
+    float v[8], u[8];
+    ld8(d + 8 * j, v);
+    ld8(pre + 8 * j, u);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] *= gelu_grad(u[i]);
+    st8(d + 8 * j, v);
+  }
 }
 template <class T>
-__global__ void cast_f2t(const float* a, T* o, int64_t total) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
-    o[i] = fromf<T>(a[i]);
+__global__ void cast_f2t(const float* a, T* o, int64_t n8) {
+  GRID_STRIDE(j, n8) {
+    float v[8];
+    ld8(a + 8 * j, v);
+    st8(o + 8 * j, v);
+  }
 }
 template <class T>
 __global__ void fill_ones(T* o, int64_t n) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    o[i] = fromf<T>(1.0f);
+  GRID_STRIDE(i, n) o[i] = fromf<T>(1.0f);
+}
+
+// Causal softmax, one warp per score row; lane owns 8-column chunks lane, lane+32, ...
+// (NCH = chunks per lane).  Chunks entirely above the diagonal are never read (exact zeros).
+template <class T, int NCH>
+__global__ void softmax_causal(const float* sc, T* p, int S, int64_t rows) {
+  const int64_t row = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (row >= rows) return;
+  const int r = (int)(row % S);
+  const float* s = sc + row * S;
+  T* o = p + row * S;
+  float v[NCH][8];
+  float m = -INFINITY;
+#pragma unroll
+  for (int k = 0; k < NCH; ++k) {
+    const int c0 = 8 * (lane + 32 * k);
+    if (c0 < S && c0 <= r) {
+      ld8(s + c0, v[k]);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        if (c0 + i > r) v[k][i] = -INFINITY;
+        m = fmaxf(m, v[k][i]);
+      }
+    }
+  }
+  m = warp_max(m);
+  float z = 0.f;
+#pragma unroll
+  for (int k = 0; k < NCH; ++k) {
+    const int c0 = 8 * (lane + 32 * k);
+    if (c0 < S && c0 <= r) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        v[k][i] = c0 + i <= r ? expf(v[k][i] - m) : 0.f;
+        z += v[k][i];
+      }
+    }
+  }
+  const float inv = 1.0f / warp_sum(z);
+#pragma unroll
+  for (int k = 0; k < NCH; ++k) {
+    const int c0 = 8 * (lane + 32 * k);
+    if (c0 < S) {
+      float w[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) w[i] = c0 <= r ? v[k][i] * inv : 0.f;
+      st8(o + c0, w);
+    }
+  }
+}
+
+// dS = P * (dP - Σ dP*P), written in place over P (chunks above the diagonal stay 0)
+template <class T, int NCH>
+__global__ void softmax_bwd(T* p, const float* dp, int S, int64_t rows) {
+  const int64_t row = blockIdx.x * (int64_t)(blockDim.x / 32) + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (row >= rows) return;
+  const int r = (int)(row % S);
+  T* pr = p + row * S;
+  const float* d = dp + row * S;
+  float pv[NCH][8], dv[NCH][8];
+  float a = 0.f;
+#pragma unroll
+  for (int k = 0; k < NCH; ++k) {
+    const int c0 = 8 * (lane + 32 * k);
+    if (c0 < S && c0 <= r) {
+      ld8(pr + c0, pv[k]);
+      ld8(d + c0, dv[k]);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) a += pv[k][i] * dv[k][i];  // P == 0 above the diagonal
+    }
+  }
+  a = warp_sum(a);
+#pragma unroll
+  for (int k = 0; k < NCH; ++k) {
+    const int c0 = 8 * (lane + 32 * k);
+    if (c0 < S && c0 <= r) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) pv[k][i] = pv[k][i] * (dv[k][i] - a);
+      st8(pr + c0, pv[k]);
+    }
+  }
 }
 
 // cross entropy per row (block of 512): loss_n, dlogits_n = (softmax - onehot)/Ntot
@@ -246,19 +356,35 @@ __global__ void __launch_bounds__(512) ce_fwd_bwd(const float* logits, const int
   const int tgt = tok[b * (S + 1) + s + 1];
   const float* l = logits + n * V;
   float m = -INFINITY;
-  for (int c = threadIdx.x; c < V; c += 512) m = fmaxf(m, l[c]);
+  for (int c = 8 * threadIdx.x; c < V; c += 8 * 512) {
+    float v[8];
+    ld8(l + c, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) m = fmaxf(m, v[i]);
+  }
   m = block_reduce<512>(m, true);
   float z = 0.f;
-  for (int c = threadIdx.x; c < V; c += 512) z += expf(l[c] - m);
+  for (int c = 8 * threadIdx.x; c < V; c += 8 * 512) {
+    float v[8];
+    ld8(l + c, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) z += expf(v[i] - m);
+  }
   z = block_reduce<512>(z, false);
   const float inv = 1.0f / z;
   const float lt = l[tgt];
   __syncthreads();  // all reads of l[] done before an in-place (fp32) overwrite
   T* d = dlogits + n * V;
-  for (int c = threadIdx.x; c < V; c += 512) {
-    float p = expf(l[c] - m) * inv;
-    if (c == tgt) p -= 1.0f;
-    d[c] = fromf<T>(p * inv_n);
+  for (int c = 8 * threadIdx.x; c < V; c += 8 * 512) {
+    float v[8];
+    ld8(l + c, v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      float pr = expf(v[i] - m) * inv;
+      if (c + i == tgt) pr -= 1.0f;
+      v[i] = pr * inv_n;
+    }
+    st8(d + c, v);
   }
   if (threadIdx.x == 0) row_loss[n] = logf(z) + m - lt;
 }
@@ -297,6 +423,26 @@ __global__ void embed_bwd_wpe(const float* dx, float* dwpe, int B, int S, int h)
   }
 }
 
+// pointer arrays of the per-(batch, head) attention operands on the [N, 3h] / [N, h] layouts
+__global__ void build_attn_ptrs(void** P, char* qkv, char* scores, char* probs, char* att, char* datt,
+                                char* dqkv, int B, int nh, int S, int h, int es) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int BH = B * nh;
+  if (i >= BH) return;
+  const int b = i / nh, hd_i = i % nh, hd = h / nh;
+  const int64_t row3 = (int64_t)b * S * 3 * h, row1 = (int64_t)b * S * h, col = (int64_t)hd_i * hd;
+  P[0 * BH + i] = qkv + es * (row3 + col);
+  P[1 * BH + i] = qkv + es * (row3 + h + col);
+  P[2 * BH + i] = qkv + es * (row3 + 2 * h + col);
+  P[3 * BH + i] = scores + 4 * (int64_t)i * S * S;
+  P[4 * BH + i] = probs + es * (int64_t)i * S * S;
+  P[5 * BH + i] = att + es * (row1 + col);
+  P[6 * BH + i] = datt + es * (row1 + col);
+  P[7 * BH + i] = dqkv + es * (row3 + col);
+  P[8 * BH + i] = dqkv + es * (row3 + h + col);
+  P[9 * BH + i] = dqkv + es * (row3 + 2 * h + col);
+}
+
 int grid_for(int64_t total, int threads = 256) {
   int64_t g = (total + threads - 1) / threads;
   const int64_t cap = 148 * 16;
@@ -315,12 +461,14 @@ struct gpt_ctx {
   void* ws = nullptr;
   size_t ws_bytes = 64u << 20;
   int B = 0, N = 0, S = 0, h = 0, nh = 0, V = 0, L = 0;
+  int ptrB = -1;
   int64_t maxN = 0;
   std::vector<void*> allocs;
   int64_t bytes = 0;
   float* x = nullptr;  // (L+1) checkpoints
-  void *ln1, *ln2, *lnf, *q, *k, *v, *probs, *atto, *att, *fc_pre, *fc_act, *dy, *d4h, *datt, *dO, *dq, *dk, *dv, *dqkv, *ones_t, *dlogits;
-  float *ln1_m, *ln1_r, *ln2_m, *ln2_r, *lnf_m, *lnf_r, *f32big, *scores, *x_mid, *dres, *dln, *tmp, *logits, *row_loss, *ones_f;
+  void *ln1, *ln2, *lnf, *qkv, *probs, *att, *fc_pre, *fc_act, *dy, *d4h, *datt, *dqkv, *ones_t, *dlogits;
+  float *ln1_m, *ln1_r, *ln2_m, *ln2_r, *lnf_m, *lnf_r, *scores, *x_mid, *dres, *dln, *tmp, *logits, *row_loss, *ones_f;
+  void** aptr = nullptr;  // 10 x BH attention operand pointers
   int *keys, *vals, *keys2, *vals2;
   void* cub_tmp = nullptr;
   size_t cub_bytes = 0;
@@ -357,21 +505,25 @@ int alloc(gpt_ctx* c, void** p, int64_t bytes) {
     }                                                             \
   } while (0)
 
-// Row-major C[M,N] = alpha op(A) op(B) + beta C.  A is [M,K] (or stored [K,M] if tA),
-// B is [K,N] (or stored [N,K] if tB).  Column-major cuBLAS computes C^T = op(B)^T op(A)^T.
+// Row-major C[M,N] (row stride ldc) = alpha op(A) op(B) + beta C.  A is [M,K] (or stored [K,M]
+// if tA) with row stride lda; B is [K,N] (or stored [N,K] if tB) with row stride ldb.
+// Column-major cuBLAS computes C^T = op(B)^T op(A)^T.
+cublasStatus_t gemm(gpt_ctx* c, bool tA, bool tB, int M, int N, int K, float alpha, const void* A, cudaDataType_t ta,
+                    int lda, const void* B, cudaDataType_t tb, int ldb, float beta, void* C, cudaDataType_t tc, int ldc) {
+  return cublasGemmEx(c->cb, tB ? CUBLAS_OP_T : CUBLAS_OP_N, tA ? CUBLAS_OP_T : CUBLAS_OP_N, N, M, K, &alpha, B, tb,
+                      ldb, A, ta, lda, &beta, C, tc, ldc, CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT);
+}
 cublasStatus_t rm_gemm(gpt_ctx* c, bool tA, bool tB, int M, int N, int K, float alpha, const void* A,
                        cudaDataType_t ta, const void* B, cudaDataType_t tb, float beta, void* C, cudaDataType_t tc) {
-  const int lda = tA ? M : K, ldb = tB ? K : N;
-  return cublasGemmEx(c->cb, tB ? CUBLAS_OP_T : CUBLAS_OP_N, tA ? CUBLAS_OP_T : CUBLAS_OP_N, N, M, K, &alpha, B, tb,
-                      ldb, A, ta, lda, &beta, C, tc, N, CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT);
+  return gemm(c, tA, tB, M, N, K, alpha, A, ta, tA ? M : K, B, tb, tB ? K : N, beta, C, tc, N);
 }
-cublasStatus_t rm_gemm_batched(gpt_ctx* c, bool tA, bool tB, int M, int N, int K, float alpha, const void* A,
-                               cudaDataType_t ta, int64_t sA, const void* B, cudaDataType_t tb, int64_t sB, float beta,
-                               void* C, cudaDataType_t tc, int64_t sC, int batch) {
-  const int lda = tA ? M : K, ldb = tB ? K : N;
-  return cublasGemmStridedBatchedEx(c->cb, tB ? CUBLAS_OP_T : CUBLAS_OP_N, tA ? CUBLAS_OP_T : CUBLAS_OP_N, N, M, K,
-                                    &alpha, B, tb, ldb, sB, A, ta, lda, sA, &beta, C, tc, N, sC, batch,
-                                    CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT);
+// batched over pointer arrays (attention): operand pointer arrays Ap, Bp, Cp on the device
+cublasStatus_t gemm_ptr(gpt_ctx* c, bool tA, bool tB, int M, int N, int K, float alpha, void* const* Ap,
+                        cudaDataType_t ta, int lda, void* const* Bp, cudaDataType_t tb, int ldb, float beta,
+                        void* const* Cp, cudaDataType_t tc, int ldc, int batch) {
+  return cublasGemmBatchedEx(c->cb, tB ? CUBLAS_OP_T : CUBLAS_OP_N, tA ? CUBLAS_OP_T : CUBLAS_OP_N, N, M, K, &alpha,
+                             (const void* const*)Bp, tb, ldb, (const void* const*)Ap, ta, lda, &beta, Cp, tc, ldc,
+                             batch, CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT);
 }
 
 // out[C] (fp32) = Σ_rows X[rows, C] (fixed-order cuBLAS reduction)
@@ -385,37 +537,58 @@ int colsum(gpt_ctx* c, const void* X, bool x_is_f32, int rows, int C, float* out
   return 0;
 }
 
+template <class T, int NCH>
+void launch_softmax(gpt_ctx* c, int64_t rows, bool bwd) {
+  if (bwd)
+    (g_launches++, 0), softmax_bwd<T, NCH><<<(int)((rows + 7) / 8), 256, 0, c->st>>>((T*)c->probs, c->scores, c->S, rows);
+  else
+    (g_launches++, 0), softmax_causal<T, NCH><<<(int)((rows + 7) / 8), 256, 0, c->st>>>(c->scores, (T*)c->probs, c->S, rows);
+}
+template <class T>
+int softmax(gpt_ctx* c, int64_t rows, bool bwd) {
+  const int nch = (c->S / 8 + 31) / 32;
+  switch (nch) {
+    case 1: launch_softmax<T, 1>(c, rows, bwd); break;
+    case 2: launch_softmax<T, 2>(c, rows, bwd); break;
+    case 4: launch_softmax<T, 4>(c, rows, bwd); break;
+    case 8: launch_softmax<T, 8>(c, rows, bwd); break;
+    default: seterr("gpt: seq %d unsupported (S/256 must be 1, 2, 4 or 8 chunks per lane)", c->S); return -1;
+  }
+  return 0;
+}
+
+void** AP(gpt_ctx* c, int k) { return c->aptr + (int64_t)k * c->B * c->nh; }
+enum { PQ = 0, PK, PV, PS, PP, PO, PDO, PDQ, PDK, PDV };
+
 template <class T>
 int layer_fwd_impl(gpt_ctx* c, int l, void* const* P, bool write_out) {
   const int N = c->N, h = c->h, S = c->S, nh = c->nh, hd = h / nh, B = c->B;
   const cudaDataType_t dt = c->dt;
   const float* xin = c->x + (int64_t)l * c->maxN * h;
   float* xout = c->x + (int64_t)(l + 1) * c->maxN * h;
-  const int rows_per_blk = 8;
-  (g_launches++, 0), ln_fwd<T><<<(N + rows_per_blk - 1) / rows_per_blk, 256, 0, c->st>>>(xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
-                                                                      c->ln1_m, c->ln1_r, N, h);
-  CB(rm_gemm(c, false, true, N, 3 * h, h, 1.f, c->ln1, dt, P[2], dt, 0.f, c->f32big, CUDA_R_32F));
-  (g_launches++, 0), qkv_split<T><<<grid_for((int64_t)N * 3 * h), 256, 0, c->st>>>(c->f32big, (const T*)P[3], (T*)c->q, (T*)c->k,
-                                                                (T*)c->v, S, h, nh, (int64_t)N * 3 * h);
+  const int64_t Nh = (int64_t)N * h;
+  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
+                                                               c->ln1_m, c->ln1_r, N, h);
+  (g_launches++, 0), bias_fill<T><<<grid_for(3 * Nh / 8), 256, 0, c->st>>>((T*)c->qkv, (const T*)P[3], 3 * h, 3 * Nh / 8);
+  CB(rm_gemm(c, false, true, N, 3 * h, h, 1.f, c->ln1, dt, P[2], dt, 1.f, c->qkv, dt));
   const int BH = B * nh;
   const float scale = 1.0f / sqrtf((float)hd);
-  CB(rm_gemm_batched(c, false, true, S, S, hd, scale, c->q, dt, (int64_t)S * hd, c->k, dt, (int64_t)S * hd, 0.f,
-                     c->scores, CUDA_R_32F, (int64_t)S * S, BH));
-  const int64_t rows = (int64_t)BH * S;
-  (g_launches++, 0), softmax_causal<T><<<(int)((rows + 7) / 8), 256, 0, c->st>>>(c->scores, (T*)c->probs, S, rows);
-  CB(rm_gemm_batched(c, false, false, S, hd, S, 1.f, c->probs, dt, (int64_t)S * S, c->v, dt, (int64_t)S * hd, 0.f,
-                     c->atto, dt, (int64_t)S * hd, BH));
-  (g_launches++, 0), heads_to_rows<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>((const T*)c->atto, (T*)c->att, S, h, nh,
-                                                                 (int64_t)N * h, h, 0);
-  (g_launches++, 0), resid_bias<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>(xin, (const T*)P[5], c->x_mid, h, (int64_t)N * h);
+  CB(gemm_ptr(c, false, true, S, S, hd, scale, AP(c, PQ), dt, 3 * h, AP(c, PK), dt, 3 * h, 0.f, AP(c, PS),
+              CUDA_R_32F, S, BH));
+  int r = softmax<T>(c, (int64_t)BH * S, false);
+  if (r) return r;
+  CB(gemm_ptr(c, false, false, S, hd, S, 1.f, AP(c, PP), dt, S, AP(c, PV), dt, 3 * h, 0.f, AP(c, PO), dt, h, BH));
+  (g_launches++, 0), resid_bias<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(xin, (const T*)P[5], c->x_mid, h, Nh / 8);
   CB(rm_gemm(c, false, true, N, h, h, 1.f, c->att, dt, P[4], dt, 1.f, c->x_mid, CUDA_R_32F));
-  (g_launches++, 0), ln_fwd<T><<<(N + rows_per_blk - 1) / rows_per_blk, 256, 0, c->st>>>(c->x_mid, (const T*)P[6], (const T*)P[7],
-                                                                      (T*)c->ln2, c->ln2_m, c->ln2_r, N, h);
-  CB(rm_gemm(c, false, true, N, 4 * h, h, 1.f, c->ln2, dt, P[8], dt, 0.f, c->f32big, CUDA_R_32F));
-  (g_launches++, 0), gelu_fwd<T><<<grid_for((int64_t)N * 4 * h), 256, 0, c->st>>>(c->f32big, (const T*)P[9], (T*)c->fc_pre,
-                                                               (T*)c->fc_act, 4 * h, (int64_t)N * 4 * h);
+  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->x_mid, (const T*)P[6], (const T*)P[7],
+                                                               (T*)c->ln2, c->ln2_m, c->ln2_r, N, h);
+  (g_launches++, 0), bias_fill<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((T*)c->fc_pre, (const T*)P[9], 4 * h,
+                                                                          4 * Nh / 8);
+  CB(rm_gemm(c, false, true, N, 4 * h, h, 1.f, c->ln2, dt, P[8], dt, 1.f, c->fc_pre, dt));
+  (g_launches++, 0), gelu_fwd<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((const T*)c->fc_pre, (T*)c->fc_act,
+                                                                         4 * Nh / 8);
   if (write_out) {
-    (g_launches++, 0), resid_bias<T><<<grid_for((int64_t)N * h), 256, 0, c->st>>>(c->x_mid, (const T*)P[11], xout, h, (int64_t)N * h);
+    (g_launches++, 0), resid_bias<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(c->x_mid, (const T*)P[11], xout, h, Nh / 8);
     CB(rm_gemm(c, false, true, N, h, 4 * h, 1.f, c->fc_act, dt, P[10], dt, 1.f, xout, CUDA_R_32F));
   }
   CK(cudaGetLastError());
@@ -431,39 +604,38 @@ int layer_bwd_impl(gpt_ctx* c, int l, void* const* P, float* const* G) {
   const float* xin = c->x + (int64_t)l * c->maxN * h;
   const int64_t Nh = (int64_t)N * h;
   // ---- MLP
-  (g_launches++, 0), cast_f2t<T><<<grid_for(Nh), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh);
+  (g_launches++, 0), cast_f2t<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh / 8);
   CB(rm_gemm(c, true, false, h, 4 * h, N, 1.f, c->dy, dt, c->fc_act, dt, 0.f, G[10], CUDA_R_32F));
   if ((r = colsum(c, c->dres, true, N, h, G[11]))) return r;
   CB(rm_gemm(c, false, false, N, 4 * h, h, 1.f, c->dy, dt, P[10], dt, 0.f, c->d4h, dt));
-  (g_launches++, 0), gelu_bwd<T><<<grid_for(4 * Nh), 256, 0, c->st>>>((T*)c->d4h, (const T*)c->fc_pre, 4 * Nh);
+  (g_launches++, 0), gelu_bwd<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((T*)c->d4h, (const T*)c->fc_pre, 4 * Nh / 8);
   CB(rm_gemm(c, true, false, 4 * h, h, N, 1.f, c->d4h, dt, c->ln2, dt, 0.f, G[8], CUDA_R_32F));
   if ((r = colsum(c, c->d4h, false, N, 4 * h, G[9]))) return r;
   CB(rm_gemm(c, false, false, N, h, 4 * h, 1.f, c->d4h, dt, P[8], dt, 0.f, c->dln, CUDA_R_32F));
-  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, c->x_mid, c->ln2_m, c->ln2_r, (const T*)P[6], c->dres, c->tmp, N, h);
+  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, c->x_mid, c->ln2_m, c->ln2_r, (const T*)P[6],
+                                                               c->dres, c->tmp, N, h);
   if ((r = colsum(c, c->tmp, true, N, h, G[6]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[7]))) return r;
   // ---- attention
-  (g_launches++, 0), cast_f2t<T><<<grid_for(Nh), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh);
+  (g_launches++, 0), cast_f2t<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh / 8);
   CB(rm_gemm(c, true, false, h, h, N, 1.f, c->dy, dt, c->att, dt, 0.f, G[4], CUDA_R_32F));
   if ((r = colsum(c, c->dres, true, N, h, G[5]))) return r;
   CB(rm_gemm(c, false, false, N, h, h, 1.f, c->dy, dt, P[4], dt, 0.f, c->datt, dt));
-  (g_launches++, 0), rows_to_heads<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->datt, (T*)c->dO, S, h, nh, Nh);
   const int BH = B * nh;
   const float scale = 1.0f / sqrtf((float)hd);
-  const int64_t sQ = (int64_t)S * hd, sS = (int64_t)S * S;
-  CB(rm_gemm_batched(c, false, true, S, S, hd, 1.f, c->dO, dt, sQ, c->v, dt, sQ, 0.f, c->scores, CUDA_R_32F, sS, BH));
-  CB(rm_gemm_batched(c, true, false, S, hd, S, 1.f, c->probs, dt, sS, c->dO, dt, sQ, 0.f, c->dv, dt, sQ, BH));
-  const int64_t rows = (int64_t)BH * S;
-  (g_launches++, 0), softmax_bwd<T><<<(int)((rows + 7) / 8), 256, 0, c->st>>>((T*)c->probs, c->scores, S, rows);
-  CB(rm_gemm_batched(c, false, false, S, hd, S, scale, c->probs, dt, sS, c->k, dt, sQ, 0.f, c->dq, dt, sQ, BH));
-  CB(rm_gemm_batched(c, true, false, S, hd, S, scale, c->probs, dt, sS, c->q, dt, sQ, 0.f, c->dk, dt, sQ, BH));
-  (g_launches++, 0), heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dq, (T*)c->dqkv, S, h, nh, Nh, 3 * h, 0);
-  (g_launches++, 0), heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dk, (T*)c->dqkv, S, h, nh, Nh, 3 * h, h);
-  (g_launches++, 0), heads_to_rows<T><<<grid_for(Nh), 256, 0, c->st>>>((const T*)c->dv, (T*)c->dqkv, S, h, nh, Nh, 3 * h, 2 * h);
+  CB(gemm_ptr(c, false, true, S, S, hd, 1.f, AP(c, PDO), dt, h, AP(c, PV), dt, 3 * h, 0.f, AP(c, PS), CUDA_R_32F, S,
+              BH));
+  CB(gemm_ptr(c, true, false, S, hd, S, 1.f, AP(c, PP), dt, S, AP(c, PDO), dt, h, 0.f, AP(c, PDV), dt, 3 * h, BH));
+  if ((r = softmax<T>(c, (int64_t)BH * S, true))) return r;
+  CB(gemm_ptr(c, false, false, S, hd, S, scale, AP(c, PP), dt, S, AP(c, PK), dt, 3 * h, 0.f, AP(c, PDQ), dt, 3 * h,
+              BH));
+  CB(gemm_ptr(c, true, false, S, hd, S, scale, AP(c, PP), dt, S, AP(c, PQ), dt, 3 * h, 0.f, AP(c, PDK), dt, 3 * h,
+              BH));
   CB(rm_gemm(c, true, false, 3 * h, h, N, 1.f, c->dqkv, dt, c->ln1, dt, 0.f, G[2], CUDA_R_32F));
   if ((r = colsum(c, c->dqkv, false, N, 3 * h, G[3]))) return r;
   CB(rm_gemm(c, false, false, N, h, 3 * h, 1.f, c->dqkv, dt, P[2], dt, 0.f, c->dln, CUDA_R_32F));
-  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xin, c->ln1_m, c->ln1_r, (const T*)P[0], c->dres, c->tmp, N, h);
+  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xin, c->ln1_m, c->ln1_r, (const T*)P[0],
+                                                               c->dres, c->tmp, N, h);
   if ((r = colsum(c, c->tmp, true, N, h, G[0]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[1]))) return r;
   CK(cudaGetLastError());
@@ -475,13 +647,15 @@ int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float
   const int N = c->N, h = c->h, V = c->V, S = c->S;
   const cudaDataType_t dt = c->dt;
   const float* xL = c->x + (int64_t)c->L * c->maxN * h;
-  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xL, (const T*)R[2], (const T*)R[3], (T*)c->lnf, c->lnf_m, c->lnf_r, N, h);
+  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xL, (const T*)R[2], (const T*)R[3], (T*)c->lnf,
+                                                               c->lnf_m, c->lnf_r, N, h);
   CB(rm_gemm(c, false, true, N, V, h, 1.f, c->lnf, dt, R[0], dt, 0.f, c->logits, CUDA_R_32F));
   (g_launches++, 0), ce_fwd_bwd<T><<<N, 512, 0, c->st>>>(c->logits, tok, S, V, 1.0f / N, c->row_loss, (T*)c->dlogits);
   (g_launches++, 0), mean_fixed<<<1, 512, 0, c->st>>>(c->row_loss, N, 1.0f / N, d_loss);
   CB(rm_gemm(c, false, false, N, h, V, 1.f, c->dlogits, dt, R[0], dt, 0.f, c->dln, CUDA_R_32F));
   CK(cudaMemsetAsync(c->dres, 0, sizeof(float) * (size_t)N * h, c->st));
-  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xL, c->lnf_m, c->lnf_r, (const T*)R[2], c->dres, c->tmp, N, h);
+  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xL, c->lnf_m, c->lnf_r, (const T*)R[2], c->dres,
+                                                               c->tmp, N, h);
   int r;
   if ((r = colsum(c, c->tmp, true, N, h, G[2]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[3]))) return r;
@@ -504,9 +678,15 @@ float* gpt_checkpoint(gpt_ctx* c, int32_t l) {
 
 int32_t gpt_create(const gpt_config* cfg, gpt_ctx** out) {
   g_err.clear();
-  if (!cfg || !out || cfg->n_layers < 1 || cfg->hidden < 1 || cfg->heads < 1 || cfg->hidden % cfg->heads ||
-      cfg->seq < 1 || cfg->max_batch < 1 || cfg->vocab < 1 || !cfg->stream) {
-    seterr("gpt_create: invalid config (hidden %% heads must be 0, stream required)");
+  if (!cfg || !out || cfg->n_layers < 1 || cfg->hidden < 8 || cfg->heads < 1 || cfg->hidden % cfg->heads ||
+      cfg->hidden % 8 || (cfg->hidden / cfg->heads) % 8 || cfg->seq < 8 || cfg->seq % 8 || cfg->max_batch < 1 ||
+      cfg->vocab < 8 || cfg->vocab % 8 || !cfg->stream) {
+    seterr("gpt_create: invalid config (hidden, head dim, seq and vocab must be multiples of 8; stream required)");
+    return -1;
+  }
+  const int nch = (cfg->seq / 8 + 31) / 32;
+  if (nch != 1 && nch != 2 && nch != 4 && nch != 8) {
+    seterr("gpt_create: seq %d unsupported by the softmax kernel", cfg->seq);
     return -1;
   }
   auto* c = new gpt_ctx();
@@ -533,16 +713,13 @@ int32_t gpt_create(const gpt_config* cfg, gpt_ctx** out) {
     if (!r) r = alloc(c, p, b);
   };
   A((void**)&c->x, 4 * (c->L + 1) * mN * h);
-  for (void** p : {&c->ln1, &c->ln2, &c->lnf, &c->q, &c->k, &c->v, &c->atto, &c->att, &c->dy, &c->datt, &c->dO, &c->dq,
-                   &c->dk, &c->dv})
-    A(p, es * mN * h);
-  A(&c->dqkv, es * mN * 3 * h);
+  for (void** p : {&c->ln1, &c->ln2, &c->lnf, &c->att, &c->dy, &c->datt}) A(p, es * mN * h);
+  for (void** p : {&c->qkv, &c->dqkv}) A(p, es * mN * 3 * h);
   for (void** p : {&c->fc_pre, &c->fc_act, &c->d4h}) A(p, es * mN * 4 * h);
   A(&c->probs, es * BHSS);
   A((void**)&c->scores, 4 * BHSS);
   for (float** p : {&c->ln1_m, &c->ln1_r, &c->ln2_m, &c->ln2_r, &c->lnf_m, &c->lnf_r, &c->row_loss, &c->ones_f})
     A((void**)p, 4 * mN);
-  A((void**)&c->f32big, 4 * mN * 4 * h);
   for (float** p : {&c->x_mid, &c->dres, &c->dln, &c->tmp}) A((void**)p, 4 * mN * h);
   A((void**)&c->logits, 4 * mN * c->V);
   if (c->bf16)
@@ -550,6 +727,7 @@ int32_t gpt_create(const gpt_config* cfg, gpt_ctx** out) {
   else
     c->dlogits = c->logits;  // fp32: dlogits overwrite logits in place
   A(&c->ones_t, es * mN);
+  A((void**)&c->aptr, 10 * 8 * (int64_t)cfg->max_batch * c->nh);
   for (int** p : {&c->keys, &c->vals, &c->keys2, &c->vals2}) A((void**)p, 4 * mN);
   A(&c->ws, c->ws_bytes);
   if (!r) {
@@ -600,10 +778,17 @@ int32_t gpt_embed_forward(gpt_ctx* c, const int32_t* tok, int32_t B, void* const
   }
   c->B = B;
   c->N = B * c->S;
+  if (c->ptrB != B) {
+    const int BH = B * c->nh;
+    (g_launches++, 0), build_attn_ptrs<<<(BH + 127) / 128, 128, 0, c->st>>>(
+        c->aptr, (char*)c->qkv, (char*)c->scores, (char*)c->probs, (char*)c->att, (char*)c->datt, (char*)c->dqkv, B,
+        c->nh, c->S, c->h, c->es);
+    c->ptrB = B;
+  }
   if (c->bf16)
-    (g_launches++, 0), embed_fwd<bf16><<<c->N, 256, 0, c->st>>>(tok, (const bf16*)R[0], (const bf16*)R[1], c->x, c->S, c->h);
+    (g_launches++, 0), embed_fwd<bf16><<<c->N, 128, 0, c->st>>>(tok, (const bf16*)R[0], (const bf16*)R[1], c->x, c->S, c->h);
   else
-    (g_launches++, 0), embed_fwd<float><<<c->N, 256, 0, c->st>>>(tok, (const float*)R[0], (const float*)R[1], c->x, c->S, c->h);
+    (g_launches++, 0), embed_fwd<float><<<c->N, 128, 0, c->st>>>(tok, (const float*)R[0], (const float*)R[1], c->x, c->S, c->h);
   CK(cudaGetLastError());
   return 0;
 }
