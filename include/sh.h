@@ -36,8 +36,9 @@
  *     g = g*coef (only when clipping is on);  m = fma(b1, m, omb1*g);
  *     v = fma(b2, v, omb2*(g*g));  d = sqrt(v)/sqrt_bc2 + eps;
  *     p = fma(-step_size, m/d, wd ? p*decay : p);  p16 = rne_bf16(p)
- *   with omb1 = 1-b1, omb2 = 1-b2, sqrt_bc2 = sqrt(1-b2^t), step_size = lr/(1-b1^t),
- *   decay = 1 - lr*lambda computed in double on the host and rounded once to fp32.
+ *   with b1, b2, eps, omb1 = 1-b1, omb2 = 1-b2, sqrt_bc2 = sqrt(1-b2^t), step_size = lr/(1-b1^t),
+ *   decay = 1 - lr*lambda computed in double from the double hyperparameters on the host and
+ *   rounded once to fp32.
  *   rne_bf16 is integer round-to-nearest-even with canonical NaN 0x7FC0.
  *
  * Errors: every call returns sh_status; no exception crosses the ABI.  The message
@@ -95,6 +96,7 @@ typedef struct {
 #define SH_FLAG_PROFILE   (1ull << 0) /* record per-layer CUDA events every step (else warm-up only) */
 #define SH_FLAG_POISON    (1ull << 1) /* debug: fill a slot's param half with NaN before every refill */
 #define SH_FLAG_DUPLEX    (1ull << 2) /* autotuner: full-duplex link, max() instead of sum in (1d)/(2d) */
+#define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
 typedef struct {
@@ -103,9 +105,9 @@ typedef struct {
   sh_layer_shape resident;          /* embedding / positions / final LN: always in HBM */
   int32_t window;                   /* 0..n_layers, or -1: w0 = min(2, w_max) then autotune after warm-up */
   int32_t precision;                /* sh_precision */
-  float lr;                         /* initial learning rate (sh_set_lr changes it) */
-  float beta1, beta2, eps, weight_decay;
-  float max_grad_norm;              /* <= 0: no clipping (throughput mode, R3) */
+  double lr;                        /* initial learning rate (sh_set_lr changes it) */
+  double beta1, beta2, eps, weight_decay;  /* doubles: the per-step scalars are derived in double */
+  double max_grad_norm;             /* <= 0: no clipping (throughput mode, R3) */
   int32_t device;                   /* CUDA ordinal */
   void* compute_stream;             /* caller-owned cudaStream_t for all layer compute (required) */
   int32_t cpu_threads;              /* CPU Adam threads; 0 = all online cores */
@@ -135,16 +137,20 @@ typedef struct {
   int64_t fixed_bytes;         /* HBM always used by the engine (resident set, scratch) */
   int64_t s_avail;             /* S_avail */
   int32_t duplex;              /* 1: soft constraints use max(Σc2g, Σg2c) (R7) */
+  int32_t cpu_hard;            /* 1: also require the CPU-update throughput form of eq. 3 (R19):
+                                  Σ_{k>=w} t_opt_cpu^k <= Σ_i (t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i */
 } sh_profile;
 
 typedef struct {
   int32_t window;          /* chosen w* */
   int32_t w_max_memory;    /* largest w meeting (1c)/(2c) */
-  int32_t reason;          /* 0: hard+soft met; 1: hard only; 2: memory fallback */
+  int32_t reason;          /* 0: hard+soft met (w < L); 1: hard only; 2: memory fallback */
   int32_t fp_hard_ok, bp_hard_ok, soft_ok;  /* at the chosen window */
   double eq3_min_slack_ms; /* min_k [Σ_{i<=k}(t_fp+t_bp) + Σ_{i<w} t_opt_gpu - t_opt_cpu_k]  (eq. 3) */
   int32_t eq3_ok;
   double eq4_lhs_ms, eq4_rhs_ms; /* 5 n t_async  vs  Σ_{i=w}^{n-1} t_opt_gpu (eq. 4) */
+  double cpu_total_ms;     /* Σ_{k>=w} t_opt_cpu^k at the chosen window */
+  double gpu_step_ms;      /* Σ_i (t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i */
 } sh_solve_report;
 
 typedef struct {
@@ -218,7 +224,7 @@ sh_status sh_backward_layer(sh_ctx* ctx, int32_t layer, int32_t phase, void** de
 sh_status sh_resident(sh_ctx* ctx, void** dev_params, float** dev_grads);
 
 /* Learning rate for the steps whose backward starts after this call. */
-sh_status sh_set_lr(sh_ctx* ctx, float lr);
+sh_status sh_set_lr(sh_ctx* ctx, double lr);
 
 /* End of step: finalize the global gradient norm in fixed order (K3
  * partials), then one fused multi-tensor AdamW (K2) over layers [0, w) and the
@@ -273,7 +279,7 @@ typedef struct {
 } sh_adam_scalars;
 
 /* Host-side derivation of the per-step fp32 scalars from (lr, t) in double. */
-sh_status sh_adam_scalars_for(float lr, float beta1, float beta2, float eps, float weight_decay,
+sh_status sh_adam_scalars_for(double lr, double beta1, double beta2, double eps, double weight_decay,
                               int64_t t, sh_adam_scalars* out);
 
 /* K2 on one flat tensor range: elements [0, n_decay) get weight decay, [n_decay, n) not.

@@ -14,7 +14,9 @@
 // link directions and the constraint is max(g2c, c2g) (a GPU-optimised entering layer is
 // restaged by K1: t_stage replaces t_c2g); the soft constraints use the paper's half-duplex
 // sum unless `duplex` is set (then max); "min m" with soft constraints is lexicographic:
-// hard and soft -> hard only -> memory maximum.  The implementation uses prefix sums; the
+// hard and soft (only for w < L: at w = L nothing moves and every window sum is empty, so the
+// soft constraint is vacuous there) -> hard only -> memory maximum.  Optional (cpu_hard, R19):
+// the CPU Adam of the host layers must fit in one step's GPU time (the throughput form of eq. 3).  The implementation uses prefix sums; the
 // oracle (oracle/autotune_oracle.py) evaluates the same definitions with plain loops.
 #include <algorithm>
 #include <cmath>
@@ -84,6 +86,15 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
     return true;
   };
 
+  auto cpu_total = [&](int w) {
+    double t = 0;
+    for (int k = w; k < L; ++k) t += at(P->t_opt_cpu, k);
+    return t;
+  };
+  auto gpu_step = [&](int w) { return fp.sum(0, L) + bp.sum(0, L) + ogpu.sum(0, w); };
+  auto hard = [&](int w) {
+    return fp_hard(w) && bp_hard(w) && (!P->cpu_hard || cpu_total(w) <= gpu_step(w));
+  };
   int wmax = -1;
   for (int w = 0; w <= L; ++w)
     if (mem_ok(w)) wmax = w;
@@ -92,10 +103,10 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
     return SH_ERR_OOM_DEVICE;
   }
   int best = -1, reason = 2;
+  for (int w = 0; w < L && best < 0; ++w)
+    if (mem_ok(w) && hard(w) && soft(w)) best = w, reason = 0;
   for (int w = 0; w <= L && best < 0; ++w)
-    if (mem_ok(w) && fp_hard(w) && bp_hard(w) && soft(w)) best = w, reason = 0;
-  for (int w = 0; w <= L && best < 0; ++w)
-    if (mem_ok(w) && fp_hard(w) && bp_hard(w)) best = w, reason = 1;
+    if (mem_ok(w) && hard(w)) best = w, reason = 1;
   if (best < 0) best = wmax, reason = 2;
 
   R->window = best;
@@ -115,5 +126,7 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
   // eq. 4: 5 n t_async ≤ Σ_{i=w}^{n-1} t_opt_gpu
   R->eq4_lhs_ms = 5.0 * L * P->t_async;
   R->eq4_rhs_ms = ogpu.sum(best, L);
+  R->cpu_total_ms = cpu_total(best);
+  R->gpu_step_ms = gpu_step(best);
   return SH_OK;
 }

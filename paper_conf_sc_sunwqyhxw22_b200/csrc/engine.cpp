@@ -260,7 +260,7 @@ struct sh_ctx {
   bool registered_all = false;
   std::vector<uint8_t> reg_done;
   bool res_reg = false;
-  float lr = 0;
+  double lr = 0;
   sh_adam_scalars sc{};
   cudaEvent_t ev_comm_done = nullptr, ev_cs_mark = nullptr;
 
@@ -903,22 +903,22 @@ sh_status sh_nccl_get_unique_id(void* out128) {
   return SH_OK;
 }
 
-sh_status sh_adam_scalars_for(float lr, float beta1, float beta2, float eps, float weight_decay,
+sh_status sh_adam_scalars_for(double lr, double beta1, double beta2, double eps, double weight_decay,
                               int64_t t, sh_adam_scalars* o) {
   if (!o || t < 1) {
     set_error("sh_adam_scalars_for: t must be >= 1");
     return SH_ERR_INVALID;
   }
-  const double bc1 = 1.0 - std::pow((double)beta1, (double)t);
-  const double bc2 = 1.0 - std::pow((double)beta2, (double)t);
-  o->beta1 = beta1;
-  o->beta2 = beta2;
-  o->omb1 = (float)(1.0 - (double)beta1);
-  o->omb2 = (float)(1.0 - (double)beta2);
-  o->eps = eps;
-  o->step_size = (float)((double)lr / bc1);
+  const double bc1 = 1.0 - std::pow(beta1, (double)t);
+  const double bc2 = 1.0 - std::pow(beta2, (double)t);
+  o->beta1 = (float)beta1;
+  o->beta2 = (float)beta2;
+  o->omb1 = (float)(1.0 - beta1);
+  o->omb2 = (float)(1.0 - beta2);
+  o->eps = (float)eps;
+  o->step_size = (float)(lr / bc1);
   o->sqrt_bc2 = (float)std::sqrt(bc2);
-  o->decay = (float)(1.0 - (double)lr * (double)weight_decay);
+  o->decay = (float)(1.0 - lr * weight_decay);
   return SH_OK;
 }
 
@@ -1182,7 +1182,7 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
   return SH_OK;
 }
 
-sh_status sh_set_lr(sh_ctx* c, float lr) {
+sh_status sh_set_lr(sh_ctx* c, double lr) {
   if (!c) return SH_ERR_INVALID;
   c->lr = lr;
   return SH_OK;
@@ -1502,6 +1502,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   o->s_avail = c->cfg.device_budget_bytes > 0 ? c->cfg.device_budget_bytes
                                               : held + (int64_t)fr - ((int64_t)2 << 30);
   o->duplex = (c->cfg.flags & SH_FLAG_DUPLEX) ? 1 : 0;
+  o->cpu_hard = (c->cfg.flags & SH_FLAG_CPU_HARD) ? 1 : 0;
   return SH_OK;
 }
 

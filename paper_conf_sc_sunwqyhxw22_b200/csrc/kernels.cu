@@ -164,7 +164,7 @@ __global__ void __launch_bounds__(256) k3_final_kernel(const double* __restrict_
   if (threadIdx.x == 0) *out = s;
 }
 
-__global__ void norm_finalize_kernel(const double* __restrict__ partials, int n, float max_norm,
+__global__ void norm_finalize_kernel(const double* __restrict__ partials, int n, double max_norm,
                                      double* norm_out, float* coef_out) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
   double s = 0.0;
@@ -172,8 +172,8 @@ __global__ void norm_finalize_kernel(const double* __restrict__ partials, int n,
   const double norm = sqrt(s);
   *norm_out = norm;
   double c = 1.0;
-  if (max_norm > 0.0f) {
-    c = (double)max_norm / (norm + 1e-6);
+  if (max_norm > 0.0) {
+    c = max_norm / (norm + 1e-6);
     if (c > 1.0) c = 1.0;
   }
   *coef_out = (float)c;
@@ -239,7 +239,7 @@ cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaS
   return cudaGetLastError();
 }
 
-cudaError_t norm_finalize(const double* partials, int n, float max_norm, double* norm_out,
+cudaError_t norm_finalize(const double* partials, int n, double max_norm, double* norm_out,
                           float* coef_out, cudaStream_t st) {
   launch_counter()++;
   norm_finalize_kernel<<<1, 32, 0, st>>>(partials, n, max_norm, norm_out, coef_out);

@@ -65,7 +65,7 @@ constexpr int kSumsqMaxBlocks = 1184;  // 148 SMs x 8
 // Deterministic Σ g^2 in fp64 -> *out (device).  scratch: kSumsqMaxBlocks doubles.
 cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaStream_t st);
 // norm = sqrt(Σ partials[0..n)) in index order; coef = min(1, max_norm/(norm+1e-6)) (fp32)
-cudaError_t norm_finalize(const double* partials, int n, float max_norm, double* norm_out,
+cudaError_t norm_finalize(const double* partials, int n, double max_norm, double* norm_out,
                           float* coef_out, cudaStream_t st);
 int sm_count();
 int64_t launches();

@@ -20,7 +20,7 @@ SH_OK, SH_ERR_INVALID, SH_ERR_CUDA, SH_ERR_OOM_DEVICE, SH_ERR_OOM_HOST, SH_ERR_N
 SH_FP32, SH_BF16_MIXED = 0, 1
 SH_PRE, SH_POST = 0, 1
 SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE = 0, 1, 2, 3
-SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU = 1, 2, 4, 8
+SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD = 1, 2, 4, 8, 16
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
@@ -43,9 +43,9 @@ class LayerShape(C.Structure):
 
 class Config(C.Structure):
     _fields_ = [("n_layers", C.c_int32), ("layers", C.POINTER(LayerShape)), ("resident", LayerShape),
-                ("window", C.c_int32), ("precision", C.c_int32), ("lr", C.c_float), ("beta1", C.c_float),
-                ("beta2", C.c_float), ("eps", C.c_float), ("weight_decay", C.c_float),
-                ("max_grad_norm", C.c_float), ("device", C.c_int32), ("compute_stream", C.c_void_p),
+                ("window", C.c_int32), ("precision", C.c_int32), ("lr", C.c_double), ("beta1", C.c_double),
+                ("beta2", C.c_double), ("eps", C.c_double), ("weight_decay", C.c_double),
+                ("max_grad_norm", C.c_double), ("device", C.c_int32), ("compute_stream", C.c_void_p),
                 ("cpu_threads", C.c_int32), ("grad_ring_depth", C.c_int32), ("warmup_steps", C.c_int32),
                 ("device_budget_bytes", C.c_int64), ("world_size", C.c_int32), ("rank", C.c_int32),
                 ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64)]
@@ -59,14 +59,14 @@ class Profile(C.Structure):
     _fields_ = [("n_layers", C.c_int32), ("t_fp", _PD), ("t_bp", _PD), ("t_c2g", _PD), ("t_g2c", _PD),
                 ("t_stage", _PD), ("t_opt_gpu", _PD), ("t_opt_cpu", _PD), ("t_async", C.c_double),
                 ("slot_bytes", _PI64), ("gstate_bytes", _PI64), ("fixed_bytes", C.c_int64),
-                ("s_avail", C.c_int64), ("duplex", C.c_int32)]
+                ("s_avail", C.c_int64), ("duplex", C.c_int32), ("cpu_hard", C.c_int32)]
 
 
 class SolveReport(C.Structure):
     _fields_ = [("window", C.c_int32), ("w_max_memory", C.c_int32), ("reason", C.c_int32),
                 ("fp_hard_ok", C.c_int32), ("bp_hard_ok", C.c_int32), ("soft_ok", C.c_int32),
                 ("eq3_min_slack_ms", C.c_double), ("eq3_ok", C.c_int32), ("eq4_lhs_ms", C.c_double),
-                ("eq4_rhs_ms", C.c_double)]
+                ("eq4_rhs_ms", C.c_double), ("cpu_total_ms", C.c_double), ("gpu_step_ms", C.c_double)]
 
 
 class Stats(C.Structure):
@@ -103,14 +103,14 @@ def lib() -> C.CDLL:
             "sh_synchronize": [vp], "sh_destroy": [vp],
             "sh_forward_layer": [vp, i32, i32, vp],
             "sh_backward_layer": [vp, i32, i32, vp, vp],
-            "sh_resident": [vp, vp, vp], "sh_set_lr": [vp, f32],
+            "sh_resident": [vp, vp, vp], "sh_set_lr": [vp, C.c_double],
             "sh_step": [vp, C.POINTER(C.c_double)],
             "sh_solve_window": [C.POINTER(Profile), C.POINTER(SolveReport)],
             "sh_autotune_window": [vp, C.POINTER(Profile), C.POINTER(i32)],
             "sh_set_window": [vp, i32], "sh_get_profile": [vp, C.POINTER(Profile)],
             "sh_read_layer": [vp, i32, i32, vp], "sh_stats": [vp, C.POINTER(Stats)],
             "sh_nccl_get_unique_id": [vp],
-            "sh_adam_scalars_for": [f32, f32, f32, f32, f32, i64, C.POINTER(AdamScalars)],
+            "sh_adam_scalars_for": [C.c_double] * 5 + [i64, C.POINTER(AdamScalars)],
             "sh_op_adamw_gpu": [vp, vp, vp, vp, vp, vp, i64, i64, C.POINTER(AdamScalars), vp, vp],
             "sh_op_adamw_cpu": [vp, vp, vp, vp, vp, i64, i64, C.POINTER(AdamScalars), i32, f32, i32],
             "sh_op_cast_bf16_gpu": [vp, vp, i64, vp], "sh_op_cast_bf16_cpu": [vp, vp, i64],
@@ -204,7 +204,8 @@ def _dbl(a, n):
 
 
 def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
-                 slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False) -> dict:
+                 slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False,
+                 cpu_hard=False) -> dict:
     """Pure call of sh_solve_window (no GPU)."""
     n = len(t_fp)
     keep = {}
@@ -223,6 +224,7 @@ def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_c
     prof.fixed_bytes = int(fixed_bytes)
     prof.s_avail = int(s_avail)
     prof.duplex = 1 if duplex else 0
+    prof.cpu_hard = 1 if cpu_hard else 0
     rep = SolveReport()
     check(lib().sh_solve_window(C.byref(prof), C.byref(rep)))
     return {f: getattr(rep, f) for f, _ in SolveReport._fields_}
@@ -359,7 +361,7 @@ class Engine:
         check(self._L.sh_get_profile(self.h, C.byref(p)))
         n = p.n_layers
         out = {"n_layers": n, "t_async": p.t_async, "s_avail": p.s_avail, "fixed_bytes": p.fixed_bytes,
-               "duplex": p.duplex}
+               "duplex": p.duplex, "cpu_hard": p.cpu_hard}
         for f in ("t_fp", "t_bp", "t_c2g", "t_g2c", "t_stage", "t_opt_gpu", "t_opt_cpu"):
             out[f] = [getattr(p, f)[i] for i in range(n)]
         for f in ("slot_bytes", "gstate_bytes"):

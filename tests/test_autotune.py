@@ -1,0 +1,107 @@
+"""Window solver (sh_solve_window, C-ABI, no GPU) vs the paper's model.
+
+Pins: homogeneous closed forms derived by hand from eq. 1b / 2b / 1d / 2d, the memory
+fallback of PAPER.md:195, and agreement with the brute-force transcription in
+oracle/autotune_oracle.py on random heterogeneous profiles.
+"""
+import math
+
+import numpy as np
+import pytest
+
+from oracle import autotune_oracle as AO
+
+sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
+
+
+def homog(L, a, c, d, **kw):
+    """t_fp = a, t_bp = 3a (recompute + 2x backward, PAPER.md:153 fn. 2), t_c2g = c, t_g2c = d."""
+    return dict(t_fp=[a] * L, t_bp=[3 * a] * L, t_c2g=[c] * L, t_g2c=[d] * L, **kw)
+
+
+def test_homogeneous_fp_bound_closed_form():
+    # soft fails (a < c + d) => w* = smallest w with w a >= c and 3 w a >= max(c, d)
+    for a, c, d in [(1.0, 2.5, 1.0), (2.0, 9.0, 3.0), (1.0, 0.9, 0.2), (0.5, 3.2, 7.0)]:
+        L = 40
+        r = sh.solve_window(**homog(L, a, c, d))
+        expect = max(math.ceil(c / a), math.ceil(max(c, d) / (3 * a)))
+        if a >= c + d:  # soft holds at the hard minimum too
+            assert r["reason"] == 0
+        else:
+            assert r["reason"] == 1
+        assert r["window"] == expect, (a, c, d, r)
+
+
+def test_soft_constraint_met_gives_reason0_and_no_jump_to_resident():
+    # a >= c + d: every w meeting hard meets soft; the solver must not pick w = L
+    r = sh.solve_window(**homog(24, 4.0, 3.0, 0.5))
+    assert r == {**r, "window": 1, "reason": 0}
+    # soft unsatisfiable: still the hard minimum, not the vacuous w = L
+    r = sh.solve_window(**homog(24, 1.0, 1.5, 2.0))
+    assert r["window"] == 2 and r["reason"] == 1
+
+
+def test_memory_fallback_largest_window():
+    # hard needs w >= 5 but memory allows only w <= 3 -> w* = 3
+    L = 20
+    prof = homog(L, 1.0, 5.0, 1.0, slot_bytes=[100] * L, gstate_bytes=[50] * L, fixed_bytes=0,
+                 s_avail=4 * 100 + 3 * 50)
+    r = sh.solve_window(**prof)
+    assert r["window"] == 3 and r["reason"] == 2 and r["w_max_memory"] == 3
+
+
+def test_oom_even_at_w0():
+    with pytest.raises(sh.ShError) as e:
+        sh.solve_window(**homog(4, 1, 1, 1, slot_bytes=[10] * 4, s_avail=5))
+    assert e.value.status == sh.SH_ERR_OOM_DEVICE
+
+
+def test_resident_when_transfers_cannot_hide_and_memory_allows():
+    # no w < L meets the FP hard constraint (c2g exceeds the whole model's FP time), memory allows L
+    L = 6
+    r = sh.solve_window(**homog(L, 1.0, 100.0, 1.0))
+    assert r["window"] == L and r["reason"] == 1
+
+
+def test_cpu_hard_pushes_window_up():
+    L = 10
+    prof = homog(L, 1.0, 0.5, 0.5, t_opt_cpu=[10.0] * L, t_opt_gpu=[0.1] * L)
+    r0 = sh.solve_window(**prof)
+    assert r0["window"] == 1
+    r1 = sh.solve_window(**prof, cpu_hard=True)
+    # (L - w) * 10 <= 4 L + 0.1 w  ->  w >= (10 L - 4 L) / 10.1
+    assert r1["window"] == math.ceil((10 * L - 4 * L) / 10.1)
+    assert r1["cpu_total_ms"] <= r1["gpu_step_ms"]
+
+
+def test_eq3_and_eq4_reports():
+    L = 8
+    prof = homog(L, 1.0, 0.5, 0.2, t_opt_cpu=[3.0] * L, t_opt_gpu=[0.25] * L, t_async=0.01)
+    r = sh.solve_window(**prof)
+    w = r["window"]
+    # slack at k = w: (w+1)*4 + 0.25 w - 3
+    assert abs(r["eq3_min_slack_ms"] - ((w + 1) * 4.0 + 0.25 * w - 3.0)) < 1e-12
+    assert abs(r["eq4_lhs_ms"] - 5 * L * 0.01) < 1e-12
+    assert abs(r["eq4_rhs_ms"] - 0.25 * (L - w)) < 1e-12
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_random_heterogeneous_matches_bruteforce(seed):
+    rng = np.random.default_rng(seed)
+    L = int(rng.integers(1, 30))
+    prof = dict(t_fp=rng.uniform(0.1, 3, L), t_bp=rng.uniform(0.3, 9, L), t_c2g=rng.uniform(0, 6, L),
+                t_g2c=rng.uniform(0, 8, L), t_stage=rng.uniform(0, 0.5, L), t_opt_gpu=rng.uniform(0, 1, L),
+                t_opt_cpu=rng.uniform(0, 20, L), t_async=float(rng.uniform(0, 0.1)),
+                slot_bytes=rng.integers(1, 100, L), gstate_bytes=rng.integers(1, 60, L),
+                fixed_bytes=int(rng.integers(0, 50)), s_avail=int(rng.integers(100, 3000)),
+                duplex=bool(rng.integers(0, 2)), cpu_hard=bool(rng.integers(0, 2)))
+    want = AO.solve(**{k: (list(v) if isinstance(v, np.ndarray) else v) for k, v in prof.items()})
+    if want is None:
+        with pytest.raises(sh.ShError):
+            sh.solve_window(**prof)
+        return
+    got = sh.solve_window(**prof)
+    for k in ("window", "reason", "w_max_memory"):
+        assert got[k] == want[k], (k, got, want)
+    for k in ("eq3_min_slack_ms", "eq4_lhs_ms", "eq4_rhs_ms"):
+        assert abs(got[k] - want[k]) <= 1e-9 * max(1.0, abs(want[k])), (k, got, want)
