@@ -58,7 +58,7 @@ __attribute__((target("avx512f"))) static inline __m256i rne_bf16_16(__m512 x) {
   return _mm512_cvtepi32_epi16(r);
 }
 
-template <bool kWd, bool kCoef, bool kOut>
+template <bool kWd, bool kCoef, bool kOut, bool kNT>
 __attribute__((target("avx512f"))) static void adam_avx512_block(
     float* __restrict p, float* __restrict m, float* __restrict v, const float* __restrict g,
     uint16_t* __restrict out16, int64_t b, int64_t e, const sh_adam_scalars& s, float coef) {
@@ -81,7 +81,11 @@ __attribute__((target("avx512f"))) static void adam_avx512_block(
     _mm512_storeu_ps(m + i, mm);
     _mm512_storeu_ps(v + i, vv);
     _mm512_storeu_ps(p + i, pp);
-    if (kOut) _mm256_storeu_si256(reinterpret_cast<__m256i*>(out16 + i), rne_bf16_16(pp));
+    if (kOut) {
+      // the shadow is written once and next read by the H2D DMA: stream it (no read-for-ownership)
+      if (kNT) _mm256_stream_si256(reinterpret_cast<__m256i*>(out16 + i), rne_bf16_16(pp));
+      else _mm256_storeu_si256(reinterpret_cast<__m256i*>(out16 + i), rne_bf16_16(pp));
+    }
   }
 }
 
@@ -89,12 +93,15 @@ template <bool kWd>
 static void adam_vec_dispatch(float* p, float* m, float* v, const float* g, uint16_t* out16,
                               int64_t b, int64_t e, const sh_adam_scalars& s, bool use_coef,
                               float coef) {
+  const bool nt = out16 && ((reinterpret_cast<uintptr_t>(out16 + b) & 31) == 0);
   if (use_coef) {
-    if (out16) adam_avx512_block<kWd, true, true>(p, m, v, g, out16, b, e, s, coef);
-    else adam_avx512_block<kWd, true, false>(p, m, v, g, out16, b, e, s, coef);
+    if (!out16) adam_avx512_block<kWd, true, false, false>(p, m, v, g, out16, b, e, s, coef);
+    else if (nt) adam_avx512_block<kWd, true, true, true>(p, m, v, g, out16, b, e, s, coef);
+    else adam_avx512_block<kWd, true, true, false>(p, m, v, g, out16, b, e, s, coef);
   } else {
-    if (out16) adam_avx512_block<kWd, false, true>(p, m, v, g, out16, b, e, s, coef);
-    else adam_avx512_block<kWd, false, false>(p, m, v, g, out16, b, e, s, coef);
+    if (!out16) adam_avx512_block<kWd, false, false, false>(p, m, v, g, out16, b, e, s, coef);
+    else if (nt) adam_avx512_block<kWd, false, true, true>(p, m, v, g, out16, b, e, s, coef);
+    else adam_avx512_block<kWd, false, true, false>(p, m, v, g, out16, b, e, s, coef);
   }
 }
 
@@ -121,6 +128,7 @@ void adamw_range(float* p, float* m, float* v, const float* g, uint16_t* out16, 
     else adam_vec_dispatch<false>(p, m, v, g, out16, b, ev, sc, use_coef, coef);
     adam_scalar_range(p, m, v, g, out16, ev, e, n_decay, sc, use_coef, coef);
   }
+  if (out16) _mm_sfence();  // order the streamed shadow before the caller's release of ready[j]
 }
 
 __attribute__((target("avx512f"))) static void cast_avx512(const float* src, uint16_t* dst,

@@ -1059,7 +1059,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->device_bytes += 16 * n + (int64_t)c->cb * n;
     CKC(c.get(), cudaMemset(p, 0, 16 * n + (int64_t)c->cb * n));
     double* d = nullptr;
-    const int64_t nd = (c->L + 1) + 2 * kern::kSumsqMaxBlocks + 1;
+    const int64_t nd = (c->L + 1) + 2 * (kern::kSumsqMaxBlocks + 1) + 1;
     if (cudaMalloc(&d, nd * 8 + 64) != cudaSuccess) {
       cudaGetLastError();
       set_error("sh_init: cudaMalloc of scratch failed");
@@ -1068,8 +1068,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     CKC(c.get(), cudaMemset(d, 0, nd * 8 + 64));
     c->partials = d;
     c->scratch_cs = d + (c->L + 1);
-    c->scratch_comm = c->scratch_cs + kern::kSumsqMaxBlocks;
-    c->norm_dev = c->scratch_comm + kern::kSumsqMaxBlocks;
+    c->scratch_comm = c->scratch_cs + kern::kSumsqMaxBlocks + 1;
+    c->norm_dev = c->scratch_comm + kern::kSumsqMaxBlocks + 1;
     c->coef_dev = reinterpret_cast<float*>(c->norm_dev + 1);
   }
   c->g.assign(c->L, GState{});
@@ -1749,9 +1749,12 @@ sh_status sh_op_sumsq_gpu(const float* g, int64_t n, double* out_dev, void* stre
   const void* ptrs[] = {g};
   if (!g || !out_dev || !ops_args_ok(n, 0, ptrs, 1)) return SH_ERR_INVALID;
   static double* scratch = nullptr;
-  if (!scratch && cudaMalloc(&scratch, 8 * kern::kSumsqMaxBlocks) != cudaSuccess) {
-    set_error("K3 scratch allocation failed");
-    return SH_ERR_OOM_DEVICE;
+  if (!scratch) {
+    if (cudaMalloc(&scratch, 8 * (kern::kSumsqMaxBlocks + 1)) != cudaSuccess ||
+        cudaMemset(scratch, 0, 8 * (kern::kSumsqMaxBlocks + 1)) != cudaSuccess) {
+      set_error("K3 scratch allocation failed");
+      return SH_ERR_OOM_DEVICE;
+    }
   }
   const cudaError_t e = kern::sumsq(g, n, scratch, out_dev, static_cast<cudaStream_t>(stream));
   if (e != cudaSuccess) {

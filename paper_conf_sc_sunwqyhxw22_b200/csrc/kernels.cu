@@ -140,28 +140,53 @@ __device__ __forceinline__ double block_sum256(double x) {
   return r;  // valid in thread 0
 }
 
-// K3 pass 1: block b sums elements of float4 groups b*256+t, stepping by grid*256.
-// The grid depends only on n (never on the device), so the tree is fixed.
-__global__ void __launch_bounds__(256) k3_partial_kernel(const float* __restrict__ g, int64_t n4,
-                                                        double* __restrict__ partial) {
-  double acc = 0.0;
-  for (int64_t j = blockIdx.x * 256ll + threadIdx.x; j < n4; j += (int64_t)gridDim.x * 256) {
-    const float4 a = ld_stream(g + 4 * j);
-    acc = fma((double)a.x, (double)a.x, acc);
-    acc = fma((double)a.y, (double)a.y, acc);
-    acc = fma((double)a.z, (double)a.z, acc);
-    acc = fma((double)a.w, (double)a.w, acc);
-  }
-  const double s = block_sum256(acc);
-  if (threadIdx.x == 0) partial[blockIdx.x] = s;
-}
-
-__global__ void __launch_bounds__(256) k3_final_kernel(const double* __restrict__ partial, int nb,
+// K3: one launch.  Block b sums float4 groups b*256+t, b*256+t+stride, ... (4 independent loads
+// in flight per thread), reduces with a fixed warp-shuffle tree, writes partial[b]; the last block
+// to finish (atomic ticket) sums partial[0..grid) in index order and resets the ticket.  The grid
+// depends only on n, so the reduction tree -- and the result bits -- are fixed.
+__global__ void __launch_bounds__(256) k3_sumsq_kernel(const float* __restrict__ g, int64_t n4,
+                                                      double* __restrict__ partial,
+                                                      unsigned int* __restrict__ ticket,
                                                       double* __restrict__ out) {
-  double acc = 0.0;
-  for (int i = threadIdx.x; i < nb; i += 256) acc += partial[i];
-  const double s = block_sum256(acc);
-  if (threadIdx.x == 0) *out = s;
+  const int64_t stride = (int64_t)gridDim.x * 256;
+  int64_t j = blockIdx.x * 256ll + threadIdx.x;
+  double acc0 = 0.0, acc1 = 0.0;
+  for (; j + 3 * stride < n4; j += 4 * stride) {
+    const float4 a = ld_stream(g + 4 * j);
+    const float4 b = ld_stream(g + 4 * (j + stride));
+    const float4 c = ld_stream(g + 4 * (j + 2 * stride));
+    const float4 d = ld_stream(g + 4 * (j + 3 * stride));
+    acc0 = fma((double)a.x, (double)a.x, acc0); acc1 = fma((double)a.y, (double)a.y, acc1);
+    acc0 = fma((double)a.z, (double)a.z, acc0); acc1 = fma((double)a.w, (double)a.w, acc1);
+    acc0 = fma((double)b.x, (double)b.x, acc0); acc1 = fma((double)b.y, (double)b.y, acc1);
+    acc0 = fma((double)b.z, (double)b.z, acc0); acc1 = fma((double)b.w, (double)b.w, acc1);
+    acc0 = fma((double)c.x, (double)c.x, acc0); acc1 = fma((double)c.y, (double)c.y, acc1);
+    acc0 = fma((double)c.z, (double)c.z, acc0); acc1 = fma((double)c.w, (double)c.w, acc1);
+    acc0 = fma((double)d.x, (double)d.x, acc0); acc1 = fma((double)d.y, (double)d.y, acc1);
+    acc0 = fma((double)d.z, (double)d.z, acc0); acc1 = fma((double)d.w, (double)d.w, acc1);
+  }
+  for (; j < n4; j += stride) {
+    const float4 a = ld_stream(g + 4 * j);
+    acc0 = fma((double)a.x, (double)a.x, acc0); acc1 = fma((double)a.y, (double)a.y, acc1);
+    acc0 = fma((double)a.z, (double)a.z, acc0); acc1 = fma((double)a.w, (double)a.w, acc1);
+  }
+  const double s = block_sum256(acc0 + acc1);
+  __shared__ bool last;
+  if (threadIdx.x == 0) {
+    partial[blockIdx.x] = s;
+    __threadfence();
+    last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  double t = 0.0;
+  for (int i = threadIdx.x; i < (int)gridDim.x; i += 256) t += __ldcg(partial + i);
+  const double tot = block_sum256(t);
+  if (threadIdx.x == 0) {
+    *out = tot;
+    *ticket = 0u;  // ready for the next launch on this scratch
+  }
 }
 
 __global__ void norm_finalize_kernel(const double* __restrict__ partials, int n, double max_norm,
@@ -231,11 +256,11 @@ cudaError_t cast_bf16(const float* src, uint16_t* dst, int64_t n, cudaStream_t s
 cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaStream_t st) {
   const int64_t n4 = n / 4;
   if (n4 == 0) return cudaMemsetAsync(out, 0, sizeof(double), st);
-  int64_t nb = (n4 + 2047) / 2048;  // >= 8 float4 per thread before striding
+  int64_t nb = (n4 + 4095) / 4096;  // >= 16 float4 per thread before the tail
   if (nb > kSumsqMaxBlocks) nb = kSumsqMaxBlocks;
-  launch_counter() += 2;
-  k3_partial_kernel<<<(int)nb, 256, 0, st>>>(g, n4, scratch);
-  k3_final_kernel<<<1, 256, 0, st>>>(scratch, (int)nb, out);
+  launch_counter()++;
+  unsigned int* ticket = reinterpret_cast<unsigned int*>(scratch + kSumsqMaxBlocks);
+  k3_sumsq_kernel<<<(int)nb, 256, 0, st>>>(g, n4, scratch, ticket, out);
   return cudaGetLastError();
 }
 

@@ -62,7 +62,8 @@ struct K2Args {
 cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out = nullptr);
 cudaError_t cast_bf16(const float* src, uint16_t* dst, int64_t n, cudaStream_t st);
 constexpr int kSumsqMaxBlocks = 1184;  // 148 SMs x 8
-// Deterministic Σ g^2 in fp64 -> *out (device).  scratch: kSumsqMaxBlocks doubles.
+// Deterministic Σ g^2 in fp64 -> *out (device).  scratch: kSumsqMaxBlocks + 1 doubles, zeroed
+// once (the last word is the block ticket, reset by the kernel); one scratch per stream.
 cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaStream_t st);
 // norm = sqrt(Σ partials[0..n)) in index order; coef = min(1, max_norm/(norm+1e-6)) (fp32)
 cudaError_t norm_finalize(const double* partials, int n, double max_norm, double* norm_out,

@@ -9,7 +9,6 @@ buffers -- plumbing, as the task's north star states.
 from __future__ import annotations
 
 import math
-from concurrent.futures import ThreadPoolExecutor
 from dataclasses import dataclass
 
 import numpy as np
@@ -75,16 +74,16 @@ class StrongholdTrainer:
             self.init_params(seed, init_threads)
 
     def init_params(self, seed: int, threads: int = 8):
+        """Seeded init (synth/, bit-identical to synth.init_layer) streamed layer by layer through
+        one reusable buffer: O(one layer) of transient host memory at any model size."""
         mc = self.mc
-
-        def one(i):
-            return i, np.concatenate([a.reshape(-1) for a in synth.init_layer(seed, i, mc.n_layers, mc.hidden)])
-
-        with ThreadPoolExecutor(max(1, threads)) as ex:
-            for i, flat in ex.map(one, range(mc.n_layers)):
-                self.engine.register(i, flat)
-        res = synth.init_resident(seed, mc.vocab, mc.seq, mc.hidden)
-        self.engine.register(-1, np.concatenate([a.reshape(-1) for a in res]))
+        flat = np.empty(mc.params_per_layer(), np.float32)
+        for i in range(mc.n_layers):
+            synth.init_layer_into(flat, seed, i, mc.n_layers, mc.hidden, threads)
+            self.engine.register(i, flat)
+        res = np.empty(sum(mc.res_numels()), np.float32)
+        synth.init_resident_into(res, seed, mc.vocab, mc.seq, mc.hidden, threads)
+        self.engine.register(-1, res)
 
     def register_state(self, layers, resident, m_layers=None, v_layers=None, m_res=None, v_res=None, step=0):
         flat = lambda ts: np.concatenate([np.asarray(a, np.float32).reshape(-1) for a in ts])

@@ -63,6 +63,30 @@ def normal(key: np.uint64, n: int, std: float) -> np.ndarray:
     return (z[:n] * std).astype(np.float32)
 
 
+def fill_normal(out: np.ndarray, key: np.uint64, std: float, threads: int = 8, chunk_pairs: int = 1 << 20):
+    """Write normal(key, out.size, std) into the float32 array `out` (bit-identical to normal()),
+    in chunks of Box-Muller pairs on `threads` threads, with O(chunk) temporary memory."""
+    from concurrent.futures import ThreadPoolExecutor
+    n = out.size
+    m = (n + 1) // 2
+    flat = out.reshape(-1)
+
+    def work(k0):
+        k1 = min(m, k0 + chunk_pairs)
+        u1 = uniform01(key, k1 - k0, k0)
+        u2 = uniform01(key, k1 - k0, m + k0)
+        r = np.sqrt(-2.0 * np.log(u1))
+        z0 = ((r * np.cos(2.0 * np.pi * u2)) * std).astype(np.float32)
+        z1 = ((r * np.sin(2.0 * np.pi * u2)) * std).astype(np.float32)
+        e0 = 2 * k1 if 2 * k1 <= n else n
+        flat[2 * k0:e0:2] = z0[: (e0 - 2 * k0 + 1) // 2]
+        flat[2 * k0 + 1:min(2 * k1, n):2] = z1[: (min(2 * k1, n) - 2 * k0) // 2]
+
+    with ThreadPoolExecutor(max(1, threads)) as ex:
+        list(ex.map(work, range(0, m, chunk_pairs)))
+    return out
+
+
 # --- GPT-2 shaped parameter sets -------------------------------------------------
 
 LAYER_TENSORS = ("ln1_g", "ln1_b", "w_qkv", "b_qkv", "w_o", "b_o",
@@ -103,6 +127,33 @@ def init_layer(seed: int, layer: int, L: int, h: int) -> list[np.ndarray]:
         else:
             out.append(np.zeros(shp, dtype=np.float32))
     return out
+
+
+def init_layer_into(flat: np.ndarray, seed: int, layer: int, L: int, h: int, threads: int = 8) -> np.ndarray:
+    """init_layer(...) concatenated in LAYER_TENSORS order, written into the float32 vector
+    `flat` (bit-identical, bounded temporaries; used for multi-billion-parameter configs)."""
+    resid_std = 0.02 / np.sqrt(2.0 * L)
+    o = 0
+    for ti, (name, shp) in enumerate(zip(LAYER_TENSORS, layer_shapes(h))):
+        n = int(np.prod(shp))
+        seg = flat[o:o + n]
+        if name.startswith("w_"):
+            std = resid_std if name in ("w_o", "w_proj") else 0.02
+            fill_normal(seg, stream_key(seed, 1, layer, ti), std, threads)
+        elif name.endswith("_g"):
+            seg[:] = 1.0
+        else:
+            seg[:] = 0.0
+        o += n
+    return flat
+
+
+def init_resident_into(flat: np.ndarray, seed: int, V: int, s: int, h: int, threads: int = 8) -> np.ndarray:
+    fill_normal(flat[:V * h], stream_key(seed, 2, 0), 0.02, threads)
+    fill_normal(flat[V * h:V * h + s * h], stream_key(seed, 2, 1), 0.02, threads)
+    flat[V * h + s * h:V * h + s * h + h] = 1.0
+    flat[V * h + s * h + h:] = 0.0
+    return flat
 
 
 def init_resident(seed: int, V: int, s: int, h: int) -> list[np.ndarray]:
