@@ -35,7 +35,12 @@ CONFIGS = {
     "tiny": (4, 256, 4, 128, 512, 2, 2, "BASELINE configs[0]: tiny GPT 4x256, seq 128"),
     "c2": (48, 1600, 25, 1024, 50304, 16, 4, "BASELINE configs[1]: GPT-2 XL-shaped 1.5B (48 x 1600, seq 1024)"),
     "c3": (48, 4096, 32, 1024, 50304, 16, 4, "BASELINE configs[2]: GPT-style ~10B (48 x 4096, seq 1024)"),
+    # 75 x 4096: 15.3 B params, fp32 params + Adam states = 184 GB > 180 GB of HBM; host store
+    # 12 B/param (fp32-fetch mode, no bf16 shadow) = 175 GB of the box's 196 GB
+    "c4": (75, 4096, 32, 1024, 50304, 16, 4, "BASELINE configs[3]: depth-scaled GPT 75 x 4096 = 15.3B, "
+                                             "states 184 GB > 180 GB HBM (max trainable on this host)"),
 }
+FETCH_FP32_DEFAULT = {"c4"}
 PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
 PROBE_D2H_GBS = 57.01
 
@@ -178,6 +183,8 @@ def main():
     ap.add_argument("--no-resident", action="store_true", help="skip the all-resident comparison run")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--fetch-fp32", type=int, default=-1, help="1: no host bf16 shadow, fp32 over the link")
+    ap.add_argument("--init-threads", type=int, default=16)
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -211,12 +218,16 @@ def main():
     mc = ModelConfig(L, h, nh, s, V)
     K, W = args.steps, args.warmup
 
+    fetch32 = args.fetch_fp32 == 1 or (args.fetch_fp32 == -1 and args.config in FETCH_FP32_DEFAULT)
+    grad_ring = args.grad_ring or (4 if args.config in ("c3", "c4") else 0)
+
     def run(window, e2e: bool):
         t_init = time.perf_counter()
+        flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
-                               flags=sh.SH_FLAG_PROFILE, world_size=world, rank=rank, nccl_id=nccl_id,
-                               cpu_threads=args.cpu_threads, grad_ring_depth=args.grad_ring,
-                               warmup_steps=W if window == -1 else 5)
+                               flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
+                               cpu_threads=args.cpu_threads, grad_ring_depth=grad_ring,
+                               warmup_steps=W if window == -1 else 5, init_threads=args.init_threads)
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
         host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + K)])
@@ -265,7 +276,7 @@ def main():
 
     r = run(w, not args.no_e2e)
     res = None
-    if not args.no_resident and w != L and args.config != "c3":
+    if not args.no_resident and w != L and args.config not in ("c3", "c4"):
         res = run(L, False)
 
     def gmax(x):
@@ -304,7 +315,11 @@ def main():
         "config": {"workload": args.config, "description": desc, "layers": L, "hidden": h, "heads": nh, "seq": s,
                    "vocab": V, "params": mc.n_params(), "batch_per_gpu": b, "global_batch": b * world,
                    "window": w, "ring_slots": w + 1, "precision": "bf16_mixed" if prec else "fp32",
-                   "parallelism": f"dp{world}", "states": "fp32 master/m/v + bf16 shadow in pinned host RAM",
+                   "parallelism": f"dp{world}",
+                   "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),
+                   "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
+                   "grad_landing_buffers": grad_ring or L, "host_store_bytes": r["st1"]["host_bytes"],
+                   "states_bytes_fp32_p_m_v": 12 * mc.n_params(),
                    "l2": "no flush: per-step traffic (GBs) >> 126 MB L2"},
         "tokens_per_s": tokens_s,
         "model_tflops": tokens_s * flops_tok / 1e12,
@@ -314,6 +329,7 @@ def main():
             "h2d_gbs_per_transfer": h2d_gbs, "d2h_gbs_per_transfer": d2h_gbs,
             "h2d_peak_gbs": PROBE_H2D_GBS, "d2h_peak_gbs": PROBE_D2H_GBS,
             "h2d_frac": h2d_gbs / PROBE_H2D_GBS if h2d_gbs else None,
+            "h2d_step_gbs": d["h2d_bytes"] / (ms / 1e3) / 1e9, "d2h_step_gbs": d["d2h_bytes"] / (ms / 1e3) / 1e9,
             "d2h_frac": d2h_gbs / PROBE_D2H_GBS if d2h_gbs else None,
             "h2d_busy_frac_of_step": d["h2d_busy_ms"] / ms, "d2h_busy_frac_of_step": d["d2h_busy_ms"] / ms,
             "peak_source": "profiles/r01_probe_box.json (pinned 1 GiB copies)"},

@@ -96,6 +96,9 @@ typedef struct {
 #define SH_FLAG_PROFILE   (1ull << 0) /* record per-layer CUDA events every step (else warm-up only) */
 #define SH_FLAG_POISON    (1ull << 1) /* debug: fill a slot's param half with NaN before every refill */
 #define SH_FLAG_DUPLEX    (1ull << 2) /* autotuner: full-duplex link, max() instead of sum in (1d)/(2d) */
+#define SH_FLAG_FETCH_FP32 (1ull << 5) /* bf16 mode: no host bf16 shadow (12 instead of 14 B/param of host
+                                          RAM); prefetch the fp32 master (4 B/param over the link) into
+                                          the slot's idle grad half and K1-cast it on the GPU */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

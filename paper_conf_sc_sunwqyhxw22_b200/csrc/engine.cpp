@@ -226,9 +226,16 @@ struct sh_ctx {
   float* coef_dev = nullptr;
   int64_t device_bytes = 0;
 
-  // ---- host store
-  char* host_base = nullptr;
+  // ---- host store: one pinned block per host-optimised layer (allocated when the layer first
+  // becomes host-optimised) + one block for the landing ring and scalars
+  struct HostBlock {
+    char* p = nullptr;
+    size_t bytes = 0;
+  };
+  std::vector<HostBlock> hblocks;  // [L]
+  HostBlock hland;
   size_t host_bytes = 0;
+  bool shadow = true;  // bf16 shadow kept in host RAM (bf16 mode without SH_FLAG_FETCH_FP32)
   std::vector<float*> h_master, h_m, h_v;
   std::vector<uint16_t*> h_shadow;
   std::vector<float*> landing;
@@ -398,6 +405,56 @@ void parallel_touch(char* p, size_t bytes, int threads) {
   for (auto& t : ts) t.join();
 }
 
+int64_t mem_available_bytes() {
+  FILE* f = fopen("/proc/meminfo", "r");
+  if (!f) return INT64_MAX;
+  char key[64];
+  long long kb = 0;
+  char unit[16];
+  int64_t avail = INT64_MAX;
+  while (fscanf(f, "%63s %lld %15s", key, &kb, unit) == 3)
+    if (strcmp(key, "MemAvailable:") == 0) {
+      avail = (int64_t)kb * 1024;
+      break;
+    }
+  fclose(f);
+  return avail;
+}
+
+// mmap + THP advice + parallel first touch + cudaHostRegister.  Refuses (instead of letting the
+// kernel OOM-kill the process) when the block would leave less than SH_HOST_MARGIN_GB free.
+sh_status host_block_alloc(size_t bytes, int threads, char** out) {
+  *out = nullptr;
+  const char* mg = getenv("SH_HOST_MARGIN_GB");
+  const int64_t margin = (int64_t)((mg ? atof(mg) : 3.0) * (1ll << 30));
+  const int64_t avail = mem_available_bytes();
+  if ((int64_t)bytes + margin > avail) {
+    set_error("host store: %lld B requested, %lld B available (margin %lld B)", (long long)bytes,
+              (long long)avail, (long long)margin);
+    return SH_ERR_OOM_HOST;
+  }
+  char* p = static_cast<char*>(host_alloc(bytes));
+  if (!p) {
+    set_error("host store: mmap of %lld B failed", (long long)bytes);
+    return SH_ERR_OOM_HOST;
+  }
+  parallel_touch(p, bytes, threads);
+  if (cudaHostRegister(p, bytes, cudaHostRegisterPortable) != cudaSuccess) {
+    cudaGetLastError();
+    munmap(p, bytes);
+    set_error("host store: cudaHostRegister of %lld B failed (memlock?)", (long long)bytes);
+    return SH_ERR_OOM_HOST;
+  }
+  *out = p;
+  return SH_OK;
+}
+
+void host_block_free(char* p, size_t bytes) {
+  if (!p) return;
+  cudaHostUnregister(p);
+  munmap(p, bytes);
+}
+
 // ---------------------------------------------------------------------------- CPU Adam pool
 void finish_job(sh_ctx* c, Job* j) {
   c->ready[j->layer].store(j->step + 1, std::memory_order_release);
@@ -438,7 +495,7 @@ void worker_loop(sh_ctx* c, int tid) {
     const LayerLayout& Lx = c->lay[x];
     const int64_t b = chunk * kCpuChunk, e = std::min(Lx.n_pad, b + kCpuChunk);
     cpu::adamw_range(c->h_master[x], c->h_m[x], c->h_v[x], c->landing[job->landing],
-                     c->bf16 ? c->h_shadow[x] : nullptr, b, e, Lx.n_decay, job->sc, c->clip, coef);
+                     c->shadow ? c->h_shadow[x] : nullptr, b, e, Lx.n_decay, job->sc, c->clip, coef);
     const double dt = now_ms() - t0;
     double cur = c->cpu_ms.load();
     while (!c->cpu_ms.compare_exchange_weak(cur, cur + dt)) {
@@ -477,7 +534,7 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
     Job* jp = j.get();
     const float coef = 1.0f;
     cpu::adamw_range(c->h_master[jp->layer], c->h_m[jp->layer], c->h_v[jp->layer],
-                     c->landing[jp->landing], c->bf16 ? c->h_shadow[jp->layer] : nullptr, 0,
+                     c->landing[jp->landing], c->shadow ? c->h_shadow[jp->layer] : nullptr, 0,
                      c->lay[jp->layer].n_pad, c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
     finish_job(c, jp);
     return;
@@ -569,7 +626,7 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
         const double ms = ev_ms(P.c2g0[ph][i], P.c2g1[ph][i]);
         c->p_c2g[i] = ms;
         c->h2d_busy += ms;
-        c->h2d_prof_bytes += (int64_t)c->cb * c->lay[i].n_pad;
+        c->h2d_prof_bytes += (int64_t)((c->bf16 && !c->shadow) ? 4 : c->cb) * c->lay[i].n_pad;
       }
     if (P.rec_g2c[i]) {
       const double ms = ev_ms(P.g2c0[i], P.g2c1[i]);
@@ -650,10 +707,16 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   }
   c->arrive_by_issuer[y] = 1;
   const int64_t need = c->step;
-  const void* src = c->bf16 ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];
-  const int64_t bytes = (int64_t)c->cb * n;
+  // bf16 mode fetches the bf16 shadow; fp32 mode the master; SH_FLAG_FETCH_FP32 fetches the fp32
+  // master into the slot's (idle) grad half and K1 casts it into the param half on the H2D stream
+  const bool cast = c->bf16 && !c->shadow;
+  const void* src = c->shadow ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];
+  const int64_t bytes = (cast ? 4 : (int64_t)c->cb) * n;
   cudaEvent_t pf = c->ev_param_free[s];
-  c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph] {
+  cudaEvent_t gf = c->ev_grad_free[s];
+  float* stage_buf = c->slot_grad(s);
+  const int64_t gf_gen = c->gradfree_gen[s];
+  c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, gf, stage_buf, gf_gen, s, n] {
     double waited = 0;
     if (!state_wait(c, [&] { return c->ready[y].load(std::memory_order_acquire) >= need; },
                     "CPU Adam of a layer to prefetch", &waited)) {
@@ -667,13 +730,22 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       }
     }
     CKA(c, cudaStreamWaitEvent(c->h2d, pf, 0));
+    if (cast) {  // the staging area (grad half) must be free of the previous occupant's offload
+      if (!state_wait(c, [&] { return c->gradfree_pub[s].load() >= gf_gen; }, "grad half for fp32 staging")) {
+        c->arrive_pub[y].store(kInf);
+        notify_state(c);
+        return;
+      }
+      CKA(c, cudaStreamWaitEvent(c->h2d, gf, 0));
+    }
     if (poison) CKA(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->h2d));
     if (P) CKA(c, cudaEventRecord(P->c2g0[ph][y], c->h2d));
-    CKA(c, cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, c->h2d));
+    CKA(c, cudaMemcpyAsync(cast ? (void*)stage_buf : dst, src, bytes, cudaMemcpyHostToDevice, c->h2d));
     if (P) {
       CKA(c, cudaEventRecord(P->c2g1[ph][y], c->h2d));
       P->rec_c2g[ph][y] = 1;
     }
+    if (cast) CKA(c, kern::cast_bf16(stage_buf, reinterpret_cast<uint16_t*>(dst), n, c->h2d));
     CKA(c, cudaEventRecord(c->ev_arrive[y], c->h2d));
     c->h2d_bytes += bytes;
     c->h2d_copies++;
@@ -772,6 +844,24 @@ void free_g(sh_ctx* c, int x) {
   c->g[x] = GState{};
 }
 
+// Host block of layer x: [master | m | v | shadow?], 2 MiB aligned.
+sh_status ensure_host_layer(sh_ctx* c, int x) {
+  if (c->h_master[x]) return SH_OK;
+  const int64_t n = c->lay[x].n_pad;
+  const size_t bytes = align_up(12 * n + (c->shadow ? 2 * n : 0), 1 << 21);
+  char* p = nullptr;
+  sh_status st = host_block_alloc(bytes, c->n_threads, &p);
+  if (st != SH_OK) return st;
+  c->hblocks[x] = {p, bytes};
+  c->host_bytes += bytes;
+  float* b = reinterpret_cast<float*>(p);
+  c->h_master[x] = b;
+  c->h_m[x] = b + n;
+  c->h_v[x] = b + 2 * n;
+  if (c->shadow) c->h_shadow[x] = reinterpret_cast<uint16_t*>(b + 3 * n);
+  return SH_OK;
+}
+
 sh_status alloc_ring(sh_ctx* c, int n_slots) {
   if (n_slots <= c->n_slots) return SH_OK;
   char* r = nullptr;
@@ -836,10 +926,12 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   // leaving G: HBM -> host store (bitwise), shadow recomputed with the same RNE
   for (int x = w_new; x < w_old; ++x) {
     const int64_t n = c->lay[x].n_pad;
+    st = ensure_host_layer(c, x);
+    if (st != SH_OK) return st;
     CKC(c, cudaMemcpy(c->h_master[x], c->g[x].master, 4 * n, cudaMemcpyDeviceToHost));
     CKC(c, cudaMemcpy(c->h_m[x], c->g[x].m, 4 * n, cudaMemcpyDeviceToHost));
     CKC(c, cudaMemcpy(c->h_v[x], c->g[x].v, 4 * n, cudaMemcpyDeviceToHost));
-    if (c->bf16) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], 0, n);
+    if (c->shadow) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], 0, n);
     c->ready[x].store(c->step);
     free_g(c, x);
   }
@@ -1000,47 +1092,28 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   // ---- host store: per layer master | m | v | shadow, plus landing buffers, 2 MiB aligned
   c->n_threads = cfg->cpu_threads > 0 ? cfg->cpu_threads : (int)std::thread::hardware_concurrency();
   if (c->n_threads < 1) c->n_threads = 1;
-  std::vector<int64_t> off(c->L);
-  int64_t hb = 0;
-  for (int x = 0; x < c->L; ++x) {
-    off[x] = hb;
-    const int64_t n = c->lay[x].n_pad;
-    hb += align_up(12 * n + (c->bf16 ? 2 * n : 0), 4096);
-  }
-  const int64_t land_off = align_up(hb, 1 << 21);
-  hb = land_off + (int64_t)c->D * align_up(4 * c->max_pad, 4096);
-  const int64_t coef_off = hb;
-  hb = align_up(hb + 4096, 1 << 21);
-  c->host_bytes = hb;
-  c->host_base = static_cast<char*>(host_alloc(hb));
-  if (!c->host_base) {
-    set_error("sh_init: mmap of %lld B host store failed", (long long)hb);
-    return SH_ERR_OOM_HOST;
-  }
-  parallel_touch(c->host_base, hb, c->n_threads);
-  if (cudaHostRegister(c->host_base, hb, cudaHostRegisterPortable) != cudaSuccess) {
-    cudaGetLastError();
-    munmap(c->host_base, hb);
-    c->host_base = nullptr;
-    set_error("sh_init: cudaHostRegister of %lld B failed (memlock?)", (long long)hb);
-    return SH_ERR_OOM_HOST;
-  }
-  c->h_master.resize(c->L);
-  c->h_m.resize(c->L);
-  c->h_v.resize(c->L);
+  c->shadow = c->bf16 && !(cfg->flags & SH_FLAG_FETCH_FP32);
+  c->hblocks.assign(c->L, {});
+  c->h_master.assign(c->L, nullptr);
+  c->h_m.assign(c->L, nullptr);
+  c->h_v.assign(c->L, nullptr);
   c->h_shadow.assign(c->L, nullptr);
-  for (int x = 0; x < c->L; ++x) {
-    const int64_t n = c->lay[x].n_pad;
-    float* b = reinterpret_cast<float*>(c->host_base + off[x]);
-    c->h_master[x] = b;
-    c->h_m[x] = b + n;
-    c->h_v[x] = b + 2 * n;
-    if (c->bf16) c->h_shadow[x] = reinterpret_cast<uint16_t*>(b + 3 * n);
+  {
+    const int64_t lb = align_up(4 * c->max_pad, 4096);
+    const size_t bytes = align_up((int64_t)c->D * lb + 4096, 1 << 21);
+    char* p = nullptr;
+    sh_status st = host_block_alloc(bytes, c->n_threads, &p);
+    if (st != SH_OK) return st;
+    c->hland = {p, bytes};
+    c->host_bytes += bytes;
+    c->landing.resize(c->D);
+    for (int k = 0; k < c->D; ++k) c->landing[k] = reinterpret_cast<float*>(p + (int64_t)k * lb);
+    c->h_coef = reinterpret_cast<float*>(p + (int64_t)c->D * lb);
   }
-  c->landing.resize(c->D);
-  for (int k = 0; k < c->D; ++k)
-    c->landing[k] = reinterpret_cast<float*>(c->host_base + land_off + (int64_t)k * align_up(4 * c->max_pad, 4096));
-  c->h_coef = reinterpret_cast<float*>(c->host_base + coef_off);
+  for (int x = w0; x < c->L; ++x) {  // host-optimised layers of the initial window
+    sh_status st = ensure_host_layer(c.get(), x);
+    if (st != SH_OK) return st;
+  }
 
   // ---- device: resident set, partials, ring, G states
   {
@@ -1158,15 +1231,23 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
   } else {
     const int x = layer;
     const int64_t n = c->lay[x].n_pad;
-    pack_layer(c->lay[x], params, c->h_master[x]);
-    pack_layer(c->lay[x], m, c->h_m[x]);
-    pack_layer(c->lay[x], v, c->h_v[x]);
-    if (c->bf16) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], 0, n);
+    std::vector<float> tmp;
+    float *hp = c->h_master[x], *hm = c->h_m[x], *hv = c->h_v[x];
+    if (!hp) {  // GPU-optimised layer without a host block: stage through a temporary
+      tmp.resize(3 * n);
+      hp = tmp.data();
+      hm = hp + n;
+      hv = hp + 2 * n;
+    }
+    pack_layer(c->lay[x], params, hp);
+    pack_layer(c->lay[x], m, hm);
+    pack_layer(c->lay[x], v, hv);
+    if (c->shadow && c->h_shadow[x]) cpu::cast_bf16_range(hp, c->h_shadow[x], 0, n);
     c->ready[x].store(step);
     if (c->is_g(x)) {
-      CKC(c, cudaMemcpy(c->g[x].master, c->h_master[x], 4 * n, cudaMemcpyHostToDevice));
-      CKC(c, cudaMemcpy(c->g[x].m, c->h_m[x], 4 * n, cudaMemcpyHostToDevice));
-      CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
+      CKC(c, cudaMemcpy(c->g[x].master, hp, 4 * n, cudaMemcpyHostToDevice));
+      CKC(c, cudaMemcpy(c->g[x].m, hm, 4 * n, cudaMemcpyHostToDevice));
+      CKC(c, cudaMemcpy(c->g[x].v, hv, 4 * n, cudaMemcpyHostToDevice));
     }
     c->reg_done[x] = 1;
   }
@@ -1466,16 +1547,17 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   if (st != SH_OK) return st;
   // t_c2g of GPU-optimised layers is not observed (they are never fetched): use the bytes
   // rate of the measured host layers (same link, same size class)
+  const double fb = (c->bf16 && !c->shadow) ? 4.0 : (double)c->cb;  // fetched bytes per element
   double rate = 0;  // ms per byte
   int nr = 0;
   for (int x = 0; x < c->L; ++x)
-    if (c->p_c2g[x] > 0) rate += c->p_c2g[x] / ((double)c->cb * c->lay[x].n_pad), nr++;
+    if (c->p_c2g[x] > 0) rate += c->p_c2g[x] / (fb * c->lay[x].n_pad), nr++;
   double grate = 0;
   int ng = 0;
   for (int x = 0; x < c->L; ++x)
     if (c->p_g2c[x] > 0) grate += c->p_g2c[x] / (4.0 * c->lay[x].n_pad), ng++;
   for (int x = 0; x < c->L; ++x) {
-    if (c->p_c2g[x] <= 0 && nr) c->p_c2g[x] = rate / nr * c->cb * c->lay[x].n_pad;
+    if (c->p_c2g[x] <= 0 && nr) c->p_c2g[x] = rate / nr * fb * c->lay[x].n_pad;
     if (c->p_g2c[x] <= 0 && ng) c->p_g2c[x] = grate / ng * 4.0 * c->lay[x].n_pad;
     c->p_ocpu[x] = c->cpu_elems.load() > 0
                        ? c->cpu_ms.load() / c->n_threads / (double)c->cpu_elems.load() * c->lay[x].n_pad
@@ -1572,7 +1654,12 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
       }
       CKC(c, cudaMemcpy(tmp.data(), c->slot_param(c->layer_slot[layer]), tmp.size(), cudaMemcpyDeviceToHost));
     } else {
-      std::memcpy(tmp.data(), c->bf16 ? (void*)c->h_shadow[layer] : (void*)c->h_master[layer], tmp.size());
+      if (c->shadow)
+        std::memcpy(tmp.data(), c->h_shadow[layer], tmp.size());
+      else if (c->bf16)
+        cpu::cast_bf16_range(c->h_master[layer], reinterpret_cast<uint16_t*>(tmp.data()), 0, n);
+      else
+        std::memcpy(tmp.data(), c->h_master[layer], tmp.size());
     }
     if (c->bf16)
       unpack_layer_u16(Lx, reinterpret_cast<uint16_t*>(tmp.data()), static_cast<uint16_t*>(dst));
@@ -1665,10 +1752,8 @@ sh_status sh_destroy(sh_ctx* c) {
   if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
     if (s) cudaStreamDestroy(s);
-  if (c->host_base) {
-    cudaHostUnregister(c->host_base);
-    munmap(c->host_base, c->host_bytes);
-  }
+  for (auto& b : c->hblocks) host_block_free(b.p, b.bytes);
+  host_block_free(c->hland.p, c->hland.bytes);
   delete c;
   return SH_OK;
 }

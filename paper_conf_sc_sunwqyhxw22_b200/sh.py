@@ -20,7 +20,8 @@ SH_OK, SH_ERR_INVALID, SH_ERR_CUDA, SH_ERR_OOM_DEVICE, SH_ERR_OOM_HOST, SH_ERR_N
 SH_FP32, SH_BF16_MIXED = 0, 1
 SH_PRE, SH_POST = 0, 1
 SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE = 0, 1, 2, 3
-SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD = 1, 2, 4, 8, 16
+SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32 = \
+    1, 2, 4, 8, 16, 32
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",

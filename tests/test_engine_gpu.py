@@ -107,6 +107,24 @@ def test_clip_windowed_bitwise_and_poison():
             tr.close()
 
 
+def test_fetch_fp32_mode_bitwise_equals_resident():
+    """SH_FLAG_FETCH_FP32: no host shadow, fp32 master over the link, K1 cast on the GPU."""
+    L = TINY["L"]
+    ref, _, _ = engine_run(TINY, STEPS, L, sh.SH_BF16_MIXED)
+    ref_state = engine_state(ref)
+    ref.close()
+    for w in (0, 1, 3):
+        tr, _, _ = engine_run(TINY, STEPS, w, sh.SH_BF16_MIXED, flags=sh.SH_FLAG_FETCH_FP32 | sh.SH_FLAG_POISON)
+        try:
+            ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+            assert ok, f"window {w}: {what}"
+            s = tr.engine.stats()
+            # 4 B/param over the link: FP fetches L-w layers
+            assert s["h2d_bytes"] % 4 == 0 and s["h2d_bytes"] > 0
+        finally:
+            tr.close()
+
+
 def test_window_change_mid_run_bitwise():
     L = TINY["L"]
     ref, _, _ = engine_run(TINY, 4, L, sh.SH_BF16_MIXED)
