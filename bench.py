@@ -34,13 +34,28 @@ CONFIGS = {
     # name: (L, h, nh, s, V, default batch, default window, description)
     "tiny": (4, 256, 4, 128, 512, 2, 2, "BASELINE configs[0]: tiny GPT 4x256, seq 128"),
     "c2": (48, 1600, 25, 1024, 50304, 16, 4, "BASELINE configs[1]: GPT-2 XL-shaped 1.5B (48 x 1600, seq 1024)"),
-    "c3": (48, 4096, 32, 1024, 50304, 16, 4, "BASELINE configs[2]: GPT-style ~10B (48 x 4096, seq 1024)"),
-    # 75 x 4096: 15.3 B params, fp32 params + Adam states = 184 GB > 180 GB of HBM; host store
-    # 12 B/param (fp32-fetch mode, no bf16 shadow) = 175 GB of the box's 196 GB
-    "c4": (75, 4096, 32, 1024, 50304, 16, 4, "BASELINE configs[3]: depth-scaled GPT 75 x 4096 = 15.3B, "
-                                             "states 184 GB > 180 GB HBM (max trainable on this host)"),
+    "c3": (48, 4096, 32, 1024, 50304, 16, -1, "BASELINE configs[2]: GPT-style ~10B (48 x 4096, seq 1024)"),
+    # depth-scaled h=4096 GPT with L = L_max(host RAM); on a 196 GB host that is
+    # 77 layers = 15.7 B params, fp32 params + Adam states 188 GB > 180 GB of HBM, host store 12 B/param
+    # (fp32-fetch mode, no bf16 shadow)
+    "c4": (0, 4096, 32, 1024, 50304, 16, -1, "BASELINE configs[3]: depth-scaled GPT h4096, L = L_max(host RAM), "
+                                            "fp32 states > 180 GB HBM, auto-tuned window"),
 }
 FETCH_FP32_DEFAULT = {"c4"}
+CPU_HARD_DEFAULT = {"c3", "c4"}   # autotune with the eq. 3 CPU-throughput constraint (R19)
+
+
+def c4_layers(h: int, ring: int, w0: int = 2, margin_gb: float = 8.0) -> int:
+    """Deepest h-wide GPT whose host store (12 B/param, per-layer 2 MiB-aligned blocks for layers
+    >= w0, plus `ring` landing buffers) fits in MemAvailable - margin."""
+    avail = None
+    for ln in open("/proc/meminfo"):
+        if ln.startswith("MemAvailable:"):
+            avail = int(ln.split()[1]) * 1024
+    n_pad = sum((n + 127) // 128 * 128 for n in (h, h, 3 * h * h, 3 * h, h * h, h, h, h, 4 * h * h, 4 * h, 4 * h * h, h))
+    per_layer = (12 * n_pad + (1 << 21) - 1) // (1 << 21) * (1 << 21)
+    budget = avail - int(margin_gb * (1 << 30)) - ring * 4 * n_pad
+    return max(w0 + 1, budget // per_layer + w0)
 PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
 PROBE_D2H_GBS = 57.01
 
@@ -185,6 +200,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--fetch-fp32", type=int, default=-1, help="1: no host bf16 shadow, fp32 over the link")
     ap.add_argument("--init-threads", type=int, default=16)
+    ap.add_argument("--layers", type=int, default=0, help="c4: override L_max(host RAM)")
+    ap.add_argument("--trace-out", default="", help="write a Chrome trace of the last profiled step")
+    ap.add_argument("--cpu-hard", type=int, default=-1, help="1: autotune with the eq. 3 CPU constraint")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -214,16 +232,20 @@ def main():
     L, h, nh, s, V, b0, w0, desc = CONFIGS[args.config]
     b = args.batch or b0
     w = w0 if args.window == -2 else args.window
+    if L == 0:
+        L = args.layers or c4_layers(h, args.grad_ring or 4)
     prec = sh.SH_BF16_MIXED if args.precision == "bf16" else sh.SH_FP32
     mc = ModelConfig(L, h, nh, s, V)
     K, W = args.steps, args.warmup
 
     fetch32 = args.fetch_fp32 == 1 or (args.fetch_fp32 == -1 and args.config in FETCH_FP32_DEFAULT)
+    cpu_hard = args.cpu_hard == 1 or (args.cpu_hard == -1 and args.config in CPU_HARD_DEFAULT)
     grad_ring = args.grad_ring or (4 if args.config in ("c3", "c4") else 0)
 
     def run(window, e2e: bool):
         t_init = time.perf_counter()
-        flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0)
+        flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
+            (sh.SH_FLAG_CPU_HARD if cpu_hard else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=args.cpu_threads, grad_ring_depth=grad_ring,
@@ -270,9 +292,22 @@ def main():
             torch.cuda.synchronize()
             e2e_ms = e0.elapsed_time(e1)
         prof = tr.engine.profile() if window != L else None
+        trace = tr.engine.trace()
+        st2 = tr.engine.stats()
+        if args.trace_out and rank == 0:
+            # Chrome trace (chrome://tracing / Perfetto) of the last profiled step: Fig. 4 analogue
+            tid = {"fp": 1, "bp": 1, "k2_adamw": 1, "h2d_fp": 2, "h2d_bp": 2, "d2h_grad": 3, "k1_stage": 4,
+                   "k3_sumsq": 5}
+            ev = [{"name": f"{e['kind']} L{e['layer']}", "ph": "X", "pid": 0, "tid": tid[e["kind"]],
+                   "ts": e["start_ms"] * 1e3, "dur": (e["end_ms"] - e["start_ms"]) * 1e3} for e in trace]
+            names = {1: "compute stream", 2: "H2D copy engine", 3: "D2H copy engine", 4: "K1 stage stream",
+                     5: "K3 (D2H stream)"}
+            ev += [{"name": "thread_name", "ph": "M", "pid": 0, "tid": k, "args": {"name": v}} for k, v in names.items()]
+            with open(args.trace_out + (f".w{window}" if window != w else ""), "w") as f:
+                json.dump({"traceEvents": ev, "displayTimeUnit": "ms"}, f)
         tr.close()
         return dict(ms=ms, e2e_ms=e2e_ms, st0=st0, st1=st1, loss=loss, launches=launches, clocks=clk.summary(),
-                    init_s=t_init, prof=prof)
+                    init_s=t_init, prof=prof, st2=st2)
 
     r = run(w, not args.no_e2e)
     res = None
@@ -314,7 +349,10 @@ def main():
         "dtype": "bf16" if prec == sh.SH_BF16_MIXED else "f32", "data": "synthetic",
         "config": {"workload": args.config, "description": desc, "layers": L, "hidden": h, "heads": nh, "seq": s,
                    "vocab": V, "params": mc.n_params(), "batch_per_gpu": b, "global_batch": b * world,
-                   "window": w, "ring_slots": w + 1, "precision": "bf16_mixed" if prec else "fp32",
+                   "window": r["st1"]["window"], "ring_slots": r["st1"]["n_slots"],
+                   "window_mode": ("autotuned (P1/P2" + (" + eq.3 CPU throughput" if cpu_hard else "") + ")")
+                   if w == -1 else "fixed",
+                   "precision": "bf16_mixed" if prec else "fp32",
                    "parallelism": f"dp{world}",
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),
                    "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
@@ -332,6 +370,8 @@ def main():
             "h2d_step_gbs": d["h2d_bytes"] / (ms / 1e3) / 1e9, "d2h_step_gbs": d["d2h_bytes"] / (ms / 1e3) / 1e9,
             "d2h_frac": d2h_gbs / PROBE_D2H_GBS if d2h_gbs else None,
             "h2d_busy_frac_of_step": d["h2d_busy_ms"] / ms, "d2h_busy_frac_of_step": d["d2h_busy_ms"] / ms,
+            "h2d_overlap_with_compute": r["st2"]["h2d_overlap_frac"],
+            "d2h_overlap_with_compute": r["st2"]["d2h_overlap_frac"],
             "peak_source": "profiles/r01_probe_box.json (pinned 1 GiB copies)"},
         "cpu_adam": {"threads": st1["cpu_threads"], "elems_per_step": d["cpu_adam_elems"] / K,
                      "thread_ms_per_step": d["cpu_adam_ms"] / K,

@@ -81,7 +81,9 @@ typedef enum {
   SH_READ_PARAM = 0,   /* fp32 master parameters (float[numel]) */
   SH_READ_M = 1,       /* fp32 Adam first moment */
   SH_READ_V = 2,       /* fp32 Adam second moment */
-  SH_READ_COMPUTE = 3  /* compute copy: uint16 bf16 bits (bf16 mode) or float (fp32 mode) */
+  SH_READ_COMPUTE = 3, /* compute copy: uint16 bf16 bits (bf16 mode) or float (fp32 mode) */
+  SH_READ_GRAD = 4     /* fp32 gradients of the last step (host layers: from the landing buffer,
+                          SH_ERR_STATE if the ring has reused it) -- diagnostics / parity tests */
 } sh_read_what;
 
 /* One layer (offload unit): its tensors in the caller's order.
@@ -180,7 +182,19 @@ typedef struct {
   double k3_ms_sum;             /* per-layer K3 (Σg²) durations summed (profiled steps) */
   int64_t k3_bytes_sum;
   int64_t k3_samples;
+  /* copy/compute overlap of the last harvested profiled step (Fig. 4 analogue):
+     |copy ∩ compute| / |copy| with compute = union of the per-layer FP/BP compute intervals */
+  double h2d_overlap_frac, d2h_overlap_frac;
+  double last_step_ms;          /* first FP hook .. end of K2 of that step (GPU time) */
 } sh_stats_t;
+
+/* One interval of a profiled step (times in ms from the step's first FP hook). */
+typedef struct {
+  int32_t kind;   /* 0 FP compute, 1 BP compute, 2 H2D (FP), 3 H2D (BP), 4 D2H grads, 5 K1 stage,
+                     6 K3 sumsq, 7 K2 */
+  int32_t layer;  /* -1 for K2 */
+  double start_ms, end_ms;
+} sh_trace_event;
 
 /* ---- lifecycle ------------------------------------------------------------------ */
 
@@ -260,6 +274,10 @@ sh_status sh_get_profile(sh_ctx* ctx, sh_profile* out);
 sh_status sh_read_layer(sh_ctx* ctx, int32_t layer, int32_t what, void* dst);
 
 sh_status sh_stats(sh_ctx* ctx, sh_stats_t* out);
+
+/* Intervals of the last harvested profiled step (SH_FLAG_PROFILE or warm-up steps); *n_out is
+ * the number available (at most cap are written).  Blocks like sh_stats (harvests first). */
+sh_status sh_get_trace(sh_ctx* ctx, sh_trace_event* out, int32_t cap, int32_t* n_out);
 
 /* Thread-local message of the last failed call ("" if none). */
 const char* sh_last_error(void);

@@ -165,8 +165,8 @@ struct ProfSet {  // CUDA timing events of one step (double-buffered by step par
   std::vector<cudaEvent_t> fp0, fp1, bp0, bp1, c2g0[2], c2g1[2], g2c0, g2c1, st0, st1, k30, k31;
   std::vector<std::atomic<uint8_t>> rec_c2g[2], rec_g2c, rec_st;
   std::vector<uint8_t> rec_fp, rec_bp, rec_k3;
-  cudaEvent_t k2a = nullptr, k2b = nullptr;
-  bool rec_k2 = false;
+  cudaEvent_t k2a = nullptr, k2b = nullptr, t0 = nullptr;
+  bool rec_k2 = false, rec_t0 = false;
   bool active = false;
   int64_t step = -1;
   int64_t k2_bytes = 0;
@@ -222,6 +222,10 @@ struct sh_ctx {
   double* partials = nullptr;  // [L+1]
   double* scratch_cs = nullptr;
   double* scratch_comm = nullptr;
+  double* scratch_d2h = nullptr;
+  cudaEvent_t ev_k3_last = nullptr;  // after the K3 of the latest host-layer offload (D2H stream)
+  int64_t k3_last_gen = 0;            // generation of that offload request
+  std::atomic<int64_t> k3_pub{0};     // latest generation whose K3 has been enqueued
   double* norm_dev = nullptr;
   float* coef_dev = nullptr;
   int64_t device_bytes = 0;
@@ -254,6 +258,7 @@ struct sh_ctx {
   std::unique_ptr<std::atomic<int64_t>[]> ready;  // updates applied to layer j
   std::unique_ptr<std::atomic<int64_t>[]> landing_done;
   std::vector<int64_t> landing_uses;
+  std::vector<int> landing_owner, last_landing;  // which layer's grads a landing buffer holds
   int64_t landing_rr = 0;
   int64_t gen = 0;
   std::mutex smu;
@@ -289,6 +294,8 @@ struct sh_ctx {
   std::vector<double> p_fp, p_bp, p_c2g, p_g2c, p_stage, p_ogpu, p_ocpu, p_slot, p_gstate;
   std::vector<int64_t> p_slot_i, p_gstate_i;
   std::vector<double> cpu_ms_layer;  // host timing of CPU Adam per layer (last)
+  std::vector<sh_trace_event> trace;
+  double h2d_overlap = 0, d2h_overlap = 0, last_step_ms = 0;
   double t_async_ms = 0.0;
   int64_t n_async = 0;
   int profiled_steps = 0;
@@ -577,6 +584,7 @@ sh_status prof_alloc(sh_ctx* c, ProfSet& P) {
     if (r == cudaSuccess) r = mk(*v);
   if (r == cudaSuccess) r = cudaEventCreate(&P.k2a);
   if (r == cudaSuccess) r = cudaEventCreate(&P.k2b);
+  if (r == cudaSuccess) r = cudaEventCreate(&P.t0);
   if (r != cudaSuccess) {
     set_error("cudaEventCreate: %s", cudaGetErrorString(r));
     return SH_ERR_CUDA;
@@ -602,6 +610,7 @@ void prof_reset(sh_ctx* c, ProfSet& P, int64_t step) {
     P.rec_k3[i] = 0;
   }
   P.rec_k2 = false;
+  P.rec_t0 = false;
   P.active = true;
   P.step = step;
 }
@@ -613,10 +622,66 @@ float ev_ms(cudaEvent_t a, cudaEvent_t b) {
   return ms;
 }
 
+float ev_at(cudaEvent_t t0, cudaEvent_t e) {
+  float ms = 0;
+  if (cudaEventSynchronize(e) != cudaSuccess) return 0;
+  if (cudaEventElapsedTime(&ms, t0, e) != cudaSuccess) return 0;
+  return ms;
+}
+
+double union_overlap(std::vector<std::pair<double, double>> comp, const std::vector<std::pair<double, double>>& cp,
+                     double* copy_total) {
+  std::sort(comp.begin(), comp.end());
+  std::vector<std::pair<double, double>> u;
+  for (auto& iv : comp) {
+    if (!u.empty() && iv.first <= u.back().second) u.back().second = std::max(u.back().second, iv.second);
+    else u.push_back(iv);
+  }
+  double ov = 0, tot = 0;
+  for (auto& c : cp) {
+    tot += c.second - c.first;
+    for (auto& v : u) ov += std::max(0.0, std::min(c.second, v.second) - std::max(c.first, v.first));
+  }
+  *copy_total = tot;
+  return ov;
+}
+
+void build_trace(sh_ctx* c, ProfSet& P) {
+  if (!P.rec_t0) return;
+  c->trace.clear();
+  auto add = [&](int kind, int layer, cudaEvent_t a, cudaEvent_t b) {
+    c->trace.push_back(sh_trace_event{kind, layer, ev_at(P.t0, a), ev_at(P.t0, b)});
+  };
+  for (int i = 0; i < c->L; ++i) {
+    if (P.rec_fp[i]) add(0, i, P.fp0[i], P.fp1[i]);
+    if (P.rec_bp[i]) add(1, i, P.bp0[i], P.bp1[i]);
+    for (int ph = 0; ph < 2; ++ph)
+      if (P.rec_c2g[ph][i]) add(2 + ph, i, P.c2g0[ph][i], P.c2g1[ph][i]);
+    if (P.rec_g2c[i]) add(4, i, P.g2c0[i], P.g2c1[i]);
+    if (P.rec_st[i]) add(5, i, P.st0[i], P.st1[i]);
+    if (P.rec_k3[i]) add(6, i, P.k30[i], P.k31[i]);
+  }
+  if (P.rec_k2) add(7, -1, P.k2a, P.k2b);
+  std::vector<std::pair<double, double>> comp, h2d, d2h;
+  double end = 0;
+  for (auto& e : c->trace) {
+    end = std::max(end, e.end_ms);
+    if (e.kind <= 1) comp.emplace_back(e.start_ms, e.end_ms);
+    if (e.kind == 2 || e.kind == 3) h2d.emplace_back(e.start_ms, e.end_ms);
+    if (e.kind == 4) d2h.emplace_back(e.start_ms, e.end_ms);
+  }
+  double th = 0, td = 0;
+  const double oh = union_overlap(comp, h2d, &th), od = union_overlap(comp, d2h, &td);
+  c->h2d_overlap = th > 0 ? oh / th : 0;
+  c->d2h_overlap = td > 0 ? od / td : 0;
+  c->last_step_ms = P.rec_k2 ? ev_at(P.t0, P.k2b) : end;
+}
+
 // Read the events of a finished profiled step into the profile arrays and the stats.
 void prof_harvest(sh_ctx* c, ProfSet& P) {
   if (!P.active) return;
   P.active = false;
+  build_trace(c, P);
   const int L = c->L;
   for (int i = 0; i < L; ++i) {
     if (P.rec_fp[i]) c->p_fp[i] = ev_ms(P.fp0[i], P.fp1[i]);
@@ -1077,6 +1142,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   CKC(c.get(), cudaStreamCreateWithFlags(&c->stage, cudaStreamNonBlocking));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_cs_mark, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
+  CKC(c.get(), cudaEventCreateWithFlags(&c->ev_k3_last, cudaEventDisableTiming));
   if (W > 1) {
     CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
     if (!g_nccl.load()) {
@@ -1132,7 +1198,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->device_bytes += 16 * n + (int64_t)c->cb * n;
     CKC(c.get(), cudaMemset(p, 0, 16 * n + (int64_t)c->cb * n));
     double* d = nullptr;
-    const int64_t nd = (c->L + 1) + 2 * (kern::kSumsqMaxBlocks + 1) + 1;
+    const int64_t nd = (c->L + 1) + 3 * (kern::kSumsqMaxBlocks + 1) + 1;
     if (cudaMalloc(&d, nd * 8 + 64) != cudaSuccess) {
       cudaGetLastError();
       set_error("sh_init: cudaMalloc of scratch failed");
@@ -1142,7 +1208,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->partials = d;
     c->scratch_cs = d + (c->L + 1);
     c->scratch_comm = c->scratch_cs + kern::kSumsqMaxBlocks + 1;
-    c->norm_dev = c->scratch_comm + kern::kSumsqMaxBlocks + 1;
+    c->scratch_d2h = c->scratch_comm + kern::kSumsqMaxBlocks + 1;
+    c->norm_dev = c->scratch_d2h + kern::kSumsqMaxBlocks + 1;
     c->coef_dev = reinterpret_cast<float*>(c->norm_dev + 1);
   }
   c->g.assign(c->L, GState{});
@@ -1161,6 +1228,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->landing_done = std::make_unique<std::atomic<int64_t>[]>(c->D);
   for (int k = 0; k < c->D; ++k) c->landing_done[k].store(0);
   c->landing_uses.assign(c->D, 0);
+  c->landing_owner.assign(c->D, -1);
+  c->last_landing.assign(c->L, -1);
   c->reg_done.assign(c->L, 0);
   c->coef_of_step.assign(2, 1.0f);
   c->coef_step.assign(2, -1);
@@ -1289,7 +1358,12 @@ sh_status sh_forward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_param
       }
       // harvest the profile of step-2 (its issuer work is complete by the ready chain)
       prof_harvest(c, c->prof[c->step & 1]);
-      if (step_profiled(c, c->step)) prof_reset(c, c->prof[c->step & 1], c->step);
+      if (step_profiled(c, c->step)) {
+        ProfSet& P = c->prof[c->step & 1];
+        prof_reset(c, P, c->step);
+        CKC(c, cudaEventRecord(P.t0, c->cs));
+        P.rec_t0 = true;
+      }
       CKC(c, cudaMemsetAsync(c->res_grad, 0, 4 * c->res.n_pad, c->cs));
       c->phase = sh_ctx::FP;
     }
@@ -1384,7 +1458,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_comm, c->partials + x, c->comm));
       CKC(c, cudaEventRecord(c->ev_reduced[s], c->comm));
       grads_ready = c->ev_reduced[s];
-    } else {
+    } else if (c->is_g(x)) {
       if (P) CKC(c, cudaEventRecord(P->k30[x], c->cs));
       CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_cs, c->partials + x, c->cs));
       if (P) {
@@ -1392,10 +1466,16 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
         P->rec_k3[x] = 1;
       }
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
+    } else {
+      // host layer: K3 runs on the D2H stream right before the offload (off the compute stream)
+      CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
     }
+    const bool k3_on_d2h = c->W == 1 && !c->is_g(x);
     if (!c->is_g(x)) {
       const int k = (int)(c->landing_rr++ % c->D);
       const int64_t use = c->landing_uses[k]++;
+      c->landing_owner[k] = x;
+      c->last_landing[x] = k;
       const int64_t gen = ++c->gen;
       c->gradfree_gen[s] = gen;
       float* src = c->slot_grad(s);
@@ -1403,14 +1483,26 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       const int64_t step = c->step;
       const sh_adam_scalars sc = c->sc;
       cudaEvent_t gf = c->ev_grad_free[s];
-      c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P] {
+      if (k3_on_d2h) c->k3_last_gen = gen;
+      c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P, k3_on_d2h] {
+        CKA(c, cudaStreamWaitEvent(c->d2h, grads_ready, 0));
+        if (k3_on_d2h) {  // K3 before any host wait: sh_step only needs the norms
+          if (P) CKA(c, cudaEventRecord(P->k30[x], c->d2h));
+          CKA(c, kern::sumsq(src, n, c->scratch_d2h, c->partials + x, c->d2h));
+          if (P) {
+            CKA(c, cudaEventRecord(P->k31[x], c->d2h));
+            P->rec_k3[x] = 1;
+          }
+          CKA(c, cudaEventRecord(c->ev_k3_last, c->d2h));
+          c->k3_pub.store(gen);
+          notify_state(c);
+        }
         if (!state_wait(c, [&] { return c->landing_done[k].load(std::memory_order_acquire) >= use; },
                         "host landing buffer")) {
           c->gradfree_pub[s].store(kInf);
           notify_state(c);
           return;
         }
-        CKA(c, cudaStreamWaitEvent(c->d2h, grads_ready, 0));
         if (P) CKA(c, cudaEventRecord(P->g2c0[x], c->d2h));
         CKA(c, cudaMemcpyAsync(dst, src, 4 * n, cudaMemcpyDeviceToHost, c->d2h));
         if (P) {
@@ -1467,6 +1559,11 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     CKC(c, cudaStreamWaitEvent(c->cs, c->ev_comm_done, 0));
   } else {
     CKC(c, kern::sumsq(c->res_grad, c->res.n_pad, c->scratch_cs, c->partials + L, c->cs));
+    if (c->w < L) {  // the host layers' K3 ran on the D2H stream: wait for the last one only
+      const int64_t gen = c->k3_last_gen;
+      if (!state_wait(c, [&] { return c->k3_pub.load() >= gen; }, "last K3 issue")) return check_failed(c);
+      CKC(c, cudaStreamWaitEvent(c->cs, c->ev_k3_last, 0));
+    }
   }
   CKC(c, kern::norm_finalize(c->partials, L + 1, c->cfg.max_grad_norm, c->norm_dev, c->coef_dev, c->cs));
   ProfSet* P = cur_prof(c);
@@ -1631,7 +1728,7 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
 sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
   clear_error();
   if (!c || !dst) return SH_ERR_INVALID;
-  if (layer < -1 || layer >= c->L || what < 0 || what > 3) {
+  if (layer < -1 || layer >= c->L || what < 0 || what > 4) {
     set_error("sh_read_layer: bad layer %d / what %d", layer, what);
     return SH_ERR_INVALID;
   }
@@ -1668,6 +1765,26 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
     return SH_OK;
   }
   std::vector<float> tmp(n);
+  if (what == SH_READ_GRAD) {  // gradients of the last completed step
+    if (layer < 0) {
+      CKC(c, cudaMemcpy(tmp.data(), c->res_grad, 4 * n, cudaMemcpyDeviceToHost));
+    } else if (c->is_g(layer)) {
+      if (c->layer_slot[layer] < 0) {
+        set_error("sh_read_layer: grads of layer %d not available", layer);
+        return SH_ERR_STATE;
+      }
+      CKC(c, cudaMemcpy(tmp.data(), c->slot_grad(c->layer_slot[layer]), 4 * n, cudaMemcpyDeviceToHost));
+    } else {
+      const int k = c->last_landing[layer];
+      if (k < 0 || c->landing_owner[k] != layer) {
+        set_error("sh_read_layer: grads of layer %d were overwritten in the landing ring (depth %d)", layer, c->D);
+        return SH_ERR_STATE;
+      }
+      std::memcpy(tmp.data(), c->landing[k], 4 * n);
+    }
+    unpack_layer(Lx, tmp.data(), static_cast<float*>(dst));
+    return SH_OK;
+  }
   if (layer < 0 || c->is_g(layer)) {
     const float* src = layer < 0 ? (what == 0 ? c->res_master : what == 1 ? c->res_m : c->res_v)
                                  : (what == 0 ? c->g[layer].master : what == 1 ? c->g[layer].m : c->g[layer].v);
@@ -1712,7 +1829,18 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->k3_ms_sum = c->k3_ms_sum;
   o->k3_bytes_sum = c->k3_bytes_sum;
   o->k3_samples = c->k3_samples;
+  o->h2d_overlap_frac = c->h2d_overlap;
+  o->d2h_overlap_frac = c->d2h_overlap;
+  o->last_step_ms = c->last_step_ms;
   return SH_OK;
+}
+
+sh_status sh_get_trace(sh_ctx* c, sh_trace_event* out, int32_t cap, int32_t* n_out) {
+  clear_error();
+  if (!c || !n_out) return SH_ERR_INVALID;
+  if (c->phase == sh_ctx::IDLE) sync_all(c);
+  *n_out = (int32_t)c->trace.size();
+  for (int i = 0; i < (int)c->trace.size() && i < cap && out; ++i) out[i] = c->trace[i];
 }
 
 sh_status sh_destroy(sh_ctx* c) {
@@ -1746,10 +1874,12 @@ sh_status sh_destroy(sh_ctx* c) {
       for (auto e : *v)
         if (e) cudaEventDestroy(e);
     if (P.k2a) cudaEventDestroy(P.k2a);
+    if (P.t0) cudaEventDestroy(P.t0);
     if (P.k2b) cudaEventDestroy(P.k2b);
   }
   if (c->ev_cs_mark) cudaEventDestroy(c->ev_cs_mark);
   if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
+  if (c->ev_k3_last) cudaEventDestroy(c->ev_k3_last);
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
     if (s) cudaStreamDestroy(s);
   for (auto& b : c->hblocks) host_block_free(b.p, b.bytes);

@@ -19,7 +19,7 @@ SH_OK, SH_ERR_INVALID, SH_ERR_CUDA, SH_ERR_OOM_DEVICE, SH_ERR_OOM_HOST, SH_ERR_N
     SH_ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6, -7
 SH_FP32, SH_BF16_MIXED = 0, 1
 SH_PRE, SH_POST = 0, 1
-SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE = 0, 1, 2, 3
+SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE, SH_READ_GRAD = 0, 1, 2, 3, 4
 SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32 = \
     1, 2, 4, 8, 16, 32
 
@@ -29,7 +29,7 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_autotune_window", "sh_set_window", "sh_get_profile", "sh_read_layer", "sh_stats",
            "sh_last_error", "sh_abi_version", "sh_nccl_get_unique_id", "sh_adam_scalars_for",
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
-           "sh_op_sumsq_gpu", "sh_kernel_launches")
+           "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace")
 
 
 class ShError(RuntimeError):
@@ -79,7 +79,15 @@ class Stats(C.Structure):
                 ("cpu_wait_ms", C.c_double), ("k2_ms_last", C.c_double), ("k2_bytes_last", C.c_int64),
                 ("k2_launches_last", C.c_int32), ("cpu_threads", C.c_int32), ("profiled_steps", C.c_int32),
                 ("k2_ms_sum", C.c_double), ("k2_bytes_sum", C.c_int64), ("k2_samples", C.c_int64),
-                ("k3_ms_sum", C.c_double), ("k3_bytes_sum", C.c_int64), ("k3_samples", C.c_int64)]
+                ("k3_ms_sum", C.c_double), ("k3_bytes_sum", C.c_int64), ("k3_samples", C.c_int64),
+                ("h2d_overlap_frac", C.c_double), ("d2h_overlap_frac", C.c_double), ("last_step_ms", C.c_double)]
+
+
+class TraceEvent(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("layer", C.c_int32), ("start_ms", C.c_double), ("end_ms", C.c_double)]
+
+
+TRACE_KINDS = ("fp", "bp", "h2d_fp", "h2d_bp", "d2h_grad", "k1_stage", "k3_sumsq", "k2_adamw")
 
 
 class AdamScalars(C.Structure):
@@ -116,6 +124,7 @@ def lib() -> C.CDLL:
             "sh_op_adamw_cpu": [vp, vp, vp, vp, vp, i64, i64, C.POINTER(AdamScalars), i32, f32, i32],
             "sh_op_cast_bf16_gpu": [vp, vp, i64, vp], "sh_op_cast_bf16_cpu": [vp, vp, i64],
             "sh_op_sumsq_gpu": [vp, i64, vp, vp],
+            "sh_get_trace": [vp, vp, i32, C.POINTER(i32)],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -378,6 +387,15 @@ class Engine:
             out = np.empty(n, dtype=np.float32)
         check(self._L.sh_read_layer(self.h, layer, what, out.ctypes.data))
         return out
+
+    def trace(self) -> list[dict]:
+        """Intervals of the last profiled step (ms from its first FP hook)."""
+        n = C.c_int32()
+        check(self._L.sh_get_trace(self.h, None, 0, C.byref(n)))
+        buf = (TraceEvent * max(1, n.value))()
+        check(self._L.sh_get_trace(self.h, buf, n.value, C.byref(n)))
+        return [{"kind": TRACE_KINDS[e.kind], "layer": e.layer, "start_ms": e.start_ms, "end_ms": e.end_ms}
+                for e in buf[:n.value]]
 
     def stats(self) -> dict:
         s = Stats()
