@@ -234,6 +234,10 @@ def main():
     w = w0 if args.window == -2 else args.window
     if L == 0:
         L = args.layers or c4_layers(h, args.grad_ring or 4)
+        if world > 1:  # one shared host store per box: every rank must build the same model
+            lt = torch.tensor([L], dtype=torch.int64, device="cuda")
+            dist.broadcast(lt, 0)
+            L = int(lt.item())
     prec = sh.SH_BF16_MIXED if args.precision == "bf16" else sh.SH_FP32
     mc = ModelConfig(L, h, nh, s, V)
     K, W = args.steps, args.warmup
@@ -242,13 +246,21 @@ def main():
     cpu_hard = args.cpu_hard == 1 or (args.cpu_hard == -1 and args.config in CPU_HARD_DEFAULT)
     grad_ring = args.grad_ring or (4 if args.config in ("c3", "c4") else 0)
 
+    shm_name = None
+    cpu_threads = args.cpu_threads
+    if world > 1:
+        import hashlib
+        shm_name = "sh_" + hashlib.sha1(nccl_id).hexdigest()[:16]  # one host store for the box
+        local_world = int(os.environ.get("LOCAL_WORLD_SIZE", world))
+        cpu_threads = cpu_threads or max(1, (os.cpu_count() or 1) // local_world)
+
     def run(window, e2e: bool):
         t_init = time.perf_counter()
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
             (sh.SH_FLAG_CPU_HARD if cpu_hard else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
-                               cpu_threads=args.cpu_threads, grad_ring_depth=grad_ring,
+                               cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads)
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
@@ -354,6 +366,7 @@ def main():
                    if w == -1 else "fixed",
                    "precision": "bf16_mixed" if prec else "fp32",
                    "parallelism": f"dp{world}",
+                   "host_store": "one shared /dev/shm store, rank-sliced offload + CPU Adam" if world > 1 else "private",
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),
                    "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
                    "grad_landing_buffers": grad_ring or L, "host_store_bytes": r["st1"]["host_bytes"],

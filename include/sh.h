@@ -101,6 +101,9 @@ typedef struct {
 #define SH_FLAG_FETCH_FP32 (1ull << 5) /* bf16 mode: no host bf16 shadow (12 instead of 14 B/param of host
                                           RAM); prefetch the fp32 master (4 B/param over the link) into
                                           the slot's idle grad half and K1-cast it on the GPU */
+#define SH_FLAG_TEST_NO_COLLECTIVE (1ull << 6) /* test: world_size > 1 without NCCL (all ranks feed identical
+                                                  data, so the average is the local gradient); exercises
+                                                  the shared store / slicing with several processes */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
@@ -123,6 +126,9 @@ typedef struct {
   int32_t rank;
   const void* nccl_unique_id;       /* 128-byte ncclUniqueId, required when world_size > 1 */
   uint64_t flags;                   /* SH_FLAG_* */
+  const char* shm_name;             /* world_size > 1: name of ONE shared host store for all ranks of the
+                                       box (/dev/shm); rank r offloads and CPU-updates only
+                                       slice r of every layer.  NULL/"": a private replica per rank */
 } sh_config;
 
 /* Per-layer profile consumed by the window solver (PAPER.md:132 notation; times in ms,

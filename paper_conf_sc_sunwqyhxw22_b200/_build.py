@@ -35,8 +35,8 @@ def _nccl_include() -> str:
 
 INCS = ["-I" + os.path.join(ROOT, "include"), "-I" + CSRC, "-I" + os.path.join(CUDA, "include")]
 CXXFLAGS = ["-O3", "-fPIC", "-std=c++17", "-ffp-contract=off", "-fno-fast-math", "-g1", "-Wall",
-            "-Wno-unused-function", "-pthread"]
-NVFLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-ffp-contract=off",
+            "-Wno-unused-function", "-Werror=return-type", "-pthread"]
+NVFLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-ffp-contract=off,-Werror=return-type",
                   "--fmad=false", "-Xptxas", "-v"]
 
 

@@ -32,7 +32,12 @@
 #include <dlfcn.h>
 #include <pthread.h>
 #include <sched.h>
+#include <fcntl.h>
 #include <sys/mman.h>
+#include <sys/stat.h>
+#include <sys/statvfs.h>
+
+#include <cerrno>
 #include <unistd.h>
 
 #include <algorithm>
@@ -185,10 +190,19 @@ struct Job {
   int layer;
   int64_t step;
   int landing;
+  int64_t lo, hi;  // element range of this rank (whole layer unless the store is shared)
   int64_t n_chunks;
   int64_t next = 0;
   std::atomic<int64_t> done{0};
   sh_adam_scalars sc;
+};
+
+// Control block of a shared (multi-process, one box) host store, in /dev/shm.
+struct ShmCtl {
+  std::atomic<int64_t> magic;
+  std::atomic<int64_t> created;    // rank 0 finished creating the layer segments
+  std::atomic<int64_t> bar[4];     // monotonic barrier counters
+  std::atomic<int64_t> cnt[1];     // [L] per-layer slice updates completed (W per step)
 };
 
 struct sh_ctx {
@@ -240,6 +254,14 @@ struct sh_ctx {
   HostBlock hland;
   size_t host_bytes = 0;
   bool shadow = true;  // bf16 shadow kept in host RAM (bf16 mode without SH_FLAG_FETCH_FP32)
+  // shared store (world_size > 1 with shm_name): rank r owns elements [slo[x], shi[x]) of layer x
+  bool shared = false;
+  bool no_collective = false;
+  std::string shm_name;
+  ShmCtl* ctl = nullptr;
+  size_t ctl_bytes = 0;
+  std::vector<int64_t> slo, shi;
+  int64_t bar_calls[4] = {0, 0, 0, 0};
   std::vector<float*> h_master, h_m, h_v;
   std::vector<uint16_t*> h_shadow;
   std::vector<float*> landing;
@@ -377,8 +399,18 @@ bool state_wait(sh_ctx* c, Pred pred, const char* what, double* waited_ms = null
   if (pred()) return true;
   const double t0 = now_ms();
   std::unique_lock<std::mutex> g(c->smu);
-  const bool ok = c->scv.wait_for(g, std::chrono::duration<double>(wait_timeout_s()),
-                                  [&] { return c->failed.load() || pred(); });
+  bool ok;
+  if (c->shared) {  // cross-process progress is only visible by polling the shared counters
+    const double deadline = t0 + 1e3 * wait_timeout_s();
+    for (;;) {
+      if (c->failed.load() || pred()) { ok = true; break; }
+      if (now_ms() > deadline) { ok = false; break; }
+      c->scv.wait_for(g, std::chrono::microseconds(50));
+    }
+  } else {
+    ok = c->scv.wait_for(g, std::chrono::duration<double>(wait_timeout_s()),
+                         [&] { return c->failed.load() || pred(); });
+  }
   if (waited_ms) *waited_ms = now_ms() - t0;
   if (!ok) {
     g.unlock();
@@ -391,6 +423,20 @@ bool state_wait(sh_ctx* c, Pred pred, const char* what, double* waited_ms = null
 void notify_state(sh_ctx* c) {
   { std::lock_guard<std::mutex> g(c->smu); }
   c->scv.notify_all();
+}
+
+// Updates applied to host layer x >= t (all W slices when the store is shared)?
+bool ready_at_least(const sh_ctx* c, int x, int64_t t) {
+  if (c->shared) return c->ctl->cnt[x].load(std::memory_order_acquire) >= (int64_t)c->W * t;
+  return c->ready[x].load(std::memory_order_acquire) >= t;
+}
+
+// Cross-process barrier on the shared control block (polling).
+bool shm_barrier(sh_ctx* c, int id, const char* what) {
+  if (!c->shared) return true;
+  const int64_t target = (int64_t)c->W * (++c->bar_calls[id]);
+  c->ctl->bar[id].fetch_add(1);
+  return state_wait(c, [&] { return c->ctl->bar[id].load() >= target; }, what);
 }
 
 // ---------------------------------------------------------------------------- host store
@@ -465,6 +511,7 @@ void host_block_free(char* p, size_t bytes) {
 // ---------------------------------------------------------------------------- CPU Adam pool
 void finish_job(sh_ctx* c, Job* j) {
   c->ready[j->layer].store(j->step + 1, std::memory_order_release);
+  if (c->shared) c->ctl->cnt[j->layer].fetch_add(1, std::memory_order_release);
   c->landing_done[j->landing].fetch_add(1, std::memory_order_release);
   notify_state(c);
 }
@@ -500,7 +547,7 @@ void worker_loop(sh_ctx* c, int tid) {
     const double t0 = now_ms();
     const int x = job->layer;
     const LayerLayout& Lx = c->lay[x];
-    const int64_t b = chunk * kCpuChunk, e = std::min(Lx.n_pad, b + kCpuChunk);
+    const int64_t b = job->lo + chunk * kCpuChunk, e = std::min(job->hi, b + kCpuChunk);
     cpu::adamw_range(c->h_master[x], c->h_m[x], c->h_v[x], c->landing[job->landing],
                      c->shadow ? c->h_shadow[x] : nullptr, b, e, Lx.n_decay, job->sc, c->clip, coef);
     const double dt = now_ms() - t0;
@@ -535,14 +582,16 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
   j->layer = L->layer;
   j->step = L->step;
   j->landing = L->landing;
-  j->n_chunks = (c->lay[L->layer].n_pad + kCpuChunk - 1) / kCpuChunk;
+  j->lo = c->slo[L->layer];
+  j->hi = c->shi[L->layer];
+  j->n_chunks = (j->hi - j->lo + kCpuChunk - 1) / kCpuChunk;
   j->sc = L->sc;
   if ((c->cfg.flags & SH_FLAG_SYNC_CPU) && !c->clip) {  // debug: inline, single-threaded
     Job* jp = j.get();
     const float coef = 1.0f;
     cpu::adamw_range(c->h_master[jp->layer], c->h_m[jp->layer], c->h_v[jp->layer],
-                     c->landing[jp->landing], c->shadow ? c->h_shadow[jp->layer] : nullptr, 0,
-                     c->lay[jp->layer].n_pad, c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
+                     c->landing[jp->landing], c->shadow ? c->h_shadow[jp->layer] : nullptr, jp->lo,
+                     jp->hi, c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
     finish_job(c, jp);
     return;
   }
@@ -697,7 +746,7 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
       const double ms = ev_ms(P.g2c0[i], P.g2c1[i]);
       c->p_g2c[i] = ms;
       c->d2h_busy += ms;
-      c->d2h_prof_bytes += 4 * c->lay[i].n_pad;
+      c->d2h_prof_bytes += 4 * (c->shi[i] - c->slo[i]);
     }
     if (P.rec_st[i]) c->p_stage[i] = ev_ms(P.st0[i], P.st1[i]);
     if (P.rec_k3[i]) {
@@ -783,8 +832,7 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   const int64_t gf_gen = c->gradfree_gen[s];
   c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, gf, stage_buf, gf_gen, s, n] {
     double waited = 0;
-    if (!state_wait(c, [&] { return c->ready[y].load(std::memory_order_acquire) >= need; },
-                    "CPU Adam of a layer to prefetch", &waited)) {
+    if (!state_wait(c, [&] { return ready_at_least(c, y, need); }, "CPU Adam of a layer to prefetch", &waited)) {
       c->arrive_pub[y].store(kInf);
       notify_state(c);
       return;
@@ -909,13 +957,73 @@ void free_g(sh_ctx* c, int x) {
   c->g[x] = GState{};
 }
 
-// Host block of layer x: [master | m | v | shadow?], 2 MiB aligned.
+std::string shm_path(const sh_ctx* c, const char* suffix, int x = -1) {
+  char b[256];
+  if (x >= 0) snprintf(b, sizeof(b), "/%s.%s%d", c->shm_name.c_str(), suffix, x);
+  else snprintf(b, sizeof(b), "/%s.%s", c->shm_name.c_str(), suffix);
+  return b;
+}
+
+// Map (rank 0: create) a /dev/shm segment of `bytes`; page-lock it in this process.
+sh_status shm_map(sh_ctx* c, const std::string& path, size_t bytes, bool create, char** out, bool touch) {
+  *out = nullptr;
+  int fd = -1;
+  if (create) {
+    if (touch) {
+      const char* mg = getenv("SH_HOST_MARGIN_GB");
+      const int64_t margin = (int64_t)((mg ? atof(mg) : 3.0) * (1ll << 30));
+      if ((int64_t)bytes + margin > mem_available_bytes()) {
+        set_error("shared host store: %lld B requested, %lld B available", (long long)bytes,
+                  (long long)mem_available_bytes());
+        return SH_ERR_OOM_HOST;
+      }
+    }
+    struct statvfs vfs;
+    if (touch && statvfs("/dev/shm", &vfs) == 0 && (int64_t)vfs.f_bavail * (int64_t)vfs.f_frsize < (int64_t)bytes) {
+      set_error("shared host store: /dev/shm has %lld B free, %lld B needed",
+                (long long)vfs.f_bavail * (long long)vfs.f_frsize, (long long)bytes);
+      return SH_ERR_OOM_HOST;
+    }
+    shm_unlink(path.c_str());
+    fd = shm_open(path.c_str(), O_CREAT | O_EXCL | O_RDWR, 0600);
+    if (fd >= 0 && ftruncate(fd, (off_t)bytes) != 0) {
+      close(fd);
+      fd = -1;
+    }
+  } else {
+    fd = shm_open(path.c_str(), O_RDWR, 0600);
+  }
+  if (fd < 0) {
+    set_error("shm_open(%s) failed: %s", path.c_str(), strerror(errno));
+    return SH_ERR_OOM_HOST;
+  }
+  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  close(fd);
+  if (p == MAP_FAILED) {
+    set_error("mmap of shared segment %s failed", path.c_str());
+    return SH_ERR_OOM_HOST;
+  }
+  madvise(p, bytes, MADV_HUGEPAGE);
+  if (create && touch) parallel_touch(static_cast<char*>(p), bytes, c->n_threads);
+  if (touch && cudaHostRegister(p, bytes, cudaHostRegisterPortable) != cudaSuccess) {
+    cudaGetLastError();
+    munmap(p, bytes);
+    set_error("cudaHostRegister of shared segment %s failed", path.c_str());
+    return SH_ERR_OOM_HOST;
+  }
+  *out = static_cast<char*>(p);
+  return SH_OK;
+}
+
+// Host block of layer x: [master | m | v | shadow?], 2 MiB aligned.  Shared stores map the
+// segment rank 0 created (all layers are created collectively in sh_init).
 sh_status ensure_host_layer(sh_ctx* c, int x) {
   if (c->h_master[x]) return SH_OK;
   const int64_t n = c->lay[x].n_pad;
   const size_t bytes = align_up(12 * n + (c->shadow ? 2 * n : 0), 1 << 21);
   char* p = nullptr;
-  sh_status st = host_block_alloc(bytes, c->n_threads, &p);
+  sh_status st = c->shared ? shm_map(c, shm_path(c, "L", x), bytes, c->rank == 0, &p, true)
+                           : host_block_alloc(bytes, c->n_threads, &p);
   if (st != SH_OK) return st;
   c->hblocks[x] = {p, bytes};
   c->host_bytes += bytes;
@@ -975,7 +1083,7 @@ sh_status sync_all(sh_ctx* c) {
   // all host layers updated for the steps taken so far
   if (!state_wait(c, [&] {
         for (int x = 0; x < c->L; ++x)
-          if (!c->is_g(x) && c->ready[x].load() < c->step) return false;
+          if (!c->is_g(x) && !ready_at_least(c, x, c->step)) return false;
         return true;
       }, "CPU Adam drain"))
     return check_failed(c);
@@ -990,15 +1098,22 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   const int w_old = c->w;
   // leaving G: HBM -> host store (bitwise), shadow recomputed with the same RNE
   for (int x = w_new; x < w_old; ++x) {
-    const int64_t n = c->lay[x].n_pad;
     st = ensure_host_layer(c, x);
     if (st != SH_OK) return st;
-    CKC(c, cudaMemcpy(c->h_master[x], c->g[x].master, 4 * n, cudaMemcpyDeviceToHost));
-    CKC(c, cudaMemcpy(c->h_m[x], c->g[x].m, 4 * n, cudaMemcpyDeviceToHost));
-    CKC(c, cudaMemcpy(c->h_v[x], c->g[x].v, 4 * n, cudaMemcpyDeviceToHost));
-    if (c->shadow) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], 0, n);
+    // every rank holds the same GPU state; each writes its own slice of the (shared) store
+    const int64_t lo = c->slo[x], nb = 4 * (c->shi[x] - c->slo[x]);
+    CKC(c, cudaMemcpy(c->h_master[x] + lo, c->g[x].master + lo, nb, cudaMemcpyDeviceToHost));
+    CKC(c, cudaMemcpy(c->h_m[x] + lo, c->g[x].m + lo, nb, cudaMemcpyDeviceToHost));
+    CKC(c, cudaMemcpy(c->h_v[x] + lo, c->g[x].v + lo, nb, cudaMemcpyDeviceToHost));
+    if (c->shadow) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], lo, c->shi[x]);
     c->ready[x].store(c->step);
     free_g(c, x);
+  }
+  if (w_new < w_old && c->shared) {
+    if (!shm_barrier(c, 2, "window change (slices written)")) return check_failed(c);
+    if (c->rank == 0)
+      for (int x = w_new; x < w_old; ++x) c->ctl->cnt[x].store((int64_t)c->W * c->step);
+    if (!shm_barrier(c, 3, "window change (counters)")) return check_failed(c);
   }
   // joining G: host store -> HBM
   for (int x = w_old; x < w_new; ++x) {
@@ -1103,7 +1218,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     return SH_ERR_INVALID;
   }
   const int W = cfg->world_size < 1 ? 1 : cfg->world_size;
-  if (W > 1 && (!cfg->nccl_unique_id || cfg->rank < 0 || cfg->rank >= W)) {
+  if (W > 1 && ((!cfg->nccl_unique_id && !(cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE)) || cfg->rank < 0 ||
+                 cfg->rank >= W)) {
     set_error("sh_init: world_size > 1 needs nccl_unique_id and 0 <= rank < world_size");
     return SH_ERR_INVALID;
   }
@@ -1112,6 +1228,9 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->L = cfg->n_layers;
   c->W = W;
   c->rank = cfg->rank;
+  c->no_collective = W > 1 && (cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE);
+  c->shared = W > 1 && cfg->shm_name && cfg->shm_name[0];
+  if (c->shared) c->shm_name = cfg->shm_name;
   c->bf16 = cfg->precision == SH_BF16_MIXED;
   c->cb = c->bf16 ? 2 : 4;
   c->clip = cfg->max_grad_norm > 0.0f;
@@ -1143,8 +1262,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_cs_mark, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_k3_last, cudaEventDisableTiming));
-  if (W > 1) {
-    CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
+  if (W > 1) CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
+  if (W > 1 && !c->no_collective) {
     if (!g_nccl.load()) {
       set_error("sh_init: world_size > 1 but libnccl.so.2 cannot be loaded");
       return SH_ERR_UNSUPPORTED;
@@ -1176,9 +1295,61 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     for (int k = 0; k < c->D; ++k) c->landing[k] = reinterpret_cast<float*>(p + (int64_t)k * lb);
     c->h_coef = reinterpret_cast<float*>(p + (int64_t)c->D * lb);
   }
-  for (int x = w0; x < c->L; ++x) {  // host-optimised layers of the initial window
-    sh_status st = ensure_host_layer(c.get(), x);
-    if (st != SH_OK) return st;
+  // rank slices (multiples of kPad so every chunk stays 16-element aligned)
+  c->slo.assign(c->L, 0);
+  c->shi.assign(c->L, 0);
+  for (int x = 0; x < c->L; ++x) {
+    const int64_t units = c->lay[x].n_pad / kPad;
+    const int R = c->shared ? c->W : 1, r = c->shared ? c->rank : 0;
+    c->slo[x] = units * r / R * kPad;
+    c->shi[x] = units * (r + 1) / R * kPad;
+  }
+  if (c->shared) {
+    // control block: rank 0 creates it, the others wait for it; then every layer segment
+    c->ctl_bytes = align_up(sizeof(ShmCtl) + 8 * (int64_t)c->L, 4096);
+    char* p = nullptr;
+    if (c->rank == 0) {
+      sh_status st = shm_map(c.get(), shm_path(c.get(), "ctl"), c->ctl_bytes, true, &p, false);
+      if (st != SH_OK) return st;
+      std::memset(p, 0, c->ctl_bytes);
+      c->ctl = reinterpret_cast<ShmCtl*>(p);
+      for (int x = 0; x < c->L; ++x) {
+        sh_status st2 = ensure_host_layer(c.get(), x);
+        if (st2 != SH_OK) return st2;
+      }
+      c->ctl->magic.store(0x5348u);
+      c->ctl->created.store(1);
+    } else {
+      const double t0 = now_ms();
+      for (;;) {  // wait for rank 0's control block and segments
+        sh_status st = shm_map(c.get(), shm_path(c.get(), "ctl"), c->ctl_bytes, false, &p, false);
+        if (st == SH_OK) {
+          c->ctl = reinterpret_cast<ShmCtl*>(p);
+          if (c->ctl->created.load() == 1) break;
+          munmap(p, c->ctl_bytes);
+          c->ctl = nullptr;
+        }
+        if (now_ms() - t0 > 1e3 * wait_timeout_s()) {
+          set_error("shared host store: rank 0 did not create %s", shm_path(c.get(), "ctl").c_str());
+          return SH_ERR_STATE;
+        }
+        usleep(2000);
+      }
+      for (int x = 0; x < c->L; ++x) {
+        sh_status st2 = ensure_host_layer(c.get(), x);
+        if (st2 != SH_OK) return st2;
+      }
+    }
+    if (!shm_barrier(c.get(), 0, "shared store mapping")) return check_failed(c.get());
+    if (c->rank == 0) {  // every rank has it mapped: remove the names (mappings persist)
+      shm_unlink(shm_path(c.get(), "ctl").c_str());
+      for (int x = 0; x < c->L; ++x) shm_unlink(shm_path(c.get(), "L", x).c_str());
+    }
+  } else {
+    for (int x = w0; x < c->L; ++x) {  // host-optimised layers of the initial window
+      sh_status st = ensure_host_layer(c.get(), x);
+      if (st != SH_OK) return st;
+    }
   }
 
   // ---- device: resident set, partials, ring, G states
@@ -1302,7 +1473,7 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
     const int64_t n = c->lay[x].n_pad;
     std::vector<float> tmp;
     float *hp = c->h_master[x], *hm = c->h_m[x], *hv = c->h_v[x];
-    if (!hp) {  // GPU-optimised layer without a host block: stage through a temporary
+    if (!hp || (c->shared && c->rank != 0)) {  // no (own) host copy to write: stage through a temporary
       tmp.resize(3 * n);
       hp = tmp.data();
       hm = hp + n;
@@ -1311,8 +1482,9 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
     pack_layer(c->lay[x], params, hp);
     pack_layer(c->lay[x], m, hm);
     pack_layer(c->lay[x], v, hv);
-    if (c->shadow && c->h_shadow[x]) cpu::cast_bf16_range(hp, c->h_shadow[x], 0, n);
+    if (c->shadow && c->h_shadow[x] && hp == c->h_master[x]) cpu::cast_bf16_range(hp, c->h_shadow[x], 0, n);
     c->ready[x].store(step);
+    if (c->shared && c->rank == 0) c->ctl->cnt[x].store((int64_t)c->W * step);
     if (c->is_g(x)) {
       CKC(c, cudaMemcpy(c->g[x].master, hp, 4 * n, cudaMemcpyHostToDevice));
       CKC(c, cudaMemcpy(c->g[x].m, hm, 4 * n, cudaMemcpyHostToDevice));
@@ -1324,6 +1496,7 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
   bool all = c->res_reg;
   for (int x = 0; x < c->L; ++x) all = all && c->reg_done[x];
   if (all && !c->registered_all) {
+    if (!shm_barrier(c, 1, "registration of the shared host store")) return check_failed(c);
     c->registered_all = true;
     st = stage_g_layers(c);
     if (st != SH_OK) return st;
@@ -1452,9 +1625,12 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       // data parallel: average this layer's grads across ranks before the offload (K-e)
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
       CKC(c, cudaStreamWaitEvent(c->comm, c->ev_grad_done[s], 0));
-      st = nccl_check(c, g_nccl.AllReduce(c->slot_grad(s), c->slot_grad(s), n, ncclFloat, ncclAvg, c->nccl, c->comm),
-                      "ncclAllReduce(layer grads)");
-      if (st != SH_OK) return st;
+      if (!c->no_collective) {
+        st = nccl_check(c, g_nccl.AllReduce(c->slot_grad(s), c->slot_grad(s), n, ncclFloat, ncclAvg, c->nccl,
+                                            c->comm),
+                        "ncclAllReduce(layer grads)");
+        if (st != SH_OK) return st;
+      }
       CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_comm, c->partials + x, c->comm));
       CKC(c, cudaEventRecord(c->ev_reduced[s], c->comm));
       grads_ready = c->ev_reduced[s];
@@ -1480,11 +1656,12 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       c->gradfree_gen[s] = gen;
       float* src = c->slot_grad(s);
       float* dst = c->landing[k];
+      const int64_t lo = c->slo[x], hi = c->shi[x];  // this rank's slice (whole layer unless shared)
       const int64_t step = c->step;
       const sh_adam_scalars sc = c->sc;
       cudaEvent_t gf = c->ev_grad_free[s];
       if (k3_on_d2h) c->k3_last_gen = gen;
-      c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P, k3_on_d2h] {
+      c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P, k3_on_d2h, lo, hi] {
         CKA(c, cudaStreamWaitEvent(c->d2h, grads_ready, 0));
         if (k3_on_d2h) {  // K3 before any host wait: sh_step only needs the norms
           if (P) CKA(c, cudaEventRecord(P->k30[x], c->d2h));
@@ -1504,14 +1681,14 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
           return;
         }
         if (P) CKA(c, cudaEventRecord(P->g2c0[x], c->d2h));
-        CKA(c, cudaMemcpyAsync(dst, src, 4 * n, cudaMemcpyDeviceToHost, c->d2h));
+        CKA(c, cudaMemcpyAsync(dst + lo, src + lo, 4 * (hi - lo), cudaMemcpyDeviceToHost, c->d2h));
         if (P) {
           CKA(c, cudaEventRecord(P->g2c1[x], c->d2h));
           P->rec_g2c[x] = 1;
         }
         CKA(c, cudaEventRecord(gf, c->d2h));
         CKA(c, cudaLaunchHostFunc(c->d2h, landed_cb, new Landed{c, x, step, k, sc}));
-        c->d2h_bytes += 4 * n;
+        c->d2h_bytes += 4 * (hi - lo);
         c->d2h_copies++;
         c->gradfree_pub[s].store(gen);
         notify_state(c);
@@ -1551,9 +1728,12 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     // resident grads: average too, on the comm stream after the caller's embedding backward
     CKC(c, cudaEventRecord(c->ev_cs_mark, c->cs));
     CKC(c, cudaStreamWaitEvent(c->comm, c->ev_cs_mark, 0));
-    st = nccl_check(c, g_nccl.AllReduce(c->res_grad, c->res_grad, c->res.n_pad, ncclFloat, ncclAvg, c->nccl, c->comm),
-                    "ncclAllReduce(resident grads)");
-    if (st != SH_OK) return st;
+    if (!c->no_collective) {
+      st = nccl_check(c, g_nccl.AllReduce(c->res_grad, c->res_grad, c->res.n_pad, ncclFloat, ncclAvg, c->nccl,
+                                          c->comm),
+                      "ncclAllReduce(resident grads)");
+      if (st != SH_OK) return st;
+    }
     CKC(c, kern::sumsq(c->res_grad, c->res.n_pad, c->scratch_comm, c->partials + L, c->comm));
     CKC(c, cudaEventRecord(c->ev_comm_done, c->comm));
     CKC(c, cudaStreamWaitEvent(c->cs, c->ev_comm_done, 0));
@@ -1841,6 +2021,7 @@ sh_status sh_get_trace(sh_ctx* c, sh_trace_event* out, int32_t cap, int32_t* n_o
   if (c->phase == sh_ctx::IDLE) sync_all(c);
   *n_out = (int32_t)c->trace.size();
   for (int i = 0; i < (int)c->trace.size() && i < cap && out; ++i) out[i] = c->trace[i];
+  return SH_OK;
 }
 
 sh_status sh_destroy(sh_ctx* c) {
@@ -1883,6 +2064,7 @@ sh_status sh_destroy(sh_ctx* c) {
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
     if (s) cudaStreamDestroy(s);
   for (auto& b : c->hblocks) host_block_free(b.p, b.bytes);
+  if (c->ctl) munmap(c->ctl, c->ctl_bytes);
   host_block_free(c->hland.p, c->hland.bytes);
   delete c;
   return SH_OK;

@@ -20,8 +20,8 @@ SH_OK, SH_ERR_INVALID, SH_ERR_CUDA, SH_ERR_OOM_DEVICE, SH_ERR_OOM_HOST, SH_ERR_N
 SH_FP32, SH_BF16_MIXED = 0, 1
 SH_PRE, SH_POST = 0, 1
 SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE, SH_READ_GRAD = 0, 1, 2, 3, 4
-SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32 = \
-    1, 2, 4, 8, 16, 32
+SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32, \
+    SH_FLAG_TEST_NO_COLLECTIVE = 1, 2, 4, 8, 16, 32, 64
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
@@ -49,7 +49,7 @@ class Config(C.Structure):
                 ("max_grad_norm", C.c_double), ("device", C.c_int32), ("compute_stream", C.c_void_p),
                 ("cpu_threads", C.c_int32), ("grad_ring_depth", C.c_int32), ("warmup_steps", C.c_int32),
                 ("device_budget_bytes", C.c_int64), ("world_size", C.c_int32), ("rank", C.c_int32),
-                ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64)]
+                ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p)]
 
 
 _PD = C.POINTER(C.c_double)
@@ -248,7 +248,7 @@ class Engine:
     def __init__(self, layer_numels, layer_wd, res_numels, res_wd, *, window, precision=SH_BF16_MIXED,
                  lr=1.5e-4, betas=(0.9, 0.999), eps=1e-8, weight_decay=0.01, max_grad_norm=0.0, device=0,
                  stream=None, cpu_threads=0, grad_ring_depth=0, warmup_steps=5, device_budget_bytes=0,
-                 world_size=1, rank=0, nccl_id: bytes | None = None, flags=0):
+                 world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None):
         L = lib()
         self.n_layers = len(layer_numels)
         self._keep = []
@@ -281,6 +281,8 @@ class Engine:
             idbuf = (C.c_uint8 * 128).from_buffer_copy(nccl_id)
             cfg.nccl_unique_id = C.cast(idbuf, C.c_void_p)
         cfg.flags = flags
+        self._shm = shm_name.encode() if shm_name else None
+        cfg.shm_name = self._shm
         self.precision = precision
         self._cfg = cfg
         self._shapes = shapes

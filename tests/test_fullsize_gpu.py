@@ -78,7 +78,9 @@ def test_fullsize_sampled_adamw(windowed_run):
                                         m1[sel].astype(np.float64), v1[sel].astype(np.float64), 2, opt, d)
             scale = np.abs(p1[sel]) + np.abs(rp - p1[sel])
             assert (np.abs(p2[sel] - rp) <= 1e-6 * scale + 1e-30).all(), (x, d)
-            assert np.allclose(m2[sel], rm, rtol=1e-6, atol=1e-30)
+            # fp32 rounding relative to the magnitudes of the two terms (m can cancel to ~0)
+            mscale = opt.beta1 * np.abs(m1[sel]) + (1 - opt.beta1) * np.abs(g2[sel])
+            assert (np.abs(m2[sel] - rm) <= 1e-6 * mscale + 1e-38).all(), (x, d)
             assert np.allclose(v2[sel], rv, rtol=1e-6, atol=1e-38)
 
 
