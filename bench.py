@@ -202,6 +202,8 @@ def main():
     ap.add_argument("--init-threads", type=int, default=16)
     ap.add_argument("--layers", type=int, default=0, help="c4: override L_max(host RAM)")
     ap.add_argument("--trace-out", default="", help="write a Chrome trace of the last profiled step")
+    ap.add_argument("--attention", default="auto", choices=["auto", "flash", "cublas"],
+                    help="attention core of the GPT driver (outside the hot path)")
     ap.add_argument("--cpu-hard", type=int, default=-1, help="1: autotune with the eq. 3 CPU constraint")
     args = ap.parse_args()
     if args.warmup < 3:
@@ -261,7 +263,9 @@ def main():
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
-                               warmup_steps=W if window == -1 else 5, init_threads=args.init_threads)
+                               warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
+                               attention=args.attention)
+        attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
         host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + K)])
@@ -319,7 +323,7 @@ def main():
                 json.dump({"traceEvents": ev, "displayTimeUnit": "ms"}, f)
         tr.close()
         return dict(ms=ms, e2e_ms=e2e_ms, st0=st0, st1=st1, loss=loss, launches=launches, clocks=clk.summary(),
-                    init_s=t_init, prof=prof, st2=st2)
+                    init_s=t_init, prof=prof, st2=st2, attn=attn_used)
 
     r = run(w, not args.no_e2e)
     res = None
@@ -365,6 +369,7 @@ def main():
                    "window_mode": ("autotuned (P1/P2" + (" + eq.3 CPU throughput" if cpu_hard else "") + ")")
                    if w == -1 else "fixed",
                    "precision": "bf16_mixed" if prec else "fp32",
+                   "gpt_driver_attention": r["attn"],
                    "parallelism": f"dp{world}",
                    "host_store": "one shared /dev/shm store, rank-sliced offload + CPU Adam" if world > 1 else "private",
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),

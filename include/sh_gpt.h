@@ -66,6 +66,19 @@ int32_t gpt_layer_backward(gpt_ctx* ctx, int32_t layer, void* const* params, flo
 /* res_grads[0][tok] += dL/dx_0 rows (stable, deterministic); res_grads[1][pos] += Σ_b rows. */
 int32_t gpt_embed_backward(gpt_ctx* ctx, const int32_t* d_tokens, float* const* res_grads);
 
+/* Staged block, for callers that substitute the attention core (e.g. a fused flash-attention
+ * library kernel on the bf16 path).  Forward: forward_qkv (LN1 + QKV GEMM -> buffer 0, [N,3h],
+ * columns [q|k|v], head j at j*hd) ; caller writes buffer 1 = causal attention output [N,h] ;
+ * forward_out(write_out) (W_o + residual, LN2, MLP; write_out = 0 during the backward recompute).
+ * Backward (after the recompute): backward_mlp (MLP, LN2, W_o grads; d_att -> buffer 2 [N,h]) ;
+ * caller writes buffer 3 = d qkv [N,3h] ; backward_qkv (W_qkv grads, LN1, residual gradient). */
+int32_t gpt_layer_forward_qkv(gpt_ctx* ctx, int32_t layer, void* const* params);
+int32_t gpt_layer_forward_out(gpt_ctx* ctx, int32_t layer, void* const* params, int32_t write_out);
+int32_t gpt_layer_backward_mlp(gpt_ctx* ctx, int32_t layer, void* const* params, float* const* grads);
+int32_t gpt_layer_backward_qkv(gpt_ctx* ctx, int32_t layer, void* const* params, float* const* grads);
+/* 0: qkv [N,3h], 1: att [N,h], 2: d_att [N,h], 3: d_qkv [N,3h] (compute dtype, device). */
+void* gpt_buffer(gpt_ctx* ctx, int32_t which);
+
 /* Device pointer of checkpoint x_l (fp32 [B*S, h]), l in 0..n_layers (diagnostics / tests). */
 float* gpt_checkpoint(gpt_ctx* ctx, int32_t l);
 

@@ -202,7 +202,8 @@ struct ShmCtl {
   std::atomic<int64_t> magic;
   std::atomic<int64_t> created;    // rank 0 finished creating the layer segments
   std::atomic<int64_t> bar[4];     // monotonic barrier counters
-  std::atomic<int64_t> cnt[1];     // [L] per-layer slice updates completed (W per step)
+  std::atomic<int64_t> cnt[1];     // [2L]: cnt[x] slice updates completed (W per step);
+                                   //       cnt[L+x] offloads landed (W per step)
 };
 
 struct sh_ctx {
@@ -524,20 +525,31 @@ void worker_loop(sh_ctx* c, int tid) {
     float coef = 1.0f;
     {
       std::unique_lock<std::mutex> g(c->pmu);
-      c->pcv.wait(g, [&] {
+      // shared store: a slice may only be rewritten once every rank's gradients of the layer have
+      // landed (then no rank can still be fetching this step's parameters of the layer for its
+      // backward).  A real all-reduce implies it; SH_FLAG_TEST_NO_COLLECTIVE relies on it.
+      auto eligible = [&](const Job* jp) {
+        if (jp->next >= jp->n_chunks) return false;
+        if (c->clip && c->coef_step[jp->step & 1] != jp->step) return false;
+        if (c->shared && c->ctl->cnt[c->L + jp->layer].load(std::memory_order_acquire) < (int64_t)c->W * (jp->step + 1))
+          return false;
+        return true;
+      };
+      auto any = [&] {
         if (c->pool_stop || c->failed.load()) return true;
-        for (auto& jp : c->jobs) {
-          if (jp->next >= jp->n_chunks) continue;
-          if (c->clip && c->coef_step[jp->step & 1] != jp->step) continue;
-          return true;
-        }
+        for (auto& jp : c->jobs)
+          if (eligible(jp.get())) return true;
         return false;
-      });
+      };
+      if (c->shared) {
+        while (!any()) c->pcv.wait_for(g, std::chrono::microseconds(100));
+      } else {
+        c->pcv.wait(g, any);
+      }
       if (c->pool_stop || c->failed.load()) return;
       // lowest layer first: it is prefetched first by the next FP (eq. 3)
       for (auto& jp : c->jobs) {
-        if (jp->next >= jp->n_chunks) continue;
-        if (c->clip && c->coef_step[jp->step & 1] != jp->step) continue;
+        if (!eligible(jp.get())) continue;
         if (!job || jp->step < job->step || (jp->step == job->step && jp->layer < job->layer))
           job = jp.get();
       }
@@ -578,6 +590,7 @@ struct Landed {
 void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA calls here
   std::unique_ptr<Landed> L(static_cast<Landed*>(arg));
   sh_ctx* c = L->c;
+  if (c->shared) c->ctl->cnt[c->L + L->layer].fetch_add(1, std::memory_order_release);
   auto j = std::make_unique<Job>();
   j->layer = L->layer;
   j->step = L->step;
@@ -586,7 +599,7 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
   j->hi = c->shi[L->layer];
   j->n_chunks = (j->hi - j->lo + kCpuChunk - 1) / kCpuChunk;
   j->sc = L->sc;
-  if ((c->cfg.flags & SH_FLAG_SYNC_CPU) && !c->clip) {  // debug: inline, single-threaded
+  if ((c->cfg.flags & SH_FLAG_SYNC_CPU) && !c->clip && !c->shared) {  // debug: inline, single-threaded
     Job* jp = j.get();
     const float coef = 1.0f;
     cpu::adamw_range(c->h_master[jp->layer], c->h_m[jp->layer], c->h_v[jp->layer],
@@ -1112,7 +1125,10 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   if (w_new < w_old && c->shared) {
     if (!shm_barrier(c, 2, "window change (slices written)")) return check_failed(c);
     if (c->rank == 0)
-      for (int x = w_new; x < w_old; ++x) c->ctl->cnt[x].store((int64_t)c->W * c->step);
+      for (int x = w_new; x < w_old; ++x) {
+        c->ctl->cnt[x].store((int64_t)c->W * c->step);
+        c->ctl->cnt[c->L + x].store((int64_t)c->W * c->step);
+      }
     if (!shm_barrier(c, 3, "window change (counters)")) return check_failed(c);
   }
   // joining G: host store -> HBM
@@ -1306,7 +1322,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   }
   if (c->shared) {
     // control block: rank 0 creates it, the others wait for it; then every layer segment
-    c->ctl_bytes = align_up(sizeof(ShmCtl) + 8 * (int64_t)c->L, 4096);
+    c->ctl_bytes = align_up(sizeof(ShmCtl) + 16 * (int64_t)c->L, 4096);
     char* p = nullptr;
     if (c->rank == 0) {
       sh_status st = shm_map(c.get(), shm_path(c.get(), "ctl"), c->ctl_bytes, true, &p, false);
@@ -1484,7 +1500,10 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
     pack_layer(c->lay[x], v, hv);
     if (c->shadow && c->h_shadow[x] && hp == c->h_master[x]) cpu::cast_bf16_range(hp, c->h_shadow[x], 0, n);
     c->ready[x].store(step);
-    if (c->shared && c->rank == 0) c->ctl->cnt[x].store((int64_t)c->W * step);
+    if (c->shared && c->rank == 0) {
+      c->ctl->cnt[x].store((int64_t)c->W * step);
+      c->ctl->cnt[c->L + x].store((int64_t)c->W * step);
+    }
     if (c->is_g(x)) {
       CKC(c, cudaMemcpy(c->g[x].master, hp, 4 * n, cudaMemcpyHostToDevice));
       CKC(c, cudaMemcpy(c->g[x].m, hm, 4 * n, cudaMemcpyHostToDevice));

@@ -560,17 +560,27 @@ int softmax(gpt_ctx* c, int64_t rows, bool bwd) {
 void** AP(gpt_ctx* c, int k) { return c->aptr + (int64_t)k * c->B * c->nh; }
 enum { PQ = 0, PK, PV, PS, PP, PO, PDO, PDQ, PDK, PDV };
 
+// Block forward in three stages so a caller can substitute the attention core (stage 2):
+//   fwd_qkv:  ln1, qkv = ln1 W_qkv^T + b_qkv                     -> c->qkv  [N, 3h]
+//   fwd_attn: att = causal softmax(q k^T / sqrt(hd)) v (cuBLAS)   -> c->att  [N, h]
+//   fwd_out:  x_mid = x + att W_o^T + b_o; ln2; MLP; x_out
 template <class T>
-int layer_fwd_impl(gpt_ctx* c, int l, void* const* P, bool write_out) {
-  const int N = c->N, h = c->h, S = c->S, nh = c->nh, hd = h / nh, B = c->B;
+int fwd_qkv(gpt_ctx* c, int l, void* const* P) {
+  const int N = c->N, h = c->h;
   const cudaDataType_t dt = c->dt;
   const float* xin = c->x + (int64_t)l * c->maxN * h;
-  float* xout = c->x + (int64_t)(l + 1) * c->maxN * h;
   const int64_t Nh = (int64_t)N * h;
   (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
                                                                c->ln1_m, c->ln1_r, N, h);
   (g_launches++, 0), bias_fill<T><<<grid_for(3 * Nh / 8), 256, 0, c->st>>>((T*)c->qkv, (const T*)P[3], 3 * h, 3 * Nh / 8);
   CB(rm_gemm(c, false, true, N, 3 * h, h, 1.f, c->ln1, dt, P[2], dt, 1.f, c->qkv, dt));
+  return 0;
+}
+
+template <class T>
+int fwd_attn(gpt_ctx* c) {
+  const int h = c->h, S = c->S, nh = c->nh, hd = h / nh, B = c->B;
+  const cudaDataType_t dt = c->dt;
   const int BH = B * nh;
   const float scale = 1.0f / sqrtf((float)hd);
   CB(gemm_ptr(c, false, true, S, S, hd, scale, AP(c, PQ), dt, 3 * h, AP(c, PK), dt, 3 * h, 0.f, AP(c, PS),
@@ -578,6 +588,16 @@ int layer_fwd_impl(gpt_ctx* c, int l, void* const* P, bool write_out) {
   int r = softmax<T>(c, (int64_t)BH * S, false);
   if (r) return r;
   CB(gemm_ptr(c, false, false, S, hd, S, 1.f, AP(c, PP), dt, S, AP(c, PV), dt, 3 * h, 0.f, AP(c, PO), dt, h, BH));
+  return 0;
+}
+
+template <class T>
+int fwd_out(gpt_ctx* c, int l, void* const* P, bool write_out) {
+  const int N = c->N, h = c->h;
+  const cudaDataType_t dt = c->dt;
+  const float* xin = c->x + (int64_t)l * c->maxN * h;
+  float* xout = c->x + (int64_t)(l + 1) * c->maxN * h;
+  const int64_t Nh = (int64_t)N * h;
   (g_launches++, 0), resid_bias<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(xin, (const T*)P[5], c->x_mid, h, Nh / 8);
   CB(rm_gemm(c, false, true, N, h, h, 1.f, c->att, dt, P[4], dt, 1.f, c->x_mid, CUDA_R_32F));
   (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->x_mid, (const T*)P[6], (const T*)P[7],
@@ -596,14 +616,24 @@ int layer_fwd_impl(gpt_ctx* c, int l, void* const* P, bool write_out) {
 }
 
 template <class T>
-int layer_bwd_impl(gpt_ctx* c, int l, void* const* P, float* const* G) {
-  int r = layer_fwd_impl<T>(c, l, P, false);  // recompute (activation checkpointing)
-  if (r) return r;
-  const int N = c->N, h = c->h, S = c->S, nh = c->nh, hd = h / nh, B = c->B;
+int layer_fwd_impl(gpt_ctx* c, int l, void* const* P, bool write_out) {
+  int r;
+  if ((r = fwd_qkv<T>(c, l, P))) return r;
+  if ((r = fwd_attn<T>(c))) return r;
+  return fwd_out<T>(c, l, P, write_out);
+}
+
+// Block backward in three stages (after the forward of the layer was recomputed):
+//   bwd_mlp:  MLP and W_o backward, LN2 backward; d_att = d(x_mid) W_o  -> c->datt [N, h]
+//   bwd_attn: dq, dk, dv of the attention core (cuBLAS path)           -> c->dqkv [N, 3h]
+//   bwd_qkv:  W_qkv backward, LN1 backward (residual gradient propagated in place)
+template <class T>
+int bwd_mlp(gpt_ctx* c, int l, void* const* P, float* const* G) {
+  (void)l;
+  const int N = c->N, h = c->h;
   const cudaDataType_t dt = c->dt;
-  const float* xin = c->x + (int64_t)l * c->maxN * h;
   const int64_t Nh = (int64_t)N * h;
-  // ---- MLP
+  int r;
   (g_launches++, 0), cast_f2t<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh / 8);
   CB(rm_gemm(c, true, false, h, 4 * h, N, 1.f, c->dy, dt, c->fc_act, dt, 0.f, G[10], CUDA_R_32F));
   if ((r = colsum(c, c->dres, true, N, h, G[11]))) return r;
@@ -616,21 +646,37 @@ int layer_bwd_impl(gpt_ctx* c, int l, void* const* P, float* const* G) {
                                                                c->dres, c->tmp, N, h);
   if ((r = colsum(c, c->tmp, true, N, h, G[6]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[7]))) return r;
-  // ---- attention
   (g_launches++, 0), cast_f2t<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh / 8);
   CB(rm_gemm(c, true, false, h, h, N, 1.f, c->dy, dt, c->att, dt, 0.f, G[4], CUDA_R_32F));
   if ((r = colsum(c, c->dres, true, N, h, G[5]))) return r;
   CB(rm_gemm(c, false, false, N, h, h, 1.f, c->dy, dt, P[4], dt, 0.f, c->datt, dt));
+  return 0;
+}
+
+template <class T>
+int bwd_attn(gpt_ctx* c) {
+  const int h = c->h, S = c->S, nh = c->nh, hd = h / nh, B = c->B;
+  const cudaDataType_t dt = c->dt;
   const int BH = B * nh;
   const float scale = 1.0f / sqrtf((float)hd);
   CB(gemm_ptr(c, false, true, S, S, hd, 1.f, AP(c, PDO), dt, h, AP(c, PV), dt, 3 * h, 0.f, AP(c, PS), CUDA_R_32F, S,
               BH));
   CB(gemm_ptr(c, true, false, S, hd, S, 1.f, AP(c, PP), dt, S, AP(c, PDO), dt, h, 0.f, AP(c, PDV), dt, 3 * h, BH));
-  if ((r = softmax<T>(c, (int64_t)BH * S, true))) return r;
+  int r = softmax<T>(c, (int64_t)BH * S, true);
+  if (r) return r;
   CB(gemm_ptr(c, false, false, S, hd, S, scale, AP(c, PP), dt, S, AP(c, PK), dt, 3 * h, 0.f, AP(c, PDQ), dt, 3 * h,
               BH));
   CB(gemm_ptr(c, true, false, S, hd, S, scale, AP(c, PP), dt, S, AP(c, PQ), dt, 3 * h, 0.f, AP(c, PDK), dt, 3 * h,
               BH));
+  return 0;
+}
+
+template <class T>
+int bwd_qkv(gpt_ctx* c, int l, void* const* P, float* const* G) {
+  const int N = c->N, h = c->h;
+  const cudaDataType_t dt = c->dt;
+  const float* xin = c->x + (int64_t)l * c->maxN * h;
+  int r;
   CB(rm_gemm(c, true, false, 3 * h, h, N, 1.f, c->dqkv, dt, c->ln1, dt, 0.f, G[2], CUDA_R_32F));
   if ((r = colsum(c, c->dqkv, false, N, 3 * h, G[3]))) return r;
   CB(rm_gemm(c, false, false, N, h, 3 * h, 1.f, c->dqkv, dt, P[2], dt, 0.f, c->dln, CUDA_R_32F));
@@ -640,6 +686,15 @@ int layer_bwd_impl(gpt_ctx* c, int l, void* const* P, float* const* G) {
   if ((r = colsum(c, c->dln, true, N, h, G[1]))) return r;
   CK(cudaGetLastError());
   return 0;
+}
+
+template <class T>
+int layer_bwd_impl(gpt_ctx* c, int l, void* const* P, float* const* G) {
+  int r = layer_fwd_impl<T>(c, l, P, false);  // recompute (activation checkpointing)
+  if (r) return r;
+  if ((r = bwd_mlp<T>(c, l, P, G))) return r;
+  if ((r = bwd_attn<T>(c))) return r;
+  return bwd_qkv<T>(c, l, P, G);
 }
 
 template <class T>
@@ -818,6 +873,49 @@ int32_t gpt_layer_backward(gpt_ctx* c, int32_t l, void* const* P, float* const* 
     return -1;
   }
   return c->bf16 ? layer_bwd_impl<bf16>(c, l, P, G) : layer_bwd_impl<float>(c, l, P, G);
+}
+
+static bool stage_ok(gpt_ctx* c, int32_t l, const void* P) {
+  if (!c || !P || l < 0 || l >= c->L || c->B == 0) {
+    seterr("gpt stage: bad layer %d or no embed_forward", l);
+    return false;
+  }
+  return true;
+}
+
+int32_t gpt_layer_forward_qkv(gpt_ctx* c, int32_t l, void* const* P) {
+  g_err.clear();
+  if (!stage_ok(c, l, P)) return -1;
+  return c->bf16 ? fwd_qkv<bf16>(c, l, P) : fwd_qkv<float>(c, l, P);
+}
+
+int32_t gpt_layer_forward_out(gpt_ctx* c, int32_t l, void* const* P, int32_t write_out) {
+  g_err.clear();
+  if (!stage_ok(c, l, P)) return -1;
+  return c->bf16 ? fwd_out<bf16>(c, l, P, write_out != 0) : fwd_out<float>(c, l, P, write_out != 0);
+}
+
+int32_t gpt_layer_backward_mlp(gpt_ctx* c, int32_t l, void* const* P, float* const* G) {
+  g_err.clear();
+  if (!stage_ok(c, l, P) || !G) return -1;
+  return c->bf16 ? bwd_mlp<bf16>(c, l, P, G) : bwd_mlp<float>(c, l, P, G);
+}
+
+int32_t gpt_layer_backward_qkv(gpt_ctx* c, int32_t l, void* const* P, float* const* G) {
+  g_err.clear();
+  if (!stage_ok(c, l, P) || !G) return -1;
+  return c->bf16 ? bwd_qkv<bf16>(c, l, P, G) : bwd_qkv<float>(c, l, P, G);
+}
+
+void* gpt_buffer(gpt_ctx* c, int32_t which) {
+  if (!c) return nullptr;
+  switch (which) {
+    case 0: return c->qkv;
+    case 1: return c->att;
+    case 2: return c->datt;
+    case 3: return c->dqkv;
+    default: return nullptr;
+  }
 }
 
 int32_t gpt_embed_backward(gpt_ctx* c, const int32_t* tok, float* const* G) {

@@ -17,7 +17,7 @@ import torch
 import synth
 
 from . import sh
-from .gpt import GPT
+from .gpt import GPT, FlashAttention
 
 
 @dataclass
@@ -52,7 +52,8 @@ class StrongholdTrainer:
 
     def __init__(self, mc: ModelConfig, *, batch: int, window: int, precision=sh.SH_BF16_MIXED, lr=1.5e-4,
                  max_grad_norm=0.0, device=0, seed=1234, cpu_threads=0, grad_ring_depth=0, warmup_steps=5,
-                 flags=0, world_size=1, rank=0, nccl_id=None, init=True, init_threads=8, shm_name=None):
+                 flags=0, world_size=1, rank=0, nccl_id=None, init=True, init_threads=8, shm_name=None,
+                 attention="auto"):
         self.mc = mc
         self.batch = batch
         self.device = torch.device("cuda", device)
@@ -67,6 +68,15 @@ class StrongholdTrainer:
                                 flags=flags, shm_name=shm_name)
         self.gpt = GPT(n_layers=L, hidden=mc.hidden, heads=mc.heads, seq=mc.seq, max_batch=batch,
                        vocab=mc.vocab, precision=precision, device=device, stream=self.stream)
+        # attention core: fused flash-attention library kernel on the bf16 path ("auto"/"flash"),
+        # else the cuBLAS batched-GEMM + softmax kernels inside libsh_gpt ("cublas", and fp32 mode)
+        self.flash = None
+        if attention == "flash" or (attention == "auto" and precision == sh.SH_BF16_MIXED):
+            try:
+                self.flash = FlashAttention(self.gpt, batch, mc.seq, mc.hidden, mc.heads)
+            except ImportError:
+                if attention == "flash":
+                    raise
         self.tok_dev = torch.empty((batch, mc.seq + 1), dtype=torch.int32, device=self.device)
         self.loss_dev = torch.zeros(1, dtype=torch.float32, device=self.device)
         self.loss_host = torch.zeros(1, dtype=torch.float32).pin_memory()
@@ -101,21 +111,35 @@ class StrongholdTrainer:
         tok = self.tok_dev.data_ptr()
         rp, rg = e.resident()
         L = self.mc.n_layers
+        fa = self.flash
+        if fa is not None:
+            fa.set_batch(B)
         with torch.cuda.stream(self.stream):
             # FP: pre_forward -> compute -> post_forward
-            P = e.forward_pre(0)
-            g.embed_forward(tok, B, rp)
-            g.layer_forward(0, P)
-            e.forward_post(0)
-            for i in range(1, L):
+            for i in range(L):
                 P = e.forward_pre(i)
-                g.layer_forward(i, P)
+                if i == 0:
+                    g.embed_forward(tok, B, rp)
+                if fa is None:
+                    g.layer_forward(i, P)
+                else:
+                    g.forward_qkv(i, P)
+                    fa.forward()
+                    g.forward_out(i, P, True)
                 e.forward_post(i)
             g.head(tok, rp, rg, self.loss_dev.data_ptr())
             # BP: pre_backward -> recompute + backward -> post (offload + CPU Adam)
             for i in range(L - 1, -1, -1):
                 P, G = e.backward_pre(i)
-                g.layer_backward(i, P, G)
+                if fa is None:
+                    g.layer_backward(i, P, G)
+                else:
+                    g.forward_qkv(i, P)       # recompute from the layer's checkpoint
+                    fa.forward()
+                    g.forward_out(i, P, False)
+                    g.backward_mlp(i, P, G)
+                    fa.backward()
+                    g.backward_qkv(i, P, G)
                 e.backward_post(i)
             g.embed_backward(tok, rg)
             return e.step(want_norm=want_norm)

@@ -51,9 +51,11 @@ def test_fp32_vs_oracle(oracle_noclip, window):
         tr.close()
 
 
-def test_bf16_vs_oracle(oracle_noclip):
+@pytest.mark.parametrize("attention", ["flash", "cublas"])
+def test_bf16_vs_oracle(oracle_noclip, attention):
     st, olosses, _ = oracle_noclip
-    tr, losses, _ = engine_run(TINY, STEPS, 2, sh.SH_BF16_MIXED)
+    tr, losses, _ = engine_run(TINY, STEPS, 2, sh.SH_BF16_MIXED, attention=attention)
+    assert (tr.flash is not None) == (attention == "flash")
     try:
         errs = _errors(tr, st)
         assert max(errs.values()) <= BF16_TOL, errs
