@@ -4,9 +4,12 @@
   python bench.py --impl reference ...     # the CPU oracle, timed on this box's host cores
 
 Metric (BASELINE.json): samples/s at max trainable size per B200; host-link GB/s vs peak.
-Workload (N=1): BASELINE.json configs[1], GPT-2 XL-shaped 1.5B (48 layers, h 1600, 25 heads,
-seq 1024, V 50304), bf16 mixed precision, batch 16 per GPU, window 4 (the paper's artifact
-default), parameters + Adam states in pinned host RAM.  A "step" is one full
+Workload (N=1, default): BASELINE.json configs[3] -- the metric is quoted "at max trainable size
+per B200": a depth-scaled GPT (h 4096, 32 heads, seq 1024, V 50304) whose depth L is the largest the
+host RAM can hold (fp32 master + Adam m, v = 12 B/param in pinned host RAM; fp32 states > 180 GB of
+HBM), bf16 mixed precision, batch 16 per GPU, window auto-tuned by the paper's model (P1/P2) plus
+the eq. 3 CPU-throughput constraint.  `--config c2` is configs[1] (GPT-2 XL-shaped 1.5B), `c3`
+configs[2] (10B), `tiny` configs[0].  A "step" is one full
 training iteration through every §8(a) row: prefetch H2D, K1 restage, per-layer K3, grad D2H,
 CPU AdamW, K2 (and, outside the hot path, the GPT block compute that drives it).
 
@@ -45,16 +48,29 @@ FETCH_FP32_DEFAULT = {"c4"}
 CPU_HARD_DEFAULT = {"c3", "c4"}   # autotune with the eq. 3 CPU-throughput constraint (R19)
 
 
-def c4_layers(h: int, ring: int, w0: int = 2, margin_gb: float = 8.0) -> int:
-    """Deepest h-wide GPT whose host store (12 B/param, per-layer 2 MiB-aligned blocks for layers
-    >= w0, plus `ring` landing buffers) fits in MemAvailable - margin."""
-    avail = None
+def mem_available() -> int:
     for ln in open("/proc/meminfo"):
         if ln.startswith("MemAvailable:"):
-            avail = int(ln.split()[1]) * 1024
+            return int(ln.split()[1]) * 1024
+    return 0
+
+
+def shm_free() -> int:
+    try:
+        st = os.statvfs("/dev/shm")
+        return st.f_bavail * st.f_frsize
+    except OSError:
+        return 0
+
+
+def c4_layers(h: int, ring: int, w0: int = 2, margin_gb: float = 8.0, ranks_sharing: int = 1,
+              budget: int | None = None) -> int:
+    """Deepest h-wide GPT whose host store (12 B/param, per-layer 2 MiB-aligned blocks for layers
+    >= w0, plus `ring` landing buffers per rank) fits in MemAvailable - margin (or `budget`)."""
+    avail = budget if budget is not None else mem_available()
     n_pad = sum((n + 127) // 128 * 128 for n in (h, h, 3 * h * h, 3 * h, h * h, h, h, h, 4 * h * h, 4 * h, 4 * h * h, h))
     per_layer = (12 * n_pad + (1 << 21) - 1) // (1 << 21) * (1 << 21)
-    budget = avail - int(margin_gb * (1 << 30)) - ring * 4 * n_pad
+    budget = avail - int(margin_gb * (1 << 30)) - ranks_sharing * ring * 4 * n_pad
     return max(w0 + 1, budget // per_layer + w0)
 PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
 PROBE_D2H_GBS = 57.01
@@ -189,7 +205,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="sh", choices=["sh", "reference"])
-    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="c4", choices=sorted(CONFIGS))
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--window", type=int, default=-2, help="-2: config default, -1: autotune, L: resident")
     ap.add_argument("--precision", default="bf16", choices=["bf16", "fp32"])
@@ -234,9 +250,22 @@ def main():
     L, h, nh, s, V, b0, w0, desc = CONFIGS[args.config]
     b = args.batch or b0
     w = w0 if args.window == -2 else args.window
+    # data parallel: one shared /dev/shm host store per box when /dev/shm can hold it, else a
+    # private replica per rank with the host RAM divided between the ranks of the box
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", world))
+    use_shm = world > 1
+    if world > 1:
+        flag = torch.tensor([1 if shm_free() > 0.8 * mem_available() else 0], dtype=torch.int64, device="cuda")
+        dist.broadcast(flag, 0)
+        use_shm = bool(flag.item())
     if L == 0:
-        L = args.layers or c4_layers(h, args.grad_ring or 4)
-        if world > 1:  # one shared host store per box: every rank must build the same model
+        if args.layers:
+            L = args.layers
+        elif not use_shm and world > 1:
+            L = c4_layers(h, args.grad_ring or 4, budget=mem_available() // local_world)
+        else:
+            L = c4_layers(h, args.grad_ring or 4, ranks_sharing=local_world)
+        if world > 1:  # every rank must build the same model
             lt = torch.tensor([L], dtype=torch.int64, device="cuda")
             dist.broadcast(lt, 0)
             L = int(lt.item())
@@ -252,8 +281,8 @@ def main():
     cpu_threads = args.cpu_threads
     if world > 1:
         import hashlib
-        shm_name = "sh_" + hashlib.sha1(nccl_id).hexdigest()[:16]  # one host store for the box
-        local_world = int(os.environ.get("LOCAL_WORLD_SIZE", world))
+        if use_shm:
+            shm_name = "sh_" + hashlib.sha1(nccl_id).hexdigest()[:16]  # one host store for the box
         cpu_threads = cpu_threads or max(1, (os.cpu_count() or 1) // local_world)
 
     def run(window, e2e: bool):
@@ -371,7 +400,8 @@ def main():
                    "precision": "bf16_mixed" if prec else "fp32",
                    "gpt_driver_attention": r["attn"],
                    "parallelism": f"dp{world}",
-                   "host_store": "one shared /dev/shm store, rank-sliced offload + CPU Adam" if world > 1 else "private",
+                   "host_store": ("one shared /dev/shm store, rank-sliced offload + CPU Adam" if shm_name else
+                                  "private per rank") if world > 1 else "private",
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),
                    "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
                    "grad_landing_buffers": grad_ring or L, "host_store_bytes": r["st1"]["host_bytes"],

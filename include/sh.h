@@ -122,6 +122,7 @@ typedef struct {
   int32_t grad_ring_depth;          /* host landing buffers for offloaded grads; 0 = one per host layer */
   int32_t warmup_steps;             /* profiled steps before autotune (default 5); 0 = default */
   int64_t device_budget_bytes;      /* S_avail for ring + G states; 0 = free memory - 2 GiB */
+  double cpu_util_max;              /* autotuner eq. 3 utilisation target rho (SH_FLAG_CPU_HARD); 0 = 0.85 */
   int32_t world_size;               /* data-parallel ranks (1 = single GPU) */
   int32_t rank;
   const void* nccl_unique_id;       /* 128-byte ncclUniqueId, required when world_size > 1 */
@@ -149,7 +150,8 @@ typedef struct {
   int64_t s_avail;             /* S_avail */
   int32_t duplex;              /* 1: soft constraints use max(Σc2g, Σg2c) (R7) */
   int32_t cpu_hard;            /* 1: also require the CPU-update throughput form of eq. 3 (R19):
-                                  Σ_{k>=w} t_opt_cpu^k <= Σ_i (t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i */
+                                  Σ_{k>=w} t_opt_cpu^k <= rho * (Σ_i (t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i) */
+  double cpu_util_max;         /* rho in (0, 1]; <= 0 means 1 (utilisation target of the CPU pool) */
 } sh_profile;
 
 typedef struct {

@@ -14,7 +14,7 @@ code shared with the C++ solver (paper_conf_sc_sunwqyhxw22_b200/csrc/autotune.cp
   (1d) sum over the same FP windows: sum t_fp >= sum t_c2g + sum t_g2c   (max() if duplex)
   (2d) sum over the same BP windows: sum t_bp >= sum t_c2g + sum t_g2c   (max() if duplex)
   rule: min{w < L : mem & hard & soft}, else min{w <= L : mem & hard}, else max{w : mem}
-  cpu_hard (optional): sum_{k>=w} t_opt_cpu[k] <= sum_i (t_fp[i] + t_bp[i]) + sum_{i<w} t_opt_gpu[i]
+  cpu_hard (optional): sum_{k>=w} t_opt_cpu[k] <= rho (sum_i (t_fp[i] + t_bp[i]) + sum_{i<w} t_opt_gpu[i])
   eq. 3 slack: min_{k in [w, L)} [ sum_{i<=k}(t_fp[i]+t_bp[i]) + sum_{i<w} t_opt_gpu[i] - t_opt_cpu[k] ]
   eq. 4: 5 L t_async  vs  sum_{i=w}^{L-1} t_opt_gpu[i]
 """
@@ -26,7 +26,8 @@ def _z(a, n):
 
 
 def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
-          slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False, cpu_hard=False):
+          slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False, cpu_hard=False,
+          cpu_util_max=1.0):
     L = len(t_fp)
     fp, bp, c2g, g2c = _z(t_fp, L), _z(t_bp, L), _z(t_c2g, L), _z(t_g2c, L)
     st, og, oc = _z(t_stage, L), _z(t_opt_gpu, L), _z(t_opt_cpu, L)
@@ -76,7 +77,8 @@ def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None
     def cpu_ok(w):
         if not cpu_hard:
             return True
-        return sum(oc[k] for k in range(w, L)) <= sum(fp) + sum(bp) + sum(og[:w])
+        rho = cpu_util_max if 0.0 < cpu_util_max < 1.0 else 1.0
+        return sum(oc[k] for k in range(w, L)) <= rho * (sum(fp) + sum(bp) + sum(og[:w]))
 
     def hard(w):
         return fp_hard(w) and bp_hard(w) and cpu_ok(w)

@@ -92,8 +92,9 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
     return t;
   };
   auto gpu_step = [&](int w) { return fp.sum(0, L) + bp.sum(0, L) + ogpu.sum(0, w); };
+  const double rho = P->cpu_util_max > 0.0 && P->cpu_util_max < 1.0 ? P->cpu_util_max : 1.0;
   auto hard = [&](int w) {
-    return fp_hard(w) && bp_hard(w) && (!P->cpu_hard || cpu_total(w) <= gpu_step(w));
+    return fp_hard(w) && bp_hard(w) && (!P->cpu_hard || cpu_total(w) <= rho * gpu_step(w));
   };
   int wmax = -1;
   for (int w = 0; w <= L; ++w)

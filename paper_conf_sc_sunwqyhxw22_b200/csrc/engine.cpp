@@ -1881,6 +1881,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
                                               : held + (int64_t)fr - ((int64_t)2 << 30);
   o->duplex = (c->cfg.flags & SH_FLAG_DUPLEX) ? 1 : 0;
   o->cpu_hard = (c->cfg.flags & SH_FLAG_CPU_HARD) ? 1 : 0;
+  o->cpu_util_max = c->cfg.cpu_util_max > 0.0 ? c->cfg.cpu_util_max : 0.85;
   return SH_OK;
 }
 

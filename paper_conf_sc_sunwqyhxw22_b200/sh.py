@@ -48,7 +48,8 @@ class Config(C.Structure):
                 ("beta2", C.c_double), ("eps", C.c_double), ("weight_decay", C.c_double),
                 ("max_grad_norm", C.c_double), ("device", C.c_int32), ("compute_stream", C.c_void_p),
                 ("cpu_threads", C.c_int32), ("grad_ring_depth", C.c_int32), ("warmup_steps", C.c_int32),
-                ("device_budget_bytes", C.c_int64), ("world_size", C.c_int32), ("rank", C.c_int32),
+                ("device_budget_bytes", C.c_int64), ("cpu_util_max", C.c_double), ("world_size", C.c_int32),
+                ("rank", C.c_int32),
                 ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p)]
 
 
@@ -60,7 +61,8 @@ class Profile(C.Structure):
     _fields_ = [("n_layers", C.c_int32), ("t_fp", _PD), ("t_bp", _PD), ("t_c2g", _PD), ("t_g2c", _PD),
                 ("t_stage", _PD), ("t_opt_gpu", _PD), ("t_opt_cpu", _PD), ("t_async", C.c_double),
                 ("slot_bytes", _PI64), ("gstate_bytes", _PI64), ("fixed_bytes", C.c_int64),
-                ("s_avail", C.c_int64), ("duplex", C.c_int32), ("cpu_hard", C.c_int32)]
+                ("s_avail", C.c_int64), ("duplex", C.c_int32), ("cpu_hard", C.c_int32),
+                ("cpu_util_max", C.c_double)]
 
 
 class SolveReport(C.Structure):
@@ -215,7 +217,7 @@ def _dbl(a, n):
 
 def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
                  slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False,
-                 cpu_hard=False) -> dict:
+                 cpu_hard=False, cpu_util_max=1.0) -> dict:
     """Pure call of sh_solve_window (no GPU)."""
     n = len(t_fp)
     keep = {}
@@ -235,6 +237,7 @@ def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_c
     prof.s_avail = int(s_avail)
     prof.duplex = 1 if duplex else 0
     prof.cpu_hard = 1 if cpu_hard else 0
+    prof.cpu_util_max = cpu_util_max
     rep = SolveReport()
     check(lib().sh_solve_window(C.byref(prof), C.byref(rep)))
     return {f: getattr(rep, f) for f, _ in SolveReport._fields_}
@@ -373,7 +376,7 @@ class Engine:
         check(self._L.sh_get_profile(self.h, C.byref(p)))
         n = p.n_layers
         out = {"n_layers": n, "t_async": p.t_async, "s_avail": p.s_avail, "fixed_bytes": p.fixed_bytes,
-               "duplex": p.duplex, "cpu_hard": p.cpu_hard}
+               "duplex": p.duplex, "cpu_hard": p.cpu_hard, "cpu_util_max": p.cpu_util_max}
         for f in ("t_fp", "t_bp", "t_c2g", "t_g2c", "t_stage", "t_opt_gpu", "t_opt_cpu"):
             out[f] = [getattr(p, f)[i] for i in range(n)]
         for f in ("slot_bytes", "gstate_bytes"):

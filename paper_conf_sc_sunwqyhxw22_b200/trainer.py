@@ -80,6 +80,9 @@ class StrongholdTrainer:
         self.tok_dev = torch.empty((batch, mc.seq + 1), dtype=torch.int32, device=self.device)
         self.loss_dev = torch.zeros(1, dtype=torch.float32, device=self.device)
         self.loss_host = torch.zeros(1, dtype=torch.float32).pin_memory()
+        # with a shared host store only rank 0 writes the host-optimised layers' initial state
+        self._w0 = window if window >= 0 else min(2, L)
+        self._host_data_skipped = bool(shm_name) and rank != 0
         if init:
             self.init_params(seed, init_threads)
 
@@ -89,7 +92,10 @@ class StrongholdTrainer:
         mc = self.mc
         flat = np.empty(mc.params_per_layer(), np.float32)
         for i in range(mc.n_layers):
-            synth.init_layer_into(flat, seed, i, mc.n_layers, mc.hidden, threads)
+            if self._host_data_skipped and i >= self._w0:
+                flat[:] = 0.0  # ignored by the engine: rank 0 writes the shared copy
+            else:
+                synth.init_layer_into(flat, seed, i, mc.n_layers, mc.hidden, threads)
             self.engine.register(i, flat)
         res = np.empty(sum(mc.res_numels()), np.float32)
         synth.init_resident_into(res, seed, mc.vocab, mc.seq, mc.hidden, threads)

@@ -72,6 +72,9 @@ def test_cpu_hard_pushes_window_up():
     # (L - w) * 10 <= 4 L + 0.1 w  ->  w >= (10 L - 4 L) / 10.1
     assert r1["window"] == math.ceil((10 * L - 4 * L) / 10.1)
     assert r1["cpu_total_ms"] <= r1["gpu_step_ms"]
+    # utilisation target rho = 0.5: (L - w) * 10 <= 0.5 (4 L + 0.1 w)
+    r2 = sh.solve_window(**prof, cpu_hard=True, cpu_util_max=0.5)
+    assert r2["window"] == math.ceil((10 * L - 2 * L) / 10.05)
 
 
 def test_eq3_and_eq4_reports():
@@ -94,7 +97,8 @@ def test_random_heterogeneous_matches_bruteforce(seed):
                 t_opt_cpu=rng.uniform(0, 20, L), t_async=float(rng.uniform(0, 0.1)),
                 slot_bytes=rng.integers(1, 100, L), gstate_bytes=rng.integers(1, 60, L),
                 fixed_bytes=int(rng.integers(0, 50)), s_avail=int(rng.integers(100, 3000)),
-                duplex=bool(rng.integers(0, 2)), cpu_hard=bool(rng.integers(0, 2)))
+                duplex=bool(rng.integers(0, 2)), cpu_hard=bool(rng.integers(0, 2)),
+                cpu_util_max=float(rng.choice([1.0, 0.85, 0.5])))
     want = AO.solve(**{k: (list(v) if isinstance(v, np.ndarray) else v) for k, v in prof.items()})
     if want is None:
         with pytest.raises(sh.ShError):
