@@ -201,7 +201,8 @@ struct Job {
 struct ShmCtl {
   std::atomic<int64_t> magic;
   std::atomic<int64_t> created;    // rank 0 finished creating the layer segments
-  std::atomic<int64_t> bar[4];     // monotonic barrier counters
+  std::atomic<int64_t> bar[6];     // monotonic barrier counters
+  std::atomic<int64_t> window;     // rank 0's autotuned window (every rank must use the same one)
   std::atomic<int64_t> cnt[1];     // [2L]: cnt[x] slice updates completed (W per step);
                                    //       cnt[L+x] offloads landed (W per step)
 };
@@ -262,7 +263,7 @@ struct sh_ctx {
   ShmCtl* ctl = nullptr;
   size_t ctl_bytes = 0;
   std::vector<int64_t> slo, shi;
-  int64_t bar_calls[4] = {0, 0, 0, 0};
+  int64_t bar_calls[6] = {0, 0, 0, 0, 0, 0};
   std::vector<float*> h_master, h_m, h_v;
   std::vector<uint16_t*> h_shadow;
   std::vector<float*> landing;
@@ -1920,8 +1921,15 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   sh_status st = sh_solve_window(&p, &rep);
   if (st != SH_OK) return st;
   c->autotune_pending = false;
-  if (wout) *wout = rep.window;
-  if (rep.window != c->w) return sh_set_window(c, rep.window);
+  int32_t w = rep.window;
+  if (c->shared) {  // one shared host store: the whole job must switch to the same window
+    if (c->rank == 0) c->ctl->window.store(w);
+    if (!shm_barrier(c, 4, "autotuned window agreement")) return check_failed(c);
+    w = (int32_t)c->ctl->window.load();
+    if (!shm_barrier(c, 5, "autotuned window read")) return check_failed(c);
+  }
+  if (wout) *wout = w;
+  if (w != c->w) return sh_set_window(c, w);
   return SH_OK;
 }
 

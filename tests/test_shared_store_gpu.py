@@ -24,8 +24,8 @@ def _rank(rank, world, name, window, q):
     os.environ["SH_WAIT_TIMEOUT_S"] = "120"
     mc = T.ModelConfig(TINY["L"], TINY["h"], TINY["nh"], TINY["s"], TINY["V"])
     tr = T.StrongholdTrainer(mc, batch=TINY["b"], window=window, precision=sh.SH_BF16_MIXED,
-                             world_size=world, rank=rank, shm_name=name, cpu_threads=2,
-                             flags=sh.SH_FLAG_TEST_NO_COLLECTIVE)
+                             world_size=world, rank=rank, shm_name=name, cpu_threads=2, warmup_steps=2,
+                             flags=sh.SH_FLAG_TEST_NO_COLLECTIVE | sh.SH_FLAG_CPU_HARD)
     for t in range(STEPS):
         tr.set_tokens(synth.tokens(t, TINY["b"], TINY["s"], TINY["V"]))
         tr.step_device()
@@ -33,12 +33,13 @@ def _rank(rank, world, name, window, q):
     stats = tr.engine.stats()
     tr.close()
     q.put((rank, {k: [[a.tobytes() for a in u] if isinstance(u, list) else u.tobytes() for u in v]
-                  for k, v in st.items()}, stats["d2h_bytes"]))
+                  for k, v in st.items()}, stats["d2h_bytes"], stats["window"]))
 
 
-@pytest.mark.parametrize("window", [0, 1, 3])
+@pytest.mark.parametrize("window", [0, 1, 3, -1])
 def test_shared_store_two_ranks_bitwise(window):
-    ref, _, _ = engine_run(TINY, STEPS, window, sh.SH_BF16_MIXED)
+    # window -1: both ranks autotune after 2 warm-up steps; rank 0's choice must be adopted by all
+    ref, _, _ = engine_run(TINY, STEPS, window if window >= 0 else TINY["L"], sh.SH_BF16_MIXED)
     want = engine_state(ref)
     ref_d2h = ref.engine.stats()["d2h_bytes"]
     ref.close()
@@ -54,8 +55,10 @@ def test_shared_store_two_ranks_bitwise(window):
         p.join(timeout=60)
         assert p.exitcode == 0
     total_d2h = 0
-    for rank, state, d2h in res:
+    for rank, state, d2h, w in res:
         assert state == want, f"rank {rank} differs from the single-process run"
         total_d2h += d2h
-    assert total_d2h == ref_d2h  # the two ranks together offload each host layer exactly once
+    assert res[0][3] == res[1][3]  # same window on every rank
+    if window >= 0:
+        assert total_d2h == ref_d2h  # the two ranks together offload each host layer exactly once
     assert not any(f.startswith(name) for f in os.listdir("/dev/shm"))  # names removed after mapping
