@@ -248,6 +248,12 @@ sh_status sh_backward_layer(sh_ctx* ctx, int32_t layer, int32_t phase, void** de
  * are zeroed at the first forward hook of every step. */
 sh_status sh_resident(sh_ctx* ctx, void** dev_params, float** dev_grads);
 
+/* FP-only pass (NEXT-4: streaming inference of a model larger than HBM, e.g. the teacher of
+ * knowledge distillation): call after sh_forward_layer(L-1, SH_POST) instead of
+ * the backward hooks.  Nothing is updated, the step counter does not advance and every layer copy
+ * in the ring stays valid for the next pass (whose prefetches reuse them). */
+sh_status sh_forward_only_end(sh_ctx* ctx);
+
 /* Learning rate for the steps whose backward starts after this call. */
 sh_status sh_set_lr(sh_ctx* ctx, double lr);
 

@@ -60,6 +60,8 @@ int32_t gpt_layer_forward(gpt_ctx* ctx, int32_t layer, void* const* params);
  * residual-gradient buffer, res_grads[2..3] (LN_f) and the head part of res_grads[0] (=). */
 int32_t gpt_head_forward_backward(gpt_ctx* ctx, const int32_t* d_tokens, void* const* res_params,
                                   float* const* res_grads, float* d_loss);
+/* Forward-only head (inference): loss = mean CE(LN_f(x_L) wte^T, targets) -> *d_loss. */
+int32_t gpt_head_forward(gpt_ctx* ctx, const int32_t* d_tokens, void* const* res_params, float* d_loss);
 /* Recompute block_l forward from x_l, then backward: fp32 weight grads written into grads[],
  * the residual gradient is propagated in place (dL/dx_{l+1} -> dL/dx_l). */
 int32_t gpt_layer_backward(gpt_ctx* ctx, int32_t layer, void* const* params, float* const* grads);

@@ -293,6 +293,7 @@ struct sh_ctx {
   int last_layer = -1;
   int last_hook = SH_POST;
   int64_t step = 0;
+  int64_t fwd_passes = 0;
   bool registered_all = false;
   std::vector<uint8_t> reg_done;
   bool res_reg = false;
@@ -1731,6 +1732,26 @@ sh_status sh_resident(sh_ctx* c, void** dev_params, float** dev_grads) {
     if (dev_params) dev_params[k] = static_cast<char*>(c->res_compute) + (int64_t)c->cb * c->res.offset[k];
     if (dev_grads) dev_grads[k] = c->res_grad + c->res.offset[k];
   }
+  return SH_OK;
+}
+
+sh_status sh_forward_only_end(sh_ctx* c) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  if (!(c->phase == sh_ctx::FP && c->last_layer == c->L - 1 && c->last_hook == SH_POST)) {
+    set_error("sh_forward_only_end: the forward of layer L-1 must be the last hook");
+    return SH_ERR_STATE;
+  }
+  // nothing was updated: every copy in the ring stays valid for the next pass; the step counter
+  // (Adam's t) does not advance.  Pending profiling of this pass is dropped.
+  ProfSet& P = c->prof[c->step & 1];
+  if (P.active && P.step == c->step) P.active = false;
+  c->phase = sh_ctx::IDLE;
+  c->last_layer = -1;
+  c->last_hook = SH_POST;
+  c->fwd_passes++;
   return SH_OK;
 }
 

@@ -698,7 +698,7 @@ int layer_bwd_impl(gpt_ctx* c, int l, void* const* P, float* const* G) {
 }
 
 template <class T>
-int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float* d_loss) {
+int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float* d_loss, bool backward = true) {
   const int N = c->N, h = c->h, V = c->V, S = c->S;
   const cudaDataType_t dt = c->dt;
   const float* xL = c->x + (int64_t)c->L * c->maxN * h;
@@ -707,6 +707,10 @@ int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float
   CB(rm_gemm(c, false, true, N, V, h, 1.f, c->lnf, dt, R[0], dt, 0.f, c->logits, CUDA_R_32F));
   (g_launches++, 0), ce_fwd_bwd<T><<<N, 512, 0, c->st>>>(c->logits, tok, S, V, 1.0f / N, c->row_loss, (T*)c->dlogits);
   (g_launches++, 0), mean_fixed<<<1, 512, 0, c->st>>>(c->row_loss, N, 1.0f / N, d_loss);
+  if (!backward) {
+    CK(cudaGetLastError());
+    return 0;
+  }
   CB(rm_gemm(c, false, false, N, h, V, 1.f, c->dlogits, dt, R[0], dt, 0.f, c->dln, CUDA_R_32F));
   CK(cudaMemsetAsync(c->dres, 0, sizeof(float) * (size_t)N * h, c->st));
   (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xL, c->lnf_m, c->lnf_r, (const T*)R[2], c->dres,
@@ -864,6 +868,16 @@ int32_t gpt_head_forward_backward(gpt_ctx* c, const int32_t* tok, void* const* R
     return -1;
   }
   return c->bf16 ? head_impl<bf16>(c, tok, R, G, d_loss) : head_impl<float>(c, tok, R, G, d_loss);
+}
+
+int32_t gpt_head_forward(gpt_ctx* c, const int32_t* tok, void* const* R, float* d_loss) {
+  g_err.clear();
+  if (!c || !tok || !R || !d_loss || c->B == 0) {
+    seterr("gpt_head_forward: bad arguments");
+    return -1;
+  }
+  return c->bf16 ? head_impl<bf16>(c, tok, R, nullptr, d_loss, false)
+                 : head_impl<float>(c, tok, R, nullptr, d_loss, false);
 }
 
 int32_t gpt_layer_backward(gpt_ctx* c, int32_t l, void* const* P, float* const* G) {

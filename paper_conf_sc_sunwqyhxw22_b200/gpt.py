@@ -10,7 +10,7 @@ from .sh import LIBDIR
 EXPORTS = ("gpt_create", "gpt_destroy", "gpt_last_error", "gpt_workspace_bytes", "gpt_embed_forward",
            "gpt_layer_forward", "gpt_head_forward_backward", "gpt_layer_backward", "gpt_embed_backward",
            "gpt_checkpoint", "gpt_kernel_launches", "gpt_layer_forward_qkv", "gpt_layer_forward_out",
-           "gpt_layer_backward_mlp", "gpt_layer_backward_qkv", "gpt_buffer")
+           "gpt_layer_backward_mlp", "gpt_layer_backward_qkv", "gpt_buffer", "gpt_head_forward")
 
 
 class GptConfig(C.Structure):
@@ -35,7 +35,7 @@ def lib() -> C.CDLL:
                "gpt_head_forward_backward": [vp, vp, vp, vp, vp], "gpt_layer_backward": [vp, i32, vp, vp],
                "gpt_embed_backward": [vp, vp, vp], "gpt_layer_forward_qkv": [vp, i32, vp],
                "gpt_layer_forward_out": [vp, i32, vp, i32], "gpt_layer_backward_mlp": [vp, i32, vp, vp],
-               "gpt_layer_backward_qkv": [vp, i32, vp, vp]}
+               "gpt_layer_backward_qkv": [vp, i32, vp, vp], "gpt_head_forward": [vp, vp, vp, vp]}
         for n, a in sig.items():
             getattr(L, n).argtypes = a
             getattr(L, n).restype = C.c_int32
@@ -80,6 +80,9 @@ class GPT:
 
     def head(self, tok_ptr: int, res_params, res_grads, loss_ptr: int):
         _check(self._L.gpt_head_forward_backward(self.h, tok_ptr, res_params, res_grads, loss_ptr))
+
+    def head_forward(self, tok_ptr: int, res_params, loss_ptr: int):
+        _check(self._L.gpt_head_forward(self.h, tok_ptr, res_params, loss_ptr))
 
     def layer_backward(self, layer: int, params, grads):
         _check(self._L.gpt_layer_backward(self.h, layer, params, grads))

@@ -29,7 +29,7 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_autotune_window", "sh_set_window", "sh_get_profile", "sh_read_layer", "sh_stats",
            "sh_last_error", "sh_abi_version", "sh_nccl_get_unique_id", "sh_adam_scalars_for",
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
-           "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace")
+           "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end")
 
 
 class ShError(RuntimeError):
@@ -127,6 +127,7 @@ def lib() -> C.CDLL:
             "sh_op_cast_bf16_gpu": [vp, vp, i64, vp], "sh_op_cast_bf16_cpu": [vp, vp, i64],
             "sh_op_sumsq_gpu": [vp, i64, vp, vp],
             "sh_get_trace": [vp, vp, i32, C.POINTER(i32)],
+            "sh_forward_only_end": [vp],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -347,6 +348,9 @@ class Engine:
 
     def backward_post(self, i: int):
         check(self._L.sh_backward_layer(self.h, i, SH_POST, None, None))
+
+    def forward_only_end(self):
+        check(self._L.sh_forward_only_end(self.h))
 
     def resident(self):
         return self._rp, self._rg

@@ -150,6 +150,31 @@ class StrongholdTrainer:
             g.embed_backward(tok, rg)
             return e.step(want_norm=want_norm)
 
+    def forward_only(self, batch: int | None = None) -> None:
+        """FP-only pass (streaming inference / KD teacher) over self.tok_dev:
+        loss -> self.loss_dev; no backward, no update (NEXT-4)."""
+        e, g = self.engine, self.gpt
+        B = batch or self.batch
+        tok = self.tok_dev.data_ptr()
+        rp, _ = e.resident()
+        fa = self.flash
+        if fa is not None:
+            fa.set_batch(B)
+        with torch.cuda.stream(self.stream):
+            for i in range(self.mc.n_layers):
+                P = e.forward_pre(i)
+                if i == 0:
+                    g.embed_forward(tok, B, rp)
+                if fa is None:
+                    g.layer_forward(i, P)
+                else:
+                    g.forward_qkv(i, P)
+                    fa.forward()
+                    g.forward_out(i, P, True)
+                e.forward_post(i)
+            g.head_forward(tok, rp, self.loss_dev.data_ptr())
+            e.forward_only_end()
+
     def step(self, tokens_host: torch.Tensor, want_norm=False) -> float:
         """End-to-end public step: pinned host tokens -> device, train, loss -> host."""
         with torch.cuda.stream(self.stream):

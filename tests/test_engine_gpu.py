@@ -182,3 +182,34 @@ def test_protocol_errors():
         assert np.isfinite(tr.loss())
     finally:
         tr.close()
+
+
+@pytest.mark.parametrize("precision", [sh.SH_FP32, sh.SH_BF16_MIXED])
+def test_forward_only_passes(precision):
+    """NEXT-4 FP-only streaming (KD teacher inference): the loss of an FP-only
+    pass equals the training step's loss at the same parameters bitwise, for every window; passes
+    update nothing; a training step after FP-only passes is unaffected by them."""
+    L = TINY["L"]
+    tok0 = synth.tokens(0, TINY["b"], TINY["s"], TINY["V"])
+    ref, ref_losses, _ = engine_run(TINY, 2, L, precision)
+    ref_state = engine_state(ref)
+    ref.close()
+    for w in (0, 1, L):
+        from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
+        mc = T.ModelConfig(L, TINY["h"], TINY["nh"], TINY["s"], TINY["V"])
+        tr = T.StrongholdTrainer(mc, batch=TINY["b"], window=w, precision=precision)
+        try:
+            tr.set_tokens(tok0)
+            losses = []
+            for _ in range(3):
+                tr.forward_only()
+                losses.append(np.float32(tr.loss()).tobytes())
+            assert len(set(losses)) == 1 and losses[0] == np.float32(ref_losses[0]).tobytes(), w
+            assert tr.engine.stats()["step"] == 0
+            for t in range(2):  # training continues exactly as if the passes never happened
+                tr.set_tokens(synth.tokens(t, TINY["b"], TINY["s"], TINY["V"]))
+                tr.step_device(want_norm=True)
+            ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+            assert ok, (w, what)
+        finally:
+            tr.close()
