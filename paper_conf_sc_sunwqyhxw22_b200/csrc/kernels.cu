@@ -21,6 +21,7 @@
 
 #include <atomic>
 #include <cstdint>
+#include <cstdlib>
 
 #include "sh_internal.hpp"
 
@@ -61,10 +62,11 @@ __device__ __forceinline__ void adam_elem(float& p, float& m, float& v, float g,
   p = __fmaf_rn(s.nss, __fdiv_rn(m, d), pp);
 }
 
-// K2: one work item = kK2Chunk consecutive elements of one entry.  Thread t of the block
-// handles elements base + u*1024 + 4t .. +3 for u in {0,1}: every float4 load/store of a
-// warp touches 512 contiguous bytes.  8 independent 16-B loads in flight per thread.
-template <bool kBf16Out>
+// K2: one work item = 1024*U consecutive elements of one entry.  Thread t of the block handles
+// elements base + u*1024 + 4t .. +3 for u in [0, U): every float4 load/store of a warp touches 512
+// contiguous bytes; 4U independent 16-B loads in flight per thread (U = 2 by default, tuned on
+// B200 with tools/bench_kernels.py).
+template <bool kBf16Out, int U>
 __global__ void __launch_bounds__(256) k2_adamw_kernel(const __grid_constant__ K2Args a) {
   const AdamS s{a.sc.beta1, a.sc.beta2, a.sc.omb1, a.sc.omb2, a.sc.eps, -a.sc.step_size,
                 a.sc.sqrt_bc2, a.sc.decay};
@@ -75,29 +77,38 @@ __global__ void __launch_bounds__(256) k2_adamw_kernel(const __grid_constant__ K
   for (int64_t item = blockIdx.x; item < n_items; item += gridDim.x) {
     while (item >= a.item_start[e + 1]) ++e;  // items are visited in increasing order
     const K2Entry& E = a.e[e];
-    const int64_t base = (item - a.item_start[e]) * kK2Chunk;
+    const int64_t base = (item - a.item_start[e]) * (1024 * U);
+    float4 p[U], m[U], v[U], g[U];
 #pragma unroll
-    for (int u = 0; u < 2; ++u) {
+    for (int u = 0; u < U; ++u) {
+      const int64_t i = base + u * 1024 + 4 * threadIdx.x;
+      if (i < E.n) {
+        p[u] = ld_rw(E.p + i);
+        m[u] = ld_rw(E.m + i);
+        v[u] = ld_rw(E.v + i);
+        g[u] = ld_stream(E.g + i);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
       const int64_t i = base + u * 1024 + 4 * threadIdx.x;
       if (i >= E.n) continue;
-      float4 p = ld_rw(E.p + i), m = ld_rw(E.m + i), v = ld_rw(E.v + i);
-      const float4 g = ld_stream(E.g + i);
       const bool wd = i < E.n_decay;  // n_decay is a multiple of 8: uniform per float4
-      adam_elem(p.x, m.x, v.x, g.x, s, wd, use_coef, coef);
-      adam_elem(p.y, m.y, v.y, g.y, s, wd, use_coef, coef);
-      adam_elem(p.z, m.z, v.z, g.z, s, wd, use_coef, coef);
-      adam_elem(p.w, m.w, v.w, g.w, s, wd, use_coef, coef);
-      st_f4(E.p + i, p);
-      st_f4(E.m + i, m);
-      st_f4(E.v + i, v);
+      adam_elem(p[u].x, m[u].x, v[u].x, g[u].x, s, wd, use_coef, coef);
+      adam_elem(p[u].y, m[u].y, v[u].y, g[u].y, s, wd, use_coef, coef);
+      adam_elem(p[u].z, m[u].z, v[u].z, g[u].z, s, wd, use_coef, coef);
+      adam_elem(p[u].w, m[u].w, v[u].w, g[u].w, s, wd, use_coef, coef);
+      st_f4(E.p + i, p[u]);
+      st_f4(E.m + i, m[u]);
+      st_f4(E.v + i, v[u]);
       if (E.out != nullptr) {
         if constexpr (kBf16Out) {
           uint2 o;
-          o.x = rne_bf16_bits(p.x) | (rne_bf16_bits(p.y) << 16);
-          o.y = rne_bf16_bits(p.z) | (rne_bf16_bits(p.w) << 16);
+          o.x = rne_bf16_bits(p[u].x) | (rne_bf16_bits(p[u].y) << 16);
+          o.y = rne_bf16_bits(p[u].z) | (rne_bf16_bits(p[u].w) << 16);
           *reinterpret_cast<uint2*>(static_cast<uint16_t*>(E.out) + i) = o;
         } else {
-          st_f4(static_cast<float*>(E.out) + i, p);
+          st_f4(static_cast<float*>(E.out) + i, p[u]);
         }
       }
     }
@@ -224,22 +235,33 @@ int sm_count() {
   return g_sm_count;
 }
 
+namespace {
+int env_int(const char* name, int dflt) {
+  const char* e = getenv(name);
+  return e ? atoi(e) : dflt;
+}
+}  // namespace
+
 cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
+  static const int U = env_int("SH_K2_U", 2) == 4 ? 4 : 2;
+  static const int bps = env_int("SH_K2_BPS", 4);
+  const int64_t chunk = 1024 * U;
   a.item_start[0] = 0;
-  for (int i = 0; i < a.n_entries; ++i)
-    a.item_start[i + 1] = a.item_start[i] + (a.e[i].n + kK2Chunk - 1) / kK2Chunk;
+  for (int i = 0; i < a.n_entries; ++i) a.item_start[i + 1] = a.item_start[i] + (a.e[i].n + chunk - 1) / chunk;
   const int64_t items = a.item_start[a.n_entries];
   if (items == 0) return cudaSuccess;
-  // Persistent-style grid: 4 resident 256-thread blocks per SM (8 KB of loads in flight per
-  // block-iteration), never more blocks than items.
-  const int64_t cap = (int64_t)sm_count() * 4;
+  // Persistent-style grid: bps resident 256-thread blocks per SM, never more blocks than items.
+  const int64_t cap = (int64_t)sm_count() * (bps > 0 ? bps : 4);
   const int grid = (int)(items < cap ? items : cap);
   if (grid_out) *grid_out = grid;
   launch_counter()++;
-  if (a.out_bf16)
-    k2_adamw_kernel<true><<<grid, 256, 0, st>>>(a);
-  else
-    k2_adamw_kernel<false><<<grid, 256, 0, st>>>(a);
+  if (U == 4) {
+    if (a.out_bf16) k2_adamw_kernel<true, 4><<<grid, 256, 0, st>>>(a);
+    else k2_adamw_kernel<false, 4><<<grid, 256, 0, st>>>(a);
+  } else {
+    if (a.out_bf16) k2_adamw_kernel<true, 2><<<grid, 256, 0, st>>>(a);
+    else k2_adamw_kernel<false, 2><<<grid, 256, 0, st>>>(a);
+  }
   return cudaGetLastError();
 }
 

@@ -49,7 +49,6 @@ struct K2Entry {
   int64_t n_decay;  // multiple of 8
 };
 constexpr int kK2MaxEntries = 40;
-constexpr int kK2Chunk = 2048;  // elements per work item (256 threads x 2 x float4)
 struct K2Args {
   sh_adam_scalars sc;
   const float* coef;  // null: no clipping

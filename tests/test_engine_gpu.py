@@ -213,3 +213,51 @@ def test_forward_only_passes(precision):
             assert ok, (w, what)
         finally:
             tr.close()
+
+
+def test_autotune_mid_run_bitwise_and_trace():
+    """window = -1: w0 = min(2, L) for the warm-up steps, then sh_autotune_window applies the solver
+    on the measured profile (P1/P2 + eq. 3 with SH_FLAG_CPU_HARD); results stay bitwise equal to the
+    resident run, and the step trace / overlap stats of the profiled steps are consistent."""
+    L = TINY["L"]
+    ref, _, _ = engine_run(TINY, 4, L, sh.SH_BF16_MIXED)
+    ref_state = engine_state(ref)
+    ref.close()
+    from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
+    mc = T.ModelConfig(L, TINY["h"], TINY["nh"], TINY["s"], TINY["V"])
+    tr = T.StrongholdTrainer(mc, batch=TINY["b"], window=-1, precision=sh.SH_BF16_MIXED, warmup_steps=2,
+                             flags=sh.SH_FLAG_CPU_HARD | sh.SH_FLAG_PROFILE)
+    try:
+        for t in range(4):
+            tr.set_tokens(synth.tokens(t, TINY["b"], TINY["s"], TINY["V"]))
+            tr.step_device(want_norm=True)
+        ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+        assert ok, what
+        st = tr.engine.stats()
+        assert 0 <= st["window"] <= L and st["profiled_steps"] >= 3
+        prof = tr.engine.profile()
+        assert all(x > 0 for x in prof["t_fp"]) and all(x > 0 for x in prof["t_bp"])
+        trace = tr.engine.trace()
+        kinds = {e["kind"] for e in trace}
+        assert {"fp", "bp", "k2_adamw"} <= kinds
+        fp = sorted((e["layer"], e["start_ms"], e["end_ms"]) for e in trace if e["kind"] == "fp")
+        assert [x[0] for x in fp] == list(range(L))
+        assert all(a[2] <= b[1] + 1e-3 for a, b in zip(fp, fp[1:]))  # FP layers run in order
+        assert all(e["end_ms"] >= e["start_ms"] >= 0 for e in trace)
+        if st["window"] < L:
+            assert 0.0 <= st["h2d_overlap_frac"] <= 1.0 and 0.0 <= st["d2h_overlap_frac"] <= 1.0
+    finally:
+        tr.close()
+
+
+def test_read_grad_after_landing_ring_reuse_is_an_error():
+    tr, _, _ = engine_run(TINY, 1, 0, sh.SH_FP32, grad_ring_depth=1)
+    try:
+        # with a 1-deep landing ring only the last offloaded layer (layer 0 in BP order) survives
+        g = tr.engine.read_layer(0, sh.SH_READ_GRAD)
+        assert np.isfinite(g).all() and np.abs(g).max() > 0
+        with pytest.raises(sh.ShError) as e:
+            tr.engine.read_layer(TINY["L"] - 1, sh.SH_READ_GRAD)
+        assert e.value.status == sh.SH_ERR_STATE
+    finally:
+        tr.close()
