@@ -177,6 +177,10 @@ def blas_threads():
 def run_reference(args, cfgname):
     L, h, nh, s, V, b, w, desc = CONFIGS[cfgname]
     b = args.batch or b
+    if args.layers:
+        L = args.layers
+    if L == 0:  # same depth rule as the CUDA arm (L_max of this host's RAM)
+        L = c4_layers(h, args.grad_ring or 4, ranks_sharing=int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
@@ -191,7 +195,8 @@ def run_reference(args, cfgname):
             "unit": "samples/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": per * 1e3 * b, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic",
-            "config": {"workload": cfgname, "description": desc, "batch_per_gpu": b, "seq": s},
+            "config": {"workload": cfgname, "description": desc, "layers": L, "hidden": h, "heads": nh,
+                       "batch_per_gpu": b, "seq": s, "vocab": V},
             "cpu_baseline": {"value": val, "unit": "samples/s", "cores": blas_threads(), "kind": "oracle",
                              "sample": "per step: one block fwd+bwd+AdamW and the head at batch 1 (numpy fp64), "
                                        f"extrapolated x{L} layers"},
@@ -216,7 +221,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--fetch-fp32", type=int, default=-1, help="1: no host bf16 shadow, fp32 over the link")
     ap.add_argument("--init-threads", type=int, default=16)
-    ap.add_argument("--layers", type=int, default=0, help="c4: override L_max(host RAM)")
+    ap.add_argument("--layers", type=int, default=0, help="override the depth (c4: L_max(host RAM))")
     ap.add_argument("--trace-out", default="", help="write a Chrome trace of the last profiled step")
     ap.add_argument("--attention", default="auto", choices=["auto", "flash", "cublas"],
                     help="attention core of the GPT driver (outside the hot path)")
@@ -258,6 +263,8 @@ def main():
         flag = torch.tensor([1 if shm_free() > 0.8 * mem_available() else 0], dtype=torch.int64, device="cuda")
         dist.broadcast(flag, 0)
         use_shm = bool(flag.item())
+    if args.layers and L != 0:
+        L = args.layers  # depth override (e.g. the resident-fit comparison model)
     if L == 0:
         if args.layers:
             L = args.layers
