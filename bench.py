@@ -72,6 +72,7 @@ def c4_layers(h: int, ring: int, w0: int = 2, margin_gb: float = 8.0, ranks_shar
     per_layer = (12 * n_pad + (1 << 21) - 1) // (1 << 21) * (1 << 21)
     budget = avail - int(margin_gb * (1 << 30)) - ranks_sharing * ring * 4 * n_pad
     return max(w0 + 1, budget // per_layer + w0)
+METRIC = "samples/s at max trainable size per B200; host-link GB/s vs peak"
 PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
 PROBE_D2H_GBS = 57.01
 
@@ -191,7 +192,7 @@ def run_reference(args, cfgname):
             times.append(per_sample)
     per = float(np.mean(times))
     val = 1.0 / per
-    line = {"impl": "reference", "metric": "samples/s (CPU oracle, extrapolated)", "value": val,
+    line = {"impl": "reference", "metric": METRIC, "value": val,
             "unit": "samples/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": per * 1e3 * b, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic",
@@ -395,7 +396,7 @@ def main():
     flops_tok = mc.flops_per_token()
     tokens_s = samples * s
     line = {
-        "metric": "samples/s at max trainable size per B200; host-link GB/s vs peak",
+        "metric": METRIC,
         "value": samples, "unit": "samples/s", "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "bf16" if prec == sh.SH_BF16_MIXED else "f32", "data": "synthetic",
