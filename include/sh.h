@@ -104,6 +104,10 @@ typedef struct {
 #define SH_FLAG_TEST_NO_COLLECTIVE (1ull << 6) /* test: world_size > 1 without NCCL (all ranks feed identical
                                                   data, so the average is the local gradient); exercises
                                                   the shared store / slicing with several processes */
+#define SH_FLAG_SLICE_FETCH (1ull << 7) /* NEXT-1 (data parallel + shm_name): each rank H2Ds only its 1/W
+                                           slice of a fetched layer; an in-place ncclAllGather over NVLink
+                                           assembles the layer in every rank's slot (PCIe bytes and host
+                                           DRAM reads per rank / W).  Needs NCCL >= 2.18 (ncclCommSplit). */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

@@ -94,6 +94,8 @@ struct Nccl {
   ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
                             cudaStream_t) = nullptr;
   ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*CommSplit)(ncclComm_t, int, int, ncclComm_t*, ncclConfig_t*) = nullptr;
   const char* (*GetErrorString)(ncclResult_t) = nullptr;
   bool load() {
     if (h) return true;
@@ -108,6 +110,8 @@ struct Nccl {
     CommInitRank = (decltype(CommInitRank))dlsym(h, "ncclCommInitRank");
     AllReduce = (decltype(AllReduce))dlsym(h, "ncclAllReduce");
     CommDestroy = (decltype(CommDestroy))dlsym(h, "ncclCommDestroy");
+    AllGather = (decltype(AllGather))dlsym(h, "ncclAllGather");
+    CommSplit = (decltype(CommSplit))dlsym(h, "ncclCommSplit");
     GetErrorString = (decltype(GetErrorString))dlsym(h, "ncclGetErrorString");
     return GetUniqueId && CommInitRank && AllReduce && CommDestroy && GetErrorString;
   }
@@ -229,6 +233,9 @@ struct sh_ctx {
   // ---- streams
   cudaStream_t cs = nullptr, h2d = nullptr, d2h = nullptr, stage = nullptr, comm = nullptr;
   ncclComm_t nccl = nullptr;
+  ncclComm_t nccl_fetch = nullptr;  // NEXT-1: collectives issued by the H2D issuer thread
+  bool slice_fetch = false;
+  int64_t cs_max = 0;               // equal slice length (elements) used by the all-gather
 
   // ---- device memory
   char* ring = nullptr;
@@ -755,7 +762,8 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
         const double ms = ev_ms(P.c2g0[ph][i], P.c2g1[ph][i]);
         c->p_c2g[i] = ms;
         c->h2d_busy += ms;
-        c->h2d_prof_bytes += (int64_t)((c->bf16 && !c->shadow) ? 4 : c->cb) * c->lay[i].n_pad;
+        c->h2d_prof_bytes += (int64_t)((c->bf16 && !c->shadow) ? 4 : c->cb) *
+                             (c->slice_fetch && !c->no_collective ? c->shi[i] - c->slo[i] : c->lay[i].n_pad);
       }
     if (P.rec_g2c[i]) {
       const double ms = ev_ms(P.g2c0[i], P.g2c1[i]);
@@ -840,12 +848,18 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   // master into the slot's (idle) grad half and K1 casts it into the param half on the H2D stream
   const bool cast = c->bf16 && !c->shadow;
   const void* src = c->shadow ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];
-  const int64_t bytes = (cast ? 4 : (int64_t)c->cb) * n;
+  const int64_t eb = cast ? 4 : (int64_t)c->cb;  // fetched bytes per element
+  const int64_t bytes = eb * n;
+  // NEXT-1 slice fetch: this rank's slice over PCIe, the rest over NVLink (in-place all-gather)
+  const bool slice = c->slice_fetch;
+  const int64_t slo = c->slo[y], shi = c->shi[y];
+  const int64_t cs = align_up((n + c->W - 1) / c->W, kPad);
   cudaEvent_t pf = c->ev_param_free[s];
   cudaEvent_t gf = c->ev_grad_free[s];
   float* stage_buf = c->slot_grad(s);
   const int64_t gf_gen = c->gradfree_gen[s];
-  c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, gf, stage_buf, gf_gen, s, n] {
+  c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, gf, stage_buf, gf_gen, s, n, eb, slice,
+                slo, shi, cs] {
     double waited = 0;
     if (!state_wait(c, [&] { return ready_at_least(c, y, need); }, "CPU Adam of a layer to prefetch", &waited)) {
       c->arrive_pub[y].store(kInf);
@@ -867,15 +881,31 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       CKA(c, cudaStreamWaitEvent(c->h2d, gf, 0));
     }
     if (poison) CKA(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->h2d));
+    char* buf = cast ? reinterpret_cast<char*>(stage_buf) : dst;
+    const char* hsrc = static_cast<const char*>(src);
     if (P) CKA(c, cudaEventRecord(P->c2g0[ph][y], c->h2d));
-    CKA(c, cudaMemcpyAsync(cast ? (void*)stage_buf : dst, src, bytes, cudaMemcpyHostToDevice, c->h2d));
+    if (!slice) {
+      CKA(c, cudaMemcpyAsync(buf, src, bytes, cudaMemcpyHostToDevice, c->h2d));
+    } else if (shi > slo) {
+      CKA(c, cudaMemcpyAsync(buf + eb * slo, hsrc + eb * slo, eb * (shi - slo), cudaMemcpyHostToDevice, c->h2d));
+    }
     if (P) {
       CKA(c, cudaEventRecord(P->c2g1[ph][y], c->h2d));
       P->rec_c2g[ph][y] = 1;
     }
+    if (slice) {
+      if (!c->no_collective) {  // every rank holds slice r at offset r*cs: gather in place
+        const ncclResult_t r = g_nccl.AllGather(buf + eb * c->rank * cs, buf, (size_t)cs,
+                                                eb == 4 ? ncclFloat32 : ncclBfloat16, c->nccl_fetch, c->h2d);
+        if (r != ncclSuccess) async_fail(c, SH_ERR_NCCL, "ncclAllGather(fetch): %s", g_nccl.GetErrorString(r));
+      } else {  // test mode (one GPU): the other ranks' slices come over PCIe as well
+        if (slo > 0) CKA(c, cudaMemcpyAsync(buf, hsrc, eb * slo, cudaMemcpyHostToDevice, c->h2d));
+        if (n > shi) CKA(c, cudaMemcpyAsync(buf + eb * shi, hsrc + eb * shi, eb * (n - shi), cudaMemcpyHostToDevice, c->h2d));
+      }
+    }
     if (cast) CKA(c, kern::cast_bf16(stage_buf, reinterpret_cast<uint16_t*>(dst), n, c->h2d));
     CKA(c, cudaEventRecord(c->ev_arrive[y], c->h2d));
-    c->h2d_bytes += bytes;
+    c->h2d_bytes += slice && !c->no_collective ? eb * (shi - slo) : bytes;
     c->h2d_copies++;
     c->arrive_pub[y].store(gen);
     notify_state(c);
@@ -1260,8 +1290,12 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->max_pad = std::max(c->max_pad, c->lay[i].n_pad);
   }
   if (!make_layout(cfg->resident, &c->res)) return SH_ERR_INVALID;
-  c->slot_param_bytes = align_up((int64_t)c->cb * c->max_pad, 256);
-  c->slot_grad_bytes = align_up(4 * c->max_pad, 256);
+  // data parallel slices: equal length cs = ceil(n_pad / W) rounded to kPad (an in-place
+  // all-gather needs equal counts), so slots hold W * cs elements
+  c->cs_max = align_up((c->max_pad + W - 1) / W, kPad);
+  const int64_t slot_elems = W > 1 ? std::max(c->max_pad, (int64_t)W * c->cs_max) : c->max_pad;
+  c->slot_param_bytes = align_up((int64_t)c->cb * slot_elems, 256);
+  c->slot_grad_bytes = align_up(4 * slot_elems, 256);
   c->slot_bytes = c->slot_param_bytes + c->slot_grad_bytes;
   const int w0 = cfg->window >= 0 ? cfg->window : std::min(2, c->L);
   c->autotune_pending = cfg->window < 0;
@@ -1291,6 +1325,16 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     sh_status s = nccl_check(c.get(), g_nccl.CommInitRank(&c->nccl, W, id, cfg->rank), "ncclCommInitRank");
     if (s != SH_OK) return s;
   }
+  c->slice_fetch = W > 1 && (cfg->flags & SH_FLAG_SLICE_FETCH) && cfg->shm_name && cfg->shm_name[0];
+  if (c->slice_fetch && !c->no_collective) {
+    if (!g_nccl.AllGather || !g_nccl.CommSplit) {
+      set_error("sh_init: SH_FLAG_SLICE_FETCH needs ncclAllGather and ncclCommSplit");
+      return SH_ERR_UNSUPPORTED;
+    }
+    sh_status s = nccl_check(c.get(), g_nccl.CommSplit(c->nccl, 0, cfg->rank, &c->nccl_fetch, nullptr),
+                             "ncclCommSplit(fetch)");
+    if (s != SH_OK) return s;
+  }
 
   // ---- host store: per layer master | m | v | shadow, plus landing buffers, 2 MiB aligned
   c->n_threads = cfg->cpu_threads > 0 ? cfg->cpu_threads : (int)std::thread::hardware_concurrency();
@@ -1317,10 +1361,15 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->slo.assign(c->L, 0);
   c->shi.assign(c->L, 0);
   for (int x = 0; x < c->L; ++x) {
-    const int64_t units = c->lay[x].n_pad / kPad;
-    const int R = c->shared ? c->W : 1, r = c->shared ? c->rank : 0;
-    c->slo[x] = units * r / R * kPad;
-    c->shi[x] = units * (r + 1) / R * kPad;
+    const int64_t n = c->lay[x].n_pad;
+    if (c->shared) {
+      const int64_t cs = align_up((n + c->W - 1) / c->W, kPad);
+      c->slo[x] = std::min(n, (int64_t)c->rank * cs);
+      c->shi[x] = std::min(n, (int64_t)(c->rank + 1) * cs);
+    } else {
+      c->slo[x] = 0;
+      c->shi[x] = n;
+    }
   }
   if (c->shared) {
     // control block: rank 0 creates it, the others wait for it; then every layer segment
@@ -2090,6 +2139,7 @@ sh_status sh_destroy(sh_ctx* c) {
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
     if (s) cudaStreamSynchronize(s);
   if (c->cs) cudaStreamSynchronize(c->cs);
+  if (c->nccl_fetch) g_nccl.CommDestroy(c->nccl_fetch);
   if (c->nccl) g_nccl.CommDestroy(c->nccl);
   for (int x = 0; x < c->L; ++x) free_g(c, x);
   if (c->ring) cudaFree(c->ring);

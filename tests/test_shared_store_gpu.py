@@ -18,14 +18,14 @@ sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
 STEPS = 3
 
 
-def _rank(rank, world, name, window, q):
+def _rank(rank, world, name, window, q, extra_flags=0):
     import synth
     from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
     os.environ["SH_WAIT_TIMEOUT_S"] = "120"
     mc = T.ModelConfig(TINY["L"], TINY["h"], TINY["nh"], TINY["s"], TINY["V"])
     tr = T.StrongholdTrainer(mc, batch=TINY["b"], window=window, precision=sh.SH_BF16_MIXED,
                              world_size=world, rank=rank, shm_name=name, cpu_threads=2, warmup_steps=2,
-                             flags=sh.SH_FLAG_TEST_NO_COLLECTIVE | sh.SH_FLAG_CPU_HARD)
+                             flags=sh.SH_FLAG_TEST_NO_COLLECTIVE | sh.SH_FLAG_CPU_HARD | extra_flags)
     for t in range(STEPS):
         tr.set_tokens(synth.tokens(t, TINY["b"], TINY["s"], TINY["V"]))
         tr.step_device()
@@ -36,8 +36,8 @@ def _rank(rank, world, name, window, q):
                   for k, v in st.items()}, stats["d2h_bytes"], stats["window"]))
 
 
-@pytest.mark.parametrize("window", [0, 1, 3, -1])
-def test_shared_store_two_ranks_bitwise(window):
+@pytest.mark.parametrize("window,extra", [(0, 0), (1, 0), (3, 0), (-1, 0), (1, "slice"), (0, "slice32")])
+def test_shared_store_two_ranks_bitwise(window, extra):
     # window -1: both ranks autotune after 2 warm-up steps; rank 0's choice must be adopted by all
     ref, _, _ = engine_run(TINY, STEPS, window if window >= 0 else TINY["L"], sh.SH_BF16_MIXED)
     want = engine_state(ref)
@@ -47,7 +47,9 @@ def test_shared_store_two_ranks_bitwise(window):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     name = f"shtest_{uuid.uuid4().hex[:12]}"
-    procs = [ctx.Process(target=_rank, args=(r, 2, name, window, q)) for r in range(2)]
+    flags = {0: 0, "slice": sh.SH_FLAG_SLICE_FETCH,
+             "slice32": sh.SH_FLAG_SLICE_FETCH | sh.SH_FLAG_FETCH_FP32}[extra]
+    procs = [ctx.Process(target=_rank, args=(r, 2, name, window, q, flags)) for r in range(2)]
     for p in procs:
         p.start()
     res = [q.get(timeout=300) for _ in range(2)]
