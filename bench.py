@@ -224,6 +224,8 @@ def main():
     ap.add_argument("--init-threads", type=int, default=16)
     ap.add_argument("--layers", type=int, default=0, help="override the depth (c4: L_max(host RAM))")
     ap.add_argument("--trace-out", default="", help="write a Chrome trace of the last profiled step")
+    ap.add_argument("--slice-fetch", action="store_true",
+                    help="N>1: NEXT-1 slice H2D + NVLink all-gather (SH_FLAG_SLICE_FETCH)")
     ap.add_argument("--attention", default="auto", choices=["auto", "flash", "cublas"],
                     help="attention core of the GPT driver (outside the hot path)")
     ap.add_argument("--cpu-hard", type=int, default=-1, help="1: autotune with the eq. 3 CPU constraint")
@@ -296,7 +298,7 @@ def main():
     def run(window, e2e: bool):
         t_init = time.perf_counter()
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
-            (sh.SH_FLAG_CPU_HARD if cpu_hard else 0)
+            (sh.SH_FLAG_CPU_HARD if cpu_hard else 0) | (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
