@@ -64,7 +64,7 @@ __device__ __forceinline__ void adam_elem(float& p, float& m, float& v, float g,
 
 // K2: one work item = 1024*U consecutive elements of one entry.  Thread t of the block handles
 // elements base + u*1024 + 4t .. +3 for u in [0, U): every float4 load/store of a warp touches 512
-// contiguous bytes; 4U independent 16-B loads in flight per thread (U = 2 by default, tuned on
+// contiguous bytes; 4U independent 16-B loads in flight per thread (U = 4 by default, tuned on
 // B200 with tools/bench_kernels.py).
 template <bool kBf16Out, int U>
 __global__ void __launch_bounds__(256) k2_adamw_kernel(const __grid_constant__ K2Args a) {
@@ -243,7 +243,7 @@ int env_int(const char* name, int dflt) {
 }  // namespace
 
 cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
-  static const int U = env_int("SH_K2_U", 2) == 4 ? 4 : 2;
+  static const int U = env_int("SH_K2_U", 4) == 2 ? 2 : 4;  // U=4: 0.93 vs 0.89 of HBM peak (profiles/r01_kernels_microbench.txt)
   static const int bps = env_int("SH_K2_BPS", 4);
   const int64_t chunk = 1024 * U;
   a.item_start[0] = 0;
