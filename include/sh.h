@@ -108,6 +108,8 @@ typedef struct {
                                            slice of a fetched layer; an in-place ncclAllGather over NVLink
                                            assembles the layer in every rank's slot (PCIe bytes and host
                                            DRAM reads per rank / W).  Needs NCCL >= 2.18 (ncclCommSplit). */
+#define SH_FLAG_DELAY_INJECT (1ull << 8) /* test: random 0-2 ms sleeps in the copy issuers and CPU Adam tasks
+                                            (ordering-race hunting; results must stay bitwise identical) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

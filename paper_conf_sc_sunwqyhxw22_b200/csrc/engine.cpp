@@ -81,6 +81,18 @@ double now_ms() {
 
 int64_t align_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
+// SH_FLAG_DELAY_INJECT: random 0..2 ms host sleeps in the issuers and CPU Adam tasks and random
+// GPU spin kernels are NOT used; the host sleeps perturb every cross-thread ordering the engine
+// relies on.  Thread-local xorshift, seeded per thread.
+void maybe_delay(uint64_t flags) {
+  if (!(flags & SH_FLAG_DELAY_INJECT)) return;
+  static thread_local uint64_t x = 0x9E3779B97F4A7C15ull ^ (uint64_t)pthread_self();
+  x ^= x << 13;
+  x ^= x >> 7;
+  x ^= x << 17;
+  if ((x & 3) == 0) usleep((useconds_t)(x % 2000));
+}
+
 double wait_timeout_s() {
   const char* e = getenv("SH_WAIT_TIMEOUT_S");
   return e ? atof(e) : 600.0;
@@ -565,6 +577,7 @@ void worker_loop(sh_ctx* c, int tid) {
       chunk = job->next++;
       if (c->clip) coef = c->coef_of_step[job->step & 1];
     }
+    maybe_delay(c->cfg.flags);
     const double t0 = now_ms();
     const int x = job->layer;
     const LayerLayout& Lx = c->lay[x];
@@ -860,6 +873,7 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   const int64_t gf_gen = c->gradfree_gen[s];
   c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, gf, stage_buf, gf_gen, s, n, eb, slice,
                 slo, shi, cs] {
+    maybe_delay(c->cfg.flags);
     double waited = 0;
     if (!state_wait(c, [&] { return ready_at_least(c, y, need); }, "CPU Adam of a layer to prefetch", &waited)) {
       c->arrive_pub[y].store(kInf);
@@ -1732,6 +1746,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       cudaEvent_t gf = c->ev_grad_free[s];
       if (k3_on_d2h) c->k3_last_gen = gen;
       c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P, k3_on_d2h, lo, hi] {
+        maybe_delay(c->cfg.flags);
         CKA(c, cudaStreamWaitEvent(c->d2h, grads_ready, 0));
         if (k3_on_d2h) {  // K3 before any host wait: sh_step only needs the norms
           if (P) CKA(c, cudaEventRecord(P->k30[x], c->d2h));

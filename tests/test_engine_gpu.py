@@ -261,3 +261,23 @@ def test_read_grad_after_landing_ring_reuse_is_an_error():
         assert e.value.status == sh.SH_ERR_STATE
     finally:
         tr.close()
+
+
+@pytest.mark.parametrize("precision,extra", [(sh.SH_BF16_MIXED, 0), (sh.SH_FP32, 0),
+                                             (sh.SH_BF16_MIXED, sh.SH_FLAG_FETCH_FP32)])
+def test_delay_injection_bitwise(precision, extra):
+    """random host delays in the H2D/D2H issuers and the CPU Adam tasks perturb every
+    cross-thread ordering; slot poisoning turns any read of a not-yet-arrived layer into NaNs.  The
+    result must still equal the resident run bitwise (small landing ring, few threads)."""
+    L = TINY["L"]
+    ref, _, _ = engine_run(TINY, STEPS, L, precision)
+    ref_state = engine_state(ref)
+    ref.close()
+    for w in (0, 1, 2):
+        tr, _, _ = engine_run(TINY, STEPS, w, precision, cpu_threads=3, grad_ring_depth=2,
+                              flags=sh.SH_FLAG_DELAY_INJECT | sh.SH_FLAG_POISON | extra)
+        try:
+            ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+            assert ok, (w, what)
+        finally:
+            tr.close()
