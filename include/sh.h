@@ -110,6 +110,8 @@ typedef struct {
                                            DRAM reads per rank / W).  Needs NCCL >= 2.18 (ncclCommSplit). */
 #define SH_FLAG_DELAY_INJECT (1ull << 8) /* test: random 0-2 ms sleeps in the copy issuers and CPU Adam tasks
                                             (ordering-race hunting; results must stay bitwise identical) */
+#define SH_FLAG_DECOUPLE  (1ull << 9) /* autotuner: decouple the ring (prefetch distance) from the
+                                         GPU-optimised set (needs no clipping; R22) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
@@ -129,6 +131,10 @@ typedef struct {
   int32_t warmup_steps;             /* profiled steps before autotune (default 5); 0 = default */
   int64_t device_budget_bytes;      /* S_avail for ring + G states; 0 = free memory - 2 GiB */
   double cpu_util_max;              /* autotuner eq. 3 utilisation target rho (SH_FLAG_CPU_HARD); 0 = 0.85 */
+  int32_t ring_slots;               /* ring size cap (0: window + 1).  Without clipping a GPU-optimised
+                                       layer is updated right after its backward, so its slot is not
+                                       pinned and the ring may be smaller than the GPU-optimised set:
+                                       prefetch distance = min(window, ring_slots - 1) (R22) */
   int32_t world_size;               /* data-parallel ranks (1 = single GPU) */
   int32_t rank;
   const void* nccl_unique_id;       /* 128-byte ncclUniqueId, required when world_size > 1 */
@@ -158,6 +164,8 @@ typedef struct {
   int32_t cpu_hard;            /* 1: also require the CPU-update throughput form of eq. 3 (R19):
                                   Σ_{k>=w} t_opt_cpu^k <= rho * (Σ_i (t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i) */
   double cpu_util_max;         /* rho in (0, 1]; <= 0 means 1 (utilisation target of the CPU pool) */
+  int32_t decouple;            /* 1: choose the prefetch distance d (ring d+1, by P1/P2) and the
+                                  GPU-optimised set g >= d (by eq. 3 + memory) separately (R22) */
 } sh_profile;
 
 typedef struct {
@@ -170,6 +178,7 @@ typedef struct {
   double eq4_lhs_ms, eq4_rhs_ms; /* 5 n t_async  vs  Σ_{i=w}^{n-1} t_opt_gpu (eq. 4) */
   double cpu_total_ms;     /* Σ_{k>=w} t_opt_cpu^k at the chosen window */
   double gpu_step_ms;      /* Σ_i (t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i */
+  int32_t ring_slots;      /* chosen ring size (prefetch distance + 1); window + 1 unless decoupled */
 } sh_solve_report;
 
 typedef struct {
@@ -283,6 +292,9 @@ sh_status sh_autotune_window(sh_ctx* ctx, const sh_profile* override_profile, in
 
 /* Change the window between steps (after sh_step, before the next forward hook). */
 sh_status sh_set_window(sh_ctx* ctx, int32_t window);
+
+/* Change the GPU-optimised set size (window) and the ring cap together (ring_slots 0: window+1). */
+sh_status sh_set_window_ring(sh_ctx* ctx, int32_t window, int32_t ring_slots);
 
 /* Fill the engine's measured profile (arrays owned by ctx, valid until the next call). */
 sh_status sh_get_profile(sh_ctx* ctx, sh_profile* out);

@@ -14,6 +14,8 @@ code shared with the C++ solver (paper_conf_sc_sunwqyhxw22_b200/csrc/autotune.cp
   (1d) sum over the same FP windows: sum t_fp >= sum t_c2g + sum t_g2c   (max() if duplex)
   (2d) sum over the same BP windows: sum t_bp >= sum t_c2g + sum t_g2c   (max() if duplex)
   rule: min{w < L : mem & hard & soft}, else min{w <= L : mem & hard}, else max{w : mem}
+  decouple (R22): prefetch distance d (ring d+1) and GPU-optimised set g = max(d, g_min) separately;
+      (1b)/(2b) fetch cost of a GPU-optimised layer is t_stage, and it has no offload (g2c = 0)
   cpu_hard (optional): sum_{k>=w} t_opt_cpu[k] <= rho (sum_i (t_fp[i] + t_bp[i]) + sum_{i<w} t_opt_gpu[i])
   eq. 3 slack: min_{k in [w, L)} [ sum_{i<=k}(t_fp[i]+t_bp[i]) + sum_{i<w} t_opt_gpu[i] - t_opt_cpu[k] ]
   eq. 4: 5 L t_async  vs  sum_{i=w}^{L-1} t_opt_gpu[i]
@@ -27,35 +29,40 @@ def _z(a, n):
 
 def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
           slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False, cpu_hard=False,
-          cpu_util_max=1.0):
+          cpu_util_max=1.0, decouple=False):
+    """d = prefetch distance (ring d+1 slots), g = GPU-optimised layers [0, g); coupled d = g = m
+    (the paper), decoupled g = max(d, smallest g meeting the CPU constraint) (R22)."""
     L = len(t_fp)
     fp, bp, c2g, g2c = _z(t_fp, L), _z(t_bp, L), _z(t_c2g, L), _z(t_g2c, L)
     st, og, oc = _z(t_stage, L), _z(t_opt_gpu, L), _z(t_opt_cpu, L)
     sb = [0] * L if slot_bytes is None else list(slot_bytes)
     gb = [0] * L if gstate_bytes is None else list(gstate_bytes)
 
-    def mem(w):
-        need = fixed_bytes + (w + 1) * max(sb)
-        for i in range(w):
+    def mem(d, g):
+        need = fixed_bytes + (d + 1) * max(sb)
+        for i in range(g):
             need += gb[i]
         return need <= s_avail
 
-    def fp_hard(w):
-        for j in range(w, L):
+    def fetch(j, g):
+        return st[j] if j < g else c2g[j]
+
+    def fp_hard(d, g):
+        for j in range(d, L):
             s = 0.0
-            for i in range(j - w, j):
+            for i in range(j - d, j):
                 s += fp[i]
-            if s < c2g[j]:
+            if s < fetch(j, g):
                 return False
         return True
 
-    def bp_hard(w):
-        for j in range(L - w - 2, -1, -1):
+    def bp_hard(d, g):
+        for j in range(L - d - 2, -1, -1):
             s = 0.0
-            for i in range(j + 1, j + w + 1):
+            for i in range(j + 1, j + d + 1):
                 s += bp[i]
-            fetch = st[j] if j < w else c2g[j]
-            if s < max(g2c[j + w + 1], fetch):
+            off = g2c[j + d + 1] if j + d + 1 >= g else 0.0   # GPU-optimised layers are not offloaded
+            if s < max(off, fetch(j, g)):
                 return False
         return True
 
@@ -65,44 +72,62 @@ def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None
         b = sum(g2c[i] for i in range(lo, hi))
         return comp >= (max(a, b) if duplex else a + b)
 
-    def soft(w):
-        for j in range(w, L):
-            if not window_ok(fp, j - w, j):
+    def soft(d):
+        for j in range(d, L):
+            if not window_ok(fp, j - d, j):
                 return False
-        for j in range(L - w - 2, -1, -1):
-            if not window_ok(bp, j + 1, j + w + 1):
+        for j in range(L - d - 2, -1, -1):
+            if not window_ok(bp, j + 1, j + d + 1):
                 return False
         return True
 
-    def cpu_ok(w):
+    def cpu_ok(g):
         if not cpu_hard:
             return True
         rho = cpu_util_max if 0.0 < cpu_util_max < 1.0 else 1.0
-        return sum(oc[k] for k in range(w, L)) <= rho * (sum(fp) + sum(bp) + sum(og[:w]))
+        return sum(oc[k] for k in range(g, L)) <= rho * (sum(fp) + sum(bp) + sum(og[:g]))
 
-    def hard(w):
-        return fp_hard(w) and bp_hard(w) and cpu_ok(w)
+    def hard(d, g):
+        return fp_hard(d, g) and bp_hard(d, g) and cpu_ok(g)
 
-    mems = [w for w in range(L + 1) if mem(w)]
+    mems = [w for w in range(L + 1) if mem(w, w)]
     if not mems:
         return None
-    best, reason = None, 2
-    for w in range(L):
-        if mem(w) and hard(w) and soft(w):
-            best, reason = w, 0
-            break
-    if best is None:
-        for w in range(L + 1):
-            if mem(w) and hard(w):
-                best, reason = w, 1
+    best = None
+    reason = 2
+    if not decouple:
+        for w in range(L):
+            if mem(w, w) and hard(w, w) and soft(w):
+                best, reason = (w, w), 0
                 break
+        if best is None:
+            for w in range(L + 1):
+                if mem(w, w) and hard(w, w):
+                    best, reason = (w, w), 1
+                    break
+    else:
+        gmin = 0
+        while gmin < L and not cpu_ok(gmin):
+            gmin += 1
+        for d in range(L):
+            g = max(d, gmin)
+            if mem(d, g) and hard(d, g) and soft(d):
+                best, reason = (d, g), 0
+                break
+        if best is None:
+            for d in range(L + 1):
+                g = max(d, gmin)
+                if mem(d, g) and hard(d, g):
+                    best, reason = (d, g), 1
+                    break
     if best is None:
-        best = max(mems)
+        best = (max(mems), max(mems))
+    d, g = best
     slack = None
-    for k in range(best, L):
-        rhs = sum(fp[i] + bp[i] for i in range(k + 1)) + sum(og[i] for i in range(best))
+    for k in range(g, L):
+        rhs = sum(fp[i] + bp[i] for i in range(k + 1)) + sum(og[i] for i in range(g))
         v = rhs - oc[k]
         slack = v if slack is None else min(slack, v)
-    return {"window": best, "reason": reason, "w_max_memory": max(mems),
+    return {"window": g, "ring_slots": d + 1, "reason": reason, "w_max_memory": max(mems),
             "eq3_min_slack_ms": 0.0 if slack is None else slack,
-            "eq4_lhs_ms": 5.0 * L * t_async, "eq4_rhs_ms": sum(og[i] for i in range(best, L))}
+            "eq4_lhs_ms": 5.0 * L * t_async, "eq4_rhs_ms": sum(og[i] for i in range(g, L))}

@@ -56,78 +56,93 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
   int64_t slot = 0;
   for (int i = 0; i < L; ++i) slot = std::max<int64_t>(slot, P->slot_bytes ? P->slot_bytes[i] : 0);
 
-  auto mem_ok = [&](int w) {
-    int64_t need = P->fixed_bytes + (int64_t)(w + 1) * slot;
-    for (int i = 0; i < w; ++i) need += P->gstate_bytes ? P->gstate_bytes[i] : 0;
+  // d = prefetch distance (ring d+1 slots), g = GPU-optimised layers [0, g).  The paper couples
+  // them (d = g = m); `decouple` (R22) lets g exceed d.
+  auto mem_ok = [&](int d, int g) {
+    int64_t need = P->fixed_bytes + (int64_t)(d + 1) * slot;
+    for (int i = 0; i < g; ++i) need += P->gstate_bytes ? P->gstate_bytes[i] : 0;
     return need <= P->s_avail;
   };
-  auto fp_hard = [&](int w) {  // (1b): ∀ j ∈ [w, L): Σ_{i=j-w}^{j-1} t_fp ≥ t_c2g[j]
-    for (int j = w; j < L; ++j)
-      if (fp.sum(j - w, j) < at(P->t_c2g, j)) return false;
+  auto fetch = [&](int j, int g) { return j < g ? at(P->t_stage, j) : at(P->t_c2g, j); };
+  auto fp_hard = [&](int d, int g) {  // (1b): ∀ j ∈ [d, L): Σ_{i=j-d}^{j-1} t_fp ≥ fetch of j
+    for (int j = d; j < L; ++j)
+      if (fp.sum(j - d, j) < fetch(j, g)) return false;
     return true;
   };
-  auto bp_hard = [&](int w) {  // (2b): ∀ j ∈ [0, L-w-2]: Σ_{i=j+1}^{j+w} t_bp ≥ max(g2c[j+w+1], fetch_j)
-    for (int j = 0; j + w + 1 < L; ++j) {
-      const double fetch = j < w ? at(P->t_stage, j) : at(P->t_c2g, j);
-      const double need = std::max(at(P->t_g2c, j + w + 1), fetch);
-      if (bp.sum(j + 1, j + w + 1) < need) return false;
+  auto bp_hard = [&](int d, int g) {  // (2b): ∀ j ∈ [0, L-d-2]: Σ_{i=j+1}^{j+d} t_bp ≥ max(g2c[j+d+1], fetch_j)
+    for (int j = 0; j + d + 1 < L; ++j) {
+      const double off = j + d + 1 >= g ? at(P->t_g2c, j + d + 1) : 0.0;  // G layers are not offloaded
+      if (bp.sum(j + 1, j + d + 1) < std::max(off, fetch(j, g))) return false;
     }
     return true;
   };
-  auto soft = [&](int w) {  // (1d) over FP windows, (2d) over BP windows
-    for (int j = w; j < L; ++j) {
-      const double a = c2g.sum(j - w, j), b = g2c.sum(j - w, j);
-      if (fp.sum(j - w, j) < (P->duplex ? std::max(a, b) : a + b)) return false;
+  auto soft = [&](int d) {  // (1d) over FP windows, (2d) over BP windows
+    for (int j = d; j < L; ++j) {
+      const double a = c2g.sum(j - d, j), b = g2c.sum(j - d, j);
+      if (fp.sum(j - d, j) < (P->duplex ? std::max(a, b) : a + b)) return false;
     }
-    for (int j = 0; j + w + 1 < L; ++j) {
-      const double a = c2g.sum(j + 1, j + w + 1), b = g2c.sum(j + 1, j + w + 1);
-      if (bp.sum(j + 1, j + w + 1) < (P->duplex ? std::max(a, b) : a + b)) return false;
+    for (int j = 0; j + d + 1 < L; ++j) {
+      const double a = c2g.sum(j + 1, j + d + 1), b = g2c.sum(j + 1, j + d + 1);
+      if (bp.sum(j + 1, j + d + 1) < (P->duplex ? std::max(a, b) : a + b)) return false;
     }
     return true;
   };
-
-  auto cpu_total = [&](int w) {
+  auto cpu_total = [&](int g) {
     double t = 0;
-    for (int k = w; k < L; ++k) t += at(P->t_opt_cpu, k);
+    for (int k = g; k < L; ++k) t += at(P->t_opt_cpu, k);
     return t;
   };
-  auto gpu_step = [&](int w) { return fp.sum(0, L) + bp.sum(0, L) + ogpu.sum(0, w); };
+  auto gpu_step = [&](int g) { return fp.sum(0, L) + bp.sum(0, L) + ogpu.sum(0, g); };
   const double rho = P->cpu_util_max > 0.0 && P->cpu_util_max < 1.0 ? P->cpu_util_max : 1.0;
-  auto hard = [&](int w) {
-    return fp_hard(w) && bp_hard(w) && (!P->cpu_hard || cpu_total(w) <= rho * gpu_step(w));
-  };
+  auto cpu_ok = [&](int g) { return !P->cpu_hard || cpu_total(g) <= rho * gpu_step(g); };
+  auto hard = [&](int d, int g) { return fp_hard(d, g) && bp_hard(d, g) && cpu_ok(g); };
+
   int wmax = -1;
   for (int w = 0; w <= L; ++w)
-    if (mem_ok(w)) wmax = w;
+    if (mem_ok(w, w)) wmax = w;
   if (wmax < 0) {
     set_error("sh_solve_window: even w=0 exceeds S_avail (%lld bytes)", (long long)P->s_avail);
     return SH_ERR_OOM_DEVICE;
   }
-  int best = -1, reason = 2;
-  for (int w = 0; w < L && best < 0; ++w)
-    if (mem_ok(w) && hard(w) && soft(w)) best = w, reason = 0;
-  for (int w = 0; w <= L && best < 0; ++w)
-    if (mem_ok(w) && hard(w)) best = w, reason = 1;
-  if (best < 0) best = wmax, reason = 2;
+  int best_d = -1, best_g = -1, reason = 2;
+  if (!P->decouple) {
+    for (int w = 0; w < L && best_d < 0; ++w)
+      if (mem_ok(w, w) && hard(w, w) && soft(w)) best_d = best_g = w, reason = 0;
+    for (int w = 0; w <= L && best_d < 0; ++w)
+      if (mem_ok(w, w) && hard(w, w)) best_d = best_g = w, reason = 1;
+  } else {
+    int gmin = 0;
+    while (gmin < L && !cpu_ok(gmin)) ++gmin;
+    for (int d = 0; d < L && best_d < 0; ++d) {
+      const int g = std::max(d, gmin);
+      if (mem_ok(d, g) && hard(d, g) && soft(d)) best_d = d, best_g = g, reason = 0;
+    }
+    for (int d = 0; d <= L && best_d < 0; ++d) {
+      const int g = std::max(d, gmin);
+      if (mem_ok(d, g) && hard(d, g)) best_d = d, best_g = g, reason = 1;
+    }
+  }
+  if (best_d < 0) best_d = best_g = wmax, reason = 2;
 
-  R->window = best;
+  R->window = best_g;
+  R->ring_slots = best_d + 1;
   R->w_max_memory = wmax;
   R->reason = reason;
-  R->fp_hard_ok = fp_hard(best);
-  R->bp_hard_ok = bp_hard(best);
-  R->soft_ok = soft(best);
-  // eq. 3: t_opt_cpu^k ≤ Σ_{i=0}^{k}(t_fp^i + t_bp^i) + Σ_{i<w} t_opt_gpu^i,  k ∈ [w, L)
+  R->fp_hard_ok = fp_hard(best_d, best_g);
+  R->bp_hard_ok = bp_hard(best_d, best_g);
+  R->soft_ok = soft(best_d);
+  // eq. 3: t_opt_cpu^k ≤ Σ_{i=0}^{k}(t_fp^i + t_bp^i) + Σ_{i<g} t_opt_gpu^i,  k ∈ [g, L)
   double slack = INFINITY;
-  for (int k = best; k < L; ++k) {
-    const double rhs = fp.sum(0, k + 1) + bp.sum(0, k + 1) + ogpu.sum(0, best);
+  for (int k = best_g; k < L; ++k) {
+    const double rhs = fp.sum(0, k + 1) + bp.sum(0, k + 1) + ogpu.sum(0, best_g);
     slack = std::min(slack, rhs - at(P->t_opt_cpu, k));
   }
   R->eq3_min_slack_ms = std::isinf(slack) ? 0.0 : slack;
   R->eq3_ok = !(slack < 0.0);
-  // eq. 4: 5 n t_async ≤ Σ_{i=w}^{n-1} t_opt_gpu
+  // eq. 4: 5 n t_async ≤ Σ_{i=g}^{n-1} t_opt_gpu
   R->eq4_lhs_ms = 5.0 * L * P->t_async;
-  R->eq4_rhs_ms = ogpu.sum(best, L);
-  R->cpu_total_ms = cpu_total(best);
-  R->gpu_step_ms = gpu_step(best);
+  R->eq4_rhs_ms = ogpu.sum(best_g, L);
+  R->cpu_total_ms = cpu_total(best_g);
+  R->gpu_step_ms = gpu_step(best_g);
   return SH_OK;
 }

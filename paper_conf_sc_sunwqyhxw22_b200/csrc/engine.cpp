@@ -183,9 +183,9 @@ class Issuer {
 };
 
 struct ProfSet {  // CUDA timing events of one step (double-buffered by step parity)
-  std::vector<cudaEvent_t> fp0, fp1, bp0, bp1, c2g0[2], c2g1[2], g2c0, g2c1, st0, st1, k30, k31;
+  std::vector<cudaEvent_t> fp0, fp1, bp0, bp1, c2g0[2], c2g1[2], g2c0, g2c1, st0, st1, k30, k31, k2l0, k2l1;
   std::vector<std::atomic<uint8_t>> rec_c2g[2], rec_g2c, rec_st;
-  std::vector<uint8_t> rec_fp, rec_bp, rec_k3;
+  std::vector<uint8_t> rec_fp, rec_bp, rec_k3, rec_k2l;
   cudaEvent_t k2a = nullptr, k2b = nullptr, t0 = nullptr;
   bool rec_k2 = false, rec_t0 = false;
   bool active = false;
@@ -235,7 +235,15 @@ struct sh_ctx {
   int64_t slot_param_bytes = 0, slot_grad_bytes = 0, slot_bytes = 0;
   int w = 0;
   int n_slots = 0;   // allocated
-  int n_active = 0;  // used = w+1
+  int n_active = 0;  // slots in use = min(w + 1, ring cap)
+  int d = 0;         // prefetch distance = n_active - 1 (the paper's window m when the ring is w+1)
+  int ring_cap = 0;  // sh_config.ring_slots / sh_set_window_ring (0: w + 1)
+  bool k2_layer = true;  // no clipping: a GPU-optimised layer is updated right after its backward
+  int ring_for(int w_) const {
+    int r = w_ + 1;
+    if (k2_layer && ring_cap > 0 && ring_cap < r) r = ring_cap;  // G grads are not pinned: ring may be smaller
+    return r;
+  }
   int D = 0;         // host landing buffers
   bool clip = false;
   int warmup = 5;
@@ -352,6 +360,7 @@ struct sh_ctx {
   int64_t h2d_prof_bytes = 0, d2h_prof_bytes = 0;
   double k2_ms_last = 0, k2_ms_sum = 0, k3_ms_sum = 0;
   int64_t k2_bytes_last = 0, k2_bytes_sum = 0, k2_samples = 0, k3_bytes_sum = 0, k3_samples = 0;
+  int64_t k2_layer_launches = 0;
   int k2_launches_last = 0;
 
   // ---- failure
@@ -664,7 +673,7 @@ sh_status prof_alloc(sh_ctx* c, ProfSet& P) {
   };
   cudaError_t r = cudaSuccess;
   for (auto* v : {&P.fp0, &P.fp1, &P.bp0, &P.bp1, &P.c2g0[0], &P.c2g1[0], &P.c2g0[1], &P.c2g1[1],
-                  &P.g2c0, &P.g2c1, &P.st0, &P.st1, &P.k30, &P.k31})
+                  &P.g2c0, &P.g2c1, &P.st0, &P.st1, &P.k30, &P.k31, &P.k2l0, &P.k2l1})
     if (r == cudaSuccess) r = mk(*v);
   if (r == cudaSuccess) r = cudaEventCreate(&P.k2a);
   if (r == cudaSuccess) r = cudaEventCreate(&P.k2b);
@@ -680,6 +689,7 @@ sh_status prof_alloc(sh_ctx* c, ProfSet& P) {
   P.rec_fp.assign(c->L, 0);
   P.rec_bp.assign(c->L, 0);
   P.rec_k3.assign(c->L, 0);
+  P.rec_k2l.assign(c->L, 0);
   return SH_OK;
 }
 
@@ -692,6 +702,7 @@ void prof_reset(sh_ctx* c, ProfSet& P, int64_t step) {
     P.rec_fp[i] = 0;
     P.rec_bp[i] = 0;
     P.rec_k3[i] = 0;
+    P.rec_k2l[i] = 0;
   }
   P.rec_k2 = false;
   P.rec_t0 = false;
@@ -744,6 +755,7 @@ void build_trace(sh_ctx* c, ProfSet& P) {
     if (P.rec_g2c[i]) add(4, i, P.g2c0[i], P.g2c1[i]);
     if (P.rec_st[i]) add(5, i, P.st0[i], P.st1[i]);
     if (P.rec_k3[i]) add(6, i, P.k30[i], P.k31[i]);
+    if (P.rec_k2l[i]) add(7, i, P.k2l0[i], P.k2l1[i]);
   }
   if (P.rec_k2) add(7, -1, P.k2a, P.k2b);
   std::vector<std::pair<double, double>> comp, h2d, d2h;
@@ -785,6 +797,13 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
       c->d2h_prof_bytes += 4 * (c->shi[i] - c->slo[i]);
     }
     if (P.rec_st[i]) c->p_stage[i] = ev_ms(P.st0[i], P.st1[i]);
+    if (P.rec_k2l[i]) {
+      const double ms = ev_ms(P.k2l0[i], P.k2l1[i]);
+      c->p_ogpu[i] = ms;
+      c->k2_ms_sum += ms;
+      c->k2_bytes_sum += (c->bf16 ? 30 : 32) * c->lay[i].n_pad;
+      c->k2_layer_launches++;
+    }
     if (P.rec_k3[i]) {
       c->k3_ms_sum += ev_ms(P.k30[i], P.k31[i]);
       c->k3_bytes_sum += 4 * c->lay[i].n_pad;
@@ -801,8 +820,9 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
     // apportion K2 time to layers by bytes (one fused launch covers all of them)
     double tot = 0;
     for (int i = 0; i < L; ++i) tot += c->lay[i].n_pad;
-    for (int i = 0; i < L; ++i)
-      c->p_ogpu[i] = P.k2_bytes > 0 ? c->k2_ms_last * (30.0 * c->lay[i].n_pad) / P.k2_bytes : 0.0;
+    if (!c->k2_layer)
+      for (int i = 0; i < L; ++i)
+        c->p_ogpu[i] = P.k2_bytes > 0 ? c->k2_ms_last * (30.0 * c->lay[i].n_pad) / P.k2_bytes : 0.0;
   }
   c->profiled_steps++;
 }
@@ -821,7 +841,10 @@ int64_t next_use(const sh_ctx* c, int x, int cur) {
   if (x >= cur) return x;  // FP use still ahead
   const int b = 2 * c->L - 1 - x;
   if (b >= cur) return b;  // BP use still ahead
-  return c->is_g(x) ? kPinned : kInf;  // G grads wait for K2; host copies go stale
+  // after its backward: a host copy goes stale; a GPU-optimised layer's copy was updated in place by
+  // its per-layer K2 (valid for the next step's FP) or, in clip mode, its grads wait for sh_step's K2
+  if (!c->is_g(x)) return kInf;
+  return c->k2_layer ? 2 * (int64_t)c->L + x : kPinned;
 }
 
 sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
@@ -948,7 +971,7 @@ bool ensure_at(sh_ctx* c, int p, int cur, sh_status* st) {
 // Common PRE work: ensure the current layer, prefetch the window ahead, wait for arrival.
 sh_status pre_common(sh_ctx* c, int x, int pos) {
   sh_status st;
-  const int last = std::min(pos + c->w, 2 * c->L - 1);
+  const int last = std::min(pos + c->d, 2 * c->L - 1);
   for (int p = pos; p <= last; ++p) {
     const bool ok = ensure_at(c, p, pos, &st);
     if (st != SH_OK) return st;
@@ -981,7 +1004,7 @@ sh_status stage_g_layers(sh_ctx* c) {
   // ring reset: G layers 0..w-1 into slots 0..w-1 (compute stream), the rest empty
   for (int s = 0; s < c->n_slots; ++s) c->slot_layer[s] = -1;
   for (int x = 0; x < c->L; ++x) c->layer_slot[x] = -1;
-  for (int x = 0; x < c->w; ++x) {
+  for (int x = 0; x < std::min(c->w, c->n_active); ++x) {  // the rest are restaged by K1 on demand
     c->slot_layer[x] = x;
     c->layer_slot[x] = x;
     char* dst = c->slot_param(x);
@@ -1186,10 +1209,11 @@ sh_status apply_window(sh_ctx* c, int w_new) {
     CKC(c, cudaMemcpy(c->g[x].m, c->h_m[x], 4 * n, cudaMemcpyHostToDevice));
     CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
   }
-  st = alloc_ring(c, w_new + 1);
+  st = alloc_ring(c, c->ring_for(w_new));
   if (st != SH_OK) return st;
   c->w = w_new;
-  c->n_active = w_new + 1;
+  c->n_active = c->ring_for(w_new);
+  c->d = c->n_active - 1;
   st = stage_g_layers(c);
   if (st != SH_OK) return st;
   CKC(c, cudaStreamSynchronize(c->cs));
@@ -1495,9 +1519,12 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     if (s != SH_OK) return s;
   }
   c->w = w0;
-  c->n_active = w0 + 1;
+  c->k2_layer = !c->clip;
+  c->ring_cap = cfg->ring_slots > 0 ? cfg->ring_slots : 0;
+  c->n_active = c->ring_for(w0);
+  c->d = c->n_active - 1;
   {
-    sh_status s = alloc_ring(c.get(), w0 + 1);
+    sh_status s = alloc_ring(c.get(), c->n_active);
     if (s != SH_OK) return s;
     for (int x = 0; x < w0; ++x) {
       s = alloc_g(c.get(), x);
@@ -1730,6 +1757,39 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       // host layer: K3 runs on the D2H stream right before the offload (off the compute stream)
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
     }
+    if (c->is_g(x) && c->k2_layer) {
+      // per-layer K2 of a GPU-optimised layer right after its backward (no clipping: the update
+      // needs no global norm; bitwise the same as the step-end K2).  Single GPU: on the compute
+      // stream, in order.  Data parallel: on the comm stream after the all-reduce and K3, so the
+      // compute stream does not wait for the collective; the next use of the slot (a fetch into it,
+      // the next FP of the layer, the next occupant's grad half) waits on events recorded after it.
+      cudaStream_t ks = c->W > 1 ? c->comm : c->cs;
+      if (P) CKC(c, cudaEventRecord(P->k2l0[x], ks));
+      kern::K2Args a{};
+      a.sc = c->sc;
+      a.coef = nullptr;
+      a.out_bf16 = c->bf16;
+      a.n_entries = 1;
+      a.e[0] = kern::K2Entry{c->g[x].master, c->g[x].m, c->g[x].v, c->slot_grad(s), c->slot_param(s), n,
+                             c->lay[x].n_decay};
+      CKC(c, kern::adamw_multi(a, ks));
+      if (P) {
+        CKC(c, cudaEventRecord(P->k2l1[x], ks));
+        P->rec_k2l[x] = 1;
+      }
+      CKC(c, cudaEventRecord(c->ev_param_free[s], ks));  // param half rewritten by K2
+      if (ks != c->cs) {
+        CKC(c, cudaEventRecord(c->ev_grad_free[s], ks));
+        const int64_t g1 = ++c->gen;
+        c->gradfree_gen[s] = g1;
+        c->gradfree_pub[s].store(g1);
+        CKC(c, cudaEventRecord(c->ev_arrive[x], ks));
+        const int64_t g2 = ++c->gen;
+        c->arrive_gen[x] = g2;
+        c->arrive_by_issuer[x] = 0;
+        c->arrive_pub[x].store(g2);
+      }
+    }
     const bool k3_on_d2h = c->W == 1 && !c->is_g(x);
     if (!c->is_g(x)) {
       const int k = (int)(c->landing_rr++ % c->D);
@@ -1859,8 +1919,9 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
   a.out_bf16 = c->bf16;
   int64_t bytes = 0;
   int launches = 0;
-  // layer 0 first: the next FP starts with it
-  for (int x = 0; x < c->w; ++x) {
+  // clip mode: the GPU-optimised layers (pinned in the ring) are updated here with the clip
+  // coefficient, layer 0 first (the next FP starts with it); otherwise they were updated per layer
+  for (int x = 0; x < (c->k2_layer ? 0 : c->w); ++x) {
     const int s = c->layer_slot[x];
     if (s < 0) {
       set_error("internal: GPU-optimised layer %d not in the ring at sh_step", x);
@@ -1968,6 +2029,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   o->duplex = (c->cfg.flags & SH_FLAG_DUPLEX) ? 1 : 0;
   o->cpu_hard = (c->cfg.flags & SH_FLAG_CPU_HARD) ? 1 : 0;
   o->cpu_util_max = c->cfg.cpu_util_max > 0.0 ? c->cfg.cpu_util_max : 0.85;
+  o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip ? 1 : 0;
   return SH_OK;
 }
 
@@ -1992,6 +2054,32 @@ sh_status sh_set_window(sh_ctx* c, int32_t w) {
   return apply_window(c, w);
 }
 
+sh_status sh_set_window_ring(sh_ctx* c, int32_t w, int32_t ring) {
+  clear_error();
+  if (!c) return SH_ERR_INVALID;
+  if (ring < 0) {
+    set_error("sh_set_window_ring: ring_slots must be >= 0");
+    return SH_ERR_INVALID;
+  }
+  if (c->clip && ring > 0 && ring < w + 1) {
+    set_error("sh_set_window_ring: clip mode pins the GPU-optimised layers' grads: ring must be >= window + 1");
+    return SH_ERR_INVALID;
+  }
+  if (c->phase != sh_ctx::IDLE) {
+    set_error("sh_set_window_ring: only between steps");
+    return SH_ERR_STATE;
+  }
+  if (w < 0 || w > c->L) {
+    set_error("sh_set_window_ring: window %d outside 0..%d", w, c->L);
+    return SH_ERR_INVALID;
+  }
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  if (w == c->w && ring == c->ring_cap) return SH_OK;
+  c->ring_cap = ring;
+  return apply_window(c, w);
+}
+
 sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   clear_error();
   if (!c) return SH_ERR_INVALID;
@@ -2007,15 +2095,17 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   if (st != SH_OK) return st;
   c->autotune_pending = false;
   int32_t w = rep.window;
+  int32_t ring = p.decouple && !c->clip ? rep.ring_slots : 0;
   if (c->shared) {  // one shared host store: the whole job must switch to the same window
-    if (c->rank == 0) c->ctl->window.store(w);
+    if (c->rank == 0) c->ctl->window.store((int64_t)w | ((int64_t)ring << 32));
     if (!shm_barrier(c, 4, "autotuned window agreement")) return check_failed(c);
-    w = (int32_t)c->ctl->window.load();
+    const int64_t v = c->ctl->window.load();
+    w = (int32_t)(v & 0xffffffff);
+    ring = (int32_t)(v >> 32);
     if (!shm_barrier(c, 5, "autotuned window read")) return check_failed(c);
   }
   if (wout) *wout = w;
-  if (w != c->w) return sh_set_window(c, w);
-  return SH_OK;
+  return sh_set_window_ring(c, w, ring);
 }
 
 sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
@@ -2165,7 +2255,7 @@ sh_status sh_destroy(sh_ctx* c) {
       if (e) cudaEventDestroy(e);
   for (auto& P : c->prof) {
     for (auto* v : {&P.fp0, &P.fp1, &P.bp0, &P.bp1, &P.c2g0[0], &P.c2g1[0], &P.c2g0[1], &P.c2g1[1],
-                    &P.g2c0, &P.g2c1, &P.st0, &P.st1, &P.k30, &P.k31})
+                    &P.g2c0, &P.g2c1, &P.st0, &P.st1, &P.k30, &P.k31, &P.k2l0, &P.k2l1})
       for (auto e : *v)
         if (e) cudaEventDestroy(e);
     if (P.k2a) cudaEventDestroy(P.k2a);

@@ -21,7 +21,8 @@ SH_FP32, SH_BF16_MIXED = 0, 1
 SH_PRE, SH_POST = 0, 1
 SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE, SH_READ_GRAD = 0, 1, 2, 3, 4
 SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32, \
-    SH_FLAG_TEST_NO_COLLECTIVE, SH_FLAG_SLICE_FETCH, SH_FLAG_DELAY_INJECT = 1, 2, 4, 8, 16, 32, 64, 128, 256
+    SH_FLAG_TEST_NO_COLLECTIVE, SH_FLAG_SLICE_FETCH, SH_FLAG_DELAY_INJECT, SH_FLAG_DECOUPLE = \
+    1, 2, 4, 8, 16, 32, 64, 128, 256, 512
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
@@ -29,7 +30,7 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_autotune_window", "sh_set_window", "sh_get_profile", "sh_read_layer", "sh_stats",
            "sh_last_error", "sh_abi_version", "sh_nccl_get_unique_id", "sh_adam_scalars_for",
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
-           "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end")
+           "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end", "sh_set_window_ring")
 
 
 class ShError(RuntimeError):
@@ -48,8 +49,8 @@ class Config(C.Structure):
                 ("beta2", C.c_double), ("eps", C.c_double), ("weight_decay", C.c_double),
                 ("max_grad_norm", C.c_double), ("device", C.c_int32), ("compute_stream", C.c_void_p),
                 ("cpu_threads", C.c_int32), ("grad_ring_depth", C.c_int32), ("warmup_steps", C.c_int32),
-                ("device_budget_bytes", C.c_int64), ("cpu_util_max", C.c_double), ("world_size", C.c_int32),
-                ("rank", C.c_int32),
+                ("device_budget_bytes", C.c_int64), ("cpu_util_max", C.c_double), ("ring_slots", C.c_int32),
+                ("world_size", C.c_int32), ("rank", C.c_int32),
                 ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p)]
 
 
@@ -62,14 +63,15 @@ class Profile(C.Structure):
                 ("t_stage", _PD), ("t_opt_gpu", _PD), ("t_opt_cpu", _PD), ("t_async", C.c_double),
                 ("slot_bytes", _PI64), ("gstate_bytes", _PI64), ("fixed_bytes", C.c_int64),
                 ("s_avail", C.c_int64), ("duplex", C.c_int32), ("cpu_hard", C.c_int32),
-                ("cpu_util_max", C.c_double)]
+                ("cpu_util_max", C.c_double), ("decouple", C.c_int32)]
 
 
 class SolveReport(C.Structure):
     _fields_ = [("window", C.c_int32), ("w_max_memory", C.c_int32), ("reason", C.c_int32),
                 ("fp_hard_ok", C.c_int32), ("bp_hard_ok", C.c_int32), ("soft_ok", C.c_int32),
                 ("eq3_min_slack_ms", C.c_double), ("eq3_ok", C.c_int32), ("eq4_lhs_ms", C.c_double),
-                ("eq4_rhs_ms", C.c_double), ("cpu_total_ms", C.c_double), ("gpu_step_ms", C.c_double)]
+                ("eq4_rhs_ms", C.c_double), ("cpu_total_ms", C.c_double), ("gpu_step_ms", C.c_double),
+                ("ring_slots", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -127,7 +129,7 @@ def lib() -> C.CDLL:
             "sh_op_cast_bf16_gpu": [vp, vp, i64, vp], "sh_op_cast_bf16_cpu": [vp, vp, i64],
             "sh_op_sumsq_gpu": [vp, i64, vp, vp],
             "sh_get_trace": [vp, vp, i32, C.POINTER(i32)],
-            "sh_forward_only_end": [vp],
+            "sh_forward_only_end": [vp], "sh_set_window_ring": [vp, i32, i32],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -218,7 +220,7 @@ def _dbl(a, n):
 
 def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
                  slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False,
-                 cpu_hard=False, cpu_util_max=1.0) -> dict:
+                 cpu_hard=False, cpu_util_max=1.0, decouple=False) -> dict:
     """Pure call of sh_solve_window (no GPU)."""
     n = len(t_fp)
     keep = {}
@@ -239,6 +241,7 @@ def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_c
     prof.duplex = 1 if duplex else 0
     prof.cpu_hard = 1 if cpu_hard else 0
     prof.cpu_util_max = cpu_util_max
+    prof.decouple = 1 if decouple else 0
     rep = SolveReport()
     check(lib().sh_solve_window(C.byref(prof), C.byref(rep)))
     return {f: getattr(rep, f) for f, _ in SolveReport._fields_}
@@ -252,7 +255,8 @@ class Engine:
     def __init__(self, layer_numels, layer_wd, res_numels, res_wd, *, window, precision=SH_BF16_MIXED,
                  lr=1.5e-4, betas=(0.9, 0.999), eps=1e-8, weight_decay=0.01, max_grad_norm=0.0, device=0,
                  stream=None, cpu_threads=0, grad_ring_depth=0, warmup_steps=5, device_budget_bytes=0,
-                 world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None):
+                 world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None,
+                 ring_slots=0, cpu_util_max=0.0):
         L = lib()
         self.n_layers = len(layer_numels)
         self._keep = []
@@ -278,6 +282,8 @@ class Engine:
         cfg.grad_ring_depth = grad_ring_depth
         cfg.warmup_steps = warmup_steps
         cfg.device_budget_bytes = device_budget_bytes
+        cfg.ring_slots = ring_slots
+        cfg.cpu_util_max = cpu_util_max
         cfg.world_size = world_size
         cfg.rank = rank
         idbuf = None
@@ -367,8 +373,11 @@ class Engine:
         return None
 
     # -- window
-    def set_window(self, w: int):
-        check(self._L.sh_set_window(self.h, w))
+    def set_window(self, w: int, ring_slots: int | None = None):
+        if ring_slots is None:
+            check(self._L.sh_set_window(self.h, w))
+        else:
+            check(self._L.sh_set_window_ring(self.h, w, ring_slots))
 
     def autotune(self) -> int:
         w = C.c_int32()
@@ -380,7 +389,7 @@ class Engine:
         check(self._L.sh_get_profile(self.h, C.byref(p)))
         n = p.n_layers
         out = {"n_layers": n, "t_async": p.t_async, "s_avail": p.s_avail, "fixed_bytes": p.fixed_bytes,
-               "duplex": p.duplex, "cpu_hard": p.cpu_hard, "cpu_util_max": p.cpu_util_max}
+               "duplex": p.duplex, "cpu_hard": p.cpu_hard, "cpu_util_max": p.cpu_util_max, "decouple": p.decouple}
         for f in ("t_fp", "t_bp", "t_c2g", "t_g2c", "t_stage", "t_opt_gpu", "t_opt_cpu"):
             out[f] = [getattr(p, f)[i] for i in range(n)]
         for f in ("slot_bytes", "gstate_bytes"):

@@ -53,7 +53,7 @@ class StrongholdTrainer:
     def __init__(self, mc: ModelConfig, *, batch: int, window: int, precision=sh.SH_BF16_MIXED, lr=1.5e-4,
                  max_grad_norm=0.0, device=0, seed=1234, cpu_threads=0, grad_ring_depth=0, warmup_steps=5,
                  flags=0, world_size=1, rank=0, nccl_id=None, init=True, init_threads=8, shm_name=None,
-                 attention="auto"):
+                 attention="auto", ring_slots=0):
         self.mc = mc
         self.batch = batch
         self.device = torch.device("cuda", device)
@@ -65,7 +65,7 @@ class StrongholdTrainer:
                                 precision=precision, lr=lr, max_grad_norm=max_grad_norm, device=device,
                                 stream=self.stream, cpu_threads=cpu_threads, grad_ring_depth=grad_ring_depth,
                                 warmup_steps=warmup_steps, world_size=world_size, rank=rank, nccl_id=nccl_id,
-                                flags=flags, shm_name=shm_name)
+                                flags=flags, shm_name=shm_name, ring_slots=ring_slots)
         self.gpt = GPT(n_layers=L, hidden=mc.hidden, heads=mc.heads, seq=mc.seq, max_batch=batch,
                        vocab=mc.vocab, precision=precision, device=device, stream=self.stream)
         # attention core: fused flash-attention library kernel on the bf16 path ("auto"/"flash"),

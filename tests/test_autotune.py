@@ -88,7 +88,22 @@ def test_eq3_and_eq4_reports():
     assert abs(r["eq4_rhs_ms"] - 0.25 * (L - w)) < 1e-12
 
 
-@pytest.mark.parametrize("seed", range(40))
+def test_decoupled_ring_smaller_than_gpu_set():
+    # transfers hide behind 2 layers (d = 2) but the CPU needs >= 7 GPU-optimised layers (eq. 3)
+    L = 10
+    prof = homog(L, 1.0, 1.5, 1.0, t_stage=[0.1] * L, t_opt_cpu=[10.0] * L, t_opt_gpu=[0.1] * L)
+    coupled = sh.solve_window(**prof, cpu_hard=True)
+    dec = sh.solve_window(**prof, cpu_hard=True, decouple=True)
+    gmin = math.ceil((10 * L - 4 * L) / 10.1)
+    assert coupled["window"] == gmin and coupled["ring_slots"] == gmin + 1
+    assert dec["window"] == gmin and dec["ring_slots"] == 3
+    # memory: the decoupled choice fits where the coupled one would not
+    prof_mem = dict(prof, slot_bytes=[10] * L, gstate_bytes=[1] * L, s_avail=3 * 10 + gmin * 1)
+    assert sh.solve_window(**prof_mem, cpu_hard=True, decouple=True)["window"] == gmin
+    assert sh.solve_window(**prof_mem, cpu_hard=True)["window"] < gmin
+
+
+@pytest.mark.parametrize("seed", range(60))
 def test_random_heterogeneous_matches_bruteforce(seed):
     rng = np.random.default_rng(seed)
     L = int(rng.integers(1, 30))
@@ -98,14 +113,14 @@ def test_random_heterogeneous_matches_bruteforce(seed):
                 slot_bytes=rng.integers(1, 100, L), gstate_bytes=rng.integers(1, 60, L),
                 fixed_bytes=int(rng.integers(0, 50)), s_avail=int(rng.integers(100, 3000)),
                 duplex=bool(rng.integers(0, 2)), cpu_hard=bool(rng.integers(0, 2)),
-                cpu_util_max=float(rng.choice([1.0, 0.85, 0.5])))
+                cpu_util_max=float(rng.choice([1.0, 0.85, 0.5])), decouple=bool(rng.integers(0, 2)))
     want = AO.solve(**{k: (list(v) if isinstance(v, np.ndarray) else v) for k, v in prof.items()})
     if want is None:
         with pytest.raises(sh.ShError):
             sh.solve_window(**prof)
         return
     got = sh.solve_window(**prof)
-    for k in ("window", "reason", "w_max_memory"):
+    for k in ("window", "reason", "w_max_memory", "ring_slots"):
         assert got[k] == want[k], (k, got, want)
     for k in ("eq3_min_slack_ms", "eq4_lhs_ms", "eq4_rhs_ms"):
         assert abs(got[k] - want[k]) <= 1e-9 * max(1.0, abs(want[k])), (k, got, want)

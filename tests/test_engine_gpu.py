@@ -281,3 +281,33 @@ def test_delay_injection_bitwise(precision, extra):
             assert ok, (w, what)
         finally:
             tr.close()
+
+
+
+@pytest.mark.parametrize("precision", [sh.SH_FP32, sh.SH_BF16_MIXED])
+def test_ring_smaller_than_gpu_set_bitwise(precision):
+    """R22: without clipping a GPU-optimised layer is updated right after its backward (per-layer
+    K2), so the ring (prefetch distance + 1) may be smaller than the GPU-optimised set; its layers
+    are then restaged by K1 from their HBM masters in FP as well.  Bitwise equal to resident."""
+    L = TINY["L"]
+    ref, _, _ = engine_run(TINY, STEPS, L, precision)
+    ref_state = engine_state(ref)
+    ref.close()
+    for w, ring in ((3, 2), (L, 1), (L, 3), (2, 1)):
+        tr, _, _ = engine_run(TINY, STEPS, w, precision, ring_slots=ring,
+                              flags=sh.SH_FLAG_POISON | sh.SH_FLAG_DELAY_INJECT)
+        try:
+            ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+            assert ok, (w, ring, what)
+            assert tr.engine.stats()["n_slots"] == min(ring, w + 1)
+        finally:
+            tr.close()
+    # ring changes mid-run, together with the GPU-optimised set
+    tr, _, _ = engine_run(TINY, 4, 1, precision, set_window_at={1: (3, 2), 2: (L, 1), 3: (0, 0)})
+    try:
+        ref2, _, _ = engine_run(TINY, 4, L, precision)
+        ok, what = states_bitwise_equal(engine_state(tr), engine_state(ref2))
+        ref2.close()
+        assert ok, what
+    finally:
+        tr.close()
