@@ -298,7 +298,8 @@ def main():
     def run(window, e2e: bool):
         t_init = time.perf_counter()
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
-            (sh.SH_FLAG_CPU_HARD if cpu_hard else 0) | (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0)
+            (sh.SH_FLAG_CPU_HARD | sh.SH_FLAG_DECOUPLE if cpu_hard else 0) | \
+            (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
@@ -405,8 +406,8 @@ def main():
         "config": {"workload": args.config, "description": desc, "layers": L, "hidden": h, "heads": nh, "seq": s,
                    "vocab": V, "params": mc.n_params(), "batch_per_gpu": b, "global_batch": b * world,
                    "window": r["st1"]["window"], "ring_slots": r["st1"]["n_slots"],
-                   "window_mode": ("autotuned (P1/P2" + (" + eq.3 CPU throughput" if cpu_hard else "") + ")")
-                   if w == -1 else "fixed",
+                   "window_mode": ("autotuned (P1/P2" + (" + eq.3 CPU throughput, ring decoupled from the GPU set"
+                                                         if cpu_hard else "") + ")") if w == -1 else "fixed",
                    "precision": "bf16_mixed" if prec else "fp32",
                    "gpt_driver_attention": r["attn"],
                    "parallelism": f"dp{world}",
