@@ -75,6 +75,7 @@ def c4_layers(h: int, ring: int, w0: int = 2, margin_gb: float = 8.0, ranks_shar
 METRIC = "samples/s at max trainable size per B200; host-link GB/s vs peak"
 PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
 PROBE_D2H_GBS = 57.01
+PROBE_HOST_TRIAD_GBS = 143.43  # profiles/r01_probe_box.json, 16-thread STREAM triad (no RFO counted)
 
 
 def measured_peaks():
@@ -436,7 +437,10 @@ def main():
                      "thread_ms_per_step": d["cpu_adam_ms"] / K,
                      "dram_gbs": 30.0 * d["cpu_adam_elems"] / (d["cpu_adam_ms"] / 1e3 / st1["cpu_threads"]) / 1e9
                      if d["cpu_adam_ms"] > 0 else None,
-                     "prefetch_wait_ms_per_step": d["cpu_wait_ms"] / K},
+                     "prefetch_wait_ms_per_step": d["cpu_wait_ms"] / K,
+                     "host_dram_triad_peak_gbs": PROBE_HOST_TRIAD_GBS,
+                     "note": "dram_gbs counts the AdamW's 30 B/param (28 without shadow) while its threads run; "
+                             "the copy engines' DMA shares the same host DRAM"},
         "roofline": {"kernel": "K2 fused multi-tensor AdamW (sh_step)", "bound": "hbm", "achieved": k2_gbs,
                      "peak": peak, "unit": "GB/s", "frac": k2_gbs / peak if k2_gbs else None, "traffic": None,
                      "peak_source": peak_kind, "algorithmic_bytes_per_elem": 30 if prec else 32,
