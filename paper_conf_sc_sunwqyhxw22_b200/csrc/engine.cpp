@@ -303,6 +303,7 @@ struct sh_ctx {
   std::vector<int64_t> gradfree_gen, gradfree_waited;
   std::unique_ptr<std::atomic<int64_t>[]> gradfree_pub;
   std::vector<cudaEvent_t> ev_arrive;
+  std::vector<cudaEvent_t> ev_upd;  // [L] after the latest K2 of a GPU-optimised layer (K1 restage waits)
   std::vector<int64_t> arrive_gen, compute_waited;
   std::vector<uint8_t> arrive_by_issuer;
   std::unique_ptr<std::atomic<int64_t>[]> arrive_pub;
@@ -860,8 +861,11 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   ProfSet* P = cur_prof(c);
   const int ph = pos < c->L ? 0 : 1;
   if (c->is_g(y)) {
-    // K1 restage from the HBM master (GPU-optimised layer evicted during FP)
+    // K1 restage from the HBM master (GPU-optimised layer evicted earlier): after the victim slot is
+    // free AND after the layer's latest K2 (its master may have been written on another stream or
+    // after the victim's release)
     CKC(c, cudaStreamWaitEvent(c->stage, c->ev_param_free[s], 0));
+    CKC(c, cudaStreamWaitEvent(c->stage, c->ev_upd[y], 0));
     if (poison) CKC(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->stage));
     if (P) CKC(c, cudaEventRecord(P->st0[y], c->stage));
     if (c->bf16)
@@ -1492,6 +1496,11 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->layer_slot.assign(c->L, -1);
   c->ev_arrive.assign(c->L, nullptr);
   for (auto& e : c->ev_arrive) CKC(c.get(), cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  c->ev_upd.assign(c->L, nullptr);
+  for (auto& e : c->ev_upd) {
+    CKC(c.get(), cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    CKC(c.get(), cudaEventRecord(e, c->cs));  // completed: nothing to wait for yet
+  }
   c->arrive_gen.assign(c->L, 0);
   c->compute_waited.assign(c->L, 0);
   c->arrive_by_issuer.assign(c->L, 0);
@@ -1778,6 +1787,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
         P->rec_k2l[x] = 1;
       }
       CKC(c, cudaEventRecord(c->ev_param_free[s], ks));  // param half rewritten by K2
+      CKC(c, cudaEventRecord(c->ev_upd[x], ks));
       if (ks != c->cs) {
         CKC(c, cudaEventRecord(c->ev_grad_free[s], ks));
         const int64_t g1 = ++c->gen;
@@ -1938,6 +1948,8 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
                                      c->res.n_pad, c->res.n_decay};
   st = push_k2(c, a, &bytes, &launches);
   if (st != SH_OK) return st;
+  if (!c->k2_layer)
+    for (int x = 0; x < c->w; ++x) CKC(c, cudaEventRecord(c->ev_upd[x], c->cs));
   if (P) {
     CKC(c, cudaEventRecord(P->k2b, c->cs));
     P->rec_k2 = true;
@@ -2250,7 +2262,7 @@ sh_status sh_destroy(sh_ctx* c) {
   if (c->ring) cudaFree(c->ring);
   if (c->res_master) cudaFree(c->res_master);
   if (c->partials) cudaFree(c->partials);
-  for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced, &c->ev_arrive})
+  for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced, &c->ev_arrive, &c->ev_upd})
     for (auto e : *v)
       if (e) cudaEventDestroy(e);
   for (auto& P : c->prof) {
