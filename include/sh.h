@@ -111,7 +111,8 @@ typedef struct {
 #define SH_FLAG_DELAY_INJECT (1ull << 8) /* test: random 0-2 ms sleeps in the copy issuers and CPU Adam tasks
                                             (ordering-race hunting; results must stay bitwise identical) */
 #define SH_FLAG_DECOUPLE  (1ull << 9) /* autotuner: decouple the ring (prefetch distance) from the
-                                         GPU-optimised set (needs no clipping; R22) */
+                                         GPU-optimised set (needs no clipping and a landing buffer per
+                                         layer, grad_ring_depth 0; R22) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

@@ -2041,7 +2041,10 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   o->duplex = (c->cfg.flags & SH_FLAG_DUPLEX) ? 1 : 0;
   o->cpu_hard = (c->cfg.flags & SH_FLAG_CPU_HARD) ? 1 : 0;
   o->cpu_util_max = c->cfg.cpu_util_max > 0.0 ? c->cfg.cpu_util_max : 0.85;
-  o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip ? 1 : 0;
+  // decoupling needs a landing buffer per host layer: otherwise the ring's grad halves are what
+  // absorbs the D2H backlog when the CPU Adam is slower than BP (measured: a 7-slot ring with a
+  // 4-deep landing ring stalled BP every 4 layers on the C4 model)
+  o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip && c->D >= c->L ? 1 : 0;
   return SH_OK;
 }
 
@@ -2140,11 +2143,16 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
     if (layer < 0) {
       CKC(c, cudaMemcpy(tmp.data(), c->res_compute, tmp.size(), cudaMemcpyDeviceToHost));
     } else if (c->is_g(layer)) {
-      if (c->layer_slot[layer] < 0) {
-        set_error("sh_read_layer: layer %d not staged", layer);
-        return SH_ERR_STATE;
+      if (c->layer_slot[layer] >= 0) {
+        CKC(c, cudaMemcpy(tmp.data(), c->slot_param(c->layer_slot[layer]), tmp.size(), cudaMemcpyDeviceToHost));
+      } else {  // outside the ring (decoupled ring): the copy K1 would stage, from the HBM master
+        std::vector<float> mst(n);
+        CKC(c, cudaMemcpy(mst.data(), c->g[layer].master, 4 * n, cudaMemcpyDeviceToHost));
+        if (c->bf16)
+          cpu::cast_bf16_range(mst.data(), reinterpret_cast<uint16_t*>(tmp.data()), 0, n);
+        else
+          std::memcpy(tmp.data(), mst.data(), 4 * n);
       }
-      CKC(c, cudaMemcpy(tmp.data(), c->slot_param(c->layer_slot[layer]), tmp.size(), cudaMemcpyDeviceToHost));
     } else {
       if (c->shadow)
         std::memcpy(tmp.data(), c->h_shadow[layer], tmp.size());
