@@ -225,6 +225,9 @@ def main():
     ap.add_argument("--init-threads", type=int, default=16)
     ap.add_argument("--layers", type=int, default=0, help="override the depth (c4: L_max(host RAM))")
     ap.add_argument("--trace-out", default="", help="write a Chrome trace of the last profiled step")
+    ap.add_argument("--resident-fit-layers", type=int, default=-1,
+                    help="c3/c4: also time the all-resident model of the same width with this depth "
+                         "(SURVEY §8(d): the >=85%% bar denominator; -1: 36 for h=4096, 0: skip)")
     ap.add_argument("--slice-fetch", action="store_true",
                     help="N>1: NEXT-1 slice H2D + NVLink all-gather (SH_FLAG_SLICE_FETCH)")
     ap.add_argument("--attention", default="auto", choices=["auto", "flash", "cublas"],
@@ -296,7 +299,8 @@ def main():
             shm_name = "sh_" + hashlib.sha1(nccl_id).hexdigest()[:16]  # one host store for the box
         cpu_threads = cpu_threads or max(1, (os.cpu_count() or 1) // local_world)
 
-    def run(window, e2e: bool):
+    def run(window, e2e: bool, mc=mc):
+        L = mc.n_layers
         t_init = time.perf_counter()
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
             (sh.SH_FLAG_CPU_HARD | sh.SH_FLAG_DECOUPLE if cpu_hard else 0) | \
@@ -370,6 +374,12 @@ def main():
     res = None
     if not args.no_resident and w != L and args.config not in ("c3", "c4"):
         res = run(L, False)
+    fit = None
+    fit_layers = args.resident_fit_layers if args.resident_fit_layers >= 0 else (36 if h == 4096 else 0)
+    if args.config in ("c3", "c4") and fit_layers > 0 and not args.no_resident:
+        mc_fit = ModelConfig(fit_layers, h, nh, s, V)
+        fit = run(fit_layers, False, mc_fit)
+        fit["tflops"] = b * world * K / (fit["ms"] / 1e3) * s * mc_fit.flops_per_token() / 1e12
 
     def gmax(x):
         if world == 1:
@@ -453,6 +463,11 @@ def main():
     if r["e2e_ms"] is not None:
         line["e2e"] = {"value": b * world * K / (e2e_ms / 1e3), "unit": "samples/s",
                        "h2d_bytes_per_step": b * (s + 1) * 4, "d2h_bytes_per_step": 4}
+    if fit:
+        line["resident_fit"] = {"layers": fit_layers, "window": fit_layers, "model_tflops": fit["tflops"],
+                                "samples_per_s": b * world * K / (fit["ms"] / 1e3),
+                                "frac_model_tflops": line["model_tflops"] / fit["tflops"],
+                                "note": "same width, all layers GPU-resident (SURVEY §8(d) C4 bar: >= 0.85)"}
     if res:
         line["resident"] = {"window": L, "samples_per_s": b * world * K / (res_ms / 1e3),
                             "ms_per_step": res_ms / K, "frac_windowed_over_resident": res_ms / ms}
