@@ -299,6 +299,8 @@ struct sh_ctx {
 
   // ---- ring state (driver thread only, except *_pub / ready / landing_done)
   std::vector<int> slot_layer, layer_slot;
+  std::vector<int64_t> slot_last_use;  // global position of the occupant's latest compute (LRU tie-break)
+  int64_t pos_clock = 0;
   std::vector<cudaEvent_t> ev_param_free, ev_grad_done, ev_grad_free, ev_reduced;
   std::vector<int64_t> gradfree_gen, gradfree_waited;
   std::unique_ptr<std::atomic<int64_t>[]> gradfree_pub;
@@ -965,7 +967,10 @@ bool ensure_at(sh_ctx* c, int p, int cur, sh_status* st) {
     const int o = c->slot_layer[s];
     const int64_t nu = o < 0 ? kInf + 1 : next_use(c, o, cur);
     if (nu == kPinned || nu <= p) continue;
-    if (nu > best_nu) best_nu = nu, best = s;
+    // farthest next use (Belady); among equals (e.g. host layers done for this step) the least
+    // recently used, whose gradient offload was requested first and is most likely complete
+    if (nu > best_nu || (nu == best_nu && c->slot_last_use[s] < c->slot_last_use[best]))
+      best_nu = nu, best = s;
   }
   if (best < 0) return false;
   *st = issue_fetch(c, y, best, p);
@@ -987,6 +992,7 @@ sh_status pre_common(sh_ctx* c, int x, int pos) {
       break;
     }
   }
+  c->slot_last_use[c->layer_slot[x]] = ++c->pos_clock;
   if (c->arrive_gen[x] > c->compute_waited[x]) {
     const int64_t gen = c->arrive_gen[x];
     if (c->arrive_by_issuer[x] &&
@@ -1138,6 +1144,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
   cudaMemset(r, 0, (int64_t)n_slots * c->slot_bytes);
   const int old = c->n_slots;
   c->slot_layer.resize(n_slots, -1);
+  c->slot_last_use.resize(n_slots, 0);
   c->ev_param_free.resize(n_slots, nullptr);
   c->ev_grad_done.resize(n_slots, nullptr);
   c->ev_grad_free.resize(n_slots, nullptr);
