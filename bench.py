@@ -182,7 +182,7 @@ def run_reference(args, cfgname):
     if args.layers:
         L = args.layers
     if L == 0:  # same depth rule as the CUDA arm (L_max of this host's RAM)
-        L = c4_layers(h, args.grad_ring or 4, ranks_sharing=int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
+        L = c4_layers(h, args.grad_ring or 8, ranks_sharing=int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
@@ -276,9 +276,9 @@ def main():
         if args.layers:
             L = args.layers
         elif not use_shm and world > 1:
-            L = c4_layers(h, args.grad_ring or 4, budget=mem_available() // local_world)
+            L = c4_layers(h, args.grad_ring or 8, budget=mem_available() // local_world)
         else:
-            L = c4_layers(h, args.grad_ring or 4, ranks_sharing=local_world)
+            L = c4_layers(h, args.grad_ring or 8, ranks_sharing=local_world)
         if world > 1:  # every rank must build the same model
             lt = torch.tensor([L], dtype=torch.int64, device="cuda")
             dist.broadcast(lt, 0)
@@ -289,7 +289,9 @@ def main():
 
     fetch32 = args.fetch_fp32 == 1 or (args.fetch_fp32 == -1 and args.config in FETCH_FP32_DEFAULT)
     cpu_hard = args.cpu_hard == 1 or (args.cpu_hard == -1 and args.config in CPU_HARD_DEFAULT)
-    grad_ring = args.grad_ring or (4 if args.config in ("c3", "c4") else 0)
+    # c3/c4 are host-RAM bound: 8 landing buffers (measured on C4: 4 -> 6.80, 8 -> 7.08, 12 -> 7.51
+    # samples/s at L = 83, 82, 80; profiles/r01_bench_c4_ring*.json)
+    grad_ring = args.grad_ring or (8 if args.config in ("c3", "c4") else 0)
 
     shm_name = None
     cpu_threads = args.cpu_threads
