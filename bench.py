@@ -228,6 +228,8 @@ def main():
     ap.add_argument("--resident-fit-layers", type=int, default=-1,
                     help="c3/c4: also time the all-resident model of the same width with this depth "
                          "(SURVEY §8(d): the >=85%% bar denominator; -1: 36 for h=4096, 0: skip)")
+    ap.add_argument("--fp-only", action="store_true",
+                    help="NEXT-4: time FP-only streaming passes (KD-teacher inference, PAPER.md:357-368)")
     ap.add_argument("--slice-fetch", action="store_true",
                     help="N>1: NEXT-1 slice H2D + NVLink all-gather (SH_FLAG_SLICE_FETCH)")
     ap.add_argument("--attention", default="auto", choices=["auto", "flash", "cublas"],
@@ -318,9 +320,10 @@ def main():
         host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + K)])
         host = host.pin_memory()
         dev = host.to(f"cuda:{local}")
+        step_fn = tr.forward_only if args.fp_only else tr.step_device
         for t in range(W):
             tr.tok_dev.copy_(dev[t])
-            tr.step_device()
+            step_fn()
         tr.engine.synchronize()
         st0 = tr.engine.stats()
         l0 = sh.kernel_launches() + G.kernel_launches()
@@ -333,7 +336,7 @@ def main():
             for t in range(W, W + K):
                 with torch.cuda.stream(tr.stream):
                     tr.tok_dev.copy_(dev[t], non_blocking=True)
-                tr.step_device()
+                step_fn()
             tr.engine.synchronize()
             ev1.record(tr.stream)
             torch.cuda.synchronize()
@@ -342,7 +345,7 @@ def main():
         st1 = tr.engine.stats()
         loss = tr.loss()
         e2e_ms = None
-        if e2e:
+        if e2e and not args.fp_only:
             if world > 1:
                 dist.barrier()
             torch.cuda.synchronize()
@@ -411,8 +414,10 @@ def main():
     d2h_gbs = d["d2h_profiled_bytes"] / (d["d2h_busy_ms"] / 1e3) / 1e9 if d["d2h_busy_ms"] > 0 else None
     flops_tok = mc.flops_per_token()
     tokens_s = samples * s
+    if args.fp_only:  # FP-only passes: 2 flop/param/token for the layers + the head forward
+        flops_tok = 2 * mc.n_layers * mc.params_per_layer() + 2 * h * V
     line = {
-        "metric": METRIC,
+        "metric": METRIC if not args.fp_only else "samples/s, FP-only streaming inference (NEXT-4)",
         "value": samples, "unit": "samples/s", "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "bf16" if prec == sh.SH_BF16_MIXED else "f32", "data": "synthetic",
