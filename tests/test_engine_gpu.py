@@ -311,3 +311,31 @@ def test_ring_smaller_than_gpu_set_bitwise(precision):
         assert ok, what
     finally:
         tr.close()
+
+
+@pytest.mark.parametrize("precision,window", [(sh.SH_BF16_MIXED, 1), (sh.SH_FP32, 2)])
+def test_checkpoint_resume_bitwise(precision, window):
+    """Save after 2 steps (sh_read_layer: master, m, v of every layer and the resident set), restore
+    into a fresh engine (sh_register_host_store with m, v and step=2, so Adam's bias correction
+    continues at t=3) and train one more step: identical to an uninterrupted 3-step run."""
+    from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
+    L = TINY["L"]
+    full, _, _ = engine_run(TINY, 3, window, precision)
+    want = engine_state(full)
+    full.close()
+    first, _, _ = engine_run(TINY, 2, window, precision)
+    saved = {what: [first.read_layer_tensors(i, what) for i in range(L)] + [first.read_layer_tensors(-1, what)]
+             for what in (sh.SH_READ_PARAM, sh.SH_READ_M, sh.SH_READ_V)}
+    first.close()
+    mc = T.ModelConfig(L, TINY["h"], TINY["nh"], TINY["s"], TINY["V"])
+    tr = T.StrongholdTrainer(mc, batch=TINY["b"], window=window, precision=precision, init=False)
+    try:
+        p, m, v = saved[sh.SH_READ_PARAM], saved[sh.SH_READ_M], saved[sh.SH_READ_V]
+        tr.register_state(p[:L], p[L], m[:L], v[:L], m[L], v[L], step=2)
+        tr.set_tokens(synth.tokens(2, TINY["b"], TINY["s"], TINY["V"]))
+        tr.step_device(want_norm=True)
+        ok, what = states_bitwise_equal(engine_state(tr), want)
+        assert ok, what
+        assert tr.engine.stats()["step"] == 3
+    finally:
+        tr.close()
