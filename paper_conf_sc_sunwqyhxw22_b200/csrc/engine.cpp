@@ -306,6 +306,13 @@ struct sh_ctx {
   std::unique_ptr<std::atomic<int64_t>[]> gradfree_pub;
   std::vector<cudaEvent_t> ev_arrive;
   std::vector<cudaEvent_t> ev_upd;  // [L] after the latest K2 of a GPU-optimised layer (K1 restage waits)
+  // no clipping: GPU-optimised layers write their grads into a small rotation of dedicated HBM
+  // buffers (not the ring's grad halves, which may still be queued for offload) consumed by their
+  // per-layer K2 on a side stream
+  std::vector<float*> gbuf;
+  std::vector<cudaEvent_t> ev_gbuf_free, ev_gbuf_ready;
+  std::vector<int> gbuf_owner, layer_gbuf;
+  int64_t gbuf_rr = 0;
   std::vector<int64_t> arrive_gen, compute_waited;
   std::vector<uint8_t> arrive_by_issuer;
   std::unique_ptr<std::atomic<int64_t>[]> arrive_pub;
@@ -1127,6 +1134,32 @@ sh_status ensure_host_layer(sh_ctx* c, int x) {
   return SH_OK;
 }
 
+sh_status ensure_gbufs(sh_ctx* c, int w) {
+  if (!c->k2_layer || w <= 0) return SH_OK;
+  const int want = std::min(std::max(w, 2), 4);
+  while ((int)c->gbuf.size() < want) {
+    float* p = nullptr;
+    if (cudaMalloc(&p, 4 * c->max_pad) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("cudaMalloc of a GPU-optimised-layer grad buffer (%lld B) failed", (long long)(4 * c->max_pad));
+      return SH_ERR_OOM_DEVICE;
+    }
+    cudaEvent_t a = nullptr, b = nullptr;
+    if (cudaEventCreateWithFlags(&a, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&b, cudaEventDisableTiming) != cudaSuccess) {
+      set_error("cudaEventCreate failed");
+      return SH_ERR_CUDA;
+    }
+    cudaEventRecord(a, c->cs);
+    c->gbuf.push_back(p);
+    c->ev_gbuf_free.push_back(a);
+    c->ev_gbuf_ready.push_back(b);
+    c->gbuf_owner.push_back(-1);
+    c->device_bytes += 4 * c->max_pad;
+  }
+  return SH_OK;
+}
+
 sh_status alloc_ring(sh_ctx* c, int n_slots) {
   if (n_slots <= c->n_slots) return SH_OK;
   char* r = nullptr;
@@ -1221,6 +1254,8 @@ sh_status apply_window(sh_ctx* c, int w_new) {
     CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
   }
   st = alloc_ring(c, c->ring_for(w_new));
+  if (st != SH_OK) return st;
+  st = ensure_gbufs(c, w_new);
   if (st != SH_OK) return st;
   c->w = w_new;
   c->n_active = c->ring_for(w_new);
@@ -1539,6 +1574,11 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->ring_cap = cfg->ring_slots > 0 ? cfg->ring_slots : 0;
   c->n_active = c->ring_for(w0);
   c->d = c->n_active - 1;
+  c->layer_gbuf.assign(c->L, -1);
+  {
+    sh_status s = ensure_gbufs(c.get(), w0);
+    if (s != SH_OK) return s;
+  }
   {
     sh_status s = alloc_ring(c.get(), c->n_active);
     if (s != SH_OK) return s;
@@ -1720,18 +1760,26 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
     st = pre_common(c, x, pos);
     if (st != SH_OK) return st;
     const int s = c->layer_slot[x];
-    if (c->gradfree_gen[s] > c->gradfree_waited[s]) {
+    float* gdst = c->slot_grad(s);
+    if (c->is_g(x) && c->k2_layer) {
+      // dedicated grad buffer: no wait on this slot's pending offload
+      const int b = (int)(c->gbuf_rr++ % (int64_t)c->gbuf.size());
+      c->layer_gbuf[x] = b;
+      c->gbuf_owner[b] = x;
+      CKC(c, cudaStreamWaitEvent(c->cs, c->ev_gbuf_free[b], 0));  // its previous K2 consumed it
+      gdst = c->gbuf[b];
+    } else if (c->gradfree_gen[s] > c->gradfree_waited[s]) {
       const int64_t gen = c->gradfree_gen[s];
       if (!state_wait(c, [&] { return c->gradfree_pub[s].load() >= gen; }, "gradient offload issue"))
         return check_failed(c);
       CKC(c, cudaStreamWaitEvent(c->cs, c->ev_grad_free[s], 0));
       c->gradfree_waited[s] = gen;
     }
-    CKC(c, cudaMemsetAsync(c->slot_grad(s), 0, 4 * c->lay[x].n_pad, c->cs));
+    CKC(c, cudaMemsetAsync(gdst, 0, 4 * c->lay[x].n_pad, c->cs));
     if (ProfSet* P = cur_prof(c)) CKC(c, cudaEventRecord(P->bp0[x], c->cs));
     fill_param_ptrs(c, x, dev_params);
     const LayerLayout& Lx = c->lay[x];
-    for (int k = 0; k < Lx.n_tensors; ++k) dev_grads[k] = c->slot_grad(s) + Lx.offset[k];
+    for (int k = 0; k < Lx.n_tensors; ++k) dev_grads[k] = gdst + Lx.offset[k];
     c->last_layer = x;
     c->last_hook = SH_PRE;
   } else if (phase == SH_POST) {
@@ -1748,7 +1796,55 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
     }
     CKC(c, cudaEventRecord(c->ev_param_free[s], c->cs));
     cudaEvent_t grads_ready = c->ev_grad_done[s];
-    if (c->W > 1) {
+    if (c->is_g(x) && c->k2_layer) {
+      // GPU-optimised layer, no clipping: grads in its dedicated buffer b; [W>1: all-reduce];
+      // K3; per-layer K2 (bitwise the same as a step-end update) on a side stream -- the stage
+      // stream (single GPU) or the comm stream (data parallel, in order after the collective) --
+      // so the compute stream goes straight on to the next layer.  The next uses of the slot (a
+      // fetch into it, the next FP of the layer) and of the buffer wait on events recorded after K2.
+      const int b = c->layer_gbuf[x];
+      float* gb = c->gbuf[b];
+      cudaStream_t ks = c->W > 1 ? c->comm : c->stage;
+      if (c->W > 1) {
+        CKC(c, cudaEventRecord(c->ev_gbuf_ready[b], c->cs));
+        CKC(c, cudaStreamWaitEvent(c->comm, c->ev_gbuf_ready[b], 0));
+        if (!c->no_collective) {
+          st = nccl_check(c, g_nccl.AllReduce(gb, gb, n, ncclFloat, ncclAvg, c->nccl, c->comm),
+                          "ncclAllReduce(layer grads)");
+          if (st != SH_OK) return st;
+        }
+        CKC(c, kern::sumsq(gb, n, c->scratch_comm, c->partials + x, c->comm));
+      } else {
+        if (P) CKC(c, cudaEventRecord(P->k30[x], c->cs));
+        CKC(c, kern::sumsq(gb, n, c->scratch_cs, c->partials + x, c->cs));
+        if (P) {
+          CKC(c, cudaEventRecord(P->k31[x], c->cs));
+          P->rec_k3[x] = 1;
+        }
+        CKC(c, cudaEventRecord(c->ev_gbuf_ready[b], c->cs));
+        CKC(c, cudaStreamWaitEvent(ks, c->ev_gbuf_ready[b], 0));
+      }
+      if (P) CKC(c, cudaEventRecord(P->k2l0[x], ks));
+      kern::K2Args a{};
+      a.sc = c->sc;
+      a.coef = nullptr;
+      a.out_bf16 = c->bf16;
+      a.n_entries = 1;
+      a.e[0] = kern::K2Entry{c->g[x].master, c->g[x].m, c->g[x].v, gb, c->slot_param(s), n, c->lay[x].n_decay};
+      CKC(c, kern::adamw_multi(a, ks));
+      if (P) {
+        CKC(c, cudaEventRecord(P->k2l1[x], ks));
+        P->rec_k2l[x] = 1;
+      }
+      CKC(c, cudaEventRecord(c->ev_param_free[s], ks));  // param half rewritten by K2
+      CKC(c, cudaEventRecord(c->ev_upd[x], ks));
+      CKC(c, cudaEventRecord(c->ev_gbuf_free[b], ks));
+      CKC(c, cudaEventRecord(c->ev_arrive[x], ks));     // the next FP of x waits for its update
+      const int64_t g2 = ++c->gen;
+      c->arrive_gen[x] = g2;
+      c->arrive_by_issuer[x] = 0;
+      c->arrive_pub[x].store(g2);
+    } else if (c->W > 1) {
       // data parallel: average this layer's grads across ranks before the offload (K-e)
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
       CKC(c, cudaStreamWaitEvent(c->comm, c->ev_grad_done[s], 0));
@@ -1761,7 +1857,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_comm, c->partials + x, c->comm));
       CKC(c, cudaEventRecord(c->ev_reduced[s], c->comm));
       grads_ready = c->ev_reduced[s];
-    } else if (c->is_g(x)) {
+    } else if (c->is_g(x)) {  // clip mode: grads stay in the slot until sh_step's K2
       if (P) CKC(c, cudaEventRecord(P->k30[x], c->cs));
       CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_cs, c->partials + x, c->cs));
       if (P) {
@@ -1772,40 +1868,6 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
     } else {
       // host layer: K3 runs on the D2H stream right before the offload (off the compute stream)
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
-    }
-    if (c->is_g(x) && c->k2_layer) {
-      // per-layer K2 of a GPU-optimised layer right after its backward (no clipping: the update
-      // needs no global norm; bitwise the same as the step-end K2).  Single GPU: on the compute
-      // stream, in order.  Data parallel: on the comm stream after the all-reduce and K3, so the
-      // compute stream does not wait for the collective; the next use of the slot (a fetch into it,
-      // the next FP of the layer, the next occupant's grad half) waits on events recorded after it.
-      cudaStream_t ks = c->W > 1 ? c->comm : c->cs;
-      if (P) CKC(c, cudaEventRecord(P->k2l0[x], ks));
-      kern::K2Args a{};
-      a.sc = c->sc;
-      a.coef = nullptr;
-      a.out_bf16 = c->bf16;
-      a.n_entries = 1;
-      a.e[0] = kern::K2Entry{c->g[x].master, c->g[x].m, c->g[x].v, c->slot_grad(s), c->slot_param(s), n,
-                             c->lay[x].n_decay};
-      CKC(c, kern::adamw_multi(a, ks));
-      if (P) {
-        CKC(c, cudaEventRecord(P->k2l1[x], ks));
-        P->rec_k2l[x] = 1;
-      }
-      CKC(c, cudaEventRecord(c->ev_param_free[s], ks));  // param half rewritten by K2
-      CKC(c, cudaEventRecord(c->ev_upd[x], ks));
-      if (ks != c->cs) {
-        CKC(c, cudaEventRecord(c->ev_grad_free[s], ks));
-        const int64_t g1 = ++c->gen;
-        c->gradfree_gen[s] = g1;
-        c->gradfree_pub[s].store(g1);
-        CKC(c, cudaEventRecord(c->ev_arrive[x], ks));
-        const int64_t g2 = ++c->gen;
-        c->arrive_gen[x] = g2;
-        c->arrive_by_issuer[x] = 0;
-        c->arrive_pub[x].store(g2);
-      }
     }
     const bool k3_on_d2h = c->W == 1 && !c->is_g(x);
     if (!c->is_g(x)) {
@@ -2178,6 +2240,14 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
   if (what == SH_READ_GRAD) {  // gradients of the last completed step
     if (layer < 0) {
       CKC(c, cudaMemcpy(tmp.data(), c->res_grad, 4 * n, cudaMemcpyDeviceToHost));
+    } else if (c->is_g(layer) && c->k2_layer) {
+      const int b = c->layer_gbuf[layer];
+      if (b < 0 || c->gbuf_owner[b] != layer) {
+        set_error("sh_read_layer: grads of layer %d were overwritten (%d GPU-layer grad buffers)", layer,
+                  (int)c->gbuf.size());
+        return SH_ERR_STATE;
+      }
+      CKC(c, cudaMemcpy(tmp.data(), c->gbuf[b], 4 * n, cudaMemcpyDeviceToHost));
     } else if (c->is_g(layer)) {
       if (c->layer_slot[layer] < 0) {
         set_error("sh_read_layer: grads of layer %d not available", layer);
@@ -2274,6 +2344,9 @@ sh_status sh_destroy(sh_ctx* c) {
   if (c->nccl_fetch) g_nccl.CommDestroy(c->nccl_fetch);
   if (c->nccl) g_nccl.CommDestroy(c->nccl);
   for (int x = 0; x < c->L; ++x) free_g(c, x);
+  for (float* p : c->gbuf) cudaFree(p);
+  for (auto e : c->ev_gbuf_free) cudaEventDestroy(e);
+  for (auto e : c->ev_gbuf_ready) cudaEventDestroy(e);
   if (c->ring) cudaFree(c->ring);
   if (c->res_master) cudaFree(c->res_master);
   if (c->partials) cudaFree(c->partials);
