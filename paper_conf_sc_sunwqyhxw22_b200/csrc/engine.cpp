@@ -234,7 +234,8 @@ struct sh_ctx {
   int64_t max_pad = 0;
   int64_t slot_param_bytes = 0, slot_grad_bytes = 0, slot_bytes = 0;
   int w = 0;
-  int n_slots = 0;   // allocated
+  int n_slots = 0;   // slots with bookkeeping (grow-only)
+  int ring_alloc = 0;  // slots currently allocated (0 while a regrow failed)
   int n_active = 0;  // slots in use = min(w + 1, ring cap)
   int d = 0;         // prefetch distance = n_active - 1 (the paper's window m when the ring is w+1)
   int ring_cap = 0;  // sh_config.ring_slots / sh_set_window_ring (0: w + 1)
@@ -1135,8 +1136,8 @@ sh_status ensure_host_layer(sh_ctx* c, int x) {
 }
 
 sh_status ensure_gbufs(sh_ctx* c, int w) {
-  if (!c->k2_layer || w <= 0) return SH_OK;
-  const int want = std::min(std::max(w, 2), 4);
+  if (!c->k2_layer || (w <= 0 && c->cfg.window == 0)) return SH_OK;
+  const int want = std::min(std::max(w, 4), 4);  // 4 up front: the window solver sees them as used
   while ((int)c->gbuf.size() < want) {
     float* p = nullptr;
     if (cudaMalloc(&p, 4 * c->max_pad) != cudaSuccess) {
@@ -1160,19 +1161,37 @@ sh_status ensure_gbufs(sh_ctx* c, int w) {
   return SH_OK;
 }
 
+// Grow-only ring.  Called with the engine idle: every slot's content can be
+// re-derived (GPU-optimised layers from their HBM masters, host layers from the host store), so
+// the old ring is released BEFORE the new one is allocated (never both at once).  On failure the
+// ring is left unallocated and the caller retries with fewer slots.
 sh_status alloc_ring(sh_ctx* c, int n_slots) {
-  if (n_slots <= c->n_slots) return SH_OK;
+  if (c->ring && n_slots <= c->n_slots) return SH_OK;
+  if (c->ring) {
+    cudaDeviceSynchronize();
+    cudaFree(c->ring);
+    c->device_bytes -= (int64_t)c->ring_alloc * c->slot_bytes;
+    c->ring = nullptr;
+    c->ring_alloc = 0;
+  }
+  n_slots = std::max(n_slots, c->n_slots);  // events / bookkeeping never shrink
   char* r = nullptr;
   if (cudaMalloc(&r, (int64_t)n_slots * c->slot_bytes) != cudaSuccess) {
     cudaGetLastError();
+    // put the previous ring back (it fitted before) so the context stays usable
+    if (c->n_slots > 0 && cudaMalloc(&r, (int64_t)c->n_slots * c->slot_bytes) == cudaSuccess) {
+      c->ring = r;
+      c->ring_alloc = c->n_slots;
+      c->device_bytes += (int64_t)c->n_slots * c->slot_bytes;
+    } else {
+      cudaGetLastError();
+      async_fail(c, SH_ERR_OOM_DEVICE, "ring re-allocation failed");
+    }
     set_error("cudaMalloc of %d ring slots (%lld B each) failed", n_slots, (long long)c->slot_bytes);
     return SH_ERR_OOM_DEVICE;
   }
-  if (c->ring) {
-    cudaFree(c->ring);
-    c->device_bytes -= (int64_t)c->n_slots * c->slot_bytes;
-  }
   c->ring = r;
+  c->ring_alloc = n_slots;
   c->device_bytes += (int64_t)n_slots * c->slot_bytes;
   cudaMemset(r, 0, (int64_t)n_slots * c->slot_bytes);
   const int old = c->n_slots;
@@ -1244,17 +1263,21 @@ sh_status apply_window(sh_ctx* c, int w_new) {
       }
     if (!shm_barrier(c, 3, "window change (counters)")) return check_failed(c);
   }
-  // joining G: host store -> HBM
+  // ring first (the old one is released inside), then the joining layers' HBM states (rolled
+  // back on failure so the caller can retry with a smaller window)
+  st = alloc_ring(c, c->ring_for(w_new));
+  if (st != SH_OK) return st;
   for (int x = w_old; x < w_new; ++x) {
     st = alloc_g(c, x);
-    if (st != SH_OK) return st;
+    if (st != SH_OK) {
+      for (int y = w_old; y < w_new; ++y) free_g(c, y);
+      return st;
+    }
     const int64_t n = c->lay[x].n_pad;
     CKC(c, cudaMemcpy(c->g[x].master, c->h_master[x], 4 * n, cudaMemcpyHostToDevice));
     CKC(c, cudaMemcpy(c->g[x].m, c->h_m[x], 4 * n, cudaMemcpyHostToDevice));
     CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
   }
-  st = alloc_ring(c, c->ring_for(w_new));
-  if (st != SH_OK) return st;
   st = ensure_gbufs(c, w_new);
   if (st != SH_OK) return st;
   c->w = w_new;
@@ -2102,7 +2125,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   size_t fr = 0, tot = 0;
   cudaMemGetInfo(&fr, &tot);
   // S_avail = what the engine holds now (ring + G states) + what is still free - margin
-  int64_t held = (int64_t)c->n_slots * c->slot_bytes;
+  int64_t held = (int64_t)c->ring_alloc * c->slot_bytes;
   for (int x = 0; x < c->L; ++x)
     if (c->g[x].master) held += 12 * c->lay[x].n_pad;
   o->s_avail = c->cfg.device_budget_bytes > 0 ? c->cfg.device_budget_bytes
@@ -2188,8 +2211,17 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
     ring = (int32_t)(v >> 32);
     if (!shm_barrier(c, 5, "autotuned window read")) return check_failed(c);
   }
-  if (wout) *wout = w;
-  return sh_set_window_ring(c, w, ring);
+  // apply; if HBM turns out short (the solver's S_avail is an estimate), step the window down
+  const int w_old = c->w;
+  st = sh_set_window_ring(c, w, ring);
+  while (st == SH_ERR_OOM_DEVICE && w > w_old) {
+    --w;
+    if (ring > 0) ring = std::min(ring, w + 1);
+    st = sh_set_window_ring(c, w, ring);
+  }
+  if (st == SH_ERR_OOM_DEVICE) st = sh_set_window_ring(c, w_old, 0);  // restore the warm-up window
+  if (wout) *wout = c->w;
+  return st;
 }
 
 sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
@@ -2283,7 +2315,7 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   if (c->phase == sh_ctx::IDLE) sync_all(c);
   o->step = c->step;
   o->window = c->w;
-  o->n_slots = c->n_slots;
+  o->n_slots = c->ring_alloc;
   o->host_bytes = (int64_t)c->host_bytes;
   o->device_bytes = c->device_bytes;
   o->h2d_bytes = c->h2d_bytes.load();
