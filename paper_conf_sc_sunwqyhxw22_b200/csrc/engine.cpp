@@ -268,6 +268,7 @@ struct sh_ctx {
   double* scratch_comm = nullptr;
   double* scratch_d2h = nullptr;
   cudaEvent_t ev_k3_last = nullptr;  // after the K3 of the latest host-layer offload (D2H stream)
+  cudaEvent_t ev_res_k3[2] = {nullptr, nullptr}, ev_norm[2] = {nullptr, nullptr};  // by step parity
   int64_t k3_last_gen = 0;            // generation of that offload request
   std::atomic<int64_t> k3_pub{0};     // latest generation whose K3 has been enqueued
   double* norm_dev = nullptr;
@@ -1421,6 +1422,10 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_cs_mark, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_k3_last, cudaEventDisableTiming));
+  for (int i = 0; i < 2; ++i) {
+    CKC(c.get(), cudaEventCreateWithFlags(&c->ev_res_k3[i], cudaEventDisableTiming));
+    CKC(c.get(), cudaEventCreateWithFlags(&c->ev_norm[i], cudaEventDisableTiming));
+  }
   if (W > 1) CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
   if (W > 1 && !c->no_collective) {
     if (!g_nccl.load()) {
@@ -1827,7 +1832,9 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       // fetch into it, the next FP of the layer) and of the buffer wait on events recorded after K2.
       const int b = c->layer_gbuf[x];
       float* gb = c->gbuf[b];
-      cudaStream_t ks = c->W > 1 ? c->comm : c->stage;
+      // (single GPU: on the compute stream -- measured on C4, K2 running beside the next layer's
+      // GEMMs slows them by about as much as it saves, and in order its roofline stays clean)
+      cudaStream_t ks = c->W > 1 ? c->comm : c->cs;
       if (c->W > 1) {
         CKC(c, cudaEventRecord(c->ev_gbuf_ready[b], c->cs));
         CKC(c, cudaStreamWaitEvent(c->comm, c->ev_gbuf_ready[b], 0));
@@ -1844,8 +1851,10 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
           CKC(c, cudaEventRecord(P->k31[x], c->cs));
           P->rec_k3[x] = 1;
         }
-        CKC(c, cudaEventRecord(c->ev_gbuf_ready[b], c->cs));
-        CKC(c, cudaStreamWaitEvent(ks, c->ev_gbuf_ready[b], 0));
+        if (ks != c->cs) {
+          CKC(c, cudaEventRecord(c->ev_gbuf_ready[b], c->cs));
+          CKC(c, cudaStreamWaitEvent(ks, c->ev_gbuf_ready[b], 0));
+        }
       }
       if (P) CKC(c, cudaEventRecord(P->k2l0[x], ks));
       kern::K2Args a{};
@@ -2006,13 +2015,30 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     CKC(c, cudaStreamWaitEvent(c->cs, c->ev_comm_done, 0));
   } else {
     CKC(c, kern::sumsq(c->res_grad, c->res.n_pad, c->scratch_cs, c->partials + L, c->cs));
-    if (c->w < L) {  // the host layers' K3 ran on the D2H stream: wait for the last one only
+  }
+  bool norm_on_d2h = false;
+  if (c->W == 1 && c->w < L && !c->clip) {
+    // no clipping: nothing on the compute stream needs the norm.  Finalize it on the D2H stream
+    // behind the host layers' K3s, queued on the D2H issuer, so the driver never waits for the
+    // issuer (which may be held back by landing-buffer waits) at the step boundary.
+    const int par = (int)(c->step & 1);
+    CKC(c, cudaEventRecord(c->ev_res_k3[par], c->cs));
+    cudaEvent_t rk = c->ev_res_k3[par], nd = c->ev_norm[par];
+    const double mx = c->cfg.max_grad_norm;
+    c->id2h.push([c, rk, nd, L, mx] {
+      CKA(c, cudaStreamWaitEvent(c->d2h, rk, 0));
+      CKA(c, kern::norm_finalize(c->partials, L + 1, mx, c->norm_dev, c->coef_dev, c->d2h));
+      CKA(c, cudaEventRecord(nd, c->d2h));
+    });
+    norm_on_d2h = true;
+  } else {
+    if (c->W == 1 && c->w < L) {  // clip mode: K2 needs the coefficient -- wait for the last K3
       const int64_t gen = c->k3_last_gen;
       if (!state_wait(c, [&] { return c->k3_pub.load() >= gen; }, "last K3 issue")) return check_failed(c);
       CKC(c, cudaStreamWaitEvent(c->cs, c->ev_k3_last, 0));
     }
+    CKC(c, kern::norm_finalize(c->partials, L + 1, c->cfg.max_grad_norm, c->norm_dev, c->coef_dev, c->cs));
   }
-  CKC(c, kern::norm_finalize(c->partials, L + 1, c->cfg.max_grad_norm, c->norm_dev, c->coef_dev, c->cs));
   ProfSet* P = cur_prof(c);
   if (P) CKC(c, cudaEventRecord(P->k2a, c->cs));
   kern::K2Args a{};
@@ -2072,6 +2098,10 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
   }
   if (grad_norm_out) {
     CKC(c, cudaStreamSynchronize(c->cs));
+    if (norm_on_d2h) {
+      c->id2h.drain();
+      CKC(c, cudaEventSynchronize(c->ev_norm[(c->step - 1) & 1]));
+    }
     CKC(c, cudaMemcpy(grad_norm_out, c->norm_dev, 8, cudaMemcpyDeviceToHost));
   }
   return check_failed(c);
@@ -2397,6 +2427,10 @@ sh_status sh_destroy(sh_ctx* c) {
   if (c->ev_cs_mark) cudaEventDestroy(c->ev_cs_mark);
   if (c->ev_comm_done) cudaEventDestroy(c->ev_comm_done);
   if (c->ev_k3_last) cudaEventDestroy(c->ev_k3_last);
+  for (int i = 0; i < 2; ++i) {
+    if (c->ev_res_k3[i]) cudaEventDestroy(c->ev_res_k3[i]);
+    if (c->ev_norm[i]) cudaEventDestroy(c->ev_norm[i]);
+  }
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
     if (s) cudaStreamDestroy(s);
   for (auto& b : c->hblocks) host_block_free(b.p, b.bytes);
