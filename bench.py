@@ -235,6 +235,11 @@ def main():
     ap.add_argument("--attention", default="auto", choices=["auto", "flash", "cublas"],
                     help="attention core of the GPT driver (outside the hot path)")
     ap.add_argument("--cpu-hard", type=int, default=-1, help="1: autotune with the eq. 3 CPU constraint")
+    ap.add_argument("--spill-dir", default="", help="NEXT-2: directory of the file-backed tier (PAPER.md:219-221)")
+    ap.add_argument("--host-pin-gb", type=float, default=0.0,
+                    help="NEXT-2: pinned host-store budget in GB (layers beyond it spill to --spill-dir)")
+    ap.add_argument("--executors", type=int, default=1,
+                    help="NEXT-3: K multi-stream executors (micro-batches of batch/K on K streams, PAPER.md:227-242)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -313,7 +318,8 @@ def main():
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
-                               attention=args.attention)
+                               attention=args.attention, executors=args.executors,
+                               spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9))
         attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
@@ -429,6 +435,9 @@ def main():
                    "precision": "bf16_mixed" if prec else "fp32",
                    "gpt_driver_attention": r["attn"],
                    "parallelism": f"dp{world}",
+                   "executors": args.executors,
+                   "spill": {"dir": args.spill_dir, "layers": r["st1"]["spilled_layers"],
+                             "bytes": r["st1"]["spill_bytes"]} if args.spill_dir else None,
                    "host_store": ("one shared /dev/shm store, rank-sliced offload + CPU Adam" if shm_name else
                                   "private per rank") if world > 1 else "private",
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),

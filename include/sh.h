@@ -143,6 +143,30 @@ typedef struct {
   const char* shm_name;             /* world_size > 1: name of ONE shared host store for all ranks of the
                                        box (/dev/shm); rank r offloads and CPU-updates only
                                        slice r of every layer.  NULL/"": a private replica per rank */
+  int32_t n_executors;              /* NEXT-3 multi-stream executors (Fig. 5): K >= 2
+                                       concurrent training workers on one GPU share ONE copy of every
+                                       layer's parameters (the ring slot) and each computes a micro-batch
+                                       on its own stream; executor e >= 1 writes its gradients into the
+                                       engine-owned buffers of sh_executor_grads, and the engine's K4
+                                       kernel averages them into executor 0's buffers ("an all-reduce
+                                       operation to synchronize the gradients among parallel training
+                                       workers before performing parameter updates") at
+                                       the backward POST (layers) and at sh_step (resident set).
+                                       0 or 1: a single worker.  At most 8. */
+  const char* spill_dir;            /* NEXT-2 secondary-storage tier: NULL/"" = off.
+                                       Otherwise a directory (NVMe or any file system): host-optimised
+                                       layers whose pinned block would exceed host_pin_budget_bytes, or
+                                       for which pinned host RAM runs out, are kept in files there,
+                                       memory-mapped (MAP_SHARED) instead of pinned ("memory-mapping a
+                                       swap file on the secondary storage to the CPU memory space").
+                                       Their prefetches are copied through two pinned bounce buffers,
+                                       the CPU Adam updates them through the page cache (read-ahead
+                                       started when the layer's gradients land, write-back started
+                                       when its update finishes).  Results are bit-identical to the
+                                       all-pinned store.  Files are created O_EXCL, unlinked at once,
+                                       space reserved with posix_fallocate.  Not with shm_name. */
+  int64_t host_pin_budget_bytes;    /* cap on pinned host-store bytes (layer blocks + landing ring);
+                                       0 = no cap (spill only when pinning fails for lack of RAM) */
 } sh_config;
 
 /* Per-layer profile consumed by the window solver (PAPER.md:132 notation; times in ms,
@@ -210,6 +234,8 @@ typedef struct {
      |copy ∩ compute| / |copy| with compute = union of the per-layer FP/BP compute intervals */
   double h2d_overlap_frac, d2h_overlap_frac;
   double last_step_ms;          /* first FP hook .. end of K2 of that step (GPU time) */
+  int64_t spill_bytes;          /* NEXT-2: bytes of host-optimised layer state in spill files */
+  int32_t spilled_layers;       /* number of layers in the spill tier */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */
@@ -264,6 +290,19 @@ sh_status sh_backward_layer(sh_ctx* ctx, int32_t layer, int32_t phase, void** de
  * are zeroed at the first forward hook of every step. */
 sh_status sh_resident(sh_ctx* ctx, void** dev_params, float** dev_grads);
 
+/* NEXT-3 executors (sh_config.n_executors = K >= 2).  Writes the n_tensors fp32 gradient
+ * pointers of executor `executor` (0..K-1) for `layer` -- which must be between its
+ * sh_backward_layer PRE and POST -- or for the resident set (layer -1, any time in a step).
+ * Executor 0's are the pointers the hooks / sh_resident return; executors >= 1 get
+ * engine-owned buffers, zeroed on the compute stream at the PRE (layers) or the first forward
+ * hook (resident set).  Contract: every executor's work on a layer is enqueued after its PRE
+ * was issued on the compute stream and joined back into the compute stream (an event wait)
+ * before the POST; every executor works on an equal share of the batch and computes the
+ * gradient of its own micro-batch MEAN loss.  At the POST (sh_step for the resident set) K4
+ * computes g = (((g_0 + g_1) + g_2) + ... + g_{K-1}) * fp32(1/K), a fixed order, so results stay
+ * bit-identical across windows.  Library-owned; valid until the POST / next sh_step. */
+sh_status sh_executor_grads(sh_ctx* ctx, int32_t layer, int32_t executor, float** dev_grads);
+
 /* FP-only pass (NEXT-4: streaming inference of a model larger than HBM, e.g. the teacher of
  * knowledge distillation): call after sh_forward_layer(L-1, SH_POST) instead of
  * the backward hooks.  Nothing is updated, the step counter does not advance and every layer copy
@@ -317,7 +356,7 @@ const char* sh_last_error(void);
 
 int32_t sh_abi_version(void);
 
-/* Number of engine kernel launches (K1, K2, K3, norm finalize) since the library was loaded. */
+/* Number of engine kernel launches (K1, K2, K3, K4, norm finalize) since the library was loaded. */
 int64_t sh_kernel_launches(void);
 
 /* Rank 0 of a data-parallel job: fill a 128-byte ncclUniqueId (dlopen'ed libnccl.so.2, the
@@ -354,6 +393,11 @@ sh_status sh_op_cast_bf16_gpu(const float* src, uint16_t* dst16, int64_t n, void
 
 /* CPU rne_bf16 (the shadow writer of the CPU Adam). */
 sh_status sh_op_cast_bf16_cpu(const float* src, uint16_t* dst16, int64_t n);
+
+/* K4 (NEXT-3): dst[i] = (((dst[i] + src[0][i]) + src[1][i]) + ... + src[n_src-1][i]) * inv_k,
+ * every op IEEE fp32 round-to-nearest; src is a HOST array of n_src (0..7) device pointers. */
+sh_status sh_op_exec_reduce_gpu(float* dst, const float* const* src, int32_t n_src, int64_t n, float inv_k,
+                                void* stream);
 
 /* K3: out[0] = Σ g[i]^2 accumulated in fp64 with a fixed reduction tree (deterministic). */
 sh_status sh_op_sumsq_gpu(const float* g, int64_t n, double* out_dev, void* stream);

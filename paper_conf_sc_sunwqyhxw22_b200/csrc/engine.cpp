@@ -262,6 +262,12 @@ struct sh_ctx {
   char* ring = nullptr;
   std::vector<GState> g;  // [L]
   float *res_master = nullptr, *res_m = nullptr, *res_v = nullptr, *res_grad = nullptr;
+  // NEXT-3 multi-stream executors: executor e >= 1 writes its micro-batch
+  // gradients into xgrad[e-1] (layer in BP) / xres[e-1] (resident set); K4 folds them into
+  // executor 0's buffers (the engine's own) at the backward POST / sh_step
+  int K = 1;
+  std::vector<float*> xgrad, xres;
+  float* cur_gdst = nullptr;  // executor 0's grad buffer of the layer between backward PRE and POST
   void* res_compute = nullptr;
   double* partials = nullptr;  // [L+1]
   double* scratch_cs = nullptr;
@@ -280,10 +286,23 @@ struct sh_ctx {
   struct HostBlock {
     char* p = nullptr;
     size_t bytes = 0;
+    int fd = -1;  // NEXT-2: >= 0 for a file-backed (spilled, pageable) block
   };
   std::vector<HostBlock> hblocks;  // [L]
   HostBlock hland;
   size_t host_bytes = 0;
+  // NEXT-2 secondary-storage tier: host-optimised layers beyond the pinned
+  // budget live in mmap'ed files (MAP_SHARED, unlinked at creation) under spill_dir; their
+  // fetches go through pinned bounce buffers, the CPU Adam works on the mapping (page cache)
+  std::string spill_dir;
+  int64_t pin_budget = 0;
+  size_t spill_bytes = 0;
+  int n_spilled = 0;
+  std::vector<uint8_t> spilled;  // [L]
+  char* bounce[2] = {nullptr, nullptr};
+  size_t bounce_bytes = 0;
+  cudaEvent_t ev_bounce[2] = {nullptr, nullptr};
+  int bounce_rr = 0;  // H2D issuer thread only
   bool shadow = true;  // bf16 shadow kept in host RAM (bf16 mode without SH_FLAG_FETCH_FP32)
   // shared store (world_size > 1 with shm_name): rank r owns elements [slo[x], shi[x]) of layer x
   bool shared = false;
@@ -553,6 +572,10 @@ void host_block_free(char* p, size_t bytes) {
 
 // ---------------------------------------------------------------------------- CPU Adam pool
 void finish_job(sh_ctx* c, Job* j) {
+  if (c->spilled[j->layer]) {  // start the write-back of the updated states now (async bulk write)
+    const auto& hb = c->hblocks[j->layer];
+    sync_file_range(hb.fd, 0, (off64_t)hb.bytes, SYNC_FILE_RANGE_WRITE);
+  }
   c->ready[j->layer].store(j->step + 1, std::memory_order_release);
   if (c->shared) c->ctl->cnt[j->layer].fetch_add(1, std::memory_order_release);
   c->landing_done[j->landing].fetch_add(1, std::memory_order_release);
@@ -634,6 +657,10 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
   std::unique_ptr<Landed> L(static_cast<Landed*>(arg));
   sh_ctx* c = L->c;
   if (c->shared) c->ctl->cnt[c->L + L->layer].fetch_add(1, std::memory_order_release);
+  if (c->spilled[L->layer]) {  // spilled layer: start reading its master / m / v before the CPU Adam
+    const auto& hb = c->hblocks[L->layer];
+    madvise(hb.p, hb.bytes, MADV_WILLNEED);
+  }
   auto j = std::make_unique<Job>();
   j->layer = L->layer;
   j->step = L->step;
@@ -935,9 +962,18 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
     if (poison) CKA(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->h2d));
     char* buf = cast ? reinterpret_cast<char*>(stage_buf) : dst;
     const char* hsrc = static_cast<const char*>(src);
+    if (c->spilled[y]) {
+      // NEXT-2: pageable source -> CPU copy into a pinned bounce buffer (reads the file through the
+      // page cache; overlaps the previous layer's H2D from the other buffer) -> async H2D
+      const int k = c->bounce_rr++ & 1;
+      CKA(c, cudaEventSynchronize(c->ev_bounce[k]));  // its previous H2D has finished
+      std::memcpy(c->bounce[k], hsrc, bytes);
+      hsrc = c->bounce[k];
+    }
     if (P) CKA(c, cudaEventRecord(P->c2g0[ph][y], c->h2d));
     if (!slice) {
-      CKA(c, cudaMemcpyAsync(buf, src, bytes, cudaMemcpyHostToDevice, c->h2d));
+      CKA(c, cudaMemcpyAsync(buf, hsrc, bytes, cudaMemcpyHostToDevice, c->h2d));
+      if (c->spilled[y]) CKA(c, cudaEventRecord(c->ev_bounce[(c->bounce_rr - 1) & 1], c->h2d));
     } else if (shi > slo) {
       CKA(c, cudaMemcpyAsync(buf + eb * slo, hsrc + eb * slo, eb * (shi - slo), cudaMemcpyHostToDevice, c->h2d));
     }
@@ -1118,16 +1154,85 @@ sh_status shm_map(sh_ctx* c, const std::string& path, size_t bytes, bool create,
 
 // Host block of layer x: [master | m | v | shadow?], 2 MiB aligned.  Shared stores map the
 // segment rank 0 created (all layers are created collectively in sh_init).
+// NEXT-2: file-backed block in spill_dir (the paper's "memory-mapping a swap file on the secondary
+// storage").  The file is unlinked right away (the mapping keeps it; nothing is left
+// behind on a crash); space is reserved with posix_fallocate so a full disk fails here, not with a
+// SIGBUS inside the CPU Adam.
+sh_status spill_block_alloc(sh_ctx* c, int x, size_t bytes, char** out, int* fd_out) {
+  *out = nullptr;
+  *fd_out = -1;
+  char path[4096];
+  snprintf(path, sizeof(path), "%s/sh_spill_%d_%p_%d.bin", c->spill_dir.c_str(), (int)getpid(), (void*)c, x);
+  const int fd = open(path, O_RDWR | O_CREAT | O_EXCL, 0600);
+  if (fd < 0) {
+    set_error("spill tier: open(%s): %s", path, strerror(errno));
+    return SH_ERR_OOM_HOST;
+  }
+  unlink(path);
+  const int e = posix_fallocate(fd, 0, (off_t)bytes);
+  if (e != 0) {
+    close(fd);
+    set_error("spill tier: posix_fallocate of %lld B in %s: %s", (long long)bytes, c->spill_dir.c_str(), strerror(e));
+    return SH_ERR_OOM_HOST;
+  }
+  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  if (p == MAP_FAILED) {
+    close(fd);
+    set_error("spill tier: mmap of %lld B failed: %s", (long long)bytes, strerror(errno));
+    return SH_ERR_OOM_HOST;
+  }
+  *out = static_cast<char*>(p);
+  *fd_out = fd;
+  return SH_OK;
+}
+
+sh_status ensure_bounce(sh_ctx* c) {
+  if (c->bounce[0]) return SH_OK;
+  const size_t b = align_up(4 * c->max_pad, 1 << 21);  // fp32 fetch is the largest
+  for (int k = 0; k < 2; ++k) {
+    sh_status st = host_block_alloc(b, c->n_threads, &c->bounce[k]);
+    if (st != SH_OK) return st;
+    CKC(c, cudaEventCreateWithFlags(&c->ev_bounce[k], cudaEventDisableTiming));
+    CKC(c, cudaEventRecord(c->ev_bounce[k], c->h2d));
+    c->host_bytes += b;
+  }
+  c->bounce_bytes = b;
+  return SH_OK;
+}
+
 sh_status ensure_host_layer(sh_ctx* c, int x) {
   if (c->h_master[x]) return SH_OK;
   const int64_t n = c->lay[x].n_pad;
   const size_t bytes = align_up(12 * n + (c->shadow ? 2 * n : 0), 1 << 21);
   char* p = nullptr;
-  sh_status st = c->shared ? shm_map(c, shm_path(c, "L", x), bytes, c->rank == 0, &p, true)
-                           : host_block_alloc(bytes, c->n_threads, &p);
+  int fd = -1;
+  sh_status st = SH_OK;
+  if (c->shared) {
+    st = shm_map(c, shm_path(c, "L", x), bytes, c->rank == 0, &p, true);
+  } else {
+    const bool can_spill = !c->spill_dir.empty();
+    bool spill = can_spill && c->pin_budget > 0 && (int64_t)(c->host_bytes + bytes) > c->pin_budget;
+    if (!spill) {
+      st = host_block_alloc(bytes, c->n_threads, &p);
+      if (st == SH_ERR_OOM_HOST && can_spill) {  // host RAM exhausted: overflow to the spill tier
+        clear_error();
+        spill = true;
+      }
+    }
+    if (spill) {
+      st = ensure_bounce(c);
+      if (st == SH_OK) st = spill_block_alloc(c, x, bytes, &p, &fd);
+    }
+  }
   if (st != SH_OK) return st;
-  c->hblocks[x] = {p, bytes};
-  c->host_bytes += bytes;
+  c->hblocks[x] = {p, bytes, fd};
+  if (fd >= 0) {
+    c->spilled[x] = 1;
+    c->spill_bytes += bytes;
+    c->n_spilled++;
+  } else {
+    c->host_bytes += bytes;
+  }
   float* b = reinterpret_cast<float*>(p);
   c->h_master[x] = b;
   c->h_m[x] = b + n;
@@ -1290,6 +1395,18 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   return SH_OK;
 }
 
+// K4 on the compute stream: dst = (dst + Σ_e src[e]) / K in a fixed order (NEXT-3).
+sh_status exec_fold(sh_ctx* c, float* dst, const std::vector<float*>& src, int64_t n) {
+  kern::K4Args a{};
+  a.dst = dst;
+  a.n_src = (int)src.size();
+  for (int e = 0; e < a.n_src; ++e) a.src[e] = src[e];
+  a.n = n;
+  a.inv_k = (float)(1.0 / (double)c->K);
+  CKC(c, kern::exec_reduce(a, c->cs));
+  return SH_OK;
+}
+
 sh_status push_k2(sh_ctx* c, kern::K2Args& a, int64_t* bytes, int* launches) {
   if (a.n_entries == 0) return SH_OK;
   for (int i = 0; i < a.n_entries; ++i) *bytes += (c->bf16 ? 30 : 32) * a.e[i].n;
@@ -1379,8 +1496,13 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     set_error("sh_init: world_size > 1 needs nccl_unique_id and 0 <= rank < world_size");
     return SH_ERR_INVALID;
   }
+  if (cfg->n_executors < 0 || cfg->n_executors > kern::kMaxExecutors) {
+    set_error("sh_init: n_executors %d outside 0..%d", cfg->n_executors, kern::kMaxExecutors);
+    return SH_ERR_INVALID;
+  }
   auto c = std::make_unique<sh_ctx>();
   c->cfg = *cfg;
+  c->K = cfg->n_executors > 1 ? cfg->n_executors : 1;
   c->L = cfg->n_layers;
   c->W = W;
   c->rank = cfg->rank;
@@ -1453,6 +1575,20 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   if (c->n_threads < 1) c->n_threads = 1;
   c->shadow = c->bf16 && !(cfg->flags & SH_FLAG_FETCH_FP32);
   c->hblocks.assign(c->L, {});
+  c->spilled.assign(c->L, 0);
+  if (cfg->spill_dir && cfg->spill_dir[0]) {
+    if (c->shared) {
+      set_error("sh_init: spill_dir is not supported with a shared (multi-rank) host store");
+      return SH_ERR_INVALID;
+    }
+    struct stat sb;
+    if (stat(cfg->spill_dir, &sb) != 0 || !S_ISDIR(sb.st_mode)) {
+      set_error("sh_init: spill_dir %s is not a directory", cfg->spill_dir);
+      return SH_ERR_INVALID;
+    }
+    c->spill_dir = cfg->spill_dir;
+  }
+  c->pin_budget = cfg->host_pin_budget_bytes > 0 ? cfg->host_pin_budget_bytes : 0;
   c->h_master.assign(c->L, nullptr);
   c->h_m.assign(c->L, nullptr);
   c->h_v.assign(c->L, nullptr);
@@ -1561,6 +1697,19 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->scratch_d2h = c->scratch_comm + kern::kSumsqMaxBlocks + 1;
     c->norm_dev = c->scratch_d2h + kern::kSumsqMaxBlocks + 1;
     c->coef_dev = reinterpret_cast<float*>(c->norm_dev + 1);
+    for (int e = 1; e < c->K; ++e) {  // executor gradient buffers (one set: K4 runs in stream order)
+      float* xg = nullptr;
+      float* xr = nullptr;
+      if (cudaMalloc(&xg, 4 * c->max_pad) != cudaSuccess || cudaMalloc(&xr, 4 * n) != cudaSuccess) {
+        cudaGetLastError();
+        if (xg) cudaFree(xg);
+        set_error("sh_init: cudaMalloc of executor %d gradient buffers failed", e);
+        return SH_ERR_OOM_DEVICE;
+      }
+      c->xgrad.push_back(xg);
+      c->xres.push_back(xr);
+      c->device_bytes += 4 * (c->max_pad + n);
+    }
   }
   c->g.assign(c->L, GState{});
   c->layer_slot.assign(c->L, -1);
@@ -1733,6 +1882,7 @@ sh_status sh_forward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_param
         P.rec_t0 = true;
       }
       CKC(c, cudaMemsetAsync(c->res_grad, 0, 4 * c->res.n_pad, c->cs));
+      for (float* xr : c->xres) CKC(c, cudaMemsetAsync(xr, 0, 4 * c->res.n_pad, c->cs));
       c->phase = sh_ctx::FP;
     }
     st = pre_common(c, x, x);
@@ -1804,6 +1954,8 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       c->gradfree_waited[s] = gen;
     }
     CKC(c, cudaMemsetAsync(gdst, 0, 4 * c->lay[x].n_pad, c->cs));
+    for (float* xg : c->xgrad) CKC(c, cudaMemsetAsync(xg, 0, 4 * c->lay[x].n_pad, c->cs));
+    c->cur_gdst = gdst;
     if (ProfSet* P = cur_prof(c)) CKC(c, cudaEventRecord(P->bp0[x], c->cs));
     fill_param_ptrs(c, x, dev_params);
     const LayerLayout& Lx = c->lay[x];
@@ -1817,6 +1969,10 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
     }
     const int s = c->layer_slot[x];
     const int64_t n = c->lay[x].n_pad;
+    if (c->K > 1) {  // K4: fold the executors' micro-batch gradients (counted as BP compute)
+      st = exec_fold(c, c->cur_gdst, c->xgrad, n);
+      if (st != SH_OK) return st;
+    }
     ProfSet* P = cur_prof(c);
     if (P) {
       CKC(c, cudaEventRecord(P->bp1[x], c->cs));
@@ -1970,6 +2126,30 @@ sh_status sh_resident(sh_ctx* c, void** dev_params, float** dev_grads) {
   return SH_OK;
 }
 
+sh_status sh_executor_grads(sh_ctx* c, int32_t layer, int32_t executor, float** dev_grads) {
+  clear_error();
+  if (!c || !dev_grads) return SH_ERR_INVALID;
+  sh_status st = check_failed(c);
+  if (st != SH_OK) return st;
+  if (executor < 0 || executor >= c->K) {
+    set_error("sh_executor_grads: executor %d outside 0..%d", executor, c->K - 1);
+    return SH_ERR_INVALID;
+  }
+  if (layer < 0) {
+    float* base = executor == 0 ? c->res_grad : c->xres[executor - 1];
+    for (int k = 0; k < c->res.n_tensors; ++k) dev_grads[k] = base + c->res.offset[k];
+    return SH_OK;
+  }
+  if (!(c->phase == sh_ctx::BP && c->last_hook == SH_PRE && layer == c->last_layer)) {
+    set_error("sh_executor_grads(%d): layer must be between its backward PRE and POST", layer);
+    return SH_ERR_STATE;
+  }
+  float* base = executor == 0 ? c->cur_gdst : c->xgrad[executor - 1];
+  const LayerLayout& Lx = c->lay[layer];
+  for (int k = 0; k < Lx.n_tensors; ++k) dev_grads[k] = base + Lx.offset[k];
+  return SH_OK;
+}
+
 sh_status sh_forward_only_end(sh_ctx* c) {
   clear_error();
   if (!c) return SH_ERR_INVALID;
@@ -2000,6 +2180,10 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     return SH_ERR_STATE;
   }
   const int L = c->L;
+  if (c->K > 1) {
+    st = exec_fold(c, c->res_grad, c->xres, c->res.n_pad);
+    if (st != SH_OK) return st;
+  }
   if (c->W > 1) {
     // resident grads: average too, on the comm stream after the caller's embedding backward
     CKC(c, cudaEventRecord(c->ev_cs_mark, c->cs));
@@ -2374,6 +2558,8 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->h2d_overlap_frac = c->h2d_overlap;
   o->d2h_overlap_frac = c->d2h_overlap;
   o->last_step_ms = c->last_step_ms;
+  o->spill_bytes = (int64_t)c->spill_bytes;
+  o->spilled_layers = c->n_spilled;
   return SH_OK;
 }
 
@@ -2407,6 +2593,8 @@ sh_status sh_destroy(sh_ctx* c) {
   if (c->nccl) g_nccl.CommDestroy(c->nccl);
   for (int x = 0; x < c->L; ++x) free_g(c, x);
   for (float* p : c->gbuf) cudaFree(p);
+  for (float* p : c->xgrad) cudaFree(p);
+  for (float* p : c->xres) cudaFree(p);
   for (auto e : c->ev_gbuf_free) cudaEventDestroy(e);
   for (auto e : c->ev_gbuf_ready) cudaEventDestroy(e);
   if (c->ring) cudaFree(c->ring);
@@ -2433,7 +2621,18 @@ sh_status sh_destroy(sh_ctx* c) {
   }
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
     if (s) cudaStreamDestroy(s);
-  for (auto& b : c->hblocks) host_block_free(b.p, b.bytes);
+  for (auto& b : c->hblocks) {
+    if (b.fd >= 0) {
+      munmap(b.p, b.bytes);
+      close(b.fd);
+    } else {
+      host_block_free(b.p, b.bytes);
+    }
+  }
+  for (int k = 0; k < 2; ++k) {
+    host_block_free(c->bounce[k], c->bounce_bytes);
+    if (c->ev_bounce[k]) cudaEventDestroy(c->ev_bounce[k]);
+  }
   if (c->ctl) munmap(c->ctl, c->ctl_bytes);
   host_block_free(c->hland.p, c->hland.bytes);
   delete c;
@@ -2508,6 +2707,30 @@ sh_status sh_op_cast_bf16_cpu(const float* src, uint16_t* dst16, int64_t n) {
   clear_error();
   if (!src || !dst16 || n < 0) return SH_ERR_INVALID;
   cpu::cast_bf16_range(src, dst16, 0, n);
+  return SH_OK;
+}
+
+sh_status sh_op_exec_reduce_gpu(float* dst, const float* const* src, int32_t n_src, int64_t n, float inv_k,
+                                void* stream) {
+  clear_error();
+  if (n_src < 0 || n_src >= kern::kMaxExecutors || (n_src > 0 && !src)) {
+    set_error("sh_op_exec_reduce_gpu: n_src %d outside 0..%d", n_src, kern::kMaxExecutors - 1);
+    return SH_ERR_INVALID;
+  }
+  kern::K4Args a{};
+  a.dst = dst;
+  a.n_src = n_src;
+  for (int e = 0; e < n_src; ++e) a.src[e] = src[e];
+  a.n = n;
+  a.inv_k = inv_k;
+  const void* ptrs[kern::kMaxExecutors + 1] = {dst};
+  for (int e = 0; e < n_src; ++e) ptrs[e + 1] = src[e];
+  if (!ops_args_ok(n, 0, ptrs, n_src + 1)) return SH_ERR_INVALID;
+  const cudaError_t e = kern::exec_reduce(a, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) {
+    set_error("sh_op_exec_reduce_gpu: %s", cudaGetErrorString(e));
+    return SH_ERR_CUDA;
+  }
   return SH_OK;
 }
 

@@ -8,6 +8,10 @@
 //                  new compute copy in place.  HBM-bound: 30 B/element (bf16 mode).
 //  K3 sumsq        per-layer Σg² in fp64 with a fixed reduction tree (grad-norm for clipping;
 //                  deterministic, no float atomics).  HBM-bound: 4 B/element.
+//  K4 exec_reduce  the in-GPU all-reduce of the multi-stream executors (NEXT-3, PAPER.md:236-240:
+//                  "an all-reduce operation to synchronize the gradients among parallel training
+//                  workers before performing parameter updates"): g0 = (((g0+g1)+g2)+...)*inv_k
+//                  in a fixed order.  HBM-bound: 4(k+1) B/element.
 //
 // None of these is a contraction, so there is no tensor-core work here: the rules that matter
 // are 128-bit coalesced accesses, enough bytes in flight per SM, and a grid sized in
@@ -200,6 +204,28 @@ __global__ void __launch_bounds__(256) k3_sumsq_kernel(const float* __restrict__
   }
 }
 
+// K4: 8 elements (2 float4) per thread per iteration; the k-1 executor buffers are streamed
+// (read once, L1 no-allocate), the destination is read and written in place.
+__global__ void __launch_bounds__(256) k4_exec_reduce_kernel(const __grid_constant__ K4Args a) {
+  const int64_t n8 = a.n / 8;
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n8;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    float4 x0 = ld_rw(a.dst + 8 * j), x1 = ld_rw(a.dst + 8 * j + 4);
+    for (int s = 0; s < a.n_src; ++s) {
+      const float4 y0 = ld_stream(a.src[s] + 8 * j), y1 = ld_stream(a.src[s] + 8 * j + 4);
+      x0.x = __fadd_rn(x0.x, y0.x); x0.y = __fadd_rn(x0.y, y0.y);
+      x0.z = __fadd_rn(x0.z, y0.z); x0.w = __fadd_rn(x0.w, y0.w);
+      x1.x = __fadd_rn(x1.x, y1.x); x1.y = __fadd_rn(x1.y, y1.y);
+      x1.z = __fadd_rn(x1.z, y1.z); x1.w = __fadd_rn(x1.w, y1.w);
+    }
+    const float f = a.inv_k;
+    x0.x = __fmul_rn(x0.x, f); x0.y = __fmul_rn(x0.y, f); x0.z = __fmul_rn(x0.z, f); x0.w = __fmul_rn(x0.w, f);
+    x1.x = __fmul_rn(x1.x, f); x1.y = __fmul_rn(x1.y, f); x1.z = __fmul_rn(x1.z, f); x1.w = __fmul_rn(x1.w, f);
+    st_f4(a.dst + 8 * j, x0);
+    st_f4(a.dst + 8 * j + 4, x1);
+  }
+}
+
 __global__ void norm_finalize_kernel(const double* __restrict__ partials, int n, double max_norm,
                                      double* norm_out, float* coef_out) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
@@ -283,6 +309,16 @@ cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaS
   launch_counter()++;
   unsigned int* ticket = reinterpret_cast<unsigned int*>(scratch + kSumsqMaxBlocks);
   k3_sumsq_kernel<<<(int)nb, 256, 0, st>>>(g, n4, scratch, ticket, out);
+  return cudaGetLastError();
+}
+
+cudaError_t exec_reduce(const K4Args& a, cudaStream_t st) {
+  const int64_t n8 = a.n / 8;
+  if (n8 == 0 || a.n_src < 0) return cudaSuccess;
+  const int64_t cap = (int64_t)sm_count() * 8;
+  const int64_t need = (n8 + 255) / 256;
+  launch_counter()++;
+  k4_exec_reduce_kernel<<<(int)(need < cap ? need : cap), 256, 0, st>>>(a);
   return cudaGetLastError();
 }
 

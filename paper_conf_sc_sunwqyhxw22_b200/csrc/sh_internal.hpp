@@ -67,6 +67,16 @@ cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaS
 // norm = sqrt(Σ partials[0..n)) in index order; coef = min(1, max_norm/(norm+1e-6)) (fp32)
 cudaError_t norm_finalize(const double* partials, int n, double max_norm, double* norm_out,
                           float* coef_out, cudaStream_t st);
+// K4 (NEXT-3 executors): dst = ((dst + src[0]) + src[1] + ...) * inv_k elementwise (n multiple of 8).
+constexpr int kMaxExecutors = 8;
+struct K4Args {
+  float* dst;
+  const float* src[kMaxExecutors];
+  int n_src;
+  int64_t n;
+  float inv_k;
+};
+cudaError_t exec_reduce(const K4Args& a, cudaStream_t st);
 int sm_count();
 int64_t launches();
 }  // namespace kern

@@ -30,7 +30,8 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_autotune_window", "sh_set_window", "sh_get_profile", "sh_read_layer", "sh_stats",
            "sh_last_error", "sh_abi_version", "sh_nccl_get_unique_id", "sh_adam_scalars_for",
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
-           "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end", "sh_set_window_ring")
+           "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end", "sh_set_window_ring",
+           "sh_executor_grads", "sh_op_exec_reduce_gpu")
 
 
 class ShError(RuntimeError):
@@ -51,7 +52,8 @@ class Config(C.Structure):
                 ("cpu_threads", C.c_int32), ("grad_ring_depth", C.c_int32), ("warmup_steps", C.c_int32),
                 ("device_budget_bytes", C.c_int64), ("cpu_util_max", C.c_double), ("ring_slots", C.c_int32),
                 ("world_size", C.c_int32), ("rank", C.c_int32),
-                ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p)]
+                ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p),
+                ("n_executors", C.c_int32), ("spill_dir", C.c_char_p), ("host_pin_budget_bytes", C.c_int64)]
 
 
 _PD = C.POINTER(C.c_double)
@@ -84,7 +86,8 @@ class Stats(C.Structure):
                 ("k2_launches_last", C.c_int32), ("cpu_threads", C.c_int32), ("profiled_steps", C.c_int32),
                 ("k2_ms_sum", C.c_double), ("k2_bytes_sum", C.c_int64), ("k2_samples", C.c_int64),
                 ("k3_ms_sum", C.c_double), ("k3_bytes_sum", C.c_int64), ("k3_samples", C.c_int64),
-                ("h2d_overlap_frac", C.c_double), ("d2h_overlap_frac", C.c_double), ("last_step_ms", C.c_double)]
+                ("h2d_overlap_frac", C.c_double), ("d2h_overlap_frac", C.c_double), ("last_step_ms", C.c_double),
+                ("spill_bytes", C.c_int64), ("spilled_layers", C.c_int32)]
 
 
 class TraceEvent(C.Structure):
@@ -130,6 +133,8 @@ def lib() -> C.CDLL:
             "sh_op_sumsq_gpu": [vp, i64, vp, vp],
             "sh_get_trace": [vp, vp, i32, C.POINTER(i32)],
             "sh_forward_only_end": [vp], "sh_set_window_ring": [vp, i32, i32],
+            "sh_executor_grads": [vp, i32, i32, vp],
+            "sh_op_exec_reduce_gpu": [vp, vp, i32, i64, f32, vp],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -195,6 +200,11 @@ def op_cast_bf16_cpu(src, dst16, n):
     check(lib().sh_op_cast_bf16_cpu(_ptr(src), _ptr(dst16), n))
 
 
+def op_exec_reduce_gpu(dst, srcs, n, inv_k, stream=None):
+    arr = (C.c_void_p * max(1, len(srcs)))(*[_ptr(x) for x in srcs])
+    check(lib().sh_op_exec_reduce_gpu(_ptr(dst), arr, len(srcs), n, inv_k, _stream_handle(stream)))
+
+
 def op_sumsq_gpu(g, n, out_dev, stream=None):
     check(lib().sh_op_sumsq_gpu(_ptr(g), n, _ptr(out_dev), _stream_handle(stream)))
 
@@ -256,7 +266,8 @@ class Engine:
                  lr=1.5e-4, betas=(0.9, 0.999), eps=1e-8, weight_decay=0.01, max_grad_norm=0.0, device=0,
                  stream=None, cpu_threads=0, grad_ring_depth=0, warmup_steps=5, device_budget_bytes=0,
                  world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None,
-                 ring_slots=0, cpu_util_max=0.0):
+                 ring_slots=0, cpu_util_max=0.0, n_executors=1, spill_dir: str | None = None,
+                 host_pin_budget_bytes=0):
         L = lib()
         self.n_layers = len(layer_numels)
         self._keep = []
@@ -291,6 +302,11 @@ class Engine:
             idbuf = (C.c_uint8 * 128).from_buffer_copy(nccl_id)
             cfg.nccl_unique_id = C.cast(idbuf, C.c_void_p)
         cfg.flags = flags
+        cfg.n_executors = n_executors
+        self._spill = spill_dir.encode() if spill_dir else None
+        cfg.spill_dir = self._spill
+        cfg.host_pin_budget_bytes = int(host_pin_budget_bytes)
+        self.n_executors = max(1, n_executors)
         self._shm = shm_name.encode() if shm_name else None
         cfg.shm_name = self._shm
         self.precision = precision
@@ -304,6 +320,11 @@ class Engine:
         self._rp = (C.c_void_p * len(res_numels))()
         self._rg = (C.c_void_p * len(res_numels))()
         check(L.sh_resident(self.h, self._rp, self._rg))
+        # executor e >= 1 gradient pointer arrays: per layer (filled at each backward PRE) and resident
+        self._xg = [[(C.c_void_p * len(n))() for n in self.layer_numels] for _ in range(self.n_executors)]
+        self._xr = [(C.c_void_p * len(res_numels))() for _ in range(self.n_executors)]
+        for e in range(1, self.n_executors):
+            check(L.sh_executor_grads(self.h, -1, e, self._xr[e]))
         self._L = L
 
     def _shape(self, nums, wds):
@@ -351,6 +372,17 @@ class Engine:
         a, g = self._p_arr[i], self._g_arr[i]
         check(self._L.sh_backward_layer(self.h, i, SH_PRE, a, g))
         return a, g
+
+    def executor_grads(self, i: int, e: int):
+        """Gradient pointers of executor e for layer i (between its backward PRE and POST)."""
+        if e == 0:
+            return self._g_arr[i]
+        g = self._xg[e][i] if 0 <= e < self.n_executors else (C.c_void_p * 64)()  # C reports the error
+        check(self._L.sh_executor_grads(self.h, i, e, g))
+        return g
+
+    def executor_resident_grads(self, e: int):
+        return self._rg if e == 0 else self._xr[e]
 
     def backward_post(self, i: int):
         check(self._L.sh_backward_layer(self.h, i, SH_POST, None, None))

@@ -53,9 +53,15 @@ class StrongholdTrainer:
     def __init__(self, mc: ModelConfig, *, batch: int, window: int, precision=sh.SH_BF16_MIXED, lr=1.5e-4,
                  max_grad_norm=0.0, device=0, seed=1234, cpu_threads=0, grad_ring_depth=0, warmup_steps=5,
                  flags=0, world_size=1, rank=0, nccl_id=None, init=True, init_threads=8, shm_name=None,
-                 attention="auto", ring_slots=0):
+                 attention="auto", ring_slots=0, executors=1, spill_dir=None, host_pin_budget_bytes=0):
         self.mc = mc
         self.batch = batch
+        # NEXT-3 multi-stream executors: K workers on K streams, one parameter copy,
+        # each on batch/K sequences; the engine's K4 averages their gradients before the update
+        self.K = max(1, int(executors))
+        if batch % self.K:
+            raise ValueError(f"batch {batch} is not a multiple of executors {self.K}")
+        self.mb = batch // self.K
         self.device = torch.device("cuda", device)
         torch.cuda.set_device(self.device)
         self.stream = torch.cuda.Stream(device=self.device)
@@ -65,20 +71,28 @@ class StrongholdTrainer:
                                 precision=precision, lr=lr, max_grad_norm=max_grad_norm, device=device,
                                 stream=self.stream, cpu_threads=cpu_threads, grad_ring_depth=grad_ring_depth,
                                 warmup_steps=warmup_steps, world_size=world_size, rank=rank, nccl_id=nccl_id,
-                                flags=flags, shm_name=shm_name, ring_slots=ring_slots)
-        self.gpt = GPT(n_layers=L, hidden=mc.hidden, heads=mc.heads, seq=mc.seq, max_batch=batch,
-                       vocab=mc.vocab, precision=precision, device=device, stream=self.stream)
+                                flags=flags, shm_name=shm_name, ring_slots=ring_slots, n_executors=self.K,
+                                spill_dir=spill_dir, host_pin_budget_bytes=host_pin_budget_bytes)
+        # executor 0 runs on the engine's compute stream, executors >= 1 on their own streams
+        self.streams = [self.stream] + [torch.cuda.Stream(device=self.device) for _ in range(self.K - 1)]
+        self.gpts = [GPT(n_layers=L, hidden=mc.hidden, heads=mc.heads, seq=mc.seq, max_batch=self.mb,
+                         vocab=mc.vocab, precision=precision, device=device, stream=st) for st in self.streams]
+        self.gpt = self.gpts[0]
         # attention core: fused flash-attention library kernel on the bf16 path ("auto"/"flash"),
         # else the cuBLAS batched-GEMM + softmax kernels inside libsh_gpt ("cublas", and fp32 mode)
-        self.flash = None
+        self.flashes = [None] * self.K
         if attention == "flash" or (attention == "auto" and precision == sh.SH_BF16_MIXED):
             try:
-                self.flash = FlashAttention(self.gpt, batch, mc.seq, mc.hidden, mc.heads)
+                self.flashes = [FlashAttention(g, self.mb, mc.seq, mc.hidden, mc.heads) for g in self.gpts]
             except ImportError:
                 if attention == "flash":
                     raise
+        self.flash = self.flashes[0]
+        self._fork = [torch.cuda.Event() for _ in range(2 * mc.n_layers + 2)]
+        self._join = [[torch.cuda.Event() for _ in range(2 * mc.n_layers + 2)] for _ in range(self.K)]
         self.tok_dev = torch.empty((batch, mc.seq + 1), dtype=torch.int32, device=self.device)
         self.loss_dev = torch.zeros(1, dtype=torch.float32, device=self.device)
+        self.loss_parts = torch.zeros(self.K, dtype=torch.float32, device=self.device)
         self.loss_host = torch.zeros(1, dtype=torch.float32).pin_memory()
         # with a shared host store only rank 0 writes the host-optimised layers' initial state
         self._w0 = window if window >= 0 else min(2, L)
@@ -110,69 +124,116 @@ class StrongholdTrainer:
                              None if v_res is None else flat(v_res), step)
 
     # ------------------------------------------------------------------ one step
+    def _run(self, k: int, fn):
+        """Run fn(e) for every executor e: executor 0 on the compute stream, executors >= 1 forked
+        from the compute stream's current position (after the hook just issued) on their own
+        streams and joined back before the next hook (the sh_executor_grads contract)."""
+        if self.K == 1:
+            fn(0)
+            return
+        cs = self.stream
+        self._fork[k].record(cs)
+        for e in range(1, self.K):
+            st = self.streams[e]
+            st.wait_event(self._fork[k])
+            with torch.cuda.stream(st):
+                fn(e)
+            self._join[e][k].record(st)
+        fn(0)
+        for e in range(1, self.K):
+            cs.wait_event(self._join[e][k])
+
+    def _tok(self, e: int, mb: int) -> int:
+        return self.tok_dev.data_ptr() + 4 * e * mb * (self.mc.seq + 1)
+
+    def _layer_fwd(self, e: int, i: int, P, write_out=True):
+        g, fa = self.gpts[e], self.flashes[e]
+        if fa is None:
+            if write_out:
+                g.layer_forward(i, P)
+            else:
+                raise AssertionError("recompute without flash goes through layer_backward")
+        else:
+            g.forward_qkv(i, P)
+            fa.forward()
+            g.forward_out(i, P, write_out)
+
     def step_device(self, batch: int | None = None, want_norm=False):
         """One training step on tokens already in self.tok_dev.  Asynchronous unless want_norm."""
-        e, g = self.engine, self.gpt
+        e = self.engine
         B = batch or self.batch
-        tok = self.tok_dev.data_ptr()
-        rp, rg = e.resident()
+        if B % self.K:
+            raise ValueError(f"batch {B} is not a multiple of executors {self.K}")
+        mb = B // self.K
         L = self.mc.n_layers
-        fa = self.flash
-        if fa is not None:
-            fa.set_batch(B)
+        for fa in self.flashes:
+            if fa is not None:
+                fa.set_batch(mb)
+        gp = self.gpts
+        loss = [self.loss_dev.data_ptr()] if self.K == 1 else \
+            [self.loss_parts.data_ptr() + 4 * x for x in range(self.K)]
         with torch.cuda.stream(self.stream):
             # FP (PAPER.md:108): pre_forward -> compute -> post_forward
             for i in range(L):
                 P = e.forward_pre(i)
-                if i == 0:
-                    g.embed_forward(tok, B, rp)
-                if fa is None:
-                    g.layer_forward(i, P)
-                else:
-                    g.forward_qkv(i, P)
-                    fa.forward()
-                    g.forward_out(i, P, True)
+
+                def fwd(x, i=i, P=P):
+                    if i == 0:
+                        gp[x].embed_forward(self._tok(x, mb), mb, e.resident()[0])
+                    self._layer_fwd(x, i, P)
+                self._run(i, fwd)
                 e.forward_post(i)
-            g.head(tok, rp, rg, self.loss_dev.data_ptr())
+            rp = e.resident()[0]
+            self._run(L, lambda x: gp[x].head(self._tok(x, mb), rp, e.executor_resident_grads(x), loss[x]))
             # BP (PAPER.md:111): pre_backward -> recompute + backward -> post (offload + CPU Adam)
             for i in range(L - 1, -1, -1):
-                P, G = e.backward_pre(i)
-                if fa is None:
-                    g.layer_backward(i, P, G)
-                else:
-                    g.forward_qkv(i, P)       # recompute from the layer's checkpoint
-                    fa.forward()
-                    g.forward_out(i, P, False)
-                    g.backward_mlp(i, P, G)
-                    fa.backward()
-                    g.backward_qkv(i, P, G)
+                P, _ = e.backward_pre(i)
+                Gs = [e.executor_grads(i, x) for x in range(self.K)]
+
+                def bwd(x, i=i, P=P):
+                    g, fa, G = gp[x], self.flashes[x], Gs[x]
+                    if fa is None:
+                        g.layer_backward(i, P, G)
+                    else:
+                        g.forward_qkv(i, P)       # recompute from the layer's checkpoint
+                        fa.forward()
+                        g.forward_out(i, P, False)
+                        g.backward_mlp(i, P, G)
+                        fa.backward()
+                        g.backward_qkv(i, P, G)
+                self._run(L + 1 + (L - 1 - i), bwd)
                 e.backward_post(i)
-            g.embed_backward(tok, rg)
+            self._run(2 * L + 1, lambda x: gp[x].embed_backward(self._tok(x, mb), e.executor_resident_grads(x)))
+            if self.K > 1:
+                torch.mean(self.loss_parts, dim=0, keepdim=True, out=self.loss_dev)  # loss report only
             return e.step(want_norm=want_norm)
 
     def forward_only(self, batch: int | None = None) -> None:
         """FP-only pass (streaming inference / KD teacher) over self.tok_dev:
         loss -> self.loss_dev; no backward, no update (NEXT-4)."""
-        e, g = self.engine, self.gpt
+        e = self.engine
         B = batch or self.batch
-        tok = self.tok_dev.data_ptr()
-        rp, _ = e.resident()
-        fa = self.flash
-        if fa is not None:
-            fa.set_batch(B)
+        mb = B // self.K
+        for fa in self.flashes:
+            if fa is not None:
+                fa.set_batch(mb)
+        gp = self.gpts
+        loss = [self.loss_dev.data_ptr()] if self.K == 1 else \
+            [self.loss_parts.data_ptr() + 4 * x for x in range(self.K)]
         with torch.cuda.stream(self.stream):
             for i in range(self.mc.n_layers):
                 P = e.forward_pre(i)
-                if i == 0:
-                    g.embed_forward(tok, B, rp)
-                if fa is None:
-                    g.layer_forward(i, P)
-                else:
-                    g.forward_qkv(i, P)
-                    fa.forward()
-                    g.forward_out(i, P, True)
+
+                def fwd(x, i=i, P=P):
+                    if i == 0:
+                        gp[x].embed_forward(self._tok(x, mb), mb, e.resident()[0])
+                    self._layer_fwd(x, i, P)
+                self._run(i, fwd)
                 e.forward_post(i)
-            g.head_forward(tok, rp, self.loss_dev.data_ptr())
+            rp = e.resident()[0]
+            self._run(self.mc.n_layers, lambda x: gp[x].head_forward(self._tok(x, mb), rp, loss[x]))
+            if self.K > 1:
+                torch.mean(self.loss_parts, dim=0, keepdim=True, out=self.loss_dev)
             e.forward_only_end()
 
     def step(self, tokens_host: torch.Tensor, want_norm=False) -> float:
@@ -209,7 +270,8 @@ class StrongholdTrainer:
 
     def close(self):
         self.engine.close()
-        self.gpt.close()
+        for g in self.gpts:
+            g.close()
 
 
 def bf16_bits_to_f32(u16: np.ndarray) -> np.ndarray:

@@ -47,13 +47,14 @@ def unit_errors(eng_layers, eng_res, st):
 
 def engine_run(cfg: dict, steps: int, window: int, precision: int, seed=1234, max_grad_norm=0.0, lr=1.5e-4,
                flags=0, tok_seed=1234, set_window_at=None, cpu_threads=0, grad_ring_depth=0, attention="auto",
-               ring_slots=0):
+               ring_slots=0, executors=1, **kw):
     """Run the CUDA path; returns (trainer, losses, norms) with the trainer still open."""
     from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
     mc = T.ModelConfig(cfg["L"], cfg["h"], cfg["nh"], cfg["s"], cfg["V"])
     tr = T.StrongholdTrainer(mc, batch=cfg["b"], window=window, precision=precision, lr=lr,
                              max_grad_norm=max_grad_norm, seed=seed, flags=flags, cpu_threads=cpu_threads,
-                             grad_ring_depth=grad_ring_depth, attention=attention, ring_slots=ring_slots)
+                             grad_ring_depth=grad_ring_depth, attention=attention, ring_slots=ring_slots,
+                             executors=executors, **kw)
     losses, norms = [], []
     for t in range(steps):
         if set_window_at and t in set_window_at:

@@ -98,3 +98,24 @@ def test_k3_sumsq_deterministic_and_exact(n):
     assert a.tobytes() == b.tobytes()
     exact = float(np.sum(g.astype(np.float64) ** 2))
     assert abs(a - exact) <= 1e-12 * exact
+
+
+@pytest.mark.parametrize("n,k", [(8, 2), (1 << 12, 3), ((1 << 22) + 8, 4), (201379840 // 64 * 8, 8)])
+def test_k4_exec_reduce_matches_plain_sum(n, k):
+    """K4 (NEXT-3 executor all-reduce): ((g0 + g1) + ...) * fp32(1/k), bitwise equal to
+    the same IEEE fp32 op sequence written with plain torch elementwise ops, and within fp32 rounding
+    of the exact fp64 mean."""
+    dev = torch.device("cuda")
+    gs = [torch.from_numpy(synth.normal(synth.stream_key(n + e, 11), n, 1e-3)).to(dev) for e in range(k)]
+    inv = np.float32(1.0 / k)
+    ref = gs[0].clone()
+    for e in range(1, k):
+        ref = ref + gs[e]
+    ref = ref * torch.tensor(inv, device=dev)
+    mean64 = sum(g.double() for g in gs) / k
+    dst = gs[0].clone()
+    sh.op_exec_reduce_gpu(dst, gs[1:], n, float(inv))
+    torch.cuda.synchronize()
+    assert torch.equal(dst.view(torch.int32), ref.view(torch.int32))
+    err = (dst.double() - mean64).abs().max().item()
+    assert err <= k * 2.0 ** -23 * mean64.abs().max().item() + 1e-30
