@@ -238,6 +238,7 @@ def main():
     ap.add_argument("--spill-dir", default="", help="NEXT-2: directory of the file-backed tier (PAPER.md:219-221)")
     ap.add_argument("--host-pin-gb", type=float, default=0.0,
                     help="NEXT-2: pinned host-store budget in GB (layers beyond it spill to --spill-dir)")
+    ap.add_argument("--spill-evict", action="store_true", help="NEXT-2: drop spilled layers from the page cache")
     ap.add_argument("--executors", type=int, default=1,
                     help="NEXT-3: K multi-stream executors (micro-batches of batch/K on K streams, PAPER.md:227-242)")
     args = ap.parse_args()
@@ -313,7 +314,8 @@ def main():
         t_init = time.perf_counter()
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
             (sh.SH_FLAG_CPU_HARD | sh.SH_FLAG_DECOUPLE if cpu_hard else 0) | \
-            (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0)
+            (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0) | \
+            (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
@@ -437,7 +439,7 @@ def main():
                    "parallelism": f"dp{world}",
                    "executors": args.executors,
                    "spill": {"dir": args.spill_dir, "layers": r["st1"]["spilled_layers"],
-                             "bytes": r["st1"]["spill_bytes"]} if args.spill_dir else None,
+                             "bytes": r["st1"]["spill_bytes"], "evict": args.spill_evict} if args.spill_dir else None,
                    "host_store": ("one shared /dev/shm store, rank-sliced offload + CPU Adam" if shm_name else
                                   "private per rank") if world > 1 else "private",
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),

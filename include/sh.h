@@ -113,6 +113,9 @@ typedef struct {
 #define SH_FLAG_DECOUPLE  (1ull << 9) /* autotuner: decouple the ring (prefetch distance) from the
                                          GPU-optimised set (needs no clipping and a landing buffer per
                                          layer, grad_ring_depth 0; R22) */
+#define SH_FLAG_SPILL_EVICT (1ull << 10) /* NEXT-2: after a spilled layer's CPU update, write it back and drop
+                                           it from the page cache (RAM held by the spill tier stays bounded;
+                                           every fetch / update of the layer reads the file) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

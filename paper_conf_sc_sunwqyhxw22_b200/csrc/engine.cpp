@@ -574,7 +574,16 @@ void host_block_free(char* p, size_t bytes) {
 void finish_job(sh_ctx* c, Job* j) {
   if (c->spilled[j->layer]) {  // start the write-back of the updated states now (async bulk write)
     const auto& hb = c->hblocks[j->layer];
-    sync_file_range(hb.fd, 0, (off64_t)hb.bytes, SYNC_FILE_RANGE_WRITE);
+    if (c->cfg.flags & SH_FLAG_SPILL_EVICT) {
+      // bounded RAM: write the layer back, then drop it from the page cache (the next fetch and
+      // update read it from the file again -- the paper's swap-file behaviour)
+      sync_file_range(hb.fd, 0, (off64_t)hb.bytes,
+                      SYNC_FILE_RANGE_WAIT_BEFORE | SYNC_FILE_RANGE_WRITE | SYNC_FILE_RANGE_WAIT_AFTER);
+      madvise(hb.p, hb.bytes, MADV_DONTNEED);
+      posix_fadvise(hb.fd, 0, (off_t)hb.bytes, POSIX_FADV_DONTNEED);
+    } else {
+      sync_file_range(hb.fd, 0, (off64_t)hb.bytes, SYNC_FILE_RANGE_WRITE);
+    }
   }
   c->ready[j->layer].store(j->step + 1, std::memory_order_release);
   if (c->shared) c->ctl->cnt[j->layer].fetch_add(1, std::memory_order_release);
@@ -1243,7 +1252,10 @@ sh_status ensure_host_layer(sh_ctx* c, int x) {
 
 sh_status ensure_gbufs(sh_ctx* c, int w) {
   if (!c->k2_layer || (w <= 0 && c->cfg.window == 0)) return SH_OK;
-  const int want = std::min(std::max(w, 4), 4);  // 4 up front: the window solver sees them as used
+  // allocated up front (the window solver sees them as used).  Single GPU: the per-layer K2 runs
+  // on the compute stream, in order, so two buffers never wait; data parallel: K2 runs on the comm
+  // stream behind the all-reduce, four keep BP from waiting on it
+  const int want = c->W > 1 ? 4 : 2;
   while ((int)c->gbuf.size() < want) {
     float* p = nullptr;
     if (cudaMalloc(&p, 4 * c->max_pad) != cudaSuccess) {

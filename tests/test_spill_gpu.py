@@ -30,7 +30,8 @@ def resident():
 
 
 @pytest.mark.parametrize("precision,flags", [(sh.SH_FP32, 0), (sh.SH_BF16_MIXED, 0),
-                                             (sh.SH_BF16_MIXED, sh.SH_FLAG_FETCH_FP32)])
+                                             (sh.SH_BF16_MIXED, sh.SH_FLAG_FETCH_FP32),
+                                             (sh.SH_FP32, sh.SH_FLAG_SPILL_EVICT)])
 @pytest.mark.parametrize("window", [0, 1])
 def test_spilled_bitwise_equals_resident(tmp_path, resident, precision, flags, window):
     ref, ref_losses, ref_norms = resident[precision]
