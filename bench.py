@@ -142,6 +142,17 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
+def k2_traffic(elems_per_launch: float):
+    """DRAM read+write bytes of one K2 launch: the per-element figure of the committed ncu --set full
+    capture (tools/ncu_kernels.sh -> tools/ncu_iso_summary.py) times this bench's elements per launch."""
+    p = os.path.join(ROOT, "profiles", "r01_ncu_iso_kernels.json")
+    try:
+        per = json.load(open(p))["k2_adamw"]["dram_bytes_per_elem"]
+    except Exception:  # noqa: BLE001
+        return None
+    return per * elems_per_launch
+
+
 def oracle_sample(L, h, nh, s, V, seed=1234):
     """Bounded CPU-oracle sample of the workload: one block fwd+bwd and its AdamW, plus the head
     (fwd+bwd) and the resident AdamW, at batch 1; extrapolated to one sample of the full model."""
@@ -463,14 +474,28 @@ def main():
             "peak_source": "profiles/r01_probe_box.json (pinned 1 GiB copies)"},
         "cpu_adam": {"threads": st1["cpu_threads"], "elems_per_step": d["cpu_adam_elems"] / K,
                      "thread_ms_per_step": d["cpu_adam_ms"] / K,
-                     "dram_gbs": 30.0 * d["cpu_adam_elems"] / (d["cpu_adam_ms"] / 1e3 / st1["cpu_threads"]) / 1e9
+                     "dram_gbs": (28 if fetch32 or not prec else 30) * d["cpu_adam_elems"] / (d["cpu_adam_ms"] / 1e3 / st1["cpu_threads"]) / 1e9
                      if d["cpu_adam_ms"] > 0 else None,
                      "prefetch_wait_ms_per_step": d["cpu_wait_ms"] / K,
                      "host_dram_triad_peak_gbs": PROBE_HOST_TRIAD_GBS,
                      "note": "dram_gbs counts the AdamW's 30 B/param (28 without shadow) while its threads run; "
                              "the copy engines' DMA shares the same host DRAM"},
+        # whole-step host-DRAM roofline: the CPU AdamW's bytes (28 B/param fp32-fetch, 30 with the bf16
+        # shadow: r p,m,v,g + w p,m,v [+ w shadow]) plus every DMA byte the copy engines move through
+        # host DRAM, over the step time, against the probe's 16-thread triad
+        "host_dram": {"bytes_per_step": ((28 if fetch32 or not prec else 30) * d["cpu_adam_elems"]
+                                         + d["h2d_bytes"] + d["d2h_bytes"]) / K,
+                      "achieved_gbs": ((28 if fetch32 or not prec else 30) * d["cpu_adam_elems"]
+                                       + d["h2d_bytes"] + d["d2h_bytes"]) / (ms / 1e3) / 1e9,
+                      "peak_gbs": PROBE_HOST_TRIAD_GBS,
+                      "frac": ((28 if fetch32 or not prec else 30) * d["cpu_adam_elems"]
+                               + d["h2d_bytes"] + d["d2h_bytes"]) / (ms / 1e3) / 1e9 / PROBE_HOST_TRIAD_GBS,
+                      "peak_source": "profiles/r01_probe_box.json (STREAM triad, 16 threads)"},
         "roofline": {"kernel": "K2 fused multi-tensor AdamW (sh_step)", "bound": "hbm", "achieved": k2_gbs,
-                     "peak": peak, "unit": "GB/s", "frac": k2_gbs / peak if k2_gbs else None, "traffic": None,
+                     "peak": peak, "unit": "GB/s", "frac": k2_gbs / peak if k2_gbs else None,
+                     "traffic": k2_traffic(d["k2_bytes_sum"] / max(1, d["k2_samples"]) / (30 if prec else 32)),
+                     "traffic_source": "profiles/r01_ncu_iso_kernels.json: ncu --set full DRAM bytes/element of an "
+                                       "isolated K2 launch (one h=4096 layer) x elements per launch",
                      "peak_source": peak_kind, "algorithmic_bytes_per_elem": 30 if prec else 32,
                      "bytes_per_launch": d["k2_bytes_sum"] / max(1, d["k2_samples"]),
                      "k3_sumsq_gbs": k3_gbs, "k3_frac": k3_gbs / peak if k3_gbs else None},

@@ -116,6 +116,9 @@ typedef struct {
 #define SH_FLAG_SPILL_EVICT (1ull << 10) /* NEXT-2: after a spilled layer's CPU update, write it back and drop
                                            it from the page cache (RAM held by the spill tier stays bounded;
                                            every fetch / update of the layer reads the file) */
+#define SH_FLAG_TEST_DP_PATH (1ull << 11) /* test: take the data-parallel path at world_size 1 (one-rank NCCL
+                                            communicator from nccl_unique_id: the per-layer and resident
+                                            all-reduces run on the comm stream and are the identity) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

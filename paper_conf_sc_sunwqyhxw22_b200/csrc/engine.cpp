@@ -306,6 +306,9 @@ struct sh_ctx {
   bool shadow = true;  // bf16 shadow kept in host RAM (bf16 mode without SH_FLAG_FETCH_FP32)
   // shared store (world_size > 1 with shm_name): rank r owns elements [slo[x], shi[x]) of layer x
   bool shared = false;
+  // the data-parallel (collective) path: world_size > 1, or SH_FLAG_TEST_DP_PATH at world_size 1
+  // (a one-rank NCCL communicator: every all-reduce runs, and is the identity)
+  bool dp = false;
   bool no_collective = false;
   std::string shm_name;
   ShmCtl* ctl = nullptr;
@@ -1255,7 +1258,7 @@ sh_status ensure_gbufs(sh_ctx* c, int w) {
   // allocated up front (the window solver sees them as used).  Single GPU: the per-layer K2 runs
   // on the compute stream, in order, so two buffers never wait; data parallel: K2 runs on the comm
   // stream behind the all-reduce, four keep BP from waiting on it
-  const int want = c->W > 1 ? 4 : 2;
+  const int want = c->dp ? 4 : 2;
   while ((int)c->gbuf.size() < want) {
     float* p = nullptr;
     if (cudaMalloc(&p, 4 * c->max_pad) != cudaSuccess) {
@@ -1503,8 +1506,9 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     return SH_ERR_INVALID;
   }
   const int W = cfg->world_size < 1 ? 1 : cfg->world_size;
-  if (W > 1 && ((!cfg->nccl_unique_id && !(cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE)) || cfg->rank < 0 ||
-                 cfg->rank >= W)) {
+  const bool dp = W > 1 || (cfg->flags & SH_FLAG_TEST_DP_PATH);
+  if (dp && ((!cfg->nccl_unique_id && !(cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE)) || cfg->rank < 0 ||
+             cfg->rank >= W)) {
     set_error("sh_init: world_size > 1 needs nccl_unique_id and 0 <= rank < world_size");
     return SH_ERR_INVALID;
   }
@@ -1518,7 +1522,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->L = cfg->n_layers;
   c->W = W;
   c->rank = cfg->rank;
-  c->no_collective = W > 1 && (cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE);
+  c->dp = dp;
+  c->no_collective = dp && (cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE);
   c->shared = W > 1 && cfg->shm_name && cfg->shm_name[0];
   if (c->shared) c->shm_name = cfg->shm_name;
   c->bf16 = cfg->precision == SH_BF16_MIXED;
@@ -1560,8 +1565,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     CKC(c.get(), cudaEventCreateWithFlags(&c->ev_res_k3[i], cudaEventDisableTiming));
     CKC(c.get(), cudaEventCreateWithFlags(&c->ev_norm[i], cudaEventDisableTiming));
   }
-  if (W > 1) CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
-  if (W > 1 && !c->no_collective) {
+  if (dp) CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
+  if (dp && !c->no_collective) {
     if (!g_nccl.load()) {
       set_error("sh_init: world_size > 1 but libnccl.so.2 cannot be loaded");
       return SH_ERR_UNSUPPORTED;
@@ -2002,8 +2007,8 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       float* gb = c->gbuf[b];
       // (single GPU: on the compute stream -- measured on C4, K2 running beside the next layer's
       // GEMMs slows them by about as much as it saves, and in order its roofline stays clean)
-      cudaStream_t ks = c->W > 1 ? c->comm : c->cs;
-      if (c->W > 1) {
+      cudaStream_t ks = c->dp ? c->comm : c->cs;
+      if (c->dp) {
         CKC(c, cudaEventRecord(c->ev_gbuf_ready[b], c->cs));
         CKC(c, cudaStreamWaitEvent(c->comm, c->ev_gbuf_ready[b], 0));
         if (!c->no_collective) {
@@ -2044,7 +2049,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       c->arrive_gen[x] = g2;
       c->arrive_by_issuer[x] = 0;
       c->arrive_pub[x].store(g2);
-    } else if (c->W > 1) {
+    } else if (c->dp) {
       // data parallel: average this layer's grads across ranks before the offload (K-e)
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
       CKC(c, cudaStreamWaitEvent(c->comm, c->ev_grad_done[s], 0));
@@ -2069,7 +2074,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       // host layer: K3 runs on the D2H stream right before the offload (off the compute stream)
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
     }
-    const bool k3_on_d2h = c->W == 1 && !c->is_g(x);
+    const bool k3_on_d2h = !c->dp && !c->is_g(x);
     if (!c->is_g(x)) {
       const int k = (int)(c->landing_rr++ % c->D);
       const int64_t use = c->landing_uses[k]++;
@@ -2196,7 +2201,7 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     st = exec_fold(c, c->res_grad, c->xres, c->res.n_pad);
     if (st != SH_OK) return st;
   }
-  if (c->W > 1) {
+  if (c->dp) {
     // resident grads: average too, on the comm stream after the caller's embedding backward
     CKC(c, cudaEventRecord(c->ev_cs_mark, c->cs));
     CKC(c, cudaStreamWaitEvent(c->comm, c->ev_cs_mark, 0));
@@ -2213,7 +2218,7 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     CKC(c, kern::sumsq(c->res_grad, c->res.n_pad, c->scratch_cs, c->partials + L, c->cs));
   }
   bool norm_on_d2h = false;
-  if (c->W == 1 && c->w < L && !c->clip) {
+  if (!c->dp && c->w < L && !c->clip) {
     // no clipping: nothing on the compute stream needs the norm.  Finalize it on the D2H stream
     // behind the host layers' K3s, queued on the D2H issuer, so the driver never waits for the
     // issuer (which may be held back by landing-buffer waits) at the step boundary.
@@ -2228,7 +2233,7 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     });
     norm_on_d2h = true;
   } else {
-    if (c->W == 1 && c->w < L) {  // clip mode: K2 needs the coefficient -- wait for the last K3
+    if (!c->dp && c->w < L) {  // clip mode: K2 needs the coefficient -- wait for the last K3
       const int64_t gen = c->k3_last_gen;
       if (!state_wait(c, [&] { return c->k3_pub.load() >= gen; }, "last K3 issue")) return check_failed(c);
       CKC(c, cudaStreamWaitEvent(c->cs, c->ev_k3_last, 0));
