@@ -23,7 +23,7 @@ def parse(path):
         except ValueError:
             continue
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-9, "usecond": 1e-6,
-                 "msecond": 1e-3}.get(u, 1)
+                 "msecond": 1e-3, "ns": 1e-9, "us": 1e-6, "ms": 1e-3}.get(u, 1)
         out[h] = x * scale
     return out
 
@@ -42,7 +42,6 @@ def main():
                   "dram_bytes_per_elem": (rd + wr) / N, "algorithmic_bytes_per_elem": alg,
                   "traffic_over_algorithmic": (rd + wr) / (alg * N),
                   "achieved_alg_gbs": alg * N / t / 1e9,
-                  "dram_pct_of_peak": m.get("dram__throughput.avg.pct_of_peak_sustained_elapsed"),
                   "grid": m.get("launch__grid_size"), "regs": m.get("launch__registers_per_thread")}
     json.dump(res, open(dst, "w"), indent=1)
     print(json.dumps(res, indent=1))

@@ -6,7 +6,7 @@ for k in k2_adamw k1_cast k3_sumsq k4_exec_reduce; do
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:$k -s 1 -c 1 \
       -o gpurun_out/ncu_iso_$k -f python tools/kernel_once.py > gpurun_out/ncu_iso_$k.log 2>&1
   ncu -i gpurun_out/ncu_iso_$k.ncu-rep --page raw --csv \
-      --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,launch__grid_size,launch__registers_per_thread,dram__throughput.avg.pct_of_peak_sustained_elapsed \
+      --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,launch__grid_size,launch__registers_per_thread \
       > gpurun_out/ncu_iso_$k.csv 2>&1
 done
 ls -la gpurun_out | tail -20
