@@ -119,6 +119,9 @@ typedef struct {
 #define SH_FLAG_TEST_DP_PATH (1ull << 11) /* test: take the data-parallel path at world_size 1 (one-rank NCCL
                                             communicator from nccl_unique_id: the per-layer and resident
                                             all-reduces run on the comm stream and are the identity) */
+#define SH_FLAG_KEEP_GRADS (1ull << 12) /* diagnostics: one gradient buffer per GPU-optimised layer (no clipping),
+                                          so SH_READ_GRAD can return every layer's gradients after a step
+                                          (default: a rotation of 2, or 4 with data parallelism) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

@@ -1259,7 +1259,8 @@ sh_status ensure_gbufs(sh_ctx* c, int w) {
   // allocated up front (the window solver sees them as used).  Single GPU: the per-layer K2 runs
   // on the compute stream, in order, so two buffers never wait; data parallel: K2 runs on the comm
   // stream behind the all-reduce, four keep BP from waiting on it
-  const int want = c->dp ? 4 : 2;
+  int want = c->dp ? 4 : 2;
+  if (c->cfg.flags & SH_FLAG_KEEP_GRADS) want = std::max(want, w);  // one per GPU-optimised layer
   while ((int)c->gbuf.size() < want) {
     float* p = nullptr;
     if (cudaMalloc(&p, 4 * c->max_pad) != cudaSuccess) {

@@ -204,25 +204,44 @@ __global__ void __launch_bounds__(256) k3_sumsq_kernel(const float* __restrict__
   }
 }
 
-// K4: 8 elements (2 float4) per thread per iteration; the k-1 executor buffers are streamed
-// (read once, L1 no-allocate), the destination is read and written in place.
+// K4: a block handles tiles of 4096 floats; thread t of the block owns the float4s at t*4 + 1024u
+// (u < 4) of a tile, so every warp access is 512 contiguous bytes and all 4(n_src+1) 16-B loads of
+// an iteration are in flight before the adds.  Executor buffers are streamed (L1 no-allocate), the
+// destination is read and written in place.  The < 4096-float tail is done one float4 per thread.
 __global__ void __launch_bounds__(256) k4_exec_reduce_kernel(const __grid_constant__ K4Args a) {
-  const int64_t n8 = a.n / 8;
-  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n8;
-       j += (int64_t)gridDim.x * blockDim.x) {
-    float4 x0 = ld_rw(a.dst + 8 * j), x1 = ld_rw(a.dst + 8 * j + 4);
+  const float f = a.inv_k;
+  const int64_t tiles = a.n / 4096;
+  for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    const int64_t base = tile * 4096 + 4 * threadIdx.x;
+    float4 x[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) x[u] = ld_rw(a.dst + base + 1024 * u);
     for (int s = 0; s < a.n_src; ++s) {
-      const float4 y0 = ld_stream(a.src[s] + 8 * j), y1 = ld_stream(a.src[s] + 8 * j + 4);
-      x0.x = __fadd_rn(x0.x, y0.x); x0.y = __fadd_rn(x0.y, y0.y);
-      x0.z = __fadd_rn(x0.z, y0.z); x0.w = __fadd_rn(x0.w, y0.w);
-      x1.x = __fadd_rn(x1.x, y1.x); x1.y = __fadd_rn(x1.y, y1.y);
-      x1.z = __fadd_rn(x1.z, y1.z); x1.w = __fadd_rn(x1.w, y1.w);
+      float4 y[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) y[u] = ld_stream(a.src[s] + base + 1024 * u);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        x[u].x = __fadd_rn(x[u].x, y[u].x); x[u].y = __fadd_rn(x[u].y, y[u].y);
+        x[u].z = __fadd_rn(x[u].z, y[u].z); x[u].w = __fadd_rn(x[u].w, y[u].w);
+      }
     }
-    const float f = a.inv_k;
-    x0.x = __fmul_rn(x0.x, f); x0.y = __fmul_rn(x0.y, f); x0.z = __fmul_rn(x0.z, f); x0.w = __fmul_rn(x0.w, f);
-    x1.x = __fmul_rn(x1.x, f); x1.y = __fmul_rn(x1.y, f); x1.z = __fmul_rn(x1.z, f); x1.w = __fmul_rn(x1.w, f);
-    st_f4(a.dst + 8 * j, x0);
-    st_f4(a.dst + 8 * j + 4, x1);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      x[u].x = __fmul_rn(x[u].x, f); x[u].y = __fmul_rn(x[u].y, f);
+      x[u].z = __fmul_rn(x[u].z, f); x[u].w = __fmul_rn(x[u].w, f);
+      st_f4(a.dst + base + 1024 * u, x[u]);
+    }
+  }
+  for (int64_t i = tiles * 4096 + 4 * (blockIdx.x * (int64_t)blockDim.x + threadIdx.x); i < a.n;
+       i += 4 * (int64_t)gridDim.x * blockDim.x) {
+    float4 x = ld_rw(a.dst + i);
+    for (int s = 0; s < a.n_src; ++s) {
+      const float4 y = ld_stream(a.src[s] + i);
+      x.x = __fadd_rn(x.x, y.x); x.y = __fadd_rn(x.y, y.y); x.z = __fadd_rn(x.z, y.z); x.w = __fadd_rn(x.w, y.w);
+    }
+    x.x = __fmul_rn(x.x, f); x.y = __fmul_rn(x.y, f); x.z = __fmul_rn(x.z, f); x.w = __fmul_rn(x.w, f);
+    st_f4(a.dst + i, x);
   }
 }
 
@@ -313,10 +332,9 @@ cudaError_t sumsq(const float* g, int64_t n, double* scratch, double* out, cudaS
 }
 
 cudaError_t exec_reduce(const K4Args& a, cudaStream_t st) {
-  const int64_t n8 = a.n / 8;
-  if (n8 == 0 || a.n_src < 0) return cudaSuccess;
-  const int64_t cap = (int64_t)sm_count() * 8;
-  const int64_t need = (n8 + 255) / 256;
+  if (a.n <= 0 || a.n_src < 0) return cudaSuccess;
+  const int64_t cap = (int64_t)sm_count() * 8;  // persistent: 8 x 256 threads per SM (44 regs)
+  const int64_t need = (a.n + 4095) / 4096;
   launch_counter()++;
   k4_exec_reduce_kernel<<<(int)(need < cap ? need : cap), 256, 0, st>>>(a);
   return cudaGetLastError();

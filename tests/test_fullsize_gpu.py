@@ -30,7 +30,7 @@ def _trainer(window):
     from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
     mc = T.ModelConfig(C2["L"], C2["h"], C2["nh"], C2["s"], C2["V"])
     return T.StrongholdTrainer(mc, batch=C2["b"], window=window, precision=sh.SH_BF16_MIXED,
-                               flags=sh.SH_FLAG_PROFILE, init_threads=16)
+                               flags=sh.SH_FLAG_PROFILE | sh.SH_FLAG_KEEP_GRADS, init_threads=16)
 
 
 def _read(tr, layer, what):
