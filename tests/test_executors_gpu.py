@@ -106,3 +106,17 @@ def test_executor_grads_protocol():
             T.StrongholdTrainer(mc, batch=3, window=2, precision=sh.SH_FP32, executors=2)
     finally:
         tr.close()
+
+
+def test_executors_clip_fp32_vs_oracle():
+    """Clip mode: the global norm is taken over the executors' AVERAGED gradients (K4 runs before K3)."""
+    st, _, onorms = oracle_run(TINY_B4, STEPS, max_grad_norm=0.5)
+    assert onorms[0] > 0.5
+    tr, _, norms = engine_run(TINY_B4, STEPS, 1, sh.SH_FP32, max_grad_norm=0.5, executors=2)
+    try:
+        errs = _errors(tr, st)
+        assert max(errs.values()) <= FP32_TOL, errs
+        for a, b in zip(norms, onorms):
+            assert abs(a - b) <= 1e-4 * b, (norms, onorms)
+    finally:
+        tr.close()

@@ -70,3 +70,19 @@ def test_bad_spill_dir(tmp_path):
     with pytest.raises(sh.ShError):
         tr, _, _ = engine_run(TINY, 1, 1, sh.SH_FP32, spill_dir=str(tmp_path / "missing"))
         tr.close()
+
+
+def test_spill_clip_mode_bitwise(tmp_path):
+    L = TINY["L"]
+    ref_tr, ref_losses, ref_norms = engine_run(TINY, STEPS, L, sh.SH_FP32, max_grad_norm=0.5)
+    ref = engine_state(ref_tr)
+    ref_tr.close()
+    tr, losses, norms = engine_run(TINY, STEPS, 1, sh.SH_FP32, max_grad_norm=0.5, spill_dir=str(tmp_path),
+                                   host_pin_budget_bytes=1)
+    try:
+        assert tr.engine.stats()["spilled_layers"] == L - 1
+        ok, what = states_bitwise_equal(engine_state(tr), ref)
+        assert ok, what
+        assert losses == ref_losses and norms == ref_norms
+    finally:
+        tr.close()
