@@ -1526,7 +1526,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->rank = cfg->rank;
   c->dp = dp;
   c->no_collective = dp && (cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE);
-  c->shared = W > 1 && cfg->shm_name && cfg->shm_name[0];
+  c->shared = dp && cfg->shm_name && cfg->shm_name[0];
   if (c->shared) c->shm_name = cfg->shm_name;
   c->bf16 = cfg->precision == SH_BF16_MIXED;
   c->cb = c->bf16 ? 2 : 4;
@@ -1578,7 +1578,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     sh_status s = nccl_check(c.get(), g_nccl.CommInitRank(&c->nccl, W, id, cfg->rank), "ncclCommInitRank");
     if (s != SH_OK) return s;
   }
-  c->slice_fetch = W > 1 && (cfg->flags & SH_FLAG_SLICE_FETCH) && cfg->shm_name && cfg->shm_name[0];
+  c->slice_fetch = dp && (cfg->flags & SH_FLAG_SLICE_FETCH) && cfg->shm_name && cfg->shm_name[0];
   if (c->slice_fetch && !c->no_collective) {
     if (!g_nccl.AllGather || !g_nccl.CommSplit) {
       set_error("sh_init: SH_FLAG_SLICE_FETCH needs ncclAllGather and ncclCommSplit");

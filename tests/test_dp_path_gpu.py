@@ -50,3 +50,27 @@ def test_dp_path_with_executors():
         assert losses == ref_losses
     finally:
         tr.close()
+
+
+@pytest.mark.parametrize("fetch32", [False, True])
+def test_dp_path_shared_store_slice_fetch_one_rank(fetch32):
+    """The whole data-parallel machinery of one rank with real NCCL calls: the shared /dev/shm host
+    store (control block, counters, barriers), NEXT-1 slice fetch (ncclCommSplit for the H2D issuer's
+    communicator, in-place ncclAllGather after the slice H2D) and the per-layer all-reduce."""
+    import os
+    import uuid
+    L = TINY["L"]
+    ref_tr, ref_losses, _ = engine_run(TINY, STEPS, L, sh.SH_BF16_MIXED)
+    ref = engine_state(ref_tr)
+    ref_tr.close()
+    name = f"shdp1_{uuid.uuid4().hex[:12]}"
+    flags = sh.SH_FLAG_TEST_DP_PATH | sh.SH_FLAG_SLICE_FETCH | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0)
+    tr, losses, _ = engine_run(TINY, STEPS, 1, sh.SH_BF16_MIXED, flags=flags, nccl_id=sh.nccl_unique_id(),
+                               shm_name=name)
+    try:
+        ok, what = states_bitwise_equal(engine_state(tr), ref)
+        assert ok, what
+        assert losses == ref_losses
+    finally:
+        tr.close()
+    assert not any(f.startswith(name) for f in os.listdir("/dev/shm"))
