@@ -249,6 +249,10 @@ def main():
     ap.add_argument("--spill-dir", default="", help="NEXT-2: directory of the file-backed tier (PAPER.md:219-221)")
     ap.add_argument("--host-pin-gb", type=float, default=0.0,
                     help="NEXT-2: pinned host-store budget in GB (layers beyond it spill to --spill-dir)")
+    ap.add_argument("--ablate-alloc", action="store_true",
+                    help="Fig. 14 ablation: cudaMalloc/cudaFree per prefetch instead of the reserved ring")
+    ap.add_argument("--sync-cpu", action="store_true",
+                    help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
     ap.add_argument("--spill-evict", action="store_true", help="NEXT-2: drop spilled layers from the page cache")
     ap.add_argument("--executors", type=int, default=1,
                     help="NEXT-3: K multi-stream executors (micro-batches of batch/K on K streams, PAPER.md:227-242)")
@@ -326,7 +330,8 @@ def main():
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
             (sh.SH_FLAG_CPU_HARD | sh.SH_FLAG_DECOUPLE if cpu_hard else 0) | \
             (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0) | \
-            (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0)
+            (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0) | \
+            (sh.SH_FLAG_ABLATE_ALLOC if args.ablate_alloc else 0) | (sh.SH_FLAG_SYNC_CPU if args.sync_cpu else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
@@ -449,6 +454,8 @@ def main():
                    "gpt_driver_attention": r["attn"],
                    "parallelism": f"dp{world}",
                    "executors": args.executors,
+                   "ablation": [k for k, v in (("alloc", args.ablate_alloc), ("sync_cpu", args.sync_cpu),
+                                               ("cpu_threads", args.cpu_threads)) if v] or None,
                    "spill": {"dir": args.spill_dir, "layers": r["st1"]["spilled_layers"],
                              "bytes": r["st1"]["spill_bytes"], "evict": args.spill_evict} if args.spill_dir else None,
                    "host_store": ("one shared /dev/shm store, rank-sliced offload + CPU Adam" if shm_name else

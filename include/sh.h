@@ -122,6 +122,8 @@ typedef struct {
 #define SH_FLAG_KEEP_GRADS (1ull << 12) /* diagnostics: one gradient buffer per GPU-optimised layer (no clipping),
                                           so SH_READ_GRAD can return every layer's gradients after a step
                                           (default: a rotation of 2, or 4 with data parallelism) */
+#define SH_FLAG_ABLATE_ALLOC (1ull << 13) /* ablation (Fig. 14): a cudaMalloc/cudaFree pair per
+                                            prefetch, as per-layer CUDA-allocator buffers would cost */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

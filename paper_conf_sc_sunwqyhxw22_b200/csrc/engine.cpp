@@ -900,6 +900,14 @@ int64_t next_use(const sh_ctx* c, int x, int cur) {
 }
 
 sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
+  if (c->cfg.flags & SH_FLAG_ABLATE_ALLOC) {
+    // ablation (Fig. 14 "memory management"): what per-layer buffers from the CUDA
+    // allocator would cost -- a cudaMalloc / cudaFree pair per prefetch; cudaFree synchronises the
+    // device, so the driver cannot run ahead of the GPU (data placement is unchanged)
+    void* tmp = nullptr;
+    CKC(c, cudaMalloc(&tmp, c->slot_bytes));
+    CKC(c, cudaFree(tmp));
+  }
   const int old = c->slot_layer[s];
   if (old >= 0) c->layer_slot[old] = -1;
   c->slot_layer[s] = y;

@@ -22,7 +22,8 @@ SH_PRE, SH_POST = 0, 1
 SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE, SH_READ_GRAD = 0, 1, 2, 3, 4
 SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32, \
     SH_FLAG_TEST_NO_COLLECTIVE, SH_FLAG_SLICE_FETCH, SH_FLAG_DELAY_INJECT, SH_FLAG_DECOUPLE, SH_FLAG_SPILL_EVICT, \
-    SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS = 1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096
+    SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS, SH_FLAG_ABLATE_ALLOC = \
+    1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
