@@ -43,9 +43,14 @@ CONFIGS = {
     # (fp32-fetch mode, no bf16 shadow)
     "c4": (0, 4096, 32, 1024, 50304, 16, -1, "BASELINE configs[3]: depth-scaled GPT h4096, L = L_max(host RAM), "
                                             "fp32 states > 180 GB HBM, auto-tuned window"),
+    # the largest model the host RAM holds once GPU-optimised layers keep no host copy: warm up with
+    # the first C4MAX_W0 layers already in HBM, so only layers >= C4MAX_W0 need host blocks
+    "c4max": (0, 4096, 32, 1024, 50304, 16, -1, "max trainable size in host RAM: depth-scaled GPT h4096, "
+                                                "L = 32 + host-RAM capacity, auto-tuned window"),
 }
-FETCH_FP32_DEFAULT = {"c4"}
-CPU_HARD_DEFAULT = {"c3", "c4"}   # autotune with the eq. 3 CPU-throughput constraint (R19)
+C4MAX_W0 = 32
+FETCH_FP32_DEFAULT = {"c4", "c4max"}
+CPU_HARD_DEFAULT = {"c3", "c4", "c4max"}   # autotune with the eq. 3 CPU-throughput constraint (R19)
 
 
 def mem_available() -> int:
@@ -193,7 +198,8 @@ def run_reference(args, cfgname):
     if args.layers:
         L = args.layers
     if L == 0:  # same depth rule as the CUDA arm (L_max of this host's RAM)
-        L = c4_layers(h, args.grad_ring or 8, ranks_sharing=int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
+        L = c4_layers(h, args.grad_ring or 8, w0=C4MAX_W0 if cfgname == "c4max" else 2,
+                      ranks_sharing=int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
@@ -296,8 +302,11 @@ def main():
     if args.layers and L != 0:
         L = args.layers  # depth override (e.g. the resident-fit comparison model)
     if L == 0:
+        w0h = C4MAX_W0 if args.config == "c4max" else 2
         if args.layers:
             L = args.layers
+        elif args.config == "c4max":
+            L = c4_layers(h, args.grad_ring or 8, w0=w0h, ranks_sharing=local_world)
         elif not use_shm and world > 1:
             L = c4_layers(h, args.grad_ring or 8, budget=mem_available() // local_world)
         else:
@@ -314,7 +323,7 @@ def main():
     cpu_hard = args.cpu_hard == 1 or (args.cpu_hard == -1 and args.config in CPU_HARD_DEFAULT)
     # c3/c4 are host-RAM bound: 8 landing buffers (measured on C4: 4 -> 6.80, 8 -> 7.08, 12 -> 7.51
     # samples/s at L = 83, 82, 80; profiles/r01_bench_c4_ring*.json)
-    grad_ring = args.grad_ring or (8 if args.config in ("c3", "c4") else 0)
+    grad_ring = args.grad_ring or (8 if args.config in ("c3", "c4", "c4max") else 0)
 
     shm_name = None
     cpu_threads = args.cpu_threads
@@ -337,7 +346,8 @@ def main():
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
                                attention=args.attention, executors=args.executors,
-                               spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9))
+                               spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9),
+                               warmup_window=C4MAX_W0 if args.config == "c4max" and window == -1 else 0)
         attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
@@ -401,11 +411,11 @@ def main():
 
     r = run(w, not args.no_e2e)
     res = None
-    if not args.no_resident and w != L and args.config not in ("c3", "c4"):
+    if not args.no_resident and w != L and args.config not in ("c3", "c4", "c4max"):
         res = run(L, False)
     fit = None
     fit_layers = args.resident_fit_layers if args.resident_fit_layers >= 0 else (36 if h == 4096 else 0)
-    if args.config in ("c3", "c4") and fit_layers > 0 and not args.no_resident:
+    if args.config in ("c3", "c4", "c4max") and fit_layers > 0 and not args.no_resident:
         mc_fit = ModelConfig(fit_layers, h, nh, s, V)
         fit = run(fit_layers, False, mc_fit)
         fit["tflops"] = b * world * K / (fit["ms"] / 1e3) * s * mc_fit.flops_per_token() / 1e12

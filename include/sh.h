@@ -178,6 +178,10 @@ typedef struct {
                                        space reserved with posix_fallocate.  Not with shm_name. */
   int64_t host_pin_budget_bytes;    /* cap on pinned host-store bytes (layer blocks + landing ring);
                                        0 = no cap (spill only when pinning fails for lack of RAM) */
+  int32_t warmup_window;            /* window of the warm-up steps when window == -1 (0: min(2, n_layers)).
+                                       Only host-optimised layers hold a host block (a layer joining the
+                                       GPU set gives its block back), so a larger warm-up window lowers
+                                       the host RAM the store needs from the start */
 } sh_config;
 
 /* Per-layer profile consumed by the window solver (PAPER.md:132 notation; times in ms,

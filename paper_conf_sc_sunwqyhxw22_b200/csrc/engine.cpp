@@ -1221,6 +1221,24 @@ sh_status ensure_bounce(sh_ctx* c) {
   return SH_OK;
 }
 
+void release_host_layer(sh_ctx* c, int x) {
+  auto& hb = c->hblocks[x];
+  if (!hb.p) return;
+  if (hb.fd >= 0) {
+    munmap(hb.p, hb.bytes);
+    close(hb.fd);
+    c->spill_bytes -= hb.bytes;
+    c->n_spilled--;
+    c->spilled[x] = 0;
+  } else {
+    host_block_free(hb.p, hb.bytes);
+    c->host_bytes -= hb.bytes;
+  }
+  hb = {};
+  c->h_master[x] = c->h_m[x] = c->h_v[x] = nullptr;
+  c->h_shadow[x] = nullptr;
+}
+
 sh_status ensure_host_layer(sh_ctx* c, int x) {
   if (c->h_master[x]) return SH_OK;
   const int64_t n = c->lay[x].n_pad;
@@ -1417,6 +1435,10 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   st = stage_g_layers(c);
   if (st != SH_OK) return st;
   CKC(c, cudaStreamSynchronize(c->cs));
+  // the joining layers' masters / m / v now live in HBM: give their host blocks back (a private
+  // store re-allocates one if the layer leaves the GPU set again; shared segments stay mapped)
+  if (!c->shared)
+    for (int x = w_old; x < w_new; ++x) release_host_layer(c, x);
   return SH_OK;
 }
 
@@ -1554,7 +1576,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->slot_param_bytes = align_up((int64_t)c->cb * slot_elems, 256);
   c->slot_grad_bytes = align_up(4 * slot_elems, 256);
   c->slot_bytes = c->slot_param_bytes + c->slot_grad_bytes;
-  const int w0 = cfg->window >= 0 ? cfg->window : std::min(2, c->L);
+  const int w0 = cfg->window >= 0 ? cfg->window
+                                   : std::min(cfg->warmup_window > 0 ? cfg->warmup_window : 2, c->L);
   c->autotune_pending = cfg->window < 0;
   c->D = cfg->grad_ring_depth > 0 ? cfg->grad_ring_depth : c->L;
   if (c->clip && c->D < c->L) {

@@ -54,7 +54,8 @@ class Config(C.Structure):
                 ("device_budget_bytes", C.c_int64), ("cpu_util_max", C.c_double), ("ring_slots", C.c_int32),
                 ("world_size", C.c_int32), ("rank", C.c_int32),
                 ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p),
-                ("n_executors", C.c_int32), ("spill_dir", C.c_char_p), ("host_pin_budget_bytes", C.c_int64)]
+                ("n_executors", C.c_int32), ("spill_dir", C.c_char_p), ("host_pin_budget_bytes", C.c_int64),
+                ("warmup_window", C.c_int32)]
 
 
 _PD = C.POINTER(C.c_double)
@@ -268,7 +269,7 @@ class Engine:
                  stream=None, cpu_threads=0, grad_ring_depth=0, warmup_steps=5, device_budget_bytes=0,
                  world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None,
                  ring_slots=0, cpu_util_max=0.0, n_executors=1, spill_dir: str | None = None,
-                 host_pin_budget_bytes=0):
+                 host_pin_budget_bytes=0, warmup_window=0):
         L = lib()
         self.n_layers = len(layer_numels)
         self._keep = []
@@ -307,6 +308,7 @@ class Engine:
         self._spill = spill_dir.encode() if spill_dir else None
         cfg.spill_dir = self._spill
         cfg.host_pin_budget_bytes = int(host_pin_budget_bytes)
+        cfg.warmup_window = int(warmup_window)
         self.n_executors = max(1, n_executors)
         self._shm = shm_name.encode() if shm_name else None
         cfg.shm_name = self._shm

@@ -53,7 +53,8 @@ class StrongholdTrainer:
     def __init__(self, mc: ModelConfig, *, batch: int, window: int, precision=sh.SH_BF16_MIXED, lr=1.5e-4,
                  max_grad_norm=0.0, device=0, seed=1234, cpu_threads=0, grad_ring_depth=0, warmup_steps=5,
                  flags=0, world_size=1, rank=0, nccl_id=None, init=True, init_threads=8, shm_name=None,
-                 attention="auto", ring_slots=0, executors=1, spill_dir=None, host_pin_budget_bytes=0):
+                 attention="auto", ring_slots=0, executors=1, spill_dir=None, host_pin_budget_bytes=0,
+                 warmup_window=0):
         self.mc = mc
         self.batch = batch
         # NEXT-3 multi-stream executors: K workers on K streams, one parameter copy,
@@ -72,7 +73,8 @@ class StrongholdTrainer:
                                 stream=self.stream, cpu_threads=cpu_threads, grad_ring_depth=grad_ring_depth,
                                 warmup_steps=warmup_steps, world_size=world_size, rank=rank, nccl_id=nccl_id,
                                 flags=flags, shm_name=shm_name, ring_slots=ring_slots, n_executors=self.K,
-                                spill_dir=spill_dir, host_pin_budget_bytes=host_pin_budget_bytes)
+                                spill_dir=spill_dir, host_pin_budget_bytes=host_pin_budget_bytes,
+                                warmup_window=warmup_window)
         # executor 0 runs on the engine's compute stream, executors >= 1 on their own streams
         self.streams = [self.stream] + [torch.cuda.Stream(device=self.device) for _ in range(self.K - 1)]
         self.gpts = [GPT(n_layers=L, hidden=mc.hidden, heads=mc.heads, seq=mc.seq, max_batch=self.mb,
@@ -95,7 +97,7 @@ class StrongholdTrainer:
         self.loss_parts = torch.zeros(self.K, dtype=torch.float32, device=self.device)
         self.loss_host = torch.zeros(1, dtype=torch.float32).pin_memory()
         # with a shared host store only rank 0 writes the host-optimised layers' initial state
-        self._w0 = window if window >= 0 else min(2, L)
+        self._w0 = window if window >= 0 else min(warmup_window if warmup_window > 0 else 2, L)
         self._host_data_skipped = bool(shm_name) and rank != 0
         if init:
             self.init_params(seed, init_threads)

@@ -1,0 +1,53 @@
+"""Host-store footprint: only host-optimised layers hold a pinned host block (a layer joining the
+GPU-optimised set gives its block back; one leaving it gets a new one), and the warm-up window of
+an autotuned run (sh_config.warmup_window) decides which layers need a block from the start.
+Footprint changes must not change a bit of the training."""
+import pytest
+
+import synth
+from tests._common import TINY, engine_run, engine_state, states_bitwise_equal
+
+pytestmark = pytest.mark.gpu
+
+sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
+
+
+def test_blocks_follow_the_gpu_set():
+    L = TINY["L"]
+    ref_tr, ref_losses, _ = engine_run(TINY, 3, L, sh.SH_FP32)
+    ref = engine_state(ref_tr)
+    ref_tr.close()
+    tr, losses, _ = engine_run(TINY, 1, 1, sh.SH_FP32)
+    try:
+        hb1 = tr.engine.stats()["host_bytes"]
+        tr.engine.set_window(3)                      # layers 1, 2 join the GPU set
+        hb3 = tr.engine.stats()["host_bytes"]
+        assert hb3 < hb1
+        per_layer = (hb1 - hb3) // 2
+        assert per_layer >= 12 * sum(tr.mc.layer_numels())
+        for t in (1, 2):
+            if t == 2:
+                tr.engine.set_window(1)              # and leave it again
+                assert tr.engine.stats()["host_bytes"] == hb1
+            tr.set_tokens(synth.tokens(t, TINY["b"], TINY["s"], TINY["V"]))
+            tr.step_device(want_norm=True)
+            losses.append(tr.loss())
+        ok, what = states_bitwise_equal(engine_state(tr), ref)
+        assert ok, what
+        assert losses == ref_losses
+    finally:
+        tr.close()
+
+
+def test_warmup_window_sets_the_initial_footprint():
+    from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
+    mc = T.ModelConfig(TINY["L"], TINY["h"], TINY["nh"], TINY["s"], TINY["V"])
+    a = T.StrongholdTrainer(mc, batch=TINY["b"], window=-1, precision=sh.SH_FP32, warmup_steps=2)
+    b = T.StrongholdTrainer(mc, batch=TINY["b"], window=-1, precision=sh.SH_FP32, warmup_steps=2, warmup_window=3)
+    try:
+        sa, sb = a.engine.stats(), b.engine.stats()
+        assert sa["window"] == 2 and sb["window"] == 3
+        assert sb["host_bytes"] < sa["host_bytes"]
+    finally:
+        a.close()
+        b.close()

@@ -8,3 +8,8 @@ for v in "base:" "threads1:--cpu-threads 1" "threads4:--cpu-threads 4" "synccpu:
   timeout 900 $B $a > gpurun_out/abl_$n.json 2> gpurun_out/abl_$n.err
   echo "$n"; tail -c 200 gpurun_out/abl_$n.json; echo
 done
+# NEXT-4 / Fig. 13 analogue: FP-only streaming inference (KD teacher) of the C2 model and of the C4 model
+timeout 900 python bench.py --config c2 --fp-only --steps 10 --no-resident --no-cpu-baseline > gpurun_out/fponly_c2.json 2> gpurun_out/fponly_c2.err
+tail -c 300 gpurun_out/fponly_c2.json; echo
+timeout 1500 python bench.py --fp-only --window 40 --steps 5 --no-resident --no-cpu-baseline > gpurun_out/fponly_c4.json 2> gpurun_out/fponly_c4.err
+tail -c 300 gpurun_out/fponly_c4.json; echo
