@@ -257,6 +257,8 @@ def main():
                     help="NEXT-2: pinned host-store budget in GB (layers beyond it spill to --spill-dir)")
     ap.add_argument("--ablate-alloc", action="store_true",
                     help="Fig. 14 ablation: cudaMalloc/cudaFree per prefetch instead of the reserved ring")
+    ap.add_argument("--grow-landing", action="store_true",
+                    help="autotune may decouple the ring by growing the landing ring (SH_FLAG_GROW_LANDING)")
     ap.add_argument("--sync-cpu", action="store_true",
                     help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
     ap.add_argument("--spill-evict", action="store_true", help="NEXT-2: drop spilled layers from the page cache")
@@ -340,7 +342,8 @@ def main():
             (sh.SH_FLAG_CPU_HARD | sh.SH_FLAG_DECOUPLE if cpu_hard else 0) | \
             (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0) | \
             (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0) | \
-            (sh.SH_FLAG_ABLATE_ALLOC if args.ablate_alloc else 0) | (sh.SH_FLAG_SYNC_CPU if args.sync_cpu else 0)
+            (sh.SH_FLAG_ABLATE_ALLOC if args.ablate_alloc else 0) | (sh.SH_FLAG_SYNC_CPU if args.sync_cpu else 0) | \
+            (sh.SH_FLAG_GROW_LANDING if args.grow_landing else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
@@ -472,7 +475,7 @@ def main():
                                   "private per rank") if world > 1 else "private",
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),
                    "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
-                   "grad_landing_buffers": grad_ring or L, "host_store_bytes": r["st1"]["host_bytes"],
+                   "grad_landing_buffers": r["st1"]["landing_buffers"], "host_store_bytes": r["st1"]["host_bytes"],
                    "states_bytes_fp32_p_m_v": 12 * mc.n_params(),
                    "l2": "no flush: per-step traffic (GBs) >> 126 MB L2"},
         "tokens_per_s": tokens_s,

@@ -124,6 +124,10 @@ typedef struct {
                                           (default: a rotation of 2, or 4 with data parallelism) */
 #define SH_FLAG_ABLATE_ALLOC (1ull << 13) /* ablation (Fig. 14): a cudaMalloc/cudaFree pair per
                                             prefetch, as per-layer CUDA-allocator buffers would cost */
+#define SH_FLAG_GROW_LANDING (1ull << 14) /* autotuner: with a private store and grad_ring_depth < n_layers, still
+                                            decouple the ring (R22) by growing the landing ring to one buffer
+                                            per host-optimised layer, in the host RAM the layers joining the
+                                            GPU set give back */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
@@ -251,6 +255,8 @@ typedef struct {
   double last_step_ms;          /* first FP hook .. end of K2 of that step (GPU time) */
   int64_t spill_bytes;          /* NEXT-2: bytes of host-optimised layer state in spill files */
   int32_t spilled_layers;       /* number of layers in the spill tier */
+  int32_t landing_buffers;      /* host landing buffers for offloaded gradients (grows when the autotuner
+                                   decouples the ring on a private store) */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */

@@ -1442,6 +1442,39 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   return SH_OK;
 }
 
+// Grow the host landing ring to D_new buffers (private store, between steps): a fresh pinned block,
+// the two clip-coefficient words carried over, every buffer's use counter restarted.  Lets the
+// autotuner decouple the ring from the GPU-optimised set (R22) once the layers joining that set
+// have given their host blocks back.
+sh_status grow_landing(sh_ctx* c, int D_new) {
+  if (D_new <= c->D || c->shared) return SH_OK;
+  sh_status st = sync_all(c);
+  if (st != SH_OK) return st;
+  const int64_t lb = align_up(4 * c->max_pad, 4096);
+  const size_t bytes = align_up((int64_t)D_new * lb + 4096, 1 << 21);
+  char* p = nullptr;
+  st = host_block_alloc(bytes, c->n_threads, &p);
+  if (st != SH_OK) return st;
+  const float coef0 = c->h_coef[0], coef1 = c->h_coef[1];
+  host_block_free(c->hland.p, c->hland.bytes);
+  c->host_bytes -= c->hland.bytes;
+  c->hland = {p, bytes};
+  c->host_bytes += bytes;
+  c->D = D_new;
+  c->landing.resize(D_new);
+  for (int k = 0; k < D_new; ++k) c->landing[k] = reinterpret_cast<float*>(p + (int64_t)k * lb);
+  c->h_coef = reinterpret_cast<float*>(p + (int64_t)D_new * lb);
+  c->h_coef[0] = coef0;
+  c->h_coef[1] = coef1;
+  c->landing_done = std::make_unique<std::atomic<int64_t>[]>(D_new);
+  for (int k = 0; k < D_new; ++k) c->landing_done[k].store(0);
+  c->landing_uses.assign(D_new, 0);
+  c->landing_owner.assign(D_new, -1);
+  c->last_landing.assign(c->L, -1);
+  c->landing_rr = 0;
+  return SH_OK;
+}
+
 // K4 on the compute stream: dst = (dst + Σ_e src[e]) / K in a fixed order (NEXT-3).
 sh_status exec_fold(sh_ctx* c, float* dst, const std::vector<float*>& src, int64_t n) {
   kern::K4Args a{};
@@ -2400,7 +2433,10 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   // decoupling needs a landing buffer per host layer: otherwise the ring's grad halves are what
   // absorbs the D2H backlog when the CPU Adam is slower than BP (measured: a 7-slot ring with a
   // 4-deep landing ring stalled BP every 4 layers on the C4 model)
-  o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip && c->D >= c->L ? 1 : 0;
+  // (with SH_FLAG_GROW_LANDING a private store grows its landing ring when the autotuner
+  // decouples, see sh_autotune_window)
+  o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip &&
+                        (c->D >= c->L || (!c->shared && (c->cfg.flags & SH_FLAG_GROW_LANDING))) ? 1 : 0;
   return SH_OK;
 }
 
@@ -2475,6 +2511,17 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
     ring = (int32_t)(v >> 32);
     if (!shm_barrier(c, 5, "autotuned window read")) return check_failed(c);
   }
+  // a decoupled ring needs a landing buffer per host-optimised layer (R22): with a private store
+  // the landing ring grows into the host RAM the layers joining the GPU set give back -- if that
+  // RAM (plus what is free now) cannot hold it, stay coupled
+  const int64_t lb = align_up(4 * c->max_pad, 4096);
+  if (ring > 0 && c->D < c->L - w) {
+    int64_t freed = 0;
+    for (int x = c->w; x < w; ++x)
+      if (c->hblocks[x].p && c->hblocks[x].fd < 0) freed += (int64_t)c->hblocks[x].bytes;
+    const int64_t need = (int64_t)(c->L - w) * lb + (int64_t)(8ll << 30);  // + headroom
+    if (c->shared || mem_available_bytes() + freed < need) ring = 0;
+  }
   // apply; if HBM turns out short (the solver's S_avail is an estimate), step the window down
   const int w_old = c->w;
   st = sh_set_window_ring(c, w, ring);
@@ -2484,6 +2531,13 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
     st = sh_set_window_ring(c, w, ring);
   }
   if (st == SH_ERR_OOM_DEVICE) st = sh_set_window_ring(c, w_old, 0);  // restore the warm-up window
+  if (st == SH_OK && c->ring_cap > 0 && c->D < c->L - c->w) {
+    st = grow_landing(c, c->L - c->w);
+    if (st != SH_OK) {  // host RAM after all too short: back to the coupled ring
+      clear_error();
+      st = sh_set_window_ring(c, c->w, 0);
+    }
+  }
   if (wout) *wout = c->w;
   return st;
 }
@@ -2609,6 +2663,7 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->d2h_overlap_frac = c->d2h_overlap;
   o->last_step_ms = c->last_step_ms;
   o->spill_bytes = (int64_t)c->spill_bytes;
+  o->landing_buffers = c->D;
   o->spilled_layers = c->n_spilled;
   return SH_OK;
 }

@@ -22,8 +22,8 @@ SH_PRE, SH_POST = 0, 1
 SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE, SH_READ_GRAD = 0, 1, 2, 3, 4
 SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32, \
     SH_FLAG_TEST_NO_COLLECTIVE, SH_FLAG_SLICE_FETCH, SH_FLAG_DELAY_INJECT, SH_FLAG_DECOUPLE, SH_FLAG_SPILL_EVICT, \
-    SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS, SH_FLAG_ABLATE_ALLOC = \
-    1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192
+    SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS, SH_FLAG_ABLATE_ALLOC, SH_FLAG_GROW_LANDING = \
+    1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192, 16384
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
@@ -89,7 +89,7 @@ class Stats(C.Structure):
                 ("k2_ms_sum", C.c_double), ("k2_bytes_sum", C.c_int64), ("k2_samples", C.c_int64),
                 ("k3_ms_sum", C.c_double), ("k3_bytes_sum", C.c_int64), ("k3_samples", C.c_int64),
                 ("h2d_overlap_frac", C.c_double), ("d2h_overlap_frac", C.c_double), ("last_step_ms", C.c_double),
-                ("spill_bytes", C.c_int64), ("spilled_layers", C.c_int32)]
+                ("spill_bytes", C.c_int64), ("spilled_layers", C.c_int32), ("landing_buffers", C.c_int32)]
 
 
 class TraceEvent(C.Structure):
@@ -230,10 +230,10 @@ def _dbl(a, n):
     return arr
 
 
-def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
+def make_profile(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
                  slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False,
-                 cpu_hard=False, cpu_util_max=1.0, decouple=False) -> dict:
-    """Pure call of sh_solve_window (no GPU)."""
+                 cpu_hard=False, cpu_util_max=1.0, decouple=False):
+    """(Profile, keep-alive arrays) for sh_solve_window / sh_autotune_window."""
     n = len(t_fp)
     keep = {}
     prof = Profile()
@@ -254,6 +254,12 @@ def solve_window(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_c
     prof.cpu_hard = 1 if cpu_hard else 0
     prof.cpu_util_max = cpu_util_max
     prof.decouple = 1 if decouple else 0
+    return prof, keep
+
+
+def solve_window(*args, **kw) -> dict:
+    """Pure call of sh_solve_window (no GPU); arguments as make_profile."""
+    prof, _keep = make_profile(*args, **kw)
     rep = SolveReport()
     check(lib().sh_solve_window(C.byref(prof), C.byref(rep)))
     return {f: getattr(rep, f) for f, _ in SolveReport._fields_}
@@ -414,9 +420,14 @@ class Engine:
         else:
             check(self._L.sh_set_window_ring(self.h, w, ring_slots))
 
-    def autotune(self) -> int:
+    def autotune(self, override: dict | None = None) -> int:
+        """Solve on the measured profile, or on `override` (make_profile keyword arguments), and apply."""
         w = C.c_int32()
-        check(self._L.sh_autotune_window(self.h, None, C.byref(w)))
+        if override is None:
+            check(self._L.sh_autotune_window(self.h, None, C.byref(w)))
+        else:
+            prof, _keep = make_profile(**override)
+            check(self._L.sh_autotune_window(self.h, C.byref(prof), C.byref(w)))
         return w.value
 
     def profile(self) -> dict:

@@ -51,3 +51,32 @@ def test_warmup_window_sets_the_initial_footprint():
     finally:
         a.close()
         b.close()
+
+
+def test_grow_landing_for_a_decoupled_ring():
+    """SH_FLAG_GROW_LANDING: an autotune that decouples the ring (R22) grows a short landing ring to
+    one buffer per host-optimised layer; the training stays bitwise equal to the resident run."""
+    L = TINY["L"]
+    ref_tr, ref_losses, _ = engine_run(TINY, 3, L, sh.SH_FP32)
+    ref = engine_state(ref_tr)
+    ref_tr.close()
+    tr, losses, _ = engine_run(TINY, 1, 1, sh.SH_FP32, grad_ring_depth=1,
+                               flags=sh.SH_FLAG_DECOUPLE | sh.SH_FLAG_GROW_LANDING)
+    try:
+        assert tr.engine.stats()["landing_buffers"] == 1
+        # a profile whose solution is prefetch distance 1 (ring 2) and GPU set 2 (CPU-update bound)
+        prof = dict(t_fp=[1.0] * L, t_bp=[3.0] * L, t_c2g=[0.1] * L, t_g2c=[0.1] * L, t_stage=[0.01] * L,
+                    t_opt_gpu=[0.0] * L, t_opt_cpu=[8.0] * L, cpu_hard=True, cpu_util_max=1.0, decouple=True)
+        assert sh.solve_window(**prof)["ring_slots"] == 2 and sh.solve_window(**prof)["window"] == 2
+        assert tr.engine.autotune(prof) == 2
+        st = tr.engine.stats()
+        assert st["landing_buffers"] == L - 2 and st["n_slots"] >= 2
+        for t in (1, 2):
+            tr.set_tokens(synth.tokens(t, TINY["b"], TINY["s"], TINY["V"]))
+            tr.step_device(want_norm=True)
+            losses.append(tr.loss())
+        ok, what = states_bitwise_equal(engine_state(tr), ref)
+        assert ok, what
+        assert losses == ref_losses
+    finally:
+        tr.close()
