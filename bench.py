@@ -259,6 +259,7 @@ def main():
                     help="Fig. 14 ablation: cudaMalloc/cudaFree per prefetch instead of the reserved ring")
     ap.add_argument("--grow-landing", action="store_true",
                     help="autotune may decouple the ring by growing the landing ring (SH_FLAG_GROW_LANDING)")
+    ap.add_argument("--no-decouple", action="store_true", help="autotune keeps the ring coupled to the GPU set")
     ap.add_argument("--sync-cpu", action="store_true",
                     help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
     ap.add_argument("--spill-evict", action="store_true", help="NEXT-2: drop spilled layers from the page cache")
@@ -339,7 +340,7 @@ def main():
         L = mc.n_layers
         t_init = time.perf_counter()
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
-            (sh.SH_FLAG_CPU_HARD | sh.SH_FLAG_DECOUPLE if cpu_hard else 0) | \
+            (sh.SH_FLAG_CPU_HARD | (0 if args.no_decouple else sh.SH_FLAG_DECOUPLE) if cpu_hard else 0) | \
             (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0) | \
             (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0) | \
             (sh.SH_FLAG_ABLATE_ALLOC if args.ablate_alloc else 0) | (sh.SH_FLAG_SYNC_CPU if args.sync_cpu else 0) | \

@@ -124,10 +124,11 @@ typedef struct {
                                           (default: a rotation of 2, or 4 with data parallelism) */
 #define SH_FLAG_ABLATE_ALLOC (1ull << 13) /* ablation (Fig. 14): a cudaMalloc/cudaFree pair per
                                             prefetch, as per-layer CUDA-allocator buffers would cost */
-#define SH_FLAG_GROW_LANDING (1ull << 14) /* autotuner: with a private store and grad_ring_depth < n_layers, still
-                                            decouple the ring (R22) by growing the landing ring to one buffer
-                                            per host-optimised layer, in the host RAM the layers joining the
-                                            GPU set give back */
+#define SH_FLAG_GROW_LANDING (1ull << 14) /* autotuner (private store, grad_ring_depth < n_layers): after the
+                                            window is applied, grow the landing ring to one buffer per
+                                            host-optimised layer in the host RAM the layers joining the GPU
+                                            set gave back (no D2H waits on the CPU Adam), and allow the
+                                            decoupled ring (R22, with SH_FLAG_DECOUPLE), which needs it */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 

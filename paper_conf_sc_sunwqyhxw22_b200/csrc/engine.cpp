@@ -2531,11 +2531,13 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
     st = sh_set_window_ring(c, w, ring);
   }
   if (st == SH_ERR_OOM_DEVICE) st = sh_set_window_ring(c, w_old, 0);  // restore the warm-up window
-  if (st == SH_OK && c->ring_cap > 0 && c->D < c->L - c->w) {
+  // one landing buffer per host layer: required by a decoupled ring; with SH_FLAG_GROW_LANDING also
+  // for a coupled one (the D2H issuer then never waits for the CPU Adam to free a buffer)
+  if (st == SH_OK && (c->ring_cap > 0 || (c->cfg.flags & SH_FLAG_GROW_LANDING)) && c->D < c->L - c->w) {
     st = grow_landing(c, c->L - c->w);
-    if (st != SH_OK) {  // host RAM after all too short: back to the coupled ring
+    if (st != SH_OK) {  // host RAM after all too short: keep the short ring (coupled)
       clear_error();
-      st = sh_set_window_ring(c, c->w, 0);
+      st = c->ring_cap > 0 ? sh_set_window_ring(c, c->w, 0) : SH_OK;
     }
   }
   if (wout) *wout = c->w;
