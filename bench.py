@@ -260,6 +260,7 @@ def main():
     ap.add_argument("--grow-landing", action="store_true",
                     help="autotune may decouple the ring by growing the landing ring (SH_FLAG_GROW_LANDING)")
     ap.add_argument("--no-decouple", action="store_true", help="autotune keeps the ring coupled to the GPU set")
+    ap.add_argument("--ring", type=int, default=0, help="fixed ring size (prefetch distance + 1) with a fixed --window")
     ap.add_argument("--sync-cpu", action="store_true",
                     help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
     ap.add_argument("--spill-evict", action="store_true", help="NEXT-2: drop spilled layers from the page cache")
@@ -349,7 +350,7 @@ def main():
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
-                               attention=args.attention, executors=args.executors,
+                               attention=args.attention, executors=args.executors, ring_slots=args.ring,
                                spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9),
                                warmup_window=C4MAX_W0 if args.config == "c4max" and window == -1 else 0)
         attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
