@@ -147,7 +147,7 @@ typedef struct {
   int32_t grad_ring_depth;          /* host landing buffers for offloaded grads; 0 = one per host layer */
   int32_t warmup_steps;             /* profiled steps before autotune (default 5); 0 = default */
   int64_t device_budget_bytes;      /* S_avail for ring + G states; 0 = free memory - 2 GiB */
-  double cpu_util_max;              /* autotuner eq. 3 utilisation target rho (SH_FLAG_CPU_HARD); 0 = 0.75 (measured: with rho 0.85 the C2 CPU Adam still saturated host DRAM, 0.98 of triad) */
+  double cpu_util_max;              /* autotuner eq. 3 utilisation target rho (SH_FLAG_CPU_HARD); 0 = 0.85 */
   int32_t ring_slots;               /* ring size cap (0: window + 1).  Without clipping a GPU-optimised
                                        layer is updated right after its backward, so its slot is not
                                        pinned and the ring may be smaller than the GPU-optimised set:

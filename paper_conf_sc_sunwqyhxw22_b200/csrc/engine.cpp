@@ -2429,7 +2429,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
                                               : held + (int64_t)fr - ((int64_t)2 << 30);
   o->duplex = (c->cfg.flags & SH_FLAG_DUPLEX) ? 1 : 0;
   o->cpu_hard = (c->cfg.flags & SH_FLAG_CPU_HARD) ? 1 : 0;
-  o->cpu_util_max = c->cfg.cpu_util_max > 0.0 ? c->cfg.cpu_util_max : 0.75;
+  o->cpu_util_max = c->cfg.cpu_util_max > 0.0 ? c->cfg.cpu_util_max : 0.85;
   // decoupling needs a landing buffer per host layer: otherwise the ring's grad halves are what
   // absorbs the D2H backlog when the CPU Adam is slower than BP (measured: a 7-slot ring with a
   // 4-deep landing ring stalled BP every 4 layers on the C4 model)
