@@ -260,6 +260,8 @@ def main():
     ap.add_argument("--grow-landing", action="store_true",
                     help="autotune may decouple the ring by growing the landing ring (SH_FLAG_GROW_LANDING)")
     ap.add_argument("--no-decouple", action="store_true", help="autotune keeps the ring coupled to the GPU set")
+    ap.add_argument("--fill-gpu", action="store_true", help="decoupled autotune fills HBM with GPU-optimised layers")
+    ap.add_argument("--late-shadow", action="store_true", help="fp32-fetch mode: bf16 host shadows after the autotune")
     ap.add_argument("--ring", type=int, default=0, help="fixed ring size (prefetch distance + 1) with a fixed --window")
     ap.add_argument("--sync-cpu", action="store_true",
                     help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
@@ -345,7 +347,8 @@ def main():
             (sh.SH_FLAG_SLICE_FETCH if args.slice_fetch else 0) | \
             (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0) | \
             (sh.SH_FLAG_ABLATE_ALLOC if args.ablate_alloc else 0) | (sh.SH_FLAG_SYNC_CPU if args.sync_cpu else 0) | \
-            (sh.SH_FLAG_GROW_LANDING if args.grow_landing else 0)
+            (sh.SH_FLAG_GROW_LANDING if args.grow_landing else 0) | (sh.SH_FLAG_FILL_GPU if args.fill_gpu else 0) | \
+            (sh.SH_FLAG_LATE_SHADOW if args.late_shadow else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,

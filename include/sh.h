@@ -129,6 +129,11 @@ typedef struct {
                                             host-optimised layer in the host RAM the layers joining the GPU
                                             set gave back (no D2H waits on the CPU Adam), and allow the
                                             decoupled ring (R22, with SH_FLAG_DECOUPLE), which needs it */
+#define SH_FLAG_FILL_GPU (1ull << 15)     /* autotuner, decoupled: the GPU-optimised set takes all the HBM the ring
+                                            leaves (sh_profile.fill_gpu) */
+#define SH_FLAG_LATE_SHADOW (1ull << 16)  /* bf16 mode with SH_FLAG_FETCH_FP32: after the autotune, give every host
+                                            layer a bf16 shadow in the host RAM the GPU set gave back (fetch 2
+                                            instead of 4 B/param; the solver already plans with that cost) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
@@ -211,6 +216,11 @@ typedef struct {
   double cpu_util_max;         /* rho in (0, 1]; <= 0 means 1 (utilisation target of the CPU pool) */
   int32_t decouple;            /* 1: choose the prefetch distance d (ring d+1, by P1/P2) and the
                                   GPU-optimised set g >= d (by eq. 3 + memory) separately (R22) */
+  int32_t fp_serial;           /* 1: (1b) also in its serialised-link form (R23): the FP fetches of the host
+                                  layers queue on one link, F(j) = max(F(j-1), S(j-d)) + t_c2g[j] <= S(j)
+                                  with S(p) = Σ_{i<p} t_fp -- a hard constraint */
+  int32_t fill_gpu;            /* decouple: g = the largest GPU-optimised set the memory leaves next to the
+                                  ring (instead of the smallest meeting eq. 3) */
 } sh_profile;
 
 typedef struct {

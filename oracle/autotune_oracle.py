@@ -19,6 +19,11 @@ code shared with the C++ solver (paper_conf_sc_sunwqyhxw22_b200/csrc/autotune.cp
   cpu_hard (optional): sum_{k>=w} t_opt_cpu[k] <= rho (sum_i (t_fp[i] + t_bp[i]) + sum_{i<w} t_opt_gpu[i])
   eq. 3 slack: min_{k in [w, L)} [ sum_{i<=k}(t_fp[i]+t_bp[i]) + sum_{i<w} t_opt_gpu[i] - t_opt_cpu[k] ]
   eq. 4: 5 L t_async  vs  sum_{i=w}^{L-1} t_opt_gpu[i]
+  fp_serial (R23, decoupled or not): the FP fetches of host layers j = g..L-1 queue on one link:
+      S(p) = sum_{i<p} t_fp[i] (compute start of FP position p with no stall)
+      F(j) = max(F(j-1), S(max(0, j-d))) + t_c2g[j]   (slot of position j-d-1 free, link free)
+      hard: F(j) <= S(j) for every host layer j
+  fill_gpu (decoupled): g = the largest g >= max(d, g_min) that fits next to the ring, not the smallest
 """
 from __future__ import annotations
 
@@ -29,7 +34,7 @@ def _z(a, n):
 
 def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
           slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False, cpu_hard=False,
-          cpu_util_max=1.0, decouple=False):
+          cpu_util_max=1.0, decouple=False, fp_serial=False, fill_gpu=False):
     """d = prefetch distance (ring d+1 slots), g = GPU-optimised layers [0, g); coupled d = g = m
     (the paper), decoupled g = max(d, smallest g meeting the CPU constraint) (R22)."""
     L = len(t_fp)
@@ -87,8 +92,26 @@ def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None
         rho = cpu_util_max if 0.0 < cpu_util_max < 1.0 else 1.0
         return sum(oc[k] for k in range(g, L)) <= rho * (sum(fp) + sum(bp) + sum(og[:g]))
 
+    def serial_ok(d, g):
+        if not fp_serial:
+            return True
+        F = None
+        for j in range(g, L):
+            q = max(0, j - d)
+            slot_free = 0.0
+            for i in range(q):
+                slot_free += fp[i]
+            start = slot_free if F is None else max(F, slot_free)
+            F = start + c2g[j]
+            s_j = 0.0
+            for i in range(j):
+                s_j += fp[i]
+            if F > s_j:
+                return False
+        return True
+
     def hard(d, g):
-        return fp_hard(d, g) and bp_hard(d, g) and cpu_ok(g)
+        return fp_hard(d, g) and bp_hard(d, g) and cpu_ok(g) and serial_ok(d, g)
 
     mems = [w for w in range(L + 1) if mem(w, w)]
     if not mems:
@@ -109,15 +132,22 @@ def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None
         gmin = 0
         while gmin < L and not cpu_ok(gmin):
             gmin += 1
+
+        def g_for(d):
+            cands = [x for x in range(max(d, gmin), L + 1) if mem(d, x)]
+            if not cands:
+                return None
+            return max(cands) if fill_gpu else (max(d, gmin) if mem(d, max(d, gmin)) else None)
+
         for d in range(L):
-            g = max(d, gmin)
-            if mem(d, g) and hard(d, g) and soft(d):
+            g = g_for(d)
+            if g is not None and hard(d, g) and soft(d):
                 best, reason = (d, g), 0
                 break
         if best is None:
             for d in range(L + 1):
-                g = max(d, gmin)
-                if mem(d, g) and hard(d, g):
+                g = g_for(d)
+                if g is not None and hard(d, g):
                     best, reason = (d, g), 1
                     break
     if best is None:

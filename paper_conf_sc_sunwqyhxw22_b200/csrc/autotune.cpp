@@ -95,7 +95,20 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
   auto gpu_step = [&](int g) { return fp.sum(0, L) + bp.sum(0, L) + ogpu.sum(0, g); };
   const double rho = P->cpu_util_max > 0.0 && P->cpu_util_max < 1.0 ? P->cpu_util_max : 1.0;
   auto cpu_ok = [&](int g) { return !P->cpu_hard || cpu_total(g) <= rho * gpu_step(g); };
-  auto hard = [&](int d, int g) { return fp_hard(d, g) && bp_hard(d, g) && cpu_ok(g); };
+  // fp_serial (R23): the FP fetches of the host layers share ONE link, so (1b) per layer is
+  // not enough when t_c2g > t_fp.  With no stalls position p starts computing at S(p) = Σ_{i<p} t_fp;
+  // the fetch of host layer j may start once its slot frees (position j-d-1 done, i.e. S(j-d)) and
+  // after the previous fetch: F(j) = max(F(j-1), S(max(0, j-d))) + t_c2g[j], and must land by S(j).
+  auto fp_serial_ok = [&](int d, int g) {
+    if (!P->fp_serial) return true;
+    double F = -INFINITY;
+    for (int j = g; j < L; ++j) {
+      F = std::max(F, fp.sum(0, std::max(0, j - d))) + at(P->t_c2g, j);
+      if (F > fp.sum(0, j)) return false;
+    }
+    return true;
+  };
+  auto hard = [&](int d, int g) { return fp_hard(d, g) && bp_hard(d, g) && cpu_ok(g) && fp_serial_ok(d, g); };
 
   int wmax = -1;
   for (int w = 0; w <= L; ++w)
@@ -113,13 +126,24 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
   } else {
     int gmin = 0;
     while (gmin < L && !cpu_ok(gmin)) ++gmin;
+    // g for a ring of d+1: the smallest meeting the CPU constraint (the paper's "min m"), or with
+    // fill_gpu the largest the memory leaves (every GPU-optimised layer takes its ~30-40 B/param of
+    // CPU-Adam + DMA traffic off the host DRAM); -1 if none fits
+    auto g_for = [&](int d) {
+      const int lo = std::max(d, gmin);
+      if (!P->fill_gpu) return mem_ok(d, lo) ? lo : -1;
+      int g = -1;
+      for (int x = lo; x <= L; ++x)
+        if (mem_ok(d, x)) g = x;
+      return g;
+    };
     for (int d = 0; d < L && best_d < 0; ++d) {
-      const int g = std::max(d, gmin);
-      if (mem_ok(d, g) && hard(d, g) && soft(d)) best_d = d, best_g = g, reason = 0;
+      const int g = g_for(d);
+      if (g >= 0 && hard(d, g) && soft(d)) best_d = d, best_g = g, reason = 0;
     }
     for (int d = 0; d <= L && best_d < 0; ++d) {
-      const int g = std::max(d, gmin);
-      if (mem_ok(d, g) && hard(d, g)) best_d = d, best_g = g, reason = 1;
+      const int g = g_for(d);
+      if (g >= 0 && hard(d, g)) best_d = d, best_g = g, reason = 1;
     }
   }
   if (best_d < 0) best_d = best_g = wmax, reason = 2;
@@ -128,7 +152,7 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
   R->ring_slots = best_d + 1;
   R->w_max_memory = wmax;
   R->reason = reason;
-  R->fp_hard_ok = fp_hard(best_d, best_g);
+  R->fp_hard_ok = fp_hard(best_d, best_g) && fp_serial_ok(best_d, best_g);
   R->bp_hard_ok = bp_hard(best_d, best_g);
   R->soft_ok = soft(best_d);
   // eq. 3: t_opt_cpu^k ≤ Σ_{i=0}^{k}(t_fp^i + t_bp^i) + Σ_{i<g} t_opt_gpu^i,  k ∈ [g, L)

@@ -289,6 +289,7 @@ struct sh_ctx {
     int fd = -1;  // NEXT-2: >= 0 for a file-backed (spilled, pageable) block
   };
   std::vector<HostBlock> hblocks;  // [L]
+  std::vector<HostBlock> hshadow;  // [L] bf16 shadows added after autotune (SH_FLAG_LATE_SHADOW)
   HostBlock hland;
   size_t host_bytes = 0;
   // NEXT-2 secondary-storage tier: host-optimised layers beyond the pinned
@@ -378,6 +379,7 @@ struct sh_ctx {
   // ---- profiling
   ProfSet prof[2];
   std::vector<double> p_fp, p_bp, p_c2g, p_g2c, p_stage, p_ogpu, p_ocpu, p_slot, p_gstate;
+  std::vector<double> p_c2g_out;  // t_c2g as handed to the solver (after the planned fetch mode)
   std::vector<int64_t> p_slot_i, p_gstate_i;
   std::vector<double> cpu_ms_layer;  // host timing of CPU Adam per layer (last)
   std::vector<sh_trace_event> trace;
@@ -640,7 +642,7 @@ void worker_loop(sh_ctx* c, int tid) {
     const LayerLayout& Lx = c->lay[x];
     const int64_t b = job->lo + chunk * kCpuChunk, e = std::min(job->hi, b + kCpuChunk);
     cpu::adamw_range(c->h_master[x], c->h_m[x], c->h_v[x], c->landing[job->landing],
-                     c->shadow ? c->h_shadow[x] : nullptr, b, e, Lx.n_decay, job->sc, c->clip, coef);
+                     c->h_shadow[x], b, e, Lx.n_decay, job->sc, c->clip, coef);
     const double dt = now_ms() - t0;
     double cur = c->cpu_ms.load();
     while (!c->cpu_ms.compare_exchange_weak(cur, cur + dt)) {
@@ -686,7 +688,7 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
     Job* jp = j.get();
     const float coef = 1.0f;
     cpu::adamw_range(c->h_master[jp->layer], c->h_m[jp->layer], c->h_v[jp->layer],
-                     c->landing[jp->landing], c->shadow ? c->h_shadow[jp->layer] : nullptr, jp->lo,
+                     c->landing[jp->landing], c->h_shadow[jp->layer], jp->lo,
                      jp->hi, c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
     finish_job(c, jp);
     return;
@@ -839,7 +841,7 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
         const double ms = ev_ms(P.c2g0[ph][i], P.c2g1[ph][i]);
         c->p_c2g[i] = ms;
         c->h2d_busy += ms;
-        c->h2d_prof_bytes += (int64_t)((c->bf16 && !c->shadow) ? 4 : c->cb) *
+        c->h2d_prof_bytes += (int64_t)((c->bf16 && !c->h_shadow[i]) ? 4 : c->cb) *
                              (c->slice_fetch && !c->no_collective ? c->shi[i] - c->slo[i] : c->lay[i].n_pad);
       }
     if (P.rec_g2c[i]) {
@@ -945,8 +947,8 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   const int64_t need = c->step;
   // bf16 mode fetches the bf16 shadow; fp32 mode the master; SH_FLAG_FETCH_FP32 fetches the fp32
   // master into the slot's (idle) grad half and K1 casts it into the param half on the H2D stream
-  const bool cast = c->bf16 && !c->shadow;
-  const void* src = c->shadow ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];
+  const bool cast = c->bf16 && !c->h_shadow[y];
+  const void* src = c->h_shadow[y] ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];
   const int64_t eb = cast ? 4 : (int64_t)c->cb;  // fetched bytes per element
   const int64_t bytes = eb * n;
   // NEXT-1 slice fetch: this rank's slice over PCIe, the rest over NVLink (in-place all-gather)
@@ -1237,6 +1239,43 @@ void release_host_layer(sh_ctx* c, int x) {
   hb = {};
   c->h_master[x] = c->h_m[x] = c->h_v[x] = nullptr;
   c->h_shadow[x] = nullptr;
+  auto& sb = c->hshadow[x];
+  if (sb.p) {
+    host_block_free(sb.p, sb.bytes);
+    c->host_bytes -= sb.bytes;
+    sb = {};
+  }
+}
+
+// SH_FLAG_LATE_SHADOW: give every host-optimised layer without one a bf16 shadow in its own pinned
+// block (the host RAM the GPU set gave back), written from the master with the CPU Adam's RNE cast,
+// so its prefetches move 2 instead of 4 B/param over the link.  Stops quietly at the first block
+// the RAM refuses (those layers keep the fp32 fetch + K1 cast).  Between steps, engine idle.
+sh_status enable_late_shadow(sh_ctx* c) {
+  if (!c->bf16 || c->shared) return SH_OK;
+  for (int x = c->w; x < c->L; ++x) {
+    if (c->h_shadow[x] || !c->h_master[x]) continue;
+    const int64_t n = c->lay[x].n_pad;
+    const size_t bytes = align_up(2 * n, 1 << 21);
+    char* p = nullptr;
+    if (host_block_alloc(bytes, c->n_threads, &p) != SH_OK) {
+      clear_error();
+      break;
+    }
+    c->hshadow[x] = {p, bytes, -1};
+    c->host_bytes += bytes;
+    uint16_t* sh16 = reinterpret_cast<uint16_t*>(p);
+    const int nt = std::max(1, c->n_threads);
+    std::vector<std::thread> ts;
+    const int64_t chunk = align_up((n + nt - 1) / nt, 16);
+    for (int t = 0; t < nt; ++t) {
+      const int64_t b = t * chunk, e = std::min(n, b + chunk);
+      if (b < e) ts.emplace_back([=] { cpu::cast_bf16_range(c->h_master[x], sh16, b, e); });
+    }
+    for (auto& th : ts) th.join();
+    c->h_shadow[x] = sh16;
+  }
+  return SH_OK;
 }
 
 sh_status ensure_host_layer(sh_ctx* c, int x) {
@@ -1399,7 +1438,7 @@ sh_status apply_window(sh_ctx* c, int w_new) {
     CKC(c, cudaMemcpy(c->h_master[x] + lo, c->g[x].master + lo, nb, cudaMemcpyDeviceToHost));
     CKC(c, cudaMemcpy(c->h_m[x] + lo, c->g[x].m + lo, nb, cudaMemcpyDeviceToHost));
     CKC(c, cudaMemcpy(c->h_v[x] + lo, c->g[x].v + lo, nb, cudaMemcpyDeviceToHost));
-    if (c->shadow) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], lo, c->shi[x]);
+    if (c->h_shadow[x]) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], lo, c->shi[x]);
     c->ready[x].store(c->step);
     free_g(c, x);
   }
@@ -1658,6 +1697,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   if (c->n_threads < 1) c->n_threads = 1;
   c->shadow = c->bf16 && !(cfg->flags & SH_FLAG_FETCH_FP32);
   c->hblocks.assign(c->L, {});
+  c->hshadow.assign(c->L, {});
   c->spilled.assign(c->L, 0);
   if (cfg->spill_dir && cfg->spill_dir[0]) {
     if (c->shared) {
@@ -2391,17 +2431,23 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   if (st != SH_OK) return st;
   // t_c2g of GPU-optimised layers is not observed (they are never fetched): use the bytes
   // rate of the measured host layers (same link, same size class)
-  const double fb = (c->bf16 && !c->shadow) ? 4.0 : (double)c->cb;  // fetched bytes per element
+  // fetched bytes per element (per layer: fp32 master + K1 cast without a shadow); with
+  // SH_FLAG_LATE_SHADOW the host layers will fetch a bf16 shadow after the autotune: solve for that
+  const bool late = c->bf16 && (c->cfg.flags & SH_FLAG_LATE_SHADOW) && !c->shared;
+  auto fbx = [&](int x) { return (c->bf16 && !c->h_shadow[x]) ? 4.0 : (double)c->cb; };
   double rate = 0;  // ms per byte
   int nr = 0;
   for (int x = 0; x < c->L; ++x)
-    if (c->p_c2g[x] > 0) rate += c->p_c2g[x] / (fb * c->lay[x].n_pad), nr++;
+    if (c->p_c2g[x] > 0) rate += c->p_c2g[x] / (fbx(x) * c->lay[x].n_pad), nr++;
   double grate = 0;
   int ng = 0;
   for (int x = 0; x < c->L; ++x)
     if (c->p_g2c[x] > 0) grate += c->p_g2c[x] / (4.0 * c->lay[x].n_pad), ng++;
+  c->p_c2g_out.assign(c->L, 0.0);
   for (int x = 0; x < c->L; ++x) {
-    if (c->p_c2g[x] <= 0 && nr) c->p_c2g[x] = rate / nr * fb * c->lay[x].n_pad;
+    const double fetch_b = late ? (double)c->cb : fbx(x);  // bytes per element the next fetch will move
+    c->p_c2g_out[x] = (c->p_c2g[x] > 0 && fetch_b == fbx(x)) ? c->p_c2g[x]
+                      : (nr ? rate / nr * fetch_b * c->lay[x].n_pad : 0.0);
     if (c->p_g2c[x] <= 0 && ng) c->p_g2c[x] = grate / ng * 4.0 * c->lay[x].n_pad;
     c->p_ocpu[x] = c->cpu_elems.load() > 0
                        ? c->cpu_ms.load() / c->n_threads / (double)c->cpu_elems.load() * c->lay[x].n_pad
@@ -2410,7 +2456,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   o->n_layers = c->L;
   o->t_fp = c->p_fp.data();
   o->t_bp = c->p_bp.data();
-  o->t_c2g = c->p_c2g.data();
+  o->t_c2g = c->p_c2g_out.data();
   o->t_g2c = c->p_g2c.data();
   o->t_stage = c->p_stage.data();
   o->t_opt_gpu = c->p_ogpu.data();
@@ -2437,6 +2483,8 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   // decouples, see sh_autotune_window)
   o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip &&
                         (c->D >= c->L || (!c->shared && (c->cfg.flags & SH_FLAG_GROW_LANDING))) ? 1 : 0;
+  o->fp_serial = o->decouple;  // R23: a decoupled (short) ring must also cover the serialised fetch queue
+  o->fill_gpu = o->decouple && (c->cfg.flags & SH_FLAG_FILL_GPU) ? 1 : 0;
   return SH_OK;
 }
 
@@ -2540,6 +2588,7 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
       st = c->ring_cap > 0 ? sh_set_window_ring(c, c->w, 0) : SH_OK;
     }
   }
+  if (st == SH_OK && (c->cfg.flags & SH_FLAG_LATE_SHADOW)) st = enable_late_shadow(c);
   if (wout) *wout = c->w;
   return st;
 }
@@ -2575,7 +2624,7 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
           std::memcpy(tmp.data(), mst.data(), 4 * n);
       }
     } else {
-      if (c->shadow)
+      if (c->h_shadow[layer])
         std::memcpy(tmp.data(), c->h_shadow[layer], tmp.size());
       else if (c->bf16)
         cpu::cast_bf16_range(c->h_master[layer], reinterpret_cast<uint16_t*>(tmp.data()), 0, n);
@@ -2728,6 +2777,7 @@ sh_status sh_destroy(sh_ctx* c) {
   }
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
     if (s) cudaStreamDestroy(s);
+  for (auto& b : c->hshadow) host_block_free(b.p, b.bytes);
   for (auto& b : c->hblocks) {
     if (b.fd >= 0) {
       munmap(b.p, b.bytes);

@@ -22,8 +22,8 @@ SH_PRE, SH_POST = 0, 1
 SH_READ_PARAM, SH_READ_M, SH_READ_V, SH_READ_COMPUTE, SH_READ_GRAD = 0, 1, 2, 3, 4
 SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_HARD, SH_FLAG_FETCH_FP32, \
     SH_FLAG_TEST_NO_COLLECTIVE, SH_FLAG_SLICE_FETCH, SH_FLAG_DELAY_INJECT, SH_FLAG_DECOUPLE, SH_FLAG_SPILL_EVICT, \
-    SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS, SH_FLAG_ABLATE_ALLOC, SH_FLAG_GROW_LANDING = \
-    1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192, 16384
+    SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS, SH_FLAG_ABLATE_ALLOC, SH_FLAG_GROW_LANDING, SH_FLAG_FILL_GPU, \
+    SH_FLAG_LATE_SHADOW = 1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192, 16384, 32768, 65536
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
@@ -67,7 +67,8 @@ class Profile(C.Structure):
                 ("t_stage", _PD), ("t_opt_gpu", _PD), ("t_opt_cpu", _PD), ("t_async", C.c_double),
                 ("slot_bytes", _PI64), ("gstate_bytes", _PI64), ("fixed_bytes", C.c_int64),
                 ("s_avail", C.c_int64), ("duplex", C.c_int32), ("cpu_hard", C.c_int32),
-                ("cpu_util_max", C.c_double), ("decouple", C.c_int32)]
+                ("cpu_util_max", C.c_double), ("decouple", C.c_int32), ("fp_serial", C.c_int32),
+                ("fill_gpu", C.c_int32)]
 
 
 class SolveReport(C.Structure):
@@ -232,7 +233,7 @@ def _dbl(a, n):
 
 def make_profile(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
                  slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False,
-                 cpu_hard=False, cpu_util_max=1.0, decouple=False):
+                 cpu_hard=False, cpu_util_max=1.0, decouple=False, fp_serial=False, fill_gpu=False):
     """(Profile, keep-alive arrays) for sh_solve_window / sh_autotune_window."""
     n = len(t_fp)
     keep = {}
@@ -254,6 +255,8 @@ def make_profile(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_c
     prof.cpu_hard = 1 if cpu_hard else 0
     prof.cpu_util_max = cpu_util_max
     prof.decouple = 1 if decouple else 0
+    prof.fp_serial = 1 if fp_serial else 0
+    prof.fill_gpu = 1 if fill_gpu else 0
     return prof, keep
 
 
@@ -435,7 +438,8 @@ class Engine:
         check(self._L.sh_get_profile(self.h, C.byref(p)))
         n = p.n_layers
         out = {"n_layers": n, "t_async": p.t_async, "s_avail": p.s_avail, "fixed_bytes": p.fixed_bytes,
-               "duplex": p.duplex, "cpu_hard": p.cpu_hard, "cpu_util_max": p.cpu_util_max, "decouple": p.decouple}
+               "duplex": p.duplex, "cpu_hard": p.cpu_hard, "cpu_util_max": p.cpu_util_max, "decouple": p.decouple,
+               "fp_serial": p.fp_serial, "fill_gpu": p.fill_gpu}
         for f in ("t_fp", "t_bp", "t_c2g", "t_g2c", "t_stage", "t_opt_gpu", "t_opt_cpu"):
             out[f] = [getattr(p, f)[i] for i in range(n)]
         for f in ("slot_bytes", "gstate_bytes"):

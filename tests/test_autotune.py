@@ -103,6 +103,29 @@ def test_decoupled_ring_smaller_than_gpu_set():
     assert sh.solve_window(**prof_mem, cpu_hard=True)["window"] < gmin
 
 
+def test_fp_serial_homogeneous_closed_form():
+    """R23 by hand: t_fp = a < t_c2g = c, no CPU constraint, decoupled (g = d).  The host fetches
+    (layers d..L-1) are link-bound from the step start: fetch j lands at (j - d + 1) c and is due at
+    S(j) = j a; the last layer binds: (L - d) c <= (L - 1) a  <=>  d >= L - (L - 1) a / c.  Together with
+    (1b) d a >= c and (2b) 3 d a >= c: d* = max(ceil(c / a), ceil(L - (L - 1) a / c))."""
+    for L, a, c in [(20, 1.0, 1.5), (40, 2.0, 3.0), (30, 1.0, 1.1), (16, 1.0, 4.0)]:
+        prof = homog(L, a, c, 0.0, t_stage=[0.0] * L)
+        d_star = max(math.ceil(c / a - 1e-12), math.ceil(L - (L - 1) * a / c - 1e-12))
+        got = sh.solve_window(**prof, decouple=True, fp_serial=True)
+        assert got["ring_slots"] == d_star + 1 and got["window"] == d_star, (L, a, c, got, d_star)
+        # without the serial form the paper's (1b) alone accepts a much shorter ring
+        assert sh.solve_window(**prof, decouple=True)["ring_slots"] == math.ceil(c / a - 1e-12) + 1
+
+
+def test_fill_gpu_takes_the_memory_left_by_the_ring():
+    L = 12
+    prof = homog(L, 1.0, 0.5, 0.5, t_stage=[0.0] * L, slot_bytes=[10] * L, gstate_bytes=[3] * L, s_avail=20 + 3 * 7)
+    small = sh.solve_window(**prof, decouple=True)
+    full = sh.solve_window(**prof, decouple=True, fill_gpu=True)
+    assert small["ring_slots"] == full["ring_slots"] == 2       # d = 1: (1b) t_fp >= t_c2g
+    assert small["window"] == 1 and full["window"] == 7         # 2 slots x 10 + 7 x 3 = 41 bytes
+
+
 @pytest.mark.parametrize("seed", range(60))
 def test_random_heterogeneous_matches_bruteforce(seed):
     rng = np.random.default_rng(seed)
@@ -113,7 +136,8 @@ def test_random_heterogeneous_matches_bruteforce(seed):
                 slot_bytes=rng.integers(1, 100, L), gstate_bytes=rng.integers(1, 60, L),
                 fixed_bytes=int(rng.integers(0, 50)), s_avail=int(rng.integers(100, 3000)),
                 duplex=bool(rng.integers(0, 2)), cpu_hard=bool(rng.integers(0, 2)),
-                cpu_util_max=float(rng.choice([1.0, 0.85, 0.5])), decouple=bool(rng.integers(0, 2)))
+                cpu_util_max=float(rng.choice([1.0, 0.85, 0.5])), decouple=bool(rng.integers(0, 2)),
+                fp_serial=bool(rng.integers(0, 2)), fill_gpu=bool(rng.integers(0, 2)))
     want = AO.solve(**{k: (list(v) if isinstance(v, np.ndarray) else v) for k, v in prof.items()})
     if want is None:
         with pytest.raises(sh.ShError):

@@ -80,3 +80,35 @@ def test_grow_landing_for_a_decoupled_ring():
         assert losses == ref_losses
     finally:
         tr.close()
+
+
+def test_late_shadow_bitwise():
+    """SH_FLAG_LATE_SHADOW: fp32-fetch mode switches the host layers to bf16-shadow fetches after the
+    autotune (shadow written from the master with the CPU Adam's RNE): bitwise the same training."""
+    L = TINY["L"]
+    ref_tr, ref_losses, _ = engine_run(TINY, 3, L, sh.SH_BF16_MIXED)
+    ref = engine_state(ref_tr)
+    ref_tr.close()
+    tr, losses, _ = engine_run(TINY, 1, 1, sh.SH_BF16_MIXED, attention="flash",
+                               flags=sh.SH_FLAG_FETCH_FP32 | sh.SH_FLAG_LATE_SHADOW | sh.SH_FLAG_GROW_LANDING,
+                               grad_ring_depth=1)
+    try:
+        hb = tr.engine.stats()["host_bytes"]
+        prof = dict(t_fp=[1.0] * L, t_bp=[3.0] * L, t_c2g=[0.1] * L, t_g2c=[0.1] * L, t_stage=[0.01] * L,
+                    t_opt_gpu=[0.0] * L, t_opt_cpu=[8.0] * L, cpu_hard=True, cpu_util_max=1.0, decouple=True)
+        assert tr.engine.autotune(prof) == 2
+        st = tr.engine.stats()
+        assert st["landing_buffers"] == L - 2
+        h2d0 = st["h2d_bytes"]
+        for t in (1, 2):
+            tr.set_tokens(synth.tokens(t, TINY["b"], TINY["s"], TINY["V"]))
+            tr.step_device(want_norm=True)
+            losses.append(tr.loss())
+        # host layers now fetch 2 B/param (bf16 shadow), not 4
+        per_fetch = (tr.engine.stats()["h2d_bytes"] - h2d0) / max(1, tr.engine.stats()["h2d_copies"] - st["h2d_copies"])
+        assert per_fetch <= 2 * sum(tr.mc.layer_numels()) * 1.01
+        ok, what = states_bitwise_equal(engine_state(tr), ref)
+        assert ok, what
+        assert losses == ref_losses
+    finally:
+        tr.close()
