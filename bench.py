@@ -541,10 +541,15 @@ def main():
                             "ms_per_step": res_ms / K, "frac_windowed_over_resident": res_ms / ms}
     if r["prof"]:
         p = r["prof"]
+        # the engine's solver re-run on the profile of the TIMED steps (steady state at the tuned window),
+        # with the same options the engine used after the warm-up
         rep = sh.solve_window(p["t_fp"], p["t_bp"], p["t_c2g"], p["t_g2c"], p["t_stage"], p["t_opt_gpu"],
                               p["t_opt_cpu"], p["t_async"], p["slot_bytes"], p["gstate_bytes"], p["fixed_bytes"],
-                              p["s_avail"], p["duplex"])
-        line["autotune"] = {"window": rep["window"], "reason": rep["reason"], "eq3_ok": rep["eq3_ok"],
+                              p["s_avail"], p["duplex"], p["cpu_hard"], p["cpu_util_max"], p["decouple"],
+                              p["fp_serial"], p["fill_gpu"])
+        line["autotune"] = {"note": "solver re-run on the timed steps' profile", "window": rep["window"],
+                            "ring_slots": rep["ring_slots"], "s_avail_gb": p["s_avail"] / 1e9,
+                            "decouple": p["decouple"], "reason": rep["reason"], "eq3_ok": rep["eq3_ok"],
                             "eq3_min_slack_ms": rep["eq3_min_slack_ms"],
                             "t_fp_ms": float(np.median(p["t_fp"])), "t_bp_ms": float(np.median(p["t_bp"])),
                             "t_c2g_ms": float(np.median(p["t_c2g"])), "t_g2c_ms": float(np.median(p["t_g2c"])),

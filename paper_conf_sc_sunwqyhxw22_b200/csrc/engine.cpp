@@ -2435,10 +2435,17 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   // SH_FLAG_LATE_SHADOW the host layers will fetch a bf16 shadow after the autotune: solve for that
   const bool late = c->bf16 && (c->cfg.flags & SH_FLAG_LATE_SHADOW) && !c->shared;
   auto fbx = [&](int x) { return (c->bf16 && !c->h_shadow[x]) ? 4.0 : (double)c->cb; };
-  double rate = 0;  // ms per byte
+  double rate = 0;  // ms per byte: mean of the measured fetches
+  double rate_min = 0;  // the fastest one: the warm-up runs with most layers on the host, so its
+                        // fetches compete with the heaviest CPU-Adam traffic; the tuned run's don't
   int nr = 0;
   for (int x = 0; x < c->L; ++x)
-    if (c->p_c2g[x] > 0) rate += c->p_c2g[x] / (fbx(x) * c->lay[x].n_pad), nr++;
+    if (c->p_c2g[x] > 0) {
+      const double r = c->p_c2g[x] / (fbx(x) * c->lay[x].n_pad);
+      rate += r;
+      rate_min = nr == 0 ? r : std::min(rate_min, r);
+      nr++;
+    }
   double grate = 0;
   int ng = 0;
   for (int x = 0; x < c->L; ++x)
@@ -2447,7 +2454,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   for (int x = 0; x < c->L; ++x) {
     const double fetch_b = late ? (double)c->cb : fbx(x);  // bytes per element the next fetch will move
     c->p_c2g_out[x] = (c->p_c2g[x] > 0 && fetch_b == fbx(x)) ? c->p_c2g[x]
-                      : (nr ? rate / nr * fetch_b * c->lay[x].n_pad : 0.0);
+                      : (nr ? (late ? rate_min : rate / nr) * fetch_b * c->lay[x].n_pad : 0.0);
     if (c->p_g2c[x] <= 0 && ng) c->p_g2c[x] = grate / ng * 4.0 * c->lay[x].n_pad;
     c->p_ocpu[x] = c->cpu_elems.load() > 0
                        ? c->cpu_ms.load() / c->n_threads / (double)c->cpu_elems.load() * c->lay[x].n_pad
@@ -2549,6 +2556,18 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   sh_status st = sh_solve_window(&p, &rep);
   if (st != SH_OK) return st;
   c->autotune_pending = false;
+  if (getenv("SH_DEBUG_AUTOTUNE")) {
+    double fp = 0, c2g = 0, g2c = 0, cpu = 0;
+    for (int x = 0; x < p.n_layers; ++x)
+      fp += p.t_fp[x], c2g += p.t_c2g ? p.t_c2g[x] : 0, g2c += p.t_g2c ? p.t_g2c[x] : 0,
+          cpu += p.t_opt_cpu ? p.t_opt_cpu[x] : 0;
+    const double n = p.n_layers;
+    fprintf(stderr, "[sh autotune] w=%d ring=%d reason=%d decouple=%d fp_serial=%d fill=%d s_avail=%.1fGB "
+            "mean t_fp=%.2f t_c2g=%.2f t_g2c=%.2f t_cpu=%.2f ms, slot=%.2fGB gstate=%.2fGB\n",
+            rep.window, rep.ring_slots, rep.reason, p.decouple, p.fp_serial, p.fill_gpu, p.s_avail / 1e9, fp / n,
+            c2g / n, g2c / n, cpu / n, p.slot_bytes ? p.slot_bytes[0] / 1e9 : 0.0,
+            p.gstate_bytes ? p.gstate_bytes[0] / 1e9 : 0.0);
+  }
   int32_t w = rep.window;
   int32_t ring = p.decouple && !c->clip ? rep.ring_slots : 0;
   if (c->shared) {  // one shared host store: the whole job must switch to the same window
