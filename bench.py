@@ -51,6 +51,10 @@ CONFIGS = {
 C4MAX_W0 = 32
 FETCH_FP32_DEFAULT = {"c4", "c4max"}
 CPU_HARD_DEFAULT = {"c3", "c4", "c4max"}   # autotune with the eq. 3 CPU-throughput constraint (R19)
+# autotune with the B200 extensions of the window model by default (R22/R23): landing-ring
+# growth, GPU set filling the HBM a decoupled ring leaves, late bf16 host shadows (C4: 7.30 -> 7.92
+# samples/s, profiles/r01_bench_default_c4_v3.json vs r01_bench_c4_tuned_coupled.json)
+TUNED_DEFAULT = {"c3", "c4"}
 
 
 def mem_available() -> int:
@@ -262,6 +266,8 @@ def main():
     ap.add_argument("--no-decouple", action="store_true", help="autotune keeps the ring coupled to the GPU set")
     ap.add_argument("--fill-gpu", action="store_true", help="decoupled autotune fills HBM with GPU-optimised layers")
     ap.add_argument("--late-shadow", action="store_true", help="fp32-fetch mode: bf16 host shadows after the autotune")
+    ap.add_argument("--plain-autotune", action="store_true",
+                    help="c3/c4: autotune without --grow-landing/--fill-gpu/--late-shadow (the round-1 default)")
     ap.add_argument("--ring", type=int, default=0, help="fixed ring size (prefetch distance + 1) with a fixed --window")
     ap.add_argument("--sync-cpu", action="store_true",
                     help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
@@ -269,6 +275,8 @@ def main():
     ap.add_argument("--executors", type=int, default=1,
                     help="NEXT-3: K multi-stream executors (micro-batches of batch/K on K streams, PAPER.md:227-242)")
     args = ap.parse_args()
+    if args.config in TUNED_DEFAULT and not args.plain_autotune and args.window in (-2, -1):
+        args.grow_landing = args.fill_gpu = args.late_shadow = True
     if args.warmup < 3:
         args.warmup = 3
     if args.impl == "reference":
@@ -478,6 +486,10 @@ def main():
                              "bytes": r["st1"]["spill_bytes"], "evict": args.spill_evict} if args.spill_dir else None,
                    "host_store": ("one shared /dev/shm store, rank-sliced offload + CPU Adam" if shm_name else
                                   "private per rank") if world > 1 else "private",
+                   "numa": {"nodes": r["st1"]["numa_nodes"],
+                            "policy": ("auto", "split", "local", "interleave", "none")[r["st1"]["numa_policy"]],
+                            "gpu_node": r["st1"]["numa_gpu_node"], "pinned_workers": r["st1"]["numa_pinned_workers"],
+                            "bound_bytes": r["st1"]["numa_bound_bytes"]},
                    "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),
                    "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
                    "grad_landing_buffers": r["st1"]["landing_buffers"], "host_store_bytes": r["st1"]["host_bytes"],

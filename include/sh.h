@@ -192,7 +192,23 @@ typedef struct {
                                        Only host-optimised layers hold a host block (a layer joining the
                                        GPU set gives its block back), so a larger warm-up window lowers
                                        the host RAM the store needs from the start */
+  int32_t numa_policy;              /* SH_NUMA_*: where the pinned host store lives and which cores update
+                                       it.  0 = SH_NUMA_AUTO */
 } sh_config;
+
+/* NUMA placement policies (sh_config.numa_policy).  Placement is an mbind(2) before the first
+ * touch (MPOL_PREFERRED: a full node spills to another instead of failing); CPU Adam workers are
+ * pinned with pthread_setaffinity_np.  On a single-node host every policy is a no-op. */
+#define SH_NUMA_AUTO 0        /* SPLIT for a private store on a multi-node host; LOCAL with data
+                                 parallelism (shared store: slice r on GPU r's node) */
+#define SH_NUMA_SPLIT 1       /* layer x's block on node x mod n_nodes; workers spread over the nodes in
+                                 proportion to their cores, each preferring the jobs of its own node's
+                                 layers (takes others only when it would idle); landing buffers
+                                 interleaved */
+#define SH_NUMA_LOCAL 2       /* every block on the GPU's node (PCI numa_node of the device), workers
+                                 pinned to that node (cpu_threads 0 = that node's cores) */
+#define SH_NUMA_INTERLEAVE 3  /* every block page-interleaved over all nodes, workers unpinned */
+#define SH_NUMA_NONE 4        /* first touch only */
 
 /* Per-layer profile consumed by the window solver (PAPER.md:132 notation; times in ms,
  * sizes in bytes).  Arrays have n_layers entries; NULL arrays are treated as zeros. */
@@ -268,6 +284,11 @@ typedef struct {
   int32_t spilled_layers;       /* number of layers in the spill tier */
   int32_t landing_buffers;      /* host landing buffers for offloaded gradients (grows when the autotuner
                                    decouples the ring on a private store) */
+  int32_t numa_nodes;           /* NUMA nodes of the host (sysfs) */
+  int32_t numa_policy;          /* policy in effect (SH_NUMA_AUTO resolved) */
+  int32_t numa_gpu_node;        /* node index of this context's GPU */
+  int32_t numa_pinned_workers;  /* CPU Adam workers pinned to a node */
+  int64_t numa_bound_bytes;     /* host-store bytes placed with mbind */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */
@@ -385,6 +406,24 @@ sh_status sh_get_trace(sh_ctx* ctx, sh_trace_event* out, int32_t cap, int32_t* n
 
 /* Thread-local message of the last failed call ("" if none). */
 const char* sh_last_error(void);
+
+/* ---- NUMA host logic; pure functions of the topology, no CUDA context needed.
+ * SH_SYSFS_ROOT (tests) prefixes every sysfs path read by them. */
+/* Online nodes: writes up to cap node ids and their CPU counts; returns the node count (>= 1; a
+ * host without NUMA sysfs is one node holding every online CPU). */
+int32_t sh_numa_topology(int32_t* node_ids, int32_t* n_cpus, int32_t cap);
+/* Node INDEX (into sh_numa_topology's order) that host-store unit `unit` (a layer) is placed on
+ * under `policy`, -1 = no binding, -2 = interleaved.  gpu_node: the GPU's node index; shared: 1
+ * for a data-parallel shared store (AUTO resolves to LOCAL there). */
+int32_t sh_numa_plan(int32_t policy, int32_t unit, int32_t n_nodes, int32_t gpu_node, int32_t shared);
+/* Node index CPU Adam worker `tid` of n_threads is pinned to (-1: not pinned). */
+int32_t sh_numa_worker_node(int32_t policy, int32_t tid, int32_t n_threads, int32_t gpu_node);
+/* Node index of a PCI device ("0000:1b:00.0", as cudaDeviceGetPCIBusId prints it); 0 if unknown. */
+int32_t sh_numa_node_of_pci(const char* bus_id);
+/* Self-check of the placement primitive: mbind(MPOL_BIND) `bytes` of fresh anonymous memory to
+ * node id `node_id`, touch it, return the node get_mempolicy reports for its first and last page
+ * (-1 if they differ or a syscall failed). */
+int32_t sh_numa_bind_check(int32_t node_id, int64_t bytes);
 
 int32_t sh_abi_version(void);
 

@@ -292,6 +292,17 @@ struct sh_ctx {
   std::vector<HostBlock> hshadow;  // [L] bf16 shadows added after autotune (SH_FLAG_LATE_SHADOW)
   HostBlock hland;
   size_t host_bytes = 0;
+  // NUMA placement (numa.cpp): resolved policy, node count, this GPU's node index,
+  // per-layer target node (index, numa::kNone / kInterleave), per-worker node, bytes bound
+  int numa_policy = SH_NUMA_NONE;
+  int numa_nodes = 1;
+  int numa_gpu = 0;
+  std::vector<int> layer_node;
+  std::vector<int> worker_node;
+  std::vector<int> slice_node;  // shared store: node index of rank r's slices
+  int land_node = -1;
+  std::atomic<int64_t> numa_bound{0};
+  std::atomic<int> numa_pinned{0};
   // NEXT-2 secondary-storage tier: host-optimised layers beyond the pinned
   // budget live in mmap'ed files (MAP_SHARED, unlinked at creation) under spill_dir; their
   // fetches go through pinned bounce buffers, the CPU Adam works on the mapping (page cache)
@@ -543,7 +554,8 @@ int64_t mem_available_bytes() {
 
 // mmap + THP advice + parallel first touch + cudaHostRegister.  Refuses (instead of letting the
 // kernel OOM-kill the process) when the block would leave less than SH_HOST_MARGIN_GB free.
-sh_status host_block_alloc(size_t bytes, int threads, char** out) {
+sh_status host_block_alloc(size_t bytes, int threads, char** out, int node = numa::kNone,
+                           std::atomic<int64_t>* bound = nullptr) {
   *out = nullptr;
   const char* mg = getenv("SH_HOST_MARGIN_GB");
   const int64_t margin = (int64_t)((mg ? atof(mg) : 3.0) * (1ll << 30));
@@ -558,6 +570,8 @@ sh_status host_block_alloc(size_t bytes, int threads, char** out) {
     set_error("host store: mmap of %lld B failed", (long long)bytes);
     return SH_ERR_OOM_HOST;
   }
+  // NUMA placement before the first touch (a no-op on a single-node host)
+  if (node != numa::kNone && numa::bind_range(p, bytes, node) && bound) bound->fetch_add((int64_t)bytes);
   parallel_touch(p, bytes, threads);
   if (cudaHostRegister(p, bytes, cudaHostRegisterPortable) != cudaSuccess) {
     cudaGetLastError();
@@ -598,7 +612,11 @@ void finish_job(sh_ctx* c, Job* j) {
 }
 
 void worker_loop(sh_ctx* c, int tid) {
-  (void)tid;
+  const int my_node = c->worker_node.empty() ? numa::kNone : c->worker_node[tid];
+  if (my_node != numa::kNone && numa::pin_thread(my_node)) c->numa_pinned.fetch_add(1);
+  // SPLIT: prefer the layers placed on this worker's node (local DRAM); take others only when
+  // none of those is eligible, so no worker idles while work is queued
+  auto local = [&](const Job* jp) { return my_node < 0 || c->layer_node[jp->layer] == my_node; };
   for (;;) {
     Job* job = nullptr;
     int64_t chunk = -1;
@@ -628,11 +646,12 @@ void worker_loop(sh_ctx* c, int tid) {
       }
       if (c->pool_stop || c->failed.load()) return;
       // lowest layer first: it is prefetched first by the next FP (eq. 3)
-      for (auto& jp : c->jobs) {
-        if (!eligible(jp.get())) continue;
-        if (!job || jp->step < job->step || (jp->step == job->step && jp->layer < job->layer))
-          job = jp.get();
-      }
+      for (int pass = 0; pass < 2 && !job; ++pass)
+        for (auto& jp : c->jobs) {
+          if (!eligible(jp.get()) || (pass == 0 && !local(jp.get()))) continue;
+          if (!job || jp->step < job->step || (jp->step == job->step && jp->layer < job->layer))
+            job = jp.get();
+        }
       chunk = job->next++;
       if (c->clip) coef = c->coef_of_step[job->step & 1];
     }
@@ -1125,7 +1144,8 @@ std::string shm_path(const sh_ctx* c, const char* suffix, int x = -1) {
 }
 
 // Map (rank 0: create) a /dev/shm segment of `bytes`; page-lock it in this process.
-sh_status shm_map(sh_ctx* c, const std::string& path, size_t bytes, bool create, char** out, bool touch) {
+sh_status shm_map(sh_ctx* c, const std::string& path, size_t bytes, bool create, char** out, bool touch,
+                  const std::function<void(char*)>& before_touch = nullptr) {
   *out = nullptr;
   int fd = -1;
   if (create) {
@@ -1164,6 +1184,7 @@ sh_status shm_map(sh_ctx* c, const std::string& path, size_t bytes, bool create,
     return SH_ERR_OOM_HOST;
   }
   madvise(p, bytes, MADV_HUGEPAGE);
+  if (create && touch && before_touch) before_touch(static_cast<char*>(p));
   if (create && touch) parallel_touch(static_cast<char*>(p), bytes, c->n_threads);
   if (touch && cudaHostRegister(p, bytes, cudaHostRegisterPortable) != cudaSuccess) {
     cudaGetLastError();
@@ -1213,7 +1234,7 @@ sh_status ensure_bounce(sh_ctx* c) {
   if (c->bounce[0]) return SH_OK;
   const size_t b = align_up(4 * c->max_pad, 1 << 21);  // fp32 fetch is the largest
   for (int k = 0; k < 2; ++k) {
-    sh_status st = host_block_alloc(b, c->n_threads, &c->bounce[k]);
+    sh_status st = host_block_alloc(b, c->n_threads, &c->bounce[k], c->land_node, &c->numa_bound);
     if (st != SH_OK) return st;
     CKC(c, cudaEventCreateWithFlags(&c->ev_bounce[k], cudaEventDisableTiming));
     CKC(c, cudaEventRecord(c->ev_bounce[k], c->h2d));
@@ -1258,7 +1279,7 @@ sh_status enable_late_shadow(sh_ctx* c) {
     const int64_t n = c->lay[x].n_pad;
     const size_t bytes = align_up(2 * n, 1 << 21);
     char* p = nullptr;
-    if (host_block_alloc(bytes, c->n_threads, &p) != SH_OK) {
+    if (host_block_alloc(bytes, c->n_threads, &p, c->layer_node[x], &c->numa_bound) != SH_OK) {
       clear_error();
       break;
     }
@@ -1286,12 +1307,27 @@ sh_status ensure_host_layer(sh_ctx* c, int x) {
   int fd = -1;
   sh_status st = SH_OK;
   if (c->shared) {
-    st = shm_map(c, shm_path(c, "L", x), bytes, c->rank == 0, &p, true);
+    // data parallel: rank r's slice of each of the four arrays on GPU r's node
+    auto place = [c, x, n](char* base) {
+      if (c->slice_node.empty()) return;
+      const int64_t cs = align_up((n + c->W - 1) / c->W, kPad);
+      const int n_arr = c->shadow ? 4 : 3;
+      for (int r = 0; r < c->W; ++r) {
+        const int64_t lo = std::min(n, (int64_t)r * cs), hi = std::min(n, (int64_t)(r + 1) * cs);
+        if (lo >= hi || c->slice_node[r] == numa::kNone) continue;
+        for (int a = 0; a < n_arr; ++a) {
+          const int64_t esz = a < 3 ? 4 : 2, off = a < 3 ? 4 * a * n : 12 * n;
+          if (numa::bind_range(base + off + esz * lo, (size_t)(esz * (hi - lo)), c->slice_node[r]))
+            c->numa_bound.fetch_add(esz * (hi - lo));
+        }
+      }
+    };
+    st = shm_map(c, shm_path(c, "L", x), bytes, c->rank == 0, &p, true, place);
   } else {
     const bool can_spill = !c->spill_dir.empty();
     bool spill = can_spill && c->pin_budget > 0 && (int64_t)(c->host_bytes + bytes) > c->pin_budget;
     if (!spill) {
-      st = host_block_alloc(bytes, c->n_threads, &p);
+      st = host_block_alloc(bytes, c->n_threads, &p, c->layer_node[x], &c->numa_bound);
       if (st == SH_ERR_OOM_HOST && can_spill) {  // host RAM exhausted: overflow to the spill tier
         clear_error();
         spill = true;
@@ -1492,7 +1528,7 @@ sh_status grow_landing(sh_ctx* c, int D_new) {
   const int64_t lb = align_up(4 * c->max_pad, 4096);
   const size_t bytes = align_up((int64_t)D_new * lb + 4096, 1 << 21);
   char* p = nullptr;
-  st = host_block_alloc(bytes, c->n_threads, &p);
+  st = host_block_alloc(bytes, c->n_threads, &p, c->land_node, &c->numa_bound);
   if (st != SH_OK) return st;
   const float coef0 = c->h_coef[0], coef1 = c->h_coef[1];
   host_block_free(c->hland.p, c->hland.bytes);
@@ -1693,8 +1729,40 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   }
 
   // ---- host store: per layer master | m | v | shadow, plus landing buffers, 2 MiB aligned
-  c->n_threads = cfg->cpu_threads > 0 ? cfg->cpu_threads : (int)std::thread::hardware_concurrency();
-  if (c->n_threads < 1) c->n_threads = 1;
+  {  // NUMA plan (numa.cpp): topology, the GPU's node, per-layer / landing / slice / worker nodes
+    const numa::Topology& topo = numa::topology();
+    c->numa_nodes = (int)topo.node_ids.size();
+    c->numa_gpu = numa::gpu_node_index(cfg->device);
+    if (cfg->numa_policy < SH_NUMA_AUTO || cfg->numa_policy > SH_NUMA_NONE) {
+      set_error("sh_init: numa_policy %d is not one of SH_NUMA_*", cfg->numa_policy);
+      return SH_ERR_INVALID;
+    }
+    c->numa_policy = numa::resolve_policy(cfg->numa_policy, c->numa_nodes, dp);
+    c->layer_node.assign(c->L, numa::kNone);
+    for (int x = 0; x < c->L; ++x) c->layer_node[x] = numa::plan_node(c->numa_policy, x, c->numa_nodes, c->numa_gpu);
+    c->land_node = c->numa_policy == SH_NUMA_SPLIT ? numa::plan_node(SH_NUMA_INTERLEAVE, 0, c->numa_nodes, 0)
+                                                    : numa::plan_node(c->numa_policy, 0, c->numa_nodes, c->numa_gpu);
+    if (c->shared && c->numa_policy != SH_NUMA_NONE) {
+      // rank r drives device (device - rank + r): one process per GPU in device order, as launched
+      // by torchrun / bench.py.  Under LOCAL slice r lives on its GPU's node; otherwise as planned.
+      int n_dev = 0;
+      if (cudaGetDeviceCount(&n_dev) != cudaSuccess) cudaGetLastError();
+      c->slice_node.assign(c->W, numa::kNone);
+      for (int r = 0; r < c->W; ++r) {
+        const int dev = cfg->device - cfg->rank + r;
+        const int gn = (dev >= 0 && dev < n_dev) ? numa::gpu_node_index(dev) : 0;
+        c->slice_node[r] = numa::plan_node(c->numa_policy, r, c->numa_nodes, gn);
+      }
+    }
+    int dflt = (int)std::thread::hardware_concurrency();
+    if (c->numa_policy == SH_NUMA_LOCAL && c->numa_nodes > 1 && !topo.cpus[c->numa_gpu].empty())
+      dflt = (int)topo.cpus[c->numa_gpu].size();  // LOCAL: the GPU node's cores
+    c->n_threads = cfg->cpu_threads > 0 ? cfg->cpu_threads : dflt;
+    if (c->n_threads < 1) c->n_threads = 1;
+    c->worker_node.assign(c->n_threads, numa::kNone);
+    for (int t = 0; t < c->n_threads; ++t)
+      c->worker_node[t] = numa::worker_node(c->numa_policy, t, c->n_threads, c->numa_gpu);
+  }
   c->shadow = c->bf16 && !(cfg->flags & SH_FLAG_FETCH_FP32);
   c->hblocks.assign(c->L, {});
   c->hshadow.assign(c->L, {});
@@ -1720,7 +1788,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     const int64_t lb = align_up(4 * c->max_pad, 4096);
     const size_t bytes = align_up((int64_t)c->D * lb + 4096, 1 << 21);
     char* p = nullptr;
-    sh_status st = host_block_alloc(bytes, c->n_threads, &p);
+    sh_status st = host_block_alloc(bytes, c->n_threads, &p, c->land_node, &c->numa_bound);
     if (st != SH_OK) return st;
     c->hland = {p, bytes};
     c->host_bytes += bytes;
@@ -2735,6 +2803,11 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->spill_bytes = (int64_t)c->spill_bytes;
   o->landing_buffers = c->D;
   o->spilled_layers = c->n_spilled;
+  o->numa_nodes = c->numa_nodes;
+  o->numa_policy = c->numa_policy;
+  o->numa_gpu_node = c->numa_gpu;
+  o->numa_pinned_workers = c->numa_pinned.load();
+  o->numa_bound_bytes = c->numa_bound.load();
   return SH_OK;
 }
 

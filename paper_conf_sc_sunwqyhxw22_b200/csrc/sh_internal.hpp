@@ -92,4 +92,23 @@ uint16_t rne_bf16(float x);
 bool has_avx512();
 }  // namespace cpu
 
+// ---- NUMA placement (numa.cpp) ---------------------------------------------------------
+namespace numa {
+constexpr int kNone = -1;        // no binding / not pinned
+constexpr int kInterleave = -2;  // page-interleaved over all nodes
+struct Topology {
+  std::vector<int> node_ids;          // online node ids (index = "node index")
+  std::vector<std::vector<int>> cpus; // CPUs of each node
+};
+bool parse_cpulist(const char* s, std::vector<int>* out);
+const Topology& topology();
+int gpu_node_index(int device);
+int resolve_policy(int policy, int n_nodes, bool shared);
+int plan_node(int policy, int unit, int n_nodes, int gpu_node);
+int worker_node(int policy, int tid, int n_threads, int gpu_node);
+bool bind_range(void* p, size_t bytes, int node_index);
+int node_of_page(const void* p);
+bool pin_thread(int node_index);
+}  // namespace numa
+
 }  // namespace sh

@@ -32,7 +32,11 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_last_error", "sh_abi_version", "sh_nccl_get_unique_id", "sh_adam_scalars_for",
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
            "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end", "sh_set_window_ring",
-           "sh_executor_grads", "sh_op_exec_reduce_gpu")
+           "sh_executor_grads", "sh_op_exec_reduce_gpu", "sh_numa_topology", "sh_numa_plan",
+           "sh_numa_worker_node", "sh_numa_node_of_pci", "sh_numa_bind_check")
+
+# NUMA placement policies (sh_config.numa_policy, include/sh.h)
+SH_NUMA_AUTO, SH_NUMA_SPLIT, SH_NUMA_LOCAL, SH_NUMA_INTERLEAVE, SH_NUMA_NONE = range(5)
 
 
 class ShError(RuntimeError):
@@ -55,7 +59,7 @@ class Config(C.Structure):
                 ("world_size", C.c_int32), ("rank", C.c_int32),
                 ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p),
                 ("n_executors", C.c_int32), ("spill_dir", C.c_char_p), ("host_pin_budget_bytes", C.c_int64),
-                ("warmup_window", C.c_int32)]
+                ("warmup_window", C.c_int32), ("numa_policy", C.c_int32)]
 
 
 _PD = C.POINTER(C.c_double)
@@ -90,7 +94,9 @@ class Stats(C.Structure):
                 ("k2_ms_sum", C.c_double), ("k2_bytes_sum", C.c_int64), ("k2_samples", C.c_int64),
                 ("k3_ms_sum", C.c_double), ("k3_bytes_sum", C.c_int64), ("k3_samples", C.c_int64),
                 ("h2d_overlap_frac", C.c_double), ("d2h_overlap_frac", C.c_double), ("last_step_ms", C.c_double),
-                ("spill_bytes", C.c_int64), ("spilled_layers", C.c_int32), ("landing_buffers", C.c_int32)]
+                ("spill_bytes", C.c_int64), ("spilled_layers", C.c_int32), ("landing_buffers", C.c_int32),
+                ("numa_nodes", C.c_int32), ("numa_policy", C.c_int32), ("numa_gpu_node", C.c_int32),
+                ("numa_pinned_workers", C.c_int32), ("numa_bound_bytes", C.c_int64)]
 
 
 class TraceEvent(C.Structure):
@@ -138,6 +144,9 @@ def lib() -> C.CDLL:
             "sh_forward_only_end": [vp], "sh_set_window_ring": [vp, i32, i32],
             "sh_executor_grads": [vp, i32, i32, vp],
             "sh_op_exec_reduce_gpu": [vp, vp, i32, i64, f32, vp],
+            "sh_numa_topology": [vp, vp, i32], "sh_numa_plan": [i32] * 5,
+            "sh_numa_worker_node": [i32] * 4, "sh_numa_node_of_pci": [C.c_char_p],
+            "sh_numa_bind_check": [i32, i64],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -212,6 +221,29 @@ def op_sumsq_gpu(g, n, out_dev, stream=None):
     check(lib().sh_op_sumsq_gpu(_ptr(g), n, _ptr(out_dev), _stream_handle(stream)))
 
 
+def numa_topology() -> list[tuple[int, int]]:
+    """[(node id, cpu count)] of the online NUMA nodes (sysfs; SH_SYSFS_ROOT prefixes it)."""
+    ids, cpus = (C.c_int32 * 1024)(), (C.c_int32 * 1024)()
+    n = lib().sh_numa_topology(C.addressof(ids), C.addressof(cpus), 1024)
+    return [(ids[k], cpus[k]) for k in range(n)]
+
+
+def numa_plan(policy: int, unit: int, n_nodes: int, gpu_node: int = 0, shared: bool = False) -> int:
+    return lib().sh_numa_plan(policy, unit, n_nodes, gpu_node, int(shared))
+
+
+def numa_worker_node(policy: int, tid: int, n_threads: int, gpu_node: int = 0) -> int:
+    return lib().sh_numa_worker_node(policy, tid, n_threads, gpu_node)
+
+
+def numa_node_of_pci(bus_id: str) -> int:
+    return lib().sh_numa_node_of_pci(bus_id.encode())
+
+
+def numa_bind_check(node_id: int, nbytes: int) -> int:
+    return lib().sh_numa_bind_check(node_id, nbytes)
+
+
 def kernel_launches() -> int:
     return int(lib().sh_kernel_launches())
 
@@ -278,7 +310,7 @@ class Engine:
                  stream=None, cpu_threads=0, grad_ring_depth=0, warmup_steps=5, device_budget_bytes=0,
                  world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None,
                  ring_slots=0, cpu_util_max=0.0, n_executors=1, spill_dir: str | None = None,
-                 host_pin_budget_bytes=0, warmup_window=0):
+                 host_pin_budget_bytes=0, warmup_window=0, numa_policy=0):
         L = lib()
         self.n_layers = len(layer_numels)
         self._keep = []
@@ -318,6 +350,7 @@ class Engine:
         cfg.spill_dir = self._spill
         cfg.host_pin_budget_bytes = int(host_pin_budget_bytes)
         cfg.warmup_window = int(warmup_window)
+        cfg.numa_policy = int(numa_policy)
         self.n_executors = max(1, n_executors)
         self._shm = shm_name.encode() if shm_name else None
         cfg.shm_name = self._shm

@@ -112,3 +112,48 @@ def test_late_shadow_bitwise():
         assert losses == ref_losses
     finally:
         tr.close()
+
+
+@pytest.mark.parametrize("policy", ["SH_NUMA_SPLIT", "SH_NUMA_LOCAL", "SH_NUMA_INTERLEAVE"])
+def test_numa_placement_bitwise(tmp_path, monkeypatch, policy):
+    """NUMA placement on a fake two-node topology that splits the box's real
+    CPUs: workers are pinned to their half, SPLIT workers prefer their node's layers, blocks are
+    mbind'ed (node 0 exists, the fake node 1 does not, so only its binds fail).  Placement and
+    job routing must not change a bit of the training."""
+    import os
+    n = os.cpu_count()
+    if n < 2:
+        pytest.skip("needs 2 CPUs")
+    root = tmp_path / "sysfs"
+    base = root / "sys/devices/system/node"
+    base.mkdir(parents=True)
+    (base / "online").write_text("0-1\n")
+    for k, cl in enumerate((f"0-{n // 2 - 1}", f"{n // 2}-{n - 1}")):
+        (base / f"node{k}").mkdir()
+        (base / f"node{k}" / "cpulist").write_text(cl + "\n")
+    L = TINY["L"]
+    ref_tr, ref_losses, _ = engine_run(TINY, 3, L, sh.SH_FP32)
+    ref = engine_state(ref_tr)
+    ref_tr.close()
+    monkeypatch.setenv("SH_SYSFS_ROOT", str(root))
+    assert len(sh.numa_topology()) == 2  # refresh the library's cached topology
+    try:
+        pol = getattr(sh, policy)
+        tr, losses, _ = engine_run(TINY, 3, 1, sh.SH_FP32, cpu_threads=4, numa_policy=pol)
+        try:
+            st = tr.engine.stats()
+            assert st["numa_nodes"] == 2 and st["numa_policy"] == pol
+            if pol == sh.SH_NUMA_INTERLEAVE:
+                assert st["numa_pinned_workers"] == 0
+            else:
+                assert st["numa_pinned_workers"] == 4
+            if pol == sh.SH_NUMA_SPLIT:
+                assert st["numa_bound_bytes"] > 0  # the node-0 layers
+            ok, what = states_bitwise_equal(engine_state(tr), ref)
+            assert ok, what
+            assert losses == ref_losses
+        finally:
+            tr.close()
+    finally:
+        monkeypatch.delenv("SH_SYSFS_ROOT")
+        sh.numa_topology()
