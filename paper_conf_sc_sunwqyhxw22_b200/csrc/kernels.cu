@@ -26,6 +26,7 @@
 #include <atomic>
 #include <cstdint>
 #include <cstdlib>
+#include <cstring>
 
 #include "sh_internal.hpp"
 
@@ -70,8 +71,8 @@ __device__ __forceinline__ void adam_elem(float& p, float& m, float& v, float g,
 // elements base + u*1024 + 4t .. +3 for u in [0, U): every float4 load/store of a warp touches 512
 // contiguous bytes; 4U independent 16-B loads in flight per thread (U = 4 by default, tuned on
 // B200 with tools/bench_kernels.py).
-template <bool kBf16Out, int U>
-__global__ void __launch_bounds__(256) k2_adamw_kernel(const __grid_constant__ K2Args a) {
+template <bool kBf16Out, int U, int kMinBlocks = 0>
+__global__ void __launch_bounds__(256, kMinBlocks) k2_adamw_kernel(const __grid_constant__ K2Args a) {
   const AdamS s{a.sc.beta1, a.sc.beta2, a.sc.omb1, a.sc.omb2, a.sc.eps, -a.sc.step_size,
                 a.sc.sqrt_bc2, a.sc.decay};
   const bool use_coef = a.coef != nullptr;
@@ -114,6 +115,139 @@ __global__ void __launch_bounds__(256) k2_adamw_kernel(const __grid_constant__ K
         } else {
           st_f4(static_cast<float*>(E.out) + i, p[u]);
         }
+      }
+    }
+  }
+}
+
+// K2, bulk-copy pipeline variant (SH_K2_IMPL=bulk).  The register-staged kernel above loads a work
+// item, then computes and stores it: while a block is in its compute/store phase its loads are
+// idle, and at 83 registers only 2 blocks fit per SM.  Here one 512-thread block per SM keeps the
+// loads continuously in flight with the Blackwell bulk-copy engine: thread 0 streams the p, m, v
+// and g slices of the next kBulkStages work items (4096 elements, 4 x 16 KB) into a ring of shared
+// memory stages with cp.async.bulk, each stage completing a transaction-count mbarrier; all
+// threads wait on the stage's barrier, run the same adam_elem on their 8 elements (conflict-free
+// 16-B shared loads) and store the results to global memory straight from registers; after a
+// block barrier thread 0 refills the stage with the item kBulkStages ahead.  Same per-element
+// arithmetic as the other kernel => bitwise identical.
+constexpr int kBulkThreads = 512;
+constexpr int kBulkStages = 3;
+template <int kItem>
+constexpr size_t bulk_smem() { return (size_t)kBulkStages * 4 * kItem * sizeof(float) + 64; }
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "LAB_WAIT:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@P1 bra DONE;\n"
+      "bra LAB_WAIT;\n"
+      "DONE:\n"
+      "}\n" ::"r"(smem_addr(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_addr(dst)),
+               "l"(src), "r"(bytes), "r"(smem_addr(bar))
+               : "memory");
+}
+__device__ __forceinline__ float4 lds_f4(const float* p) { return *reinterpret_cast<const float4*>(p); }
+
+template <bool kBf16Out, int kBulkItem, int kMinBlocks>
+__global__ void __launch_bounds__(kBulkThreads, kMinBlocks) k2_adamw_bulk_kernel(const __grid_constant__ K2Args a) {
+  constexpr int kU = kBulkItem / (4 * kBulkThreads);  // float4 per thread per array
+  extern __shared__ __align__(128) unsigned char k2_smem[];
+  float* stage_buf = reinterpret_cast<float*>(k2_smem);  // [kBulkStages][4 arrays][kBulkItem]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(k2_smem + (size_t)kBulkStages * 4 * kBulkItem * sizeof(float));
+  const AdamS s{a.sc.beta1, a.sc.beta2, a.sc.omb1, a.sc.omb2, a.sc.eps, -a.sc.step_size,
+                a.sc.sqrt_bc2, a.sc.decay};
+  const bool use_coef = a.coef != nullptr;
+  const float coef = use_coef ? *a.coef : 1.0f;
+  const int64_t n_items = a.item_start[a.n_entries];
+  if (threadIdx.x == 0) {
+    for (int k = 0; k < kBulkStages; ++k) mbar_init(&bar[k], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  int e_prod = 0;  // producer's entry cursor (runs kBulkStages items ahead of the consumers)
+  auto issue = [&](int64_t item, int stage) {
+    while (item >= a.item_start[e_prod + 1]) ++e_prod;
+    const K2Entry& E = a.e[e_prod];
+    const int64_t base = (item - a.item_start[e_prod]) * kBulkItem;
+    const int64_t cnt = E.n - base < kBulkItem ? E.n - base : kBulkItem;  // multiple of 8 elements
+    const uint32_t bytes = (uint32_t)(cnt * sizeof(float));
+    float* d = stage_buf + (size_t)stage * 4 * kBulkItem;
+    mbar_expect_tx(&bar[stage], 4 * bytes);
+    bulk_g2s(d, E.p + base, bytes, &bar[stage]);
+    bulk_g2s(d + kBulkItem, E.m + base, bytes, &bar[stage]);
+    bulk_g2s(d + 2 * kBulkItem, E.v + base, bytes, &bar[stage]);
+    bulk_g2s(d + 3 * kBulkItem, E.g + base, bytes, &bar[stage]);
+  };
+  if (threadIdx.x == 0)
+    for (int k = 0; k < kBulkStages; ++k) {
+      const int64_t item = blockIdx.x + (int64_t)k * gridDim.x;
+      if (item < n_items) issue(item, k);
+    }
+  int e = 0;
+  int j = 0;
+  for (int64_t item = blockIdx.x; item < n_items; item += gridDim.x, ++j) {
+    const int stage = j % kBulkStages;
+    while (item >= a.item_start[e + 1]) ++e;
+    const K2Entry& E = a.e[e];
+    const int64_t base = (item - a.item_start[e]) * kBulkItem;
+    mbar_wait(&bar[stage], (uint32_t)((j / kBulkStages) & 1));
+    const float* sp = stage_buf + (size_t)stage * 4 * kBulkItem;
+    float4 p[kU], m[kU], v[kU], g[kU];
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const int o = u * 4 * kBulkThreads + 4 * threadIdx.x;
+      p[u] = lds_f4(sp + o);
+      m[u] = lds_f4(sp + kBulkItem + o);
+      v[u] = lds_f4(sp + 2 * kBulkItem + o);
+      g[u] = lds_f4(sp + 3 * kBulkItem + o);
+    }
+#pragma unroll
+    for (int u = 0; u < kU; ++u) {
+      const int64_t i = base + u * 4 * kBulkThreads + 4 * threadIdx.x;
+      if (i >= E.n) continue;
+      const bool wd = i < E.n_decay;  // n_decay is a multiple of 8: uniform per float4
+      adam_elem(p[u].x, m[u].x, v[u].x, g[u].x, s, wd, use_coef, coef);
+      adam_elem(p[u].y, m[u].y, v[u].y, g[u].y, s, wd, use_coef, coef);
+      adam_elem(p[u].z, m[u].z, v[u].z, g[u].z, s, wd, use_coef, coef);
+      adam_elem(p[u].w, m[u].w, v[u].w, g[u].w, s, wd, use_coef, coef);
+      st_f4(E.p + i, p[u]);
+      st_f4(E.m + i, m[u]);
+      st_f4(E.v + i, v[u]);
+      if (E.out != nullptr) {
+        if constexpr (kBf16Out) {
+          uint2 o;
+          o.x = rne_bf16_bits(p[u].x) | (rne_bf16_bits(p[u].y) << 16);
+          o.y = rne_bf16_bits(p[u].z) | (rne_bf16_bits(p[u].w) << 16);
+          *reinterpret_cast<uint2*>(static_cast<uint16_t*>(E.out) + i) = o;
+        } else {
+          st_f4(static_cast<float*>(E.out) + i, p[u]);
+        }
+      }
+    }
+    __syncthreads();  // every thread is done reading this stage
+    if (threadIdx.x == 0) {
+      const int64_t nx = item + (int64_t)kBulkStages * gridDim.x;
+      if (nx < n_items) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic reads before async writes
+        issue(nx, stage);
       }
     }
   }
@@ -290,6 +424,44 @@ int env_int(const char* name, int dflt) {
 cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
   static const int U = env_int("SH_K2_U", 4) == 2 ? 2 : 4;  // U=4: 0.93 vs 0.89 of HBM peak (profiles/r01_kernels_microbench.txt)
   static const int bps = env_int("SH_K2_BPS", 4);
+  // SH_K2_IMPL: "bulk4k" / "bulk2k" = bulk-copy pipeline (4096-element items, 1 block/SM, or
+  // 2048-element items, 2 blocks/SM); "ldg3" = register-staged kernel capped at 80 registers (3
+  // blocks/SM); default: register-staged, 2 blocks/SM
+  static const int impl = [] {
+    const char* e = getenv("SH_K2_IMPL");
+    if (!e) return 0;
+    if (strcmp(e, "bulk4k") == 0 || strcmp(e, "bulk") == 0) return 1;
+    if (strcmp(e, "bulk2k") == 0) return 2;
+    if (strcmp(e, "ldg3") == 0) return 3;
+    return 0;
+  }();
+  if (impl == 1 || impl == 2) {
+    const int item = impl == 1 ? 4096 : 2048;
+    a.item_start[0] = 0;
+    for (int i = 0; i < a.n_entries; ++i) a.item_start[i + 1] = a.item_start[i] + (a.e[i].n + item - 1) / item;
+    const int64_t items = a.item_start[a.n_entries];
+    if (items == 0) return cudaSuccess;
+    static bool attr_done = false;
+    if (!attr_done) {
+      cudaFuncSetAttribute(k2_adamw_bulk_kernel<true, 4096, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bulk_smem<4096>());
+      cudaFuncSetAttribute(k2_adamw_bulk_kernel<false, 4096, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bulk_smem<4096>());
+      cudaFuncSetAttribute(k2_adamw_bulk_kernel<true, 2048, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bulk_smem<2048>());
+      cudaFuncSetAttribute(k2_adamw_bulk_kernel<false, 2048, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bulk_smem<2048>());
+      attr_done = true;
+    }
+    const int64_t cap = (int64_t)sm_count() * (impl == 1 ? 1 : 2);
+    const int grid = (int)(items < cap ? items : cap);
+    if (grid_out) *grid_out = grid;
+    launch_counter()++;
+    if (impl == 1) {
+      if (a.out_bf16) k2_adamw_bulk_kernel<true, 4096, 1><<<grid, kBulkThreads, bulk_smem<4096>(), st>>>(a);
+      else k2_adamw_bulk_kernel<false, 4096, 1><<<grid, kBulkThreads, bulk_smem<4096>(), st>>>(a);
+    } else {
+      if (a.out_bf16) k2_adamw_bulk_kernel<true, 2048, 2><<<grid, kBulkThreads, bulk_smem<2048>(), st>>>(a);
+      else k2_adamw_bulk_kernel<false, 2048, 2><<<grid, kBulkThreads, bulk_smem<2048>(), st>>>(a);
+    }
+    return cudaGetLastError();
+  }
   const int64_t chunk = 1024 * U;
   a.item_start[0] = 0;
   for (int i = 0; i < a.n_entries; ++i) a.item_start[i + 1] = a.item_start[i] + (a.e[i].n + chunk - 1) / chunk;
@@ -300,7 +472,10 @@ cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
   const int grid = (int)(items < cap ? items : cap);
   if (grid_out) *grid_out = grid;
   launch_counter()++;
-  if (U == 4) {
+  if (impl == 3) {
+    if (a.out_bf16) k2_adamw_kernel<true, 4, 3><<<grid, 256, 0, st>>>(a);
+    else k2_adamw_kernel<false, 4, 3><<<grid, 256, 0, st>>>(a);
+  } else if (U == 4) {
     if (a.out_bf16) k2_adamw_kernel<true, 4><<<grid, 256, 0, st>>>(a);
     else k2_adamw_kernel<false, 4><<<grid, 256, 0, st>>>(a);
   } else {
