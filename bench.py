@@ -509,6 +509,12 @@ def main():
             "h2d_overlap_with_compute": r["st2"]["h2d_overlap_frac"],
             "d2h_overlap_with_compute": r["st2"]["d2h_overlap_frac"],
             "peak_source": "profiles/r01_probe_box.json (pinned 1 GiB copies)"},
+        # compute-stream stall of the last profiled step: step time minus the union of
+        # the layer compute intervals and K2 on the compute stream (engine CUDA events)
+        "compute_stream": {"step_ms": r["st2"]["last_step_ms"], "busy_ms": r["st2"]["compute_busy_ms"],
+                           "stall_ms": r["st2"]["last_step_ms"] - r["st2"]["compute_busy_ms"],
+                           "stall_frac": (1 - r["st2"]["compute_busy_ms"] / r["st2"]["last_step_ms"])
+                           if r["st2"]["last_step_ms"] > 0 else None},
         "cpu_adam": {"threads": st1["cpu_threads"], "elems_per_step": d["cpu_adam_elems"] / K,
                      "thread_ms_per_step": d["cpu_adam_ms"] / K,
                      "dram_gbs": (28 if fetch32 or not prec else 30) * d["cpu_adam_elems"] / (d["cpu_adam_ms"] / 1e3 / st1["cpu_threads"]) / 1e9

@@ -289,6 +289,9 @@ typedef struct {
   int32_t numa_gpu_node;        /* node index of this context's GPU */
   int32_t numa_pinned_workers;  /* CPU Adam workers pinned to a node */
   int64_t numa_bound_bytes;     /* host-store bytes placed with mbind */
+  double compute_busy_ms;       /* last harvested profiled step: union of the compute-stream intervals
+                                   (layer FP/BP compute, K2); last_step_ms - compute_busy_ms is the
+                                   compute stream's stall (waiting on fetches, restages, updates) */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */

@@ -394,7 +394,7 @@ struct sh_ctx {
   std::vector<int64_t> p_slot_i, p_gstate_i;
   std::vector<double> cpu_ms_layer;  // host timing of CPU Adam per layer (last)
   std::vector<sh_trace_event> trace;
-  double h2d_overlap = 0, d2h_overlap = 0, last_step_ms = 0;
+  double h2d_overlap = 0, d2h_overlap = 0, last_step_ms = 0, compute_busy_ms = 0;
   double t_async_ms = 0.0;
   int64_t n_async = 0;
   int profiled_steps = 0;
@@ -844,6 +844,14 @@ void build_trace(sh_ctx* c, ProfSet& P) {
   c->h2d_overlap = th > 0 ? oh / th : 0;
   c->d2h_overlap = td > 0 ? od / td : 0;
   c->last_step_ms = P.rec_k2 ? ev_at(P.t0, P.k2b) : end;
+  // compute-stream busy time: union of the layer compute intervals and the K2 launches on it
+  // (the step-end K2 and, single GPU, the per-layer K2); the rest of the step is stall
+  std::vector<std::pair<double, double>> busy = comp;
+  for (auto& e : c->trace)
+    if (e.kind == 7) busy.emplace_back(e.start_ms, e.end_ms);
+  double tb = 0;
+  const double whole = union_overlap(busy, {{0.0, std::max(end, c->last_step_ms)}}, &tb);
+  c->compute_busy_ms = whole;
 }
 
 // Read the events of a finished profiled step into the profile arrays and the stats.
@@ -2800,6 +2808,7 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->h2d_overlap_frac = c->h2d_overlap;
   o->d2h_overlap_frac = c->d2h_overlap;
   o->last_step_ms = c->last_step_ms;
+  o->compute_busy_ms = c->compute_busy_ms;
   o->spill_bytes = (int64_t)c->spill_bytes;
   o->landing_buffers = c->D;
   o->spilled_layers = c->n_spilled;

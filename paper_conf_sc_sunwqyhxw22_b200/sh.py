@@ -96,7 +96,8 @@ class Stats(C.Structure):
                 ("h2d_overlap_frac", C.c_double), ("d2h_overlap_frac", C.c_double), ("last_step_ms", C.c_double),
                 ("spill_bytes", C.c_int64), ("spilled_layers", C.c_int32), ("landing_buffers", C.c_int32),
                 ("numa_nodes", C.c_int32), ("numa_policy", C.c_int32), ("numa_gpu_node", C.c_int32),
-                ("numa_pinned_workers", C.c_int32), ("numa_bound_bytes", C.c_int64)]
+                ("numa_pinned_workers", C.c_int32), ("numa_bound_bytes", C.c_int64),
+                ("compute_busy_ms", C.c_double)]
 
 
 class TraceEvent(C.Structure):

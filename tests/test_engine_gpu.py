@@ -246,6 +246,19 @@ def test_autotune_mid_run_bitwise_and_trace():
         assert all(e["end_ms"] >= e["start_ms"] >= 0 for e in trace)
         if st["window"] < L:
             assert 0.0 <= st["h2d_overlap_frac"] <= 1.0 and 0.0 <= st["d2h_overlap_frac"] <= 1.0
+        # compute-stream busy time = union of the fp / bp / K2 intervals, within the step
+        busy = sorted((e["start_ms"], e["end_ms"]) for e in trace if e["kind"] in ("fp", "bp", "k2_adamw"))
+        union, cur = 0.0, None
+        for a0, a1 in busy:
+            if cur and a0 <= cur[1]:
+                cur[1] = max(cur[1], a1)
+            else:
+                if cur:
+                    union += cur[1] - cur[0]
+                cur = [a0, a1]
+        union += cur[1] - cur[0]
+        assert 0 < st["compute_busy_ms"] <= st["last_step_ms"] + 1e-3
+        assert abs(st["compute_busy_ms"] - union) <= 1e-3 * max(1.0, union)
     finally:
         tr.close()
 
