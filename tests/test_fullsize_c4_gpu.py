@@ -1,0 +1,116 @@
+"""Parity at the size and in the launch configuration the default `bench.py` times: configs[3] C4
+(h=4096 GPT, L = 82, 16.7 B params, fp32 states 201 GB > 180 GB of HBM, bf16 mixed, batch 16) with
+the window the autotuner picked in profiles/r01_bench_default_c4_v4.json: 53 GPU-optimised layers,
+a decoupled ring of 15 slots (R22), bf16 host shadows, one landing buffer per host layer.
+
+The fp64 oracle cannot run this model, so (as for C2 in test_fullsize_gpu.py) this checks:
+  * sampled AdamW at step 2 against the oracle's update, element by element, on the first GPU
+    layer (its gradients are in the last-used GPU grad buffer), both ends of the host range and
+    the resident set: the right gradients reach the right layer's GPU / CPU update;
+  * bitwise equality of every sampled layer's p / m / v with a DIFFERENT split of the same model
+    (44 GPU-optimised layers, ring 21, fp32 fetch + K1 cast instead of bf16 shadows): layers that
+    are host-optimised in one run and GPU-optimised in the other (44-52) cross the CPU/GPU Adam
+    boundary, so this is the bit-exact-across-windows bar at full size;
+  * step-1 loss is ln V + O(init noise).
+"""
+import hashlib
+import math
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import gpt_oracle as O
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
+C4 = dict(L=82, h=4096, nh=32, s=1024, V=50304, b=16)
+SAMPLED = (0, 53, 81, -1)                  # oracle-checked (grads readable at step 2)
+HASHED = (0, 43, 44, 52, 53, 81, -1)       # compared bitwise between the two splits
+N_SAMPLE = 4096
+
+
+def _trainer(window, ring, flags):
+    from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
+    mc = T.ModelConfig(C4["L"], C4["h"], C4["nh"], C4["s"], C4["V"])
+    return T.StrongholdTrainer(mc, batch=C4["b"], window=window, precision=sh.SH_BF16_MIXED,
+                               flags=sh.SH_FLAG_PROFILE | flags, ring_slots=ring, grad_ring_depth=0,
+                               init_threads=16)
+
+
+def _run(window, ring, flags, sample_idx=None):
+    """2 steps; returns losses, sha1 of p/m/v of the HASHED layers, and (if sample_idx) the sampled
+    p/m/v after step 1 and p/m/v/g after step 2 of the SAMPLED layers."""
+    tr = _trainer(window, ring, flags)
+    out = {"loss": [], "s1": {}, "s2": {}, "sha": {}}
+    try:
+        for t in range(2):
+            tr.set_tokens(synth.tokens(t, C4["b"], C4["s"], C4["V"]))
+            tr.step_device()
+            out["loss"].append(tr.loss())
+            if sample_idx is not None:
+                whats = (sh.SH_READ_PARAM, sh.SH_READ_M, sh.SH_READ_V) + ((sh.SH_READ_GRAD,) if t == 1 else ())
+                for x in SAMPLED:
+                    out["s1" if t == 0 else "s2"][x] = [tr.engine.read_layer(x, w)[sample_idx[x]] for w in whats]
+        for x in HASHED:
+            out["sha"][x] = [hashlib.sha1(tr.engine.read_layer(x, w).tobytes()).hexdigest()
+                             for w in (sh.SH_READ_PARAM, sh.SH_READ_M, sh.SH_READ_V)]
+        out["window"] = tr.engine.stats()["window"]
+    finally:
+        tr.close()
+    return out
+
+
+@pytest.fixture(scope="module")
+def runs():
+    rng = np.random.default_rng(0)
+    h = C4["h"]
+    idx = {}
+    for x in SAMPLED:
+        n = sum(int(np.prod(s)) for s in (synth.layer_shapes(h) if x >= 0 else
+                                          synth.resident_shapes(C4["V"], C4["s"], h)))
+        idx[x] = np.sort(rng.choice(n, N_SAMPLE, replace=False))
+    a = _run(53, 15, 0, idx)                      # the bench's autotuned configuration
+    b = _run(44, 21, sh.SH_FLAG_FETCH_FP32)       # another split, fp32 fetch + K1 cast
+    return idx, a, b
+
+
+def test_c4_sampled_adamw_vs_oracle(runs):
+    idx, a, _ = runs
+    assert a["window"] == 53
+    opt = O.AdamWConfig()
+    h = C4["h"]
+    for x in SAMPLED:
+        p1, m1, v1 = a["s1"][x]
+        p2, m2, v2, g2 = a["s2"][x]
+        numels = [int(np.prod(s)) for s in (synth.layer_shapes(h) if x >= 0 else
+                                            synth.resident_shapes(C4["V"], C4["s"], h))]
+        wd = synth.layer_weight_decay(h) if x >= 0 else synth.resident_weight_decay()
+        decay = np.concatenate([np.full(n, d) for n, d in zip(numels, wd)])[idx[x]]
+        assert np.abs(g2).max() > 0, x  # the step-2 gradients really are there
+        for d in (True, False):
+            sel = decay == d
+            if not sel.any():
+                continue
+            rp, rm, rv = O.adamw_update(p1[sel].astype(np.float64), g2[sel].astype(np.float64),
+                                        m1[sel].astype(np.float64), v1[sel].astype(np.float64), 2, opt, d)
+            scale = np.abs(p1[sel]) + np.abs(rp - p1[sel])
+            assert (np.abs(p2[sel] - rp) <= 1e-6 * scale + 1e-30).all(), (x, d)
+            mscale = opt.beta1 * np.abs(m1[sel]) + (1 - opt.beta1) * np.abs(g2[sel])
+            assert (np.abs(m2[sel] - rm) <= 1e-6 * mscale + 1e-38).all(), (x, d)
+            assert np.allclose(v2[sel], rv, rtol=1e-6, atol=1e-38), (x, d)
+
+
+def test_c4_splits_bitwise_equal(runs):
+    _, a, b = runs
+    assert b["window"] == 44
+    for x in HASHED:
+        assert a["sha"][x] == b["sha"][x], x
+    assert a["loss"] == b["loss"]
+
+
+def test_c4_loss(runs):
+    _, a, _ = runs
+    assert math.log(C4["V"]) - 0.1 < a["loss"][0] < math.log(C4["V"]) + 0.5
+    assert all(np.isfinite(a["loss"]))
