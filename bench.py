@@ -55,6 +55,7 @@ CPU_HARD_DEFAULT = {"c3", "c4", "c4max"}   # autotune with the eq. 3 CPU-through
 # growth, GPU set filling the HBM a decoupled ring leaves, late bf16 host shadows (C4: 7.30 -> 7.92
 # samples/s, profiles/r01_bench_default_c4_v3.json vs r01_bench_c4_tuned_coupled.json)
 TUNED_DEFAULT = {"c3", "c4"}
+SETTLE_STEPS = 2  # untimed steps after the autotuner's window change (before the K timed steps)
 
 
 def mem_available() -> int:
@@ -367,11 +368,15 @@ def main():
         attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
-        host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + K)])
+        # an autotuned run changes its window (and with the extensions its landing ring and host
+        # shadows) at the end of warm-up step W; S more untimed steps let the new configuration reach
+        # its steady state (GPU-set uploads, ring refill) so the timed steps measure it, not the switch
+        S = SETTLE_STEPS if window == -1 else 0
+        host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + S + K)])
         host = host.pin_memory()
         dev = host.to(f"cuda:{local}")
         step_fn = tr.forward_only if args.fp_only else tr.step_device
-        for t in range(W):
+        for t in range(W + S):
             tr.tok_dev.copy_(dev[t])
             step_fn()
         tr.engine.synchronize()
@@ -383,7 +388,7 @@ def main():
         torch.cuda.synchronize()
         with ClockSampler(local) as clk:
             ev0.record(tr.stream)
-            for t in range(W, W + K):
+            for t in range(W + S, W + S + K):
                 with torch.cuda.stream(tr.stream):
                     tr.tok_dev.copy_(dev[t], non_blocking=True)
                 step_fn()
@@ -401,7 +406,7 @@ def main():
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(tr.stream)
-            for t in range(W, W + K):
+            for t in range(W + S, W + S + K):
                 tr.step(host[t])  # public API: pinned host tokens -> H2D, step, loss -> host
             tr.engine.synchronize()
             e1.record(tr.stream)
@@ -494,7 +499,8 @@ def main():
                    "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
                    "grad_landing_buffers": r["st1"]["landing_buffers"], "host_store_bytes": r["st1"]["host_bytes"],
                    "states_bytes_fp32_p_m_v": 12 * mc.n_params(),
-                   "l2": "no flush: per-step traffic (GBs) >> 126 MB L2"},
+                   "l2": "no flush: per-step traffic (GBs) >> 126 MB L2",
+                   "settle_steps": SETTLE_STEPS if w == -1 else 0},
         "tokens_per_s": tokens_s,
         "model_tflops": tokens_s * flops_tok / 1e12,
         "final_loss": r["loss"],
