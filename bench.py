@@ -294,14 +294,19 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
-    nccl_id = None
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    def fresh_nccl_id():
+        # an ncclUniqueId bootstraps ONE communicator: every engine context (the timed run, the
+        # resident-fit run) gets its own, created on rank 0 and broadcast over torch.distributed
         idt = torch.zeros(128, dtype=torch.uint8, device="cuda")
         if rank == 0:
             idt.copy_(torch.frombuffer(bytearray(sh.nccl_unique_id()), dtype=torch.uint8))
         dist.broadcast(idt, 0)
-        nccl_id = bytes(idt.cpu().numpy().tobytes())
+        return bytes(idt.cpu().numpy().tobytes())
+
+    nccl_id = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        nccl_id = fresh_nccl_id()
 
     L, h, nh, s, V, b0, w0, desc = CONFIGS[args.config]
     b = args.batch or b0
@@ -342,14 +347,22 @@ def main():
 
     shm_name = None
     cpu_threads = args.cpu_threads
+    import hashlib
     if world > 1:
-        import hashlib
         if use_shm:
             shm_name = "sh_" + hashlib.sha1(nccl_id).hexdigest()[:16]  # one host store for the box
         cpu_threads = cpu_threads or max(1, (os.cpu_count() or 1) // local_world)
 
+    first_run = [True]
+
     def run(window, e2e: bool, mc=mc):
         L = mc.n_layers
+        nid, shm = nccl_id, shm_name
+        if world > 1 and not first_run[0]:
+            nid = fresh_nccl_id()
+            if shm_name:
+                shm = "sh_" + hashlib.sha1(nid).hexdigest()[:16]
+        first_run[0] = False
         t_init = time.perf_counter()
         flags = sh.SH_FLAG_PROFILE | (sh.SH_FLAG_FETCH_FP32 if fetch32 else 0) | \
             (sh.SH_FLAG_CPU_HARD | (0 if args.no_decouple else sh.SH_FLAG_DECOUPLE) if cpu_hard else 0) | \
@@ -359,8 +372,8 @@ def main():
             (sh.SH_FLAG_GROW_LANDING if args.grow_landing else 0) | (sh.SH_FLAG_FILL_GPU if args.fill_gpu else 0) | \
             (sh.SH_FLAG_LATE_SHADOW if args.late_shadow else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
-                               flags=flags, world_size=world, rank=rank, nccl_id=nccl_id,
-                               cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm_name,
+                               flags=flags, world_size=world, rank=rank, nccl_id=nid,
+                               cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm,
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
                                attention=args.attention, executors=args.executors, ring_slots=args.ring,
                                spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9),
