@@ -194,6 +194,15 @@ typedef struct {
                                        the host RAM the store needs from the start */
   int32_t numa_policy;              /* SH_NUMA_*: where the pinned host store lives and which cores update
                                        it.  0 = SH_NUMA_AUTO */
+  int64_t ring_bytes;               /* NEXT-4 fixed-byte window: 0 = off (w + 1 slots sized for
+                                       the largest layer).  > 0: ONE device buffer of at most ring_bytes
+                                       holding variable-capacity slots -- slot 0 fits the largest layer,
+                                       slot x >= 1 is sized for layer x (execution order) while the bytes
+                                       last -- and the prefetch runs ahead until no evictable slot fits
+                                       the next layer, so the number of buffered layers follows the
+                                       layer sizes (heterogeneous stacks).  window still sets the
+                                       GPU-optimised set.  Needs no clipping, world_size 1, window >= 0,
+                                       ring_slots 0; SH_ERR_INVALID if the largest layer does not fit */
 } sh_config;
 
 /* NUMA placement policies (sh_config.numa_policy).  Placement is an mbind(2) before the first
@@ -292,6 +301,7 @@ typedef struct {
   double compute_busy_ms;       /* last harvested profiled step: union of the compute-stream intervals
                                    (layer FP/BP compute, K2); last_step_ms - compute_busy_ms is the
                                    compute stream's stall (waiting on fetches, restages, updates) */
+  int64_t ring_bytes;           /* device bytes of the slot ring */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */

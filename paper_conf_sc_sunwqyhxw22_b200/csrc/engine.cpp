@@ -239,8 +239,16 @@ struct sh_ctx {
   int n_active = 0;  // slots in use = min(w + 1, ring cap)
   int d = 0;         // prefetch distance = n_active - 1 (the paper's window m when the ring is w+1)
   int ring_cap = 0;  // sh_config.ring_slots / sh_set_window_ring (0: w + 1)
+  // NEXT-4 fixed-byte window (sh_config.ring_bytes): variable-capacity slots packed
+  // into one buffer of a fixed byte size; empty = fixed-size slots
+  std::vector<int64_t> slot_off, slot_cap, slot_pb;  // byte offset, capacity (elements), param-half bytes
+  int64_t byte_ring_total = 0;
+  bool byte_ring() const { return !slot_off.empty(); }
+  int64_t ring_bytes_for(int n) const { return byte_ring() ? byte_ring_total : (int64_t)n * slot_bytes; }
+  int64_t slot_param_bytes_of(int s) const { return byte_ring() ? slot_pb[s] : slot_param_bytes; }
   bool k2_layer = true;  // no clipping: a GPU-optimised layer is updated right after its backward
   int ring_for(int w_) const {
+    if (byte_ring()) return (int)slot_off.size();  // the whole fixed-size buffer is always in use
     int r = w_ + 1;
     if (k2_layer && ring_cap > 0 && ring_cap < r) r = ring_cap;  // G grads are not pinned: ring may be smaller
     return r;
@@ -417,8 +425,9 @@ struct sh_ctx {
   int async_status = SH_OK;
 
   bool is_g(int x) const { return x < w; }
-  char* slot_param(int s) const { return ring + (int64_t)s * slot_bytes; }
+  char* slot_param(int s) const { return byte_ring() ? ring + slot_off[s] : ring + (int64_t)s * slot_bytes; }
   float* slot_grad(int s) const {
+    if (byte_ring()) return reinterpret_cast<float*>(ring + slot_off[s] + slot_pb[s]);
     return reinterpret_cast<float*>(ring + (int64_t)s * slot_bytes + slot_param_bytes);
   }
   int layer_at(int pos) const { return pos < L ? pos : 2 * L - 1 - pos; }
@@ -954,7 +963,7 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
     // after the victim's release)
     CKC(c, cudaStreamWaitEvent(c->stage, c->ev_param_free[s], 0));
     CKC(c, cudaStreamWaitEvent(c->stage, c->ev_upd[y], 0));
-    if (poison) CKC(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->stage));
+    if (poison) CKC(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes_of(s), c->stage));
     if (P) CKC(c, cudaEventRecord(P->st0[y], c->stage));
     if (c->bf16)
       CKC(c, kern::cast_bf16(c->g[y].master, reinterpret_cast<uint16_t*>(dst), n, c->stage));
@@ -986,8 +995,9 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   cudaEvent_t gf = c->ev_grad_free[s];
   float* stage_buf = c->slot_grad(s);
   const int64_t gf_gen = c->gradfree_gen[s];
+  const int64_t pbytes = c->slot_param_bytes_of(s);
   c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, gf, stage_buf, gf_gen, s, n, eb, slice,
-                slo, shi, cs] {
+                slo, shi, cs, pbytes] {
     maybe_delay(c->cfg.flags);
     double waited = 0;
     if (!state_wait(c, [&] { return ready_at_least(c, y, need); }, "CPU Adam of a layer to prefetch", &waited)) {
@@ -1009,7 +1019,7 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       }
       CKA(c, cudaStreamWaitEvent(c->h2d, gf, 0));
     }
-    if (poison) CKA(c, cudaMemsetAsync(dst, 0xff, c->slot_param_bytes, c->h2d));
+    if (poison) CKA(c, cudaMemsetAsync(dst, 0xff, pbytes, c->h2d));
     char* buf = cast ? reinterpret_cast<char*>(stage_buf) : dst;
     const char* hsrc = static_cast<const char*>(src);
     if (c->spilled[y]) {
@@ -1059,12 +1069,18 @@ bool ensure_at(sh_ctx* c, int p, int cur, sh_status* st) {
   int best = -1;
   int64_t best_nu = -2;
   for (int s = 0; s < c->n_active; ++s) {
+    if (c->byte_ring() && c->slot_cap[s] < c->lay[y].n_pad) continue;  // too small for this layer
     const int o = c->slot_layer[s];
     const int64_t nu = o < 0 ? kInf + 1 : next_use(c, o, cur);
     if (nu == kPinned || nu <= p) continue;
     // farthest next use (Belady); among equals (e.g. host layers done for this step) the least
     // recently used, whose gradient offload was requested first and is most likely complete
-    if (nu > best_nu || (nu == best_nu && c->slot_last_use[s] < c->slot_last_use[best]))
+    // (fixed-byte ring: among equal next uses the smallest slot that fits -- best fit keeps the
+    // large slots for the large layers)
+    const bool tie_better = c->byte_ring() && best >= 0 && c->slot_cap[s] != c->slot_cap[best]
+                                ? c->slot_cap[s] < c->slot_cap[best]
+                                : best >= 0 && c->slot_last_use[s] < c->slot_last_use[best];
+    if (nu > best_nu || (nu == best_nu && tie_better))
       best_nu = nu, best = s;
   }
   if (best < 0) return false;
@@ -1402,19 +1418,19 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
   if (c->ring) {
     cudaDeviceSynchronize();
     cudaFree(c->ring);
-    c->device_bytes -= (int64_t)c->ring_alloc * c->slot_bytes;
+    c->device_bytes -= c->ring_bytes_for(c->ring_alloc);
     c->ring = nullptr;
     c->ring_alloc = 0;
   }
   n_slots = std::max(n_slots, c->n_slots);  // events / bookkeeping never shrink
   char* r = nullptr;
-  if (cudaMalloc(&r, (int64_t)n_slots * c->slot_bytes) != cudaSuccess) {
+  if (cudaMalloc(&r, c->ring_bytes_for(n_slots)) != cudaSuccess) {
     cudaGetLastError();
     // put the previous ring back (it fitted before) so the context stays usable
-    if (c->n_slots > 0 && cudaMalloc(&r, (int64_t)c->n_slots * c->slot_bytes) == cudaSuccess) {
+    if (c->n_slots > 0 && cudaMalloc(&r, c->ring_bytes_for(c->n_slots)) == cudaSuccess) {
       c->ring = r;
       c->ring_alloc = c->n_slots;
-      c->device_bytes += (int64_t)c->n_slots * c->slot_bytes;
+      c->device_bytes += c->ring_bytes_for(c->n_slots);
     } else {
       cudaGetLastError();
       async_fail(c, SH_ERR_OOM_DEVICE, "ring re-allocation failed");
@@ -1424,8 +1440,8 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
   }
   c->ring = r;
   c->ring_alloc = n_slots;
-  c->device_bytes += (int64_t)n_slots * c->slot_bytes;
-  cudaMemset(r, 0, (int64_t)n_slots * c->slot_bytes);
+  c->device_bytes += c->ring_bytes_for(n_slots);
+  cudaMemset(r, 0, c->ring_bytes_for(n_slots));
   const int old = c->n_slots;
   c->slot_layer.resize(n_slots, -1);
   c->slot_last_use.resize(n_slots, 0);
@@ -1948,6 +1964,42 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->w = w0;
   c->k2_layer = !c->clip;
   c->ring_cap = cfg->ring_slots > 0 ? cfg->ring_slots : 0;
+  if (cfg->ring_bytes > 0) {
+    // NEXT-4 fixed-byte window ("a fixed-size GPU buffer where the number of DNN layers
+    // stored can dynamically change ... for DNN models with a heterogeneous layer structure").
+    // Slot 0 can hold the largest layer (progress is guaranteed at every position); slot x >= 1 is
+    // sized for layer x, in execution order, while the buffer has room -- a window of consecutive
+    // layers therefore fits in the slots of any stretch with the same size mix, and the prefetch
+    // stops at the first upcoming layer no evictable slot can hold (pre_common), so the number of
+    // layers in the buffer follows their sizes.  G layers 0..w-1 are staged into slots 0..w-1,
+    // which fit by construction.
+    if (c->clip || c->dp || c->autotune_pending || cfg->ring_slots > 0) {
+      set_error("sh_init: ring_bytes needs no clipping, a single rank, a fixed window and ring_slots 0");
+      return SH_ERR_INVALID;
+    }
+    auto slot_sz = [&](int64_t cap, int64_t* pb) {
+      *pb = align_up((int64_t)c->cb * cap, 256);
+      return *pb + align_up(4 * cap, 256);
+    };
+    int64_t pb = 0, total = slot_sz(c->max_pad, &pb);
+    if (total > cfg->ring_bytes) {
+      set_error("sh_init: ring_bytes %lld cannot hold the largest layer (%lld B)", (long long)cfg->ring_bytes,
+                (long long)total);
+      return SH_ERR_INVALID;
+    }
+    c->slot_off.push_back(0);
+    c->slot_cap.push_back(c->max_pad);
+    c->slot_pb.push_back(pb);
+    for (int x = 1; x < c->L; ++x) {
+      const int64_t b = slot_sz(c->lay[x].n_pad, &pb);
+      if (total + b > cfg->ring_bytes) break;
+      c->slot_off.push_back(total);
+      c->slot_cap.push_back(c->lay[x].n_pad);
+      c->slot_pb.push_back(pb);
+      total += b;
+    }
+    c->byte_ring_total = total;
+  }
   c->n_active = c->ring_for(w0);
   c->d = c->n_active - 1;
   c->layer_gbuf.assign(c->L, -1);
@@ -2551,7 +2603,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   size_t fr = 0, tot = 0;
   cudaMemGetInfo(&fr, &tot);
   // S_avail = what the engine holds now (ring + G states) + what is still free - margin
-  int64_t held = (int64_t)c->ring_alloc * c->slot_bytes;
+  int64_t held = c->ring_bytes_for(c->ring_alloc);
   for (int x = 0; x < c->L; ++x)
     if (c->g[x].master) held += 12 * c->lay[x].n_pad;
   o->s_avail = c->cfg.device_budget_bytes > 0 ? c->cfg.device_budget_bytes
@@ -2603,6 +2655,10 @@ sh_status sh_set_window_ring(sh_ctx* c, int32_t w, int32_t ring) {
     set_error("sh_set_window_ring: clip mode pins the GPU-optimised layers' grads: ring must be >= window + 1");
     return SH_ERR_INVALID;
   }
+  if (c->byte_ring() && ring > 0) {
+    set_error("sh_set_window_ring: the ring is a fixed-byte buffer (ring_bytes); ring_slots must be 0");
+    return SH_ERR_INVALID;
+  }
   if (c->phase != sh_ctx::IDLE) {
     set_error("sh_set_window_ring: only between steps");
     return SH_ERR_STATE;
@@ -2621,6 +2677,10 @@ sh_status sh_set_window_ring(sh_ctx* c, int32_t w, int32_t ring) {
 sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   clear_error();
   if (!c) return SH_ERR_INVALID;
+  if (c->byte_ring()) {
+    set_error("sh_autotune_window: a fixed-byte ring (ring_bytes) sets the window by bytes, not by the P1/P2 search");
+    return SH_ERR_UNSUPPORTED;
+  }
   sh_profile p{};
   if (ov) {
     p = *ov;
@@ -2809,6 +2869,7 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->d2h_overlap_frac = c->d2h_overlap;
   o->last_step_ms = c->last_step_ms;
   o->compute_busy_ms = c->compute_busy_ms;
+  o->ring_bytes = c->ring_bytes_for(c->ring_alloc);
   o->spill_bytes = (int64_t)c->spill_bytes;
   o->landing_buffers = c->D;
   o->spilled_layers = c->n_spilled;

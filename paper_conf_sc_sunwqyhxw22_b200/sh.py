@@ -59,7 +59,7 @@ class Config(C.Structure):
                 ("world_size", C.c_int32), ("rank", C.c_int32),
                 ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p),
                 ("n_executors", C.c_int32), ("spill_dir", C.c_char_p), ("host_pin_budget_bytes", C.c_int64),
-                ("warmup_window", C.c_int32), ("numa_policy", C.c_int32)]
+                ("warmup_window", C.c_int32), ("numa_policy", C.c_int32), ("ring_bytes", C.c_int64)]
 
 
 _PD = C.POINTER(C.c_double)
@@ -97,7 +97,7 @@ class Stats(C.Structure):
                 ("spill_bytes", C.c_int64), ("spilled_layers", C.c_int32), ("landing_buffers", C.c_int32),
                 ("numa_nodes", C.c_int32), ("numa_policy", C.c_int32), ("numa_gpu_node", C.c_int32),
                 ("numa_pinned_workers", C.c_int32), ("numa_bound_bytes", C.c_int64),
-                ("compute_busy_ms", C.c_double)]
+                ("compute_busy_ms", C.c_double), ("ring_bytes", C.c_int64)]
 
 
 class TraceEvent(C.Structure):
@@ -311,7 +311,7 @@ class Engine:
                  stream=None, cpu_threads=0, grad_ring_depth=0, warmup_steps=5, device_budget_bytes=0,
                  world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None,
                  ring_slots=0, cpu_util_max=0.0, n_executors=1, spill_dir: str | None = None,
-                 host_pin_budget_bytes=0, warmup_window=0, numa_policy=0):
+                 host_pin_budget_bytes=0, warmup_window=0, numa_policy=0, ring_bytes=0):
         L = lib()
         self.n_layers = len(layer_numels)
         self._keep = []
@@ -352,6 +352,7 @@ class Engine:
         cfg.host_pin_budget_bytes = int(host_pin_budget_bytes)
         cfg.warmup_window = int(warmup_window)
         cfg.numa_policy = int(numa_policy)
+        cfg.ring_bytes = int(ring_bytes)
         self.n_executors = max(1, n_executors)
         self._shm = shm_name.encode() if shm_name else None
         cfg.shm_name = self._shm

@@ -51,11 +51,11 @@ def _init():
             [rng.standard_normal(n).astype(np.float32) * np.float32(0.02) for n in RES])
 
 
-def _engine_run(window, precision, ring_slots=0):
+def _engine_run(window, precision, ring_slots=0, ring_bytes=0, stats=None, flags=0):
     bf16 = precision == sh.SH_BF16_MIXED
     stream = torch.cuda.Stream()
     eng = sh.Engine(LAYERS, WD, RES, RES_WD, window=window, precision=precision, lr=LR, stream=stream,
-                    ring_slots=ring_slots, cpu_threads=4)
+                    ring_slots=ring_slots, cpu_threads=4, ring_bytes=ring_bytes, flags=flags)
     try:
         lay, res = _init()
         for i, ts in enumerate(lay):
@@ -81,6 +81,8 @@ def _engine_run(window, precision, ring_slots=0):
                     _view(rg[k], n, False).add_(c * float(a) + float(b))
             eng.step()
         eng.synchronize()
+        if stats is not None:
+            stats.update(eng.stats())
         out = [eng.read_layer(i, w) for i in range(L) for w in (sh.SH_READ_PARAM, sh.SH_READ_M, sh.SH_READ_V)]
         out += [eng.read_layer(-1, w) for w in (sh.SH_READ_PARAM, sh.SH_READ_M, sh.SH_READ_V)]
         return out
@@ -124,3 +126,46 @@ def test_heterogeneous_units_vs_oracle_and_bitwise_windows(precision):
         out = _engine_run(w, prec, ring)
         for k, (x, y) in enumerate(zip(out, ref)):
             assert x.tobytes() == y.tobytes(), (w, ring, k // 3, k % 3)
+
+
+def _pad(n):
+    return (n + 127) // 128 * 128
+
+
+@pytest.mark.parametrize("precision", ["SH_FP32", "SH_BF16_MIXED"])
+def test_fixed_byte_window_heterogeneous(precision):
+    """NEXT-4 fixed-byte window: one buffer of ring_bytes holds a variable number of
+    layers.  2.5 largest-layer slots of bytes hold 5 slots here (the largest, then layers 1-4 at
+    their own sizes), where fixed-size slots would hold 2; training is bitwise the resident run's
+    for any GPU-optimised set, with slot poisoning on (a slot reused by a smaller layer must never
+    expose stale bytes)."""
+    prec = getattr(sh, precision)
+    L = len(LAYERS)
+    cb = 2 if prec == sh.SH_BF16_MIXED else 4
+    npad = [sum(_pad(n) for n in lay) for lay in LAYERS]
+    slot = lambda n: (cb * n + 255) // 256 * 256 + (4 * n + 255) // 256 * 256  # noqa: E731
+    budget = int(2.5 * slot(max(npad)))
+    caps, total = [max(npad)], slot(max(npad))
+    for x in range(1, L):
+        if total + slot(npad[x]) > budget:
+            break
+        caps.append(npad[x])
+        total += slot(npad[x])
+    assert len(caps) >= 4  # many more layers than the 2 fixed-size slots the same bytes would hold
+    ref = _engine_run(L, prec)
+    for w in (0, 1, 3, 6):
+        st = {}
+        out = _engine_run(w, prec, ring_bytes=budget, stats=st, flags=sh.SH_FLAG_POISON)
+        assert st["n_slots"] == len(caps) and st["ring_bytes"] == total <= budget, (st["n_slots"], st["ring_bytes"])
+        for k, (x, y) in enumerate(zip(out, ref)):
+            assert x.tobytes() == y.tobytes(), (w, k // 3, k % 3)
+
+
+def test_fixed_byte_window_rejects_too_small_and_autotune():
+    stream = torch.cuda.Stream()
+    with pytest.raises(sh.ShError) as e:
+        sh.Engine(LAYERS, WD, RES, RES_WD, window=0, precision=sh.SH_FP32, stream=stream, ring_bytes=4096)
+    assert e.value.status == sh.SH_ERR_INVALID and "largest layer" in str(e.value)
+    with pytest.raises(sh.ShError) as e:
+        sh.Engine(LAYERS, WD, RES, RES_WD, window=-1, precision=sh.SH_FP32, stream=stream, ring_bytes=1 << 30)
+    assert e.value.status == sh.SH_ERR_INVALID
