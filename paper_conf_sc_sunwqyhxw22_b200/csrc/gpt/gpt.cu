@@ -14,6 +14,7 @@
 #include <cub/device/device_radix_sort.cuh>
 
 #include <atomic>
+#include <type_traits>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -122,6 +123,8 @@ __global__ void ln_fwd(const float* x, const T* g, const T* b, T* out, float* me
   if (row >= N) return;
   const float* xr = x + (int64_t)row * h;
   float s = 0.f;
+  // unrolled for memory-level parallelism; each lane still accumulates in index order
+#pragma unroll 4
   for (int c = 8 * lane; c < h; c += 256) {
     float v[8];
     ld8(xr + c, v);
@@ -130,6 +133,8 @@ __global__ void ln_fwd(const float* x, const T* g, const T* b, T* out, float* me
   }
   const float mu = warp_sum(s) / h;
   float var = 0.f;
+  // unrolled for memory-level parallelism; each lane still accumulates in index order
+#pragma unroll 4
   for (int c = 8 * lane; c < h; c += 256) {
     float v[8];
     ld8(xr + c, v);
@@ -138,6 +143,8 @@ __global__ void ln_fwd(const float* x, const T* g, const T* b, T* out, float* me
   }
   const float rs = 1.0f / sqrtf(warp_sum(var) / h + kLnEps);
   T* o = out + (int64_t)row * h;
+  // unrolled for memory-level parallelism; each lane still accumulates in index order
+#pragma unroll 4
   for (int c = 8 * lane; c < h; c += 256) {
     float v[8], gg[8], bb[8];
     ld8(xr + c, v);
@@ -164,6 +171,8 @@ __global__ void ln_bwd(const float* dy, const float* x, const float* mean, const
   const float* xr = x + (int64_t)row * h;
   const float mu = mean[row], rs = rstd[row];
   float a = 0.f, bb = 0.f;
+  // unrolled for memory-level parallelism; each lane still accumulates in index order
+#pragma unroll 4
   for (int c = 8 * lane; c < h; c += 256) {
     float d[8], xv[8], gg[8];
     ld8(dr + c, d);
@@ -180,6 +189,8 @@ __global__ void ln_bwd(const float* dy, const float* x, const float* mean, const
   bb = warp_sum(bb) / h;
   float* o = dres + (int64_t)row * h;
   float* t = tmp + (int64_t)row * h;
+  // unrolled for memory-level parallelism; each lane still accumulates in index order
+#pragma unroll 4
   for (int c = 8 * lane; c < h; c += 256) {
     float d[8], xv[8], gg[8], ov[8], tv[8];
     ld8(dr + c, d);
@@ -220,13 +231,28 @@ __global__ void resid_bias(const float* x, const T* bias, float* out, int C, int
   }
 }
 
+// tanh: the accurate tanhf in fp32 mode; MUFU.TANH (tanh.approx.f32, |rel err| ~ 2^-11) for bf16
+// activations, whose own rounding is 2^-9 -- the accurate tanhf made the GELU kernels
+// issue-bound (4 TB/s at h 4096)
+template <class T>
+__device__ __forceinline__ float tanh_t(float x) {
+  if constexpr (std::is_same<T, bf16>::value) {
+    float y;
+    asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+  } else {
+    return tanhf(x);
+  }
+}
+template <class T>
 __device__ __forceinline__ float gelu_f(float u) {
   const float k = 0.7978845608028654f;  // sqrt(2/pi)
-  return 0.5f * u * (1.0f + tanhf(k * (u + 0.044715f * u * u * u)));
+  return 0.5f * u * (1.0f + tanh_t<T>(k * (u + 0.044715f * u * u * u)));
 }
+template <class T>
 __device__ __forceinline__ float gelu_grad(float u) {
   const float k = 0.7978845608028654f;
-  const float t = tanhf(k * (u + 0.044715f * u * u * u));
+  const float t = tanh_t<T>(k * (u + 0.044715f * u * u * u));
   return 0.5f * (1.0f + t) + 0.5f * u * (1.0f - t * t) * k * (1.0f + 3.0f * 0.044715f * u * u);
 }
 
@@ -236,7 +262,7 @@ __global__ void gelu_fwd(const T* pre, T* act, int64_t n8) {
     float v[8];
     ld8(pre + 8 * j, v);
 #pragma unroll
-    for (int i = 0; i < 8; ++i) v[i] = gelu_f(v[i]);
+    for (int i = 0; i < 8; ++i) v[i] = gelu_f<T>(v[i]);
     st8(act + 8 * j, v);
   }
 }
@@ -247,7 +273,7 @@ __global__ void gelu_bwd(T* d, const T* pre, int64_t n8) {
     ld8(d + 8 * j, v);
     ld8(pre + 8 * j, u);
 #pragma unroll
-    for (int i = 0; i < 8; ++i) v[i] *= gelu_grad(u[i]);
+    for (int i = 0; i < 8; ++i) v[i] *= gelu_grad<T>(u[i]);
     st8(d + 8 * j, v);
   }
 }
