@@ -7,17 +7,20 @@
 // broadcast prefill + beta = 1 (one rounding of acc + bias).  The remaining SIMT kernels are
 // HBM-bound and move 16-byte vectors (8 bf16 / 2 x 4 fp32) with fixed reduction orders.
 // The math is DESIGN.md reading R1 / oracle/gpt_oracle.py (shared by definition, not code).
+#include <cublasLt.h>
 #include <cublas_v2.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
 #include <cub/device/device_radix_sort.cuh>
 
+#include <algorithm>
 #include <atomic>
 #include <type_traits>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <string>
 #include <vector>
 
@@ -498,6 +501,15 @@ struct gpt_ctx {
   int *keys, *vals, *keys2, *vals2;
   void* cub_tmp = nullptr;
   size_t cub_bytes = 0;
+  // bf16 path: cuBLASLt GEMMs with fused epilogues (bias; bias + GELU with the pre-activation kept
+  // for the backward; GELU gradient) replace the bias-fill / GELU SIMT passes
+  cublasLtHandle_t lt = nullptr;
+  int use_lt = 0;  // bit 1: qkv bias epilogue, 2: fc bias + GELU, 4: dGELU (SH_GPT_LT, default all)
+  struct LtAlgo {
+    int64_t key[7];
+    cublasLtMatmulAlgo_t algo;
+  };
+  std::vector<LtAlgo> lt_algos;
 };
 
 namespace {
@@ -543,6 +555,72 @@ cublasStatus_t rm_gemm(gpt_ctx* c, bool tA, bool tB, int M, int N, int K, float 
                        cudaDataType_t ta, const void* B, cudaDataType_t tb, float beta, void* C, cudaDataType_t tc) {
   return gemm(c, tA, tB, M, N, K, alpha, A, ta, tA ? M : K, B, tb, tB ? K : N, beta, C, tc, N);
 }
+// Row-major bf16 D[M x N] = op(A)[M x K] op(B)[K x N] through cuBLASLt with an epilogue:
+//   CUBLASLT_EPILOGUE_BIAS           D = AB + bias[N]
+//   CUBLASLT_EPILOGUE_GELU_AUX_BIAS  aux = AB + bias[N] (pre-activation, kept for the backward),
+//                                    D = GELU(aux)
+//   CUBLASLT_EPILOGUE_DGELU          D = AB * GELU'(aux)
+// Same column-major mapping as gemm(): D^T = op(B)^T op(A)^T.  fp32 accumulate; the algorithm is
+// chosen once per shape by the heuristic and cached (same shape -> same algorithm -> same bits).
+cublasStatus_t lt_gemm(gpt_ctx* c, bool tA, bool tB, int M, int N, int K, const void* A, const void* B, void* D,
+                       cublasLtEpilogue_t epi, const void* bias, void* aux) {
+  const cublasOperation_t ta = tB ? CUBLAS_OP_T : CUBLAS_OP_N, tb = tA ? CUBLAS_OP_T : CUBLAS_OP_N;
+  cublasLtMatmulDesc_t op = nullptr;
+  cublasLtMatrixLayout_t la = nullptr, lb = nullptr, ld = nullptr;
+  cublasStatus_t st = cublasLtMatmulDescCreate(&op, CUBLAS_COMPUTE_32F, CUDA_R_32F);
+  auto set = [&](cublasLtMatmulDescAttributes_t a, const void* v, size_t n) {
+    if (st == CUBLAS_STATUS_SUCCESS) st = cublasLtMatmulDescSetAttribute(op, a, v, n);
+  };
+  set(CUBLASLT_MATMUL_DESC_TRANSA, &ta, sizeof(ta));
+  set(CUBLASLT_MATMUL_DESC_TRANSB, &tb, sizeof(tb));
+  set(CUBLASLT_MATMUL_DESC_EPILOGUE, &epi, sizeof(epi));
+  if (bias) set(CUBLASLT_MATMUL_DESC_BIAS_POINTER, &bias, sizeof(bias));
+  if (aux) {
+    const int64_t ald = N;
+    const int32_t adt = CUDA_R_16BF;
+    set(CUBLASLT_MATMUL_DESC_EPILOGUE_AUX_POINTER, &aux, sizeof(aux));
+    set(CUBLASLT_MATMUL_DESC_EPILOGUE_AUX_LD, &ald, sizeof(ald));
+    set(CUBLASLT_MATMUL_DESC_EPILOGUE_AUX_DATA_TYPE, &adt, sizeof(adt));
+  }
+  if (st == CUBLAS_STATUS_SUCCESS)
+    st = cublasLtMatrixLayoutCreate(&la, CUDA_R_16BF, ta == CUBLAS_OP_T ? K : N, ta == CUBLAS_OP_T ? N : K, tB ? K : N);
+  if (st == CUBLAS_STATUS_SUCCESS)
+    st = cublasLtMatrixLayoutCreate(&lb, CUDA_R_16BF, tb == CUBLAS_OP_T ? M : K, tb == CUBLAS_OP_T ? K : M, tA ? M : K);
+  if (st == CUBLAS_STATUS_SUCCESS) st = cublasLtMatrixLayoutCreate(&ld, CUDA_R_16BF, N, M, N);
+  const int64_t key[7] = {M, N, K, tA, tB, (int64_t)epi, (int64_t)(bias != nullptr)};
+  const cublasLtMatmulAlgo_t* algo = nullptr;
+  for (auto& a : c->lt_algos)
+    if (std::equal(key, key + 7, a.key)) algo = &a.algo;
+  if (st == CUBLAS_STATUS_SUCCESS && !algo) {
+    cublasLtMatmulPreference_t pref = nullptr;
+    st = cublasLtMatmulPreferenceCreate(&pref);
+    const uint64_t wsb = c->ws_bytes;
+    if (st == CUBLAS_STATUS_SUCCESS)
+      st = cublasLtMatmulPreferenceSetAttribute(pref, CUBLASLT_MATMUL_PREF_MAX_WORKSPACE_BYTES, &wsb, sizeof(wsb));
+    cublasLtMatmulHeuristicResult_t res{};
+    int n_res = 0;
+    if (st == CUBLAS_STATUS_SUCCESS)
+      st = cublasLtMatmulAlgoGetHeuristic(c->lt, op, la, lb, ld, ld, pref, 1, &res, &n_res);
+    if (pref) cublasLtMatmulPreferenceDestroy(pref);
+    if (st == CUBLAS_STATUS_SUCCESS && n_res < 1) st = CUBLAS_STATUS_NOT_SUPPORTED;
+    if (st == CUBLAS_STATUS_SUCCESS) {
+      gpt_ctx::LtAlgo e;
+      std::copy(key, key + 7, e.key);
+      e.algo = res.algo;
+      c->lt_algos.push_back(e);
+      algo = &c->lt_algos.back().algo;
+    }
+  }
+  const float one = 1.f, zero = 0.f;
+  if (st == CUBLAS_STATUS_SUCCESS)
+    st = cublasLtMatmul(c->lt, op, &one, B, la, A, lb, &zero, D, ld, D, ld, algo, c->ws, c->ws_bytes, c->st);
+  if (ld) cublasLtMatrixLayoutDestroy(ld);
+  if (lb) cublasLtMatrixLayoutDestroy(lb);
+  if (la) cublasLtMatrixLayoutDestroy(la);
+  if (op) cublasLtMatmulDescDestroy(op);
+  return st;
+}
+
 // batched over pointer arrays (attention): operand pointer arrays Ap, Bp, Cp on the device
 cublasStatus_t gemm_ptr(gpt_ctx* c, bool tA, bool tB, int M, int N, int K, float alpha, void* const* Ap,
                         cudaDataType_t ta, int lda, void* const* Bp, cudaDataType_t tb, int ldb, float beta,
@@ -598,8 +676,12 @@ int fwd_qkv(gpt_ctx* c, int l, void* const* P) {
   const int64_t Nh = (int64_t)N * h;
   (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
                                                                c->ln1_m, c->ln1_r, N, h);
-  (g_launches++, 0), bias_fill<T><<<grid_for(3 * Nh / 8), 256, 0, c->st>>>((T*)c->qkv, (const T*)P[3], 3 * h, 3 * Nh / 8);
-  CB(rm_gemm(c, false, true, N, 3 * h, h, 1.f, c->ln1, dt, P[2], dt, 1.f, c->qkv, dt));
+  if (c->use_lt & 1) {
+    CB(lt_gemm(c, false, true, N, 3 * h, h, c->ln1, P[2], c->qkv, CUBLASLT_EPILOGUE_BIAS, P[3], nullptr));
+  } else {
+    (g_launches++, 0), bias_fill<T><<<grid_for(3 * Nh / 8), 256, 0, c->st>>>((T*)c->qkv, (const T*)P[3], 3 * h, 3 * Nh / 8);
+    CB(rm_gemm(c, false, true, N, 3 * h, h, 1.f, c->ln1, dt, P[2], dt, 1.f, c->qkv, dt));
+  }
   return 0;
 }
 
@@ -628,11 +710,15 @@ int fwd_out(gpt_ctx* c, int l, void* const* P, bool write_out) {
   CB(rm_gemm(c, false, true, N, h, h, 1.f, c->att, dt, P[4], dt, 1.f, c->x_mid, CUDA_R_32F));
   (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->x_mid, (const T*)P[6], (const T*)P[7],
                                                                (T*)c->ln2, c->ln2_m, c->ln2_r, N, h);
-  (g_launches++, 0), bias_fill<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((T*)c->fc_pre, (const T*)P[9], 4 * h,
-                                                                          4 * Nh / 8);
-  CB(rm_gemm(c, false, true, N, 4 * h, h, 1.f, c->ln2, dt, P[8], dt, 1.f, c->fc_pre, dt));
-  (g_launches++, 0), gelu_fwd<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((const T*)c->fc_pre, (T*)c->fc_act,
-                                                                         4 * Nh / 8);
+  if (c->use_lt & 2) {
+    CB(lt_gemm(c, false, true, N, 4 * h, h, c->ln2, P[8], c->fc_act, CUBLASLT_EPILOGUE_GELU_AUX_BIAS, P[9], c->fc_pre));
+  } else {
+    (g_launches++, 0), bias_fill<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((T*)c->fc_pre, (const T*)P[9], 4 * h,
+                                                                            4 * Nh / 8);
+    CB(rm_gemm(c, false, true, N, 4 * h, h, 1.f, c->ln2, dt, P[8], dt, 1.f, c->fc_pre, dt));
+    (g_launches++, 0), gelu_fwd<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((const T*)c->fc_pre, (T*)c->fc_act,
+                                                                           4 * Nh / 8);
+  }
   if (write_out) {
     (g_launches++, 0), resid_bias<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(c->x_mid, (const T*)P[11], xout, h, Nh / 8);
     CB(rm_gemm(c, false, true, N, h, 4 * h, 1.f, c->fc_act, dt, P[10], dt, 1.f, xout, CUDA_R_32F));
@@ -663,8 +749,12 @@ int bwd_mlp(gpt_ctx* c, int l, void* const* P, float* const* G) {
   (g_launches++, 0), cast_f2t<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(c->dres, (T*)c->dy, Nh / 8);
   CB(rm_gemm(c, true, false, h, 4 * h, N, 1.f, c->dy, dt, c->fc_act, dt, 0.f, G[10], CUDA_R_32F));
   if ((r = colsum(c, c->dres, true, N, h, G[11]))) return r;
-  CB(rm_gemm(c, false, false, N, 4 * h, h, 1.f, c->dy, dt, P[10], dt, 0.f, c->d4h, dt));
-  (g_launches++, 0), gelu_bwd<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((T*)c->d4h, (const T*)c->fc_pre, 4 * Nh / 8);
+  if (c->use_lt & 4) {
+    CB(lt_gemm(c, false, false, N, 4 * h, h, c->dy, P[10], c->d4h, CUBLASLT_EPILOGUE_DGELU, nullptr, c->fc_pre));
+  } else {
+    CB(rm_gemm(c, false, false, N, 4 * h, h, 1.f, c->dy, dt, P[10], dt, 0.f, c->d4h, dt));
+    (g_launches++, 0), gelu_bwd<T><<<grid_for(4 * Nh / 8), 256, 0, c->st>>>((T*)c->d4h, (const T*)c->fc_pre, 4 * Nh / 8);
+  }
   CB(rm_gemm(c, true, false, 4 * h, h, N, 1.f, c->d4h, dt, c->ln2, dt, 0.f, G[8], CUDA_R_32F));
   if ((r = colsum(c, c->d4h, false, N, 4 * h, G[9]))) return r;
   CB(rm_gemm(c, false, false, N, h, 4 * h, 1.f, c->d4h, dt, P[8], dt, 0.f, c->dln, CUDA_R_32F));
@@ -832,6 +922,11 @@ int32_t gpt_create(const gpt_config* cfg, gpt_ctx** out) {
   cublasSetWorkspace(c->cb, c->ws, c->ws_bytes);
   cublasSetMathMode(c->cb, CUBLAS_DEFAULT_MATH);  // no TF32 in fp32 mode
   cublasSetAtomicsMode(c->cb, CUBLAS_ATOMICS_NOT_ALLOWED);
+  if (c->bf16) {
+    const char* e = getenv("SH_GPT_LT");
+    const int mask = e ? atoi(e) : 7;
+    c->use_lt = mask != 0 && cublasLtCreate(&c->lt) == CUBLAS_STATUS_SUCCESS ? mask : 0;
+  }
   (g_launches++, 0), fill_ones<float><<<grid_for(mN), 256, 0, c->st>>>(c->ones_f, mN);
   if (c->bf16)
     (g_launches++, 0), fill_ones<bf16><<<grid_for(mN), 256, 0, c->st>>>((bf16*)c->ones_t, mN);
@@ -850,6 +945,7 @@ int32_t gpt_destroy(gpt_ctx* c) {
   if (!c) return 0;
   if (c->st) cudaStreamSynchronize(c->st);
   if (c->cb) cublasDestroy(c->cb);
+  if (c->lt) cublasLtDestroy(c->lt);
   for (void* p : c->allocs) cudaFree(p);
   delete c;
   return 0;
