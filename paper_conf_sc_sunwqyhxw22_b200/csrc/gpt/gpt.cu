@@ -163,6 +163,113 @@ __global__ void ln_fwd(const float* x, const T* g, const T* b, T* out, float* me
   }
 }
 
+// Register-cached LN (h <= 8192): one 128-thread block per row, thread t holds elements
+// 8t + 1024k (k < K) of the row, so x (and dy) are read from DRAM once; the two-pass warp-per-row
+// kernels re-read the row from DRAM (measured: 2x the algorithmic bytes at h 4096).  Block sums
+// are a fixed tree (warp shuffle, then the 4 warp partials in order): deterministic.
+__device__ __forceinline__ float block_sum128(float x, float* red) {
+  x = warp_sum(x);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = x;
+  __syncthreads();
+  const float r = (red[0] + red[1]) + (red[2] + red[3]);
+  __syncthreads();  // red is reused by the next reduction
+  return r;
+}
+
+template <class T, int K>
+__global__ void __launch_bounds__(128) ln_fwd_reg(const float* x, const T* g, const T* b, T* out, float* mean,
+                                                  float* rstd, int N, int h) {
+  __shared__ float red[4];
+  const int row = blockIdx.x;
+  const float* xr = x + (int64_t)row * h;
+  float v[K][8];
+  float s = 0.f;
+#pragma unroll
+  for (int k = 0; k < K; ++k) {
+    const int c = 8 * threadIdx.x + 1024 * k;
+    if (c < h) {
+      ld8(xr + c, v[k]);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) s += v[k][i];
+    }
+  }
+  const float mu = block_sum128(s, red) / h;
+  float var = 0.f;
+#pragma unroll
+  for (int k = 0; k < K; ++k)
+    if (8 * threadIdx.x + 1024 * k < h)
+#pragma unroll
+      for (int i = 0; i < 8; ++i) var += (v[k][i] - mu) * (v[k][i] - mu);
+  const float rs = 1.0f / sqrtf(block_sum128(var, red) / h + kLnEps);
+  T* o = out + (int64_t)row * h;
+#pragma unroll
+  for (int k = 0; k < K; ++k) {
+    const int c = 8 * threadIdx.x + 1024 * k;
+    if (c < h) {
+      float gg[8], bb[8];
+      ld8(g + c, gg);
+      ld8(b + c, bb);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) v[k][i] = (v[k][i] - mu) * rs * gg[i] + bb[i];
+      st8(o + c, v[k]);
+    }
+  }
+  if (threadIdx.x == 0) {
+    mean[row] = mu;
+    rstd[row] = rs;
+  }
+}
+
+template <class T, int K>
+__global__ void __launch_bounds__(128) ln_bwd_reg(const float* dy, const float* x, const float* mean,
+                                                  const float* rstd, const T* g, float* dres, float* tmp, int N,
+                                                  int h) {
+  __shared__ float red[4];
+  const int row = blockIdx.x;
+  const float* dr = dy + (int64_t)row * h;
+  const float* xr = x + (int64_t)row * h;
+  const float mu = mean[row], rs = rstd[row];
+  float d[K][8], xh[K][8];
+  float a = 0.f, bb = 0.f;
+#pragma unroll
+  for (int k = 0; k < K; ++k) {
+    const int c = 8 * threadIdx.x + 1024 * k;
+    if (c < h) {
+      float gg[8];
+      ld8(dr + c, d[k]);
+      ld8(xr + c, xh[k]);
+      ld8(g + c, gg);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        xh[k][i] = (xh[k][i] - mu) * rs;
+        const float dxh = d[k][i] * gg[i];
+        a += dxh;
+        bb += dxh * xh[k][i];
+      }
+    }
+  }
+  a = block_sum128(a, red) / h;
+  bb = block_sum128(bb, red) / h;
+  float* o = dres + (int64_t)row * h;
+  float* t = tmp + (int64_t)row * h;
+#pragma unroll
+  for (int k = 0; k < K; ++k) {
+    const int c = 8 * threadIdx.x + 1024 * k;
+    if (c < h) {
+      float gg[8], ov[8], tv[8];
+      ld8(g + c, gg);
+      ld8(o + c, ov);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        ov[i] += rs * (d[k][i] * gg[i] - a - xh[k][i] * bb);
+        tv[i] = d[k][i] * xh[k][i];
+      }
+      st8(o + c, ov);
+      st8(t + c, tv);
+    }
+  }
+}
+
 // dres += LN backward(dy); tmp = dy * xhat (for dgamma); dbeta = colsum(dy) done by cuBLAS
 template <class T>
 __global__ void ln_bwd(const float* dy, const float* x, const float* mean, const float* rstd, const T* g,
@@ -478,6 +585,33 @@ int grid_for(int64_t total, int threads = 256) {
   return (int)(g < cap ? (g > 0 ? g : 1) : cap);
 }
 
+// LN launchers: the register-cached kernels for h <= 8192 (K = ceil(h / 1024) groups of 8 per thread)
+template <class T>
+void launch_ln_fwd(cudaStream_t st, const float* x, const T* g, const T* b, T* out, float* m, float* r, int N, int h) {
+  static const bool reg = !(getenv("SH_GPT_LN_REG") && getenv("SH_GPT_LN_REG")[0] == '0');  // A/B switch
+  const int K = reg ? (h + 1023) / 1024 : 0;
+  g_launches++;
+  switch (K) {
+#define LNF(k) case k: ln_fwd_reg<T, k><<<N, 128, 0, st>>>(x, g, b, out, m, r, N, h); break;
+    LNF(1) LNF(2) LNF(3) LNF(4) LNF(5) LNF(6) LNF(7) LNF(8)
+#undef LNF
+    default: ln_fwd<T><<<(N + 7) / 8, 256, 0, st>>>(x, g, b, out, m, r, N, h);
+  }
+}
+template <class T>
+void launch_ln_bwd(cudaStream_t st, const float* dy, const float* x, const float* m, const float* r, const T* g,
+                   float* dres, float* tmp, int N, int h) {
+  static const bool reg = !(getenv("SH_GPT_LN_REG") && getenv("SH_GPT_LN_REG")[0] == '0');  // A/B switch
+  const int K = reg ? (h + 1023) / 1024 : 0;
+  g_launches++;
+  switch (K) {
+#define LNB(k) case k: ln_bwd_reg<T, k><<<N, 128, 0, st>>>(dy, x, m, r, g, dres, tmp, N, h); break;
+    LNB(1) LNB(2) LNB(3) LNB(4) LNB(5) LNB(6) LNB(7) LNB(8)
+#undef LNB
+    default: ln_bwd<T><<<(N + 7) / 8, 256, 0, st>>>(dy, x, m, r, g, dres, tmp, N, h);
+  }
+}
+
 }  // namespace
 
 struct gpt_ctx {
@@ -674,7 +808,7 @@ int fwd_qkv(gpt_ctx* c, int l, void* const* P) {
   const cudaDataType_t dt = c->dt;
   const float* xin = c->x + (int64_t)l * c->maxN * h;
   const int64_t Nh = (int64_t)N * h;
-  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
+  launch_ln_fwd<T>(c->st, xin, (const T*)P[0], (const T*)P[1], (T*)c->ln1,
                                                                c->ln1_m, c->ln1_r, N, h);
   if (c->use_lt & 1) {
     CB(lt_gemm(c, false, true, N, 3 * h, h, c->ln1, P[2], c->qkv, CUBLASLT_EPILOGUE_BIAS, P[3], nullptr));
@@ -708,7 +842,7 @@ int fwd_out(gpt_ctx* c, int l, void* const* P, bool write_out) {
   const int64_t Nh = (int64_t)N * h;
   (g_launches++, 0), resid_bias<T><<<grid_for(Nh / 8), 256, 0, c->st>>>(xin, (const T*)P[5], c->x_mid, h, Nh / 8);
   CB(rm_gemm(c, false, true, N, h, h, 1.f, c->att, dt, P[4], dt, 1.f, c->x_mid, CUDA_R_32F));
-  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->x_mid, (const T*)P[6], (const T*)P[7],
+  launch_ln_fwd<T>(c->st, c->x_mid, (const T*)P[6], (const T*)P[7],
                                                                (T*)c->ln2, c->ln2_m, c->ln2_r, N, h);
   if (c->use_lt & 2) {
     CB(lt_gemm(c, false, true, N, 4 * h, h, c->ln2, P[8], c->fc_act, CUBLASLT_EPILOGUE_GELU_AUX_BIAS, P[9], c->fc_pre));
@@ -758,7 +892,7 @@ int bwd_mlp(gpt_ctx* c, int l, void* const* P, float* const* G) {
   CB(rm_gemm(c, true, false, 4 * h, h, N, 1.f, c->d4h, dt, c->ln2, dt, 0.f, G[8], CUDA_R_32F));
   if ((r = colsum(c, c->d4h, false, N, 4 * h, G[9]))) return r;
   CB(rm_gemm(c, false, false, N, h, 4 * h, 1.f, c->d4h, dt, P[8], dt, 0.f, c->dln, CUDA_R_32F));
-  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, c->x_mid, c->ln2_m, c->ln2_r, (const T*)P[6],
+  launch_ln_bwd<T>(c->st, c->dln, c->x_mid, c->ln2_m, c->ln2_r, (const T*)P[6],
                                                                c->dres, c->tmp, N, h);
   if ((r = colsum(c, c->tmp, true, N, h, G[6]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[7]))) return r;
@@ -796,7 +930,7 @@ int bwd_qkv(gpt_ctx* c, int l, void* const* P, float* const* G) {
   CB(rm_gemm(c, true, false, 3 * h, h, N, 1.f, c->dqkv, dt, c->ln1, dt, 0.f, G[2], CUDA_R_32F));
   if ((r = colsum(c, c->dqkv, false, N, 3 * h, G[3]))) return r;
   CB(rm_gemm(c, false, false, N, h, 3 * h, 1.f, c->dqkv, dt, P[2], dt, 0.f, c->dln, CUDA_R_32F));
-  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xin, c->ln1_m, c->ln1_r, (const T*)P[0],
+  launch_ln_bwd<T>(c->st, c->dln, xin, c->ln1_m, c->ln1_r, (const T*)P[0],
                                                                c->dres, c->tmp, N, h);
   if ((r = colsum(c, c->tmp, true, N, h, G[0]))) return r;
   if ((r = colsum(c, c->dln, true, N, h, G[1]))) return r;
@@ -818,7 +952,7 @@ int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float
   const int N = c->N, h = c->h, V = c->V, S = c->S;
   const cudaDataType_t dt = c->dt;
   const float* xL = c->x + (int64_t)c->L * c->maxN * h;
-  (g_launches++, 0), ln_fwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(xL, (const T*)R[2], (const T*)R[3], (T*)c->lnf,
+  launch_ln_fwd<T>(c->st, xL, (const T*)R[2], (const T*)R[3], (T*)c->lnf,
                                                                c->lnf_m, c->lnf_r, N, h);
   CB(rm_gemm(c, false, true, N, V, h, 1.f, c->lnf, dt, R[0], dt, 0.f, c->logits, CUDA_R_32F));
   (g_launches++, 0), ce_fwd_bwd<T><<<N, 512, 0, c->st>>>(c->logits, tok, S, V, 1.0f / N, c->row_loss, (T*)c->dlogits);
@@ -829,7 +963,7 @@ int head_impl(gpt_ctx* c, const int* tok, void* const* R, float* const* G, float
   }
   CB(rm_gemm(c, false, false, N, h, V, 1.f, c->dlogits, dt, R[0], dt, 0.f, c->dln, CUDA_R_32F));
   CK(cudaMemsetAsync(c->dres, 0, sizeof(float) * (size_t)N * h, c->st));
-  (g_launches++, 0), ln_bwd<T><<<(N + 7) / 8, 256, 0, c->st>>>(c->dln, xL, c->lnf_m, c->lnf_r, (const T*)R[2], c->dres,
+  launch_ln_bwd<T>(c->st, c->dln, xL, c->lnf_m, c->lnf_r, (const T*)R[2], c->dres,
                                                                c->tmp, N, h);
   int r;
   if ((r = colsum(c, c->tmp, true, N, h, G[2]))) return r;
