@@ -2,10 +2,16 @@
 //
 // Paper mechanism -> this file:
 //   pinned per-layer CPU buffers            -> HostStore: one mmap'ed, THP-advised,
-//                                                              page-locked region; per layer fp32
-//                                                              master | m | v | bf16 shadow
+//                                                              page-locked block per host layer;
+//                                                              fp32 master | m | v | bf16 shadow;
+//                                                              NUMA placement by mbind before first
+//                                                              touch (numa.cpp, sh_config.numa_policy)
 //   reserved round-robin GPU buffer queue -> ring of w+1 slots, one cudaMalloc,
 //                                                              grow-only; param half + grad half
+//                                                              (or decoupled from the GPU set, R22)
+//   fixed-size buffer, variable layer count  -> sh_config.ring_bytes: variable-capacity
+//                                                              slots in one buffer, capacity-filtered
+//                                                              Belady (NEXT-4)
 //   pre_forward / post_forward (Fig. 3b)      -> sh_forward_layer PRE/POST
 //   pre_backward (Fig. 3c)                    -> sh_backward_layer PRE/POST
 //   "idle CUDA stream" async copies          -> H2D and D2H copy-engine streams, each
