@@ -55,7 +55,7 @@ CPU_HARD_DEFAULT = {"c3", "c4", "c4max"}   # autotune with the eq. 3 CPU-through
 # growth, GPU set filling the HBM a decoupled ring leaves, late bf16 host shadows (C4: 7.30 -> 7.92
 # samples/s, profiles/r01_bench_default_c4_v3.json vs r01_bench_c4_tuned_coupled.json)
 TUNED_DEFAULT = {"c3", "c4"}
-SETTLE_STEPS = 2  # untimed steps after the autotuner's window change (before the K timed steps)
+SETTLE_STEPS = 4  # untimed steps after the autotuner's window change (before the K timed steps)
 
 
 def mem_available() -> int:

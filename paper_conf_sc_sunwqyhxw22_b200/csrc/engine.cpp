@@ -267,6 +267,7 @@ struct sh_ctx {
 
   // ---- streams
   cudaStream_t cs = nullptr, h2d = nullptr, d2h = nullptr, stage = nullptr, comm = nullptr;
+  cudaStream_t k3s = nullptr;  // K3 of host layers, beside the D2H copy of the same gradients
   ncclComm_t nccl = nullptr;
   ncclComm_t nccl_fetch = nullptr;  // NEXT-1: collectives issued by the H2D issuer thread
   bool slice_fetch = false;
@@ -1477,7 +1478,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
 sh_status sync_all(sh_ctx* c) {
   c->ih2d.drain();
   c->id2h.drain();
-  for (cudaStream_t s : {c->cs, c->h2d, c->d2h, c->stage, c->comm})
+  for (cudaStream_t s : {c->cs, c->h2d, c->d2h, c->stage, c->comm, c->k3s})
     if (s) CKC(c, cudaStreamSynchronize(s));
   // all host layers updated for the steps taken so far
   if (!state_wait(c, [&] {
@@ -1728,6 +1729,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->cs = static_cast<cudaStream_t>(cfg->compute_stream);
   CKC(c.get(), cudaStreamCreateWithFlags(&c->h2d, cudaStreamNonBlocking));
   CKC(c.get(), cudaStreamCreateWithFlags(&c->d2h, cudaStreamNonBlocking));
+  CKC(c.get(), cudaStreamCreateWithFlags(&c->k3s, cudaStreamNonBlocking));
   CKC(c.get(), cudaStreamCreateWithFlags(&c->stage, cudaStreamNonBlocking));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_cs_mark, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
@@ -2332,14 +2334,17 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P, k3_on_d2h, lo, hi] {
         maybe_delay(c->cfg.flags);
         CKA(c, cudaStreamWaitEvent(c->d2h, grads_ready, 0));
-        if (k3_on_d2h) {  // K3 before any host wait: sh_step only needs the norms
-          if (P) CKA(c, cudaEventRecord(P->k30[x], c->d2h));
-          CKA(c, kern::sumsq(src, n, c->scratch_d2h, c->partials + x, c->d2h));
+        if (k3_on_d2h) {  // K3 before any host wait (sh_step only needs the norms), on its own
+                          // stream so the copy engine does not queue behind it; the grad half is
+                          // released only after both have read it
+          CKA(c, cudaStreamWaitEvent(c->k3s, grads_ready, 0));
+          if (P) CKA(c, cudaEventRecord(P->k30[x], c->k3s));
+          CKA(c, kern::sumsq(src, n, c->scratch_d2h, c->partials + x, c->k3s));
           if (P) {
-            CKA(c, cudaEventRecord(P->k31[x], c->d2h));
+            CKA(c, cudaEventRecord(P->k31[x], c->k3s));
             P->rec_k3[x] = 1;
           }
-          CKA(c, cudaEventRecord(c->ev_k3_last, c->d2h));
+          CKA(c, cudaEventRecord(c->ev_k3_last, c->k3s));
           c->k3_pub.store(gen);
           notify_state(c);
         }
@@ -2355,6 +2360,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
           CKA(c, cudaEventRecord(P->g2c1[x], c->d2h));
           P->rec_g2c[x] = 1;
         }
+        if (k3_on_d2h) CKA(c, cudaStreamWaitEvent(c->d2h, c->ev_k3_last, 0));  // this layer's K3
         CKA(c, cudaEventRecord(gf, c->d2h));
         CKA(c, cudaLaunchHostFunc(c->d2h, landed_cb, new Landed{c, x, step, k, sc}));
         c->d2h_bytes += 4 * (hi - lo);
@@ -2468,6 +2474,7 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     const double mx = c->cfg.max_grad_norm;
     c->id2h.push([c, rk, nd, L, mx] {
       CKA(c, cudaStreamWaitEvent(c->d2h, rk, 0));
+      CKA(c, cudaStreamWaitEvent(c->d2h, c->ev_k3_last, 0));  // every host layer's K3 (k3 stream)
       CKA(c, kern::norm_finalize(c->partials, L + 1, mx, c->norm_dev, c->coef_dev, c->d2h));
       CKA(c, cudaEventRecord(nd, c->d2h));
     });
@@ -2910,7 +2917,7 @@ sh_status sh_destroy(sh_ctx* c) {
   notify_state(c);
   c->ih2d.stop();
   c->id2h.stop();
-  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
+  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s})
     if (s) cudaStreamSynchronize(s);
   if (c->cs) cudaStreamSynchronize(c->cs);
   if (c->nccl_fetch) g_nccl.CommDestroy(c->nccl_fetch);
@@ -2943,7 +2950,7 @@ sh_status sh_destroy(sh_ctx* c) {
     if (c->ev_res_k3[i]) cudaEventDestroy(c->ev_res_k3[i]);
     if (c->ev_norm[i]) cudaEventDestroy(c->ev_norm[i]);
   }
-  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm})
+  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s})
     if (s) cudaStreamDestroy(s);
   for (auto& b : c->hshadow) host_block_free(b.p, b.bytes);
   for (auto& b : c->hblocks) {
