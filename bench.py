@@ -390,7 +390,8 @@ def main():
         dev = host.to(f"cuda:{local}")
         step_fn = tr.forward_only if args.fp_only else tr.step_device
         for t in range(W + S):
-            tr.tok_dev.copy_(dev[t])
+            with torch.cuda.stream(tr.stream):  # ordered after the previous step's reads of tok_dev
+                tr.tok_dev.copy_(dev[t], non_blocking=True)
             step_fn()
         tr.engine.synchronize()
         st0 = tr.engine.stats()

@@ -158,6 +158,11 @@ def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None
         rhs = sum(fp[i] + bp[i] for i in range(k + 1)) + sum(og[i] for i in range(g))
         v = rhs - oc[k]
         slack = v if slack is None else min(slack, v)
+    cpu_total = 0.0
+    for k in range(g, L):
+        cpu_total += oc[k]
+    gpu_step = sum(fp[i] + bp[i] for i in range(L)) + sum(og[i] for i in range(g))
     return {"window": g, "ring_slots": d + 1, "reason": reason, "w_max_memory": max(mems),
+            "cpu_total_ms": cpu_total, "gpu_step_ms": gpu_step,
             "eq3_min_slack_ms": 0.0 if slack is None else slack,
             "eq4_lhs_ms": 5.0 * L * t_async, "eq4_rhs_ms": sum(og[i] for i in range(g, L))}

@@ -621,9 +621,12 @@ void finish_job(sh_ctx* c, Job* j) {
   // (without SH_FLAG_SPILL_EVICT the kernel's flusher writes the layer back lazily: forcing an
   // early write-back made the next step's CPU update wait on pages still under write-back --
   // C2 with 8 spilled layers ran at 15.5 instead of ~47 samples/s, profiles/r01_bench_c2_spill8_*)
+  // landing buffer first, readiness last: sync_all (and so grow_landing, which replaces the
+  // landing_done array) returns once every layer is ready, so no worker may still be about to
+  // touch a landing counter at that point
+  c->landing_done[j->landing].fetch_add(1, std::memory_order_release);
   c->ready[j->layer].store(j->step + 1, std::memory_order_release);
   if (c->shared) c->ctl->cnt[j->layer].fetch_add(1, std::memory_order_release);
-  c->landing_done[j->landing].fetch_add(1, std::memory_order_release);
   notify_state(c);
 }
 
@@ -1491,6 +1494,13 @@ sh_status sync_all(sh_ctx* c) {
   return check_failed(c);
 }
 
+// Forget every ring mapping: each layer is fetched / K1-restaged again at its next use (always
+// valid between steps: GPU-optimised layers restage from their HBM masters, host layers fetch).
+void clear_ring_map(sh_ctx* c) {
+  for (int s = 0; s < (int)c->slot_layer.size(); ++s) c->slot_layer[s] = -1;
+  for (int x = 0; x < c->L; ++x) c->layer_slot[x] = -1;
+}
+
 // Move the G boundary from c->w to w_new (between steps, everything idle).
 sh_status apply_window(sh_ctx* c, int w_new) {
   sh_status st = sync_all(c);
@@ -1521,11 +1531,15 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   // ring first (the old one is released inside), then the joining layers' HBM states (rolled
   // back on failure so the caller can retry with a smaller window)
   st = alloc_ring(c, c->ring_for(w_new));
-  if (st != SH_OK) return st;
+  if (st != SH_OK) {
+    clear_ring_map(c);  // a re-allocated ring holds no valid copy
+    return st;
+  }
   for (int x = w_old; x < w_new; ++x) {
     st = alloc_g(c, x);
     if (st != SH_OK) {
       for (int y = w_old; y < w_new; ++y) free_g(c, y);
+      clear_ring_map(c);
       return st;
     }
     const int64_t n = c->lay[x].n_pad;
@@ -1534,7 +1548,11 @@ sh_status apply_window(sh_ctx* c, int w_new) {
     CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
   }
   st = ensure_gbufs(c, w_new);
-  if (st != SH_OK) return st;
+  if (st != SH_OK) {
+    for (int y = w_old; y < w_new; ++y) free_g(c, y);
+    clear_ring_map(c);
+    return st;
+  }
   c->w = w_new;
   c->n_active = c->ring_for(w_new);
   c->d = c->n_active - 1;
@@ -2053,6 +2071,14 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
   sh_status st = check_failed(c);
   if (st != SH_OK) return st;
   if (step < 0) step = 0;
+  // re-registration after the store is live (resume / state reload between steps): the previous
+  // step's CPU updates, prefetches and per-layer K2s may still read or write this layer's state --
+  // drain them first; the ring's compute copies are re-staged below
+  const bool live = c->registered_all;
+  if (live) {
+    st = sync_all(c);
+    if (st != SH_OK) return st;
+  }
   if (layer == -1) {
     const int64_t n = c->res.n_pad;
     std::vector<float> tmp(n);
@@ -2101,6 +2127,12 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
   if (all && !c->registered_all) {
     if (!shm_barrier(c, 1, "registration of the shared host store")) return check_failed(c);
     c->registered_all = true;
+    st = stage_g_layers(c);
+    if (st != SH_OK) return st;
+    CKC(c, cudaStreamSynchronize(c->cs));
+  } else if (live && layer >= 0) {
+    // every ring copy of the layer is stale: drop the host-layer mapping (the next use fetches
+    // the new state) and re-stage the GPU-optimised layers from their (new) HBM masters
     st = stage_g_layers(c);
     if (st != SH_OK) return st;
     CKC(c, cudaStreamSynchronize(c->cs));
@@ -2683,8 +2715,15 @@ sh_status sh_set_window_ring(sh_ctx* c, int32_t w, int32_t ring) {
   sh_status st = check_failed(c);
   if (st != SH_OK) return st;
   if (w == c->w && ring == c->ring_cap) return SH_OK;
+  const int old_cap = c->ring_cap;
   c->ring_cap = ring;
-  return apply_window(c, w);
+  st = apply_window(c, w);
+  if (st != SH_OK) {  // the window did not change: neither does the ring cap
+    c->ring_cap = old_cap;
+    c->n_active = std::min(c->ring_for(c->w), std::max(c->ring_alloc, 1));
+    c->d = c->n_active - 1;
+  }
+  return st;
 }
 
 sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
@@ -3070,15 +3109,20 @@ sh_status sh_op_sumsq_gpu(const float* g, int64_t n, double* out_dev, void* stre
   clear_error();
   const void* ptrs[] = {g};
   if (!g || !out_dev || !ops_args_ok(n, 0, ptrs, 1)) return SH_ERR_INVALID;
-  static double* scratch = nullptr;
-  if (!scratch) {
-    if (cudaMalloc(&scratch, 8 * (kern::kSumsqMaxBlocks + 1)) != cudaSuccess ||
-        cudaMemset(scratch, 0, 8 * (kern::kSumsqMaxBlocks + 1)) != cudaSuccess) {
-      set_error("K3 scratch allocation failed");
-      return SH_ERR_OOM_DEVICE;
-    }
+  // private, stream-ordered scratch (partials + completion ticket) per call: concurrent calls on
+  // other streams or devices never share it
+  double* scratch = nullptr;
+  const size_t sb = 8 * (kern::kSumsqMaxBlocks + 1);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (cudaMallocAsync(reinterpret_cast<void**>(&scratch), sb, st) != cudaSuccess ||
+      cudaMemsetAsync(scratch, 0, sb, st) != cudaSuccess) {
+    cudaGetLastError();
+    set_error("K3 scratch allocation failed");
+    return SH_ERR_OOM_DEVICE;
   }
-  const cudaError_t e = kern::sumsq(g, n, scratch, out_dev, static_cast<cudaStream_t>(stream));
+  cudaError_t e = kern::sumsq(g, n, scratch, out_dev, st);
+  const cudaError_t e2 = cudaFreeAsync(scratch, st);
+  if (e == cudaSuccess) e = e2;
   if (e != cudaSuccess) {
     set_error("K3 launch: %s", cudaGetErrorString(e));
     return SH_ERR_CUDA;
