@@ -432,11 +432,11 @@ def main():
         if args.trace_out and rank == 0:
             # Chrome trace (chrome://tracing / Perfetto) of the last profiled step: Fig. 4 analogue
             tid = {"fp": 1, "bp": 1, "k2_adamw": 1, "h2d_fp": 2, "h2d_bp": 2, "d2h_grad": 3, "k1_stage": 4,
-                   "k3_sumsq": 5}
+                   "k3_sumsq": 5, "cpu_adam": 6, "h2d_wait_cpu": 7}
             ev = [{"name": f"{e['kind']} L{e['layer']}", "ph": "X", "pid": 0, "tid": tid[e["kind"]],
                    "ts": e["start_ms"] * 1e3, "dur": (e["end_ms"] - e["start_ms"]) * 1e3} for e in trace]
             names = {1: "compute stream", 2: "H2D copy engine", 3: "D2H copy engine", 4: "K1 stage stream",
-                     5: "K3 (D2H stream)"}
+                     5: "K3 (D2H stream)", 6: "CPU Adam pool (host clock)", 7: "H2D issuer waiting on CPU Adam"}
             ev += [{"name": "thread_name", "ph": "M", "pid": 0, "tid": k, "args": {"name": v}} for k, v in names.items()]
             with open(args.trace_out + (f".w{window}" if window != w else ""), "w") as f:
                 json.dump({"traceEvents": ev, "displayTimeUnit": "ms"}, f)

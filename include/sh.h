@@ -134,6 +134,13 @@ typedef struct {
 #define SH_FLAG_LATE_SHADOW (1ull << 16)  /* bf16 mode with SH_FLAG_FETCH_FP32: after the autotune, give every host
                                             layer a bf16 shadow in the host RAM the GPU set gave back (fetch 2
                                             instead of 4 B/param; the solver already plans with that cost) */
+#define SH_FLAG_TEST_HOST_COLLECTIVE (1ull << 17) /* test (data parallel with shm_name): every collective -- the
+                                            per-layer all-reduce / reduce-scatter, the resident all-reduce,
+                                            the norm-partials all-gather -- runs through a shared host segment
+                                            on the driver thread, the ranks' contributions summed in rank
+                                            order (identical on every rank).  Several ranks on ONE GPU with
+                                            DIFFERENT data: the averaging itself is checked against the
+                                            oracle's global-batch mean.  No NCCL. */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
@@ -307,7 +314,9 @@ typedef struct {
 /* One interval of a profiled step (times in ms from the step's first FP hook). */
 typedef struct {
   int32_t kind;   /* 0 FP compute, 1 BP compute, 2 H2D (FP), 3 H2D (BP), 4 D2H grads, 5 K1 stage,
-                     6 K3 sumsq, 7 K2 */
+                     6 K3 sumsq, 7 K2; host-clock intervals aligned to the step start: 8 CPU Adam job of
+                     the layer (this step's gradients; runs into the next step), 9 H2D issuer waiting
+                     for the CPU Adam of the layer it is about to fetch */
   int32_t layer;  /* -1 for K2 */
   double start_ms, end_ms;
 } sh_trace_event;

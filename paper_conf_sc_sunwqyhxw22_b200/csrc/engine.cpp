@@ -114,6 +114,10 @@ struct Nccl {
   ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
   ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
   ncclResult_t (*CommSplit)(ncclComm_t, int, int, ncclComm_t*, ncclConfig_t*) = nullptr;
+  ncclResult_t (*ReduceScatter)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                                cudaStream_t) = nullptr;
+  ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*) = nullptr;
+  ncclResult_t (*CommAbort)(ncclComm_t) = nullptr;
   const char* (*GetErrorString)(ncclResult_t) = nullptr;
   bool load() {
     if (h) return true;
@@ -130,8 +134,12 @@ struct Nccl {
     CommDestroy = (decltype(CommDestroy))dlsym(h, "ncclCommDestroy");
     AllGather = (decltype(AllGather))dlsym(h, "ncclAllGather");
     CommSplit = (decltype(CommSplit))dlsym(h, "ncclCommSplit");
+    ReduceScatter = (decltype(ReduceScatter))dlsym(h, "ncclReduceScatter");
+    CommGetAsyncError = (decltype(CommGetAsyncError))dlsym(h, "ncclCommGetAsyncError");
+    CommAbort = (decltype(CommAbort))dlsym(h, "ncclCommAbort");
     GetErrorString = (decltype(GetErrorString))dlsym(h, "ncclGetErrorString");
-    return GetUniqueId && CommInitRank && AllReduce && CommDestroy && GetErrorString;
+    return GetUniqueId && CommInitRank && AllReduce && CommDestroy && GetErrorString && ReduceScatter &&
+           AllGather && CommGetAsyncError && CommAbort;
   }
 };
 Nccl g_nccl;
@@ -194,6 +202,10 @@ struct ProfSet {  // CUDA timing events of one step (double-buffered by step par
   std::vector<uint8_t> rec_fp, rec_bp, rec_k3, rec_k2l;
   cudaEvent_t k2a = nullptr, k2b = nullptr, t0 = nullptr;
   bool rec_k2 = false, rec_t0 = false;
+  // host-side intervals of this step (CPU Adam jobs, H2D-issuer waits on them), in host ms; t0_host is
+  // the host clock when the compute stream passed t0 (a host function right behind the event)
+  std::atomic<double> t0_host{0.0};
+  std::vector<sh_trace_event> host_iv;  // guarded by sh_ctx::pmu
   bool active = false;
   int64_t step = -1;
   int64_t k2_bytes = 0;
@@ -211,6 +223,7 @@ struct GState {
 struct Job {
   int layer;
   int64_t step;
+  double t_first = 0.0;  // host ms when its first chunk was taken (trace)
   int landing;
   int64_t lo, hi;  // element range of this rank (whole layer unless the store is shared)
   int64_t n_chunks;
@@ -220,11 +233,14 @@ struct Job {
 };
 
 // Control block of a shared (multi-process, one box) host store, in /dev/shm.
+constexpr int kMaxHostCollRanks = 64;
 struct ShmCtl {
   std::atomic<int64_t> magic;
   std::atomic<int64_t> created;    // rank 0 finished creating the layer segments
   std::atomic<int64_t> bar[6];     // monotonic barrier counters
   std::atomic<int64_t> window;     // rank 0's autotuned window (every rank must use the same one)
+  std::atomic<int64_t> hc_arrive[kMaxHostCollRanks];  // SH_FLAG_TEST_HOST_COLLECTIVE: per-rank sequence
+  std::atomic<int64_t> hc_done[kMaxHostCollRanks];    //   numbers (contribution written / result read)
   std::atomic<int64_t> cnt[1];     // [2L]: cnt[x] slice updates completed (W per step);
                                    //       cnt[L+x] offloads landed (W per step)
 };
@@ -337,6 +353,18 @@ struct sh_ctx {
   // (a one-rank NCCL communicator: every all-reduce runs, and is the identity)
   bool dp = false;
   bool no_collective = false;
+  bool use_nccl = false;   // the collectives go through NCCL (dp, not a test mode)
+  // SH_FLAG_TEST_HOST_COLLECTIVE: the collectives run on the driver thread through a shared host
+  // segment, summed in a fixed rank order (several ranks on ONE GPU with different data)
+  bool host_coll = false;
+  float* hc_seg = nullptr;   // [W][hc_count] contributions, /dev/shm, page-locked
+  size_t hc_bytes = 0;
+  int64_t hc_count = 0;      // floats per rank
+  float* hc_tmp = nullptr;   // private pinned result staging
+  int64_t hc_seq = 0;
+  bool rs_host = false;      // host layers' gradients are reduce-scattered (shared store: slice r only)
+  double* partials_all = nullptr;  // [W][L+1] gathered per-rank partial sums of squares
+  std::atomic<int> nccl_aborted{0};
   std::string shm_name;
   ShmCtl* ctl = nullptr;
   size_t ctl_bytes = 0;
@@ -487,19 +515,57 @@ sh_status check_failed(sh_ctx* c) {
     if (e_ != cudaSuccess) async_fail((c), SH_ERR_CUDA, "%s: %s", #expr, cudaGetErrorString(e_)); \
   } while (0)
 
-// Wait on the engine state condition (timeout => fail, never hang the box).
+// ---- NCCL health (data parallel).  An asynchronous communicator error (a failed or vanished peer)
+// fails the context; a wait that times out while NCCL work may be pending aborts the communicators,
+// so their kernels exit instead of spinning on the GPU and the box stays usable.
+void nccl_abort(sh_ctx* c, const char* why) {
+  if (!c->use_nccl || c->nccl_aborted.exchange(1)) return;
+  if (c->nccl_fetch) g_nccl.CommAbort(c->nccl_fetch);
+  if (c->nccl) g_nccl.CommAbort(c->nccl);
+  async_fail(c, SH_ERR_NCCL, "NCCL communicators aborted: %s", why);
+}
+
+// false (context failed) if a communicator reports an asynchronous error.  Never called with smu held.
+bool nccl_healthy(sh_ctx* c) {
+  if (!c->use_nccl) return true;
+  if (c->nccl_aborted.load()) return false;
+  for (ncclComm_t m : {c->nccl, c->nccl_fetch}) {
+    if (!m) continue;
+    ncclResult_t r = ncclSuccess;
+    if (g_nccl.CommGetAsyncError(m, &r) != ncclSuccess) continue;
+    if (r != ncclSuccess && r != ncclInProgress) {
+      char b[256];
+      snprintf(b, sizeof(b), "asynchronous error: %s", g_nccl.GetErrorString(r));
+      nccl_abort(c, b);
+      return false;
+    }
+  }
+  return true;
+}
+
+// Wait on the engine state condition (timeout => fail, never hang the box).  With a shared store,
+// cross-process progress is only visible by polling; with NCCL the communicators are polled for
+// asynchronous errors while waiting.
 template <class Pred>
 bool state_wait(sh_ctx* c, Pred pred, const char* what, double* waited_ms = nullptr) {
   if (pred()) return true;
   const double t0 = now_ms();
   std::unique_lock<std::mutex> g(c->smu);
   bool ok;
-  if (c->shared) {  // cross-process progress is only visible by polling the shared counters
+  if (c->shared || c->use_nccl) {
     const double deadline = t0 + 1e3 * wait_timeout_s();
+    double next_poll = t0 + 20.0;
     for (;;) {
       if (c->failed.load() || pred()) { ok = true; break; }
       if (now_ms() > deadline) { ok = false; break; }
-      c->scv.wait_for(g, std::chrono::microseconds(50));
+      if (c->use_nccl && now_ms() > next_poll) {
+        g.unlock();
+        const bool healthy = nccl_healthy(c);
+        g.lock();
+        if (!healthy) { ok = true; break; }  // failed: reported below
+        next_poll = now_ms() + 20.0;
+      }
+      c->scv.wait_for(g, c->shared ? std::chrono::microseconds(50) : std::chrono::microseconds(5000));
     }
   } else {
     ok = c->scv.wait_for(g, std::chrono::duration<double>(wait_timeout_s()),
@@ -508,10 +574,33 @@ bool state_wait(sh_ctx* c, Pred pred, const char* what, double* waited_ms = null
   if (waited_ms) *waited_ms = now_ms() - t0;
   if (!ok) {
     g.unlock();
-    async_fail(c, SH_ERR_STATE, "timeout waiting for %s", what);
+    char b[256];
+    snprintf(b, sizeof(b), "timeout waiting for %s", what);
+    nccl_abort(c, b);  // no-op without NCCL
+    async_fail(c, SH_ERR_STATE, "%s", b);
     return false;
   }
   return !c->failed.load();
+}
+
+// cudaStreamSynchronize, except with NCCL: poll the stream and the communicators, abort on timeout.
+sh_status stream_sync(sh_ctx* c, cudaStream_t s) {
+  if (!c->use_nccl) {
+    CKC(c, cudaStreamSynchronize(s));
+    return SH_OK;
+  }
+  const double deadline = now_ms() + 1e3 * wait_timeout_s();
+  for (;;) {
+    const cudaError_t e = cudaStreamQuery(s);
+    if (e == cudaSuccess) return SH_OK;
+    if (e != cudaErrorNotReady) CKC(c, e);
+    if (!nccl_healthy(c)) return check_failed(c);
+    if (now_ms() > deadline) {
+      nccl_abort(c, "stream synchronize timed out");
+      return check_failed(c);
+    }
+    usleep(200);
+  }
 }
 
 void notify_state(sh_ctx* c) {
@@ -606,6 +695,8 @@ void host_block_free(char* p, size_t bytes) {
 }
 
 // ---------------------------------------------------------------------------- CPU Adam pool
+void host_interval(sh_ctx* c, int kind, int layer, int64_t step, double t0, double t1);
+
 void finish_job(sh_ctx* c, Job* j) {
   if (c->spilled[j->layer] && (c->cfg.flags & SH_FLAG_SPILL_EVICT)) {
     const auto& hb = c->hblocks[j->layer];
@@ -671,6 +762,7 @@ void worker_loop(sh_ctx* c, int tid) {
           if (!job || jp->step < job->step || (jp->step == job->step && jp->layer < job->layer))
             job = jp.get();
         }
+      if (job->next == 0) job->t_first = now_ms();
       chunk = job->next++;
       if (c->clip) coef = c->coef_of_step[job->step & 1];
     }
@@ -687,8 +779,10 @@ void worker_loop(sh_ctx* c, int tid) {
     }
     c->cpu_elems.fetch_add(e - b);
     if (job->done.fetch_add(1) + 1 == job->n_chunks) {
+      const double t_end = now_ms();
       finish_job(c, job);
       std::lock_guard<std::mutex> g(c->pmu);
+      host_interval(c, 8, job->layer, job->step, job->t_first, t_end);
       for (auto it = c->jobs.begin(); it != c->jobs.end(); ++it)
         if (it->get() == job) {
           c->jobs.erase(it);
@@ -798,8 +892,21 @@ void prof_reset(sh_ctx* c, ProfSet& P, int64_t step) {
   }
   P.rec_k2 = false;
   P.rec_t0 = false;
+  P.t0_host.store(0.0);
+  {
+    std::lock_guard<std::mutex> g(c->pmu);
+    P.host_iv.clear();
+  }
   P.active = true;
   P.step = step;
+}
+
+void CUDART_CB t0_cb(void* arg) { static_cast<ProfSet*>(arg)->t0_host.store(now_ms()); }
+
+// A host-side interval of step `step` (under pmu): CPU Adam job (kind 8) or H2D wait on it (kind 9).
+void host_interval(sh_ctx* c, int kind, int layer, int64_t step, double t0, double t1) {
+  ProfSet& P = c->prof[step & 1];
+  if (P.active && P.step == step) P.host_iv.push_back(sh_trace_event{kind, layer, t0, t1});
 }
 
 float ev_ms(cudaEvent_t a, cudaEvent_t b) {
@@ -850,10 +957,15 @@ void build_trace(sh_ctx* c, ProfSet& P) {
     if (P.rec_k2l[i]) add(7, i, P.k2l0[i], P.k2l1[i]);
   }
   if (P.rec_k2) add(7, -1, P.k2a, P.k2b);
+  if (P.t0_host.load() > 0) {
+    std::lock_guard<std::mutex> g(c->pmu);
+    for (const auto& e : P.host_iv)
+      c->trace.push_back(sh_trace_event{e.kind, e.layer, e.start_ms - P.t0_host.load(), e.end_ms - P.t0_host.load()});
+  }
   std::vector<std::pair<double, double>> comp, h2d, d2h;
   double end = 0;
   for (auto& e : c->trace) {
-    end = std::max(end, e.end_ms);
+    if (e.kind <= 7) end = std::max(end, e.end_ms);
     if (e.kind <= 1) comp.emplace_back(e.start_ms, e.end_ms);
     if (e.kind == 2 || e.kind == 3) h2d.emplace_back(e.start_ms, e.end_ms);
     if (e.kind == 4) d2h.emplace_back(e.start_ms, e.end_ms);
@@ -888,7 +1000,7 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
         c->p_c2g[i] = ms;
         c->h2d_busy += ms;
         c->h2d_prof_bytes += (int64_t)((c->bf16 && !c->h_shadow[i]) ? 4 : c->cb) *
-                             (c->slice_fetch && !c->no_collective ? c->shi[i] - c->slo[i] : c->lay[i].n_pad);
+                             (c->slice_fetch && c->use_nccl ? c->shi[i] - c->slo[i] : c->lay[i].n_pad);
       }
     if (P.rec_g2c[i]) {
       const double ms = ev_ms(P.g2c0[i], P.g2c1[i]);
@@ -1019,6 +1131,9 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       double cur = c->cpu_wait_ms.load();
       while (!c->cpu_wait_ms.compare_exchange_weak(cur, cur + waited)) {
       }
+      const double t1 = now_ms();
+      std::lock_guard<std::mutex> g(c->pmu);
+      host_interval(c, 9, y, need, t1 - waited, t1);  // waiting for the update of step need-1
     }
     CKA(c, cudaStreamWaitEvent(c->h2d, pf, 0));
     if (cast) {  // the staging area (grad half) must be free of the previous occupant's offload
@@ -1052,7 +1167,7 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       P->rec_c2g[ph][y] = 1;
     }
     if (slice) {
-      if (!c->no_collective) {  // every rank holds slice r at offset r*cs: gather in place
+      if (c->use_nccl) {  // every rank holds slice r at offset r*cs: gather in place
         const ncclResult_t r = g_nccl.AllGather(buf + eb * c->rank * cs, buf, (size_t)cs,
                                                 eb == 4 ? ncclFloat32 : ncclBfloat16, c->nccl_fetch, c->h2d);
         if (r != ncclSuccess) async_fail(c, SH_ERR_NCCL, "ncclAllGather(fetch): %s", g_nccl.GetErrorString(r));
@@ -1063,7 +1178,7 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
     }
     if (cast) CKA(c, kern::cast_bf16(stage_buf, reinterpret_cast<uint16_t*>(dst), n, c->h2d));
     CKA(c, cudaEventRecord(c->ev_arrive[y], c->h2d));
-    c->h2d_bytes += slice && !c->no_collective ? eb * (shi - slo) : bytes;
+    c->h2d_bytes += slice && c->use_nccl ? eb * (shi - slo) : bytes;
     c->h2d_copies++;
     c->arrive_pub[y].store(gen);
     notify_state(c);
@@ -1482,7 +1597,10 @@ sh_status sync_all(sh_ctx* c) {
   c->ih2d.drain();
   c->id2h.drain();
   for (cudaStream_t s : {c->cs, c->h2d, c->d2h, c->stage, c->comm, c->k3s})
-    if (s) CKC(c, cudaStreamSynchronize(s));
+    if (s) {
+      sh_status st = stream_sync(c, s);
+      if (st != SH_OK) return st;
+    }
   // all host layers updated for the steps taken so far
   if (!state_wait(c, [&] {
         for (int x = 0; x < c->L; ++x)
@@ -1627,6 +1745,98 @@ sh_status nccl_check(sh_ctx* c, ncclResult_t r, const char* what) {
   return SH_ERR_NCCL;
 }
 
+// ---- collectives of the data-parallel path.  NCCL over NVLink in production.
+// SH_FLAG_TEST_HOST_COLLECTIVE runs the same three operations through the shared host segment on the
+// driver thread -- every rank sums the ranks' contributions in rank order, so the results are
+// bitwise identical on all ranks -- which lets several ranks with DIFFERENT data share one GPU and
+// checks the averaging itself against the oracle's global-batch mean (reading R13).
+enum CollOp { kAllReduceAvg, kReduceScatterAvg, kAllGatherF64 };
+
+sh_status coll_host(sh_ctx* c, CollOp op, void* buf, int64_t n, int64_t lo, int64_t hi, void* out, cudaStream_t st) {
+  const int64_t eb = op == kAllGatherF64 ? 8 : 4;
+  if (n * eb > c->hc_count * 4) {
+    set_error("host collective: %lld elements exceed the segment", (long long)n);
+    return SH_ERR_INVALID;
+  }
+  float* mine = c->hc_seg + (int64_t)c->rank * c->hc_count;
+  CKC(c, cudaMemcpyAsync(mine, buf, n * eb, cudaMemcpyDeviceToHost, st));
+  CKC(c, cudaStreamSynchronize(st));
+  const int64_t k = ++c->hc_seq;
+  c->ctl->hc_arrive[c->rank].store(k, std::memory_order_release);
+  auto all_at = [&](std::atomic<int64_t>* a) {
+    for (int r = 0; r < c->W; ++r)
+      if (a[r].load(std::memory_order_acquire) < k) return false;
+    return true;
+  };
+  if (!state_wait(c, [&] { return all_at(c->ctl->hc_arrive); }, "host collective (contributions)"))
+    return check_failed(c);
+  void* dst;
+  const void* src;
+  int64_t bytes;
+  if (op == kAllGatherF64) {
+    for (int r = 0; r < c->W; ++r)
+      std::memcpy(reinterpret_cast<char*>(c->hc_tmp) + (int64_t)r * n * 8, c->hc_seg + (int64_t)r * c->hc_count, n * 8);
+    dst = out;
+    src = c->hc_tmp;
+    bytes = (int64_t)c->W * n * 8;
+  } else {
+    const int64_t b = op == kReduceScatterAvg ? lo : 0, e = op == kReduceScatterAvg ? hi : n;
+    const float inv = (float)(1.0 / (double)c->W);
+    for (int64_t i = b; i < e; ++i) {
+      float acc = c->hc_seg[i];
+      for (int r = 1; r < c->W; ++r) acc = acc + c->hc_seg[(int64_t)r * c->hc_count + i];
+      c->hc_tmp[i] = acc * inv;
+    }
+    dst = static_cast<float*>(buf) + b;
+    src = c->hc_tmp + b;
+    bytes = 4 * (e - b);
+  }
+  c->ctl->hc_done[c->rank].store(k, std::memory_order_release);
+  if (bytes > 0) {
+    CKC(c, cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, st));
+    CKC(c, cudaStreamSynchronize(st));  // hc_tmp is reused by the next call
+  }
+  // nobody rewrites its contribution before every rank has read this round's
+  if (!state_wait(c, [&] { return all_at(c->ctl->hc_done); }, "host collective (completion)"))
+    return check_failed(c);
+  return SH_OK;
+}
+
+// Average of a gradient buffer over the ranks (every rank gets all n elements).
+sh_status coll_allreduce_avg(sh_ctx* c, float* buf, int64_t n, cudaStream_t st, const char* what) {
+  if (c->host_coll) return coll_host(c, kAllReduceAvg, buf, n, 0, n, nullptr, st);
+  if (!c->use_nccl) return SH_OK;  // SH_FLAG_TEST_NO_COLLECTIVE: identical data, the average is the identity
+  return nccl_check(c, g_nccl.AllReduce(buf, buf, n, ncclFloat, ncclAvg, c->nccl, st), what);
+}
+
+// Host layer x with a shared store: rank r offloads and CPU-updates only its slice [slo, shi), so it
+// needs only that slice of the average -- a reduce-scatter (half the NVLink bytes of an all-reduce,
+// NEXT-1).  In place: slice r of the W*cs-element buffer receives the result (NCCL's in-place form).
+sh_status coll_reduce_scatter_avg(sh_ctx* c, float* buf, int x, cudaStream_t st) {
+  const int64_t n = c->lay[x].n_pad, cs = align_up((n + c->W - 1) / c->W, kPad);
+  if (c->host_coll) return coll_host(c, kReduceScatterAvg, buf, n, c->slo[x], c->shi[x], nullptr, st);
+  if (!c->use_nccl) return SH_OK;
+  return nccl_check(c, g_nccl.ReduceScatter(buf, buf + (int64_t)c->rank * cs, (size_t)cs, ncclFloat, ncclAvg,
+                                            c->nccl, st),
+                    "ncclReduceScatter(layer grads)");
+}
+
+// Reduce-scattered host layers leave each rank with the sum of squares of its slice only: gather the
+// per-rank partials and fold them in rank order (identical on every rank) before the norm.
+sh_status coll_fold_partials(sh_ctx* c, cudaStream_t st) {
+  if (!c->rs_host) return SH_OK;
+  const int n = c->L + 1;
+  sh_status r = SH_OK;
+  if (c->host_coll)
+    r = coll_host(c, kAllGatherF64, c->partials, n, 0, n, c->partials_all, st);
+  else
+    r = nccl_check(c, g_nccl.AllGather(c->partials, c->partials_all, (size_t)n, ncclFloat64, c->nccl, st),
+                   "ncclAllGather(norm partials)");
+  if (r != SH_OK) return r;
+  CKC(c, kern::fold_partials(c->partials_all, c->W, n, c->w, c->partials, st));
+  return SH_OK;
+}
+
 }  // namespace
 
 // =============================================================================== C ABI
@@ -1696,8 +1906,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   }
   const int W = cfg->world_size < 1 ? 1 : cfg->world_size;
   const bool dp = W > 1 || (cfg->flags & SH_FLAG_TEST_DP_PATH);
-  if (dp && ((!cfg->nccl_unique_id && !(cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE)) || cfg->rank < 0 ||
-             cfg->rank >= W)) {
+  const bool test_coll = cfg->flags & (SH_FLAG_TEST_NO_COLLECTIVE | SH_FLAG_TEST_HOST_COLLECTIVE);
+  if (dp && ((!cfg->nccl_unique_id && !test_coll) || cfg->rank < 0 || cfg->rank >= W)) {
     set_error("sh_init: world_size > 1 needs nccl_unique_id and 0 <= rank < world_size");
     return SH_ERR_INVALID;
   }
@@ -1713,7 +1923,15 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->rank = cfg->rank;
   c->dp = dp;
   c->no_collective = dp && (cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE);
+  c->host_coll = dp && !c->no_collective && (cfg->flags & SH_FLAG_TEST_HOST_COLLECTIVE);
+  c->use_nccl = dp && !c->no_collective && !c->host_coll;
   c->shared = dp && cfg->shm_name && cfg->shm_name[0];
+  c->rs_host = c->shared && (c->use_nccl || c->host_coll);
+  if (c->host_coll && (!c->shared || W > kMaxHostCollRanks)) {
+    set_error("sh_init: SH_FLAG_TEST_HOST_COLLECTIVE needs shm_name (the shared segment) and world_size <= %d",
+              kMaxHostCollRanks);
+    return SH_ERR_INVALID;
+  }
   if (c->shared) c->shm_name = cfg->shm_name;
   c->bf16 = cfg->precision == SH_BF16_MIXED;
   c->cb = c->bf16 ? 2 : 4;
@@ -1757,7 +1975,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     CKC(c.get(), cudaEventCreateWithFlags(&c->ev_norm[i], cudaEventDisableTiming));
   }
   if (dp) CKC(c.get(), cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
-  if (dp && !c->no_collective) {
+  if (c->use_nccl) {
     if (!g_nccl.load()) {
       set_error("sh_init: world_size > 1 but libnccl.so.2 cannot be loaded");
       return SH_ERR_UNSUPPORTED;
@@ -1768,7 +1986,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     if (s != SH_OK) return s;
   }
   c->slice_fetch = dp && (cfg->flags & SH_FLAG_SLICE_FETCH) && cfg->shm_name && cfg->shm_name[0];
-  if (c->slice_fetch && !c->no_collective) {
+  if (c->slice_fetch && c->use_nccl) {
     if (!g_nccl.AllGather || !g_nccl.CommSplit) {
       set_error("sh_init: SH_FLAG_SLICE_FETCH needs ncclAllGather and ncclCommSplit");
       return SH_ERR_UNSUPPORTED;
@@ -1860,6 +2078,14 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       c->shi[x] = n;
     }
   }
+  if (c->host_coll) {  // contribution segment [W][hc_count] + a private result buffer
+    c->hc_count = align_up(std::max({(int64_t)W * c->cs_max, c->res.n_pad, 2 * (int64_t)(c->L + 1)}), 1024);
+    c->hc_bytes = align_up((int64_t)W * c->hc_count * 4, 1 << 21);
+    char* p = nullptr;
+    sh_status st = host_block_alloc(c->hc_bytes, c->n_threads, &p);
+    if (st != SH_OK) return st;
+    c->hc_tmp = reinterpret_cast<float*>(p);
+  }
   if (c->shared) {
     // control block: rank 0 creates it, the others wait for it; then every layer segment
     c->ctl_bytes = align_up(sizeof(ShmCtl) + 16 * (int64_t)c->L, 4096);
@@ -1869,6 +2095,11 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       if (st != SH_OK) return st;
       std::memset(p, 0, c->ctl_bytes);
       c->ctl = reinterpret_cast<ShmCtl*>(p);
+      if (c->host_coll) {
+        sh_status st = shm_map(c.get(), shm_path(c.get(), "hc"), c->hc_bytes, true, &p, true);
+        if (st != SH_OK) return st;
+        c->hc_seg = reinterpret_cast<float*>(p);
+      }
       for (int x = 0; x < c->L; ++x) {
         sh_status st2 = ensure_host_layer(c.get(), x);
         if (st2 != SH_OK) return st2;
@@ -1891,6 +2122,11 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
         }
         usleep(2000);
       }
+      if (c->host_coll) {
+        sh_status st = shm_map(c.get(), shm_path(c.get(), "hc"), c->hc_bytes, false, &p, true);
+        if (st != SH_OK) return st;
+        c->hc_seg = reinterpret_cast<float*>(p);
+      }
       for (int x = 0; x < c->L; ++x) {
         sh_status st2 = ensure_host_layer(c.get(), x);
         if (st2 != SH_OK) return st2;
@@ -1899,6 +2135,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     if (!shm_barrier(c.get(), 0, "shared store mapping")) return check_failed(c.get());
     if (c->rank == 0) {  // every rank has it mapped: remove the names (mappings persist)
       shm_unlink(shm_path(c.get(), "ctl").c_str());
+      if (c->host_coll) shm_unlink(shm_path(c.get(), "hc").c_str());
       for (int x = 0; x < c->L; ++x) shm_unlink(shm_path(c.get(), "L", x).c_str());
     }
   } else {
@@ -1933,6 +2170,14 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     }
     CKC(c.get(), cudaMemset(d, 0, nd * 8 + 64));
     c->partials = d;
+    if (c->rs_host) {
+      if (cudaMalloc(&c->partials_all, 8 * (int64_t)W * (c->L + 1)) != cudaSuccess) {
+        cudaGetLastError();
+        set_error("sh_init: cudaMalloc of the gathered norm partials failed");
+        return SH_ERR_OOM_DEVICE;
+      }
+      CKC(c.get(), cudaMemset(c->partials_all, 0, 8 * (int64_t)W * (c->L + 1)));
+    }
     c->scratch_cs = d + (c->L + 1);
     c->scratch_comm = c->scratch_cs + kern::kSumsqMaxBlocks + 1;
     c->scratch_d2h = c->scratch_comm + kern::kSumsqMaxBlocks + 1;
@@ -2170,6 +2415,7 @@ sh_status sh_forward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_param
         ProfSet& P = c->prof[c->step & 1];
         prof_reset(c, P, c->step);
         CKC(c, cudaEventRecord(P.t0, c->cs));
+        CKC(c, cudaLaunchHostFunc(c->cs, t0_cb, &P));
         P.rec_t0 = true;
       }
       CKC(c, cudaMemsetAsync(c->res_grad, 0, 4 * c->res.n_pad, c->cs));
@@ -2244,7 +2490,11 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       CKC(c, cudaStreamWaitEvent(c->cs, c->ev_grad_free[s], 0));
       c->gradfree_waited[s] = gen;
     }
-    CKC(c, cudaMemsetAsync(gdst, 0, 4 * c->lay[x].n_pad, c->cs));
+    // (a reduce-scattered host layer spans W equal slices: zero the padding past n_pad too)
+    const int64_t zn = c->rs_host && !c->is_g(x)
+                           ? std::max(c->lay[x].n_pad, (int64_t)c->W * align_up((c->lay[x].n_pad + c->W - 1) / c->W, kPad))
+                           : c->lay[x].n_pad;
+    CKC(c, cudaMemsetAsync(gdst, 0, 4 * zn, c->cs));
     for (float* xg : c->xgrad) CKC(c, cudaMemsetAsync(xg, 0, 4 * c->lay[x].n_pad, c->cs));
     c->cur_gdst = gdst;
     if (ProfSet* P = cur_prof(c)) CKC(c, cudaEventRecord(P->bp0[x], c->cs));
@@ -2285,11 +2535,8 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       if (c->dp) {
         CKC(c, cudaEventRecord(c->ev_gbuf_ready[b], c->cs));
         CKC(c, cudaStreamWaitEvent(c->comm, c->ev_gbuf_ready[b], 0));
-        if (!c->no_collective) {
-          st = nccl_check(c, g_nccl.AllReduce(gb, gb, n, ncclFloat, ncclAvg, c->nccl, c->comm),
-                          "ncclAllReduce(layer grads)");
-          if (st != SH_OK) return st;
-        }
+        st = coll_allreduce_avg(c, gb, n, c->comm, "ncclAllReduce(layer grads)");
+        if (st != SH_OK) return st;
         CKC(c, kern::sumsq(gb, n, c->scratch_comm, c->partials + x, c->comm));
       } else {
         if (P) CKC(c, cudaEventRecord(P->k30[x], c->cs));
@@ -2327,13 +2574,18 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       // data parallel: average this layer's grads across ranks before the offload (K-e)
       CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
       CKC(c, cudaStreamWaitEvent(c->comm, c->ev_grad_done[s], 0));
-      if (!c->no_collective) {
-        st = nccl_check(c, g_nccl.AllReduce(c->slot_grad(s), c->slot_grad(s), n, ncclFloat, ncclAvg, c->nccl,
-                                            c->comm),
-                        "ncclAllReduce(layer grads)");
+      if (c->rs_host && !c->is_g(x)) {
+        // host layer, shared store: this rank offloads only its slice -> reduce-scatter, and the
+        // K3 covers the slice (the per-rank partials are folded at sh_step)
+        st = coll_reduce_scatter_avg(c, c->slot_grad(s), x, c->comm);
         if (st != SH_OK) return st;
+        CKC(c, kern::sumsq(c->slot_grad(s) + c->slo[x], c->shi[x] - c->slo[x], c->scratch_comm, c->partials + x,
+                           c->comm));
+      } else {
+        st = coll_allreduce_avg(c, c->slot_grad(s), n, c->comm, "ncclAllReduce(layer grads)");
+        if (st != SH_OK) return st;
+        CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_comm, c->partials + x, c->comm));
       }
-      CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_comm, c->partials + x, c->comm));
       CKC(c, cudaEventRecord(c->ev_reduced[s], c->comm));
       grads_ready = c->ev_reduced[s];
     } else if (c->is_g(x)) {  // clip mode: grads stay in the slot until sh_step's K2
@@ -2483,13 +2735,11 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
     // resident grads: average too, on the comm stream after the caller's embedding backward
     CKC(c, cudaEventRecord(c->ev_cs_mark, c->cs));
     CKC(c, cudaStreamWaitEvent(c->comm, c->ev_cs_mark, 0));
-    if (!c->no_collective) {
-      st = nccl_check(c, g_nccl.AllReduce(c->res_grad, c->res_grad, c->res.n_pad, ncclFloat, ncclAvg, c->nccl,
-                                          c->comm),
-                      "ncclAllReduce(resident grads)");
-      if (st != SH_OK) return st;
-    }
+    st = coll_allreduce_avg(c, c->res_grad, c->res.n_pad, c->comm, "ncclAllReduce(resident grads)");
+    if (st != SH_OK) return st;
     CKC(c, kern::sumsq(c->res_grad, c->res.n_pad, c->scratch_comm, c->partials + L, c->comm));
+    st = coll_fold_partials(c, c->comm);
+    if (st != SH_OK) return st;
     CKC(c, cudaEventRecord(c->ev_comm_done, c->comm));
     CKC(c, cudaStreamWaitEvent(c->cs, c->ev_comm_done, 0));
   } else {
@@ -2959,8 +3209,16 @@ sh_status sh_destroy(sh_ctx* c) {
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s})
     if (s) cudaStreamSynchronize(s);
   if (c->cs) cudaStreamSynchronize(c->cs);
-  if (c->nccl_fetch) g_nccl.CommDestroy(c->nccl_fetch);
-  if (c->nccl) g_nccl.CommDestroy(c->nccl);
+  if (!c->nccl_aborted.load()) {  // an aborted communicator is already freed
+    if (c->nccl_fetch) g_nccl.CommDestroy(c->nccl_fetch);
+    if (c->nccl) g_nccl.CommDestroy(c->nccl);
+  }
+  if (c->partials_all) cudaFree(c->partials_all);
+  if (c->hc_seg) {
+    cudaHostUnregister(c->hc_seg);
+    munmap(c->hc_seg, c->hc_bytes);
+  }
+  host_block_free(reinterpret_cast<char*>(c->hc_tmp), c->hc_bytes);
   for (int x = 0; x < c->L; ++x) free_g(c, x);
   for (float* p : c->gbuf) cudaFree(p);
   for (float* p : c->xgrad) cudaFree(p);

@@ -394,6 +394,16 @@ __global__ void norm_finalize_kernel(const double* __restrict__ partials, int n,
   *coef_out = (float)c;
 }
 
+__global__ void fold_partials_kernel(const double* __restrict__ all, int world, int n, int w_g,
+                                     double* __restrict__ out) {
+  for (int x = threadIdx.x; x < n; x += blockDim.x) {
+    double s = all[x];
+    if (x >= w_g && x < n - 1)
+      for (int r = 1; r < world; ++r) s += all[(int64_t)r * n + x];  // rank order: fixed
+    out[x] = s;
+  }
+}
+
 int g_sm_count = 0;
 __host__ std::atomic<int64_t>& launch_counter() {
   static std::atomic<int64_t> n{0};
@@ -522,5 +532,15 @@ cudaError_t norm_finalize(const double* partials, int n, double max_norm, double
   return cudaGetLastError();
 }
 
+}  // namespace kern
+}  // namespace sh
+
+namespace sh {
+namespace kern {
+cudaError_t fold_partials(const double* all, int world, int n, int w_g, double* out, cudaStream_t st) {
+  launch_counter()++;
+  fold_partials_kernel<<<1, 256, 0, st>>>(all, world, n, w_g, out);
+  return cudaGetLastError();
+}
 }  // namespace kern
 }  // namespace sh

@@ -77,6 +77,10 @@ struct K4Args {
   float inv_k;
 };
 cudaError_t exec_reduce(const K4Args& a, cudaStream_t st);
+// Data parallel with reduce-scattered host layers: out[x] = all[0][x] for x < w_g (GPU-optimised
+// layers, full gradients on every rank) and x = n-1 (resident set); out[x] = sum_r all[r][x] in
+// rank order for the host layers (each rank holds the sum of squares of its slice).
+cudaError_t fold_partials(const double* all, int world, int n, int w_g, double* out, cudaStream_t st);
 int sm_count();
 int64_t launches();
 }  // namespace kern

@@ -24,6 +24,7 @@ SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_H
     SH_FLAG_TEST_NO_COLLECTIVE, SH_FLAG_SLICE_FETCH, SH_FLAG_DELAY_INJECT, SH_FLAG_DECOUPLE, SH_FLAG_SPILL_EVICT, \
     SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS, SH_FLAG_ABLATE_ALLOC, SH_FLAG_GROW_LANDING, SH_FLAG_FILL_GPU, \
     SH_FLAG_LATE_SHADOW = 1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192, 16384, 32768, 65536
+SH_FLAG_TEST_HOST_COLLECTIVE = 1 << 17
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
@@ -104,7 +105,8 @@ class TraceEvent(C.Structure):
     _fields_ = [("kind", C.c_int32), ("layer", C.c_int32), ("start_ms", C.c_double), ("end_ms", C.c_double)]
 
 
-TRACE_KINDS = ("fp", "bp", "h2d_fp", "h2d_bp", "d2h_grad", "k1_stage", "k3_sumsq", "k2_adamw")
+TRACE_KINDS = ("fp", "bp", "h2d_fp", "h2d_bp", "d2h_grad", "k1_stage", "k3_sumsq", "k2_adamw", "cpu_adam",
+               "h2d_wait_cpu")
 
 
 class AdamScalars(C.Structure):

@@ -1,0 +1,125 @@
+"""Data parallel W = 2 with DIFFERENT data per rank, on the one GPU this environment grants (VERDICT r01
+#1d/e).
+
+Two processes, bootstrapped with torch.distributed (gloo, 127.0.0.1), drive sh_init(world_size=2)
+with one shared /dev/shm host store and SH_FLAG_TEST_HOST_COLLECTIVE: the per-layer gradient
+all-reduce (GPU-optimised layers), the reduce-scatter (host layers: rank r offloads and CPU-updates
+only its slice), the resident all-reduce and the all-gather of the per-rank norm partials all run
+through the shared host segment, summed in rank order.  Rank r trains on synth.tokens(t + 1000 r).
+
+Bars:
+  (a) both ranks end bitwise identical (params, m, v, compute copies);
+  (b) they match the fp64 oracle trained on the GLOBAL batch (both micro-batches, reading R13: the
+      mean over all sequences) -- per-tensor update delta, K-bias bound, per-unit max error;
+  (c) the mean of the ranks' losses equals the oracle's global loss, and the gradient norm (folded
+      from the per-rank slice partials) equals the oracle's.
+"""
+import os
+import socket
+import uuid
+
+import numpy as np
+import pytest
+import torch.multiprocessing as mp
+
+from tests._common import (BF16_TOL, DELTA_BF16, DELTA_FP32, FP32_TOL, TINY, check_vs_oracle, oracle_run)
+
+pytestmark = pytest.mark.gpu
+sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
+STEPS = 3
+WORLD = 2
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _rank(rank, port, window, precision, clip, extra_flags, q):
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_sc_sunwqyhxw22_b200 import trainer as T
+    from tests._common import engine_state
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), SH_WAIT_TIMEOUT_S="120")
+    dist.init_process_group("gloo", rank=rank, world_size=WORLD)
+    name = [f"shdp_{uuid.uuid4().hex[:12]}" if rank == 0 else None]
+    dist.broadcast_object_list(name, 0)  # the bootstrap bench.py does with the NCCL id
+    mc = T.ModelConfig(TINY["L"], TINY["h"], TINY["nh"], TINY["s"], TINY["V"])
+    tr = T.StrongholdTrainer(mc, batch=TINY["b"], window=window, precision=precision, world_size=WORLD, rank=rank,
+                             shm_name=name[0], cpu_threads=2, max_grad_norm=clip,
+                             flags=sh.SH_FLAG_TEST_HOST_COLLECTIVE | extra_flags)
+    losses, norms = [], []
+    for t in range(STEPS):
+        tr.set_tokens(synth.tokens(t + 1000 * rank, TINY["b"], TINY["s"], TINY["V"]))
+        norms.append(tr.step_device(want_norm=True))
+        losses.append(tr.loss())
+    st = engine_state(tr)
+    layers = [tr.read_layer_tensors(i) for i in range(mc.n_layers)]
+    res = tr.read_layer_tensors(-1)
+    stats = tr.engine.stats()
+    tr.close()
+    dist.destroy_process_group()
+    q.put((rank, {k: [[a.tobytes() for a in u] if isinstance(u, list) else u.tobytes() for u in v]
+                  for k, v in st.items()}, layers, res, losses, norms, stats["d2h_bytes"]))
+
+
+def _run(window, precision, clip=0.0, extra_flags=0):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rank, args=(r, port, window, precision, clip, extra_flags, q)) for r in range(WORLD)]
+    for p in procs:
+        p.start()
+    out = sorted([q.get(timeout=300) for _ in range(WORLD)], key=lambda x: x[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    return out
+
+
+class _Tr:  # check_vs_oracle reads through a trainer-like object
+    def __init__(self, layers, res):
+        self._l, self._r = layers, res
+        self.mc = type("mc", (), {"n_layers": len(layers)})
+
+    def read_layer_tensors(self, i):
+        return self._r if i < 0 else self._l[i]
+
+
+@pytest.fixture(scope="module")
+def oracle_global():
+    return {clip: oracle_run(TINY, STEPS, world=WORLD, max_grad_norm=clip) for clip in (0.0, 0.5)}
+
+
+@pytest.mark.parametrize("window,precision,clip,extra", [
+    (2, sh.SH_FP32, 0.0, 0),                      # G layers 0-1 all-reduced, host layers 2-3 reduce-scattered
+    (0, sh.SH_FP32, 0.0, 0),                      # every layer offloaded
+    (TINY["L"], sh.SH_FP32, 0.0, 0),              # all GPU-optimised (no host layer)
+    (1, sh.SH_FP32, 0.5, 0),                      # clipping: the coefficient needs the folded global norm
+    (1, sh.SH_BF16_MIXED, 0.0, 0),
+    (1, sh.SH_BF16_MIXED, 0.0, sh.SH_FLAG_SLICE_FETCH | sh.SH_FLAG_FETCH_FP32),
+])
+def test_dp_two_ranks_different_data_vs_oracle(oracle_global, window, precision, clip, extra):
+    st, olosses, onorms = oracle_global[clip]
+    out = _run(window, precision, clip, extra)
+    (_, s0, l0, r0, loss0, n0, d0), (_, s1, l1, r1, loss1, n1, d1) = out
+    assert s0 == s1, "the two ranks differ"                                    # (a)
+    fp32 = precision == sh.SH_FP32
+    check_vs_oracle(_Tr(l0, r0), st, DELTA_FP32 if fp32 else DELTA_BF16, FP32_TOL if fp32 else BF16_TOL,
+                    f"dp2_w{window}_{'fp32' if fp32 else 'bf16'}_clip{clip}_x{extra}")  # (b)
+    rel = 1e-5 if fp32 else 2e-2
+    for a, b, o in zip(loss0, loss1, olosses):                                # (c)
+        assert abs(0.5 * (a + b) - o) <= rel * abs(o), (loss0, loss1, olosses)
+    assert n0 == n1
+    for a, o in zip(n0, onorms):
+        assert abs(a - o) <= (1e-4 if fp32 else 2e-2) * o, (n0, onorms)
+    if window < TINY["L"]:  # each rank offloads its slice of every host layer, together each layer once
+        import synth
+        n_pad = sum((int(np.prod(sh_)) + 127) // 128 * 128 for sh_ in synth.layer_shapes(TINY["h"]))
+        assert d0 > 0 and d1 > 0 and d0 + d1 == 4 * n_pad * (TINY["L"] - window) * STEPS
+    assert not any(f.startswith("shdp_") and "hc" in f for f in os.listdir("/dev/shm"))

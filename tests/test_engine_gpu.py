@@ -1,16 +1,18 @@
 """End-to-end parity of the CUDA path (engine + GPT driver) on the tiny configuration.
 
-Bars (BASELINE.json north_star, R16):
+Bars (BASELINE.json north_star; R16, R24; tests/_common.py):
   * windowed == all-resident (w = L) BITWISE for every window 0..L: params, m, v, compute copies
-  * vs the fp64 oracle after 3 steps: per offload unit ∞-norm relative error <= 1e-4 (fp32),
-    <= 2e-2 (bf16 mixed); loss per step within 1e-5 relative (fp32)
+  * vs the fp64 oracle after 3 steps, per TENSOR update delta ||dx - dy|| / ||dy|| <= 1e-3 (fp32),
+    <= 5e-2 (bf16 mixed); K bias bounded by the Adam step bound; per offload unit max|x-y|/max|y|
+    <= 1e-4 / 2e-2; loss per step within 1e-5 relative (fp32)
+  * step-1 gradients per tensor vs the oracle (tests/test_parity_l8_gpu.py)
 """
 import numpy as np
 import pytest
 
 import synth
-from tests._common import (BF16_TOL, FP32_TOL, TINY, engine_run, engine_state, oracle_run, states_bitwise_equal,
-                           unit_errors)
+from tests._common import (BF16_TOL, DELTA_BF16, DELTA_FP32, FP32_TOL, TINY, check_vs_oracle, engine_run,
+                           engine_state, oracle_run, states_bitwise_equal)
 
 pytestmark = pytest.mark.gpu
 
@@ -29,20 +31,12 @@ def oracle_clip():
     return oracle_run(TINY, STEPS, max_grad_norm=0.5)
 
 
-def _errors(tr, st):
-    L = tr.mc.n_layers
-    layers = [tr.read_layer_tensors(i) for i in range(L)]
-    res = tr.read_layer_tensors(-1)
-    return unit_errors(layers, res, st)
-
-
 @pytest.mark.parametrize("window", [TINY["L"], 2])
 def test_fp32_vs_oracle(oracle_noclip, window):
     st, olosses, onorms = oracle_noclip
     tr, losses, norms = engine_run(TINY, STEPS, window, sh.SH_FP32)
     try:
-        errs = _errors(tr, st)
-        assert max(errs.values()) <= FP32_TOL, errs
+        check_vs_oracle(tr, st, DELTA_FP32, FP32_TOL, f"tiny_fp32_w{window}")
         for a, b in zip(losses, olosses):
             assert abs(a - b) <= 1e-5 * abs(b), (losses, olosses)
         for a, b in zip(norms, onorms):
@@ -57,8 +51,7 @@ def test_bf16_vs_oracle(oracle_noclip, attention):
     tr, losses, _ = engine_run(TINY, STEPS, 2, sh.SH_BF16_MIXED, attention=attention)
     assert (tr.flash is not None) == (attention == "flash")
     try:
-        errs = _errors(tr, st)
-        assert max(errs.values()) <= BF16_TOL, errs
+        check_vs_oracle(tr, st, DELTA_BF16, BF16_TOL, f"tiny_bf16_{attention}")
         for a, b in zip(losses, olosses):
             assert abs(a - b) <= 2e-2 * abs(b)
     finally:
@@ -70,8 +63,9 @@ def test_clip_fp32_vs_oracle(oracle_clip):
     assert onorms[0] > 0.5  # clipping is active in this run
     tr, losses, norms = engine_run(TINY, STEPS, 1, sh.SH_FP32, max_grad_norm=0.5)
     try:
-        errs = _errors(tr, st)
-        assert max(errs.values()) <= FP32_TOL, errs
+        check_vs_oracle(tr, st, DELTA_FP32, FP32_TOL, "tiny_fp32_clip")
+        for a, b in zip(norms, onorms):
+            assert abs(a - b) <= 1e-4 * b, (norms, onorms)
     finally:
         tr.close()
 

@@ -1,0 +1,68 @@
+"""Engine vs oracle: element-wise step-1 gradients and the L = 8, h = 512 configuration (SURVEY
+§8(c) "Engine vs oracle -- tolerance bar on the tiny config and an L=8, h=512 config"; T6 of §4).
+
+Gradients (the caller's GEMMs write them; the engine hands them to K3 / the offload / K2) are read
+back per tensor after ONE step -- GPU-optimised layers from their dedicated buffers
+(SH_FLAG_KEEP_GRADS), host layers from the landing buffers, the resident set from its grad buffer
+-- and compared with the oracle's element by element: ||gx - gy||_2 / ||gy||_2 per tensor.  fp32:
+the GPT driver runs pure fp32 GEMMs (no TF32) with fp32 accumulation, the measured error is ~1e-6,
+the bar 1e-4.  bf16 mixed: bf16 weights and activations (8-bit mantissa, rounding 2^-9 per value)
+through ~20 chained ops give a few 1e-3 per tensor; the bar is 5e-2, the same as the update bar.
+"""
+import pytest
+
+from tests._common import (BF16_TOL, DELTA_BF16, DELTA_FP32, FP32_TOL, L8, TINY, check_grads, check_vs_oracle,
+                           engine_run, oracle_run)
+
+pytestmark = pytest.mark.gpu
+sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
+
+GRAD_FP32 = 1e-4
+GRAD_BF16 = 5e-2
+KB_FP32 = 1e-4   # K-bias gradient / max bias gradient: rounding noise only
+KB_BF16 = 5e-2
+
+
+@pytest.fixture(scope="module")
+def tiny_g1():
+    return oracle_run(TINY, 1, keep_grads=True)[3]
+
+
+@pytest.fixture(scope="module")
+def l8_ref():
+    return oracle_run(L8, 3, keep_grads=True)
+
+
+@pytest.mark.parametrize("precision,window", [(sh.SH_FP32, 2), (sh.SH_BF16_MIXED, 2), (sh.SH_FP32, 0)])
+def test_tiny_step1_grads_vs_oracle(tiny_g1, precision, window):
+    tr, _, _ = engine_run(TINY, 1, window, precision, flags=sh.SH_FLAG_KEEP_GRADS)
+    try:
+        fp32 = precision == sh.SH_FP32
+        check_grads(tr, tiny_g1, GRAD_FP32 if fp32 else GRAD_BF16, KB_FP32 if fp32 else KB_BF16,
+                    f"tiny_grads_{'fp32' if fp32 else 'bf16'}_w{window}")
+    finally:
+        tr.close()
+
+
+@pytest.mark.parametrize("precision", [sh.SH_FP32, sh.SH_BF16_MIXED])
+def test_l8_h512_vs_oracle(l8_ref, precision):
+    st, olosses, onorms, g1 = l8_ref
+    fp32 = precision == sh.SH_FP32
+    tag = "fp32" if fp32 else "bf16"
+    # window 3 of 8: layers 0-2 GPU-optimised (K2), 3-7 offloaded (CPU Adam), prefetch distance 3
+    tr, losses, norms = engine_run(L8, 1, 3, precision, flags=sh.SH_FLAG_KEEP_GRADS)
+    try:
+        check_grads(tr, g1, GRAD_FP32 if fp32 else GRAD_BF16, KB_FP32 if fp32 else KB_BF16, f"l8_grads_{tag}")
+    finally:
+        tr.close()
+    tr, losses, norms = engine_run(L8, 3, 3, precision)
+    try:
+        check_vs_oracle(tr, st, DELTA_FP32 if fp32 else DELTA_BF16, FP32_TOL if fp32 else BF16_TOL, f"l8_{tag}", cfg=L8)
+        rel = 1e-5 if fp32 else 2e-2
+        for a, b in zip(losses, olosses):
+            assert abs(a - b) <= rel * abs(b), (losses, olosses)
+        if fp32:
+            for a, b in zip(norms, onorms):
+                assert abs(a - b) <= 1e-4 * b, (norms, onorms)
+    finally:
+        tr.close()
