@@ -55,7 +55,8 @@ CPU_HARD_DEFAULT = {"c3", "c4", "c4max"}   # autotune with the eq. 3 CPU-through
 # growth, GPU set filling the HBM a decoupled ring leaves, late bf16 host shadows (C4: 7.30 -> 7.92
 # samples/s, profiles/r01_bench_default_c4_v3.json vs r01_bench_c4_tuned_coupled.json)
 TUNED_DEFAULT = {"c3", "c4"}
-SETTLE_STEPS = 4  # untimed steps after the autotuner's window change (before the K timed steps)
+SETTLE_MAX = 10   # at most this many untimed settle steps after the autotuner's window change
+RUNS = 3          # the K timed steps are timed as RUNS consecutive segments (median / geomean reported)
 
 
 def mem_available() -> int:
@@ -86,6 +87,11 @@ METRIC = "samples/s at max trainable size per B200; host-link GB/s vs peak"
 PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
 PROBE_D2H_GBS = 57.01
 PROBE_HOST_TRIAD_GBS = 143.43  # profiles/r01_probe_box.json, 16-thread STREAM triad (no RFO counted)
+# profiles/r02_host_mix.json (tools/probe_host_mix.py): the engine's real host-DRAM mix -- the CPU AdamW
+# (16 B read + 14 B written per element) running concurrently with H2D + D2H DMA on pinned memory.  The
+# highest total host-DRAM throughput of that mix over thread counts (T14: Adam 115.9 + H2D 34.4 + D2H
+# 34.4 GB/s); the 16-thread STREAM triad alone reaches 143.
+PROBE_HOST_MIX_GBS = 184.7
 
 
 def measured_peaks():
@@ -163,12 +169,13 @@ def k2_traffic(elems_per_launch: float):
     return per * elems_per_launch
 
 
-def oracle_sample(L, h, nh, s, V, seed=1234):
-    """Bounded CPU-oracle sample of the workload: one block fwd+bwd and its AdamW, plus the head
-    (fwd+bwd) and the resident AdamW, at batch 1; extrapolated to one sample of the full model."""
+def oracle_sample(L, h, nh, s, V, b, seed=1234):
+    """Bounded CPU-oracle sample of the workload: one block's fwd+bwd at batch 1 and its AdamW, the
+    head's fwd+bwd at batch 1 and the resident AdamW, each timed once.  One training step of the full
+    model at batch b costs L (b t_fb + t_adam) + b t_head + t_adam_res (the AdamW runs once per STEP,
+    not per sample); returns (seconds per step, parts)."""
     from oracle import gpt_oracle as O
     import synth
-    cfg = O.GPTConfig(1, h, nh, s, V)
     P = [a.astype(np.float64) for a in synth.init_layer(seed, 0, L, h)]
     R = [a.astype(np.float64) for a in synth.init_resident(seed, V, s, h)]
     tok = synth.tokens(0, 1, s, V)
@@ -177,16 +184,26 @@ def oracle_sample(L, h, nh, s, V, seed=1234):
     t0 = time.perf_counter()
     y, cache = O.block_fwd(x, P, nh)
     dx, grads = O.block_bwd(np.ones_like(y) * 1e-3, cache, P)
+    t_fb = time.perf_counter() - t0
+    t0 = time.perf_counter()
     for k, (p, g) in enumerate(zip(P, grads)):
         O.adamw_update(p, g, np.zeros_like(p), np.zeros_like(p), 1, opt, p.ndim == 2)
-    t_layer = time.perf_counter() - t0
+    t_adam = time.perf_counter() - t0
     t0 = time.perf_counter()
     O.forward_backward(O.GPTConfig(0, h, nh, s, V), [], R, tok)
+    t_head = time.perf_counter() - t0
+    t0 = time.perf_counter()
     for p in R:
         O.adamw_update(p, p, np.zeros_like(p), np.zeros_like(p), 1, opt, True)
-    t_head = time.perf_counter() - t0
-    per_sample = L * t_layer + t_head
-    return per_sample, t_layer, t_head
+    t_adam_res = time.perf_counter() - t0
+    per_step = L * (b * t_fb + t_adam) + b * t_head + t_adam_res
+    return per_step, dict(t_fb=t_fb, t_adam=t_adam, t_head=t_head, t_adam_res=t_adam_res)
+
+
+def oracle_desc(L, b, parts):
+    return (f"one block fwd+bwd at batch 1 ({parts['t_fb']:.2f} s) and its AdamW ({parts['t_adam']:.2f} s), the head "
+            f"fwd+bwd at batch 1 ({parts['t_head']:.2f} s) and the resident AdamW ({parts['t_adam_res']:.2f} s), numpy "
+            f"fp64, extrapolated to one step: L x (b x fwd+bwd + AdamW) + b x head + resident AdamW, L={L}, b={b}")
 
 
 def blas_threads():
@@ -210,20 +227,19 @@ def run_reference(args, cfgname):
         return
     times = []
     for i in range(args.warmup + args.steps):
-        per_sample, tl, th = oracle_sample(L, h, nh, s, V)
+        per_step, parts = oracle_sample(L, h, nh, s, V, b)
         if i >= args.warmup:
-            times.append(per_sample)
+            times.append(per_step)
     per = float(np.mean(times))
-    val = 1.0 / per
+    val = b / per
     line = {"impl": "reference", "metric": METRIC, "value": val,
             "unit": "samples/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": per * 1e3 * b, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "ms_per_step": per * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic",
             "config": {"workload": cfgname, "description": desc, "layers": L, "hidden": h, "heads": nh,
                        "batch_per_gpu": b, "seq": s, "vocab": V},
             "cpu_baseline": {"value": val, "unit": "samples/s", "cores": blas_threads(), "kind": "oracle",
-                             "sample": "per step: one block fwd+bwd+AdamW and the head at batch 1 (numpy fp64), "
-                                       f"extrapolated x{L} layers"},
+                             "sample": "per timed step: " + oracle_desc(L, b, parts)},
             "e2e": {"value": val, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -384,32 +400,63 @@ def main():
         # an autotuned run changes its window (and with the extensions its landing ring and host
         # shadows) at the end of warm-up step W; S more untimed steps let the new configuration reach
         # its steady state (GPU-set uploads, ring refill) so the timed steps measure it, not the switch
-        S = SETTLE_STEPS if window == -1 else 0
-        host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + S + K)])
+        S_max = SETTLE_MAX if window == -1 else 0
+        host = torch.stack([torch.from_numpy(synth.tokens(t + 1000 * rank, b, s, V)) for t in range(W + S_max + K)])
         host = host.pin_memory()
         dev = host.to(f"cuda:{local}")
         step_fn = tr.forward_only if args.fp_only else tr.step_device
-        for t in range(W + S):
+
+        def one(t):
             with torch.cuda.stream(tr.stream):  # ordered after the previous step's reads of tok_dev
                 tr.tok_dev.copy_(dev[t], non_blocking=True)
             step_fn()
+
+        def mark():
+            e = torch.cuda.Event(enable_timing=True)
+            e.record(tr.stream)
+            return e
+
+        for t in range(W):
+            one(t)
+        # settle (autotuned runs switch window / landing ring / shadows at the end of warm-up): untimed
+        # steps until two consecutive step times agree within 3 % -- step i's time is read once step
+        # i+1 is issued, so the host never starves the GPU to measure it
+        t = W
+        settle_ms = []
+        if S_max:
+            marks = [mark()]
+            while t < W + S_max:
+                one(t)
+                t += 1
+                marks.append(mark())
+                if len(marks) >= 3:
+                    marks[-2].synchronize()
+                    settle_ms.append(marks[-3].elapsed_time(marks[-2]))
+                    if len(settle_ms) >= 2 and abs(settle_ms[-1] - settle_ms[-2]) <= 0.03 * settle_ms[-2]:
+                        break
+        S = t - W
         tr.engine.synchronize()
         st0 = tr.engine.stats()
         l0 = sh.kernel_launches() + G.kernel_launches()
-        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        # K timed steps in R segments (the runs of the protocol: median / geomean over >= 3)
+        R = max(1, min(RUNS, K // 3))
+        bounds = [t + (K * r) // R for r in range(R + 1)]
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
         with ClockSampler(local) as clk:
-            ev0.record(tr.stream)
-            for t in range(W + S, W + S + K):
-                with torch.cuda.stream(tr.stream):
-                    tr.tok_dev.copy_(dev[t], non_blocking=True)
-                step_fn()
-            tr.engine.synchronize()
-            ev1.record(tr.stream)
+            seg = [mark()]
+            for r in range(R):
+                for tt in range(bounds[r], bounds[r + 1]):
+                    one(tt)
+                if r < R - 1:
+                    seg.append(mark())
+            tr.engine.synchronize()  # every copy and CPU update of the K steps
+            seg.append(mark())
             torch.cuda.synchronize()
-        ms = ev0.elapsed_time(ev1)
+        ms = seg[0].elapsed_time(seg[-1])
+        seg_ms = [seg[r].elapsed_time(seg[r + 1]) for r in range(R)]
+        seg_sps = [b * world * (bounds[r + 1] - bounds[r]) / (seg_ms[r] / 1e3) for r in range(R)]
         launches = sh.kernel_launches() + G.kernel_launches() - l0
         st1 = tr.engine.stats()
         loss = tr.loss()
@@ -420,8 +467,8 @@ def main():
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(tr.stream)
-            for t in range(W + S, W + S + K):
-                tr.step(host[t])  # public API: pinned host tokens -> H2D, step, loss -> host
+            for tt in range(W + S, W + S + K):
+                tr.step(host[tt])  # public API: pinned host tokens -> H2D, step, loss -> host
             tr.engine.synchronize()
             e1.record(tr.stream)
             torch.cuda.synchronize()
@@ -442,7 +489,7 @@ def main():
                 json.dump({"traceEvents": ev, "displayTimeUnit": "ms"}, f)
         tr.close()
         return dict(ms=ms, e2e_ms=e2e_ms, st0=st0, st1=st1, loss=loss, launches=launches, clocks=clk.summary(),
-                    init_s=t_init, prof=prof, st2=st2, attn=attn_used)
+                    init_s=t_init, prof=prof, st2=st2, attn=attn_used, seg_sps=seg_sps, settle_ms=settle_ms, S=S)
 
     r = run(w, not args.no_e2e)
     res = None
@@ -472,8 +519,12 @@ def main():
     st0, st1 = r["st0"], r["st1"]
     d = {k: st1[k] - st0[k] for k in ("h2d_bytes", "d2h_bytes", "h2d_busy_ms", "d2h_busy_ms",
                                       "h2d_profiled_bytes", "d2h_profiled_bytes", "cpu_adam_ms",
-                                      "cpu_adam_elems", "cpu_wait_ms", "k2_ms_sum", "k2_bytes_sum",
-                                      "k2_samples", "k3_ms_sum", "k3_bytes_sum", "k3_samples")}
+                                      "cpu_adam_elems", "cpu_adam_shadow_elems", "cpu_wait_ms", "k2_ms_sum",
+                                      "k2_bytes_sum", "k2_samples", "k3_ms_sum", "k3_bytes_sum", "k3_samples")}
+    # host-DRAM bytes of the CPU AdamW: 28 B/element (r p, m, v, g + w p, m, v), +2 for the elements
+    # whose layer also has a bf16 shadow (counted by the engine per element)
+    adam_bytes = 28 * d["cpu_adam_elems"] + 2 * d["cpu_adam_shadow_elems"]
+    host_dram_bytes = adam_bytes + d["h2d_bytes"] + d["d2h_bytes"]
     step_ms = ms / K
     samples = b * world * K / (ms / 1e3)
     peak, peak_kind = measured_peaks()
@@ -509,12 +560,20 @@ def main():
                             "policy": ("auto", "split", "local", "interleave", "none")[r["st1"]["numa_policy"]],
                             "gpu_node": r["st1"]["numa_gpu_node"], "pinned_workers": r["st1"]["numa_pinned_workers"],
                             "bound_bytes": r["st1"]["numa_bound_bytes"]},
-                   "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 else " + bf16 shadow"),
-                   "fetch": "fp32 master, K1 cast on GPU" if fetch32 else "bf16 shadow",
+                   "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 and not st1["shadow_layers"]
+                                                                     else " + bf16 shadow"),
+                   "fetch": ("bf16 shadow" if not fetch32 else
+                             f"bf16 shadow for {st1['shadow_layers']} of {L - st1['window']} host layers (late "
+                             "shadows), fp32 master + K1 cast on the GPU for the rest" if st1["shadow_layers"] else
+                             "fp32 master, K1 cast on GPU"),
                    "grad_landing_buffers": r["st1"]["landing_buffers"], "host_store_bytes": r["st1"]["host_bytes"],
                    "states_bytes_fp32_p_m_v": 12 * mc.n_params(),
                    "l2": "no flush: per-step traffic (GBs) >> 126 MB L2",
-                   "settle_steps": SETTLE_STEPS if w == -1 else 0},
+                   "settle_steps": r["S"], "settle_step_ms": r["settle_ms"]},
+        "runs": {"n": len(r["seg_sps"]), "samples_per_s": r["seg_sps"], "median": float(np.median(r["seg_sps"])),
+                 "geomean": float(np.exp(np.mean(np.log(r["seg_sps"])))),
+                 "note": "the K timed steps as consecutive segments of one process (the last one includes the "
+                         "drain of the CPU updates); value = all K steps"},
         "tokens_per_s": tokens_s,
         "model_tflops": tokens_s * flops_tok / 1e12,
         "final_loss": r["loss"],
@@ -537,23 +596,23 @@ def main():
                            if r["st2"]["last_step_ms"] > 0 else None},
         "cpu_adam": {"threads": st1["cpu_threads"], "elems_per_step": d["cpu_adam_elems"] / K,
                      "thread_ms_per_step": d["cpu_adam_ms"] / K,
-                     "dram_gbs": (28 if fetch32 or not prec else 30) * d["cpu_adam_elems"] / (d["cpu_adam_ms"] / 1e3 / st1["cpu_threads"]) / 1e9
+                     "dram_gbs": adam_bytes / (d["cpu_adam_ms"] / 1e3 / st1["cpu_threads"]) / 1e9
                      if d["cpu_adam_ms"] > 0 else None,
                      "prefetch_wait_ms_per_step": d["cpu_wait_ms"] / K,
                      "host_dram_triad_peak_gbs": PROBE_HOST_TRIAD_GBS,
-                     "note": "dram_gbs counts the AdamW's 30 B/param (28 without shadow) while its threads run; "
-                             "the copy engines' DMA shares the same host DRAM"},
+                     "note": "dram_gbs counts the AdamW's 28 B/param (+2 where a bf16 shadow is written) while its "
+                             "threads run; the copy engines' DMA shares the same host DRAM"},
         # whole-step host-DRAM roofline: the CPU AdamW's bytes (28 B/param fp32-fetch, 30 with the bf16
         # shadow: r p,m,v,g + w p,m,v [+ w shadow]) plus every DMA byte the copy engines move through
         # host DRAM, over the step time, against the probe's 16-thread triad
-        "host_dram": {"bytes_per_step": ((28 if fetch32 or not prec else 30) * d["cpu_adam_elems"]
-                                         + d["h2d_bytes"] + d["d2h_bytes"]) / K,
-                      "achieved_gbs": ((28 if fetch32 or not prec else 30) * d["cpu_adam_elems"]
-                                       + d["h2d_bytes"] + d["d2h_bytes"]) / (ms / 1e3) / 1e9,
-                      "peak_gbs": PROBE_HOST_TRIAD_GBS,
-                      "frac": ((28 if fetch32 or not prec else 30) * d["cpu_adam_elems"]
-                               + d["h2d_bytes"] + d["d2h_bytes"]) / (ms / 1e3) / 1e9 / PROBE_HOST_TRIAD_GBS,
-                      "peak_source": "profiles/r01_probe_box.json (STREAM triad, 16 threads)"},
+        "host_dram": {"bytes_per_step": host_dram_bytes / K,
+                      "bytes_per_host_param": host_dram_bytes / max(1, d["cpu_adam_elems"]),
+                      "achieved_gbs": host_dram_bytes / (ms / 1e3) / 1e9,
+                      "peak_gbs": PROBE_HOST_MIX_GBS,
+                      "frac": host_dram_bytes / (ms / 1e3) / 1e9 / PROBE_HOST_MIX_GBS,
+                      "triad_gbs": PROBE_HOST_TRIAD_GBS,
+                      "peak_source": "profiles/r02_host_mix.json: CPU AdamW + H2D + D2H DMA concurrently (the "
+                                     "engine's own mix), best total over thread counts"},
         "roofline": {"kernel": "K2 fused multi-tensor AdamW (sh_step)", "bound": "hbm", "achieved": k2_gbs,
                      "peak": peak, "unit": "GB/s", "frac": k2_gbs / peak if k2_gbs else None,
                      "traffic": k2_traffic(d["k2_bytes_sum"] / max(1, d["k2_samples"]) / (30 if prec else 32)),
@@ -593,11 +652,9 @@ def main():
                             "t_c2g_ms": float(np.median(p["t_c2g"])), "t_g2c_ms": float(np.median(p["t_g2c"])),
                             "t_opt_cpu_ms": float(np.median(p["t_opt_cpu"]))}
     if world == 1 and not args.no_cpu_baseline:
-        per_sample, tl, th = oracle_sample(L, h, nh, s, V)
-        line["cpu_baseline"] = {"value": 1.0 / per_sample, "unit": "samples/s", "cores": blas_threads(),
-                                "kind": "oracle",
-                                "sample": f"one block fwd+bwd+AdamW ({tl:.2f} s) and the head ({th:.2f} s) at batch 1, "
-                                          f"numpy fp64, extrapolated x{L} layers"}
+        per_step, parts = oracle_sample(L, h, nh, s, V, b)
+        line["cpu_baseline"] = {"value": b / per_step, "unit": "samples/s", "cores": blas_threads(),
+                                "kind": "oracle", "sample": oracle_desc(L, b, parts)}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

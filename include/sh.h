@@ -309,6 +309,9 @@ typedef struct {
                                    (layer FP/BP compute, K2); last_step_ms - compute_busy_ms is the
                                    compute stream's stall (waiting on fetches, restages, updates) */
   int64_t ring_bytes;           /* device bytes of the slot ring */
+  int64_t cpu_adam_shadow_elems;  /* of cpu_adam_elems, those that also wrote a bf16 shadow (30 instead of
+                                     28 B of host DRAM per element) */
+  int32_t shadow_layers;        /* host-optimised layers holding a bf16 shadow (fetched at 2 B/param) */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */

@@ -444,7 +444,7 @@ struct sh_ctx {
 
   // ---- stats
   std::atomic<int64_t> h2d_bytes{0}, d2h_bytes{0}, h2d_copies{0}, d2h_copies{0}, stage_launches{0};
-  std::atomic<int64_t> cpu_elems{0};
+  std::atomic<int64_t> cpu_elems{0}, cpu_shadow_elems{0};
   std::atomic<double> cpu_ms{0.0}, cpu_wait_ms{0.0};
   double h2d_busy = 0, d2h_busy = 0;
   int64_t h2d_prof_bytes = 0, d2h_prof_bytes = 0;
@@ -778,6 +778,7 @@ void worker_loop(sh_ctx* c, int tid) {
     while (!c->cpu_ms.compare_exchange_weak(cur, cur + dt)) {
     }
     c->cpu_elems.fetch_add(e - b);
+    if (c->h_shadow[x]) c->cpu_shadow_elems.fetch_add(e - b);
     if (job->done.fetch_add(1) + 1 == job->n_chunks) {
       const double t_end = now_ms();
       finish_job(c, job);
@@ -3155,6 +3156,12 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->d2h_profiled_bytes = c->d2h_prof_bytes;
   o->cpu_adam_ms = c->cpu_ms.load();
   o->cpu_adam_elems = c->cpu_elems.load();
+  o->cpu_adam_shadow_elems = c->cpu_shadow_elems.load();
+  {
+    int n = 0;
+    for (int x = c->w; x < c->L; ++x) n += c->h_shadow[x] != nullptr;
+    o->shadow_layers = n;
+  }
   o->cpu_wait_ms = c->cpu_wait_ms.load();
   o->k2_ms_last = c->k2_ms_last;
   o->k2_bytes_last = c->k2_bytes_last;
