@@ -113,9 +113,9 @@ typedef struct {
 #define SH_FLAG_DECOUPLE  (1ull << 9) /* autotuner: decouple the ring (prefetch distance) from the
                                          GPU-optimised set (needs no clipping and a landing buffer per
                                          layer, grad_ring_depth 0; R22) */
-#define SH_FLAG_SPILL_EVICT (1ull << 10) /* NEXT-2: after a spilled layer's CPU update, write it back and drop
-                                           it from the page cache (RAM held by the spill tier stays bounded;
-                                           every fetch / update of the layer reads the file) */
+#define SH_FLAG_SPILL_EVICT (1ull << 10) /* NEXT-2, no effect since ABI round 2: the spill tier always reads and
+                                           writes its files with O_DIRECT (no page cache), so the RAM it holds
+                                           is bounded by its pinned staging buffers */
 #define SH_FLAG_TEST_DP_PATH (1ull << 11) /* test: take the data-parallel path at world_size 1 (one-rank NCCL
                                             communicator from nccl_unique_id: the per-layer and resident
                                             all-reduces run on the comm stream and are the identity) */
@@ -187,12 +187,18 @@ typedef struct {
                                        for which pinned host RAM runs out, are kept in files there,
                                        memory-mapped (MAP_SHARED) instead of pinned ("memory-mapping a
                                        swap file on the secondary storage to the CPU memory space").
-                                       Their prefetches are copied through two pinned bounce buffers,
-                                       the CPU Adam updates them through the page cache (read-ahead
-                                       started when the layer's gradients land, write-back started
-                                       when its update finishes).  Results are bit-identical to the
-                                       all-pinned store.  Files are created O_EXCL, unlinked at once,
-                                       space reserved with posix_fallocate.  Not with shm_name. */
+                                       Files are read and written with O_DIRECT bulk requests through
+                                       io_uring ("asynchronous bulk read/write requests"),
+                                       no page cache: a prefetch reads the layer's fetch region into one
+                                       of two pinned bounce buffers, then H2D; when its gradients land
+                                       a spill-read thread reads master / m / v into one of
+                                       SH_SPILL_STAGING (env, default 3) pinned staging copies, the CPU
+                                       Adam updates that copy, a spill-write thread writes master / m /
+                                       v / shadow back, and only then is the layer updated for the next
+                                       fetch.  Results are bit-identical to the all-pinned store.  Files
+                                       are created O_EXCL, unlinked at once, space reserved with
+                                       posix_fallocate; file systems without O_DIRECT get the same
+                                       aligned transfers through the page cache.  Not with shm_name. */
   int64_t host_pin_budget_bytes;    /* cap on pinned host-store bytes (layer blocks + landing ring);
                                        0 = no cap (spill only when pinning fails for lack of RAM) */
   int32_t warmup_window;            /* window of the warm-up steps when window == -1 (0: min(2, n_layers)).
@@ -312,6 +318,11 @@ typedef struct {
   int64_t cpu_adam_shadow_elems;  /* of cpu_adam_elems, those that also wrote a bf16 shadow (30 instead of
                                      28 B of host DRAM per element) */
   int32_t shadow_layers;        /* host-optimised layers holding a bf16 shadow (fetched at 2 B/param) */
+  int32_t spill_direct;         /* NEXT-2: the spill files are O_DIRECT (0: the file system refused it) */
+  int64_t spill_read_bytes;     /* NEXT-2: cumulative bytes read from / written to the spill files */
+  int64_t spill_write_bytes;
+  double spill_io_ms;           /* cumulative duration of those transfers (summed over the I/O threads) */
+  int32_t spill_uring;          /* 1: transfers go through io_uring (else pread / pwrite) */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */

@@ -73,7 +73,7 @@ def build(verbose: bool = False) -> dict:
     headers = glob.glob(os.path.join(ROOT, "include", "*.h")) + glob.glob(os.path.join(CSRC, "*.hpp"))
     nccl = ["-I" + _nccl_include()]
     srcs = [os.path.join(CSRC, f) for f in ("engine.cpp", "layout.cpp", "autotune.cpp", "cpu_adam.cpp", "numa.cpp",
-                                            "kernels.cu")]
+                                            "spill_io.cpp", "kernels.cu")]
     objs = [_compile(s, headers, nccl, log) for s in srcs]
     lib = os.path.join(OUT, "libsh.so")
     if _newer(lib, objs):

@@ -224,6 +224,11 @@ struct Job {
   int layer;
   int64_t step;
   double t_first = 0.0;  // host ms when its first chunk was taken (trace)
+  // the arrays the update works on: the layer's pinned host block, or (NEXT-2 spilled layer) a pinned
+  // staging copy its optimizer state was read into
+  float *p = nullptr, *m = nullptr, *v = nullptr;
+  uint16_t* sh16 = nullptr;
+  char* staging = nullptr;
   int landing;
   int64_t lo, hi;  // element range of this rank (whole layer unless the store is shared)
   int64_t n_chunks;
@@ -346,6 +351,16 @@ struct sh_ctx {
   size_t bounce_bytes = 0;
   cudaEvent_t ev_bounce[2] = {nullptr, nullptr};
   int bounce_rr = 0;  // H2D issuer thread only
+  // O_DIRECT spill files: [master | m | v | shadow?] regions, each kAlign-aligned; a spilled layer's
+  // CPU update reads master/m/v into a pinned staging buffer (spill_rd thread), updates it there and
+  // writes master/m/v/shadow back (spill_wr thread) before the layer counts as updated
+  bool spill_direct = false;          // the spill files are O_DIRECT (else the file system refused it)
+  std::vector<char*> stg_free, stg_all;
+  size_t stg_bytes = 0;
+  std::mutex stg_mu;
+  std::condition_variable stg_cv;
+  std::atomic<int64_t> spill_rd_bytes{0}, spill_wr_bytes{0};
+  std::atomic<double> spill_io_ms{0.0};
   bool shadow = true;  // bf16 shadow kept in host RAM (bf16 mode without SH_FLAG_FETCH_FP32)
   // shared store (world_size > 1 with shm_name): rank r owns elements [slo[x], shi[x]) of layer x
   bool shared = false;
@@ -429,6 +444,8 @@ struct sh_ctx {
 
   // ---- issuers
   Issuer ih2d, id2h;
+  Issuer spill_rd, spill_wr;  // NEXT-2 spill-file reads / write-backs (started with the first spilled layer)
+  bool spill_threads = false;
 
   // ---- profiling
   ProfSet prof[2];
@@ -697,28 +714,84 @@ void host_block_free(char* p, size_t bytes) {
 // ---------------------------------------------------------------------------- CPU Adam pool
 void host_interval(sh_ctx* c, int kind, int layer, int64_t step, double t0, double t1);
 
-void finish_job(sh_ctx* c, Job* j) {
-  if (c->spilled[j->layer] && (c->cfg.flags & SH_FLAG_SPILL_EVICT)) {
-    const auto& hb = c->hblocks[j->layer];
-    {
-      // bounded RAM: write the layer back, then drop it from the page cache (the next fetch and
-      // update read it from the file again -- the paper's swap-file behaviour)
-      sync_file_range(hb.fd, 0, (off64_t)hb.bytes,
-                      SYNC_FILE_RANGE_WAIT_BEFORE | SYNC_FILE_RANGE_WRITE | SYNC_FILE_RANGE_WAIT_AFTER);
-      madvise(hb.p, hb.bytes, MADV_DONTNEED);
-      posix_fadvise(hb.fd, 0, (off_t)hb.bytes, POSIX_FADV_DONTNEED);
-    }
+// ---- NEXT-2 spill files (O_DIRECT): region k of layer x (0 master, 1 m, 2 v, 3 bf16 shadow) starts at
+// k * sp_rb(x); every region length and offset is a multiple of spill::kAlign
+int64_t sp_rb(const sh_ctx* c, int x) { return align_up(4 * c->lay[x].n_pad, (int64_t)spill::kAlign); }
+int64_t sp_sb(const sh_ctx* c, int x) {
+  return c->shadow ? align_up(2 * c->lay[x].n_pad, (int64_t)spill::kAlign) : 0;
+}
+int64_t sp_file_bytes(const sh_ctx* c, int x) { return 3 * sp_rb(c, x) + sp_sb(c, x); }
+bool has_shadow(const sh_ctx* c, int x) { return c->h_shadow[x] != nullptr || (c->spilled[x] && c->shadow); }
+
+// Blocking O_DIRECT transfer of `bytes` (rounded up to kAlign) between buf and layer x's spill file at
+// byte offset off.  Any thread; failures fail the context.
+sh_status spill_file_io(sh_ctx* c, bool write, int x, void* buf, int64_t bytes, int64_t off = 0) {
+  const double t0 = now_ms();
+  const int64_t n = align_up(bytes, (int64_t)spill::kAlign);
+  const int r = spill::transfer(write, c->hblocks[x].fd, buf, (size_t)n, off);
+  if (r != 0) {
+    async_fail(c, SH_ERR_OOM_HOST, "spill tier: %s of %lld B (layer %d): %s", write ? "write" : "read",
+               (long long)n, x, strerror(-r));
+    set_error("spill tier: %s of layer %d failed: %s", write ? "write" : "read", x, strerror(-r));
+    return SH_ERR_OOM_HOST;
   }
-  // (without SH_FLAG_SPILL_EVICT the kernel's flusher writes the layer back lazily: forcing an
-  // early write-back made the next step's CPU update wait on pages still under write-back --
-  // C2 with 8 spilled layers ran at 15.5 instead of ~47 samples/s, profiles/r01_bench_c2_spill8_*)
+  (write ? c->spill_wr_bytes : c->spill_rd_bytes).fetch_add(n);
+  const double dt = now_ms() - t0;
+  double cur = c->spill_io_ms.load();
+  while (!c->spill_io_ms.compare_exchange_weak(cur, cur + dt)) {
+  }
+  return SH_OK;
+}
+
+char* acquire_staging(sh_ctx* c) {
+  std::unique_lock<std::mutex> g(c->stg_mu);
+  const bool ok = c->stg_cv.wait_for(g, std::chrono::duration<double>(wait_timeout_s()),
+                                     [&] { return !c->stg_free.empty() || c->failed.load(); });
+  if (!ok) {
+    g.unlock();
+    async_fail(c, SH_ERR_STATE, "timeout waiting for a spill staging buffer");
+    return nullptr;
+  }
+  if (c->failed.load()) return nullptr;
+  char* p = c->stg_free.back();
+  c->stg_free.pop_back();
+  return p;
+}
+
+void release_staging(sh_ctx* c, char* p) {
+  {
+    std::lock_guard<std::mutex> g(c->stg_mu);
+    c->stg_free.push_back(p);
+  }
+  c->stg_cv.notify_all();
+}
+
+// The update of `layer` for step `step` is visible to the prefetches (and to the other ranks).
+void mark_updated(sh_ctx* c, int layer, int64_t step) {
+  c->ready[layer].store(step + 1, std::memory_order_release);
+  if (c->shared) c->ctl->cnt[layer].fetch_add(1, std::memory_order_release);
+  notify_state(c);
+}
+
+void finish_job(sh_ctx* c, Job* j) {
   // landing buffer first, readiness last: sync_all (and so grow_landing, which replaces the
   // landing_done array) returns once every layer is ready, so no worker may still be about to
   // touch a landing counter at that point
   c->landing_done[j->landing].fetch_add(1, std::memory_order_release);
-  c->ready[j->layer].store(j->step + 1, std::memory_order_release);
-  if (c->shared) c->ctl->cnt[j->layer].fetch_add(1, std::memory_order_release);
-  notify_state(c);
+  if (j->staging) {
+    // spilled layer: updated in its staging copy; it counts as updated once master / m / v / shadow
+    // are back in the file (the next fetch reads the file)
+    const int x = j->layer;
+    const int64_t step = j->step;
+    char* stg = j->staging;
+    c->spill_wr.push([c, x, step, stg] {
+      if (spill_file_io(c, true, x, stg, sp_file_bytes(c, x)) != SH_OK) return;
+      release_staging(c, stg);
+      mark_updated(c, x, step);
+    });
+    return;
+  }
+  mark_updated(c, j->layer, j->step);
 }
 
 void worker_loop(sh_ctx* c, int tid) {
@@ -771,14 +844,14 @@ void worker_loop(sh_ctx* c, int tid) {
     const int x = job->layer;
     const LayerLayout& Lx = c->lay[x];
     const int64_t b = job->lo + chunk * kCpuChunk, e = std::min(job->hi, b + kCpuChunk);
-    cpu::adamw_range(c->h_master[x], c->h_m[x], c->h_v[x], c->landing[job->landing],
-                     c->h_shadow[x], b, e, Lx.n_decay, job->sc, c->clip, coef);
+    cpu::adamw_range(job->p, job->m, job->v, c->landing[job->landing], job->sh16, b, e, Lx.n_decay, job->sc,
+                     c->clip, coef);
     const double dt = now_ms() - t0;
     double cur = c->cpu_ms.load();
     while (!c->cpu_ms.compare_exchange_weak(cur, cur + dt)) {
     }
     c->cpu_elems.fetch_add(e - b);
-    if (c->h_shadow[x]) c->cpu_shadow_elems.fetch_add(e - b);
+    if (job->sh16) c->cpu_shadow_elems.fetch_add(e - b);
     if (job->done.fetch_add(1) + 1 == job->n_chunks) {
       const double t_end = now_ms();
       finish_job(c, job);
@@ -805,10 +878,6 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
   std::unique_ptr<Landed> L(static_cast<Landed*>(arg));
   sh_ctx* c = L->c;
   if (c->shared) c->ctl->cnt[c->L + L->layer].fetch_add(1, std::memory_order_release);
-  if (c->spilled[L->layer]) {  // spilled layer: start reading its master / m / v before the CPU Adam
-    const auto& hb = c->hblocks[L->layer];
-    madvise(hb.p, hb.bytes, MADV_WILLNEED);
-  }
   auto j = std::make_unique<Job>();
   j->layer = L->layer;
   j->step = L->step;
@@ -817,12 +886,42 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
   j->hi = c->shi[L->layer];
   j->n_chunks = (j->hi - j->lo + kCpuChunk - 1) / kCpuChunk;
   j->sc = L->sc;
+  const int x = L->layer;
+  if (c->spilled[x]) {
+    // NEXT-2: the spill-read thread reads master / m / v into a pinned staging buffer, then queues the
+    // update on it ("asynchronous bulk read/write requests")
+    Job* raw = j.release();
+    c->spill_rd.push([c, raw, x] {
+      std::unique_ptr<Job> jb(raw);
+      char* stg = acquire_staging(c);
+      if (!stg) return;
+      if (spill_file_io(c, false, x, stg, 3 * sp_rb(c, x)) != SH_OK) {
+        release_staging(c, stg);
+        return;
+      }
+      const int64_t rb = sp_rb(c, x);
+      jb->staging = stg;
+      jb->p = reinterpret_cast<float*>(stg);
+      jb->m = reinterpret_cast<float*>(stg + rb);
+      jb->v = reinterpret_cast<float*>(stg + 2 * rb);
+      jb->sh16 = c->shadow ? reinterpret_cast<uint16_t*>(stg + 3 * rb) : nullptr;
+      {
+        std::lock_guard<std::mutex> g(c->pmu);
+        c->jobs.push_back(std::move(jb));
+      }
+      c->pcv.notify_all();
+    });
+    return;
+  }
+  j->p = c->h_master[x];
+  j->m = c->h_m[x];
+  j->v = c->h_v[x];
+  j->sh16 = c->h_shadow[x];
   if ((c->cfg.flags & SH_FLAG_SYNC_CPU) && !c->clip && !c->shared) {  // debug: inline, single-threaded
     Job* jp = j.get();
     const float coef = 1.0f;
-    cpu::adamw_range(c->h_master[jp->layer], c->h_m[jp->layer], c->h_v[jp->layer],
-                     c->landing[jp->landing], c->h_shadow[jp->layer], jp->lo,
-                     jp->hi, c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
+    cpu::adamw_range(jp->p, jp->m, jp->v, c->landing[jp->landing], jp->sh16, jp->lo, jp->hi,
+                     c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
     finish_job(c, jp);
     return;
   }
@@ -1000,7 +1099,7 @@ void prof_harvest(sh_ctx* c, ProfSet& P) {
         const double ms = ev_ms(P.c2g0[ph][i], P.c2g1[ph][i]);
         c->p_c2g[i] = ms;
         c->h2d_busy += ms;
-        c->h2d_prof_bytes += (int64_t)((c->bf16 && !c->h_shadow[i]) ? 4 : c->cb) *
+        c->h2d_prof_bytes += (int64_t)((c->bf16 && !has_shadow(c, i)) ? 4 : c->cb) *
                              (c->slice_fetch && c->use_nccl ? c->shi[i] - c->slo[i] : c->lay[i].n_pad);
       }
     if (P.rec_g2c[i]) {
@@ -1106,8 +1205,8 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   const int64_t need = c->step;
   // bf16 mode fetches the bf16 shadow; fp32 mode the master; SH_FLAG_FETCH_FP32 fetches the fp32
   // master into the slot's (idle) grad half and K1 casts it into the param half on the H2D stream
-  const bool cast = c->bf16 && !c->h_shadow[y];
-  const void* src = c->h_shadow[y] ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];
+  const bool cast = c->bf16 && !has_shadow(c, y);
+  const void* src = c->h_shadow[y] ? (const void*)c->h_shadow[y] : (const void*)c->h_master[y];  // null: spilled
   const int64_t eb = cast ? 4 : (int64_t)c->cb;  // fetched bytes per element
   const int64_t bytes = eb * n;
   // NEXT-1 slice fetch: this rank's slice over PCIe, the rest over NVLink (in-place all-gather)
@@ -1149,11 +1248,16 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
     char* buf = cast ? reinterpret_cast<char*>(stage_buf) : dst;
     const char* hsrc = static_cast<const char*>(src);
     if (c->spilled[y]) {
-      // NEXT-2: pageable source -> CPU copy into a pinned bounce buffer (reads the file through the
-      // page cache; overlaps the previous layer's H2D from the other buffer) -> async H2D
+      // NEXT-2: O_DIRECT read of the layer's fetch region (bf16 shadow, else fp32 master) from its
+      // spill file straight into a pinned bounce buffer (io_uring, no page cache; overlaps the
+      // previous layer's H2D from the other buffer) -> async H2D
       const int k = c->bounce_rr++ & 1;
       CKA(c, cudaEventSynchronize(c->ev_bounce[k]));  // its previous H2D has finished
-      std::memcpy(c->bounce[k], hsrc, bytes);
+      if (spill_file_io(c, false, y, c->bounce[k], bytes, cast ? 0 : 3 * sp_rb(c, y)) != SH_OK) {
+        c->arrive_pub[y].store(kInf);
+        notify_state(c);
+        return;
+      }
       hsrc = c->bounce[k];
     }
     if (P) CKA(c, cudaEventRecord(P->c2g0[ph][y], c->h2d));
@@ -1348,16 +1452,19 @@ sh_status shm_map(sh_ctx* c, const std::string& path, size_t bytes, bool create,
 
 // Host block of layer x: [master | m | v | shadow?], 2 MiB aligned.  Shared stores map the
 // segment rank 0 created (all layers are created collectively in sh_init).
-// NEXT-2: file-backed block in spill_dir (the paper's "memory-mapping a swap file on the secondary
-// storage").  The file is unlinked right away (the mapping keeps it; nothing is left
-// behind on a crash); space is reserved with posix_fallocate so a full disk fails here, not with a
-// SIGBUS inside the CPU Adam.
-sh_status spill_block_alloc(sh_ctx* c, int x, size_t bytes, char** out, int* fd_out) {
-  *out = nullptr;
+// NEXT-2: a layer beyond the pinned budget lives in a file in spill_dir -- the paper's swap file on the
+// secondary storage -- read and written with O_DIRECT bulk requests (io_uring), so
+// the tier's RAM is bounded by its pinned staging / bounce buffers instead of the page cache.  The file
+// is unlinked right away (nothing is left behind on a crash); space is reserved with posix_fallocate so
+// a full disk fails here, not in the middle of a step.  File systems without O_DIRECT (tmpfs) get a
+// plain descriptor and the same aligned transfers.
+sh_status spill_block_alloc(sh_ctx* c, int x, size_t bytes, int* fd_out) {
   *fd_out = -1;
   char path[4096];
   snprintf(path, sizeof(path), "%s/sh_spill_%d_%p_%d.bin", c->spill_dir.c_str(), (int)getpid(), (void*)c, x);
-  const int fd = open(path, O_RDWR | O_CREAT | O_EXCL, 0600);
+  int fd = open(path, O_RDWR | O_CREAT | O_EXCL | O_DIRECT, 0600);
+  bool direct = fd >= 0;
+  if (fd < 0 && errno == EINVAL) fd = open(path, O_RDWR | O_CREAT | O_EXCL, 0600);
   if (fd < 0) {
     set_error("spill tier: open(%s): %s", path, strerror(errno));
     return SH_ERR_OOM_HOST;
@@ -1369,17 +1476,14 @@ sh_status spill_block_alloc(sh_ctx* c, int x, size_t bytes, char** out, int* fd_
     set_error("spill tier: posix_fallocate of %lld B in %s: %s", (long long)bytes, c->spill_dir.c_str(), strerror(e));
     return SH_ERR_OOM_HOST;
   }
-  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
-  if (p == MAP_FAILED) {
-    close(fd);
-    set_error("spill tier: mmap of %lld B failed: %s", (long long)bytes, strerror(errno));
-    return SH_ERR_OOM_HOST;
-  }
-  *out = static_cast<char*>(p);
+  if (c->n_spilled == 0) c->spill_direct = direct;
+  else c->spill_direct = c->spill_direct && direct;
   *fd_out = fd;
   return SH_OK;
 }
 
+// Pinned buffers of the tier, allocated with the first spilled layer: two bounce buffers for fetches
+// and SH_SPILL_STAGING (default 3) staging copies for the CPU updates, plus its two I/O threads.
 sh_status ensure_bounce(sh_ctx* c) {
   if (c->bounce[0]) return SH_OK;
   const size_t b = align_up(4 * c->max_pad, 1 << 21);  // fp32 fetch is the largest
@@ -1391,14 +1495,42 @@ sh_status ensure_bounce(sh_ctx* c) {
     c->host_bytes += b;
   }
   c->bounce_bytes = b;
+  const char* e = getenv("SH_SPILL_STAGING");
+  const int n_stg = std::max(1, e ? atoi(e) : 3);
+  int64_t fb = 0;
+  for (int x = 0; x < c->L; ++x) fb = std::max(fb, sp_file_bytes(c, x));
+  c->stg_bytes = align_up(fb, 1 << 21);
+  for (int k = 0; k < n_stg; ++k) {
+    char* p = nullptr;
+    sh_status st = host_block_alloc(c->stg_bytes, c->n_threads, &p, c->land_node, &c->numa_bound);
+    if (st != SH_OK) return st;
+    c->stg_all.push_back(p);
+    c->stg_free.push_back(p);
+    c->host_bytes += c->stg_bytes;
+  }
+  if (!c->spill_threads) {
+    c->spill_rd.start();
+    c->spill_wr.start();
+    c->spill_threads = true;
+  }
   return SH_OK;
 }
 
+// A kAlign-aligned temporary host buffer (registration, window changes and reads of spilled layers).
+struct AlignedBuf {
+  void* p = nullptr;
+  explicit AlignedBuf(size_t bytes) {
+    if (posix_memalign(&p, spill::kAlign, align_up((int64_t)bytes, (int64_t)spill::kAlign)) != 0) p = nullptr;
+  }
+  ~AlignedBuf() { free(p); }
+  float* f() const { return static_cast<float*>(p); }
+  char* b() const { return static_cast<char*>(p); }
+};
+
 void release_host_layer(sh_ctx* c, int x) {
   auto& hb = c->hblocks[x];
-  if (!hb.p) return;
+  if (!hb.p && hb.fd < 0) return;
   if (hb.fd >= 0) {
-    munmap(hb.p, hb.bytes);
     close(hb.fd);
     c->spill_bytes -= hb.bytes;
     c->n_spilled--;
@@ -1450,9 +1582,9 @@ sh_status enable_late_shadow(sh_ctx* c) {
 }
 
 sh_status ensure_host_layer(sh_ctx* c, int x) {
-  if (c->h_master[x]) return SH_OK;
+  if (c->hblocks[x].p || c->hblocks[x].fd >= 0) return SH_OK;
   const int64_t n = c->lay[x].n_pad;
-  const size_t bytes = align_up(12 * n + (c->shadow ? 2 * n : 0), 1 << 21);
+  size_t bytes = align_up(12 * n + (c->shadow ? 2 * n : 0), 1 << 21);
   char* p = nullptr;
   int fd = -1;
   sh_status st = SH_OK;
@@ -1484,19 +1616,20 @@ sh_status ensure_host_layer(sh_ctx* c, int x) {
       }
     }
     if (spill) {
+      bytes = (size_t)sp_file_bytes(c, x);
       st = ensure_bounce(c);
-      if (st == SH_OK) st = spill_block_alloc(c, x, bytes, &p, &fd);
+      if (st == SH_OK) st = spill_block_alloc(c, x, bytes, &fd);
     }
   }
   if (st != SH_OK) return st;
   c->hblocks[x] = {p, bytes, fd};
-  if (fd >= 0) {
+  if (fd >= 0) {  // no host mapping: h_master / m / v / shadow stay null
     c->spilled[x] = 1;
     c->spill_bytes += bytes;
     c->n_spilled++;
-  } else {
-    c->host_bytes += bytes;
+    return SH_OK;
   }
+  c->host_bytes += bytes;
   float* b = reinterpret_cast<float*>(p);
   c->h_master[x] = b;
   c->h_m[x] = b + n;
@@ -1629,6 +1762,24 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   for (int x = w_new; x < w_old; ++x) {
     st = ensure_host_layer(c, x);
     if (st != SH_OK) return st;
+    if (c->spilled[x]) {  // NEXT-2: into the layer's spill file
+      const int64_t n = c->lay[x].n_pad, rb = sp_rb(c, x), fb = sp_file_bytes(c, x);
+      AlignedBuf t(fb);
+      if (!t.p) {
+        set_error("apply_window: no memory for a %lld B spill staging copy", (long long)fb);
+        return SH_ERR_OOM_HOST;
+      }
+      std::memset(t.p, 0, fb);
+      CKC(c, cudaMemcpy(t.b(), c->g[x].master, 4 * n, cudaMemcpyDeviceToHost));
+      CKC(c, cudaMemcpy(t.b() + rb, c->g[x].m, 4 * n, cudaMemcpyDeviceToHost));
+      CKC(c, cudaMemcpy(t.b() + 2 * rb, c->g[x].v, 4 * n, cudaMemcpyDeviceToHost));
+      if (c->shadow) cpu::cast_bf16_range(t.f(), reinterpret_cast<uint16_t*>(t.b() + 3 * rb), 0, n);
+      st = spill_file_io(c, true, x, t.p, fb);
+      if (st != SH_OK) return st;
+      c->ready[x].store(c->step);
+      free_g(c, x);
+      continue;
+    }
     // every rank holds the same GPU state; each writes its own slice of the (shared) store
     const int64_t lo = c->slo[x], nb = 4 * (c->shi[x] - c->slo[x]);
     CKC(c, cudaMemcpy(c->h_master[x] + lo, c->g[x].master + lo, nb, cudaMemcpyDeviceToHost));
@@ -1662,6 +1813,20 @@ sh_status apply_window(sh_ctx* c, int w_new) {
       return st;
     }
     const int64_t n = c->lay[x].n_pad;
+    if (c->spilled[x]) {  // NEXT-2: from the layer's spill file
+      const int64_t rb = sp_rb(c, x);
+      AlignedBuf t(3 * rb);
+      if (!t.p) {
+        set_error("apply_window: no memory for a spill staging copy");
+        return SH_ERR_OOM_HOST;
+      }
+      st = spill_file_io(c, false, x, t.p, 3 * rb);
+      if (st != SH_OK) return st;
+      CKC(c, cudaMemcpy(c->g[x].master, t.b(), 4 * n, cudaMemcpyHostToDevice));
+      CKC(c, cudaMemcpy(c->g[x].m, t.b() + rb, 4 * n, cudaMemcpyHostToDevice));
+      CKC(c, cudaMemcpy(c->g[x].v, t.b() + 2 * rb, 4 * n, cudaMemcpyHostToDevice));
+      continue;
+    }
     CKC(c, cudaMemcpy(c->g[x].master, c->h_master[x], 4 * n, cudaMemcpyHostToDevice));
     CKC(c, cudaMemcpy(c->g[x].m, c->h_m[x], 4 * n, cudaMemcpyHostToDevice));
     CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
@@ -2345,7 +2510,17 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
     const int64_t n = c->lay[x].n_pad;
     std::vector<float> tmp;
     float *hp = c->h_master[x], *hm = c->h_m[x], *hv = c->h_v[x];
-    if (!hp || (c->shared && c->rank != 0)) {  // no (own) host copy to write: stage through a temporary
+    AlignedBuf sbuf(c->spilled[x] ? sp_file_bytes(c, x) : 0);
+    if (c->spilled[x]) {  // NEXT-2: staged in the file's layout, written with one O_DIRECT request
+      if (!sbuf.p) {
+        set_error("sh_register_host_store: no memory for a spill staging copy");
+        return SH_ERR_OOM_HOST;
+      }
+      std::memset(sbuf.p, 0, sp_file_bytes(c, x));
+      hp = sbuf.f();
+      hm = reinterpret_cast<float*>(sbuf.b() + sp_rb(c, x));
+      hv = reinterpret_cast<float*>(sbuf.b() + 2 * sp_rb(c, x));
+    } else if (!hp || (c->shared && c->rank != 0)) {  // no (own) host copy to write: stage through a temporary
       tmp.resize(3 * n);
       hp = tmp.data();
       hm = hp + n;
@@ -2355,6 +2530,11 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
     pack_layer(c->lay[x], m, hm);
     pack_layer(c->lay[x], v, hv);
     if (c->shadow && c->h_shadow[x] && hp == c->h_master[x]) cpu::cast_bf16_range(hp, c->h_shadow[x], 0, n);
+    if (c->spilled[x]) {
+      if (c->shadow) cpu::cast_bf16_range(hp, reinterpret_cast<uint16_t*>(sbuf.b() + 3 * sp_rb(c, x)), 0, n);
+      st = spill_file_io(c, true, x, sbuf.p, sp_file_bytes(c, x));
+      if (st != SH_OK) return st;
+    }
     c->ready[x].store(step);
     if (c->shared && c->rank == 0) {
       c->ctl->cnt[x].store((int64_t)c->W * step);
@@ -2858,7 +3038,7 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   // fetched bytes per element (per layer: fp32 master + K1 cast without a shadow); with
   // SH_FLAG_LATE_SHADOW the host layers will fetch a bf16 shadow after the autotune: solve for that
   const bool late = c->bf16 && (c->cfg.flags & SH_FLAG_LATE_SHADOW) && !c->shared;
-  auto fbx = [&](int x) { return (c->bf16 && !c->h_shadow[x]) ? 4.0 : (double)c->cb; };
+  auto fbx = [&](int x) { return (c->bf16 && !has_shadow(c, x)) ? 4.0 : (double)c->cb; };
   double rate = 0;  // ms per byte: mean of the measured fetches
   double rate_min = 0;  // the fastest one: the warm-up runs with most layers on the host, so its
                         // fetches compete with the heaviest CPU-Adam traffic; the tuned run's don't
@@ -3066,6 +3246,26 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
   if (st != SH_OK && !c->failed.load()) return st;
   const LayerLayout& Lx = layer < 0 ? c->res : c->lay[layer];
   const int64_t n = Lx.n_pad;
+  if (layer >= 0 && !c->is_g(layer) && c->spilled[layer] && what != SH_READ_GRAD) {  // NEXT-2: from the file
+    const int64_t rb = sp_rb(c, layer), fb = sp_file_bytes(c, layer);
+    AlignedBuf t(fb);
+    if (!t.p) return SH_ERR_OOM_HOST;
+    st = spill_file_io(c, false, layer, t.p, fb);
+    if (st != SH_OK) return st;
+    if (what == SH_READ_COMPUTE) {
+      if (c->bf16) {
+        std::vector<uint16_t> b16(n);
+        if (c->shadow) std::memcpy(b16.data(), t.b() + 3 * rb, 2 * n);
+        else cpu::cast_bf16_range(t.f(), b16.data(), 0, n);
+        unpack_layer_u16(Lx, b16.data(), static_cast<uint16_t*>(dst));
+      } else {
+        unpack_layer(Lx, t.f(), static_cast<float*>(dst));
+      }
+      return SH_OK;
+    }
+    unpack_layer(Lx, reinterpret_cast<const float*>(t.b() + what * rb), static_cast<float*>(dst));
+    return SH_OK;
+  }
   if (what == SH_READ_COMPUTE) {
     std::vector<uint8_t> tmp((size_t)c->cb * n);
     if (layer < 0) {
@@ -3157,6 +3357,11 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->cpu_adam_ms = c->cpu_ms.load();
   o->cpu_adam_elems = c->cpu_elems.load();
   o->cpu_adam_shadow_elems = c->cpu_shadow_elems.load();
+  o->spill_read_bytes = c->spill_rd_bytes.load();
+  o->spill_write_bytes = c->spill_wr_bytes.load();
+  o->spill_io_ms = c->spill_io_ms.load();
+  o->spill_direct = c->spill_direct ? 1 : 0;
+  o->spill_uring = c->n_spilled > 0 && spill::uring_available() ? 1 : 0;
   {
     int n = 0;
     for (int x = c->w; x < c->L; ++x) n += c->h_shadow[x] != nullptr;
@@ -3257,9 +3462,12 @@ sh_status sh_destroy(sh_ctx* c) {
   for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s})
     if (s) cudaStreamDestroy(s);
   for (auto& b : c->hshadow) host_block_free(b.p, b.bytes);
+  c->stg_cv.notify_all();
+  c->spill_rd.stop();
+  c->spill_wr.stop();
+  for (char* p : c->stg_all) host_block_free(p, c->stg_bytes);
   for (auto& b : c->hblocks) {
     if (b.fd >= 0) {
-      munmap(b.p, b.bytes);
       close(b.fd);
     } else {
       host_block_free(b.p, b.bytes);

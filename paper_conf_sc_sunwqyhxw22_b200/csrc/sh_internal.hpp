@@ -38,6 +38,15 @@ void unpack_layer(const LayerLayout& L, const float* src, float* dst);  // padde
 void unpack_layer_u16(const LayerLayout& L, const uint16_t* src, uint16_t* dst);
 
 // ---- kernels (kernels.cu) -----------------------------------------------------------
+namespace spill {
+constexpr size_t kAlign = 4096;  // O_DIRECT granularity (buffer address, length and file offset)
+// true if this thread can use io_uring (else transfer() falls back to pread / pwrite)
+bool uring_available();
+// Blocking O_DIRECT transfer of bytes (multiple of kAlign) between buf (kAlign-aligned, ideally page-locked)
+// and file offset off of fd (opened O_DIRECT).  0 or -errno.
+int transfer(bool write, int fd, void* buf, size_t bytes, int64_t off);
+}  // namespace spill
+
 namespace kern {
 struct K2Entry {
   float* p;

@@ -99,7 +99,8 @@ class Stats(C.Structure):
                 ("numa_nodes", C.c_int32), ("numa_policy", C.c_int32), ("numa_gpu_node", C.c_int32),
                 ("numa_pinned_workers", C.c_int32), ("numa_bound_bytes", C.c_int64),
                 ("compute_busy_ms", C.c_double), ("ring_bytes", C.c_int64), ("cpu_adam_shadow_elems", C.c_int64),
-                ("shadow_layers", C.c_int32)]
+                ("shadow_layers", C.c_int32), ("spill_direct", C.c_int32), ("spill_read_bytes", C.c_int64),
+                ("spill_write_bytes", C.c_int64), ("spill_io_ms", C.c_double), ("spill_uring", C.c_int32)]
 
 
 class TraceEvent(C.Structure):

