@@ -206,6 +206,28 @@ def oracle_desc(L, b, parts):
             f"fp64, extrapolated to one step: L x (b x fwd+bwd + AdamW) + b x head + resident AdamW, L={L}, b={b}")
 
 
+def spill_line(args, r, K):
+    """NEXT-2: the spill tier's disk traffic per step and its rate vs the same O_DIRECT io_uring path probed on
+    a fresh file in the same directory (sh_spill_probe)."""
+    from paper_conf_sc_sunwqyhxw22_b200 import sh
+    st0, st1 = r["st0"], r["st1"]
+    rd, wr = st1["spill_read_bytes"] - st0["spill_read_bytes"], st1["spill_write_bytes"] - st0["spill_write_bytes"]
+    io_ms = st1["spill_io_ms"] - st0["spill_io_ms"]
+    try:
+        probe = sh.spill_probe(args.spill_dir, 2 << 30)
+    except Exception as e:  # noqa: BLE001
+        probe = {"error": str(e)}
+    out = {"dir": args.spill_dir, "layers": st1["spilled_layers"], "bytes": st1["spill_bytes"],
+           "o_direct": bool(st1["spill_direct"]), "io_uring": bool(st1["spill_uring"]),
+           "read_bytes_per_step": rd / K, "write_bytes_per_step": wr / K,
+           "disk_gbs_while_busy": (rd + wr) / (io_ms / 1e3) / 1e9 if io_ms > 0 else None,
+           "disk_gbs_per_step": (rd + wr) / (r["ms"] / 1e3) / 1e9, "probe": probe}
+    if "read_gbs" in probe and out["disk_gbs_while_busy"]:
+        out["frac_of_probe"] = (rd + wr) / (io_ms / 1e3) / 1e9 / (
+            (rd * probe["read_gbs"] + wr * probe["write_gbs"]) / max(1, rd + wr))
+    return out
+
+
 def blas_threads():
     try:
         from threadpoolctl import threadpool_info
@@ -552,8 +574,7 @@ def main():
                    "executors": args.executors,
                    "ablation": [k for k, v in (("alloc", args.ablate_alloc), ("sync_cpu", args.sync_cpu),
                                                ("cpu_threads", args.cpu_threads)) if v] or None,
-                   "spill": {"dir": args.spill_dir, "layers": r["st1"]["spilled_layers"],
-                             "bytes": r["st1"]["spill_bytes"], "evict": args.spill_evict} if args.spill_dir else None,
+                   "spill": spill_line(args, r, K) if args.spill_dir else None,
                    "host_store": ("one shared /dev/shm store, rank-sliced offload + CPU Adam" if shm_name else
                                   "private per rank") if world > 1 else "private",
                    "numa": {"nodes": r["st1"]["numa_nodes"],

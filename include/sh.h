@@ -461,6 +461,11 @@ int32_t sh_numa_node_of_pci(const char* bus_id);
  * (-1 if they differ or a syscall failed). */
 int32_t sh_numa_bind_check(int32_t node_id, int64_t bytes);
 
+/* NEXT-2 disk probe: write then read `bytes` of a fresh file in dir with the spill tier's own O_DIRECT
+ * io_uring transfers (write timed through fdatasync); GB/s each way; *direct = 1 if O_DIRECT was
+ * accepted.  The file is unlinked at creation.  No CUDA context needed. */
+sh_status sh_spill_probe(const char* dir, int64_t bytes, double* read_gbs, double* write_gbs, int32_t* direct);
+
 int32_t sh_abi_version(void);
 
 /* Number of engine kernel launches (K1, K2, K3, K4, norm finalize) since the library was loaded. */

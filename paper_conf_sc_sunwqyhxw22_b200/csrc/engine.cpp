@@ -396,7 +396,7 @@ struct sh_ctx {
   std::vector<int64_t> slot_last_use;  // global position of the occupant's latest compute (LRU tie-break)
   int64_t pos_clock = 0;
   std::vector<cudaEvent_t> ev_param_free, ev_grad_done, ev_grad_free, ev_reduced;
-  std::vector<int64_t> gradfree_gen, gradfree_waited;
+  std::vector<int64_t> gradfree_gen, gradfree_waited;  // per gradient-pool buffer (slot index)
   std::unique_ptr<std::atomic<int64_t>[]> gradfree_pub;
   std::vector<cudaEvent_t> ev_arrive;
   std::vector<cudaEvent_t> ev_upd;  // [L] after the latest K2 of a GPU-optimised layer (K1 restage waits)
@@ -411,10 +411,27 @@ struct sh_ctx {
   std::vector<uint8_t> arrive_by_issuer;
   std::unique_ptr<std::atomic<int64_t>[]> arrive_pub;
   std::unique_ptr<std::atomic<int64_t>[]> ready;  // updates applied to layer j
-  std::unique_ptr<std::atomic<int64_t>[]> landing_done;
-  std::vector<int64_t> landing_uses;
-  std::vector<int> landing_owner, last_landing;  // which layer's grads a landing buffer holds
-  int64_t landing_rr = 0;
+  // host landing buffers: free list (guarded by smu; a CPU update returns its buffer, the D2H
+  // scheduler takes one per offload); landing_owner / last_landing: which layer's grads a buffer holds
+  std::vector<int> land_free;
+  std::vector<int> landing_owner, last_landing;
+  // gradient pool (DESIGN.md §6 "gradient pool"): the grad halves of the ring's slots are a pool of
+  // gradient buffers not tied to the slot a layer's parameters sit in -- a layer in BP takes any free
+  // one, the D2H scheduler frees it once its offload is issued.  gb_owner[b] = layer holding b (-1:
+  // free, guarded by smu); layer_gb[x] = buffer of layer x's last backward
+  std::vector<int> gb_owner, layer_gb;
+  struct PendD2H {                 // a host layer's gradients waiting for their offload
+    int x, b;
+    int64_t step, gen, lo, hi;
+    sh_adam_scalars sc;
+    void* prof;
+    cudaEvent_t ready;
+    bool k3_on_d2h, k3_done;
+  };
+  std::mutex dmu;
+  std::deque<PendD2H> pend;        // guarded by dmu, in backward (POST) order
+  std::atomic<int64_t> pend_posted{0}, pend_k3{0};
+  float* fp32_stage = nullptr;     // SH_FLAG_FETCH_FP32: fp32 master staging for the K1 cast (h2d stream)
   int64_t gen = 0;
   std::mutex smu;
   std::condition_variable scv;
@@ -774,10 +791,13 @@ void mark_updated(sh_ctx* c, int layer, int64_t step) {
 }
 
 void finish_job(sh_ctx* c, Job* j) {
-  // landing buffer first, readiness last: sync_all (and so grow_landing, which replaces the
-  // landing_done array) returns once every layer is ready, so no worker may still be about to
-  // touch a landing counter at that point
-  c->landing_done[j->landing].fetch_add(1, std::memory_order_release);
+  // landing buffer first, readiness last: sync_all (and so grow_landing, which rebuilds the landing
+  // free list) returns once every layer is ready, so no worker may still be about to return a buffer
+  {
+    std::lock_guard<std::mutex> g(c->smu);
+    c->land_free.push_back(j->landing);
+  }
+  c->scv.notify_all();
   if (j->staging) {
     // spilled layer: updated in its staging copy; it counts as updated once master / m / v / shadow
     // are back in the file (the next fetch reads the file)
@@ -1214,12 +1234,10 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
   const int64_t slo = c->slo[y], shi = c->shi[y];
   const int64_t cs = align_up((n + c->W - 1) / c->W, kPad);
   cudaEvent_t pf = c->ev_param_free[s];
-  cudaEvent_t gf = c->ev_grad_free[s];
-  float* stage_buf = c->slot_grad(s);
-  const int64_t gf_gen = c->gradfree_gen[s];
+  float* stage_buf = c->fp32_stage;  // one buffer: the copy into it and the K1 cast out of it are both on the h2d stream
   const int64_t pbytes = c->slot_param_bytes_of(s);
-  c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, gf, stage_buf, gf_gen, s, n, eb, slice,
-                slo, shi, cs, pbytes] {
+  c->ih2d.push([c, y, need, src, dst, bytes, pf, gen, poison, P, ph, cast, stage_buf, n, eb, slice, slo, shi, cs,
+                pbytes] {
     maybe_delay(c->cfg.flags);
     double waited = 0;
     if (!state_wait(c, [&] { return ready_at_least(c, y, need); }, "CPU Adam of a layer to prefetch", &waited)) {
@@ -1236,14 +1254,6 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       host_interval(c, 9, y, need, t1 - waited, t1);  // waiting for the update of step need-1
     }
     CKA(c, cudaStreamWaitEvent(c->h2d, pf, 0));
-    if (cast) {  // the staging area (grad half) must be free of the previous occupant's offload
-      if (!state_wait(c, [&] { return c->gradfree_pub[s].load() >= gf_gen; }, "grad half for fp32 staging")) {
-        c->arrive_pub[y].store(kInf);
-        notify_state(c);
-        return;
-      }
-      CKA(c, cudaStreamWaitEvent(c->h2d, gf, 0));
-    }
     if (poison) CKA(c, cudaMemsetAsync(dst, 0xff, pbytes, c->h2d));
     char* buf = cast ? reinterpret_cast<char*>(stage_buf) : dst;
     const char* hsrc = static_cast<const char*>(src);
@@ -1253,7 +1263,8 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       // previous layer's H2D from the other buffer) -> async H2D
       const int k = c->bounce_rr++ & 1;
       CKA(c, cudaEventSynchronize(c->ev_bounce[k]));  // its previous H2D has finished
-      if (spill_file_io(c, false, y, c->bounce[k], bytes, cast ? 0 : 3 * sp_rb(c, y)) != SH_OK) {
+      const int64_t off = c->bf16 && has_shadow(c, y) ? 3 * sp_rb(c, y) : 0;  // shadow region, else the master
+      if (spill_file_io(c, false, y, c->bounce[k], bytes, off) != SH_OK) {
         c->arrive_pub[y].store(kInf);
         notify_state(c);
         return;
@@ -1710,6 +1721,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
   c->ev_reduced.resize(n_slots, nullptr);
   c->gradfree_gen.resize(n_slots, 0);
   c->gradfree_waited.resize(n_slots, 0);
+  c->gb_owner.assign(n_slots, -1);  // (engine idle: every pool buffer is free)
   auto pub = std::make_unique<std::atomic<int64_t>[]>(n_slots);
   for (int s = 0; s < n_slots; ++s) pub[s].store(s < old ? c->gradfree_pub[s].load() : 0);
   c->gradfree_pub = std::move(pub);
@@ -1874,12 +1886,13 @@ sh_status grow_landing(sh_ctx* c, int D_new) {
   c->h_coef = reinterpret_cast<float*>(p + (int64_t)D_new * lb);
   c->h_coef[0] = coef0;
   c->h_coef[1] = coef1;
-  c->landing_done = std::make_unique<std::atomic<int64_t>[]>(D_new);
-  for (int k = 0; k < D_new; ++k) c->landing_done[k].store(0);
-  c->landing_uses.assign(D_new, 0);
+  {
+    std::lock_guard<std::mutex> g(c->smu);
+    c->land_free.clear();
+    for (int k = D_new - 1; k >= 0; --k) c->land_free.push_back(k);
+  }
   c->landing_owner.assign(D_new, -1);
   c->last_landing.assign(c->L, -1);
-  c->landing_rr = 0;
   return SH_OK;
 }
 
@@ -2001,6 +2014,145 @@ sh_status coll_fold_partials(sh_ctx* c, cudaStream_t st) {
   if (r != SH_OK) return r;
   CKC(c, kern::fold_partials(c->partials_all, c->W, n, c->w, c->partials, st));
   return SH_OK;
+}
+
+// ---- gradient pool + offload scheduler.  Without enough host landing buffers the CPU
+// Adam paces the offloads; a FIFO offload queue then leaves the LOWEST layers' gradients (produced
+// last in BP) waiting in HBM behind the high ones at the end of BP, so the next FP -- which needs the
+// lowest layer first -- waits for the whole backlog (measured: 0.78 s of a 3.76 s c4max step).  The
+// scheduler offloads the lowest pending layer whenever a landing buffer is free, so the layers the
+// next FP needs first are updated first and the high layers' updates overlap that FP.  Gradients
+// wait in the pool (the ring's grad halves, any buffer for any layer), not in the slot their
+// layer's parameters happened to occupy, so the out-of-order offloads never block BP.
+
+// A free pool buffer of at least n elements for layer x (blocks until one's offload is issued).
+int take_grad_buffer(sh_ctx* c, int x, int64_t n) {
+  int b = -1;
+  auto pick = [&] {
+    b = -1;
+    for (int k = 0; k < c->n_slots; ++k) {
+      if (c->gb_owner[k] != -1 || c->gradfree_pub[k].load() < c->gradfree_gen[k]) continue;
+      if (c->byte_ring() && c->slot_cap[k] < n) continue;
+      if (b < 0 || (c->byte_ring() && c->slot_cap[k] < c->slot_cap[b])) b = k;  // best fit
+    }
+    return b >= 0;
+  };
+  {
+    std::unique_lock<std::mutex> g(c->smu);
+    if (pick()) {
+      c->gb_owner[b] = x;
+      return b;
+    }
+  }
+  if (!state_wait(c, pick, "a free gradient buffer")) return -1;
+  std::lock_guard<std::mutex> g(c->smu);
+  if (!pick()) return -1;  // (failed meanwhile)
+  c->gb_owner[b] = x;
+  return b;
+}
+
+void release_grad_buffer(sh_ctx* c, int b) {
+  {
+    std::lock_guard<std::mutex> g(c->smu);
+    c->gb_owner[b] = -1;
+  }
+  c->scv.notify_all();
+}
+
+// D2H issuer thread: offload pending host-layer gradients, lowest layer first, one per free landing
+// buffer; K3 (the layer's sum of squares, needed by sh_step) is enqueued for every pending layer in
+// backward order as soon as it is posted, before any wait for a landing buffer.
+void d2h_pump(sh_ctx* c) {
+  for (;;) {
+    std::vector<sh_ctx::PendD2H*> k3todo;
+    {
+      std::lock_guard<std::mutex> g(c->dmu);
+      for (auto& p : c->pend)
+        if (!p.k3_done) k3todo.push_back(&p);  // deque elements do not move on push_back
+    }
+    for (auto* p : k3todo) {
+      if (p->k3_on_d2h) {  // on its own stream so the copy engine does not queue behind it
+        ProfSet* P = static_cast<ProfSet*>(p->prof);
+        CKA(c, cudaStreamWaitEvent(c->k3s, p->ready, 0));
+        if (P) CKA(c, cudaEventRecord(P->k30[p->x], c->k3s));
+        CKA(c, kern::sumsq(c->slot_grad(p->b), c->lay[p->x].n_pad, c->scratch_d2h, c->partials + p->x, c->k3s));
+        if (P) {
+          CKA(c, cudaEventRecord(P->k31[p->x], c->k3s));
+          P->rec_k3[p->x] = 1;
+        }
+        CKA(c, cudaEventRecord(c->ev_k3_last, c->k3s));
+        c->k3_pub.store(p->gen);
+      }
+      p->k3_done = true;
+      c->pend_k3.fetch_add(1);
+    }
+    if (!k3todo.empty()) notify_state(c);
+    {
+      std::lock_guard<std::mutex> g(c->dmu);
+      if (c->pend.empty()) return;
+    }
+    // a free landing buffer, or new posts whose K3 must go out first
+    if (!state_wait(c, [&] { return !c->land_free.empty() || c->pend_posted.load() > c->pend_k3.load(); },
+                    "host landing buffer")) {
+      std::lock_guard<std::mutex> g(c->dmu);
+      for (auto& p : c->pend) c->gradfree_pub[p.b].store(kInf);
+      c->pend.clear();
+      notify_state(c);
+      return;
+    }
+    int k = -1;
+    {
+      std::lock_guard<std::mutex> g(c->smu);
+      if (c->land_free.empty()) continue;  // woken for K3s
+      k = c->land_free.back();
+      c->land_free.pop_back();
+    }
+    sh_ctx::PendD2H p{};
+    {
+      std::lock_guard<std::mutex> g(c->dmu);
+      // lowest layer first -- except with a shared store, where a slice update needs every rank's
+      // offload of the layer: all ranks then keep the backward (POST) order, so the landing buffers
+      // every rank holds always wait for the same layers
+      auto best = c->pend.end();
+      for (auto it = c->pend.begin(); it != c->pend.end(); ++it) {
+        if (!it->k3_done) continue;
+        if (c->shared) {
+          best = it;
+          break;
+        }
+        if (best == c->pend.end() || it->step < best->step || (it->step == best->step && it->x < best->x)) best = it;
+      }
+      if (best == c->pend.end()) {  // only fresh posts: their K3 first
+        std::lock_guard<std::mutex> g2(c->smu);
+        c->land_free.push_back(k);
+        continue;
+      }
+      p = *best;
+      c->pend.erase(best);
+    }
+    maybe_delay(c->cfg.flags);
+    ProfSet* P = static_cast<ProfSet*>(p.prof);
+    const int x = p.x;
+    c->landing_owner[k] = x;
+    c->last_landing[x] = k;
+    float* src = c->slot_grad(p.b);
+    CKA(c, cudaStreamWaitEvent(c->d2h, p.ready, 0));
+    if (P) CKA(c, cudaEventRecord(P->g2c0[x], c->d2h));
+    CKA(c, cudaMemcpyAsync(c->landing[k] + p.lo, src + p.lo, 4 * (p.hi - p.lo), cudaMemcpyDeviceToHost, c->d2h));
+    if (P) {
+      CKA(c, cudaEventRecord(P->g2c1[x], c->d2h));
+      P->rec_g2c[x] = 1;
+    }
+    // the buffer is reusable after the copy and this layer's K3 (k3s is in order: the latest K3
+    // event covers it)
+    if (p.k3_on_d2h) CKA(c, cudaStreamWaitEvent(c->d2h, c->ev_k3_last, 0));
+    CKA(c, cudaEventRecord(c->ev_grad_free[p.b], c->d2h));
+    CKA(c, cudaLaunchHostFunc(c->d2h, landed_cb, new Landed{c, x, p.step, k, p.sc}));
+    c->d2h_bytes += 4 * (p.hi - p.lo);
+    c->d2h_copies++;
+    c->gradfree_pub[p.b].store(p.gen);
+    release_grad_buffer(c, p.b);
+  }
 }
 
 }  // namespace
@@ -2363,6 +2515,14 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       c->device_bytes += 4 * (c->max_pad + n);
     }
   }
+  if (c->bf16 && !c->shadow) {  // SH_FLAG_FETCH_FP32: fp32 master staging of the fetches (h2d stream)
+    if (cudaMalloc(&c->fp32_stage, c->slot_grad_bytes) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("sh_init: cudaMalloc of the fp32 fetch staging buffer failed");
+      return SH_ERR_OOM_DEVICE;
+    }
+    c->device_bytes += c->slot_grad_bytes;
+  }
   c->g.assign(c->L, GState{});
   c->layer_slot.assign(c->L, -1);
   c->ev_arrive.assign(c->L, nullptr);
@@ -2381,11 +2541,10 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->arrive_pub[x].store(0);
     c->ready[x].store(0);
   }
-  c->landing_done = std::make_unique<std::atomic<int64_t>[]>(c->D);
-  for (int k = 0; k < c->D; ++k) c->landing_done[k].store(0);
-  c->landing_uses.assign(c->D, 0);
+  for (int k = c->D - 1; k >= 0; --k) c->land_free.push_back(k);
   c->landing_owner.assign(c->D, -1);
   c->last_landing.assign(c->L, -1);
+  c->layer_gb.assign(c->L, -1);
   c->reg_done.assign(c->L, 0);
   c->coef_of_step.assign(2, 1.0f);
   c->coef_step.assign(2, -1);
@@ -2655,8 +2814,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
     const int pos = 2 * L - 1 - x;
     st = pre_common(c, x, pos);
     if (st != SH_OK) return st;
-    const int s = c->layer_slot[x];
-    float* gdst = c->slot_grad(s);
+    float* gdst = nullptr;
     if (c->is_g(x) && c->k2_layer) {
       // dedicated grad buffer: no wait on this slot's pending offload
       const int b = (int)(c->gbuf_rr++ % (int64_t)c->gbuf.size());
@@ -2664,12 +2822,19 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       c->gbuf_owner[b] = x;
       CKC(c, cudaStreamWaitEvent(c->cs, c->ev_gbuf_free[b], 0));  // its previous K2 consumed it
       gdst = c->gbuf[b];
-    } else if (c->gradfree_gen[s] > c->gradfree_waited[s]) {
-      const int64_t gen = c->gradfree_gen[s];
-      if (!state_wait(c, [&] { return c->gradfree_pub[s].load() >= gen; }, "gradient offload issue"))
-        return check_failed(c);
-      CKC(c, cudaStreamWaitEvent(c->cs, c->ev_grad_free[s], 0));
-      c->gradfree_waited[s] = gen;
+    } else {
+      // any free buffer of the gradient pool (its previous offload issued; the GPU waits for it)
+      const int64_t need_n = c->rs_host && !c->is_g(x)
+                                 ? (int64_t)c->W * align_up((c->lay[x].n_pad + c->W - 1) / c->W, kPad)
+                                 : c->lay[x].n_pad;
+      const int b = take_grad_buffer(c, x, need_n);
+      if (b < 0) return check_failed(c);
+      c->layer_gb[x] = b;
+      if (c->gradfree_gen[b] > c->gradfree_waited[b]) {
+        CKC(c, cudaStreamWaitEvent(c->cs, c->ev_grad_free[b], 0));
+        c->gradfree_waited[b] = c->gradfree_gen[b];
+      }
+      gdst = c->slot_grad(b);
     }
     // (a reduce-scattered host layer spans W equal slices: zero the padding past n_pad too)
     const int64_t zn = c->rs_host && !c->is_g(x)
@@ -2690,6 +2855,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       return SH_ERR_STATE;
     }
     const int s = c->layer_slot[x];
+    const int gb = c->is_g(x) && c->k2_layer ? -1 : c->layer_gb[x];  // gradient-pool buffer
     const int64_t n = c->lay[x].n_pad;
     if (c->K > 1) {  // K4: fold the executors' micro-batch gradients (counted as BP compute)
       st = exec_fold(c, c->cur_gdst, c->xgrad, n);
@@ -2701,7 +2867,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       P->rec_bp[x] = 1;
     }
     CKC(c, cudaEventRecord(c->ev_param_free[s], c->cs));
-    cudaEvent_t grads_ready = c->ev_grad_done[s];
+    cudaEvent_t grads_ready = gb >= 0 ? c->ev_grad_done[gb] : nullptr;
     if (c->is_g(x) && c->k2_layer) {
       // GPU-optimised layer, no clipping: grads in its dedicated buffer b; [W>1: all-reduce];
       // K3; per-layer K2 (bitwise the same as a step-end update) on a side stream -- the stage
@@ -2753,86 +2919,47 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       c->arrive_pub[x].store(g2);
     } else if (c->dp) {
       // data parallel: average this layer's grads across ranks before the offload (K-e)
-      CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
-      CKC(c, cudaStreamWaitEvent(c->comm, c->ev_grad_done[s], 0));
+      float* g = c->slot_grad(gb);
+      CKC(c, cudaEventRecord(c->ev_grad_done[gb], c->cs));
+      CKC(c, cudaStreamWaitEvent(c->comm, c->ev_grad_done[gb], 0));
       if (c->rs_host && !c->is_g(x)) {
         // host layer, shared store: this rank offloads only its slice -> reduce-scatter, and the
         // K3 covers the slice (the per-rank partials are folded at sh_step)
-        st = coll_reduce_scatter_avg(c, c->slot_grad(s), x, c->comm);
+        st = coll_reduce_scatter_avg(c, g, x, c->comm);
         if (st != SH_OK) return st;
-        CKC(c, kern::sumsq(c->slot_grad(s) + c->slo[x], c->shi[x] - c->slo[x], c->scratch_comm, c->partials + x,
-                           c->comm));
+        CKC(c, kern::sumsq(g + c->slo[x], c->shi[x] - c->slo[x], c->scratch_comm, c->partials + x, c->comm));
       } else {
-        st = coll_allreduce_avg(c, c->slot_grad(s), n, c->comm, "ncclAllReduce(layer grads)");
+        st = coll_allreduce_avg(c, g, n, c->comm, "ncclAllReduce(layer grads)");
         if (st != SH_OK) return st;
-        CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_comm, c->partials + x, c->comm));
+        CKC(c, kern::sumsq(g, n, c->scratch_comm, c->partials + x, c->comm));
       }
-      CKC(c, cudaEventRecord(c->ev_reduced[s], c->comm));
-      grads_ready = c->ev_reduced[s];
-    } else if (c->is_g(x)) {  // clip mode: grads stay in the slot until sh_step's K2
+      CKC(c, cudaEventRecord(c->ev_reduced[gb], c->comm));
+      grads_ready = c->ev_reduced[gb];
+    } else if (c->is_g(x)) {  // clip mode: grads stay in their pool buffer until sh_step's K2
       if (P) CKC(c, cudaEventRecord(P->k30[x], c->cs));
-      CKC(c, kern::sumsq(c->slot_grad(s), n, c->scratch_cs, c->partials + x, c->cs));
+      CKC(c, kern::sumsq(c->slot_grad(gb), n, c->scratch_cs, c->partials + x, c->cs));
       if (P) {
         CKC(c, cudaEventRecord(P->k31[x], c->cs));
         P->rec_k3[x] = 1;
       }
-      CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
+      CKC(c, cudaEventRecord(c->ev_grad_done[gb], c->cs));
     } else {
-      // host layer: K3 runs on the D2H stream right before the offload (off the compute stream)
-      CKC(c, cudaEventRecord(c->ev_grad_done[s], c->cs));
+      // host layer: K3 runs on its own stream beside the offload (off the compute stream)
+      CKC(c, cudaEventRecord(c->ev_grad_done[gb], c->cs));
     }
     const bool k3_on_d2h = !c->dp && !c->is_g(x);
-    if (!c->is_g(x)) {
-      const int k = (int)(c->landing_rr++ % c->D);
-      const int64_t use = c->landing_uses[k]++;
-      c->landing_owner[k] = x;
-      c->last_landing[x] = k;
+    if (!c->is_g(x)) {  // post the offload: the D2H scheduler issues it lowest layer first (d2h_pump)
       const int64_t gen = ++c->gen;
-      c->gradfree_gen[s] = gen;
-      float* src = c->slot_grad(s);
-      float* dst = c->landing[k];
-      const int64_t lo = c->slo[x], hi = c->shi[x];  // this rank's slice (whole layer unless shared)
-      const int64_t step = c->step;
-      const sh_adam_scalars sc = c->sc;
-      cudaEvent_t gf = c->ev_grad_free[s];
+      c->gradfree_gen[gb] = gen;
       if (k3_on_d2h) c->k3_last_gen = gen;
-      c->id2h.push([c, k, use, grads_ready, src, dst, n, gf, x, step, sc, s, gen, P, k3_on_d2h, lo, hi] {
-        maybe_delay(c->cfg.flags);
-        CKA(c, cudaStreamWaitEvent(c->d2h, grads_ready, 0));
-        if (k3_on_d2h) {  // K3 before any host wait (sh_step only needs the norms), on its own
-                          // stream so the copy engine does not queue behind it; the grad half is
-                          // released only after both have read it
-          CKA(c, cudaStreamWaitEvent(c->k3s, grads_ready, 0));
-          if (P) CKA(c, cudaEventRecord(P->k30[x], c->k3s));
-          CKA(c, kern::sumsq(src, n, c->scratch_d2h, c->partials + x, c->k3s));
-          if (P) {
-            CKA(c, cudaEventRecord(P->k31[x], c->k3s));
-            P->rec_k3[x] = 1;
-          }
-          CKA(c, cudaEventRecord(c->ev_k3_last, c->k3s));
-          c->k3_pub.store(gen);
-          notify_state(c);
-        }
-        if (!state_wait(c, [&] { return c->landing_done[k].load(std::memory_order_acquire) >= use; },
-                        "host landing buffer")) {
-          c->gradfree_pub[s].store(kInf);
-          notify_state(c);
-          return;
-        }
-        if (P) CKA(c, cudaEventRecord(P->g2c0[x], c->d2h));
-        CKA(c, cudaMemcpyAsync(dst + lo, src + lo, 4 * (hi - lo), cudaMemcpyDeviceToHost, c->d2h));
-        if (P) {
-          CKA(c, cudaEventRecord(P->g2c1[x], c->d2h));
-          P->rec_g2c[x] = 1;
-        }
-        if (k3_on_d2h) CKA(c, cudaStreamWaitEvent(c->d2h, c->ev_k3_last, 0));  // this layer's K3
-        CKA(c, cudaEventRecord(gf, c->d2h));
-        CKA(c, cudaLaunchHostFunc(c->d2h, landed_cb, new Landed{c, x, step, k, sc}));
-        c->d2h_bytes += 4 * (hi - lo);
-        c->d2h_copies++;
-        c->gradfree_pub[s].store(gen);
-        notify_state(c);
-      });
+      {
+        std::lock_guard<std::mutex> g(c->dmu);
+        c->pend.push_back(sh_ctx::PendD2H{x, gb, c->step, gen, c->slo[x], c->shi[x], c->sc, P, grads_ready,
+                                          k3_on_d2h, false});
+      }
+      c->pend_posted.fetch_add(1);
+      notify_state(c);
+      c->id2h.push([c] { d2h_pump(c); });
     }
     c->last_hook = SH_POST;
   } else {
@@ -2966,7 +3093,7 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
       set_error("internal: GPU-optimised layer %d not in the ring at sh_step", x);
       return SH_ERR_STATE;
     }
-    a.e[a.n_entries++] = kern::K2Entry{c->g[x].master, c->g[x].m, c->g[x].v, c->slot_grad(s),
+    a.e[a.n_entries++] = kern::K2Entry{c->g[x].master, c->g[x].m, c->g[x].v, c->slot_grad(c->layer_gb[x]),
                                        c->slot_param(s), c->lay[x].n_pad, c->lay[x].n_decay};
     if (a.n_entries == kern::kK2MaxEntries) {
       st = push_k2(c, a, &bytes, &launches);
@@ -2978,7 +3105,16 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
   st = push_k2(c, a, &bytes, &launches);
   if (st != SH_OK) return st;
   if (!c->k2_layer)
-    for (int x = 0; x < c->w; ++x) CKC(c, cudaEventRecord(c->ev_upd[x], c->cs));
+    for (int x = 0; x < c->w; ++x) {
+      CKC(c, cudaEventRecord(c->ev_upd[x], c->cs));
+      // clip mode: the layer's pool buffer is free again once this K2 has read it
+      const int b = c->layer_gb[x];
+      CKC(c, cudaEventRecord(c->ev_grad_free[b], c->cs));
+      const int64_t g2 = ++c->gen;
+      c->gradfree_gen[b] = g2;
+      c->gradfree_pub[b].store(g2);
+      release_grad_buffer(c, b);
+    }
   if (P) {
     CKC(c, cudaEventRecord(P->k2b, c->cs));
     P->rec_k2 = true;
@@ -3307,12 +3443,13 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
         return SH_ERR_STATE;
       }
       CKC(c, cudaMemcpy(tmp.data(), c->gbuf[b], 4 * n, cudaMemcpyDeviceToHost));
-    } else if (c->is_g(layer)) {
-      if (c->layer_slot[layer] < 0) {
+    } else if (c->is_g(layer)) {  // clip mode: the pool buffer its K2 read (until another layer takes it)
+      const int b = c->layer_gb[layer];
+      if (b < 0 || c->gb_owner[b] != -1 || c->gradfree_gen[b] <= 0) {
         set_error("sh_read_layer: grads of layer %d not available", layer);
         return SH_ERR_STATE;
       }
-      CKC(c, cudaMemcpy(tmp.data(), c->slot_grad(c->layer_slot[layer]), 4 * n, cudaMemcpyDeviceToHost));
+      CKC(c, cudaMemcpy(tmp.data(), c->slot_grad(b), 4 * n, cudaMemcpyDeviceToHost));
     } else {
       const int k = c->last_landing[layer];
       if (k < 0 || c->landing_owner[k] != layer) {
@@ -3426,6 +3563,7 @@ sh_status sh_destroy(sh_ctx* c) {
     if (c->nccl) g_nccl.CommDestroy(c->nccl);
   }
   if (c->partials_all) cudaFree(c->partials_all);
+  if (c->fp32_stage) cudaFree(c->fp32_stage);
   if (c->hc_seg) {
     cudaHostUnregister(c->hc_seg);
     munmap(c->hc_seg, c->hc_bytes);
@@ -3480,6 +3618,48 @@ sh_status sh_destroy(sh_ctx* c) {
   if (c->ctl) munmap(c->ctl, c->ctl_bytes);
   host_block_free(c->hland.p, c->hland.bytes);
   delete c;
+  return SH_OK;
+}
+
+sh_status sh_spill_probe(const char* dir, int64_t bytes, double* read_gbs, double* write_gbs, int32_t* direct) {
+  clear_error();
+  if (!dir || bytes <= 0 || !read_gbs || !write_gbs) return SH_ERR_INVALID;
+  char path[4096];
+  snprintf(path, sizeof(path), "%s/sh_spill_probe_%d.bin", dir, (int)getpid());
+  int fd = open(path, O_RDWR | O_CREAT | O_EXCL | O_DIRECT, 0600);
+  const int d = fd >= 0;
+  if (fd < 0 && errno == EINVAL) fd = open(path, O_RDWR | O_CREAT | O_EXCL, 0600);
+  if (fd < 0) {
+    set_error("sh_spill_probe: open(%s): %s", path, strerror(errno));
+    return SH_ERR_INVALID;
+  }
+  unlink(path);
+  const size_t n = (size_t)align_up(bytes, 1 << 21);
+  void* p = mmap(nullptr, n, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+  if (p == MAP_FAILED || posix_fallocate(fd, 0, (off_t)n) != 0) {
+    if (p != MAP_FAILED) munmap(p, n);
+    close(fd);
+    set_error("sh_spill_probe: no memory / disk space for %lld B", (long long)n);
+    return SH_ERR_OOM_HOST;
+  }
+  std::memset(p, 0x5a, n);
+  double t0 = now_ms();
+  int r = spill::transfer(true, fd, p, n, 0);
+  if (r == 0) fdatasync(fd);
+  const double tw = now_ms() - t0;
+  posix_fadvise(fd, 0, (off_t)n, POSIX_FADV_DONTNEED);
+  t0 = now_ms();
+  if (r == 0) r = spill::transfer(false, fd, p, n, 0);
+  const double tr = now_ms() - t0;
+  munmap(p, n);
+  close(fd);
+  if (r != 0) {
+    set_error("sh_spill_probe: I/O failed: %s", strerror(-r));
+    return SH_ERR_OOM_HOST;
+  }
+  *write_gbs = n / (tw / 1e3) / 1e9;
+  *read_gbs = n / (tr / 1e3) / 1e9;
+  if (direct) *direct = d;
   return SH_OK;
 }
 

@@ -34,7 +34,7 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
            "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end", "sh_set_window_ring",
            "sh_executor_grads", "sh_op_exec_reduce_gpu", "sh_numa_topology", "sh_numa_plan",
-           "sh_numa_worker_node", "sh_numa_node_of_pci", "sh_numa_bind_check")
+           "sh_numa_worker_node", "sh_numa_node_of_pci", "sh_numa_bind_check", "sh_spill_probe")
 
 # NUMA placement policies (sh_config.numa_policy, include/sh.h)
 SH_NUMA_AUTO, SH_NUMA_SPLIT, SH_NUMA_LOCAL, SH_NUMA_INTERLEAVE, SH_NUMA_NONE = range(5)
@@ -152,6 +152,7 @@ def lib() -> C.CDLL:
             "sh_numa_topology": [vp, vp, i32], "sh_numa_plan": [i32] * 5,
             "sh_numa_worker_node": [i32] * 4, "sh_numa_node_of_pci": [C.c_char_p],
             "sh_numa_bind_check": [i32, i64],
+            "sh_spill_probe": [C.c_char_p, i64, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(i32)],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -224,6 +225,13 @@ def op_exec_reduce_gpu(dst, srcs, n, inv_k, stream=None):
 
 def op_sumsq_gpu(g, n, out_dev, stream=None):
     check(lib().sh_op_sumsq_gpu(_ptr(g), n, _ptr(out_dev), _stream_handle(stream)))
+
+
+def spill_probe(directory: str, nbytes: int = 1 << 30) -> dict:
+    """NEXT-2 disk probe: O_DIRECT io_uring write / read GB/s of a fresh file in `directory`."""
+    r, w, d = C.c_double(), C.c_double(), C.c_int32()
+    check(lib().sh_spill_probe(directory.encode(), nbytes, C.byref(r), C.byref(w), C.byref(d)))
+    return {"read_gbs": r.value, "write_gbs": w.value, "direct": bool(d.value)}
 
 
 def numa_topology() -> list[tuple[int, int]]:
