@@ -413,7 +413,7 @@ struct sh_ctx {
   std::unique_ptr<std::atomic<int64_t>[]> ready;  // updates applied to layer j
   // host landing buffers: free list (guarded by smu; a CPU update returns its buffer, the D2H
   // scheduler takes one per offload); landing_owner / last_landing: which layer's grads a buffer holds
-  std::vector<int> land_free;
+  std::deque<int> land_free;  // FIFO: a buffer is reused as late as possible (SH_READ_GRAD diagnostics)
   std::vector<int> landing_owner, last_landing;
   // gradient pool (DESIGN.md §6 "gradient pool"): the grad halves of the ring's slots are a pool of
   // gradient buffers not tied to the slot a layer's parameters sit in -- a layer in BP takes any free
@@ -431,6 +431,7 @@ struct sh_ctx {
   std::mutex dmu;
   std::deque<PendD2H> pend;        // guarded by dmu, in backward (POST) order
   std::atomic<int64_t> pend_posted{0}, pend_k3{0};
+  bool d2h_fifo = false;           // SH_D2H_ORDER=fifo: offload in backward order (A/B of the scheduler)
   float* fp32_stage = nullptr;     // SH_FLAG_FETCH_FP32: fp32 master staging for the K1 cast (h2d stream)
   int64_t gen = 0;
   std::mutex smu;
@@ -1889,7 +1890,7 @@ sh_status grow_landing(sh_ctx* c, int D_new) {
   {
     std::lock_guard<std::mutex> g(c->smu);
     c->land_free.clear();
-    for (int k = D_new - 1; k >= 0; --k) c->land_free.push_back(k);
+    for (int k = 0; k < D_new; ++k) c->land_free.push_back(k);
   }
   c->landing_owner.assign(D_new, -1);
   c->last_landing.assign(c->L, -1);
@@ -2104,8 +2105,8 @@ void d2h_pump(sh_ctx* c) {
     {
       std::lock_guard<std::mutex> g(c->smu);
       if (c->land_free.empty()) continue;  // woken for K3s
-      k = c->land_free.back();
-      c->land_free.pop_back();
+      k = c->land_free.front();
+      c->land_free.pop_front();
     }
     sh_ctx::PendD2H p{};
     {
@@ -2116,7 +2117,7 @@ void d2h_pump(sh_ctx* c) {
       auto best = c->pend.end();
       for (auto it = c->pend.begin(); it != c->pend.end(); ++it) {
         if (!it->k3_done) continue;
-        if (c->shared) {
+        if (c->shared || c->d2h_fifo) {
           best = it;
           break;
         }
@@ -2124,7 +2125,7 @@ void d2h_pump(sh_ctx* c) {
       }
       if (best == c->pend.end()) {  // only fresh posts: their K3 first
         std::lock_guard<std::mutex> g2(c->smu);
-        c->land_free.push_back(k);
+        c->land_free.push_front(k);
         continue;
       }
       p = *best;
@@ -2240,6 +2241,10 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->W = W;
   c->rank = cfg->rank;
   c->dp = dp;
+  {
+    const char* e = getenv("SH_D2H_ORDER");
+    c->d2h_fifo = e && strcmp(e, "fifo") == 0;
+  }
   c->no_collective = dp && (cfg->flags & SH_FLAG_TEST_NO_COLLECTIVE);
   c->host_coll = dp && !c->no_collective && (cfg->flags & SH_FLAG_TEST_HOST_COLLECTIVE);
   c->use_nccl = dp && !c->no_collective && !c->host_coll;
@@ -2541,7 +2546,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->arrive_pub[x].store(0);
     c->ready[x].store(0);
   }
-  for (int k = c->D - 1; k >= 0; --k) c->land_free.push_back(k);
+  for (int k = 0; k < c->D; ++k) c->land_free.push_back(k);
   c->landing_owner.assign(c->D, -1);
   c->last_landing.assign(c->L, -1);
   c->layer_gb.assign(c->L, -1);
