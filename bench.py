@@ -49,7 +49,9 @@ CONFIGS = {
                                                 "L = 32 + host-RAM capacity, auto-tuned window"),
 }
 C4MAX_W0 = 32
-FETCH_FP32_DEFAULT = {"c4", "c4max"}
+# bf16 host layout: the split master (R25: hi plane = the bf16 compute copy, fetched at 2 B/param;
+# 12 B/param of host RAM) for every config; --fetch-fp32 1 / --bf16-shadow select the round-1 layouts
+FETCH_FP32_DEFAULT: set = set()
 CPU_HARD_DEFAULT = {"c3", "c4", "c4max"}   # autotune with the eq. 3 CPU-throughput constraint (R19)
 # autotune with the B200 extensions of the window model by default (R22/R23): landing-ring
 # growth, GPU set filling the HBM a decoupled ring leaves, late bf16 host shadows (C4: 7.30 -> 7.92
@@ -281,7 +283,8 @@ def main():
     ap.add_argument("--no-resident", action="store_true", help="skip the all-resident comparison run")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--fetch-fp32", type=int, default=-1, help="1: no host bf16 shadow, fp32 over the link")
+    ap.add_argument("--fetch-fp32", type=int, default=-1, help="1: fp32 master in host RAM, fp32 over the link + K1")
+    ap.add_argument("--bf16-shadow", action="store_true", help="fp32 master + bf16 shadow in host RAM (14 B/param)")
     ap.add_argument("--init-threads", type=int, default=16)
     ap.add_argument("--layers", type=int, default=0, help="override the depth (c4: L_max(host RAM))")
     ap.add_argument("--trace-out", default="", help="write a Chrome trace of the last profiled step")
@@ -408,7 +411,7 @@ def main():
             (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0) | \
             (sh.SH_FLAG_ABLATE_ALLOC if args.ablate_alloc else 0) | (sh.SH_FLAG_SYNC_CPU if args.sync_cpu else 0) | \
             (sh.SH_FLAG_GROW_LANDING if args.grow_landing else 0) | (sh.SH_FLAG_FILL_GPU if args.fill_gpu else 0) | \
-            (sh.SH_FLAG_LATE_SHADOW if args.late_shadow else 0)
+            (sh.SH_FLAG_LATE_SHADOW if args.late_shadow else 0) | (sh.SH_FLAG_BF16_SHADOW if args.bf16_shadow else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
                                flags=flags, world_size=world, rank=rank, nccl_id=nid,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm,
@@ -581,12 +584,14 @@ def main():
                             "policy": ("auto", "split", "local", "interleave", "none")[r["st1"]["numa_policy"]],
                             "gpu_node": r["st1"]["numa_gpu_node"], "pinned_workers": r["st1"]["numa_pinned_workers"],
                             "bound_bytes": r["st1"]["numa_bound_bytes"]},
-                   "states": "fp32 master/m/v in pinned host RAM" + ("" if fetch32 and not st1["shadow_layers"]
-                                                                     else " + bf16 shadow"),
-                   "fetch": ("bf16 shadow" if not fetch32 else
+                   "states": (("split fp32 master (bf16 hi plane = compute copy + 16-bit lo plane), m, v in pinned "
+                               "host RAM, 12 B/param") if prec == sh.SH_BF16_MIXED and not fetch32 and not args.bf16_shadow
+                              else "fp32 master/m/v in pinned host RAM" + ("" if not st1["shadow_layers"] else " + bf16 shadow")),
+                   "fetch": ("hi plane of the split master (bf16, 2 B/param)" if prec == sh.SH_BF16_MIXED and not fetch32
+                             and not args.bf16_shadow else "bf16 shadow" if args.bf16_shadow else
                              f"bf16 shadow for {st1['shadow_layers']} of {L - st1['window']} host layers (late "
                              "shadows), fp32 master + K1 cast on the GPU for the rest" if st1["shadow_layers"] else
-                             "fp32 master, K1 cast on GPU"),
+                             "fp32 master, K1 cast on GPU" if prec == sh.SH_BF16_MIXED else "fp32 master"),
                    "grad_landing_buffers": r["st1"]["landing_buffers"], "host_store_bytes": r["st1"]["host_bytes"],
                    "states_bytes_fp32_p_m_v": 12 * mc.n_params(),
                    "l2": "no flush: per-step traffic (GBs) >> 126 MB L2",

@@ -35,11 +35,18 @@
  * element, in IEEE fp32 round-to-nearest, no FTZ/DAZ:
  *     g = g*coef (only when clipping is on);  m = fma(b1, m, omb1*g);
  *     v = fma(b2, v, omb2*(g*g));  d = sqrt(v)/sqrt_bc2 + eps;
- *     p = fma(-step_size, m/d, wd ? p*decay : p);  p16 = rne_bf16(p)
+ *     p = fma(-step_size, m/d, wd ? p*decay : p);  p16 = rna_bf16(p)
  *   with b1, b2, eps, omb1 = 1-b1, omb2 = 1-b2, sqrt_bc2 = sqrt(1-b2^t), step_size = lr/(1-b1^t),
  *   decay = 1 - lr*lambda computed in double from the double hyperparameters on the host and
  *   rounded once to fp32.
- *   rne_bf16 is integer round-to-nearest-even with canonical NaN 0x7FC0.
+ *   rna_bf16 is round-to-nearest, ties away from zero: (bits(p) + 0x8000) >> 16, canonical NaN 0x7FC0
+ *   (R25: the rounding under which the split master below is lossless).
+ *
+ * bf16 host layout (default, R25): a host-optimised layer keeps its fp32 master as two 16-bit
+ *   planes, hi = rna_bf16(p) -- which IS the compute copy the prefetch moves, 2 B/param -- and lo = the
+ *   low 16 bits of bits(p); p = (hi << 16) + sext16(lo) exactly (a NaN comes back as a NaN).  12 B/param of
+ *   host RAM (hi, lo, m, v) with a 2 B/param fetch and no shadow copy.  SH_FLAG_FETCH_FP32 keeps an fp32
+ *   master (fetch 4 B + K1 cast on the GPU), SH_FLAG_BF16_SHADOW an fp32 master + a bf16 shadow (14 B).
  *
  * Errors: every call returns sh_status; no exception crosses the ABI.  The message
  * of the last failing call on this thread is sh_last_error().  After SH_ERR_CUDA /
@@ -141,6 +148,8 @@ typedef struct {
                                             order (identical on every rank).  Several ranks on ONE GPU with
                                             DIFFERENT data: the averaging itself is checked against the
                                             oracle's global-batch mean.  No NCCL. */
+#define SH_FLAG_BF16_SHADOW (1ull << 18) /* bf16 mode: fp32 master + separate bf16 shadow in host RAM (14 B/param)
+                                           instead of the split master (the round-1 layout) */
 #define SH_FLAG_CPU_HARD  (1ull << 4) /* autotuner: CPU-update throughput (eq. 3, R19) is a hard constraint */
 #define SH_FLAG_SYNC_CPU  (1ull << 3) /* debug: run each CPU Adam task inline when its grads land (no pool; ignored in clip mode) */
 
@@ -500,11 +509,21 @@ sh_status sh_op_adamw_cpu(float* p, float* m, float* v, const float* g, uint16_t
                           int64_t n, int64_t n_decay, const sh_adam_scalars* sc, int32_t use_coef,
                           float coef, int32_t n_threads);
 
-/* K1: dst16[i] = rne_bf16(src[i]) on the device. */
+/* K1: dst16[i] = rna_bf16(src[i]) on the device. */
 sh_status sh_op_cast_bf16_gpu(const float* src, uint16_t* dst16, int64_t n, void* stream);
 
-/* CPU rne_bf16 (the shadow writer of the CPU Adam). */
+/* CPU rna_bf16 (the shadow writer of the CPU Adam). */
 sh_status sh_op_cast_bf16_cpu(const float* src, uint16_t* dst16, int64_t n);
+
+/* Split master (host arrays, R25): hi[i] = rna_bf16(p[i]), lo[i] = low 16 bits of bits(p[i]) ... */
+sh_status sh_op_master_split_cpu(const float* p, uint16_t* hi, uint16_t* lo, int64_t n);
+/* ... and back: p[i] = bits((hi[i] << 16) + sext16(lo[i])). */
+sh_status sh_op_master_join_cpu(const uint16_t* hi, const uint16_t* lo, float* p, int64_t n);
+/* The CPU AdamW of the pool on a split master (hi, lo in/out; m, v in/out; g in), same contract as
+ * sh_op_adamw_cpu: the joined result equals sh_op_adamw_cpu's p bitwise and hi its bf16 output. */
+sh_status sh_op_adamw_split_cpu(uint16_t* hi, uint16_t* lo, float* m, float* v, const float* g, int64_t n,
+                                int64_t n_decay, const sh_adam_scalars* sc, int32_t use_coef, float coef,
+                                int32_t n_threads);
 
 /* K4 (NEXT-3): dst[i] = (((dst[i] + src[0][i]) + src[1][i]) + ... + src[n_src-1][i]) * inv_k,
  * every op IEEE fp32 round-to-nearest; src is a HOST array of n_src (0..7) device pointers. */

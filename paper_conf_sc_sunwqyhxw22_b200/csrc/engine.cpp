@@ -227,7 +227,8 @@ struct Job {
   // the arrays the update works on: the layer's pinned host block, or (NEXT-2 spilled layer) a pinned
   // staging copy its optimizer state was read into
   float *p = nullptr, *m = nullptr, *v = nullptr;
-  uint16_t* sh16 = nullptr;
+  uint16_t* sh16 = nullptr;  // bf16 shadow out, or (split master) the hi plane in/out
+  uint16_t* lo16 = nullptr;  // split master: the lo plane in/out (then p is unused)
   char* staging = nullptr;
   int landing;
   int64_t lo, hi;  // element range of this rank (whole layer unless the store is shared)
@@ -361,7 +362,8 @@ struct sh_ctx {
   std::condition_variable stg_cv;
   std::atomic<int64_t> spill_rd_bytes{0}, spill_wr_bytes{0};
   std::atomic<double> spill_io_ms{0.0};
-  bool shadow = true;  // bf16 shadow kept in host RAM (bf16 mode without SH_FLAG_FETCH_FP32)
+  bool shadow = false;  // SH_FLAG_BF16_SHADOW: fp32 master + a bf16 shadow in host RAM (14 B/param)
+  bool split = false;   // bf16 default: split master, hi plane = the compute copy (12 B/param, R25)
   // shared store (world_size > 1 with shm_name): rank r owns elements [slo[x], shi[x]) of layer x
   bool shared = false;
   // the data-parallel (collective) path: world_size > 1, or SH_FLAG_TEST_DP_PATH at world_size 1
@@ -386,7 +388,8 @@ struct sh_ctx {
   std::vector<int64_t> slo, shi;
   int64_t bar_calls[6] = {0, 0, 0, 0, 0, 0};
   std::vector<float*> h_master, h_m, h_v;
-  std::vector<uint16_t*> h_shadow;
+  std::vector<uint16_t*> h_shadow;  // bf16 copy the prefetch moves: the shadow, or the split master's hi plane
+  std::vector<uint16_t*> h_lo;      // split master: low 16 bits of the fp32 pattern (R25)
   std::vector<float*> landing;
   float* h_coef = nullptr;  // pinned [2]
   std::vector<uint8_t> registered;
@@ -420,6 +423,8 @@ struct sh_ctx {
   // one, the D2H scheduler frees it once its offload is issued.  gb_owner[b] = layer holding b (-1:
   // free, guarded by smu); layer_gb[x] = buffer of layer x's last backward
   std::vector<int> gb_owner, layer_gb;
+  std::vector<int64_t> gb_free_seq;  // release order (smu): the longest-free buffer is taken first
+  int64_t gb_free_ctr = 0;
   struct PendD2H {                 // a host layer's gradients waiting for their offload
     int x, b;
     int64_t step, gen, lo, hi;
@@ -739,7 +744,10 @@ int64_t sp_sb(const sh_ctx* c, int x) {
   return c->shadow ? align_up(2 * c->lay[x].n_pad, (int64_t)spill::kAlign) : 0;
 }
 int64_t sp_file_bytes(const sh_ctx* c, int x) { return 3 * sp_rb(c, x) + sp_sb(c, x); }
-bool has_shadow(const sh_ctx* c, int x) { return c->h_shadow[x] != nullptr || (c->spilled[x] && c->shadow); }
+bool has_shadow(const sh_ctx* c, int x) {
+  return c->h_shadow[x] != nullptr || (c->spilled[x] && (c->shadow || c->split));
+}
+// (a split-master spill file holds [hi | lo] in region 0: the fetch reads its first 2n bytes)
 
 // Blocking O_DIRECT transfer of `bytes` (rounded up to kAlign) between buf and layer x's spill file at
 // byte offset off.  Any thread; failures fail the context.
@@ -865,14 +873,18 @@ void worker_loop(sh_ctx* c, int tid) {
     const int x = job->layer;
     const LayerLayout& Lx = c->lay[x];
     const int64_t b = job->lo + chunk * kCpuChunk, e = std::min(job->hi, b + kCpuChunk);
-    cpu::adamw_range(job->p, job->m, job->v, c->landing[job->landing], job->sh16, b, e, Lx.n_decay, job->sc,
-                     c->clip, coef);
+    if (job->lo16)
+      cpu::adamw_range_split(job->sh16, job->lo16, job->m, job->v, c->landing[job->landing], b, e, Lx.n_decay,
+                             job->sc, c->clip, coef);
+    else
+      cpu::adamw_range(job->p, job->m, job->v, c->landing[job->landing], job->sh16, b, e, Lx.n_decay, job->sc,
+                       c->clip, coef);
     const double dt = now_ms() - t0;
     double cur = c->cpu_ms.load();
     while (!c->cpu_ms.compare_exchange_weak(cur, cur + dt)) {
     }
     c->cpu_elems.fetch_add(e - b);
-    if (job->sh16) c->cpu_shadow_elems.fetch_add(e - b);
+    if (job->sh16 && !job->lo16) c->cpu_shadow_elems.fetch_add(e - b);
     if (job->done.fetch_add(1) + 1 == job->n_chunks) {
       const double t_end = now_ms();
       finish_job(c, job);
@@ -926,6 +938,11 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
       jb->m = reinterpret_cast<float*>(stg + rb);
       jb->v = reinterpret_cast<float*>(stg + 2 * rb);
       jb->sh16 = c->shadow ? reinterpret_cast<uint16_t*>(stg + 3 * rb) : nullptr;
+      if (c->split) {  // region 0 = [hi | lo]
+        jb->p = nullptr;
+        jb->sh16 = reinterpret_cast<uint16_t*>(stg);
+        jb->lo16 = reinterpret_cast<uint16_t*>(stg) + c->lay[x].n_pad;
+      }
       {
         std::lock_guard<std::mutex> g(c->pmu);
         c->jobs.push_back(std::move(jb));
@@ -938,11 +955,16 @@ void CUDART_CB landed_cb(void* arg) {  // runs on a CUDA driver thread: no CUDA 
   j->m = c->h_m[x];
   j->v = c->h_v[x];
   j->sh16 = c->h_shadow[x];
+  j->lo16 = c->h_lo[x];
   if ((c->cfg.flags & SH_FLAG_SYNC_CPU) && !c->clip && !c->shared) {  // debug: inline, single-threaded
     Job* jp = j.get();
     const float coef = 1.0f;
-    cpu::adamw_range(jp->p, jp->m, jp->v, c->landing[jp->landing], jp->sh16, jp->lo, jp->hi,
-                     c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
+    if (jp->lo16)
+      cpu::adamw_range_split(jp->sh16, jp->lo16, jp->m, jp->v, c->landing[jp->landing], jp->lo, jp->hi,
+                             c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
+    else
+      cpu::adamw_range(jp->p, jp->m, jp->v, c->landing[jp->landing], jp->sh16, jp->lo, jp->hi,
+                       c->lay[jp->layer].n_decay, jp->sc, c->clip, coef);
     finish_job(c, jp);
     return;
   }
@@ -1264,7 +1286,8 @@ sh_status issue_fetch(sh_ctx* c, int y, int s, int pos) {
       // previous layer's H2D from the other buffer) -> async H2D
       const int k = c->bounce_rr++ & 1;
       CKA(c, cudaEventSynchronize(c->ev_bounce[k]));  // its previous H2D has finished
-      const int64_t off = c->bf16 && has_shadow(c, y) ? 3 * sp_rb(c, y) : 0;  // shadow region, else the master
+      // the shadow region; else the master, or a split master's hi plane, both at 0
+      const int64_t off = c->shadow ? 3 * sp_rb(c, y) : 0;
       if (spill_file_io(c, false, y, c->bounce[k], bytes, off) != SH_OK) {
         c->arrive_pub[y].store(kInf);
         notify_state(c);
@@ -1528,6 +1551,24 @@ sh_status ensure_bounce(sh_ctx* c) {
   return SH_OK;
 }
 
+// Split master (R25) on n elements in parallel: fp32 -> (hi, lo) planes, and back.
+void split_par(sh_ctx* c, const float* src, uint16_t* hi, uint16_t* lo, int64_t b, int64_t e) {
+  const int nt = std::max(1, std::min(c->n_threads, 16));
+  const int64_t chunk = align_up((e - b + nt - 1) / nt, 16);
+  std::vector<std::thread> ts;
+  for (int64_t x0 = b; x0 < e; x0 += chunk)
+    ts.emplace_back([=] { cpu::split_range(src, hi, lo, x0, std::min(e, x0 + chunk)); });
+  for (auto& t : ts) t.join();
+}
+void join_par(sh_ctx* c, const uint16_t* hi, const uint16_t* lo, float* dst, int64_t b, int64_t e) {
+  const int nt = std::max(1, std::min(c->n_threads, 16));
+  const int64_t chunk = align_up((e - b + nt - 1) / nt, 16);
+  std::vector<std::thread> ts;
+  for (int64_t x0 = b; x0 < e; x0 += chunk)
+    ts.emplace_back([=] { cpu::join_range(hi, lo, dst, x0, std::min(e, x0 + chunk)); });
+  for (auto& t : ts) t.join();
+}
+
 // A kAlign-aligned temporary host buffer (registration, window changes and reads of spilled layers).
 struct AlignedBuf {
   void* p = nullptr;
@@ -1554,6 +1595,7 @@ void release_host_layer(sh_ctx* c, int x) {
   hb = {};
   c->h_master[x] = c->h_m[x] = c->h_v[x] = nullptr;
   c->h_shadow[x] = nullptr;
+  c->h_lo[x] = nullptr;
   auto& sb = c->hshadow[x];
   if (sb.p) {
     host_block_free(sb.p, sb.bytes);
@@ -1596,7 +1638,7 @@ sh_status enable_late_shadow(sh_ctx* c) {
 sh_status ensure_host_layer(sh_ctx* c, int x) {
   if (c->hblocks[x].p || c->hblocks[x].fd >= 0) return SH_OK;
   const int64_t n = c->lay[x].n_pad;
-  size_t bytes = align_up(12 * n + (c->shadow ? 2 * n : 0), 1 << 21);
+  size_t bytes = align_up(12 * n + (c->shadow ? 2 * n : 0), 1 << 21);  // split: [hi | lo | m | v], 12 B
   char* p = nullptr;
   int fd = -1;
   sh_status st = SH_OK;
@@ -1605,12 +1647,14 @@ sh_status ensure_host_layer(sh_ctx* c, int x) {
     auto place = [c, x, n](char* base) {
       if (c->slice_node.empty()) return;
       const int64_t cs = align_up((n + c->W - 1) / c->W, kPad);
-      const int n_arr = c->shadow ? 4 : 3;
+      const int n_arr = c->split ? 4 : c->shadow ? 4 : 3;
       for (int r = 0; r < c->W; ++r) {
         const int64_t lo = std::min(n, (int64_t)r * cs), hi = std::min(n, (int64_t)(r + 1) * cs);
         if (lo >= hi || c->slice_node[r] == numa::kNone) continue;
         for (int a = 0; a < n_arr; ++a) {
-          const int64_t esz = a < 3 ? 4 : 2, off = a < 3 ? 4 * a * n : 12 * n;
+          // arrays: master, m, v[, shadow]  or (split) hi, lo, m, v
+          const int64_t esz = c->split ? (a < 2 ? 2 : 4) : (a < 3 ? 4 : 2);
+          const int64_t off = c->split ? (a < 2 ? 2 * a * n : 4 * (a - 1) * n) : (a < 3 ? 4 * a * n : 12 * n);
           if (numa::bind_range(base + off + esz * lo, (size_t)(esz * (hi - lo)), c->slice_node[r]))
             c->numa_bound.fetch_add(esz * (hi - lo));
         }
@@ -1643,6 +1687,13 @@ sh_status ensure_host_layer(sh_ctx* c, int x) {
   }
   c->host_bytes += bytes;
   float* b = reinterpret_cast<float*>(p);
+  if (c->split) {
+    c->h_shadow[x] = reinterpret_cast<uint16_t*>(p);
+    c->h_lo[x] = reinterpret_cast<uint16_t*>(p) + n;
+    c->h_m[x] = b + n;
+    c->h_v[x] = b + 2 * n;
+    return SH_OK;
+  }
   c->h_master[x] = b;
   c->h_m[x] = b + n;
   c->h_v[x] = b + 2 * n;
@@ -1723,6 +1774,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
   c->gradfree_gen.resize(n_slots, 0);
   c->gradfree_waited.resize(n_slots, 0);
   c->gb_owner.assign(n_slots, -1);  // (engine idle: every pool buffer is free)
+  c->gb_free_seq.assign(n_slots, 0);
   auto pub = std::make_unique<std::atomic<int64_t>[]>(n_slots);
   for (int s = 0; s < n_slots; ++s) pub[s].store(s < old ? c->gradfree_pub[s].load() : 0);
   c->gradfree_pub = std::move(pub);
@@ -1783,7 +1835,14 @@ sh_status apply_window(sh_ctx* c, int w_new) {
         return SH_ERR_OOM_HOST;
       }
       std::memset(t.p, 0, fb);
-      CKC(c, cudaMemcpy(t.b(), c->g[x].master, 4 * n, cudaMemcpyDeviceToHost));
+      if (c->split) {  // region 0 = [hi | lo]
+        std::vector<float> mst(n);
+        CKC(c, cudaMemcpy(mst.data(), c->g[x].master, 4 * n, cudaMemcpyDeviceToHost));
+        uint16_t* h16 = reinterpret_cast<uint16_t*>(t.b());
+        split_par(c, mst.data(), h16, h16 + n, 0, n);
+      } else {
+        CKC(c, cudaMemcpy(t.b(), c->g[x].master, 4 * n, cudaMemcpyDeviceToHost));
+      }
       CKC(c, cudaMemcpy(t.b() + rb, c->g[x].m, 4 * n, cudaMemcpyDeviceToHost));
       CKC(c, cudaMemcpy(t.b() + 2 * rb, c->g[x].v, 4 * n, cudaMemcpyDeviceToHost));
       if (c->shadow) cpu::cast_bf16_range(t.f(), reinterpret_cast<uint16_t*>(t.b() + 3 * rb), 0, n);
@@ -1795,10 +1854,16 @@ sh_status apply_window(sh_ctx* c, int w_new) {
     }
     // every rank holds the same GPU state; each writes its own slice of the (shared) store
     const int64_t lo = c->slo[x], nb = 4 * (c->shi[x] - c->slo[x]);
-    CKC(c, cudaMemcpy(c->h_master[x] + lo, c->g[x].master + lo, nb, cudaMemcpyDeviceToHost));
+    if (c->split) {
+      std::vector<float> mst(c->shi[x] - lo);
+      CKC(c, cudaMemcpy(mst.data(), c->g[x].master + lo, nb, cudaMemcpyDeviceToHost));
+      split_par(c, mst.data() - lo, c->h_shadow[x], c->h_lo[x], lo, c->shi[x]);
+    } else {
+      CKC(c, cudaMemcpy(c->h_master[x] + lo, c->g[x].master + lo, nb, cudaMemcpyDeviceToHost));
+    }
     CKC(c, cudaMemcpy(c->h_m[x] + lo, c->g[x].m + lo, nb, cudaMemcpyDeviceToHost));
     CKC(c, cudaMemcpy(c->h_v[x] + lo, c->g[x].v + lo, nb, cudaMemcpyDeviceToHost));
-    if (c->h_shadow[x]) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], lo, c->shi[x]);
+    if (c->h_shadow[x] && !c->split) cpu::cast_bf16_range(c->h_master[x], c->h_shadow[x], lo, c->shi[x]);
     c->ready[x].store(c->step);
     free_g(c, x);
   }
@@ -1835,12 +1900,25 @@ sh_status apply_window(sh_ctx* c, int w_new) {
       }
       st = spill_file_io(c, false, x, t.p, 3 * rb);
       if (st != SH_OK) return st;
-      CKC(c, cudaMemcpy(c->g[x].master, t.b(), 4 * n, cudaMemcpyHostToDevice));
+      if (c->split) {
+        std::vector<float> mst(n);
+        const uint16_t* h16 = reinterpret_cast<const uint16_t*>(t.b());
+        join_par(c, h16, h16 + n, mst.data(), 0, n);
+        CKC(c, cudaMemcpy(c->g[x].master, mst.data(), 4 * n, cudaMemcpyHostToDevice));
+      } else {
+        CKC(c, cudaMemcpy(c->g[x].master, t.b(), 4 * n, cudaMemcpyHostToDevice));
+      }
       CKC(c, cudaMemcpy(c->g[x].m, t.b() + rb, 4 * n, cudaMemcpyHostToDevice));
       CKC(c, cudaMemcpy(c->g[x].v, t.b() + 2 * rb, 4 * n, cudaMemcpyHostToDevice));
       continue;
     }
-    CKC(c, cudaMemcpy(c->g[x].master, c->h_master[x], 4 * n, cudaMemcpyHostToDevice));
+    if (c->split) {
+      std::vector<float> mst(n);
+      join_par(c, c->h_shadow[x], c->h_lo[x], mst.data(), 0, n);
+      CKC(c, cudaMemcpy(c->g[x].master, mst.data(), 4 * n, cudaMemcpyHostToDevice));
+    } else {
+      CKC(c, cudaMemcpy(c->g[x].master, c->h_master[x], 4 * n, cudaMemcpyHostToDevice));
+    }
     CKC(c, cudaMemcpy(c->g[x].m, c->h_m[x], 4 * n, cudaMemcpyHostToDevice));
     CKC(c, cudaMemcpy(c->g[x].v, c->h_v[x], 4 * n, cudaMemcpyHostToDevice));
   }
@@ -2028,13 +2106,24 @@ sh_status coll_fold_partials(sh_ctx* c, cudaStream_t st) {
 
 // A free pool buffer of at least n elements for layer x (blocks until one's offload is issued).
 int take_grad_buffer(sh_ctx* c, int x, int64_t n) {
+  // among the free buffers (offload issued) prefer one whose offload has already COMPLETED, then the
+  // one released longest ago: taking the buffer of the offload issued last would make the compute
+  // stream wait for that copy (~17 ms for an h4096 layer)
   int b = -1;
   auto pick = [&] {
     b = -1;
+    bool b_done = false;
     for (int k = 0; k < c->n_slots; ++k) {
       if (c->gb_owner[k] != -1 || c->gradfree_pub[k].load() < c->gradfree_gen[k]) continue;
       if (c->byte_ring() && c->slot_cap[k] < n) continue;
-      if (b < 0 || (c->byte_ring() && c->slot_cap[k] < c->slot_cap[b])) b = k;  // best fit
+      const bool done = cudaEventQuery(c->ev_grad_free[k]) == cudaSuccess;
+      if (!done) cudaGetLastError();  // (cudaErrorNotReady is not sticky; clear it anyway)
+      bool better;
+      if (b < 0) better = true;
+      else if (c->byte_ring() && c->slot_cap[k] != c->slot_cap[b]) better = c->slot_cap[k] < c->slot_cap[b];  // best fit
+      else if (done != b_done) better = done;
+      else better = c->gb_free_seq[k] < c->gb_free_seq[b];
+      if (better) b = k, b_done = done;
     }
     return b >= 0;
   };
@@ -2056,6 +2145,7 @@ void release_grad_buffer(sh_ctx* c, int b) {
   {
     std::lock_guard<std::mutex> g(c->smu);
     c->gb_owner[b] = -1;
+    c->gb_free_seq[b] = ++c->gb_free_ctr;
   }
   c->scv.notify_all();
 }
@@ -2354,7 +2444,8 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     for (int t = 0; t < c->n_threads; ++t)
       c->worker_node[t] = numa::worker_node(c->numa_policy, t, c->n_threads, c->numa_gpu);
   }
-  c->shadow = c->bf16 && !(cfg->flags & SH_FLAG_FETCH_FP32);
+  c->shadow = c->bf16 && !(cfg->flags & SH_FLAG_FETCH_FP32) && (cfg->flags & SH_FLAG_BF16_SHADOW);
+  c->split = c->bf16 && !(cfg->flags & SH_FLAG_FETCH_FP32) && !(cfg->flags & SH_FLAG_BF16_SHADOW);
   c->hblocks.assign(c->L, {});
   c->hshadow.assign(c->L, {});
   c->spilled.assign(c->L, 0);
@@ -2375,6 +2466,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->h_m.assign(c->L, nullptr);
   c->h_v.assign(c->L, nullptr);
   c->h_shadow.assign(c->L, nullptr);
+  c->h_lo.assign(c->L, nullptr);
   {
     const int64_t lb = align_up(4 * c->max_pad, 4096);
     const size_t bytes = align_up((int64_t)c->D * lb + 4096, 1 << 21);
@@ -2520,7 +2612,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       c->device_bytes += 4 * (c->max_pad + n);
     }
   }
-  if (c->bf16 && !c->shadow) {  // SH_FLAG_FETCH_FP32: fp32 master staging of the fetches (h2d stream)
+  if (c->bf16 && !c->shadow && !c->split) {  // SH_FLAG_FETCH_FP32: fp32 master staging of the fetches (h2d stream)
     if (cudaMalloc(&c->fp32_stage, c->slot_grad_bytes) != cudaSuccess) {
       cudaGetLastError();
       set_error("sh_init: cudaMalloc of the fp32 fetch staging buffer failed");
@@ -2672,8 +2764,9 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
   } else {
     const int x = layer;
     const int64_t n = c->lay[x].n_pad;
-    std::vector<float> tmp;
+    std::vector<float> tmp, mst;
     float *hp = c->h_master[x], *hm = c->h_m[x], *hv = c->h_v[x];
+    const bool own = c->hblocks[x].p && !(c->shared && c->rank != 0);  // this rank writes the host copy
     AlignedBuf sbuf(c->spilled[x] ? sp_file_bytes(c, x) : 0);
     if (c->spilled[x]) {  // NEXT-2: staged in the file's layout, written with one O_DIRECT request
       if (!sbuf.p) {
@@ -2684,18 +2777,30 @@ sh_status sh_register_host_store(sh_ctx* c, int32_t layer, const float* params, 
       hp = sbuf.f();
       hm = reinterpret_cast<float*>(sbuf.b() + sp_rb(c, x));
       hv = reinterpret_cast<float*>(sbuf.b() + 2 * sp_rb(c, x));
-    } else if (!hp || (c->shared && c->rank != 0)) {  // no (own) host copy to write: stage through a temporary
+      if (c->split) {  // region 0 holds [hi | lo]: the fp32 master goes through a temporary
+        mst.resize(n);
+        hp = mst.data();
+      }
+    } else if (!own) {  // no (own) host copy to write: stage through a temporary
       tmp.resize(3 * n);
       hp = tmp.data();
       hm = hp + n;
       hv = hp + 2 * n;
+    } else if (c->split) {  // split master: the fp32 master through a temporary, m / v in place
+      mst.resize(n);
+      hp = mst.data();
     }
     pack_layer(c->lay[x], params, hp);
     pack_layer(c->lay[x], m, hm);
     pack_layer(c->lay[x], v, hv);
     if (c->shadow && c->h_shadow[x] && hp == c->h_master[x]) cpu::cast_bf16_range(hp, c->h_shadow[x], 0, n);
+    if (c->split && own) split_par(c, hp, c->h_shadow[x], c->h_lo[x], 0, n);
     if (c->spilled[x]) {
       if (c->shadow) cpu::cast_bf16_range(hp, reinterpret_cast<uint16_t*>(sbuf.b() + 3 * sp_rb(c, x)), 0, n);
+      if (c->split) {
+        uint16_t* h16 = reinterpret_cast<uint16_t*>(sbuf.b());
+        split_par(c, hp, h16, h16 + n, 0, n);
+      }
       st = spill_file_io(c, true, x, sbuf.p, sp_file_bytes(c, x));
       if (st != SH_OK) return st;
     }
@@ -3397,11 +3502,19 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
       if (c->bf16) {
         std::vector<uint16_t> b16(n);
         if (c->shadow) std::memcpy(b16.data(), t.b() + 3 * rb, 2 * n);
+        else if (c->split) std::memcpy(b16.data(), t.b(), 2 * n);
         else cpu::cast_bf16_range(t.f(), b16.data(), 0, n);
         unpack_layer_u16(Lx, b16.data(), static_cast<uint16_t*>(dst));
       } else {
         unpack_layer(Lx, t.f(), static_cast<float*>(dst));
       }
+      return SH_OK;
+    }
+    if (what == SH_READ_PARAM && c->split) {
+      std::vector<float> mst(n);
+      const uint16_t* h16 = reinterpret_cast<const uint16_t*>(t.b());
+      join_par(c, h16, h16 + n, mst.data(), 0, n);
+      unpack_layer(Lx, mst.data(), static_cast<float*>(dst));
       return SH_OK;
     }
     unpack_layer(Lx, reinterpret_cast<const float*>(t.b() + what * rb), static_cast<float*>(dst));
@@ -3470,6 +3583,8 @@ sh_status sh_read_layer(sh_ctx* c, int32_t layer, int32_t what, void* dst) {
     const float* src = layer < 0 ? (what == 0 ? c->res_master : what == 1 ? c->res_m : c->res_v)
                                  : (what == 0 ? c->g[layer].master : what == 1 ? c->g[layer].m : c->g[layer].v);
     CKC(c, cudaMemcpy(tmp.data(), src, 4 * n, cudaMemcpyDeviceToHost));
+  } else if (what == SH_READ_PARAM && c->split) {
+    join_par(c, c->h_shadow[layer], c->h_lo[layer], tmp.data(), 0, n);
   } else {
     const float* src = what == 0 ? c->h_master[layer] : what == 1 ? c->h_m[layer] : c->h_v[layer];
     std::memcpy(tmp.data(), src, 4 * n);
@@ -3736,6 +3851,37 @@ sh_status sh_op_cast_bf16_cpu(const float* src, uint16_t* dst16, int64_t n) {
   clear_error();
   if (!src || !dst16 || n < 0) return SH_ERR_INVALID;
   cpu::cast_bf16_range(src, dst16, 0, n);
+  return SH_OK;
+}
+
+sh_status sh_op_master_split_cpu(const float* p, uint16_t* hi, uint16_t* lo, int64_t n) {
+  clear_error();
+  if (!p || !hi || !lo || n < 0) return SH_ERR_INVALID;
+  cpu::split_range(p, hi, lo, 0, n);
+  return SH_OK;
+}
+
+sh_status sh_op_master_join_cpu(const uint16_t* hi, const uint16_t* lo, float* p, int64_t n) {
+  clear_error();
+  if (!p || !hi || !lo || n < 0) return SH_ERR_INVALID;
+  cpu::join_range(hi, lo, p, 0, n);
+  return SH_OK;
+}
+
+sh_status sh_op_adamw_split_cpu(uint16_t* hi, uint16_t* lo, float* m, float* v, const float* g, int64_t n,
+                                int64_t n_decay, const sh_adam_scalars* sc, int32_t use_coef, float coef,
+                                int32_t n_threads) {
+  clear_error();
+  if (!hi || !lo || !m || !v || !g || !sc || !ops_args_ok(n, n_decay, nullptr, 0)) return SH_ERR_INVALID;
+  int T = n_threads > 0 ? n_threads : (int)std::thread::hardware_concurrency();
+  if (T < 1) T = 1;
+  const int64_t per = align_up(n / T + 1, 16);
+  std::vector<std::thread> ts;
+  for (int64_t b = 0; b < n; b += per) {
+    const int64_t e = std::min(n, b + per);
+    ts.emplace_back([=] { cpu::adamw_range_split(hi, lo, m, v, g, b, e, n_decay, *sc, use_coef != 0, coef); });
+  }
+  for (auto& t : ts) t.join();
   return SH_OK;
 }
 

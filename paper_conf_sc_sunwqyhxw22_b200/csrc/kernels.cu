@@ -35,10 +35,13 @@ namespace kern {
 
 namespace {
 
-__device__ __forceinline__ uint32_t rne_bf16_bits(float x) {
+// bf16 rounding of every compute copy: round to nearest, ties away from zero (RNA, R25) --
+// the rounding under which the host store's split master (hi = the compute copy, lo = the low 16
+// bits) is lossless; identical to cpu::rna_bf16.
+__device__ __forceinline__ uint32_t rna_bf16_bits(float x) {
   uint32_t u = __float_as_uint(x);
   if ((u & 0x7fffffffu) > 0x7f800000u) return 0x7fc0u;  // canonical quiet NaN
-  return (u + 0x7fffu + ((u >> 16) & 1u)) >> 16;
+  return (u + 0x8000u) >> 16;
 }
 
 __device__ __forceinline__ float4 ld_stream(const float* p) {
@@ -109,8 +112,8 @@ __global__ void __launch_bounds__(256, kMinBlocks) k2_adamw_kernel(const __grid_
       if (E.out != nullptr) {
         if constexpr (kBf16Out) {
           uint2 o;
-          o.x = rne_bf16_bits(p[u].x) | (rne_bf16_bits(p[u].y) << 16);
-          o.y = rne_bf16_bits(p[u].z) | (rne_bf16_bits(p[u].w) << 16);
+          o.x = rna_bf16_bits(p[u].x) | (rna_bf16_bits(p[u].y) << 16);
+          o.y = rna_bf16_bits(p[u].z) | (rna_bf16_bits(p[u].w) << 16);
           *reinterpret_cast<uint2*>(static_cast<uint16_t*>(E.out) + i) = o;
         } else {
           st_f4(static_cast<float*>(E.out) + i, p[u]);
@@ -234,8 +237,8 @@ __global__ void __launch_bounds__(kBulkThreads, kMinBlocks) k2_adamw_bulk_kernel
       if (E.out != nullptr) {
         if constexpr (kBf16Out) {
           uint2 o;
-          o.x = rne_bf16_bits(p[u].x) | (rne_bf16_bits(p[u].y) << 16);
-          o.y = rne_bf16_bits(p[u].z) | (rne_bf16_bits(p[u].w) << 16);
+          o.x = rna_bf16_bits(p[u].x) | (rna_bf16_bits(p[u].y) << 16);
+          o.y = rna_bf16_bits(p[u].z) | (rna_bf16_bits(p[u].w) << 16);
           *reinterpret_cast<uint2*>(static_cast<uint16_t*>(E.out) + i) = o;
         } else {
           st_f4(static_cast<float*>(E.out) + i, p[u]);
@@ -261,10 +264,10 @@ __global__ void __launch_bounds__(256) k1_cast_kernel(const float* __restrict__ 
     const float4 a = ld_stream(src + 8 * j);
     const float4 b = ld_stream(src + 8 * j + 4);
     uint4 o;
-    o.x = rne_bf16_bits(a.x) | (rne_bf16_bits(a.y) << 16);
-    o.y = rne_bf16_bits(a.z) | (rne_bf16_bits(a.w) << 16);
-    o.z = rne_bf16_bits(b.x) | (rne_bf16_bits(b.y) << 16);
-    o.w = rne_bf16_bits(b.z) | (rne_bf16_bits(b.w) << 16);
+    o.x = rna_bf16_bits(a.x) | (rna_bf16_bits(a.y) << 16);
+    o.y = rna_bf16_bits(a.z) | (rna_bf16_bits(a.w) << 16);
+    o.z = rna_bf16_bits(b.x) | (rna_bf16_bits(b.y) << 16);
+    o.w = rna_bf16_bits(b.z) | (rna_bf16_bits(b.w) << 16);
     *reinterpret_cast<uint4*>(dst + 8 * j) = o;
   }
 }

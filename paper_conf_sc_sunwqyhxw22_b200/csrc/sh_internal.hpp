@@ -101,7 +101,12 @@ void adamw_range(float* p, float* m, float* v, const float* g, uint16_t* out16, 
                  int64_t end, int64_t n_decay, const sh_adam_scalars& sc, bool use_coef,
                  float coef);
 void cast_bf16_range(const float* src, uint16_t* dst, int64_t begin, int64_t end);
-uint16_t rne_bf16(float x);
+uint16_t rna_bf16(float x);
+// Split master (R25): hi = rna_bf16(p), lo = low 16 bits of p; p = (hi << 16) + sext16(lo).
+void adamw_range_split(uint16_t* hi, uint16_t* lo, float* m, float* v, const float* g, int64_t begin, int64_t end,
+                       int64_t n_decay, const sh_adam_scalars& sc, bool use_coef, float coef);
+void split_range(const float* src, uint16_t* hi, uint16_t* lo, int64_t begin, int64_t end);
+void join_range(const uint16_t* hi, const uint16_t* lo, float* dst, int64_t begin, int64_t end);
 bool has_avx512();
 }  // namespace cpu
 

@@ -25,6 +25,7 @@ SH_FLAG_PROFILE, SH_FLAG_POISON, SH_FLAG_DUPLEX, SH_FLAG_SYNC_CPU, SH_FLAG_CPU_H
     SH_FLAG_TEST_DP_PATH, SH_FLAG_KEEP_GRADS, SH_FLAG_ABLATE_ALLOC, SH_FLAG_GROW_LANDING, SH_FLAG_FILL_GPU, \
     SH_FLAG_LATE_SHADOW = 1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048, 4096, 8192, 16384, 32768, 65536
 SH_FLAG_TEST_HOST_COLLECTIVE = 1 << 17
+SH_FLAG_BF16_SHADOW = 1 << 18
 
 # Every symbol include/sh.h declares (tests check the .so exports them all).
 EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", "sh_forward_layer",
@@ -34,7 +35,8 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_op_adamw_gpu", "sh_op_adamw_cpu", "sh_op_cast_bf16_gpu", "sh_op_cast_bf16_cpu",
            "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end", "sh_set_window_ring",
            "sh_executor_grads", "sh_op_exec_reduce_gpu", "sh_numa_topology", "sh_numa_plan",
-           "sh_numa_worker_node", "sh_numa_node_of_pci", "sh_numa_bind_check", "sh_spill_probe")
+           "sh_numa_worker_node", "sh_numa_node_of_pci", "sh_numa_bind_check", "sh_spill_probe", "sh_op_master_split_cpu",
+           "sh_op_master_join_cpu", "sh_op_adamw_split_cpu")
 
 # NUMA placement policies (sh_config.numa_policy, include/sh.h)
 SH_NUMA_AUTO, SH_NUMA_SPLIT, SH_NUMA_LOCAL, SH_NUMA_INTERLEAVE, SH_NUMA_NONE = range(5)
@@ -153,6 +155,8 @@ def lib() -> C.CDLL:
             "sh_numa_worker_node": [i32] * 4, "sh_numa_node_of_pci": [C.c_char_p],
             "sh_numa_bind_check": [i32, i64],
             "sh_spill_probe": [C.c_char_p, i64, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(i32)],
+            "sh_op_master_split_cpu": [vp, vp, vp, i64], "sh_op_master_join_cpu": [vp, vp, vp, i64],
+            "sh_op_adamw_split_cpu": [vp, vp, vp, vp, vp, i64, i64, vp, i32, f32, i32],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -208,6 +212,19 @@ def op_adamw_gpu(p, m, v, g, out16, out32, n, n_decay, sc: AdamScalars, coef=Non
 def op_adamw_cpu(p, m, v, g, out16, n, n_decay, sc: AdamScalars, coef=None, threads=0):
     check(lib().sh_op_adamw_cpu(_ptr(p), _ptr(m), _ptr(v), _ptr(g), _ptr(out16), n, n_decay, C.byref(sc),
                                 0 if coef is None else 1, 1.0 if coef is None else float(coef), threads))
+
+
+def op_master_split_cpu(p, hi, lo, n):
+    check(lib().sh_op_master_split_cpu(_ptr(p), _ptr(hi), _ptr(lo), n))
+
+
+def op_master_join_cpu(hi, lo, p, n):
+    check(lib().sh_op_master_join_cpu(_ptr(hi), _ptr(lo), _ptr(p), n))
+
+
+def op_adamw_split_cpu(hi, lo, m, v, g, n, n_decay, sc: AdamScalars, coef=None, threads=0):
+    check(lib().sh_op_adamw_split_cpu(_ptr(hi), _ptr(lo), _ptr(m), _ptr(v), _ptr(g), n, n_decay, C.byref(sc),
+                                      0 if coef is None else 1, 1.0 if coef is None else float(coef), threads))
 
 
 def op_cast_bf16_gpu(src, dst16, n, stream=None):

@@ -115,6 +115,26 @@ def grad_errors(x_layers, x_res, y_layers, y_res):
     return out, kb / ref
 
 
+def rna_bf16_bits(x: np.ndarray) -> np.ndarray:
+    """Reference bf16 rounding of the engine's compute copies (R25): round to nearest, ties away
+    from zero, canonical NaN 0x7FC0.  Built from torch's round-to-nearest-EVEN (a library routine) plus
+    the textbook tie rule, not from the engine's integer formula: the two agree except on exact ties,
+    where RNA takes the larger magnitude."""
+    import torch
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    u = x.view(np.uint32)
+    out = torch.from_numpy(x).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16).copy()
+    tie = ((u & 0xFFFF) == 0x8000) & ~np.isnan(x)
+    out[tie] = ((u[tie] >> 16) + 1).astype(np.uint16)
+    out[np.isnan(x)] = 0x7FC0
+    return out
+
+
+def rna_bf16_f32(x: np.ndarray) -> np.ndarray:
+    """rna_bf16_bits as float32 values."""
+    return (rna_bf16_bits(x).astype(np.uint32) << 16).view(np.float32)
+
+
 def log_metric(test: str, **vals):
     """Append measured parity values to $SH_PARITY_LOG (JSON lines) -- the record behind the bars."""
     import json

@@ -12,6 +12,7 @@ import pytest
 import torch
 
 import synth
+from tests._common import rna_bf16_bits
 from oracle import gpt_oracle as O
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -83,9 +84,8 @@ def test_cpu_adam_matches_oracle_and_is_thread_invariant(n, n_decay):
         assert (np.abs(cp[dec == d] - rp) <= 1e-6 * scale + 1e-30).all()
         assert np.abs(cm[dec == d] - rm).max() <= 1e-6 * np.abs(rm).max()
         assert np.abs(cv[dec == d] - rv).max() <= 1e-6 * np.abs(rv).max()
-    # the shadow is the bf16 RNE of the new master
-    ref = torch.from_numpy(cp).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
-    assert np.array_equal(c16, ref)
+    # the shadow is the bf16 (RNA, R25) of the new master
+    assert np.array_equal(c16, rna_bf16_bits(cp))
 
 
 def test_cpu_adam_clip_coefficient_scales_gradient():
@@ -101,16 +101,67 @@ def test_cpu_adam_clip_coefficient_scales_gradient():
         assert x.tobytes() == y.tobytes()
 
 
-def test_bf16_rne_cpu_matches_torch_and_canonical_nan():
+def _special_values():
     x = synth.normal(synth.stream_key(1, 2), 1 << 15, 10.0)
     x[:10] = [np.nan, -np.nan, np.inf, -np.inf, 0.0, -0.0, 1e-40, -1e-41, 3.3895314e38, 1.0000001]
-    ties = ((np.arange(1, 200, dtype=np.uint32) << 16) | 0x8000).view(np.float32)
+    ties = ((np.arange(1, 200, dtype=np.uint32) << 16) | 0x8000).view(np.float32)  # exact ties, both parities
     x[10:10 + ties.size] = ties
+    x[300:300 + ties.size] = -ties
+    return x, ties
+
+
+def test_bf16_rna_cpu_matches_reference_and_canonical_nan():
+    x, ties = _special_values()
     d = np.empty(x.size, np.uint16)
     sh.op_cast_bf16_cpu(x, d, x.size)
     assert d[0] == 0x7FC0 and d[1] == 0x7FC0
-    ref = torch.from_numpy(x[2:]).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
-    assert np.array_equal(d[2:], ref)
+    assert np.array_equal(d, rna_bf16_bits(x))
+    # round to nearest: equal to torch's RNE everywhere except exact ties with an even truncation, where
+    # RNA moves away from zero; no result is farther than half a bf16 ulp from x
+    rne = torch.from_numpy(x[2:]).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
+    diff = d[2:] != rne
+    u = x[2:].view(np.uint32)
+    assert np.array_equal(diff, ((u & 0xFFFF) == 0x8000) & ((u >> 16) & 1 == 0))
+    fin = np.isfinite(x[2:]) & np.isfinite((d[2:].astype(np.uint32) << 16).view(np.float32))
+    r = (d[2:].astype(np.uint32) << 16).view(np.float32)[fin].astype(np.float64)
+    ulp = np.abs(np.spacing(r.astype(np.float32)).astype(np.float64)) * 2 ** 16
+    assert (np.abs(r - x[2:][fin]) <= 0.5 * ulp + 1e-45).all()
+
+
+def test_split_master_is_lossless():
+    """R25: hi = the compute copy (RNA), lo = the low 16 bits; join(split(p)) == p for every non-NaN fp32
+    pattern (specials, ties of both parities, random bit patterns), NaN -> NaN."""
+    x, _ = _special_values()
+    rnd = synth.uniform_u64(synth.stream_key(9, 9), 1 << 16).astype(np.uint32).view(np.float32)
+    x = np.concatenate([x, rnd, (np.arange(0, 1 << 16, dtype=np.uint32) | 0x3F800000).view(np.float32)])
+    n = x.size
+    hi, lo, back = np.empty(n, np.uint16), np.empty(n, np.uint16), np.empty(n, np.float32)
+    sh.op_master_split_cpu(x, hi, lo, n)
+    sh.op_master_join_cpu(hi, lo, back, n)
+    assert np.array_equal(hi, rna_bf16_bits(x))
+    assert np.array_equal(lo, (x.view(np.uint32) & 0xFFFF).astype(np.uint16))
+    ok = ~np.isnan(x)
+    assert np.array_equal(back[ok].view(np.uint32), x[ok].view(np.uint32))
+    assert np.isnan(back[~ok]).all()
+
+
+@pytest.mark.parametrize("coef", [None, 0.3])
+def test_cpu_adam_on_split_master_equals_fp32(coef):
+    """The pool's AdamW on a split master == the fp32 AdamW bitwise (joined p, m, v) and hi == its bf16."""
+    n, n_decay = 1 << 16, 1 << 15
+    p, g, m, v = synth.random_adam_state(11, n)
+    sc = sh.adam_scalars(1e-3, 0.9, 0.999, 1e-8, 0.01, 5)
+    a = [x.copy() for x in (p, m, v)]
+    s16 = np.empty(n, np.uint16)
+    sh.op_adamw_cpu(a[0], a[1], a[2], g, s16, n, n_decay, sc, coef=coef, threads=3)
+    hi, lo = np.empty(n, np.uint16), np.empty(n, np.uint16)
+    sh.op_master_split_cpu(p, hi, lo, n)
+    bm, bv = m.copy(), v.copy()
+    sh.op_adamw_split_cpu(hi, lo, bm, bv, g, n, n_decay, sc, coef=coef, threads=2)
+    back = np.empty(n, np.float32)
+    sh.op_master_join_cpu(hi, lo, back, n)
+    assert back.tobytes() == a[0].tobytes() and bm.tobytes() == a[1].tobytes() and bv.tobytes() == a[2].tobytes()
+    assert np.array_equal(hi, s16)
 
 
 def test_op_argument_validation():

@@ -8,9 +8,15 @@ Bar: results bitwise equal to the single-GPU all-resident run for every window, 
 clip mode (the comm-stream ordering must not let K3 / D2H / K2 read a gradient before the
 collective wrote it, nor a slot be refilled before they finished).
 """
+import os
+
 import pytest
 
 from tests._common import TINY, engine_run, engine_state, states_bitwise_equal
+
+# parity runs pin NCCL's algorithm and protocol (DESIGN.md §11): results must not depend on its tuner
+os.environ.setdefault("NCCL_ALGO", "Ring")
+os.environ.setdefault("NCCL_PROTO", "Simple")
 
 pytestmark = pytest.mark.gpu
 

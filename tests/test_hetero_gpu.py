@@ -4,7 +4,7 @@ P:195: models "with a heterogeneous layer structure").  Every ring slot is sized
 unit, so small units must come and go through the same slots as large ones.
 
 The "model" is a toy whose backward writes g = c * a_t + b_k (two IEEE fp32 ops on the compute
-copy c the engine hands out: fp32 master, or its bf16 RNE copy), so the host side can reproduce
+copy c the engine hands out: fp32 master, or its bf16 (RNA) copy), so the host side can reproduce
 every gradient exactly with plain PyTorch CPU ops and the fp64 oracle AdamW
 (oracle.gpt_oracle.adamw_update) gives the reference parameters.  Bars: engine vs oracle per unit
 (∞-norm relative ≤ 1e-5 after 3 steps), and every window / decoupled ring bitwise equal to the
@@ -14,6 +14,7 @@ import pytest
 import torch
 
 from oracle import gpt_oracle as O
+from tests._common import rna_bf16_f32
 
 pytestmark = pytest.mark.gpu
 sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
@@ -104,8 +105,8 @@ def _oracle(bf16):
             for k, x in enumerate(u):
                 a, b = _coef(t, i, k)
                 c = torch.from_numpy(x.astype(np.float32))
-                if bf16:
-                    c = c.to(torch.bfloat16).float()
+                if bf16:  # the engine's compute copy: bf16 round-to-nearest, ties away (R25)
+                    c = torch.from_numpy(rna_bf16_f32(x.astype(np.float32)))
                 g = (c * float(a) + float(b)).numpy().astype(np.float64)
                 p[i][k], m[i][k], v[i][k] = O.adamw_update(x, g, m[i][k], v[i][k], t + 1, opt, bool(wds[i][k]))
     return [np.concatenate(u) for u in p]

@@ -10,6 +10,7 @@ import torch
 
 import synth
 from oracle import gpt_oracle as O
+from tests._common import rna_bf16_bits
 
 pytestmark = pytest.mark.gpu
 
@@ -68,10 +69,12 @@ def test_k2_bitwise_equals_cpu_adam(n, n_decay, use_coef, out):
         assert np.abs(cp[sel][mask] - rp).max() <= 1e-6 * max(1.0, np.abs(rp).max())
 
 
-def test_k1_cast_matches_cpu_rne_and_torch():
+def test_k1_cast_matches_cpu_and_rna_reference():
     n = 1 << 16
     x = synth.normal(synth.stream_key(9, 9), n, 3.0)
     x[:8] = [np.nan, np.inf, -np.inf, 1e-40, -1e-40, 0.0, -0.0, 3.4e38]
+    ties = ((np.arange(1, 200, dtype=np.uint32) << 16) | 0x8000).view(np.float32)
+    x[8:8 + ties.size] = ties  # exact ties of both parities
     dev = torch.device("cuda")
     d16 = torch.empty(n, dtype=torch.int16, device=dev)
     sh.op_cast_bf16_gpu(torch.from_numpy(x).to(dev), d16, n)
@@ -81,8 +84,7 @@ def test_k1_cast_matches_cpu_rne_and_torch():
     g16 = d16.cpu().numpy().view(np.uint16)
     assert np.array_equal(g16, c16)
     assert g16[0] == 0x7FC0
-    ref = torch.from_numpy(x[1:]).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
-    assert np.array_equal(g16[1:], ref)  # torch's RNE (library routine) on non-NaN values
+    assert np.array_equal(g16, rna_bf16_bits(x))  # torch's RNE + the ties-away rule (R25)
 
 
 @pytest.mark.parametrize("n", [8, 1 << 12, (1 << 22) + 8, 50304 * 256])
