@@ -3338,8 +3338,14 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   // 4-deep landing ring stalled BP every 4 layers on the C4 model)
   // (with SH_FLAG_GROW_LANDING a private store grows its landing ring when the autotuner
   // decouples, see sh_autotune_window)
+  // SH_DECOUPLE_ANY=1 (A/B): decouple with the gradient pool alone (the pool and the lowest-first offload
+  // order change the R22 finding, which was measured with slot-bound grad halves and a FIFO queue)
+  static const bool any = [] {
+    const char* e = getenv("SH_DECOUPLE_ANY");
+    return e && e[0] == '1';
+  }();
   o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip &&
-                        (c->D >= c->L || (!c->shared && (c->cfg.flags & SH_FLAG_GROW_LANDING))) ? 1 : 0;
+                        (c->D >= c->L || (!c->shared && (c->cfg.flags & SH_FLAG_GROW_LANDING)) || any) ? 1 : 0;
   o->fp_serial = o->decouple;  // R23: a decoupled (short) ring must also cover the serialised fetch queue
   o->fill_gpu = o->decouple && (c->cfg.flags & SH_FLAG_FILL_GPU) ? 1 : 0;
   return SH_OK;
@@ -3447,7 +3453,9 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   // the landing ring grows into the host RAM the layers joining the GPU set give back -- if that
   // RAM (plus what is free now) cannot hold it, stay coupled
   const int64_t lb = align_up(4 * c->max_pad, 4096);
-  if (ring > 0 && c->D < c->L - w) {
+  const char* any_e = getenv("SH_DECOUPLE_ANY");
+  const bool any = any_e && any_e[0] == '1';  // decouple on the gradient pool alone (no landing growth)
+  if (ring > 0 && c->D < c->L - w && !any) {
     int64_t freed = 0;
     for (int x = c->w; x < w; ++x)
       if (c->hblocks[x].p && c->hblocks[x].fd < 0) freed += (int64_t)c->hblocks[x].bytes;
@@ -3465,7 +3473,7 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   if (st == SH_ERR_OOM_DEVICE) st = sh_set_window_ring(c, w_old, 0);  // restore the warm-up window
   // one landing buffer per host layer: required by a decoupled ring; with SH_FLAG_GROW_LANDING also
   // for a coupled one (the D2H issuer then never waits for the CPU Adam to free a buffer)
-  if (st == SH_OK && (c->ring_cap > 0 || (c->cfg.flags & SH_FLAG_GROW_LANDING)) && c->D < c->L - c->w) {
+  if (st == SH_OK && ((c->ring_cap > 0 && !any) || (c->cfg.flags & SH_FLAG_GROW_LANDING)) && c->D < c->L - c->w) {
     st = grow_landing(c, c->L - c->w);
     if (st != SH_OK) {  // host RAM after all too short: keep the short ring (coupled)
       clear_error();
