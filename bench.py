@@ -4,12 +4,15 @@
   python bench.py --impl reference ...     # the CPU oracle, timed on this box's host cores
 
 Metric (BASELINE.json): samples/s at max trainable size per B200; host-link GB/s vs peak.
-Workload (N=1, default): BASELINE.json configs[3] -- the metric is quoted "at max trainable size
-per B200": a depth-scaled GPT (h 4096, 32 heads, seq 1024, V 50304) whose depth L is the largest the
-host RAM can hold (fp32 master + Adam m, v = 12 B/param in pinned host RAM; fp32 states > 180 GB of
-HBM), bf16 mixed precision, batch 16 per GPU, window auto-tuned by the paper's model (P1/P2) plus
-the eq. 3 CPU-throughput constraint.  `--config c2` is configs[1] (GPT-2 XL-shaped 1.5B), `c3`
-configs[2] (10B), `tiny` configs[0].  A "step" is one full
+Workload (N=1, default `--config c4max`): BASELINE.json configs[3] at the size the metric is quoted
+at, "max trainable size per B200": a depth-scaled GPT (h 4096, 32 heads, seq 1024, V 50304) of
+L = 106 layers (21.6 B params; pinned -- the deepest this pool's 196 GB hosts hold beside a 32-layer
+warm-up GPU set; a smaller host falls back to its own maximum), fp32 p/m/v 259 GB > 180 GB of HBM,
+the host-optimised layers' split fp32 master + Adam m, v in pinned host RAM (12 B/param), bf16 mixed
+precision, batch 16 per GPU, window auto-tuned by the paper's model (P1/P2) plus the eq. 3
+CPU-throughput constraint.  `--config c4` is the same width at L = L_max(host RAM) with a 2-layer
+warm-up set (round-1 default), `c2` configs[1] (GPT-2 XL-shaped 1.5B), `c3` configs[2] (10B), `tiny`
+configs[0].  A "step" is one full
 training iteration through every §8(a) row: prefetch H2D, K1 restage, per-layer K3, grad D2H,
 CPU AdamW, K2 (and, outside the hot path, the GPT block compute that drives it).
 
@@ -49,6 +52,11 @@ CONFIGS = {
                                                 "L = 32 + host-RAM capacity, auto-tuned window"),
 }
 C4MAX_W0 = 32
+# the depth the default line is quoted at: 106 x 4096 = 21.6 B params, fp32 p/m/v 259 GB (> 180 GB of HBM);
+# what the 196 GB host of this pool's B200 boxes holds beside a 32-layer warm-up GPU set (MemAvailable
+# varied 193-200 GB between boxes, giving 106-112 unpinned).  A box with less RAM falls back to its own
+# L_max and says so (config.layers_pinned).
+C4MAX_LAYERS = 106
 # bf16 host layout: the split master (R25: hi plane = the bf16 compute copy, fetched at 2 B/param;
 # 12 B/param of host RAM) for every config; --fetch-fp32 1 / --bf16-shadow select the round-1 layouts
 FETCH_FP32_DEFAULT: set = set()
@@ -243,9 +251,11 @@ def run_reference(args, cfgname):
     b = args.batch or b
     if args.layers:
         L = args.layers
-    if L == 0:  # same depth rule as the CUDA arm (L_max of this host's RAM)
+    if L == 0:  # same depth rule as the CUDA arm (L_max of this host's RAM; c4max pinned)
         L = c4_layers(h, args.grad_ring or 8, w0=C4MAX_W0 if cfgname == "c4max" else 2,
                       ranks_sharing=int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
+        if cfgname == "c4max":
+            L = min(L, C4MAX_LAYERS)
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
@@ -274,7 +284,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="sh", choices=["sh", "reference"])
-    ap.add_argument("--config", default="c4", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="c4max", choices=sorted(CONFIGS))
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--window", type=int, default=-2, help="-2: config default, -1: autotune, L: resident")
     ap.add_argument("--precision", default="bf16", choices=["bf16", "fp32"])
@@ -367,7 +377,7 @@ def main():
         if args.layers:
             L = args.layers
         elif args.config == "c4max":
-            L = c4_layers(h, args.grad_ring or 8, w0=w0h, ranks_sharing=local_world)
+            L = min(C4MAX_LAYERS, c4_layers(h, args.grad_ring or 8, w0=w0h, ranks_sharing=local_world))
         elif not use_shm and world > 1:
             L = c4_layers(h, args.grad_ring or 8, budget=mem_available() // local_world)
         else:
@@ -566,7 +576,9 @@ def main():
         "value": samples, "unit": "samples/s", "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "bf16" if prec == sh.SH_BF16_MIXED else "f32", "data": "synthetic",
-        "config": {"workload": args.config, "description": desc, "layers": L, "hidden": h, "heads": nh, "seq": s,
+        "config": {"workload": args.config, "description": desc, "layers": L,
+                   "layers_pinned": (L == C4MAX_LAYERS) if args.config == "c4max" and not args.layers else None,
+                   "hidden": h, "heads": nh, "seq": s,
                    "vocab": V, "params": mc.n_params(), "batch_per_gpu": b, "global_batch": b * world,
                    "window": r["st1"]["window"], "ring_slots": r["st1"]["n_slots"],
                    "window_mode": ("autotuned (P1/P2" + (" + eq.3 CPU throughput, ring decoupled from the GPU set"

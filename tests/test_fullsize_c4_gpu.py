@@ -1,14 +1,16 @@
 """Parity at the size and in the launch configuration the default `bench.py` times: configs[3] C4
 (h=4096 GPT, L = 82, 16.7 B params, fp32 states 201 GB > 180 GB of HBM, bf16 mixed, batch 16) with
 the window the autotuner picked in profiles/r01_bench_default_c4_v4.json: 53 GPU-optimised layers,
-a decoupled ring of 15 slots (R22), bf16 host shadows, one landing buffer per host layer.
+a decoupled ring of 15 slots (R22), the split host master (R25: the bf16 hi plane is the compute copy
+the prefetch moves), one landing buffer per host layer.
 
 The fp64 oracle cannot run this model, so (as for C2 in test_fullsize_gpu.py) this checks:
   * sampled AdamW at step 2 against the oracle's update, element by element, on the first GPU
     layer (its gradients are in the last-used GPU grad buffer), both ends of the host range and
     the resident set: the right gradients reach the right layer's GPU / CPU update;
   * bitwise equality of every sampled layer's p / m / v with a DIFFERENT split of the same model
-    (44 GPU-optimised layers, ring 21, fp32 fetch + K1 cast instead of bf16 shadows): layers that
+    (44 GPU-optimised layers, ring 21, an fp32 host master fetched at 4 B/param + K1 cast instead of
+    the split master): layers that
     are host-optimised in one run and GPU-optimised in the other (44-52) cross the CPU/GPU Adam
     boundary, so this is the bit-exact-across-windows bar at full size;
   * step-1 loss = ln V + h·0.02²/2 (Gaussian-logit closed form of the tied head at init).
