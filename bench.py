@@ -65,6 +65,10 @@ CPU_HARD_DEFAULT = {"c3", "c4", "c4max"}   # autotune with the eq. 3 CPU-through
 # growth, GPU set filling the HBM a decoupled ring leaves, late bf16 host shadows (C4: 7.30 -> 7.92
 # samples/s, profiles/r01_bench_default_c4_v3.json vs r01_bench_c4_tuned_coupled.json)
 TUNED_DEFAULT = {"c3", "c4"}
+# c4max: no host RAM is left to grow the landing ring, so the decoupled ring is sized as a gradient pool
+# for the backward backlog and the GPU set fills the rest of the HBM (R27; profiles/r02_ab4:
+# 44-47 GPU layers / ring 20-26 beat the coupled 38 / 39 by 3.5 %)
+FILL_DEFAULT = {"c4max"}
 SETTLE_MAX = 10   # at most this many untimed settle steps after the autotuner's window change
 RUNS = 3          # the K timed steps are timed as RUNS consecutive segments (median / geomean reported)
 
@@ -329,6 +333,8 @@ def main():
     args = ap.parse_args()
     if args.config in TUNED_DEFAULT and not args.plain_autotune and args.window in (-2, -1):
         args.grow_landing = args.fill_gpu = args.late_shadow = True
+    if args.config in FILL_DEFAULT and not args.plain_autotune and args.window in (-2, -1):
+        args.fill_gpu = True
     if args.warmup < 3:
         args.warmup = 3
     if args.impl == "reference":

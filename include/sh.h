@@ -268,12 +268,17 @@ typedef struct {
                                   with S(p) = Σ_{i<p} t_fp -- a hard constraint */
   int32_t fill_gpu;            /* decouple: g = the largest GPU-optimised set the memory leaves next to the
                                   ring (instead of the smallest meeting eq. 3) */
+  int32_t landing_buffers;     /* host landing buffers (0: unknown).  With fill_gpu, when no ring meets the
+                                  hard constraints (a link-bound FP, R27): the smallest ring whose gradient
+                                  pool holds the BP backlog ceil(Σ_{k>=g} max(0, 1 - t_bp/t_opt_cpu)) -
+                                  landing_buffers, the GPU set filling the rest (reason 3) */
 } sh_profile;
 
 typedef struct {
   int32_t window;          /* chosen w* */
   int32_t w_max_memory;    /* largest w meeting (1c)/(2c) */
-  int32_t reason;          /* 0: hard+soft met (w < L); 1: hard only; 2: memory fallback */
+  int32_t reason;          /* 0: hard+soft met (w < L); 1: hard only; 2: memory fallback;
+                              3: link-bound FP, pool-sized decoupled ring + filled GPU set (R27) */
   int32_t fp_hard_ok, bp_hard_ok, soft_ok;  /* at the chosen window */
   double eq3_min_slack_ms; /* min_k [Σ_{i<=k}(t_fp+t_bp) + Σ_{i<w} t_opt_gpu - t_opt_cpu_k]  (eq. 3) */
   int32_t eq3_ok;

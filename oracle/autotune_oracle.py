@@ -24,8 +24,14 @@ code shared with the C++ solver (paper_conf_sc_sunwqyhxw22_b200/csrc/autotune.cp
       F(j) = max(F(j-1), S(max(0, j-d))) + t_c2g[j]   (slot of position j-d-1 free, link free)
       hard: F(j) <= S(j) for every host layer j
   fill_gpu (decoupled): g = the largest g >= max(d, g_min) that fits next to the ring, not the smallest
+  link-bound fallback (R27, decoupled + fill_gpu + landing_buffers > 0, no (d, g) meets the hard
+      constraints): the smallest d whose ring d+1 holds the backward backlog
+      B(g) = ceil(sum_{k>=g} max(0, 1 - t_bp[k] / t_opt_cpu[k])) - landing_buffers, g = g_for(d), with the
+      per-window (1b) / (2b) and the CPU constraint met -> reason 3
 """
 from __future__ import annotations
+
+import math
 
 
 def _z(a, n):
@@ -34,7 +40,7 @@ def _z(a, n):
 
 def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
           slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False, cpu_hard=False,
-          cpu_util_max=1.0, decouple=False, fp_serial=False, fill_gpu=False):
+          cpu_util_max=1.0, decouple=False, fp_serial=False, fill_gpu=False, landing_buffers=0):
     """d = prefetch distance (ring d+1 slots), g = GPU-optimised layers [0, g); coupled d = g = m
     (the paper), decoupled g = max(d, smallest g meeting the CPU constraint) (R22)."""
     L = len(t_fp)
@@ -149,6 +155,19 @@ def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None
                 g = g_for(d)
                 if g is not None and hard(d, g):
                     best, reason = (d, g), 1
+                    break
+        if best is None and fill_gpu and landing_buffers > 0:
+            def backlog(g):
+                b = 0.0
+                for k in range(g, L):
+                    if oc[k] > 0:
+                        b += max(0.0, 1.0 - bp[k] / oc[k])
+                return math.ceil(b - 1e-9) - landing_buffers
+
+            for d in range(L + 1):
+                g = g_for(d)
+                if g is not None and d + 1 >= backlog(g) and fp_hard(d, g) and bp_hard(d, g) and cpu_ok(g):
+                    best, reason = (d, g), 3
                     break
     if best is None:
         best = (max(mems), max(mems))

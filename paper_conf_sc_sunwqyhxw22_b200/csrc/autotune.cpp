@@ -145,6 +145,27 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
       const int g = g_for(d);
       if (g >= 0 && hard(d, g)) best_d = d, best_g = g, reason = 1;
     }
+    // R27, link-bound FP (no ring meets the serial form of (1b)): extra slots no longer shorten the FP,
+    // they only hold gradients.  The gradient pool (the ring's grad halves) must absorb the backlog of
+    // a backward pass that outruns the CPU Adam beyond what the host landing buffers take:
+    // B(g) = ceil(Σ_{k>=g} max(0, 1 - t_bp^k / t_opt_cpu^k)) - landing_buffers; every other byte goes to
+    // the GPU-optimised set (fill_gpu).  Smallest d with d + 1 >= B(g_for(d)) meeting the per-window
+    // (1b) / (2b).
+    if (best_d < 0 && P->fill_gpu && P->landing_buffers > 0) {
+      auto backlog = [&](int g) {
+        double b = 0.0;
+        for (int k = g; k < L; ++k) {
+          const double tc = at(P->t_opt_cpu, k);
+          if (tc > 0.0) b += std::max(0.0, 1.0 - at(P->t_bp, k) / tc);
+        }
+        return (int)std::ceil(b - 1e-9) - P->landing_buffers;
+      };
+      for (int d = 0; d <= L && best_d < 0; ++d) {
+        const int g = g_for(d);
+        if (g >= 0 && d + 1 >= backlog(g) && fp_hard(d, g) && bp_hard(d, g) && cpu_ok(g))
+          best_d = d, best_g = g, reason = 3;
+      }
+    }
   }
   if (best_d < 0) best_d = best_g = wmax, reason = 2;
 

@@ -1735,8 +1735,10 @@ sh_status ensure_gbufs(sh_ctx* c, int w) {
 // re-derived (GPU-optimised layers from their HBM masters, host layers from the host store), so
 // the old ring is released BEFORE the new one is allocated (never both at once).  On failure the
 // ring is left unallocated and the caller retries with fewer slots.
-sh_status alloc_ring(sh_ctx* c, int n_slots) {
-  if (c->ring && n_slots <= c->n_slots) return SH_OK;
+// shrink (a decoupled ring, engine idle): allocate exactly n_slots even if fewer than now -- the HBM
+// goes to the GPU-optimised set the solver sized next to it (R27); bookkeeping vectors keep their size.
+sh_status alloc_ring(sh_ctx* c, int n_slots, bool shrink = false) {
+  if (c->ring && (n_slots == c->n_slots || (n_slots < c->n_slots && !shrink))) return SH_OK;
   if (c->ring) {
     cudaDeviceSynchronize();
     cudaFree(c->ring);
@@ -1744,7 +1746,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
     c->ring = nullptr;
     c->ring_alloc = 0;
   }
-  n_slots = std::max(n_slots, c->n_slots);  // events / bookkeeping never shrink
+  if (!shrink) n_slots = std::max(n_slots, c->n_slots);
   char* r = nullptr;
   if (cudaMalloc(&r, c->ring_bytes_for(n_slots)) != cudaSuccess) {
     cudaGetLastError();
@@ -1764,21 +1766,23 @@ sh_status alloc_ring(sh_ctx* c, int n_slots) {
   c->ring_alloc = n_slots;
   c->device_bytes += c->ring_bytes_for(n_slots);
   cudaMemset(r, 0, c->ring_bytes_for(n_slots));
-  const int old = c->n_slots;
-  c->slot_layer.resize(n_slots, -1);
-  c->slot_last_use.resize(n_slots, 0);
-  c->ev_param_free.resize(n_slots, nullptr);
-  c->ev_grad_done.resize(n_slots, nullptr);
-  c->ev_grad_free.resize(n_slots, nullptr);
-  c->ev_reduced.resize(n_slots, nullptr);
-  c->gradfree_gen.resize(n_slots, 0);
-  c->gradfree_waited.resize(n_slots, 0);
-  c->gb_owner.assign(n_slots, -1);  // (engine idle: every pool buffer is free)
-  c->gb_free_seq.assign(n_slots, 0);
-  auto pub = std::make_unique<std::atomic<int64_t>[]>(n_slots);
-  for (int s = 0; s < n_slots; ++s) pub[s].store(s < old ? c->gradfree_pub[s].load() : 0);
+  const int cap = std::max((int)c->slot_layer.size(), n_slots);  // bookkeeping vectors never shrink
+  const int old_cap = (int)c->slot_layer.size();
+  c->slot_layer.assign(cap, -1);  // (a re-allocated ring holds nothing)
+  c->slot_last_use.resize(cap, 0);
+  c->ev_param_free.resize(cap, nullptr);
+  c->ev_grad_done.resize(cap, nullptr);
+  c->ev_grad_free.resize(cap, nullptr);
+  c->ev_reduced.resize(cap, nullptr);
+  c->gradfree_gen.resize(cap, 0);
+  c->gradfree_waited.resize(cap, 0);
+  c->gb_owner.assign(cap, -1);  // (engine idle: every pool buffer is free)
+  c->gb_free_seq.assign(cap, 0);
+  auto pub = std::make_unique<std::atomic<int64_t>[]>(cap);
+  for (int s = 0; s < cap; ++s) pub[s].store(s < old_cap ? c->gradfree_pub[s].load() : 0);
   c->gradfree_pub = std::move(pub);
-  for (int s = old; s < n_slots; ++s) {
+  for (int s = 0; s < cap; ++s) {
+    if (c->ev_param_free[s]) continue;
     for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced})
       if (cudaEventCreateWithFlags(&(*v)[s], cudaEventDisableTiming) != cudaSuccess) {
         set_error("cudaEventCreate failed");
@@ -1878,7 +1882,7 @@ sh_status apply_window(sh_ctx* c, int w_new) {
   }
   // ring first (the old one is released inside), then the joining layers' HBM states (rolled
   // back on failure so the caller can retry with a smaller window)
-  st = alloc_ring(c, c->ring_for(w_new));
+  st = alloc_ring(c, c->ring_for(w_new), c->ring_cap > 0 && !c->byte_ring());
   if (st != SH_OK) {
     clear_ring_map(c);  // a re-allocated ring holds no valid copy
     return st;
@@ -3338,14 +3342,17 @@ sh_status sh_get_profile(sh_ctx* c, sh_profile* o) {
   // 4-deep landing ring stalled BP every 4 layers on the C4 model)
   // (with SH_FLAG_GROW_LANDING a private store grows its landing ring when the autotuner
   // decouples, see sh_autotune_window)
-  // SH_DECOUPLE_ANY=1 (A/B): decouple with the gradient pool alone (the pool and the lowest-first offload
-  // order change the R22 finding, which was measured with slot-bound grad halves and a FIFO queue)
+  // ... or, with SH_FLAG_FILL_GPU, a gradient pool sized for the backward backlog (R27): the pool and the
+  // lowest-first offload order change the R22 finding, which was measured with slot-bound grad halves
+  // and a FIFO queue (SH_DECOUPLE_ANY=1 forces decoupling for A/B runs)
   static const bool any = [] {
     const char* e = getenv("SH_DECOUPLE_ANY");
     return e && e[0] == '1';
   }();
   o->decouple = (c->cfg.flags & SH_FLAG_DECOUPLE) && !c->clip &&
-                        (c->D >= c->L || (!c->shared && (c->cfg.flags & SH_FLAG_GROW_LANDING)) || any) ? 1 : 0;
+                        (c->D >= c->L || (!c->shared && (c->cfg.flags & SH_FLAG_GROW_LANDING)) ||
+                         (c->cfg.flags & SH_FLAG_FILL_GPU) || any) ? 1 : 0;
+  o->landing_buffers = c->D;
   o->fp_serial = o->decouple;  // R23: a decoupled (short) ring must also cover the serialised fetch queue
   o->fill_gpu = o->decouple && (c->cfg.flags & SH_FLAG_FILL_GPU) ? 1 : 0;
   return SH_OK;
@@ -3454,7 +3461,8 @@ sh_status sh_autotune_window(sh_ctx* c, const sh_profile* ov, int32_t* wout) {
   // RAM (plus what is free now) cannot hold it, stay coupled
   const int64_t lb = align_up(4 * c->max_pad, 4096);
   const char* any_e = getenv("SH_DECOUPLE_ANY");
-  const bool any = any_e && any_e[0] == '1';  // decouple on the gradient pool alone (no landing growth)
+  // decouple on the gradient pool alone (no landing growth): forced, or a pool-sized ring (R27)
+  const bool any = (any_e && any_e[0] == '1') || rep.reason == 3;
   if (ring > 0 && c->D < c->L - w && !any) {
     int64_t freed = 0;
     for (int x = c->w; x < w; ++x)

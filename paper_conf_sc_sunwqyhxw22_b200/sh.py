@@ -75,7 +75,7 @@ class Profile(C.Structure):
                 ("slot_bytes", _PI64), ("gstate_bytes", _PI64), ("fixed_bytes", C.c_int64),
                 ("s_avail", C.c_int64), ("duplex", C.c_int32), ("cpu_hard", C.c_int32),
                 ("cpu_util_max", C.c_double), ("decouple", C.c_int32), ("fp_serial", C.c_int32),
-                ("fill_gpu", C.c_int32)]
+                ("fill_gpu", C.c_int32), ("landing_buffers", C.c_int32)]
 
 
 class SolveReport(C.Structure):
@@ -295,7 +295,8 @@ def _dbl(a, n):
 
 def make_profile(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None, t_async=0.0,
                  slot_bytes=None, gstate_bytes=None, fixed_bytes=0, s_avail=2 ** 62, duplex=False,
-                 cpu_hard=False, cpu_util_max=1.0, decouple=False, fp_serial=False, fill_gpu=False):
+                 cpu_hard=False, cpu_util_max=1.0, decouple=False, fp_serial=False, fill_gpu=False,
+                 landing_buffers=0):
     """(Profile, keep-alive arrays) for sh_solve_window / sh_autotune_window."""
     n = len(t_fp)
     keep = {}
@@ -319,6 +320,7 @@ def make_profile(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_c
     prof.decouple = 1 if decouple else 0
     prof.fp_serial = 1 if fp_serial else 0
     prof.fill_gpu = 1 if fill_gpu else 0
+    prof.landing_buffers = int(landing_buffers)
     return prof, keep
 
 
@@ -503,7 +505,7 @@ class Engine:
         n = p.n_layers
         out = {"n_layers": n, "t_async": p.t_async, "s_avail": p.s_avail, "fixed_bytes": p.fixed_bytes,
                "duplex": p.duplex, "cpu_hard": p.cpu_hard, "cpu_util_max": p.cpu_util_max, "decouple": p.decouple,
-               "fp_serial": p.fp_serial, "fill_gpu": p.fill_gpu}
+               "fp_serial": p.fp_serial, "fill_gpu": p.fill_gpu, "landing_buffers": p.landing_buffers}
         for f in ("t_fp", "t_bp", "t_c2g", "t_g2c", "t_stage", "t_opt_gpu", "t_opt_cpu"):
             out[f] = [getattr(p, f)[i] for i in range(n)]
         for f in ("slot_bytes", "gstate_bytes"):

@@ -153,6 +153,29 @@ def test_fill_gpu_takes_the_memory_left_by_the_ring(solve):
     assert small["window"] == 1 and full["window"] == 7         # 2 slots x 10 + 7 x 3 = 41 bytes
 
 
+def test_link_bound_pool_sized_ring(solve):
+    """R27 by hand: homogeneous, t_fp = 1 < t_c2g = 4 (every ring fails the serial form of (1b): the FP is
+    link-bound), t_bp = 3, t_opt_cpu = 30 (BP outruns the CPU: backlog 1 - 3/30 = 0.9 per host layer),
+    1 landing buffer, slots of 1 byte and GPU states of 10 bytes in S_avail = 300, decoupled + fill_gpu.
+    g_for(d) = floor((300 - (d + 1)) / 10); the pool of d + 1 grad halves must hold
+    B = ceil(0.9 (L - g)) - 1; the per-window (1b) needs d >= 4."""
+    L, D = 40, 1
+    prof = homog(L, 1.0, 4.0, 0.0, t_stage=[0.0] * L, t_opt_cpu=[30.0] * L, slot_bytes=[1] * L,
+                 gstate_bytes=[10] * L, s_avail=300)
+    want = None
+    for d in range(L):
+        g = min(L, (300 - (d + 1)) // 10)
+        if d >= 4 and d + 1 >= math.ceil(0.9 * (L - g) - 1e-9) - D:
+            want = (d, g)
+            break
+    assert want == (8, 29)
+    r = solve(**prof, decouple=True, fp_serial=True, fill_gpu=True, landing_buffers=D)
+    assert (r["ring_slots"] - 1, r["window"], r["reason"]) == (want[0], want[1], 3), r
+    # without the landing-buffer count the solver keeps the memory fallback (coupled)
+    r0 = solve(**prof, decouple=True, fp_serial=True, fill_gpu=True)
+    assert r0["reason"] == 2 and r0["ring_slots"] == r0["window"] + 1
+
+
 @pytest.mark.parametrize("seed", range(60))
 def test_random_heterogeneous_matches_bruteforce(seed):
     rng = np.random.default_rng(seed)
@@ -164,7 +187,8 @@ def test_random_heterogeneous_matches_bruteforce(seed):
                 fixed_bytes=int(rng.integers(0, 50)), s_avail=int(rng.integers(100, 3000)),
                 duplex=bool(rng.integers(0, 2)), cpu_hard=bool(rng.integers(0, 2)),
                 cpu_util_max=float(rng.choice([1.0, 0.85, 0.5])), decouple=bool(rng.integers(0, 2)),
-                fp_serial=bool(rng.integers(0, 2)), fill_gpu=bool(rng.integers(0, 2)))
+                fp_serial=bool(rng.integers(0, 2)), fill_gpu=bool(rng.integers(0, 2)),
+                landing_buffers=int(rng.integers(0, 6)))
     want = AO.solve(**{k: (list(v) if isinstance(v, np.ndarray) else v) for k, v in prof.items()})
     if want is None:
         with pytest.raises(sh.ShError):
@@ -175,3 +199,24 @@ def test_random_heterogeneous_matches_bruteforce(seed):
         assert got[k] == want[k], (k, got, want)
     for k in ("eq3_min_slack_ms", "eq4_lhs_ms", "eq4_rhs_ms"):
         assert abs(got[k] - want[k]) <= 1e-9 * max(1.0, abs(want[k])), (k, got, want)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_random_link_bound_profiles_match_bruteforce(seed):
+    """Profiles where the FP is link-bound (t_c2g >> t_fp) and the GPU set fills the memory, so the R27
+    tier decides: the C++ solver agrees with the brute-force oracle."""
+    rng = np.random.default_rng(1000 + seed)
+    L = int(rng.integers(8, 40))
+    prof = dict(t_fp=rng.uniform(0.5, 1.5, L), t_bp=rng.uniform(1.5, 4.5, L), t_c2g=rng.uniform(2.0, 6.0, L),
+                t_g2c=rng.uniform(0, 4, L), t_stage=rng.uniform(0, 0.2, L), t_opt_cpu=rng.uniform(3, 30, L),
+                slot_bytes=[int(rng.integers(1, 4))] * L, gstate_bytes=rng.integers(5, 15, L),
+                s_avail=int(rng.integers(60, 400)), decouple=True, fp_serial=True, fill_gpu=True,
+                landing_buffers=int(rng.integers(1, 8)))
+    want = AO.solve(**{k: (list(v) if isinstance(v, np.ndarray) else v) for k, v in prof.items()})
+    if want is None:
+        with pytest.raises(sh.ShError):
+            sh.solve_window(**prof)
+        return
+    got = sh.solve_window(**prof)
+    for k in ("window", "reason", "w_max_memory", "ring_slots"):
+        assert got[k] == want[k], (k, got, want)

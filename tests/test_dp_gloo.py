@@ -1,5 +1,9 @@
 """Data-parallel host-side logic with world_size 2 on CPU (gloo), no GPU.
 
+(The engine itself at world_size 2 -- sh_init(world_size=2) in two processes bootstrapped with gloo,
+different data per rank, the collectives through a shared host segment, parity with the oracle's
+global batch -- is tests/test_dp_host_gpu.py; sh_init needs a CUDA device.)
+
 On a B200 box each rank averages a layer's gradients with ncclAllReduce(avg) before the offload
  and its CPU AdamW pool updates its replica of the host store.  Here the
 collective is gloo and the update is the same native CPU AdamW (sh_op_adamw_cpu): the test pins
