@@ -26,8 +26,9 @@ code shared with the C++ solver (paper_conf_sc_sunwqyhxw22_b200/csrc/autotune.cp
   fill_gpu (decoupled): g = the largest g >= max(d, g_min) that fits next to the ring, not the smallest
   link-bound fallback (R27, decoupled + fill_gpu + landing_buffers > 0, no (d, g) meets the hard
       constraints): the smallest d whose ring d+1 holds the backward backlog
-      B(g) = ceil(sum_{k>=g} max(0, 1 - t_bp[k] / t_opt_cpu[k])) - landing_buffers, g = g_for(d), with the
-      per-window (1b) / (2b) and the CPU constraint met -> reason 3
+      B(g) = ceil(sum_{k>=g} max(0, 1 - t_bp[k] / t_opt_cpu[k])) - landing_buffers, g = the largest GPU set
+      the memory leaves next to the ring (no CPU constraint: the CPU is then the bottleneck anyway), with
+      the per-window (1b) / (2b) met -> reason 3
 """
 from __future__ import annotations
 
@@ -165,8 +166,9 @@ def solve(t_fp, t_bp, t_c2g, t_g2c, t_stage=None, t_opt_gpu=None, t_opt_cpu=None
                 return math.ceil(b - 1e-9) - landing_buffers
 
             for d in range(L + 1):
-                g = g_for(d)
-                if g is not None and d + 1 >= backlog(g) and fp_hard(d, g) and bp_hard(d, g) and cpu_ok(g):
+                fits = [x for x in range(d, L + 1) if mem(d, x)]
+                g = max(fits) if fits else None
+                if g is not None and d + 1 >= backlog(g) and fp_hard(d, g) and bp_hard(d, g):
                     best, reason = (d, g), 3
                     break
     if best is None:

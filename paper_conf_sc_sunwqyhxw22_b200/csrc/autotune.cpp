@@ -150,7 +150,7 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
     // a backward pass that outruns the CPU Adam beyond what the host landing buffers take:
     // B(g) = ceil(Σ_{k>=g} max(0, 1 - t_bp^k / t_opt_cpu^k)) - landing_buffers; every other byte goes to
     // the GPU-optimised set (fill_gpu).  Smallest d with d + 1 >= B(g_for(d)) meeting the per-window
-    // (1b) / (2b).
+    // (1b) / (2b), g = the largest GPU set the memory leaves next to the ring.
     if (best_d < 0 && P->fill_gpu && P->landing_buffers > 0) {
       auto backlog = [&](int g) {
         double b = 0.0;
@@ -160,10 +160,13 @@ extern "C" sh_status sh_solve_window(const sh_profile* P, sh_solve_report* R) {
         }
         return (int)std::ceil(b - 1e-9) - P->landing_buffers;
       };
+      // (no CPU constraint here: when no ring meets the hard constraints the CPU Adam is typically the
+      // bottleneck too, and then the largest GPU set is what relieves it)
       for (int d = 0; d <= L && best_d < 0; ++d) {
-        const int g = g_for(d);
-        if (g >= 0 && d + 1 >= backlog(g) && fp_hard(d, g) && bp_hard(d, g) && cpu_ok(g))
-          best_d = d, best_g = g, reason = 3;
+        int g = -1;
+        for (int x = d; x <= L; ++x)
+          if (mem_ok(d, x)) g = x;
+        if (g >= 0 && d + 1 >= backlog(g) && fp_hard(d, g) && bp_hard(d, g)) best_d = d, best_g = g, reason = 3;
       }
     }
   }

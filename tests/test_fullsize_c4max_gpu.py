@@ -1,14 +1,14 @@
 """Parity at the size and in the launch configuration the DEFAULT `bench.py` times: c4max, BASELINE.json
 configs[3] at "max trainable size per B200" -- h = 4096 GPT, L = 106 (21.6 B params, fp32 p/m/v 259 GB
-> 180 GB of HBM), bf16 mixed, batch 16, the configuration the autotuner settles on (38 GPU-optimised
-layers, ring 39; profiles/r02_bench_c4max_*.json), 8 host landing buffers, the split host master
-(R25) and the lowest-first offload order (R26).
+> 180 GB of HBM), bf16 mixed, batch 16, the configuration the autotuner settles on (R27: 45
+GPU-optimised layers, a decoupled ring of 26 slots; profiles/r02_bench_default_c4max*.json), 8 host
+landing buffers, the split host master (R25) and the lowest-first offload order (R26).
 
 The fp64 oracle cannot run this model, so (as test_fullsize_c4_gpu.py does for the 82-layer C4):
   * sampled AdamW at step 2 against the oracle's update, element by element, on a GPU-optimised layer
-    (layer 0: its gradients are in the last-used GPU grad buffer), on the host layers whose gradients
-    are still in one of the 8 landing buffers after the step (at least one of the candidates at both
-    ends of the host range; the scheduler offloads the high layers last) and on the resident set --
+    (layer 0: its gradients are in the last-used GPU grad buffer), on every host layer whose gradients
+    are still in one of the 8 landing buffers after the step (which ones depends on the offload
+    timing: the step-1 state of every host layer is sampled) and on the resident set --
     the right gradients reach the right layer's GPU / CPU update at full size;
   * the split master at full size: the compute copy the engine hands out (SH_READ_COMPUTE) is the
     RNA bf16 of the fp32 master it reconstructs (SH_READ_PARAM), for a host layer and a GPU layer;
@@ -27,9 +27,9 @@ pytestmark = [pytest.mark.gpu, pytest.mark.slow]
 
 sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
 C4MAX = dict(L=106, h=4096, nh=32, s=1024, V=50304, b=16)
-G_LAYERS, RING, LANDING = 38, 39, 8
-SAMPLED = (0, 38, 39, 104, 105, -1)
-HOST = (38, 39, 104, 105)
+G_LAYERS, RING, LANDING = 45, 26, 8
+HOST = tuple(range(G_LAYERS, 106))
+SAMPLED = (0,) + HOST + (-1,)
 N_SAMPLE = 4096
 
 
@@ -62,7 +62,7 @@ def run():
                     except sh.ShError as e:  # a host layer's landing buffer was reused in this step
                         assert e.status == sh.SH_ERR_STATE and x in HOST, (x, e)
         out["split"] = {x: (tr.engine.read_layer(x, sh.SH_READ_PARAM), tr.engine.read_layer(x, sh.SH_READ_COMPUTE))
-                        for x in (0, 105)}
+                        for x in (0, G_LAYERS, 105)}
         out["stats"] = tr.engine.stats()
     finally:
         tr.close()
