@@ -399,6 +399,7 @@ struct sh_ctx {
   std::vector<int64_t> slot_last_use;  // global position of the occupant's latest compute (LRU tie-break)
   int64_t pos_clock = 0;
   std::vector<cudaEvent_t> ev_param_free, ev_grad_done, ev_grad_free, ev_reduced;
+  std::vector<cudaEvent_t> ev_k3_buf;  // per pool buffer: after the K3 of the layer it holds (D2H issuer)
   std::vector<int64_t> gradfree_gen, gradfree_waited;  // per gradient-pool buffer (slot index)
   std::unique_ptr<std::atomic<int64_t>[]> gradfree_pub;
   std::vector<cudaEvent_t> ev_arrive;
@@ -1774,6 +1775,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots, bool shrink = false) {
   c->ev_grad_done.resize(cap, nullptr);
   c->ev_grad_free.resize(cap, nullptr);
   c->ev_reduced.resize(cap, nullptr);
+  c->ev_k3_buf.resize(cap, nullptr);
   c->gradfree_gen.resize(cap, 0);
   c->gradfree_waited.resize(cap, 0);
   c->gb_owner.assign(cap, -1);  // (engine idle: every pool buffer is free)
@@ -1783,7 +1785,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots, bool shrink = false) {
   c->gradfree_pub = std::move(pub);
   for (int s = 0; s < cap; ++s) {
     if (c->ev_param_free[s]) continue;
-    for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced})
+    for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced, &c->ev_k3_buf})
       if (cudaEventCreateWithFlags(&(*v)[s], cudaEventDisableTiming) != cudaSuccess) {
         set_error("cudaEventCreate failed");
         return SH_ERR_CUDA;
@@ -2158,6 +2160,7 @@ void release_grad_buffer(sh_ctx* c, int b) {
 // buffer; K3 (the layer's sum of squares, needed by sh_step) is enqueued for every pending layer in
 // backward order as soon as it is posted, before any wait for a landing buffer.
 void d2h_pump(sh_ctx* c) {
+  static const bool dbg = getenv("SH_DEBUG_PUMP") != nullptr;
   for (;;) {
     std::vector<sh_ctx::PendD2H*> k3todo;
     {
@@ -2165,6 +2168,7 @@ void d2h_pump(sh_ctx* c) {
       for (auto& p : c->pend)
         if (!p.k3_done) k3todo.push_back(&p);  // deque elements do not move on push_back
     }
+    if (dbg && !k3todo.empty()) fprintf(stderr, "[pump %.1f] k3 x%zu first L%d\n", now_ms(), k3todo.size(), k3todo[0]->x);
     for (auto* p : k3todo) {
       if (p->k3_on_d2h) {  // on its own stream so the copy engine does not queue behind it
         ProfSet* P = static_cast<ProfSet*>(p->prof);
@@ -2175,6 +2179,7 @@ void d2h_pump(sh_ctx* c) {
           CKA(c, cudaEventRecord(P->k31[p->x], c->k3s));
           P->rec_k3[p->x] = 1;
         }
+        CKA(c, cudaEventRecord(c->ev_k3_buf[p->b], c->k3s));
         CKA(c, cudaEventRecord(c->ev_k3_last, c->k3s));
         c->k3_pub.store(p->gen);
       }
@@ -2187,6 +2192,7 @@ void d2h_pump(sh_ctx* c) {
       if (c->pend.empty()) return;
     }
     // a free landing buffer, or new posts whose K3 must go out first
+    if (dbg) fprintf(stderr, "[pump %.1f] wait landing (free %zu)\n", now_ms(), c->land_free.size());
     if (!state_wait(c, [&] { return !c->land_free.empty() || c->pend_posted.load() > c->pend_k3.load(); },
                     "host landing buffer")) {
       std::lock_guard<std::mutex> g(c->dmu);
@@ -2205,17 +2211,27 @@ void d2h_pump(sh_ctx* c) {
     sh_ctx::PendD2H p{};
     {
       std::lock_guard<std::mutex> g(c->dmu);
-      // lowest layer first -- except with a shared store, where a slice update needs every rank's
-      // offload of the layer: all ranks then keep the backward (POST) order, so the landing buffers
-      // every rank holds always wait for the same layers
+      // lowest layer first among the layers whose gradients are COMPUTED (the driver posts layers well
+      // ahead of the GPU: offloading the lowest posted one would park the copy engine behind that
+      // layer's backward while earlier gradients wait), else the earliest posted -- except with a shared
+      // store, where a slice update needs every rank's offload of the layer: all ranks then keep the
+      // backward (POST) order, so the landing buffers every rank holds always wait for the same layers
       auto best = c->pend.end();
+      bool best_ready = false;
       for (auto it = c->pend.begin(); it != c->pend.end(); ++it) {
         if (!it->k3_done) continue;
         if (c->shared || c->d2h_fifo) {
           best = it;
           break;
         }
-        if (best == c->pend.end() || it->step < best->step || (it->step == best->step && it->x < best->x)) best = it;
+        const bool ready = cudaEventQuery(it->ready) == cudaSuccess;
+        if (!ready) cudaGetLastError();
+        if (best == c->pend.end()) {
+          best = it, best_ready = ready;  // the earliest posted (deque order)
+          continue;
+        }
+        if (ready && (!best_ready || it->step < best->step || (it->step == best->step && it->x < best->x)))
+          best = it, best_ready = true;
       }
       if (best == c->pend.end()) {  // only fresh posts: their K3 first
         std::lock_guard<std::mutex> g2(c->smu);
@@ -2226,6 +2242,7 @@ void d2h_pump(sh_ctx* c) {
       c->pend.erase(best);
     }
     maybe_delay(c->cfg.flags);
+    if (dbg) fprintf(stderr, "[pump %.1f] d2h L%d landing %d\n", now_ms(), p.x, k);
     ProfSet* P = static_cast<ProfSet*>(p.prof);
     const int x = p.x;
     c->landing_owner[k] = x;
@@ -2238,9 +2255,8 @@ void d2h_pump(sh_ctx* c) {
       CKA(c, cudaEventRecord(P->g2c1[x], c->d2h));
       P->rec_g2c[x] = 1;
     }
-    // the buffer is reusable after the copy and this layer's K3 (k3s is in order: the latest K3
-    // event covers it)
-    if (p.k3_on_d2h) CKA(c, cudaStreamWaitEvent(c->d2h, c->ev_k3_last, 0));
+    // the buffer is reusable after the copy and this layer's K3
+    if (p.k3_on_d2h) CKA(c, cudaStreamWaitEvent(c->d2h, c->ev_k3_buf[p.b], 0));
     CKA(c, cudaEventRecord(c->ev_grad_free[p.b], c->d2h));
     CKA(c, cudaLaunchHostFunc(c->d2h, landed_cb, new Landed{c, x, p.step, k, p.sc}));
     c->d2h_bytes += 4 * (p.hi - p.lo);
@@ -3714,7 +3730,8 @@ sh_status sh_destroy(sh_ctx* c) {
   if (c->ring) cudaFree(c->ring);
   if (c->res_master) cudaFree(c->res_master);
   if (c->partials) cudaFree(c->partials);
-  for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced, &c->ev_arrive, &c->ev_upd})
+  for (auto* v : {&c->ev_param_free, &c->ev_grad_done, &c->ev_grad_free, &c->ev_reduced, &c->ev_k3_buf, &c->ev_arrive,
+                  &c->ev_upd})
     for (auto e : *v)
       if (e) cudaEventDestroy(e);
   for (auto& P : c->prof) {
