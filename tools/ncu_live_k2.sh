@@ -4,7 +4,7 @@
 # the HBM and the host RAM are full, and ncu's save/restore of the kernel's in-place p / m / v for the
 # replay passes got the process killed.  Writes gpurun_out/ncu_live_k2.{ncu-rep,csv,log}.
 mkdir -p gpurun_out
-timeout 1500 ncu --set full --clock-control none --import-source on -k regex:k2_adamw_kernel --launch-skip 60 -c 1 \
+timeout 1500 ncu --set full --clock-control none --import-source on -k regex:k2_adamw_kernel --launch-skip 20 -c 1 \
     -o gpurun_out/ncu_live_k2 -f python bench.py --config c2 --steps 3 --no-e2e --no-resident --no-cpu-baseline \
     > gpurun_out/ncu_live_k2.log 2>&1
 ncu -i gpurun_out/ncu_live_k2.ncu-rep --page raw --csv \
