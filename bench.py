@@ -328,6 +328,10 @@ def main():
     ap.add_argument("--sync-cpu", action="store_true",
                     help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
     ap.add_argument("--spill-evict", action="store_true", help="NEXT-2: drop spilled layers from the page cache")
+    ap.add_argument("--dp-test-host-collective", action="store_true",
+                    help="TEST ONLY (N > 1 ranks on ONE GPU): gloo bootstrap, every rank on cuda:0, the engine's "
+                         "collectives through SH_FLAG_TEST_HOST_COLLECTIVE -- exercises the multi-rank bench "
+                         "orchestration where NCCL cannot run (not a performance number)")
     ap.add_argument("--executors", type=int, default=1,
                     help="NEXT-3: K multi-stream executors (micro-batches of batch/K on K streams, PAPER.md:227-242)")
     args = ap.parse_args()
@@ -350,19 +354,28 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    host_coll = args.dp_test_host_collective and world > 1
+    if host_coll:
+        local = 0  # every rank on the one GPU
     torch.cuda.set_device(local)
+    tdev = torch.device("cpu") if host_coll else torch.device("cuda", local)  # torch.distributed tensors
+
     def fresh_nccl_id():
         # an ncclUniqueId bootstraps ONE communicator: every engine context (the timed run, the
         # resident-fit run) gets its own, created on rank 0 and broadcast over torch.distributed
-        idt = torch.zeros(128, dtype=torch.uint8, device="cuda")
+        idt = torch.zeros(128, dtype=torch.uint8, device=tdev)
         if rank == 0:
-            idt.copy_(torch.frombuffer(bytearray(sh.nccl_unique_id()), dtype=torch.uint8))
+            raw = os.urandom(128) if host_coll else sh.nccl_unique_id()
+            idt.copy_(torch.frombuffer(bytearray(raw), dtype=torch.uint8))
         dist.broadcast(idt, 0)
         return bytes(idt.cpu().numpy().tobytes())
 
     nccl_id = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if host_coll:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         nccl_id = fresh_nccl_id()
 
     L, h, nh, s, V, b0, w0, desc = CONFIGS[args.config]
@@ -373,7 +386,8 @@ def main():
     local_world = int(os.environ.get("LOCAL_WORLD_SIZE", world))
     use_shm = world > 1
     if world > 1:
-        flag = torch.tensor([1 if shm_free() > 0.8 * mem_available() else 0], dtype=torch.int64, device="cuda")
+        flag = torch.tensor([1 if host_coll or shm_free() > 0.8 * mem_available() else 0], dtype=torch.int64,
+                            device=tdev)
         dist.broadcast(flag, 0)
         use_shm = bool(flag.item())
     if args.layers and L != 0:
@@ -389,7 +403,7 @@ def main():
         else:
             L = c4_layers(h, args.grad_ring or 8, ranks_sharing=local_world)
         if world > 1:  # every rank must build the same model
-            lt = torch.tensor([L], dtype=torch.int64, device="cuda")
+            lt = torch.tensor([L], dtype=torch.int64, device=tdev)
             dist.broadcast(lt, 0)
             L = int(lt.item())
     prec = sh.SH_BF16_MIXED if args.precision == "bf16" else sh.SH_FP32
@@ -427,9 +441,10 @@ def main():
             (sh.SH_FLAG_SPILL_EVICT if args.spill_evict else 0) | \
             (sh.SH_FLAG_ABLATE_ALLOC if args.ablate_alloc else 0) | (sh.SH_FLAG_SYNC_CPU if args.sync_cpu else 0) | \
             (sh.SH_FLAG_GROW_LANDING if args.grow_landing else 0) | (sh.SH_FLAG_FILL_GPU if args.fill_gpu else 0) | \
-            (sh.SH_FLAG_LATE_SHADOW if args.late_shadow else 0) | (sh.SH_FLAG_BF16_SHADOW if args.bf16_shadow else 0)
+            (sh.SH_FLAG_LATE_SHADOW if args.late_shadow else 0) | (sh.SH_FLAG_BF16_SHADOW if args.bf16_shadow else 0) | \
+            (sh.SH_FLAG_TEST_HOST_COLLECTIVE if host_coll else 0)
         tr = StrongholdTrainer(mc, batch=b, window=window, precision=prec, device=local,
-                               flags=flags, world_size=world, rank=rank, nccl_id=nid,
+                               flags=flags, world_size=world, rank=rank, nccl_id=None if host_coll else nid,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm,
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
                                attention=args.attention, executors=args.executors, ring_slots=args.ring,
@@ -546,7 +561,7 @@ def main():
     def gmax(x):
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        t = torch.tensor([x], dtype=torch.float64, device=tdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
@@ -591,7 +606,7 @@ def main():
                                                          if cpu_hard else "") + ")") if w == -1 else "fixed",
                    "precision": "bf16_mixed" if prec else "fp32",
                    "gpt_driver_attention": r["attn"],
-                   "parallelism": f"dp{world}",
+                   "parallelism": f"dp{world}" + (" (TEST: host collective, all ranks on one GPU)" if host_coll else ""),
                    "executors": args.executors,
                    "ablation": [k for k, v in (("alloc", args.ablate_alloc), ("sync_cpu", args.sync_cpu),
                                                ("cpu_threads", args.cpu_threads)) if v] or None,
