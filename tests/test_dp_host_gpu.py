@@ -103,6 +103,7 @@ def oracle_global():
     (1, sh.SH_FP32, 0.5, 0),                      # clipping: the coefficient needs the folded global norm
     (1, sh.SH_BF16_MIXED, 0.0, 0),
     (1, sh.SH_BF16_MIXED, 0.0, sh.SH_FLAG_SLICE_FETCH | sh.SH_FLAG_FETCH_FP32),
+    (2, sh.SH_BF16_MIXED, 0.0, sh.SH_FLAG_SLICE_FETCH),  # slices of the split master's hi plane
 ])
 def test_dp_two_ranks_different_data_vs_oracle(oracle_global, window, precision, clip, extra):
     st, olosses, onorms = oracle_global[clip]
