@@ -324,7 +324,10 @@ def main():
     ap.add_argument("--late-shadow", action="store_true", help="fp32-fetch mode: bf16 host shadows after the autotune")
     ap.add_argument("--plain-autotune", action="store_true",
                     help="c3/c4: autotune without --grow-landing/--fill-gpu/--late-shadow (the round-1 default)")
-    ap.add_argument("--ring", type=int, default=0, help="fixed ring size (prefetch distance + 1) with a fixed --window")
+    ap.add_argument("--ring", type=int, default=0, help="ring size (prefetch distance + 1): with a fixed --window, or the "
+                                                        "warm-up ring of an autotuned run")
+    ap.add_argument("--warmup-window", type=int, default=0,
+                    help="GPU-optimised layers during an autotuned run's warm-up (c4max default: %d)" % C4MAX_W0)
     ap.add_argument("--sync-cpu", action="store_true",
                     help="Fig. 14 ablation: one CPU Adam at a time, inline when a layer's grads land (no pool)")
     ap.add_argument("--spill-evict", action="store_true", help="NEXT-2: drop spilled layers from the page cache")
@@ -397,7 +400,8 @@ def main():
         if args.layers:
             L = args.layers
         elif args.config == "c4max":
-            L = min(C4MAX_LAYERS, c4_layers(h, args.grad_ring or 8, w0=w0h, ranks_sharing=local_world))
+            L = min(C4MAX_LAYERS, c4_layers(h, args.grad_ring or 8, w0=args.warmup_window or w0h,
+                                            ranks_sharing=local_world))
         elif not use_shm and world > 1:
             L = c4_layers(h, args.grad_ring or 8, budget=mem_available() // local_world)
         else:
@@ -449,7 +453,8 @@ def main():
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
                                attention=args.attention, executors=args.executors, ring_slots=args.ring,
                                spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9),
-                               warmup_window=C4MAX_W0 if args.config == "c4max" and window == -1 else 0)
+                               warmup_window=(args.warmup_window or (C4MAX_W0 if args.config == "c4max" else 0))
+                               if window == -1 else 0)
         attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
