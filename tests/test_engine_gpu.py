@@ -136,6 +136,27 @@ def test_fetch_fp32_mode_bitwise_equals_resident():
             tr.close()
 
 
+def test_host_layouts_bitwise_equal_and_fetch_bytes():
+    """The three bf16 host layouts train bitwise alike (the resident run has no host layout at all):
+    split master (default, R25; fetch = hi plane, 2 B/param), fp32 master + bf16 shadow
+    (SH_FLAG_BF16_SHADOW; 2 B/param), fp32 master (SH_FLAG_FETCH_FP32; 4 B/param + K1 cast).  Every
+    prefetch of the split layout moves exactly the bf16 compute copy."""
+    L, w = TINY["L"], 1
+    ref, _, _ = engine_run(TINY, STEPS, L, sh.SH_BF16_MIXED)
+    ref_state = engine_state(ref)
+    ref.close()
+    h2d = {}
+    for name, flags in (("split", 0), ("shadow", sh.SH_FLAG_BF16_SHADOW), ("fp32", sh.SH_FLAG_FETCH_FP32)):
+        tr, _, _ = engine_run(TINY, STEPS, w, sh.SH_BF16_MIXED, flags=flags | sh.SH_FLAG_POISON)
+        try:
+            ok, what = states_bitwise_equal(engine_state(tr), ref_state)
+            assert ok, f"{name}: {what}"
+            h2d[name] = tr.engine.stats()["h2d_bytes"]
+        finally:
+            tr.close()
+    assert h2d["split"] == h2d["shadow"] and h2d["fp32"] == 2 * h2d["split"], h2d
+
+
 def test_window_change_mid_run_bitwise():
     L = TINY["L"]
     ref, _, _ = engine_run(TINY, 4, L, sh.SH_BF16_MIXED)
