@@ -6,9 +6,9 @@
 Metric (BASELINE.json): samples/s at max trainable size per B200; host-link GB/s vs peak.
 Workload (N=1, default `--config c4max`): BASELINE.json configs[3] at the size the metric is quoted
 at, "max trainable size per B200": a depth-scaled GPT (h 4096, 32 heads, seq 1024, V 50304) of
-L = 106 layers (21.6 B params; pinned -- the deepest this pool's 196 GB hosts hold beside a 32-layer
-warm-up GPU set; a smaller host falls back to its own maximum), fp32 p/m/v 259 GB > 180 GB of HBM,
-the host-optimised layers' split fp32 master + Adam m, v in pinned host RAM (12 B/param), bf16 mixed
+L = 112 layers (22.8 B params; pinned -- what this pool's 196 GB hosts and the HBM hold together, warming
+up with 42 GPU-optimised layers beside a 26-slot ring; a smaller host falls back to its own maximum),
+fp32 p/m/v 273 GB > 180 GB of HBM, the host-optimised layers' split fp32 master + Adam m, v in pinned host RAM (12 B/param), bf16 mixed
 precision, batch 16 per GPU, window auto-tuned by the paper's model (P1/P2) plus the eq. 3
 CPU-throughput constraint.  `--config c4` is the same width at L = L_max(host RAM) with a 2-layer
 warm-up set (round-1 default), `c2` configs[1] (GPT-2 XL-shaped 1.5B), `c3` configs[2] (10B), `tiny`
@@ -46,17 +46,19 @@ CONFIGS = {
     # (fp32-fetch mode, no bf16 shadow)
     "c4": (0, 4096, 32, 1024, 50304, 16, -1, "BASELINE configs[3]: depth-scaled GPT h4096, L = L_max(host RAM), "
                                             "fp32 states > 180 GB HBM, auto-tuned window"),
-    # the largest model the host RAM holds once GPU-optimised layers keep no host copy: warm up with
-    # the first C4MAX_W0 layers already in HBM, so only layers >= C4MAX_W0 need host blocks
-    "c4max": (0, 4096, 32, 1024, 50304, 16, -1, "max trainable size in host RAM: depth-scaled GPT h4096, "
-                                                "L = 32 + host-RAM capacity, auto-tuned window"),
+    # the largest model HBM + host RAM hold together: GPU-optimised layers keep no host copy, so the run
+    # warms up with the first C4MAX_W0 layers already in HBM beside a decoupled C4MAX_RING0-slot ring
+    # (the configuration R27 settles on) and only layers >= C4MAX_W0 need host blocks
+    "c4max": (0, 4096, 32, 1024, 50304, 16, -1, "max trainable size: depth-scaled GPT h4096, 112 layers "
+                                                "(22.8 B params), auto-tuned window"),
 }
-C4MAX_W0 = 32
-# the depth the default line is quoted at: 106 x 4096 = 21.6 B params, fp32 p/m/v 259 GB (> 180 GB of HBM);
-# what the 196 GB host of this pool's B200 boxes holds beside a 32-layer warm-up GPU set (MemAvailable
-# varied 193-200 GB between boxes, giving 106-112 unpinned).  A box with less RAM falls back to its own
-# L_max and says so (config.layers_pinned).
-C4MAX_LAYERS = 106
+C4MAX_W0 = 42
+C4MAX_RING0 = 26
+# the depth the default line is quoted at: 112 x 4096 = 22.8 B params, fp32 p/m/v 273 GB (> 180 GB of HBM);
+# 70 host layers (170 GB of pinned state) beside the 42-layer warm-up GPU set on this pool's 196 GB hosts
+# (118 layers do not fit the HBM next to the activations; profiles/r02_ab_c4max_L112.txt).  A box with
+# less RAM falls back to its own L_max and says so (config.layers_pinned).
+C4MAX_LAYERS = 112
 # bf16 host layout: the split master (R25: hi plane = the bf16 compute copy, fetched at 2 B/param;
 # 12 B/param of host RAM) for every config; --fetch-fp32 1 / --bf16-shadow select the round-1 layouts
 FETCH_FP32_DEFAULT: set = set()
@@ -451,7 +453,8 @@ def main():
                                flags=flags, world_size=world, rank=rank, nccl_id=None if host_coll else nid,
                                cpu_threads=cpu_threads, grad_ring_depth=grad_ring, shm_name=shm,
                                warmup_steps=W if window == -1 else 5, init_threads=args.init_threads,
-                               attention=args.attention, executors=args.executors, ring_slots=args.ring,
+                               attention=args.attention, executors=args.executors,
+                               ring_slots=args.ring or (C4MAX_RING0 if args.config == "c4max" and window == -1 else 0),
                                spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9),
                                warmup_window=(args.warmup_window or (C4MAX_W0 if args.config == "c4max" else 0))
                                if window == -1 else 0)

@@ -1,8 +1,8 @@
 """Parity at the size and in the launch configuration the DEFAULT `bench.py` times: c4max, BASELINE.json
-configs[3] at "max trainable size per B200" -- h = 4096 GPT, L = 106 (21.6 B params, fp32 p/m/v 259 GB
-> 180 GB of HBM), bf16 mixed, batch 16, the configuration the autotuner settles on (R27: 45
-GPU-optimised layers, a decoupled ring of 26 slots; profiles/r02_bench_default_c4max*.json), 8 host
-landing buffers, the split host master (R25) and the lowest-first offload order (R26).
+configs[3] at "max trainable size per B200" -- h = 4096 GPT, L = 112 (22.8 B params, fp32 p/m/v 273 GB
+> 180 GB of HBM), bf16 mixed, batch 16, the configuration the autotuner settles on (R27: 42
+GPU-optimised layers, a decoupled ring of 26 slots; profiles/r02_ab_c4max_L112.txt), 8 host landing
+buffers, the split host master (R25) and the lowest-computed-first offload order (R26).
 
 The fp64 oracle cannot run this model, so (as test_fullsize_c4_gpu.py does for the 82-layer C4):
   * sampled AdamW at step 2 against the oracle's update, element by element, on a GPU-optimised layer
@@ -26,9 +26,9 @@ from tests._common import rna_bf16_bits
 pytestmark = [pytest.mark.gpu, pytest.mark.slow]
 
 sh = pytest.importorskip("paper_conf_sc_sunwqyhxw22_b200.sh")
-C4MAX = dict(L=106, h=4096, nh=32, s=1024, V=50304, b=16)
-G_LAYERS, RING, LANDING = 45, 26, 8
-HOST = tuple(range(G_LAYERS, 106))
+C4MAX = dict(L=112, h=4096, nh=32, s=1024, V=50304, b=16)
+G_LAYERS, RING, LANDING = 42, 26, 8
+HOST = tuple(range(G_LAYERS, 112))
 SAMPLED = (0,) + HOST + (-1,)
 N_SAMPLE = 4096
 
@@ -65,7 +65,7 @@ def run():
                 else:
                     out["s1"][x] = [tr.engine.read_layer(x, w)[idx[x]] for w in whats]
         out["split"] = {x: (tr.engine.read_layer(x, sh.SH_READ_PARAM), tr.engine.read_layer(x, sh.SH_READ_COMPUTE))
-                        for x in (0, G_LAYERS, 105)}
+                        for x in (0, G_LAYERS, C4MAX["L"] - 1)}
         out["stats"] = tr.engine.stats()
     finally:
         tr.close()
