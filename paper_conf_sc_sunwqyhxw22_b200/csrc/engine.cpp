@@ -3,7 +3,9 @@
 // Paper mechanism -> this file:
 //   pinned per-layer CPU buffers            -> HostStore: one mmap'ed, THP-advised,
 //                                                              page-locked block per host layer;
-//                                                              fp32 master | m | v | bf16 shadow;
+//                                                              bf16: split master hi | lo | m | v (the hi
+//                                                              plane IS the compute copy, R25), or
+//                                                              fp32 master | m | v [| bf16 shadow];
 //                                                              NUMA placement by mbind before first
 //                                                              touch (numa.cpp, sh_config.numa_policy)
 //   reserved round-robin GPU buffer queue -> ring of w+1 slots, one cudaMalloc,
@@ -15,7 +17,10 @@
 //   pre_forward / post_forward (Fig. 3b)      -> sh_forward_layer PRE/POST
 //   pre_backward (Fig. 3c)                    -> sh_backward_layer PRE/POST
 //   "idle CUDA stream" async copies          -> H2D and D2H copy-engine streams, each
-//                                                              owned by an issuer thread
+//                                                              owned by an issuer thread; gradients wait
+//                                                              in a pool (the ring's grad halves) and
+//                                                              are offloaded lowest computed layer
+//                                                              first (d2h_pump, R26)
 //   concurrent CPU optimizers            -> AdamPool: worker threads, per-layer
 //                                                              jobs split into chunks, lowest layer
 //                                                              (needed first by the next FP) first
@@ -341,8 +346,8 @@ struct sh_ctx {
   std::atomic<int64_t> numa_bound{0};
   std::atomic<int> numa_pinned{0};
   // NEXT-2 secondary-storage tier: host-optimised layers beyond the pinned
-  // budget live in mmap'ed files (MAP_SHARED, unlinked at creation) under spill_dir; their
-  // fetches go through pinned bounce buffers, the CPU Adam works on the mapping (page cache)
+  // budget live in O_DIRECT files (unlinked at creation) under spill_dir; their fetches go through
+  // pinned bounce buffers, their CPU updates through pinned staging copies (no page cache)
   std::string spill_dir;
   int64_t pin_budget = 0;
   size_t spill_bytes = 0;
@@ -394,7 +399,7 @@ struct sh_ctx {
   float* h_coef = nullptr;  // pinned [2]
   std::vector<uint8_t> registered;
 
-  // ---- ring state (driver thread only, except *_pub / ready / landing_done)
+  // ---- ring state (driver thread only, except *_pub / ready / the landing free list)
   std::vector<int> slot_layer, layer_slot;
   std::vector<int64_t> slot_last_use;  // global position of the occupant's latest compute (LRU tie-break)
   int64_t pos_clock = 0;
