@@ -65,7 +65,7 @@
 extern "C" {
 #endif
 
-#define SH_ABI_VERSION 1
+#define SH_ABI_VERSION 2  /* 2: sh_stats_t / sh_profile grew (round 2), bf16 rounding RNA, split host master */
 
 typedef struct sh_ctx sh_ctx;
 
