@@ -321,6 +321,10 @@ struct sh_ctx {
   std::atomic<int64_t> k3_pub{0};     // latest generation whose K3 has been enqueued
   double* norm_dev = nullptr;
   float* coef_dev = nullptr;
+  // K2 dynamic-schedule counters (kernels.cu kDyn), one pair per stream K2 runs on; zeroed at init and
+  // left zeroed by every launch (null: static schedule, SH_K2_SCHED=static)
+  unsigned int* k2_sched_cs = nullptr;
+  unsigned int* k2_sched_comm = nullptr;
   int64_t device_bytes = 0;
 
   // ---- host store: one pinned block per host-optimised layer (allocated when the layer first
@@ -2001,6 +2005,7 @@ sh_status exec_fold(sh_ctx* c, float* dst, const std::vector<float*>& src, int64
 sh_status push_k2(sh_ctx* c, kern::K2Args& a, int64_t* bytes, int* launches) {
   if (a.n_entries == 0) return SH_OK;
   for (int i = 0; i < a.n_entries; ++i) *bytes += (c->bf16 ? 30 : 32) * a.e[i].n;
+  a.sched = c->k2_sched_cs;
   CKC(c, kern::adamw_multi(a, c->cs));
   (*launches)++;
   a.n_entries = 0;
@@ -2623,6 +2628,10 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
     c->scratch_d2h = c->scratch_comm + kern::kSumsqMaxBlocks + 1;
     c->norm_dev = c->scratch_d2h + kern::kSumsqMaxBlocks + 1;
     c->coef_dev = reinterpret_cast<float*>(c->norm_dev + 1);
+    if (kern::k2_dynamic()) {  // in the 64-B slack after coef_dev (zeroed above)
+      c->k2_sched_cs = reinterpret_cast<unsigned int*>(c->norm_dev + 2);
+      c->k2_sched_comm = c->k2_sched_cs + 2;
+    }
     for (int e = 1; e < c->K; ++e) {  // executor gradient buffers (one set: K4 runs in stream order)
       float* xg = nullptr;
       float* xr = nullptr;
@@ -3039,6 +3048,7 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
       a.out_bf16 = c->bf16;
       a.n_entries = 1;
       a.e[0] = kern::K2Entry{c->g[x].master, c->g[x].m, c->g[x].v, gb, c->slot_param(s), n, c->lay[x].n_decay};
+      a.sched = ks == c->cs ? c->k2_sched_cs : c->k2_sched_comm;
       CKC(c, kern::adamw_multi(a, ks));
       if (P) {
         CKC(c, cudaEventRecord(P->k2l1[x], ks));
@@ -3848,7 +3858,17 @@ sh_status sh_op_adamw_gpu(float* p, float* m, float* v, const float* g, uint16_t
   a.out_bf16 = out16 != nullptr;
   a.n_entries = 1;
   a.e[0] = kern::K2Entry{p, m, v, g, out16 ? (void*)out16 : (void*)out32, n, n_decay};
-  const cudaError_t e = kern::adamw_multi(a, static_cast<cudaStream_t>(stream));
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaSuccess;
+  if (kern::k2_dynamic()) {  // per-call zeroed counters (the op has no context to own them)
+    e = cudaMallocAsync(reinterpret_cast<void**>(&a.sched), 8, st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(a.sched, 0, 8, st);
+  }
+  if (e == cudaSuccess) e = kern::adamw_multi(a, st);
+  if (a.sched) {
+    const cudaError_t f = cudaFreeAsync(a.sched, st);
+    if (e == cudaSuccess) e = f;
+  }
   if (e != cudaSuccess) {
     set_error("K2 launch: %s", cudaGetErrorString(e));
     return SH_ERR_CUDA;

@@ -74,7 +74,16 @@ __device__ __forceinline__ void adam_elem(float& p, float& m, float& v, float g,
 // elements base + u*1024 + 4t .. +3 for u in [0, U): every float4 load/store of a warp touches 512
 // contiguous bytes; 4U independent 16-B loads in flight per thread (U = 4 by default, tuned on
 // B200 with tools/bench_kernels.py).
-template <bool kBf16Out, int U, int kMinBlocks = 0>
+//
+// kDyn: dynamic work distribution.  Instead of the static grid stride, each block takes its next
+// item from a global counter (a.sched[0], one atomicAdd per 4096-element item, broadcast through
+// shared memory).  Under concurrency -- a K3 / K1 / GEMM on another stream holding some SMs when K2
+// starts, copy-engine traffic -- blocks that start late simply take fewer items instead of
+// leaving a tail of statically assigned work.  Items still arrive in increasing order per block,
+// so the entry cursor stays monotone.  The last block to finish (a.sched[1] ticket) resets both
+// counters for the next launch on the same stream.  Same per-element arithmetic => bitwise
+// identical to the static kernel.
+template <bool kBf16Out, int U, int kMinBlocks = 0, bool kDyn = false>
 __global__ void __launch_bounds__(256, kMinBlocks) k2_adamw_kernel(const __grid_constant__ K2Args a) {
   const AdamS s{a.sc.beta1, a.sc.beta2, a.sc.omb1, a.sc.omb2, a.sc.eps, -a.sc.step_size,
                 a.sc.sqrt_bc2, a.sc.decay};
@@ -82,7 +91,19 @@ __global__ void __launch_bounds__(256, kMinBlocks) k2_adamw_kernel(const __grid_
   const float coef = use_coef ? *a.coef : 1.0f;
   const int64_t n_items = a.item_start[a.n_entries];
   int e = 0;
-  for (int64_t item = blockIdx.x; item < n_items; item += gridDim.x) {
+  __shared__ unsigned int s_item[2];
+  int64_t item;
+  int parity = 0;
+  auto grab = [&]() -> int64_t {
+    if (threadIdx.x == 0) s_item[parity] = atomicAdd(a.sched, 1u);
+    __syncthreads();  // s_item[parity ^ 1] is free again: every thread read it before this barrier
+    const int64_t it = s_item[parity];
+    parity ^= 1;
+    return it;
+  };
+  if constexpr (kDyn) item = grab();
+  else item = blockIdx.x;
+  for (; item < n_items; item = kDyn ? grab() : item + gridDim.x) {
     while (item >= a.item_start[e + 1]) ++e;  // items are visited in increasing order
     const K2Entry& E = a.e[e];
     const int64_t base = (item - a.item_start[e]) * (1024 * U);
@@ -118,6 +139,16 @@ __global__ void __launch_bounds__(256, kMinBlocks) k2_adamw_kernel(const __grid_
         } else {
           st_f4(static_cast<float*>(E.out) + i, p[u]);
         }
+      }
+    }
+  }
+  if constexpr (kDyn) {
+    if (threadIdx.x == 0) {
+      __threadfence();
+      if (atomicAdd(a.sched + 1, 1u) == gridDim.x - 1) {  // every block has made its last grab
+        a.sched[0] = 0;
+        a.sched[1] = 0;
+        __threadfence();
       }
     }
   }
@@ -434,6 +465,14 @@ int env_int(const char* name, int dflt) {
 }
 }  // namespace
 
+bool k2_dynamic() {
+  static const bool dyn = [] {
+    const char* e = getenv("SH_K2_SCHED");
+    return !(e && strcmp(e, "static") == 0);
+  }();
+  return dyn;
+}
+
 cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
   static const int U = env_int("SH_K2_U", 4) == 2 ? 2 : 4;  // U=4: 0.93 vs 0.89 of HBM peak (profiles/r01_kernels_microbench.txt)
   static const int bps = env_int("SH_K2_BPS", 4);
@@ -485,7 +524,31 @@ cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
   const int grid = (int)(items < cap ? items : cap);
   if (grid_out) *grid_out = grid;
   launch_counter()++;
-  if (impl == 3) {
+  if (a.sched != nullptr && (impl == 0 || impl == 3) && U == 4) {
+    if (items >= (int64_t)1 << 32) return cudaErrorInvalidValue;  // 32-bit counter
+    // exactly the resident blocks (2 per SM at this register count): a late block would only find
+    // the counter exhausted
+    static const int per_sm = [] {
+      int nb = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, impl == 3 ? k2_adamw_kernel<true, 4, 3, true>
+                                                                       : k2_adamw_kernel<true, 4, 0, true>, 256, 0) != cudaSuccess ||
+          nb <= 0) {
+        cudaGetLastError();
+        nb = 2;
+      }
+      return nb;
+    }();
+    const int64_t dcap = (int64_t)sm_count() * per_sm;
+    const int dgrid = (int)(items < dcap ? items : dcap);
+    if (grid_out) *grid_out = dgrid;
+    if (impl == 3) {
+      if (a.out_bf16) k2_adamw_kernel<true, 4, 3, true><<<dgrid, 256, 0, st>>>(a);
+      else k2_adamw_kernel<false, 4, 3, true><<<dgrid, 256, 0, st>>>(a);
+    } else {
+      if (a.out_bf16) k2_adamw_kernel<true, 4, 0, true><<<dgrid, 256, 0, st>>>(a);
+      else k2_adamw_kernel<false, 4, 0, true><<<dgrid, 256, 0, st>>>(a);
+    }
+  } else if (impl == 3) {
     if (a.out_bf16) k2_adamw_kernel<true, 4, 3><<<grid, 256, 0, st>>>(a);
     else k2_adamw_kernel<false, 4, 3><<<grid, 256, 0, st>>>(a);
   } else if (U == 4) {

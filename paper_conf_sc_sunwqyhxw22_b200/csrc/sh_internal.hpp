@@ -61,11 +61,17 @@ constexpr int kK2MaxEntries = 40;
 struct K2Args {
   sh_adam_scalars sc;
   const float* coef;  // null: no clipping
+  // null: static grid-stride schedule; else 2 zeroed device counters owned by the caller for this
+  // stream (dynamic item distribution; the kernel leaves them zeroed); never shared by launches that
+  // may run concurrently
+  unsigned int* sched;
   int n_entries;
   int out_bf16;
   K2Entry e[kK2MaxEntries];
   int64_t item_start[kK2MaxEntries + 1];
 };
+// true unless SH_K2_SCHED=static: K2 launches that carry counters use the dynamic item schedule
+bool k2_dynamic();
 // Launch K2 over args (item_start filled by the callee).  Returns the grid used.
 cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out = nullptr);
 cudaError_t cast_bf16(const float* src, uint16_t* dst, int64_t n, cudaStream_t st);
