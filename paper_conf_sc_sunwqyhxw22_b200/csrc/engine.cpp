@@ -62,6 +62,7 @@
 #include <cstring>
 #include <deque>
 #include <functional>
+#include <map>
 #include <memory>
 #include <mutex>
 #include <string>
@@ -3845,6 +3846,43 @@ static bool ops_args_ok(int64_t n, int64_t n_decay, const void* const* ptrs, int
   return true;
 }
 
+}  // extern "C"
+
+namespace {
+// Per-(device, stream) device scratch of the op entry points: K3's partials + completion ticket and
+// K2's two dynamic-schedule counters.  Allocated and zeroed once (synchronously) on first use; every
+// kernel leaves its part reset, so launches in stream order reuse it and launches on other streams or
+// devices never share it.  Never freed (a few KB per stream handle).
+struct OpScratch {
+  double* k3 = nullptr;        // kSumsqMaxBlocks partials + ticket
+  unsigned int* k2 = nullptr;  // 2 counters
+};
+OpScratch op_scratch(cudaStream_t st) {
+  static std::mutex mu;
+  static std::map<std::pair<int, cudaStream_t>, OpScratch> m;
+  int dev = -1;
+  if (cudaGetDevice(&dev) != cudaSuccess) {
+    cudaGetLastError();
+    return {};
+  }
+  std::lock_guard<std::mutex> g(mu);
+  auto it = m.find({dev, st});
+  if (it != m.end()) return it->second;
+  const size_t k3b = 8 * (kern::kSumsqMaxBlocks + 1);
+  void* p = nullptr;
+  if (cudaMalloc(&p, k3b + 64) != cudaSuccess || cudaMemset(p, 0, k3b + 64) != cudaSuccess) {
+    cudaGetLastError();
+    if (p) cudaFree(p);
+    return {};
+  }
+  OpScratch o{static_cast<double*>(p), reinterpret_cast<unsigned int*>(static_cast<char*>(p) + k3b)};
+  m[{dev, st}] = o;
+  return o;
+}
+}  // namespace
+
+extern "C" {
+
 sh_status sh_op_adamw_gpu(float* p, float* m, float* v, const float* g, uint16_t* out16, float* out32,
                           int64_t n, int64_t n_decay, const sh_adam_scalars* sc, const float* coef,
                           void* stream) {
@@ -3859,16 +3897,14 @@ sh_status sh_op_adamw_gpu(float* p, float* m, float* v, const float* g, uint16_t
   a.n_entries = 1;
   a.e[0] = kern::K2Entry{p, m, v, g, out16 ? (void*)out16 : (void*)out32, n, n_decay};
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  cudaError_t e = cudaSuccess;
-  if (kern::k2_dynamic()) {  // per-call zeroed counters (the op has no context to own them)
-    e = cudaMallocAsync(reinterpret_cast<void**>(&a.sched), 8, st);
-    if (e == cudaSuccess) e = cudaMemsetAsync(a.sched, 0, 8, st);
+  if (kern::k2_dynamic()) {
+    a.sched = op_scratch(st).k2;
+    if (!a.sched) {
+      set_error("K2 schedule counters: allocation failed");
+      return SH_ERR_OOM_DEVICE;
+    }
   }
-  if (e == cudaSuccess) e = kern::adamw_multi(a, st);
-  if (a.sched) {
-    const cudaError_t f = cudaFreeAsync(a.sched, st);
-    if (e == cudaSuccess) e = f;
-  }
+  const cudaError_t e = kern::adamw_multi(a, st);
   if (e != cudaSuccess) {
     set_error("K2 launch: %s", cudaGetErrorString(e));
     return SH_ERR_CUDA;
@@ -3971,20 +4007,15 @@ sh_status sh_op_sumsq_gpu(const float* g, int64_t n, double* out_dev, void* stre
   clear_error();
   const void* ptrs[] = {g};
   if (!g || !out_dev || !ops_args_ok(n, 0, ptrs, 1)) return SH_ERR_INVALID;
-  // private, stream-ordered scratch (partials + completion ticket) per call: concurrent calls on
+  // scratch (partials + completion ticket) private to this device and stream: concurrent calls on
   // other streams or devices never share it
-  double* scratch = nullptr;
-  const size_t sb = 8 * (kern::kSumsqMaxBlocks + 1);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (cudaMallocAsync(reinterpret_cast<void**>(&scratch), sb, st) != cudaSuccess ||
-      cudaMemsetAsync(scratch, 0, sb, st) != cudaSuccess) {
-    cudaGetLastError();
+  double* scratch = op_scratch(st).k3;
+  if (!scratch) {
     set_error("K3 scratch allocation failed");
     return SH_ERR_OOM_DEVICE;
   }
-  cudaError_t e = kern::sumsq(g, n, scratch, out_dev, st);
-  const cudaError_t e2 = cudaFreeAsync(scratch, st);
-  if (e == cudaSuccess) e = e2;
+  const cudaError_t e = kern::sumsq(g, n, scratch, out_dev, st);
   if (e != cudaSuccess) {
     set_error("K3 launch: %s", cudaGetErrorString(e));
     return SH_ERR_CUDA;

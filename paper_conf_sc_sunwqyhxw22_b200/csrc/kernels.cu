@@ -478,13 +478,15 @@ cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
   static const int bps = env_int("SH_K2_BPS", 4);
   // SH_K2_IMPL: "bulk4k" / "bulk2k" = bulk-copy pipeline (4096-element items, 1 block/SM, or
   // 2048-element items, 2 blocks/SM); "ldg3" = register-staged kernel capped at 80 registers (3
-  // blocks/SM); default: register-staged, 2 blocks/SM
+  // blocks/SM); "dyn2" = dynamic schedule at 2 blocks/SM; default: register-staged, dynamic schedule,
+  // 3 blocks/SM when the caller passes counters (SH_K2_SCHED=static: never), else static, 2 blocks/SM
   static const int impl = [] {
     const char* e = getenv("SH_K2_IMPL");
     if (!e) return 0;
     if (strcmp(e, "bulk4k") == 0 || strcmp(e, "bulk") == 0) return 1;
     if (strcmp(e, "bulk2k") == 0) return 2;
     if (strcmp(e, "ldg3") == 0) return 3;
+    if (strcmp(e, "dyn2") == 0) return 4;
     return 0;
   }();
   if (impl == 1 || impl == 2) {
@@ -524,24 +526,28 @@ cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
   const int grid = (int)(items < cap ? items : cap);
   if (grid_out) *grid_out = grid;
   launch_counter()++;
-  if (a.sched != nullptr && (impl == 0 || impl == 3) && U == 4) {
+  // Default with counters (the engine's K2): dynamic schedule, 80-register build, 3 resident blocks per
+  // SM, grid = exactly the resident blocks.  Isolated h=4096 layer (201 M elements): 6.75 TB/s vs 6.03
+  // static (2 blocks/SM, two static waves); beside a D2H copy (the live step's usual neighbour) 6.47 vs
+  // 5.82 TB/s (profiles/r02_k2_contention.jsonl).  SH_K2_IMPL=dyn2: dynamic, 2 blocks/SM.
+  if (a.sched != nullptr && (impl == 0 || impl == 3 || impl == 4) && U == 4) {
     if (items >= (int64_t)1 << 32) return cudaErrorInvalidValue;  // 32-bit counter
-    // exactly the resident blocks (2 per SM at this register count): a late block would only find
+    // exactly the resident blocks (the occupancy of the chosen build): a late block would only find
     // the counter exhausted
     static const int per_sm = [] {
       int nb = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, impl == 3 ? k2_adamw_kernel<true, 4, 3, true>
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, impl != 4 ? k2_adamw_kernel<true, 4, 3, true>
                                                                        : k2_adamw_kernel<true, 4, 0, true>, 256, 0) != cudaSuccess ||
           nb <= 0) {
         cudaGetLastError();
-        nb = 2;
+        nb = impl != 4 ? 3 : 2;
       }
       return nb;
     }();
     const int64_t dcap = (int64_t)sm_count() * per_sm;
     const int dgrid = (int)(items < dcap ? items : dcap);
     if (grid_out) *grid_out = dgrid;
-    if (impl == 3) {
+    if (impl != 4) {
       if (a.out_bf16) k2_adamw_kernel<true, 4, 3, true><<<dgrid, 256, 0, st>>>(a);
       else k2_adamw_kernel<false, 4, 3, true><<<dgrid, 256, 0, st>>>(a);
     } else {
