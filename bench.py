@@ -82,6 +82,26 @@ def mem_available() -> int:
     return 0
 
 
+def host_pages() -> dict:
+    """Huge-page backing of the process's host memory while the engine holds its pinned store (the host
+    store is mmap'ed with MADV_HUGEPAGE: whether the kernel could back it with 2 MiB pages is a property
+    of the box -- THP mode, fragmentation -- that the DMA rates may depend on)."""
+    out = {}
+    try:
+        for ln in open("/proc/self/smaps_rollup"):
+            k = ln.split(":")[0]
+            if k in ("Rss", "AnonHugePages"):
+                out[k.lower() + "_gb"] = int(ln.split()[1]) * 1024 / 1e9
+    except OSError:
+        pass
+    for k in ("enabled", "defrag"):
+        try:
+            out["thp_" + k] = open(f"/sys/kernel/mm/transparent_hugepage/{k}").read().strip()
+        except OSError:
+            pass
+    return out
+
+
 def shm_free() -> int:
     try:
         st = os.statvfs("/dev/shm")
@@ -177,12 +197,13 @@ class ClockSampler:
 def k2_traffic(elems_per_launch: float):
     """DRAM read+write bytes of one K2 launch: the per-element figure of the committed ncu --set full
     capture (tools/ncu_kernels.sh -> tools/ncu_iso_summary.py) times this bench's elements per launch."""
-    p = os.path.join(ROOT, "profiles", "r01_ncu_iso_kernels.json")
-    try:
-        per = json.load(open(p))["k2_adamw"]["dram_bytes_per_elem"]
-    except Exception:  # noqa: BLE001
-        return None
-    return per * elems_per_launch
+    for name in ("r02_ncu_iso_kernels.json", "r01_ncu_iso_kernels.json"):
+        try:
+            per = json.load(open(os.path.join(ROOT, "profiles", name)))["k2_adamw"]["dram_bytes_per_elem"]
+        except Exception:  # noqa: BLE001
+            continue
+        return per * elems_per_launch, "profiles/" + name
+    return None, None
 
 
 def oracle_sample(L, h, nh, s, V, b, seed=1234):
@@ -540,6 +561,7 @@ def main():
         prof = tr.engine.profile() if window != L else None
         trace = tr.engine.trace()
         st2 = tr.engine.stats()
+        hostmem = host_pages()
         if args.trace_out and rank == 0:
             # Chrome trace (chrome://tracing / Perfetto) of the last profiled step: Fig. 4 analogue
             tid = {"fp": 1, "bp": 1, "k2_adamw": 1, "h2d_fp": 2, "h2d_bp": 2, "d2h_grad": 3, "k1_stage": 4,
@@ -553,6 +575,7 @@ def main():
                 json.dump({"traceEvents": ev, "displayTimeUnit": "ms"}, f)
         tr.close()
         return dict(ms=ms, e2e_ms=e2e_ms, st0=st0, st1=st1, loss=loss, launches=launches, clocks=clk.summary(),
+                    hostmem=hostmem,
                     init_s=t_init, prof=prof, st2=st2, attn=attn_used, seg_sps=seg_sps, settle_ms=settle_ms, S=S)
 
     r = run(w, not args.no_e2e)
@@ -593,6 +616,7 @@ def main():
     samples = b * world * K / (ms / 1e3)
     peak, peak_kind = measured_peaks()
     k2_gbs = d["k2_bytes_sum"] / (d["k2_ms_sum"] / 1e3) / 1e9 if d["k2_ms_sum"] > 0 else None
+    k2_tr, k2_tr_src = k2_traffic(d["k2_bytes_sum"] / max(1, d["k2_samples"]) / (30 if prec else 32))
     k3_gbs = d["k3_bytes_sum"] / (d["k3_ms_sum"] / 1e3) / 1e9 if d["k3_ms_sum"] > 0 else None
     h2d_gbs = d["h2d_profiled_bytes"] / (d["h2d_busy_ms"] / 1e3) / 1e9 if d["h2d_busy_ms"] > 0 else None
     d2h_gbs = d["d2h_profiled_bytes"] / (d["d2h_busy_ms"] / 1e3) / 1e9 if d["d2h_busy_ms"] > 0 else None
@@ -644,6 +668,7 @@ def main():
         "tokens_per_s": tokens_s,
         "model_tflops": tokens_s * flops_tok / 1e12,
         "final_loss": r["loss"],
+        "host_memory": r.get("hostmem"),
         "host_link": {
             "h2d_bytes_per_step": d["h2d_bytes"] / K, "d2h_bytes_per_step": d["d2h_bytes"] / K,
             "h2d_gbs_per_transfer": h2d_gbs, "d2h_gbs_per_transfer": d2h_gbs,
@@ -680,13 +705,16 @@ def main():
                       "triad_gbs": PROBE_HOST_TRIAD_GBS,
                       "peak_source": "profiles/r02_host_mix.json: CPU AdamW + H2D + D2H DMA concurrently (the "
                                      "engine's own mix), best total over thread counts"},
-        "roofline": {"kernel": "K2 fused multi-tensor AdamW (sh_step)", "bound": "hbm", "achieved": k2_gbs,
+        "roofline": {"kernel": "K2 fused AdamW: the per-layer launches of the GPU-optimised layers in the "
+                               "backward + the resident-set launch at sh_step (CUDA events on their stream)",
+                     "bound": "hbm", "achieved": k2_gbs,
                      "peak": peak, "unit": "GB/s", "frac": k2_gbs / peak if k2_gbs else None,
-                     "traffic": k2_traffic(d["k2_bytes_sum"] / max(1, d["k2_samples"]) / (30 if prec else 32)),
-                     "traffic_source": "profiles/r01_ncu_iso_kernels.json: ncu --set full DRAM bytes/element of an "
-                                       "isolated K2 launch (one h=4096 layer) x elements per launch",
+                     "traffic": k2_tr,
+                     "traffic_source": (f"{k2_tr_src}: ncu --set full DRAM bytes/element of an isolated K2 launch "
+                                        "(one h=4096 layer) x the K2 elements of one step") if k2_tr_src else None,
+                     "traffic_per": "step",
                      "peak_source": peak_kind, "algorithmic_bytes_per_elem": 30 if prec else 32,
-                     "bytes_per_launch": d["k2_bytes_sum"] / max(1, d["k2_samples"]),
+                     "bytes_per_step": d["k2_bytes_sum"] / max(1, d["k2_samples"]),
                      "k3_sumsq_gbs": k3_gbs, "k3_frac": k3_gbs / peak if k3_gbs else None},
         "gpu_launches": r["launches"],
         "clocks": r["clocks"],

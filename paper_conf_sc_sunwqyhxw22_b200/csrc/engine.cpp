@@ -2409,8 +2409,17 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
   c->cs = static_cast<cudaStream_t>(cfg->compute_stream);
   CKC(c.get(), cudaStreamCreateWithFlags(&c->h2d, cudaStreamNonBlocking));
   CKC(c.get(), cudaStreamCreateWithFlags(&c->d2h, cudaStreamNonBlocking));
-  CKC(c.get(), cudaStreamCreateWithFlags(&c->k3s, cudaStreamNonBlocking));
-  CKC(c.get(), cudaStreamCreateWithFlags(&c->stage, cudaStreamNonBlocking));
+  {
+    // K3 (host layers' Σg², beside the offload) and K1 (restage ahead of a layer's backward) are short
+    // HBM-bound launches that run beside the compute stream's GEMMs: at the greatest stream priority
+    // their blocks are scheduled as SMs free up instead of queueing behind a GEMM's remaining tiles
+    // (SH_SIDE_PRIO=0: default priority, the round-1 behaviour)
+    int lo = 0, hi = 0;
+    const char* e = getenv("SH_SIDE_PRIO");
+    if (!(e && atoi(e) == 0)) CKC(c.get(), cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    CKC(c.get(), cudaStreamCreateWithPriority(&c->k3s, cudaStreamNonBlocking, hi));
+    CKC(c.get(), cudaStreamCreateWithPriority(&c->stage, cudaStreamNonBlocking, hi));
+  }
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_cs_mark, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_comm_done, cudaEventDisableTiming));
   CKC(c.get(), cudaEventCreateWithFlags(&c->ev_k3_last, cudaEventDisableTiming));
