@@ -18,6 +18,7 @@
 
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 
 #include "sh_internal.hpp"
@@ -176,8 +177,18 @@ static void adam_split_scalar_range(uint16_t* hi, uint16_t* lo, float* m, float*
   }
 }
 
+// SH_CPU_PF: software-prefetch distance of the split-master AdamW in elements (0: off)
+static int64_t split_prefetch_distance() {
+  static const int64_t d = [] {
+    const char* e = getenv("SH_CPU_PF");
+    const long long x = e ? atoll(e) : 0;
+    return (int64_t)(x > 0 ? (x + 31) / 32 * 32 : 0);
+  }();
+  return d;
+}
+
 template <bool kWd, bool kCoef>
-__attribute__((target("avx512f,avx512bw"))) static void adam_split_avx512_block(
+__attribute__((target("avx512f,avx512bw,prfchw"))) static void adam_split_avx512_block(
     uint16_t* __restrict hi, uint16_t* __restrict lo, float* __restrict m, float* __restrict v,
     const float* __restrict g, int64_t b, int64_t e, const sh_adam_scalars& s, float coef) {
   const __m512 b1 = _mm512_set1_ps(s.beta1), b2 = _mm512_set1_ps(s.beta2);
@@ -185,7 +196,20 @@ __attribute__((target("avx512f,avx512bw"))) static void adam_split_avx512_block(
   const __m512 eps = _mm512_set1_ps(s.eps), nss = _mm512_set1_ps(-s.step_size);
   const __m512 sbc2 = _mm512_set1_ps(s.sqrt_bc2), decay = _mm512_set1_ps(s.decay);
   const __m512 vc = _mm512_set1_ps(coef);
+  const int64_t pf = split_prefetch_distance();
   for (int64_t i = b; i < e; i += 16) {
+    if (pf > 0 && i + pf < e) {
+      // software prefetch pf elements ahead on all five streams: the L2 streamer stops at every 4 KiB
+      // page boundary, which these nine concurrent streams (5 read, 4 written) cross every 64-128
+      // iterations; prefetchw for the read-modify-write ones
+      _mm_prefetch(reinterpret_cast<const char*>(g + i + pf), _MM_HINT_T0);
+      _mm_prefetch(reinterpret_cast<const char*>(m + i + pf), _MM_HINT_T0);
+      _mm_prefetch(reinterpret_cast<const char*>(v + i + pf), _MM_HINT_T0);
+      if ((i & 31) == 0) {
+        _mm_prefetch(reinterpret_cast<const char*>(hi + i + pf), _MM_HINT_T0);
+        _mm_prefetch(reinterpret_cast<const char*>(lo + i + pf), _MM_HINT_T0);
+      }
+    }
     const __m512i h = _mm512_cvtepu16_epi32(_mm256_loadu_si256(reinterpret_cast<const __m256i*>(hi + i)));
     const __m512i l = _mm512_cvtepi16_epi32(_mm256_loadu_si256(reinterpret_cast<const __m256i*>(lo + i)));
     __m512 pp = _mm512_castsi512_ps(_mm512_add_epi32(_mm512_slli_epi32(h, 16), l));
