@@ -123,11 +123,12 @@ METRIC = "samples/s at max trainable size per B200; host-link GB/s vs peak"
 PROBE_H2D_GBS = 55.58   # profiles/r01_probe_box.json, pinned 1 GiB H2D, best of 5
 PROBE_D2H_GBS = 57.01
 PROBE_HOST_TRIAD_GBS = 143.43  # profiles/r01_probe_box.json, 16-thread STREAM triad (no RFO counted)
-# profiles/r02_host_mix.json (tools/probe_host_mix.py): the engine's real host-DRAM mix -- the CPU AdamW
-# (16 B read + 14 B written per element) running concurrently with H2D + D2H DMA on pinned memory.  The
-# highest total host-DRAM throughput of that mix over thread counts (T14: Adam 115.9 + H2D 34.4 + D2H
-# 34.4 GB/s); the 16-thread STREAM triad alone reaches 143.
-PROBE_HOST_MIX_GBS = 184.7
+# The engine's real host-DRAM mix -- the pool's split-master CPU AdamW (16 B read + 12 B written per
+# element) running concurrently with H2D + D2H DMA on pinned memory: the highest total host-DRAM
+# throughput measured over thread counts and software-prefetch distances (profiles/r02_cpu_pf.jsonl,
+# tools/probe_cpu_pf.py: 14 threads, prefetch 1024: Adam 142.5 + H2D 27.7 + D2H 27.7 GB/s).  Round-2
+# first probe without the prefetch (profiles/r02_host_mix.json): 184.7; the 16-thread STREAM triad: 143.
+PROBE_HOST_MIX_GBS = 197.9
 
 
 def measured_peaks():
@@ -703,8 +704,9 @@ def main():
                       "peak_gbs": PROBE_HOST_MIX_GBS,
                       "frac": host_dram_bytes / (ms / 1e3) / 1e9 / PROBE_HOST_MIX_GBS,
                       "triad_gbs": PROBE_HOST_TRIAD_GBS,
-                      "peak_source": "profiles/r02_host_mix.json: CPU AdamW + H2D + D2H DMA concurrently (the "
-                                     "engine's own mix), best total over thread counts"},
+                      "peak_source": "profiles/r02_cpu_pf.jsonl: the split-master CPU AdamW + H2D + D2H DMA "
+                                     "concurrently (the engine's own mix), best total over thread counts and "
+                                     "prefetch distances"},
         "roofline": {"kernel": "K2 fused AdamW: the per-layer launches of the GPU-optimised layers in the "
                                "backward + the resident-set launch at sh_step (CUDA events on their stream)",
                      "bound": "hbm", "achieved": k2_gbs,

@@ -78,6 +78,21 @@ __attribute__((target("avx512f"))) static inline __m256i rna_bf16_16(__m512 x) {
   return _mm512_cvtepi32_epi16(r);
 }
 
+// Software-prefetch distance of the AVX-512 AdamW in elements (SH_CPU_PF, default 512; 0: off).  The
+// L2 streamer stops at every 4 KiB page boundary, which the kernel's concurrent streams (5 read + 4
+// written on the split master) cross every 64-128 iterations; prefetching 512 elements ahead on every
+// read stream keeps each core's misses in flight across them.  Measured on the B200 box
+// (profiles/r02_cpu_pf.jsonl): the split AdamW alone 143-165 -> 176-180 GB/s at 12 threads, beside
+// H2D + D2H DMA 187-192 -> 196-198 GB/s of host-DRAM total; c4max 5.31-5.46 -> 5.61 samples/s.
+static int64_t prefetch_distance() {
+  static const int64_t d = [] {
+    const char* e = getenv("SH_CPU_PF");
+    const long long x = e ? atoll(e) : 512;
+    return (int64_t)(x > 0 ? (x + 31) / 32 * 32 : 0);
+  }();
+  return d;
+}
+
 template <bool kWd, bool kCoef, bool kOut, bool kNT>
 __attribute__((target("avx512f"))) static void adam_avx512_block(
     float* __restrict p, float* __restrict m, float* __restrict v, const float* __restrict g,
@@ -87,7 +102,14 @@ __attribute__((target("avx512f"))) static void adam_avx512_block(
   const __m512 eps = _mm512_set1_ps(s.eps), nss = _mm512_set1_ps(-s.step_size);
   const __m512 sbc2 = _mm512_set1_ps(s.sqrt_bc2), decay = _mm512_set1_ps(s.decay);
   const __m512 vc = _mm512_set1_ps(coef);
+  const int64_t pf = prefetch_distance();
   for (int64_t i = b; i < e; i += 16) {
+    if (pf > 0 && i + pf < e) {
+      _mm_prefetch(reinterpret_cast<const char*>(g + i + pf), _MM_HINT_T0);
+      _mm_prefetch(reinterpret_cast<const char*>(m + i + pf), _MM_HINT_T0);
+      _mm_prefetch(reinterpret_cast<const char*>(v + i + pf), _MM_HINT_T0);
+      _mm_prefetch(reinterpret_cast<const char*>(p + i + pf), _MM_HINT_T0);
+    }
     __m512 gg = _mm512_loadu_ps(g + i);
     if (kCoef) gg = _mm512_mul_ps(gg, vc);
     __m512 mm = _mm512_loadu_ps(m + i);
@@ -177,18 +199,8 @@ static void adam_split_scalar_range(uint16_t* hi, uint16_t* lo, float* m, float*
   }
 }
 
-// SH_CPU_PF: software-prefetch distance of the split-master AdamW in elements (0: off)
-static int64_t split_prefetch_distance() {
-  static const int64_t d = [] {
-    const char* e = getenv("SH_CPU_PF");
-    const long long x = e ? atoll(e) : 0;
-    return (int64_t)(x > 0 ? (x + 31) / 32 * 32 : 0);
-  }();
-  return d;
-}
-
 template <bool kWd, bool kCoef>
-__attribute__((target("avx512f,avx512bw,prfchw"))) static void adam_split_avx512_block(
+__attribute__((target("avx512f,avx512bw"))) static void adam_split_avx512_block(
     uint16_t* __restrict hi, uint16_t* __restrict lo, float* __restrict m, float* __restrict v,
     const float* __restrict g, int64_t b, int64_t e, const sh_adam_scalars& s, float coef) {
   const __m512 b1 = _mm512_set1_ps(s.beta1), b2 = _mm512_set1_ps(s.beta2);
@@ -196,12 +208,9 @@ __attribute__((target("avx512f,avx512bw,prfchw"))) static void adam_split_avx512
   const __m512 eps = _mm512_set1_ps(s.eps), nss = _mm512_set1_ps(-s.step_size);
   const __m512 sbc2 = _mm512_set1_ps(s.sqrt_bc2), decay = _mm512_set1_ps(s.decay);
   const __m512 vc = _mm512_set1_ps(coef);
-  const int64_t pf = split_prefetch_distance();
+  const int64_t pf = prefetch_distance();
   for (int64_t i = b; i < e; i += 16) {
-    if (pf > 0 && i + pf < e) {
-      // software prefetch pf elements ahead on all five streams: the L2 streamer stops at every 4 KiB
-      // page boundary, which these nine concurrent streams (5 read, 4 written) cross every 64-128
-      // iterations; prefetchw for the read-modify-write ones
+    if (pf > 0 && i + pf < e) {  // the five read streams (hi / lo: one line per 32 elements)
       _mm_prefetch(reinterpret_cast<const char*>(g + i + pf), _MM_HINT_T0);
       _mm_prefetch(reinterpret_cast<const char*>(m + i + pf), _MM_HINT_T0);
       _mm_prefetch(reinterpret_cast<const char*>(v + i + pf), _MM_HINT_T0);
