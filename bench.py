@@ -102,6 +102,20 @@ def host_pages() -> dict:
     return out
 
 
+def layer_n_pad(h: int) -> int:
+    """Elements of one GPT block's packed layout (every tensor padded to 128 elements)."""
+    return sum((n + 127) // 128 * 128 for n in (h, h, 3 * h * h, 3 * h, h * h, h, h, h, 4 * h * h, 4 * h, 4 * h * h, h))
+
+
+def ring_bytes_of(mc, bf16: bool, slots: float) -> int:
+    """Device bytes of `slots` largest-layer slots of the fixed-byte ring (engine.cpp slot_sz:
+    the compute copy and the fp32 gradient half, each 256-B aligned)."""
+    n = layer_n_pad(mc.hidden)
+    cb = 2 if bf16 else 4
+    slot = (cb * n + 255) // 256 * 256 + (4 * n + 255) // 256 * 256
+    return int(slots * slot)
+
+
 def shm_free() -> int:
     try:
         st = os.statvfs("/dev/shm")
@@ -359,6 +373,8 @@ def main():
                     help="TEST ONLY (N > 1 ranks on ONE GPU): gloo bootstrap, every rank on cuda:0, the engine's "
                          "collectives through SH_FLAG_TEST_HOST_COLLECTIVE -- exercises the multi-rank bench "
                          "orchestration where NCCL cannot run (not a performance number)")
+    ap.add_argument("--ring-bytes-slots", type=float, default=0.0,
+                    help="NEXT-4 fixed-byte window: ring_bytes = this many largest-layer slots (param + grad halves)")
     ap.add_argument("--executors", type=int, default=1,
                     help="NEXT-3: K multi-stream executors (micro-batches of batch/K on K streams, PAPER.md:227-242)")
     args = ap.parse_args()
@@ -479,7 +495,8 @@ def main():
                                ring_slots=args.ring or (C4MAX_RING0 if args.config == "c4max" and window == -1 else 0),
                                spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9),
                                warmup_window=(args.warmup_window or (C4MAX_W0 if args.config == "c4max" else 0))
-                               if window == -1 else 0)
+                               if window == -1 else 0,
+                               ring_bytes=ring_bytes_of(mc, prec == sh.SH_BF16_MIXED, args.ring_bytes_slots) if args.ring_bytes_slots > 0 else 0)
         attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
         t_init = time.perf_counter() - t_init
         # tokens: step t uses synth.tokens(t) (rank-offset seeds for DP)
@@ -635,6 +652,8 @@ def main():
                    "hidden": h, "heads": nh, "seq": s,
                    "vocab": V, "params": mc.n_params(), "batch_per_gpu": b, "global_batch": b * world,
                    "window": r["st1"]["window"], "ring_slots": r["st1"]["n_slots"],
+                   "ring_bytes": r["st1"].get("ring_bytes"),
+                   "fixed_byte_ring": args.ring_bytes_slots or None,
                    "window_mode": ("autotuned (P1/P2" + (" + eq.3 CPU throughput, ring decoupled from the GPU set"
                                                          if cpu_hard else "") + ")") if w == -1 else "fixed",
                    "precision": "bf16_mixed" if prec else "fp32",
