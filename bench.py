@@ -53,6 +53,7 @@ CONFIGS = {
                                                 "(22.8 B params), auto-tuned window"),
 }
 C4MAX_W0 = 42
+C4MAX_HYB_W0_COST = 2  # the hybrid update's 3 HBM staging buffers (10 B/param each) displace ~2 GPU layers
 C4MAX_RING0 = 26
 # the depth the default line is quoted at: 112 x 4096 = 22.8 B params, fp32 p/m/v 273 GB (> 180 GB of HBM);
 # 70 host layers (170 GB of pinned state) beside the 42-layer warm-up GPU set on this pool's 196 GB hosts
@@ -373,6 +374,8 @@ def main():
                     help="TEST ONLY (N > 1 ranks on ONE GPU): gloo bootstrap, every rank on cuda:0, the engine's "
                          "collectives through SH_FLAG_TEST_HOST_COLLECTIVE -- exercises the multi-rank bench "
                          "orchestration where NCCL cannot run (not a performance number)")
+    ap.add_argument("--hybrid-layers", type=int, default=0,
+                    help="R28: the lowest K host-optimised layers are updated on the GPU (states stay in host RAM)")
     ap.add_argument("--ring-bytes-slots", type=float, default=0.0,
                     help="NEXT-4 fixed-byte window: ring_bytes = this many largest-layer slots (param + grad halves)")
     ap.add_argument("--executors", type=int, default=1,
@@ -436,7 +439,7 @@ def main():
     if args.layers and L != 0:
         L = args.layers  # depth override (e.g. the resident-fit comparison model)
     if L == 0:
-        w0h = C4MAX_W0 if args.config == "c4max" else 2
+        w0h = (C4MAX_W0 - (C4MAX_HYB_W0_COST if args.hybrid_layers else 0)) if args.config == "c4max" else 2
         if args.layers:
             L = args.layers
         elif args.config == "c4max":
@@ -494,8 +497,11 @@ def main():
                                attention=args.attention, executors=args.executors,
                                ring_slots=args.ring or (C4MAX_RING0 if args.config == "c4max" and window == -1 else 0),
                                spill_dir=args.spill_dir or None, host_pin_budget_bytes=int(args.host_pin_gb * 1e9),
-                               warmup_window=(args.warmup_window or (C4MAX_W0 if args.config == "c4max" else 0))
+                               warmup_window=(args.warmup_window or
+                                              (C4MAX_W0 - (C4MAX_HYB_W0_COST if args.hybrid_layers else 0)
+                                               if args.config == "c4max" else 0))
                                if window == -1 else 0,
+                               hybrid_layers=args.hybrid_layers,
                                ring_bytes=ring_bytes_of(mc, prec == sh.SH_BF16_MIXED, args.ring_bytes_slots) if args.ring_bytes_slots > 0 else 0)
         attn_used = "flash_attn 2.8 (library, deterministic bwd)" if tr.flash is not None else "cuBLAS batched + softmax"
         t_init = time.perf_counter() - t_init
@@ -654,6 +660,7 @@ def main():
                    "window": r["st1"]["window"], "ring_slots": r["st1"]["n_slots"],
                    "ring_bytes": r["st1"].get("ring_bytes"),
                    "fixed_byte_ring": args.ring_bytes_slots or None,
+                   "hybrid_layers": args.hybrid_layers or None,
                    "window_mode": ("autotuned (P1/P2" + (" + eq.3 CPU throughput, ring decoupled from the GPU set"
                                                          if cpu_hard else "") + ")") if w == -1 else "fixed",
                    "precision": "bf16_mixed" if prec else "fp32",

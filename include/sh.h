@@ -65,7 +65,8 @@
 extern "C" {
 #endif
 
-#define SH_ABI_VERSION 2  /* 2: sh_stats_t / sh_profile grew (round 2), bf16 rounding RNA, split host master */
+#define SH_ABI_VERSION 3  /* 2: sh_stats_t / sh_profile grew (round 2), bf16 rounding RNA, split host master;
+                            3: sh_config.hybrid_layers, sh_stats_t hybrid counters, sh_op_adamw_split_gpu */
 
 typedef struct sh_ctx sh_ctx;
 
@@ -225,6 +226,17 @@ typedef struct {
                                        layer sizes (heterogeneous stacks).  window still sets the
                                        GPU-optimised set.  Needs no clipping, world_size 1, window >= 0,
                                        ring_slots 0; SH_ERR_INVALID if the largest layer does not fit */
+  int32_t hybrid_layers;            /* R28 hybrid update: the lowest `hybrid_layers` host-optimised layers
+                                       (w .. w+hybrid_layers-1) keep their states in host RAM but are
+                                       updated on the GPU: their lo / m / v planes are fetched into HBM
+                                       staging during the backward, K2S updates the split master right
+                                       after the layer's backward (the compute copy in its ring slot in
+                                       place), and hi / lo / m / v are written back to host RAM; the updated
+                                       compute copy stays in the ring for the next forward.  Takes the CPU
+                                       AdamW of the layers the next forward needs first off the step
+                                       boundary (eq. 3).  Bitwise the CPU update.  Needs
+                                       the split host master (bf16 mode), no clipping, world_size 1, no
+                                       spill tier, no fixed-byte ring; 0 = off */
 } sh_config;
 
 /* NUMA placement policies (sh_config.numa_policy).  Placement is an mbind(2) before the first
@@ -337,6 +349,10 @@ typedef struct {
   int64_t spill_write_bytes;
   double spill_io_ms;           /* cumulative duration of those transfers (summed over the I/O threads) */
   int32_t spill_uring;          /* 1: transfers go through io_uring (else pread / pwrite) */
+  int32_t hybrid_layers;        /* host layers updated on the GPU (sh_config.hybrid_layers, R28) */
+  int64_t hybrid_updates;       /* cumulative K2S launches of the hybrid update */
+  int64_t hybrid_h2d_bytes;     /* of h2d_bytes / d2h_bytes: the hybrid update's lo / m / v fetches and */
+  int64_t hybrid_d2h_bytes;     /* hi / lo / m / v write-backs */
 } sh_stats_t;
 
 /* One interval of a profiled step (times in ms from the step's first FP hook). */
@@ -529,6 +545,11 @@ sh_status sh_op_master_join_cpu(const uint16_t* hi, const uint16_t* lo, float* p
 sh_status sh_op_adamw_split_cpu(uint16_t* hi, uint16_t* lo, float* m, float* v, const float* g, int64_t n,
                                 int64_t n_decay, const sh_adam_scalars* sc, int32_t use_coef, float coef,
                                 int32_t n_threads);
+
+/* K2S (R28): the same split-master AdamW on the GPU (device pointers, no clipping), bitwise
+ * sh_op_adamw_split_cpu; n, n_decay multiples of 8, 16-byte aligned pointers; enqueued on `stream`. */
+sh_status sh_op_adamw_split_gpu(uint16_t* hi, uint16_t* lo, float* m, float* v, const float* g, int64_t n,
+                                int64_t n_decay, const sh_adam_scalars* sc, void* stream);
 
 /* K4 (NEXT-3): dst[i] = (((dst[i] + src[0][i]) + src[1][i]) + ... + src[n_src-1][i]) * inv_k,
  * every op IEEE fp32 round-to-nearest; src is a HOST array of n_src (0..7) device pointers. */

@@ -296,6 +296,16 @@ struct sh_ctx {
   // ---- streams
   cudaStream_t cs = nullptr, h2d = nullptr, d2h = nullptr, stage = nullptr, comm = nullptr;
   cudaStream_t k3s = nullptr;  // K3 of host layers, beside the D2H copy of the same gradients
+  // R28 hybrid update: lo / m / v fetches into HBM staging, K2S, write-backs (one stream each, so a
+  // layer's K2S never queues behind the previous layer's write-back)
+  cudaStream_t hyb_in = nullptr, hyb_k = nullptr, hyb_out = nullptr;
+  std::vector<char*> hyb_stg;  // staging buffers [lo 2n | m 4n | v 4n] of the largest layer
+  std::vector<cudaEvent_t> ev_stg_in, ev_stg_k2, ev_stg_free;
+  std::vector<int> hyb_stg_of;         // per layer: staging buffer of its current update
+  std::vector<int64_t> hyb_issued;     // per layer: step whose staging fetch was issued (-1: none)
+  int64_t hyb_rr = 0;
+  unsigned int* k2_sched_hyb = nullptr;
+  std::atomic<int64_t> hyb_updates{0}, hyb_h2d{0}, hyb_d2h{0};
   ncclComm_t nccl = nullptr;
   ncclComm_t nccl_fetch = nullptr;  // NEXT-1: collectives issued by the H2D issuer thread
   bool slice_fetch = false;
@@ -511,6 +521,9 @@ struct sh_ctx {
   int async_status = SH_OK;
 
   bool is_g(int x) const { return x < w; }
+  // R28 hybrid update: the lowest n_hyb host-optimised layers are updated on the GPU (include/sh.h)
+  int n_hyb = 0;
+  bool is_hyb(int x) const { return n_hyb > 0 && x >= w && x < w + n_hyb; }
   char* slot_param(int s) const { return byte_ring() ? ring + slot_off[s] : ring + (int64_t)s * slot_bytes; }
   float* slot_grad(int s) const {
     if (byte_ring()) return reinterpret_cast<float*>(ring + slot_off[s] + slot_pb[s]);
@@ -1209,7 +1222,8 @@ int64_t next_use(const sh_ctx* c, int x, int cur) {
   if (b >= cur) return b;  // BP use still ahead
   // after its backward: a host copy goes stale; a GPU-optimised layer's copy was updated in place by
   // its per-layer K2 (valid for the next step's FP) or, in clip mode, its grads wait for sh_step's K2
-  if (!c->is_g(x)) return kInf;
+  // (a hybrid layer's copy was updated in place by its K2S: valid for the next step's FP, like a G layer's)
+  if (!c->is_g(x)) return c->is_hyb(x) ? 2 * (int64_t)c->L + x : kInf;
   return c->k2_layer ? 2 * (int64_t)c->L + x : kPinned;
 }
 
@@ -1811,7 +1825,7 @@ sh_status alloc_ring(sh_ctx* c, int n_slots, bool shrink = false) {
 sh_status sync_all(sh_ctx* c) {
   c->ih2d.drain();
   c->id2h.drain();
-  for (cudaStream_t s : {c->cs, c->h2d, c->d2h, c->stage, c->comm, c->k3s})
+  for (cudaStream_t s : {c->cs, c->h2d, c->d2h, c->stage, c->comm, c->k3s, c->hyb_in, c->hyb_k, c->hyb_out})
     if (s) {
       sh_status st = stream_sync(c, s);
       if (st != SH_OK) return st;
@@ -2165,6 +2179,96 @@ void release_grad_buffer(sh_ctx* c, int b) {
     c->gb_free_seq[b] = ++c->gb_free_ctr;
   }
   c->scv.notify_all();
+}
+
+// ---------------------------------------------------------------------------- R28 hybrid update
+struct HybDone {
+  sh_ctx* c;
+  int layer;
+  int64_t step;
+};
+
+void CUDART_CB hyb_done_cb(void* arg) {  // CUDA driver thread: no CUDA calls
+  std::unique_ptr<HybDone> h(static_cast<HybDone*>(arg));
+  mark_updated(h->c, h->layer, h->step);  // host hi / lo / m / v written back: fetchable again
+}
+
+// At BP PRE(y): issue the staging fetch (host lo / m / v -> HBM) of every hybrid layer among the next
+// D = S - 1 backward positions (y, y-1, ..., y-D) not yet issued this step, into the staging buffers
+// round-robin.  A buffer's previous user is the hybrid layer S fetches back, whose K2S and write-back
+// were enqueued at its POST (it is above y - D); the copy waits for that write-back on the GPU.
+sh_status hyb_issue(sh_ctx* c, int y) {
+  const int S = (int)c->hyb_stg.size();
+  for (int x = y; x >= std::max(c->w, y - (S - 1)); --x) {
+    if (!c->is_hyb(x) || c->hyb_issued[x] == c->step) continue;
+    // the host planes are current once the layer's previous update (CPU or write-back) has landed
+    if (!state_wait(c, [&] { return ready_at_least(c, x, c->step); }, "host update before a hybrid fetch"))
+      return check_failed(c);
+    const int i = (int)(c->hyb_rr++ % S);
+    const int64_t n = c->lay[x].n_pad;
+    CKC(c, cudaStreamWaitEvent(c->hyb_in, c->ev_stg_free[i], 0));
+    CKC(c, cudaMemcpyAsync(c->hyb_stg[i], c->h_lo[x], 10 * n, cudaMemcpyHostToDevice, c->hyb_in));  // [lo | m | v]
+    CKC(c, cudaEventRecord(c->ev_stg_in[i], c->hyb_in));
+    c->hyb_stg_of[x] = i;
+    c->hyb_issued[x] = c->step;
+    c->h2d_bytes += 10 * n;
+    c->hyb_h2d += 10 * n;
+    c->h2d_copies++;
+  }
+  return SH_OK;
+}
+
+// At BP POST(x) of a hybrid layer (its K3 already on the compute stream): K2S on the split master --
+// hi = the compute copy in ring slot s (updated in place), lo / m / v in the staging buffer, grads in
+// pool buffer gb -- then the write-back of hi / lo / m / v to the host block; the layer counts as
+// updated (ready) when the write-back lands, and the next FP of x uses the updated slot copy.
+sh_status hyb_update(sh_ctx* c, int x, int s, int gb) {
+  const int i = c->hyb_stg_of[x];
+  if (i < 0 || c->hyb_issued[x] != c->step) {
+    set_error("internal: hybrid layer %d has no staging fetch for step %lld", x, (long long)c->step);
+    return SH_ERR_STATE;
+  }
+  const int64_t n = c->lay[x].n_pad;
+  char* stg = c->hyb_stg[i];
+  CKC(c, cudaEventRecord(c->ev_grad_done[gb], c->cs));
+  CKC(c, cudaStreamWaitEvent(c->hyb_k, c->ev_grad_done[gb], 0));
+  CKC(c, cudaStreamWaitEvent(c->hyb_k, c->ev_stg_in[i], 0));
+  kern::K2SplitArgs a{};
+  a.sc = c->sc;
+  a.hi = reinterpret_cast<uint16_t*>(c->slot_param(s));
+  a.lo = reinterpret_cast<uint16_t*>(stg);
+  a.m = reinterpret_cast<float*>(stg + 2 * n);
+  a.v = reinterpret_cast<float*>(stg + 6 * n);
+  a.g = c->slot_grad(gb);
+  a.n = n;
+  a.n_decay = c->lay[x].n_decay;
+  a.sched = c->k2_sched_hyb;
+  CKC(c, kern::adamw_split(a, c->hyb_k));
+  c->hyb_updates++;
+  CKC(c, cudaEventRecord(c->ev_stg_k2[i], c->hyb_k));
+  // the pool buffer is free once K2S has read it
+  CKC(c, cudaEventRecord(c->ev_grad_free[gb], c->hyb_k));
+  const int64_t g1 = ++c->gen;
+  c->gradfree_gen[gb] = g1;
+  c->gradfree_pub[gb].store(g1);
+  release_grad_buffer(c, gb);
+  // write-back: hi from the slot, [lo | m | v] from the staging buffer (contiguous in the host block)
+  CKC(c, cudaStreamWaitEvent(c->hyb_out, c->ev_stg_k2[i], 0));
+  CKC(c, cudaMemcpyAsync(c->h_shadow[x], a.hi, 2 * n, cudaMemcpyDeviceToHost, c->hyb_out));
+  CKC(c, cudaMemcpyAsync(c->h_lo[x], stg, 10 * n, cudaMemcpyDeviceToHost, c->hyb_out));
+  CKC(c, cudaEventRecord(c->ev_stg_free[i], c->hyb_out));
+  // the slot's param half may be refilled (and the next FP of x may run) only after the write-back read it
+  CKC(c, cudaEventRecord(c->ev_param_free[s], c->hyb_out));
+  CKC(c, cudaEventRecord(c->ev_arrive[x], c->hyb_out));
+  const int64_t g2 = ++c->gen;
+  c->arrive_gen[x] = g2;
+  c->arrive_by_issuer[x] = 0;
+  c->arrive_pub[x].store(g2);
+  CKC(c, cudaLaunchHostFunc(c->hyb_out, hyb_done_cb, new HybDone{c, x, c->step}));
+  c->d2h_bytes += 12 * n;
+  c->hyb_d2h += 12 * n;
+  c->d2h_copies += 2;
+  return SH_OK;
 }
 
 // D2H issuer thread: offload pending host-layer gradients, lowest layer first, one per free landing
@@ -2642,6 +2746,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       c->k2_sched_cs = reinterpret_cast<unsigned int*>(c->norm_dev + 2);
       c->k2_sched_comm = c->k2_sched_cs + 2;
     }
+    c->k2_sched_hyb = reinterpret_cast<unsigned int*>(c->norm_dev + 2) + 4;  // K2S: always dynamic
     for (int e = 1; e < c->K; ++e) {  // executor gradient buffers (one set: K4 runs in stream order)
       float* xg = nullptr;
       float* xr = nullptr;
@@ -2736,6 +2841,44 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       total += b;
     }
     c->byte_ring_total = total;
+  }
+  if (cfg->hybrid_layers < 0) {
+    set_error("sh_init: hybrid_layers must be >= 0");
+    return SH_ERR_INVALID;
+  }
+  if (cfg->hybrid_layers > 0) {
+    // R28 hybrid update (include/sh.h sh_config.hybrid_layers)
+    if (!c->split || c->clip || c->dp || c->byte_ring() || (cfg->spill_dir && cfg->spill_dir[0])) {
+      set_error("sh_init: hybrid_layers needs the split host master (bf16), no clipping, world_size 1, "
+                "no fixed-byte ring and no spill tier");
+      return SH_ERR_INVALID;
+    }
+    c->n_hyb = cfg->hybrid_layers;
+    const char* e = getenv("SH_HYB_STAGING");
+    const int S = std::max(2, e ? atoi(e) : 3);
+    int lo = 0, hi = 0;
+    CKC(c.get(), cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    CKC(c.get(), cudaStreamCreateWithFlags(&c->hyb_in, cudaStreamNonBlocking));
+    CKC(c.get(), cudaStreamCreateWithPriority(&c->hyb_k, cudaStreamNonBlocking, hi));
+    CKC(c.get(), cudaStreamCreateWithFlags(&c->hyb_out, cudaStreamNonBlocking));
+    for (int i = 0; i < S; ++i) {
+      char* p = nullptr;
+      if (cudaMalloc(&p, 10 * c->max_pad) != cudaSuccess) {
+        cudaGetLastError();
+        set_error("sh_init: cudaMalloc of a hybrid-update staging buffer (%lld B) failed", (long long)(10 * c->max_pad));
+        return SH_ERR_OOM_DEVICE;
+      }
+      c->hyb_stg.push_back(p);
+      c->device_bytes += 10 * c->max_pad;
+      for (auto* v : {&c->ev_stg_in, &c->ev_stg_k2, &c->ev_stg_free}) {
+        cudaEvent_t ev = nullptr;
+        CKC(c.get(), cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        v->push_back(ev);
+      }
+      CKC(c.get(), cudaEventRecord(c->ev_stg_free[i], c->hyb_out));  // free: every wait has a completed event
+    }
+    c->hyb_stg_of.assign(c->L, -1);
+    c->hyb_issued.assign(c->L, -1);
   }
   c->n_active = c->ring_for(w0);
   c->d = c->n_active - 1;
@@ -2968,6 +3111,10 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
     const int pos = 2 * L - 1 - x;
     st = pre_common(c, x, pos);
     if (st != SH_OK) return st;
+    if (c->n_hyb > 0) {
+      st = hyb_issue(c, x);
+      if (st != SH_OK) return st;
+    }
     float* gdst = nullptr;
     if (c->is_g(x) && c->k2_layer) {
       // dedicated grad buffer: no wait on this slot's pending offload
@@ -3098,12 +3245,21 @@ sh_status sh_backward_layer(sh_ctx* c, int32_t x, int32_t phase, void** dev_para
         P->rec_k3[x] = 1;
       }
       CKC(c, cudaEventRecord(c->ev_grad_done[gb], c->cs));
+    } else if (c->is_hyb(x)) {  // R28: K3 on the compute stream (as for a G layer), then the GPU update
+      if (P) CKC(c, cudaEventRecord(P->k30[x], c->cs));
+      CKC(c, kern::sumsq(c->slot_grad(gb), n, c->scratch_cs, c->partials + x, c->cs));
+      if (P) {
+        CKC(c, cudaEventRecord(P->k31[x], c->cs));
+        P->rec_k3[x] = 1;
+      }
+      st = hyb_update(c, x, s, gb);
+      if (st != SH_OK) return st;
     } else {
       // host layer: K3 runs on its own stream beside the offload (off the compute stream)
       CKC(c, cudaEventRecord(c->ev_grad_done[gb], c->cs));
     }
     const bool k3_on_d2h = !c->dp && !c->is_g(x);
-    if (!c->is_g(x)) {  // post the offload: the D2H scheduler issues it lowest layer first (d2h_pump)
+    if (!c->is_g(x) && !c->is_hyb(x)) {  // post the offload: the D2H scheduler issues it lowest layer first (d2h_pump)
       const int64_t gen = ++c->gen;
       c->gradfree_gen[gb] = gen;
       if (k3_on_d2h) c->k3_last_gen = gen;
@@ -3284,7 +3440,7 @@ sh_status sh_step(sh_ctx* c, double* grad_norm_out) {
   // host-optimised copies in the ring are stale after this step's CPU update
   for (int s = 0; s < c->n_active; ++s) {
     const int o = c->slot_layer[s];
-    if (o >= 0 && !c->is_g(o)) {
+    if (o >= 0 && !c->is_g(o) && !c->is_hyb(o)) {  // (a hybrid layer's copy is the updated one)
       c->layer_slot[o] = -1;
       c->slot_layer[s] = -1;
     }
@@ -3676,6 +3832,10 @@ sh_status sh_stats(sh_ctx* c, sh_stats_t* o) {
   o->spill_io_ms = c->spill_io_ms.load();
   o->spill_direct = c->spill_direct ? 1 : 0;
   o->spill_uring = c->n_spilled > 0 && spill::uring_available() ? 1 : 0;
+  o->hybrid_layers = c->n_hyb;
+  o->hybrid_updates = c->hyb_updates.load();
+  o->hybrid_h2d_bytes = c->hyb_h2d.load();
+  o->hybrid_d2h_bytes = c->hyb_d2h.load();
   {
     int n = 0;
     for (int x = c->w; x < c->L; ++x) n += c->h_shadow[x] != nullptr;
@@ -3732,7 +3892,7 @@ sh_status sh_destroy(sh_ctx* c) {
   notify_state(c);
   c->ih2d.stop();
   c->id2h.stop();
-  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s})
+  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s, c->hyb_in, c->hyb_k, c->hyb_out})
     if (s) cudaStreamSynchronize(s);
   if (c->cs) cudaStreamSynchronize(c->cs);
   if (!c->nccl_aborted.load()) {  // an aborted communicator is already freed
@@ -3741,6 +3901,10 @@ sh_status sh_destroy(sh_ctx* c) {
   }
   if (c->partials_all) cudaFree(c->partials_all);
   if (c->fp32_stage) cudaFree(c->fp32_stage);
+  for (char* p : c->hyb_stg) cudaFree(p);
+  for (auto* v : {&c->ev_stg_in, &c->ev_stg_k2, &c->ev_stg_free})
+    for (cudaEvent_t e : *v)
+      if (e) cudaEventDestroy(e);
   if (c->hc_seg) {
     cudaHostUnregister(c->hc_seg);
     munmap(c->hc_seg, c->hc_bytes);
@@ -3775,7 +3939,7 @@ sh_status sh_destroy(sh_ctx* c) {
     if (c->ev_res_k3[i]) cudaEventDestroy(c->ev_res_k3[i]);
     if (c->ev_norm[i]) cudaEventDestroy(c->ev_norm[i]);
   }
-  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s})
+  for (cudaStream_t s : {c->h2d, c->d2h, c->stage, c->comm, c->k3s, c->hyb_in, c->hyb_k, c->hyb_out})
     if (s) cudaStreamDestroy(s);
   for (auto& b : c->hshadow) host_block_free(b.p, b.bytes);
   c->stg_cv.notify_all();
@@ -3985,6 +4149,34 @@ sh_status sh_op_adamw_split_cpu(uint16_t* hi, uint16_t* lo, float* m, float* v, 
     ts.emplace_back([=] { cpu::adamw_range_split(hi, lo, m, v, g, b, e, n_decay, *sc, use_coef != 0, coef); });
   }
   for (auto& t : ts) t.join();
+  return SH_OK;
+}
+
+sh_status sh_op_adamw_split_gpu(uint16_t* hi, uint16_t* lo, float* m, float* v, const float* g, int64_t n,
+                                int64_t n_decay, const sh_adam_scalars* sc, void* stream) {
+  clear_error();
+  const void* ptrs[] = {hi, lo, m, v, g};
+  if (!hi || !lo || !m || !v || !g || !sc || !ops_args_ok(n, n_decay, ptrs, 5)) return SH_ERR_INVALID;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  kern::K2SplitArgs a{};
+  a.sc = *sc;
+  a.hi = hi;
+  a.lo = lo;
+  a.m = m;
+  a.v = v;
+  a.g = g;
+  a.n = n;
+  a.n_decay = n_decay;
+  a.sched = op_scratch(st).k2;
+  if (!a.sched) {
+    set_error("K2S schedule counters: allocation failed");
+    return SH_ERR_OOM_DEVICE;
+  }
+  const cudaError_t e = kern::adamw_split(a, st);
+  if (e != cudaSuccess) {
+    set_error("K2S launch: %s", cudaGetErrorString(e));
+    return SH_ERR_CUDA;
+  }
   return SH_OK;
 }
 

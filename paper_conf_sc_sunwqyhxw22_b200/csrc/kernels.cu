@@ -154,6 +154,74 @@ __global__ void __launch_bounds__(256, kMinBlocks) k2_adamw_kernel(const __grid_
   }
 }
 
+// K2S: K2 on a host layer's SPLIT master (R25 / R28 "hybrid update"): the fp32 master is
+// held as hi = rna_bf16(p) (the bf16 compute copy, here the layer's ring slot, updated in place) and
+// lo = the low 16 bits of p (staged in HBM with m and v).  Per element: p = bits((hi << 16) + sext(lo)),
+// the same adam_elem as K2, then hi' = rna_bf16(p), lo' = low 16 bits of p' -- exactly the CPU pool's
+// split AdamW (cpu_adam.cpp adam_split_*), so a layer updated here or on the CPU ends bit-identical.
+// HBM-bound: r hi 2 + lo 2 + m 4 + v 4 + g 4, w hi 2 + lo 2 + m 4 + v 4 = 28 B/element.  Same dynamic
+// item schedule as K2 (one 4096-element item per block grab).
+__global__ void __launch_bounds__(256, 3) k2_split_kernel(const __grid_constant__ K2SplitArgs a) {
+  const AdamS s{a.sc.beta1, a.sc.beta2, a.sc.omb1, a.sc.omb2, a.sc.eps, -a.sc.step_size,
+                a.sc.sqrt_bc2, a.sc.decay};
+  constexpr int U = 4;
+  const int64_t n_items = (a.n + 1024 * U - 1) / (1024 * U);
+  __shared__ unsigned int s_item[2];
+  int parity = 0;
+  for (;;) {
+    if (threadIdx.x == 0) s_item[parity] = atomicAdd(a.sched, 1u);
+    __syncthreads();
+    const int64_t item = s_item[parity];
+    parity ^= 1;
+    if (item >= n_items) break;
+    const int64_t base = item * (1024 * U);
+    float4 p[U], m[U], v[U], g[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t i = base + u * 1024 + 4 * threadIdx.x;
+      if (i < a.n) {
+        const uint2 h = *reinterpret_cast<const uint2*>(a.hi + i);
+        const uint2 l = *reinterpret_cast<const uint2*>(a.lo + i);
+        auto join = [](uint32_t hh, uint32_t ll) {
+          return __uint_as_float((hh << 16) + (uint32_t)(int32_t)(int16_t)(uint16_t)ll);
+        };
+        p[u] = make_float4(join(h.x & 0xffffu, l.x & 0xffffu), join(h.x >> 16, l.x >> 16),
+                           join(h.y & 0xffffu, l.y & 0xffffu), join(h.y >> 16, l.y >> 16));
+        m[u] = ld_rw(a.m + i);
+        v[u] = ld_rw(a.v + i);
+        g[u] = ld_stream(a.g + i);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t i = base + u * 1024 + 4 * threadIdx.x;
+      if (i >= a.n) continue;
+      const bool wd = i < a.n_decay;  // n_decay is a multiple of 8: uniform per float4
+      adam_elem(p[u].x, m[u].x, v[u].x, g[u].x, s, wd, false, 1.0f);
+      adam_elem(p[u].y, m[u].y, v[u].y, g[u].y, s, wd, false, 1.0f);
+      adam_elem(p[u].z, m[u].z, v[u].z, g[u].z, s, wd, false, 1.0f);
+      adam_elem(p[u].w, m[u].w, v[u].w, g[u].w, s, wd, false, 1.0f);
+      st_f4(a.m + i, m[u]);
+      st_f4(a.v + i, v[u]);
+      uint2 h, l;
+      h.x = rna_bf16_bits(p[u].x) | (rna_bf16_bits(p[u].y) << 16);
+      h.y = rna_bf16_bits(p[u].z) | (rna_bf16_bits(p[u].w) << 16);
+      l.x = (__float_as_uint(p[u].x) & 0xffffu) | (__float_as_uint(p[u].y) << 16);
+      l.y = (__float_as_uint(p[u].z) & 0xffffu) | (__float_as_uint(p[u].w) << 16);
+      *reinterpret_cast<uint2*>(a.hi + i) = h;
+      *reinterpret_cast<uint2*>(a.lo + i) = l;
+    }
+  }
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(a.sched + 1, 1u) == gridDim.x - 1) {  // every block has made its last grab
+      a.sched[0] = 0;
+      a.sched[1] = 0;
+      __threadfence();
+    }
+  }
+}
+
 // K2, bulk-copy pipeline variant (SH_K2_IMPL=bulk).  The register-staged kernel above loads a work
 // item, then computes and stores it: while a block is in its compute/store phase its loads are
 // idle, and at 83 registers only 2 blocks fit per SM.  Here one 512-thread block per SM keeps the
@@ -564,6 +632,25 @@ cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out) {
     if (a.out_bf16) k2_adamw_kernel<true, 2><<<grid, 256, 0, st>>>(a);
     else k2_adamw_kernel<false, 2><<<grid, 256, 0, st>>>(a);
   }
+  return cudaGetLastError();
+}
+
+cudaError_t adamw_split(const K2SplitArgs& a, cudaStream_t st) {
+  if (a.n <= 0) return cudaSuccess;
+  if (!a.sched) return cudaErrorInvalidValue;
+  const int64_t items = (a.n + 4095) / 4096;
+  if (items >= (int64_t)1 << 32) return cudaErrorInvalidValue;
+  static const int per_sm = [] {
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k2_split_kernel, 256, 0) != cudaSuccess || nb <= 0) {
+      cudaGetLastError();
+      nb = 3;
+    }
+    return nb;
+  }();
+  const int64_t cap = (int64_t)sm_count() * per_sm;
+  launch_counter()++;
+  k2_split_kernel<<<(int)(items < cap ? items : cap), 256, 0, st>>>(a);
   return cudaGetLastError();
 }
 

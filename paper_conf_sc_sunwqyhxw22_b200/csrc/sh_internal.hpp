@@ -74,6 +74,21 @@ struct K2Args {
 bool k2_dynamic();
 // Launch K2 over args (item_start filled by the callee).  Returns the grid used.
 cudaError_t adamw_multi(K2Args& a, cudaStream_t st, int* grid_out = nullptr);
+// K2S: AdamW on a split master (hi = bf16 compute copy, lo = low 16 bits; m, v fp32), updated in place;
+// bitwise the CPU pool's split AdamW.  No clipping.  sched: 2 zeroed device counters owned by the caller
+// for this stream (left zeroed).  n, n_decay multiples of 8; pointers 16-byte aligned.
+struct K2SplitArgs {
+  sh_adam_scalars sc;
+  uint16_t* hi;
+  uint16_t* lo;
+  float* m;
+  float* v;
+  const float* g;
+  int64_t n;
+  int64_t n_decay;
+  unsigned int* sched;
+};
+cudaError_t adamw_split(const K2SplitArgs& a, cudaStream_t st);
 cudaError_t cast_bf16(const float* src, uint16_t* dst, int64_t n, cudaStream_t st);
 constexpr int kSumsqMaxBlocks = 1184;  // 148 SMs x 8
 // Deterministic Σ g^2 in fp64 -> *out (device).  scratch: kSumsqMaxBlocks + 1 doubles, zeroed

@@ -36,7 +36,7 @@ EXPORTS = ("sh_init", "sh_register_host_store", "sh_synchronize", "sh_destroy", 
            "sh_op_sumsq_gpu", "sh_kernel_launches", "sh_get_trace", "sh_forward_only_end", "sh_set_window_ring",
            "sh_executor_grads", "sh_op_exec_reduce_gpu", "sh_numa_topology", "sh_numa_plan",
            "sh_numa_worker_node", "sh_numa_node_of_pci", "sh_numa_bind_check", "sh_spill_probe", "sh_op_master_split_cpu",
-           "sh_op_master_join_cpu", "sh_op_adamw_split_cpu")
+           "sh_op_master_join_cpu", "sh_op_adamw_split_cpu", "sh_op_adamw_split_gpu")
 
 # NUMA placement policies (sh_config.numa_policy, include/sh.h)
 SH_NUMA_AUTO, SH_NUMA_SPLIT, SH_NUMA_LOCAL, SH_NUMA_INTERLEAVE, SH_NUMA_NONE = range(5)
@@ -62,7 +62,8 @@ class Config(C.Structure):
                 ("world_size", C.c_int32), ("rank", C.c_int32),
                 ("nccl_unique_id", C.c_void_p), ("flags", C.c_uint64), ("shm_name", C.c_char_p),
                 ("n_executors", C.c_int32), ("spill_dir", C.c_char_p), ("host_pin_budget_bytes", C.c_int64),
-                ("warmup_window", C.c_int32), ("numa_policy", C.c_int32), ("ring_bytes", C.c_int64)]
+                ("warmup_window", C.c_int32), ("numa_policy", C.c_int32), ("ring_bytes", C.c_int64),
+                ("hybrid_layers", C.c_int32)]
 
 
 _PD = C.POINTER(C.c_double)
@@ -102,7 +103,9 @@ class Stats(C.Structure):
                 ("numa_pinned_workers", C.c_int32), ("numa_bound_bytes", C.c_int64),
                 ("compute_busy_ms", C.c_double), ("ring_bytes", C.c_int64), ("cpu_adam_shadow_elems", C.c_int64),
                 ("shadow_layers", C.c_int32), ("spill_direct", C.c_int32), ("spill_read_bytes", C.c_int64),
-                ("spill_write_bytes", C.c_int64), ("spill_io_ms", C.c_double), ("spill_uring", C.c_int32)]
+                ("spill_write_bytes", C.c_int64), ("spill_io_ms", C.c_double), ("spill_uring", C.c_int32),
+                ("hybrid_layers", C.c_int32), ("hybrid_updates", C.c_int64), ("hybrid_h2d_bytes", C.c_int64),
+                ("hybrid_d2h_bytes", C.c_int64)]
 
 
 class TraceEvent(C.Structure):
@@ -157,6 +160,7 @@ def lib() -> C.CDLL:
             "sh_spill_probe": [C.c_char_p, i64, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(i32)],
             "sh_op_master_split_cpu": [vp, vp, vp, i64], "sh_op_master_join_cpu": [vp, vp, vp, i64],
             "sh_op_adamw_split_cpu": [vp, vp, vp, vp, vp, i64, i64, vp, i32, f32, i32],
+            "sh_op_adamw_split_gpu": [vp, vp, vp, vp, vp, i64, i64, vp, vp],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -220,6 +224,11 @@ def op_master_split_cpu(p, hi, lo, n):
 
 def op_master_join_cpu(hi, lo, p, n):
     check(lib().sh_op_master_join_cpu(_ptr(hi), _ptr(lo), _ptr(p), n))
+
+
+def op_adamw_split_gpu(hi, lo, m, v, g, n, n_decay, sc: AdamScalars, stream=None):
+    check(lib().sh_op_adamw_split_gpu(_ptr(hi), _ptr(lo), _ptr(m), _ptr(v), _ptr(g), n, n_decay, C.byref(sc),
+                                      _stream_handle(stream)))
 
 
 def op_adamw_split_cpu(hi, lo, m, v, g, n, n_decay, sc: AdamScalars, coef=None, threads=0):
@@ -342,7 +351,7 @@ class Engine:
                  stream=None, cpu_threads=0, grad_ring_depth=0, warmup_steps=5, device_budget_bytes=0,
                  world_size=1, rank=0, nccl_id: bytes | None = None, flags=0, shm_name: str | None = None,
                  ring_slots=0, cpu_util_max=0.0, n_executors=1, spill_dir: str | None = None,
-                 host_pin_budget_bytes=0, warmup_window=0, numa_policy=0, ring_bytes=0):
+                 host_pin_budget_bytes=0, warmup_window=0, numa_policy=0, ring_bytes=0, hybrid_layers=0):
         L = lib()
         self.n_layers = len(layer_numels)
         self._keep = []
@@ -384,6 +393,7 @@ class Engine:
         cfg.warmup_window = int(warmup_window)
         cfg.numa_policy = int(numa_policy)
         cfg.ring_bytes = int(ring_bytes)
+        cfg.hybrid_layers = int(hybrid_layers)
         self.n_executors = max(1, n_executors)
         self._shm = shm_name.encode() if shm_name else None
         cfg.shm_name = self._shm

@@ -54,7 +54,7 @@ class StrongholdTrainer:
                  max_grad_norm=0.0, device=0, seed=1234, cpu_threads=0, grad_ring_depth=0, warmup_steps=5,
                  flags=0, world_size=1, rank=0, nccl_id=None, init=True, init_threads=8, shm_name=None,
                  attention="auto", ring_slots=0, executors=1, spill_dir=None, host_pin_budget_bytes=0,
-                 warmup_window=0, numa_policy=0, ring_bytes=0):
+                 warmup_window=0, numa_policy=0, ring_bytes=0, hybrid_layers=0):
         self.mc = mc
         self.batch = batch
         # NEXT-3 multi-stream executors: K workers on K streams, one parameter copy,
@@ -74,7 +74,8 @@ class StrongholdTrainer:
                                 warmup_steps=warmup_steps, world_size=world_size, rank=rank, nccl_id=nccl_id,
                                 flags=flags, shm_name=shm_name, ring_slots=ring_slots, n_executors=self.K,
                                 spill_dir=spill_dir, host_pin_budget_bytes=host_pin_budget_bytes,
-                                warmup_window=warmup_window, numa_policy=numa_policy, ring_bytes=ring_bytes)
+                                warmup_window=warmup_window, numa_policy=numa_policy, ring_bytes=ring_bytes,
+                                hybrid_layers=hybrid_layers)
         # executor 0 runs on the engine's compute stream, executors >= 1 on their own streams
         self.streams = [self.stream] + [torch.cuda.Stream(device=self.device) for _ in range(self.K - 1)]
         self.gpts = [GPT(n_layers=L, hidden=mc.hidden, heads=mc.heads, seq=mc.seq, max_batch=self.mb,

@@ -43,7 +43,7 @@ def test_library_exports_every_declared_symbol(header, libname, py):
 
 
 def test_abi_version_and_error_string():
-    assert sh.lib().sh_abi_version() == 2
+    assert sh.lib().sh_abi_version() == 3
     with pytest.raises(sh.ShError) as e:
         sh.adam_scalars(1e-3, 0.9, 0.999, 1e-8, 0.0, 0)  # t must be >= 1
     assert e.value.status == sh.SH_ERR_INVALID and "t must be" in str(e.value)
