@@ -6,6 +6,7 @@
 #   bash tools/gpu_runs.sh ncu        ncu iso captures of K1-K4 + the c4max launch list (tools/ncu_c4max.sh)
 #   bash tools/gpu_runs.sh cpu_pf     CPU AdamW prefetch probe + DMA page-size probe + c4max A/B
 #   bash tools/gpu_runs.sh next4      NEXT-4 fixed-byte window vs the layer-count ring on C2
+#   bash tools/gpu_runs.sh hybrid     R28 hybrid-update GPU tests + c4max A/B over the number of hybrid layers
 #   bash tools/gpu_runs.sh ab NAME|ENV|ARGS ...   c4max A/B (tools/ab_c4max.sh, L = 112)
 # Outputs land in gpurun_out/; the summaries worth keeping are copied to profiles/ by hand.
 set -u
@@ -71,6 +72,12 @@ case "${1:-}" in
     cat gpurun_out/cpu_pf.jsonl
     bash tools/ab_c4max.sh 112 "pf0|SH_CPU_PF=0|" "pf512|SH_CPU_PF=512|" ;;
   next4) build; next4 ;;
+  hybrid)
+    smoke
+    timeout 1200 python -m pytest tests/test_hybrid_gpu.py tests/test_kernels_gpu.py tests/test_engine_gpu.py -x -q -m gpu \
+      > gpurun_out/pytest_hybrid.log 2>&1; echo "pytest rc $?"; tail -15 gpurun_out/pytest_hybrid.log
+    grep -q "passed" gpurun_out/pytest_hybrid.log && ! grep -q "failed\|error" gpurun_out/pytest_hybrid.log || exit 1
+    bash tools/ab_c4max.sh 112 "hyb0||" "hyb4||--hybrid-layers 4" "hyb8||--hybrid-layers 8" "hyb12||--hybrid-layers 12" ;;
   ab) shift; build; bash tools/ab_c4max.sh 112 "$@" ;;
   *) sed -n 2,10p "$0"; exit 2 ;;
 esac
