@@ -79,5 +79,10 @@ case "${1:-}" in
     grep -q "passed" gpurun_out/pytest_hybrid.log && ! grep -q "failed\|error" gpurun_out/pytest_hybrid.log || exit 1
     bash tools/ab_c4max.sh 112 "hyb0||" "hyb4||--hybrid-layers 4" "hyb8||--hybrid-layers 8" "hyb12||--hybrid-layers 12" ;;
   ab) shift; build; bash tools/ab_c4max.sh 112 "$@" ;;
+  hybrid2)
+    build
+    bash tools/ab_c4max.sh 112 "hyb0b||" "hyb6s2|SH_HYB_STAGING=2|--hybrid-layers 6"
+    timeout 2400 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu_full.log 2>&1
+    echo "pytest rc $?"; tail -1 gpurun_out/pytest_gpu_full.log ;;
   *) sed -n 2,10p "$0"; exit 2 ;;
 esac
