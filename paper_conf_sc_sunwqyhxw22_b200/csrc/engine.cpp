@@ -522,6 +522,10 @@ struct sh_ctx {
 
   bool is_g(int x) const { return x < w; }
   // R28 hybrid update: the lowest n_hyb host-optimised layers are updated on the GPU (include/sh.h)
+  // SH_CPU_THROTTLE=T (> 0): while the driver waits for a free gradient buffer (the offloads are the
+  // bottleneck), CPU AdamW workers with index >= T pause, leaving host DRAM to the D2H copies
+  int cpu_throttle = 0;
+  std::atomic<int> grad_starved{0};
   int n_hyb = 0;
   bool is_hyb(int x) const { return n_hyb > 0 && x >= w && x < w + n_hyb; }
   char* slot_param(int s) const { return byte_ring() ? ring + slot_off[s] : ring + (int64_t)s * slot_bytes; }
@@ -875,6 +879,9 @@ void worker_loop(sh_ctx* c, int tid) {
           if (eligible(jp.get())) return true;
         return false;
       };
+      if (c->cpu_throttle > 0 && tid >= c->cpu_throttle)
+        while (c->grad_starved.load() && !c->pool_stop && !c->failed.load())
+          c->pcv.wait_for(g, std::chrono::microseconds(200));
       if (c->shared) {
         while (!any()) c->pcv.wait_for(g, std::chrono::microseconds(100));
       } else {
@@ -2165,7 +2172,11 @@ int take_grad_buffer(sh_ctx* c, int x, int64_t n) {
       return b;
     }
   }
-  if (!state_wait(c, pick, "a free gradient buffer")) return -1;
+  c->grad_starved.store(1);
+  const bool got = state_wait(c, pick, "a free gradient buffer");
+  c->grad_starved.store(0);
+  if (c->cpu_throttle > 0) c->pcv.notify_all();
+  if (!got) return -1;
   std::lock_guard<std::mutex> g(c->smu);
   if (!pick()) return -1;  // (failed meanwhile)
   c->gb_owner[b] = x;
@@ -2584,6 +2595,7 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       dflt = (int)topo.cpus[c->numa_gpu].size();  // LOCAL: the GPU node's cores
     c->n_threads = cfg->cpu_threads > 0 ? cfg->cpu_threads : dflt;
     if (c->n_threads < 1) c->n_threads = 1;
+    if (const char* e = getenv("SH_CPU_THROTTLE")) c->cpu_throttle = std::max(0, atoi(e));
     c->worker_node.assign(c->n_threads, numa::kNone);
     for (int t = 0; t < c->n_threads; ++t)
       c->worker_node[t] = numa::worker_node(c->numa_policy, t, c->n_threads, c->numa_gpu);
