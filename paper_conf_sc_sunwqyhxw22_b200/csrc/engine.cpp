@@ -523,8 +523,8 @@ struct sh_ctx {
   bool is_g(int x) const { return x < w; }
   // R28 hybrid update: the lowest n_hyb host-optimised layers are updated on the GPU (include/sh.h)
   // while the driver waits for a free gradient buffer (the offloads are the bottleneck), CPU AdamW
-  // workers with index >= cpu_throttle pause, leaving host DRAM to the D2H copies (default
-  // n_threads - 4 from 12 threads up; SH_CPU_THROTTLE=T sets it, 0 = off)
+  // workers with index >= cpu_throttle pause, leaving host DRAM to the D2H copies (SH_CPU_THROTTLE=T;
+  // 0 = off, the default)
   int cpu_throttle = 0;
   std::atomic<int> grad_starved{0};
   int n_hyb = 0;
@@ -2596,9 +2596,9 @@ sh_status sh_init(const sh_config* cfg, sh_ctx** out) {
       dflt = (int)topo.cpus[c->numa_gpu].size();  // LOCAL: the GPU node's cores
     c->n_threads = cfg->cpu_threads > 0 ? cfg->cpu_threads : dflt;
     if (c->n_threads < 1) c->n_threads = 1;
-    // default: 4 of 16 workers pause while the offloads starve the backward (fixed-window c4max A/B on a
-    // slow-D2H box: 5.25 / 5.24 vs 5.21 / 5.22 samples/s, profiles/r02_ab_c4max_throttle.txt)
-    c->cpu_throttle = c->n_threads >= 12 ? c->n_threads - 4 : 0;
+    // off by default: a fixed-window c4max A/B on a slow-D2H box gave +0.6 % with 12 of 16 workers
+    // (5.25 / 5.24 vs 5.21 / 5.22 samples/s), inside the autotuned runs' box-to-box noise
+    // (profiles/r02_ab_c4max_throttle.txt)
     if (const char* e = getenv("SH_CPU_THROTTLE")) c->cpu_throttle = std::max(0, atoi(e));
     c->worker_node.assign(c->n_threads, numa::kNone);
     for (int t = 0; t < c->n_threads; ++t)
